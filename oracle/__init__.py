@@ -1,0 +1,180 @@
+"""CPU oracle for the GPL hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` legs may import this package. The
+product package (``paper_conf_sigmod_paulhh16_b200``) never imports it and
+shares no code with it; both consume only ``tpchgen`` output.
+
+``oracle.cpp`` evaluates each paper Listing as
+plain SQL semantics row-at-a-time (see its header for the exact rules and the
+readings of garbled passages). ``bruteforce.py`` is an independent pin written
+as nested loops straight from the SQL text.
+
+Pins: tests/test_oracle_pins.py (brute force, worked examples W1-W4 in
+tests/golden/, numpy/pandas special cases, invariants).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import time
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+# Query parameters exactly as printed in the Listings (dates as yyyymmdd).
+DEFAULT_PARAMS = {
+    "L1": (19881101,),             # P:158  l_shipdate <= '1988-11-01' (reading #1)
+    "Q5": (19940101, 19950101),    # P:603-604  [1994-01-01, 1995-01-01)
+    "Q7": (19950101, 19961231),    # P:626-627  between (inclusive, reading #9)
+    "Q8": (19950101, 19961231),    # P:650-651  between (inclusive)
+    "Q9": (1000,),                 # P:677  p_partKey < 1000 (reading #5)
+    "Q14": (19950901, 19951001),   # P:688-689  [1995-09-01, 1995-10-01)
+}
+QUERY_IDS = {"L1": 1, "Q5": 5, "Q7": 7, "Q8": 8, "Q9": 9, "Q14": 14}
+# Result schema (keys, aggs) per query: count(*) first, then the SUMs.
+SCHEMA = {
+    "L1": ((), ("count", "sum_charge")),
+    "Q5": (("n_name",), ("count", "revenue")),
+    "Q7": (("supp_nation", "cust_nation", "l_year"), ("count", "revenue")),
+    "Q8": (("o_year",), ("count", "brazil_volume", "volume")),
+    "Q9": (("nation", "o_year"), ("count", "sum_profit")),
+    "Q14": ((), ("count", "promo_volume", "total_volume")),
+}
+
+
+class _OracleDB(ctypes.Structure):
+    P = ctypes.c_void_p
+    I = ctypes.c_int64
+    _fields_ = [
+        ("n_region", I), ("r_regionkey", P), ("r_name", P),
+        ("n_nation", I), ("n_nationkey", P), ("n_name", P), ("n_regionkey", P),
+        ("n_supplier", I), ("s_suppkey", P), ("s_nationkey", P),
+        ("n_customer", I), ("c_custkey", P), ("c_nationkey", P),
+        ("n_part", I), ("p_partkey", P), ("p_type", P),
+        ("n_partsupp", I), ("ps_partkey", P), ("ps_suppkey", P), ("ps_supplycost", P),
+        ("n_orders", I), ("o_orderkey", P), ("o_custkey", P), ("o_orderdate", P),
+        ("n_lineitem", I), ("l_orderkey", P), ("l_partkey", P), ("l_suppkey", P),
+        ("l_quantity", P), ("l_extendedprice", P), ("l_discount", P), ("l_tax", P),
+        ("l_shipdate", P),
+        ("dict_r_name", P), ("n_dict_r_name", ctypes.c_int32),
+        ("dict_n_name", P), ("n_dict_n_name", ctypes.c_int32),
+        ("dict_p_type", P), ("n_dict_p_type", ctypes.c_int32),
+    ]
+
+
+class _OracleResult(ctypes.Structure):
+    _fields_ = [("n_rows", ctypes.c_int32), ("n_keys", ctypes.c_int32), ("n_aggs", ctypes.c_int32),
+                ("cap_rows", ctypes.c_int32), ("keys", ctypes.c_void_p), ("aggs", ctypes.c_void_p),
+                ("err", ctypes.c_char * 256)]
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_LIB_PATH):
+            raise RuntimeError(f"{_LIB_PATH} missing: run `make` (or __graft_entry__.build())")
+        lib = ctypes.CDLL(_LIB_PATH)
+        lib.oracle_run.argtypes = [ctypes.c_int, ctypes.POINTER(_OracleDB), ctypes.c_void_p,
+                                   ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(_OracleResult)]
+        lib.oracle_run.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+@dataclass
+class Result:
+    """Query result: rows sorted by group key; every aggregate an exact Python int."""
+    query: str
+    keys: list      # list of tuples (dictionary codes / years)
+    aggs: list      # list of lists of int (count, sums...)
+
+    def as_dict(self):
+        return {k: a for k, a in zip(self.keys, self.aggs)}
+
+
+def _strings(lst):
+    arr = (ctypes.c_char_p * len(lst))(*[s.encode() for s in lst])
+    return arr
+
+
+def _db_struct(db):
+    keep = []
+
+    def p(table, col):
+        t = db.tables.get(table)
+        if t is None or col not in t:
+            return None
+        a = np.ascontiguousarray(t[col])
+        keep.append(a)
+        return ctypes.c_void_p(a.ctypes.data)
+
+    def n(table):
+        t = db.tables.get(table)
+        return 0 if not t else len(next(iter(t.values())))
+
+    s = _OracleDB()
+    s.n_region, s.r_regionkey, s.r_name = n("region"), p("region", "r_regionkey"), p("region", "r_name")
+    s.n_nation = n("nation")
+    s.n_nationkey, s.n_name, s.n_regionkey = (p("nation", "n_nationkey"), p("nation", "n_name"),
+                                              p("nation", "n_regionkey"))
+    s.n_supplier, s.s_suppkey, s.s_nationkey = n("supplier"), p("supplier", "s_suppkey"), p("supplier", "s_nationkey")
+    s.n_customer, s.c_custkey, s.c_nationkey = n("customer"), p("customer", "c_custkey"), p("customer", "c_nationkey")
+    s.n_part, s.p_partkey, s.p_type = n("part"), p("part", "p_partkey"), p("part", "p_type")
+    s.n_partsupp = n("partsupp")
+    s.ps_partkey, s.ps_suppkey, s.ps_supplycost = (p("partsupp", "ps_partkey"), p("partsupp", "ps_suppkey"),
+                                                   p("partsupp", "ps_supplycost"))
+    s.n_orders = n("orders")
+    s.o_orderkey, s.o_custkey, s.o_orderdate = (p("orders", "o_orderkey"), p("orders", "o_custkey"),
+                                                p("orders", "o_orderdate"))
+    s.n_lineitem = n("lineitem")
+    for c in ("l_orderkey", "l_partkey", "l_suppkey", "l_quantity", "l_extendedprice", "l_discount",
+              "l_tax", "l_shipdate"):
+        setattr(s, c, p("lineitem", c))
+    d1, d2, d3 = _strings(db.r_name), _strings(db.n_name), _strings(db.p_type)
+    keep += [d1, d2, d3]
+    s.dict_r_name, s.n_dict_r_name = ctypes.cast(d1, ctypes.c_void_p), len(db.r_name)
+    s.dict_n_name, s.n_dict_n_name = ctypes.cast(d2, ctypes.c_void_p), len(db.n_name)
+    s.dict_p_type, s.n_dict_p_type = ctypes.cast(d3, ctypes.c_void_p), len(db.p_type)
+    return s, keep
+
+
+def run(query: str, db, params=None, lineitem_range=None) -> Result:
+    """Evaluate `query` ("L1", "Q5", "Q7", "Q8", "Q9", "Q14") on `db` (tpchgen.Database)."""
+    lib = _load()
+    params = tuple(params) if params is not None else DEFAULT_PARAMS[query]
+    pr = np.array(list(params) + [0] * (4 - len(params)), dtype=np.int32)
+    s, keep = _db_struct(db)
+    lb, le = lineitem_range if lineitem_range is not None else (0, s.n_lineitem)
+    cap = 4096
+    keys = np.zeros(cap * 4, dtype=np.int32)
+    aggs = np.zeros(cap * 4 * 2, dtype=np.int64)
+    r = _OracleResult()
+    r.cap_rows = cap
+    r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data
+    rc = lib.oracle_run(QUERY_IDS[query], ctypes.byref(s), pr.ctypes.data, lb, le, ctypes.byref(r))
+    if rc != 0:
+        raise RuntimeError("oracle: " + r.err.decode())
+    nk, na = r.n_keys, r.n_aggs
+    out_k, out_a = [], []
+    for i in range(r.n_rows):
+        out_k.append(tuple(int(x) for x in keys[i * nk:(i + 1) * nk]))
+        row = []
+        for j in range(na):
+            lo = int(aggs[(i * na + j) * 2]) & ((1 << 64) - 1)
+            hi = int(aggs[(i * na + j) * 2 + 1])
+            row.append((hi << 64) | lo)
+        out_a.append(row)
+    del keep
+    return Result(query, out_k, out_a)
+
+
+def timed_run(query: str, db, params=None, lineitem_range=None):
+    """(Result, seconds) — wall time of one oracle evaluation (single thread)."""
+    t0 = time.perf_counter()
+    r = run(query, db, params, lineitem_range)
+    return r, time.perf_counter() - t0
