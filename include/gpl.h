@@ -1,0 +1,216 @@
+/*
+ * gpl.h — C ABI of the B200-native GPL hot path (pipelined scan -> probe ->
+ * aggregate over columnar in-memory relations).
+ *
+ * Paper: J. Paul, J. He, B. He, "GPL: A GPU-based Pipelined Query Processing
+ * Engine", SIGMOD'16 (PAPER.md; cited as P:<line>).
+ *
+ * The calls follow the paper's problem statement:
+ *   - a query plan over columnar in-memory relations is split into segments,
+ *     each ending at a blocking kernel; hash build is blocking, probe is not
+ *     (§3.1 "segments", §3.2 "Hash join ... requires a blocking
+ *     barrier after hash build");
+ *   - the input of a segment is processed tile by tile, the tile size coming
+ *     from a cost model (§3.1, §3.3, §4 Eqs 1-9);
+ *   - only the outputs of blocking kernels are materialised in global memory
+ *     (P:135); the rest passes through on-chip channels (P:179-189
+ *     §3.4), here shared-memory rings inside one fused sm_100a kernel;
+ *   - data is resident on the device (App. A).
+ *
+ * Conventions
+ *   - Every call returns gpl_status (0 = GPL_OK). No C++ exception crosses the
+ *     ABI; the message of the last failure is gpl_last_error(ctx).
+ *   - One context = one CUDA device + one stream, used by one host thread at a
+ *     time. All device work is enqueued on that stream, in call order; stream
+ *     order is the "blocking barrier" between segments.
+ *   - Types: keys, dates (int32 yyyymmdd) and dictionary codes are int32;
+ *     decimals are scaled int64 (scale stated per column). Sums are exact:
+ *     int64 on chip, int128 in the partials and the result.
+ *   - Plan texts: see DESIGN.md §4 (grammar) and paper_conf_sigmod_paulhh16_b200/plans/.
+ */
+#ifndef GPL_H
+#define GPL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t gpl_status;
+enum {
+  GPL_OK = 0,
+  GPL_E_ARG = 1,       /* bad argument (NULL, type, alignment, size)                */
+  GPL_E_CUDA = 2,      /* CUDA runtime error (message has the CUDA error string)    */
+  GPL_E_NOMEM = 3,     /* device allocation failed                                  */
+  GPL_E_STATE = 4,     /* missing table / hash table / no run to fetch              */
+  GPL_E_DUPKEY = 5,    /* build key not unique (all paper joins are FK->PK)         */
+  GPL_E_CAPACITY = 6,  /* caller buffer too small (n_groups / nbytes set)           */
+  GPL_E_OVERFLOW = 7,  /* a value bound exceeds exact int64 arithmetic              */
+  GPL_E_DOMAIN = 8,    /* a row's group value fell outside the declared domain      */
+  GPL_E_NODEV = 9,     /* operation needs a device but the context has none         */
+  GPL_E_PLAN = 10      /* plan text: syntax or semantic error                        */
+};
+
+/* Column types. */
+enum { GPL_I32 = 1, GPL_I64 = 2, GPL_DATE32 = 3, GPL_DEC64 = 4, GPL_DICT32 = 5 };
+
+/* gpl_load_columns flags */
+enum { GPL_COPY = 0, GPL_BORROW = 1 };
+
+typedef struct {
+  const char* name;       /* column name, unique within the table                          */
+  int32_t type;           /* GPL_I32 .. GPL_DICT32                                           */
+  int32_t scale;          /* decimal scale (informational; 0 for non-decimals)              */
+  const void* data;       /* host or device pointer to nrows values                          */
+  int32_t on_device;      /* 1: data is a device pointer on the context's device            */
+  int32_t reserved;
+  int64_t capacity_rows;  /* BORROW only: rows allocated behind data (0 = nrows).           */
+} gpl_column;
+
+typedef struct gpl_ctx gpl_ctx;
+
+/* Statistics of the last gpl_run_plan (filled by gpl_fetch_result). */
+typedef struct {
+  int64_t rows_scanned;        /* fact rows streamed through the pipeline                        */
+  int64_t tile_rows_used;      /* Δ actually used (rows per scheduling claim)                    */
+  int32_t stage_rows;          /* rows per TMA stage                                              */
+  int32_t ring_depth;          /* stages in the shared-memory ring ("channels")            */
+  int32_t consumer_warps;      /* consumer warps per CTA                                          */
+  int32_t grid;                /* persistent CTAs                                                 */
+  int32_t n_ops;               /* entries used in op_pass                                         */
+  int32_t probe_split;         /* probes run before the survivor queue (-1: none)                */
+  int64_t op_pass[16];         /* rows passing each operator in plan order (filters, probes, where) */
+  double kernel_ms;            /* fused pipeline kernel time (CUDA events on the ctx stream)      */
+  double predicted_ms;         /* A9 model estimate for this run                                   */
+  double bytes_scanned;        /* algorithmic bytes: rows x bytes/row of staged columns           */
+  int32_t agg_mode;            /* 0 registers (1 group), 1 smem table, 2 global int128 atomics   */
+  int32_t kbe;                 /* 1 if produced by gpl_run_plan_kbe                               */
+  double intermediate_bytes;   /* bytes of operator outputs materialised in HBM (fused path: 0)   */
+} gpl_stats;
+
+/* Result of the last run. Arrays are CALLER-owned with capacity cap_groups. */
+typedef struct {
+  int32_t cap_groups;          /* in: rows the arrays can hold                                    */
+  int32_t n_groups;            /* out: non-empty groups (1 row when the plan has no GROUP BY)    */
+  int32_t n_keys;              /* out: group key columns                                          */
+  int32_t n_aggs;              /* out: aggregates per row; agg 0 is COUNT(*)                      */
+  int32_t* keys;               /* out: [cap_groups][n_keys] decoded key values, rows sorted by key */
+  int64_t* aggs;               /* out: [cap_groups][n_aggs][2] int128 as (lo, hi) little-endian   */
+  gpl_stats stats;             /* out */
+} gpl_result;
+
+/* A9 model report (gpl_choose_tile_rows). */
+typedef struct {
+  int64_t tile_rows;
+  int32_t stage_rows, ring_depth, consumer_warps, grid;
+  double predicted_ms;
+  double t_stream_ms, t_probe_ms, t_tail_ms, t_launch_ms;
+  double bw_gbs;               /* effective HBM bandwidth the model used                           */
+  int32_t smem_bytes;
+  int32_t feasible;
+} gpl_model_report;
+
+/* Create a context on CUDA device `device` enqueuing on `cuda_stream` (a
+ * cudaStream_t, e.g. torch.cuda.current_stream().cuda_stream; NULL = the
+ * library creates its own non-blocking stream). device = -1 creates a
+ * HOST-ONLY context (no CUDA calls): plans can be parsed/validated and the
+ * cost model queried; gpl_build_hash only validates and registers the
+ * table's shape (no data), run/fetch return GPL_E_NODEV. Platform facts (SMs,
+ * shared memory, L2) are queried from the device.
+ * Errors: GPL_E_ARG (out == NULL), GPL_E_CUDA (bad device). */
+gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out);
+
+/* Free every ctx-owned device allocation (copied columns, hash tables,
+ * partials). Borrowed column memory is untouched. NULL is a no-op. */
+void gpl_destroy(gpl_ctx* ctx);
+
+/* Place a table's columns in HBM (SoA). Replaces an
+ * existing table of that name and invalidates hash tables built from it.
+ *   GPL_COPY:   data may be host or device memory; the ctx owns a padded
+ *               (64-row, zero-filled) 256-B-aligned copy.
+ *   GPL_BORROW: data must be device memory, 16-B aligned, with
+ *               capacity_rows >= nrows rounded up to 4 rows; the caller keeps
+ *               it alive and unchanged while any run may read it.
+ * Per-column min/max are computed on load (validator bounds).
+ * Errors: GPL_E_ARG (type, alignment, duplicate name, nrows < 0), GPL_E_NOMEM. */
+gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nrows, int32_t ncols,
+                            const gpl_column* cols, uint32_t flags);
+
+/* Run one BUILD segment (scan -> filter -> probe earlier hash tables ->
+ * insert): open addressing, linear probing, power-of-two slots sized
+ * exactly from a device-side count pass (load <= 0.5). Asynchronous; later
+ * segments see the table by stream order. *ht_id receives the table's id
+ * (also addressable by name from plan texts). A table of the same name is
+ * replaced. Errors: GPL_E_PLAN, GPL_E_STATE (unknown table/column/hash table).
+ * Duplicate keys are detected on device and reported by the next
+ * gpl_fetch_result (GPL_E_DUPKEY) or gpl_sync(). */
+gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32_t* ht_id);
+
+/* Run the PROBE segment (the fused pipeline: TMA-staged tiles -> filter ->
+ * survivor queue -> probe(s) -> where -> group-by aggregate; no
+ * inter-operator HBM traffic). tile_rows = 0 lets the A9 cost model choose
+ * Δ; otherwise it is rounded up to a multiple of the stage rows.
+ * Asynchronous on the ctx stream. Errors: GPL_E_PLAN, GPL_E_STATE,
+ * GPL_E_OVERFLOW (value bound not provably exact). */
+gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows);
+
+/* Same plan, executed kernel-at-a-time with every operator's output
+ * materialised in HBM: the paper's KBE baseline (§2.2, Fig 7). Same
+ * result contract; stats.op_pass holds the same counts. For comparison only. */
+gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment);
+
+/* Synchronise the stream and return the last run's result (host decode of
+ * the int128 partials; empty groups dropped; ordered by key). Device error
+ * flags latched during builds/run are returned here (GPL_E_DUPKEY,
+ * GPL_E_DOMAIN, GPL_E_OVERFLOW). GPL_E_CAPACITY if out->cap_groups is too
+ * small (out->n_groups then holds the needed rows). */
+gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out);
+
+/* Raw dense partial aggregates of the last run, for a cross-GPU merge:
+ * n_groups_declared x n_aggs int128 (lo, hi), row-major. Copied
+ * (stream-ordered, asynchronous) into `dst` (device pointer if
+ * dst_on_device, else host; then the call synchronises). *nbytes = size.
+ * GPL_E_CAPACITY if cap_bytes is too small. */
+gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_device, size_t cap_bytes,
+                              size_t* nbytes);
+
+/* Decode merged partials (host memory, the layout above, for the plan of the
+ * context's last run) into out, exactly like gpl_fetch_result. */
+gpl_status gpl_decode_partials(gpl_ctx* ctx, const void* host_partials, size_t nbytes,
+                               gpl_result* out);
+
+/* Fixed-order exact int128 sum of `nranks` partial vectors laid out back to
+ * back in host memory (the all-gather output): out[i] = sum_r in[r][i].
+ * Pure host function (no context). */
+gpl_status gpl_merge_partials(const void* gathered, int32_t nranks, size_t nbytes_each, void* out);
+
+/* Synchronise the ctx stream; returns latched device errors. */
+gpl_status gpl_sync(gpl_ctx* ctx);
+
+/* A9: the B200 re-derivation of the paper's model (Eqs 2-9) for
+ * `probe_segment` over n_rows fact rows (n_rows <= 0: the loaded table).
+ * Fills the chosen configuration and its predicted time. */
+gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t n_rows,
+                                gpl_model_report* out);
+
+/* Tuning knobs (tests / sweeps): "stage_rows", "ring_depth",
+ * "consumer_warps", "ctas_per_sm", "probe_split" (-1 = auto), "hash_load_pct".
+ * value < 0 restores automatic selection. */
+gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value);
+
+/* Validate a plan segment against the loaded tables (host only). */
+gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment);
+
+/* Message of the last failed call on ctx (ctx-owned, valid until the next
+ * call). gpl_last_error(NULL) reports gpl_create failures. */
+const char* gpl_last_error(const gpl_ctx* ctx);
+
+/* "gpl-b200 <version> sm_100a". */
+const char* gpl_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GPL_H */

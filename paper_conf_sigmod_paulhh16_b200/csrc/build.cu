@@ -1,0 +1,280 @@
+// build.cu — A1 build segment: scan a build relation through its filters and
+// probes into earlier hash tables, then insert key -> payload into an
+// open-addressing, linear-probing, power-of-two table (load <= load_pct).
+//
+// Paper: "We implement the simple hash join with two phases, i.e., hash build
+// and hash probe ... it requires a blocking barrier after hash build"
+// (§3.2). The barrier is stream order: every later segment is
+// enqueued after this one. Hash tables are the only materialised segment
+// output.
+//
+// Sizing is exact and stays on the device: a count pass accumulates the
+// number of qualifying rows and their key range into the table's header; its
+// last block computes nslots = next_pow2(count * 100 / load_pct) and the
+// ordered-hash multiplier. The clear and insert kernels read the header, so
+// the whole build is asynchronous (no host round trip).
+#include <climits>
+
+#include "device_common.cuh"
+#include "kernels.h"
+
+namespace gpl {
+namespace {
+
+constexpr int kThreads = 256;
+
+__device__ __forceinline__ long long sel_slot(const long long (&s)[MAXP], int i) {
+  long long v = s[0];
+#pragma unroll
+  for (int k = 1; k < MAXP; k++) v = (i == k) ? s[k] : v;
+  return v;
+}
+
+// Evaluate one build row: filters, probes into earlier tables, key and payload.
+__device__ __forceinline__ bool build_row(const BuildDesc& d, const HTP* src, long long row,
+                                          unsigned long long* key, long long* payload) {
+  for (int f = 0; f < d.nfilt; f++) {
+    const Filt& F = d.filt[f];
+    if (!filt_pass(F, ld_col_global(d.col[F.ref], d.colw[F.ref], row))) return false;
+  }
+  long long slot[MAXP] = {0, 0, 0, 0};
+#pragma unroll
+  for (int p = 0; p < MAXP; p++) {
+    if (p < d.nprobe) {
+      const Probe& P = d.probe[p];
+      unsigned long long k = (uint32_t)ld_col_global(d.col[P.k1], d.colw[P.k1], row);
+      if (P.k2 >= 0) k = (k << 32) | (uint32_t)ld_col_global(d.col[P.k2], d.colw[P.k2], row);
+      long long v = 0;
+      if (!ht_probe(src[P.ht], k, &v)) return false;  // inner / semi: a miss drops the row
+      slot[p] = v;
+    }
+  }
+  unsigned long long k = (uint32_t)ld_col_global(d.col[d.k1], d.colw[d.k1], row);
+  if (d.k2 >= 0) k = (k << 32) | (uint32_t)ld_col_global(d.col[d.k2], d.colw[d.k2], row);
+  *key = k;
+  long long pay = 0;
+  if (d.pay_kind == PAY_COL) pay = ld_col_global(d.col[d.pay_ref], d.colw[d.pay_ref], row);
+  else if (d.pay_kind == PAY_SLOT) pay = sel_slot(slot, d.pay_ref);
+  else if (d.pay_kind == PAY_YEARCOL) pay = (int)ld_col_global(d.col[d.pay_ref], d.colw[d.pay_ref], row) / 10000;
+  *payload = pay;
+  return true;
+}
+
+__device__ __forceinline__ void finalize_header(HTHeader* h, unsigned long long count, long long kmin,
+                                                long long kmax, long long cap_slots, int load_pct) {
+  unsigned long long need = (count * 100ull + (unsigned long long)load_pct - 1) / (unsigned long long)load_pct;
+  uint32_t log2 = 4;
+  while ((1ull << log2) < need) log2++;
+  while ((1ll << log2) > cap_slots && log2 > 4) log2--;
+  const unsigned long long nslots = 1ull << log2;
+  if (count == 0) { kmin = 0; kmax = 0; }
+  const unsigned long long range = (unsigned long long)(kmax - kmin) + 1ull;
+  h->count = count;
+  h->kmin = kmin;
+  h->kmax = kmax;
+  h->mult = (nslots << 32) / range;
+  h->log2 = log2;
+  h->mask = (uint32_t)(nslots - 1);
+}
+
+__global__ void header_init_kernel(HTHeader* h) {
+  h->acc_count = 0;
+  h->acc_kmin = LLONG_MAX;
+  h->acc_kmax = LLONG_MIN;
+  h->done = 0;
+  h->count = 0;
+  h->kmin = h->kmax = 0;
+  h->mult = 1ull << 32;
+  h->log2 = 4;
+  h->mask = 15;
+}
+
+__global__ void __launch_bounds__(kThreads) build_count_kernel(const __grid_constant__ BuildDesc d) {
+  __shared__ HTP src[MAXHT];
+  __shared__ unsigned long long s_cnt;
+  __shared__ long long s_min, s_max;
+  if (threadIdx.x < d.nht) src[threadIdx.x] = load_htp(d.src[threadIdx.x]);
+  if (threadIdx.x == 0) { s_cnt = 0; s_min = LLONG_MAX; s_max = LLONG_MIN; }
+  __syncthreads();
+  unsigned long long cnt = 0;
+  long long mn = LLONG_MAX, mx = LLONG_MIN;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long row = (long long)blockIdx.x * blockDim.x + threadIdx.x; row < d.nrows; row += stride) {
+    unsigned long long k;
+    long long pay;
+    if (build_row(d, src, row, &k, &pay)) {
+      cnt++;
+      mn = min(mn, (long long)k);
+      mx = max(mx, (long long)k);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+    mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+    mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  }
+  if ((threadIdx.x & 31) == 0 && cnt) {
+    atomicAdd(&s_cnt, cnt);
+    atomicMin(&s_min, mn);
+    atomicMax(&s_max, mx);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    HTHeader* h = d.hdr;
+    if (s_cnt) {
+      atomicAdd(&h->acc_count, s_cnt);
+      atomicMin(&h->acc_kmin, s_min);
+      atomicMax(&h->acc_kmax, s_max);
+    }
+    __threadfence();
+    const uint32_t prev = atomicAdd(&h->done, 1u);
+    if (prev == gridDim.x - 1) {  // last block: publish the exact size
+      __threadfence();
+      const unsigned long long c = atomicAdd(&h->acc_count, 0ull);
+      const long long lo = atomicMin(&h->acc_kmin, LLONG_MAX);
+      const long long hi = atomicMax(&h->acc_kmax, LLONG_MIN);
+      finalize_header(h, c, lo, hi, d.cap_slots, d.load_pct);
+      h->acc_count = 0;
+      h->acc_kmin = LLONG_MAX;
+      h->acc_kmax = LLONG_MIN;
+      h->done = 0;
+      __threadfence();
+    }
+  }
+}
+
+__global__ void __launch_bounds__(kThreads) build_clear_kernel(const __grid_constant__ BuildDesc d, int has_known,
+                                                                const __grid_constant__ HTHeader known) {
+  uint32_t mask;
+  if (has_known) {
+    mask = known.mask;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      HTHeader* h = d.hdr;
+      h->count = known.count;
+      h->kmin = known.kmin;
+      h->kmax = known.kmax;
+      h->mult = known.mult;
+      h->log2 = known.log2;
+      h->mask = known.mask;
+    }
+  } else {
+    mask = d.hdr->mask;
+  }
+  const int slot_bytes = d.kind == HT_SET32 ? 4 : d.kind == HT_MAP32 ? 8 : 16;
+  const unsigned long long n16 = ((unsigned long long)mask + 1ull) * slot_bytes / 16ull;
+  uint4* p = (uint4*)d.slots;
+  const uint4 ones = make_uint4(~0u, ~0u, ~0u, ~0u);
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n16;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    p[i] = ones;
+}
+
+__global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_constant__ BuildDesc d) {
+  __shared__ HTP src[MAXHT];
+  __shared__ HTP dst;
+  if (threadIdx.x < d.nht) src[threadIdx.x] = load_htp(d.src[threadIdx.x]);
+  if (threadIdx.x == 0) {
+    HTRef r;
+    r.slots = d.slots;
+    r.hdr = d.hdr;
+    r.kind = d.kind;
+    r.hash = d.hash;
+    dst = load_htp(r);
+  }
+  __syncthreads();
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long row = (long long)blockIdx.x * blockDim.x + threadIdx.x; row < d.nrows; row += stride) {
+    unsigned long long key;
+    long long pay;
+    if (!build_row(d, src, row, &key, &pay)) continue;
+    uint32_t i = ht_home(dst, key);
+    if (d.kind == HT_MAP32) {
+      if ((uint32_t)key == EMPTY32) { atomicOr(d.err, ERR_RESERVED_KEY); continue; }
+      unsigned long long* s = (unsigned long long*)d.slots;
+      const unsigned long long nv = ((unsigned long long)(uint32_t)(int32_t)pay << 32) | (uint32_t)key;
+      for (;;) {
+        const unsigned long long old = atomicCAS(s + i, EMPTY64, nv);
+        if (old == EMPTY64) break;
+        if ((uint32_t)old == (uint32_t)key) { atomicOr(d.err, ERR_DUPKEY); break; }
+        i = (i + 1) & dst.mask;
+      }
+    } else if (d.kind == HT_SET32) {
+      if ((uint32_t)key == EMPTY32) { atomicOr(d.err, ERR_RESERVED_KEY); continue; }
+      uint32_t* s = (uint32_t*)d.slots;
+      for (;;) {
+        const uint32_t old = atomicCAS(s + i, EMPTY32, (uint32_t)key);
+        if (old == EMPTY32) break;
+        if (old == (uint32_t)key) { atomicOr(d.err, ERR_DUPKEY); break; }
+        i = (i + 1) & dst.mask;
+      }
+    } else {
+      if (key == EMPTY64) { atomicOr(d.err, ERR_RESERVED_KEY); continue; }
+      ulonglong2* s = (ulonglong2*)d.slots;
+      for (;;) {
+        const unsigned long long old = atomicCAS(&s[i].x, EMPTY64, key);
+        if (old == EMPTY64) { s[i].y = (unsigned long long)pay; break; }
+        if (old == key) { atomicOr(d.err, ERR_DUPKEY); break; }
+        i = (i + 1) & dst.mask;
+      }
+    }
+  }
+}
+
+__global__ void minmax_init_kernel(long long* out) {
+  out[0] = LLONG_MAX;
+  out[1] = LLONG_MIN;
+}
+
+__global__ void __launch_bounds__(kThreads) minmax_kernel(const char* col, int w, long long n, long long* out) {
+  long long mn = LLONG_MAX, mx = LLONG_MIN;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const long long v = ld_col_global(col, w, i);
+    mn = min(mn, v);
+    mx = max(mx, v);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+    mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMin(&out[0], mn);
+    atomicMax(&out[1], mx);
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_header_init(HTHeader* hdr, cudaStream_t s) {
+  header_init_kernel<<<1, 1, 0, s>>>(hdr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_build(const BuildDesc& d, bool trivial, const HTHeader& known, int num_sms, cudaStream_t s) {
+  long long work = d.nrows > 0 ? d.nrows : 1;
+  int grid = (int)std::min<long long>((work + kThreads - 1) / kThreads, (long long)num_sms * 8);
+  if (grid < 1) grid = 1;
+  if (!trivial) build_count_kernel<<<grid, kThreads, 0, s>>>(d);
+  long long clear_blocks = std::min<long long>((d.cap_slots * 16 / 16 + kThreads - 1) / kThreads, (long long)num_sms * 8);
+  if (trivial) {
+    const int sb = d.kind == HT_SET32 ? 4 : d.kind == HT_MAP32 ? 8 : 16;
+    clear_blocks = std::min<long long>(((long long)(known.mask + 1ull) * sb / 16 + kThreads - 1) / kThreads,
+                                       (long long)num_sms * 8);
+  }
+  if (clear_blocks < 1) clear_blocks = 1;
+  build_clear_kernel<<<(int)clear_blocks, kThreads, 0, s>>>(d, trivial ? 1 : 0, known);
+  if (d.nrows > 0) build_insert_kernel<<<grid, kThreads, 0, s>>>(d);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s) {
+  minmax_init_kernel<<<1, 1, 0, s>>>(out);
+  if (n > 0) {
+    int grid = (int)std::min<long long>((n + kThreads - 1) / kThreads, 148LL * 8);
+    minmax_kernel<<<grid, kThreads, 0, s>>>((const char*)col, width, n, out);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace gpl

@@ -1,0 +1,652 @@
+// capi.cpp — the extern "C" boundary (include/gpl.h). Argument checking,
+// column store (A0), build/run orchestration on the ctx stream, result decode
+// (A10). No exception crosses the ABI.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstring>
+#include <new>
+#include <set>
+#include <string>
+
+#include "costmodel.h"
+#include "ctx.h"
+#include "gpl.h"
+#include "kernels.h"
+#include "lower.h"
+#include "plan.h"
+
+#define GPL_API extern "C" __attribute__((visibility("default")))
+
+using namespace gpl;
+
+namespace {
+
+std::string g_create_error;
+
+gpl_status fail(gpl_ctx* ctx, gpl_status st, const std::string& msg) {
+  if (ctx) ctx->err = msg;
+  else g_create_error = msg;
+  return st;
+}
+
+#define CK(call)                                                                            \
+  do {                                                                                      \
+    cudaError_t e_ = (call);                                                                \
+    if (e_ != cudaSuccess) return fail(ctx, GPL_E_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+int type_width(int t) {
+  switch (t) {
+    case GPL_I32: case GPL_DATE32: case GPL_DICT32: return 4;
+    case GPL_I64: case GPL_DEC64: return 8;
+    default: return 0;
+  }
+}
+
+constexpr int kScratchWords = MAXOPS + 4;  // [0] tile counter, [1..MAXOPS] op_pass, [MAXOPS+1] err bits
+
+unsigned long long* op_pass_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 1; }
+unsigned int* err_ptr(gpl_ctx* ctx) { return (unsigned int*)(ctx->d_scratch + MAXOPS + 1); }
+
+gpl_status check_dev(gpl_ctx* ctx) {
+  if (!ctx) return GPL_E_ARG;
+  if (ctx->host_only) return fail(ctx, GPL_E_NODEV, "host-only context (device -1)");
+  CK(cudaSetDevice(ctx->device));
+  return GPL_OK;
+}
+
+void free_column(gpl_ctx* ctx, Column& c) {
+  if (c.owned && c.dev && !ctx->host_only) cudaFree(c.dev);
+  c.dev = nullptr;
+}
+
+// Read latched device error bits (syncs) and clear them.
+gpl_status take_device_errors(gpl_ctx* ctx) {
+  unsigned int bits = 0;
+  CK(cudaMemcpyAsync(&bits, err_ptr(ctx), sizeof(bits), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  if (bits) {
+    CK(cudaMemsetAsync(err_ptr(ctx), 0, sizeof(unsigned int), ctx->stream));
+    if (bits & ERR_DUPKEY) return fail(ctx, GPL_E_DUPKEY, "duplicate build key (joins must be FK->PK)");
+    if (bits & ERR_RESERVED_KEY) return fail(ctx, GPL_E_ARG, "a build key equals the reserved empty-slot value");
+    if (bits & ERR_DOMAIN) return fail(ctx, GPL_E_DOMAIN, "a group value fell outside its declared domain");
+    return fail(ctx, GPL_E_CAPACITY, "device capacity error");
+  }
+  return GPL_OK;
+}
+
+gpl_status decode(gpl_ctx* ctx, const unsigned long long* part, gpl_result* out) {
+  const LowerInfo& li = ctx->last.li;
+  const int G = li.ngroups_total, A = li.nagg;
+  out->n_keys = li.ngroup_dims;
+  out->n_aggs = A;
+  int rows = 0;
+  for (int g = 0; g < G; g++) {
+    const bool nonempty = part[2 * (g * A)] != 0 || part[2 * (g * A) + 1] != 0;
+    if (nonempty || !li.has_groups) rows++;
+  }
+  out->n_groups = rows;
+  if (rows > out->cap_groups) return fail(ctx, GPL_E_CAPACITY, "result capacity too small");
+  if (rows && (!out->aggs || (li.ngroup_dims && !out->keys))) return fail(ctx, GPL_E_ARG, "NULL result arrays");
+  int r = 0;
+  for (int g = 0; g < G; g++) {
+    const bool nonempty = part[2 * (g * A)] != 0 || part[2 * (g * A) + 1] != 0;
+    if (!nonempty && li.has_groups) continue;
+    for (int k = 0; k < li.ngroup_dims; k++) out->keys[r * li.ngroup_dims + k] = li.glo[k] + (g / li.gstride[k]) % li.gsize[k];
+    for (int a = 0; a < A; a++) {
+      out->aggs[(r * A + a) * 2] = (int64_t)part[2 * (g * A + a)];
+      out->aggs[(r * A + a) * 2 + 1] = (int64_t)part[2 * (g * A + a) + 1];
+    }
+    r++;
+  }
+  return GPL_OK;
+}
+
+}  // namespace
+
+GPL_API const char* gpl_version(void) { return "gpl-b200 0.1 sm_100a"; }
+
+GPL_API const char* gpl_last_error(const gpl_ctx* ctx) { return ctx ? ctx->err.c_str() : g_create_error.c_str(); }
+
+GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
+  gpl_ctx* ctx = nullptr;
+  if (!out) return fail(nullptr, GPL_E_ARG, "out is NULL");
+  *out = nullptr;
+  ctx = new (std::nothrow) gpl_ctx();
+  if (!ctx) return fail(nullptr, GPL_E_NOMEM, "host allocation failed");
+  if (device < 0) {
+    ctx->host_only = true;
+    *out = ctx;
+    return GPL_OK;
+  }
+  ctx->host_only = false;
+  ctx->device = device;
+  auto bad = [&](cudaError_t e, const char* what) {
+    std::string m = std::string(what) + ": " + cudaGetErrorString(e);
+    delete ctx;
+    return fail(nullptr, GPL_E_CUDA, m);
+  };
+  cudaError_t e;
+  if ((e = cudaSetDevice(device)) != cudaSuccess) return bad(e, "cudaSetDevice");
+  cudaDeviceProp p;
+  if ((e = cudaGetDeviceProperties(&p, device)) != cudaSuccess) return bad(e, "cudaGetDeviceProperties");
+  if (p.major < 10) {
+    delete ctx;
+    return fail(nullptr, GPL_E_CUDA, "device is not sm_100 class (this build targets sm_100a only)");
+  }
+  ctx->sms = p.multiProcessorCount;
+  ctx->smem_optin = (int)p.sharedMemPerBlockOptin;
+  ctx->l2_bytes = p.l2CacheSize;
+  if (cuda_stream) {
+    ctx->stream = (cudaStream_t)cuda_stream;
+  } else {
+    if ((e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking)) != cudaSuccess) return bad(e, "stream");
+    ctx->own_stream = true;
+  }
+  if ((e = cudaMalloc(&ctx->d_scratch, kScratchWords * sizeof(unsigned long long))) != cudaSuccess) return bad(e, "scratch");
+  if ((e = cudaMemset(ctx->d_scratch, 0, kScratchWords * sizeof(unsigned long long))) != cudaSuccess) return bad(e, "scratch");
+  if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
+  if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
+  *out = ctx;
+  return GPL_OK;
+}
+
+GPL_API void gpl_destroy(gpl_ctx* ctx) {
+  if (!ctx) return;
+  if (!ctx->host_only) {
+    cudaSetDevice(ctx->device);
+    cudaStreamSynchronize(ctx->stream);
+    for (auto& kv : ctx->tables)
+      for (auto& c : kv.second.cols) free_column(ctx, c);
+    for (auto& h : ctx->hts) {
+      if (h.slots) cudaFree(h.slots);
+      if (h.hdr) cudaFree(h.hdr);
+    }
+    if (ctx->d_scratch) cudaFree(ctx->d_scratch);
+    if (ctx->d_partials) cudaFree(ctx->d_partials);
+    if (ctx->d_minmax) cudaFree(ctx->d_minmax);
+    if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
+    if (ctx->ev0) cudaEventDestroy(ctx->ev0);
+    if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+    if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
+  }
+  delete ctx;
+}
+
+GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) {
+  if (!ctx || !key) return GPL_E_ARG;
+  std::string k = key;
+  Options& o = ctx->opt;
+  int64_t v = value;
+  if (k == "stage_rows") {
+    if (v >= 0 && (v % 32 || v < 32 || v > 8192)) return fail(ctx, GPL_E_ARG, "stage_rows: multiple of 32 in [32, 8192]");
+    o.stage_rows = v;
+  } else if (k == "ring_depth") {
+    if (v >= 0 && (v < 2 || v > 8)) return fail(ctx, GPL_E_ARG, "ring_depth in [2, 8]");
+    o.ring_depth = v;
+  } else if (k == "consumer_warps") {
+    if (v >= 0 && (v < 1 || v > 16)) return fail(ctx, GPL_E_ARG, "consumer_warps in [1, 16]");
+    o.consumer_warps = v;
+  } else if (k == "ctas_per_sm") {
+    if (v >= 0 && (v < 1 || v > 4)) return fail(ctx, GPL_E_ARG, "ctas_per_sm in [1, 4]");
+    o.ctas_per_sm = v;
+  } else if (k == "probe_split") {
+    o.probe_split = v < -1 ? -2 : v;  // -1 = after every probe, >= 0 = count, < -1 auto
+  } else if (k == "hash_load_pct") {
+    if (v >= 0 && (v < 10 || v > 90)) return fail(ctx, GPL_E_ARG, "hash_load_pct in [10, 90]");
+    o.hash_load_pct = v;
+  } else if (k == "hbm_mbs") {
+    o.hbm_gbs = v > 0 ? v / 1000.0 : -1;
+  } else {
+    return fail(ctx, GPL_E_ARG, "unknown option '" + k + "'");
+  }
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nrows, int32_t ncols,
+                                    const gpl_column* cols, uint32_t flags) {
+  if (!ctx) return GPL_E_ARG;
+  ctx->err.clear();
+  if (!table || !*table) return fail(ctx, GPL_E_ARG, "table name is empty");
+  if (nrows < 0 || nrows > ((int64_t)1 << 40)) return fail(ctx, GPL_E_ARG, "nrows out of range");
+  if (ncols < 1 || ncols > 64 || !cols) return fail(ctx, GPL_E_ARG, "ncols must be in [1, 64] with a column array");
+  if (flags != GPL_COPY && flags != GPL_BORROW) return fail(ctx, GPL_E_ARG, "flags must be GPL_COPY or GPL_BORROW");
+  std::set<std::string> names;
+  for (int i = 0; i < ncols; i++) {
+    if (!cols[i].name || !*cols[i].name) return fail(ctx, GPL_E_ARG, "column name is empty");
+    if (!names.insert(cols[i].name).second) return fail(ctx, GPL_E_ARG, std::string("duplicate column ") + cols[i].name);
+    if (!type_width(cols[i].type)) return fail(ctx, GPL_E_ARG, std::string("bad type for column ") + cols[i].name);
+    if (nrows > 0 && !cols[i].data) return fail(ctx, GPL_E_ARG, std::string("NULL data for column ") + cols[i].name);
+    if (ctx->host_only && cols[i].on_device) return fail(ctx, GPL_E_NODEV, "device data given to a host-only context");
+  }
+  Table t;
+  t.name = table;
+  t.nrows = nrows;
+  t.version = ctx->next_version++;
+  if (ctx->host_only) {
+    for (int i = 0; i < ncols; i++) {
+      Column c;
+      c.name = cols[i].name;
+      c.type = cols[i].type;
+      c.scale = cols[i].scale;
+      c.width = type_width(c.type);
+      c.host.assign((const char*)cols[i].data, (const char*)cols[i].data + nrows * c.width);
+      c.vmin = LLONG_MAX;
+      c.vmax = LLONG_MIN;
+      for (int64_t r = 0; r < nrows; r++) {
+        long long v = c.width == 4 ? (long long)((const int32_t*)c.host.data())[r] : ((const int64_t*)c.host.data())[r];
+        c.vmin = std::min<long long>(c.vmin, v);
+        c.vmax = std::max<long long>(c.vmax, v);
+      }
+      if (nrows == 0) c.vmin = c.vmax = 0;
+      t.cols.push_back(std::move(c));
+    }
+  } else {
+    gpl_status st = check_dev(ctx);
+    if (st) return st;
+    if (ctx->minmax_cap < (size_t)ncols) {
+      if (ctx->d_minmax) cudaFree(ctx->d_minmax);
+      ctx->d_minmax = nullptr;
+      ctx->minmax_cap = 0;
+      CK(cudaMalloc(&ctx->d_minmax, 64 * 2 * sizeof(long long)));
+      ctx->minmax_cap = 64;
+    }
+    auto cleanup = [&]() {
+      for (auto& c : t.cols) free_column(ctx, c);
+    };
+    for (int i = 0; i < ncols; i++) {
+      Column c;
+      c.name = cols[i].name;
+      c.type = cols[i].type;
+      c.scale = cols[i].scale;
+      c.width = type_width(c.type);
+      const int64_t need_cap = (nrows + 3) / 4 * 4;
+      const int64_t cap = cols[i].capacity_rows > 0 ? cols[i].capacity_rows : nrows;
+      bool borrow = flags == GPL_BORROW && cols[i].on_device && ((uintptr_t)cols[i].data % 16 == 0) && cap >= need_cap;
+      if (flags == GPL_BORROW && !cols[i].on_device) {
+        cleanup();
+        return fail(ctx, GPL_E_ARG, std::string("GPL_BORROW needs device data: ") + c.name);
+      }
+      if (borrow) {
+        c.dev = (char*)cols[i].data;
+        c.owned = false;
+        c.cap_rows = cap;
+      } else {
+        const int64_t rows = std::max<int64_t>(64, (nrows + 63) / 64 * 64);
+        cudaError_t e = cudaMalloc(&c.dev, (size_t)rows * c.width);
+        if (e != cudaSuccess) {
+          cleanup();
+          return fail(ctx, GPL_E_NOMEM, std::string("cudaMalloc for column ") + c.name + ": " + cudaGetErrorString(e));
+        }
+        c.owned = true;
+        c.cap_rows = rows;
+        t.cols.push_back(c);  // owned from here on (cleanup frees it)
+        if (nrows > 0)
+          CK(cudaMemcpyAsync(c.dev, cols[i].data, (size_t)nrows * c.width, cudaMemcpyDefault, ctx->stream));
+        CK(cudaMemsetAsync(c.dev + (size_t)nrows * c.width, 0, (size_t)(rows - nrows) * c.width, ctx->stream));
+        t.cols.pop_back();
+      }
+      t.cols.push_back(c);
+      CK(launch_minmax(c.dev, c.width, nrows, ctx->d_minmax + 2 * i, ctx->stream));
+    }
+    long long mm[128];
+    CK(cudaMemcpyAsync(mm, ctx->d_minmax, sizeof(long long) * 2 * ncols, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    for (int i = 0; i < ncols; i++) {
+      t.cols[i].vmin = nrows ? mm[2 * i] : 0;
+      t.cols[i].vmax = nrows ? mm[2 * i + 1] : 0;
+    }
+  }
+  auto old = ctx->tables.find(t.name);
+  if (old != ctx->tables.end()) {
+    if (!ctx->host_only) cudaStreamSynchronize(ctx->stream);
+    for (auto& c : old->second.cols) free_column(ctx, c);
+    for (auto& h : ctx->hts)
+      if (h.src_table == t.name) h.valid = false;
+  }
+  ctx->tables[t.name] = std::move(t);
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment) {
+  if (!ctx || !segment) return GPL_E_ARG;
+  ctx->err.clear();
+  Segment s;
+  std::string err;
+  if (!parse_segment(segment, &s, &err)) return fail(ctx, GPL_E_PLAN, err);
+  gpl_status st;
+  if (s.is_build) {
+    BuildDesc d;
+    HashTable shape;
+    bool trivial;
+    st = lower_build(ctx, s, &d, &shape, &trivial, &err);
+  } else {
+    PipeDesc d;
+    LowerInfo li;
+    st = lower_probe(ctx, s, choose_split(ctx, s), &d, &li, &err);
+  }
+  return st ? fail(ctx, st, err) : GPL_OK;
+}
+
+GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32_t* ht_id) {
+  if (!ctx || !build_segment) return GPL_E_ARG;
+  ctx->err.clear();
+  Segment s;
+  std::string err;
+  if (!parse_segment(build_segment, &s, &err)) return fail(ctx, GPL_E_PLAN, err);
+  if (!s.is_build) return fail(ctx, GPL_E_PLAN, "expected a build segment ('build NAME')");
+  gpl_status st;
+  BuildDesc d;
+  HashTable shape;
+  bool trivial = false;
+  if ((st = lower_build(ctx, s, &d, &shape, &trivial, &err))) return fail(ctx, st, err);
+  if (ctx->host_only) {  // dry run: register the table's shape so later segments validate
+    auto it = ctx->ht_by_name.find(s.name);
+    int idx = it == ctx->ht_by_name.end() ? (int)ctx->hts.size() : it->second;
+    if (it == ctx->ht_by_name.end()) {
+      ctx->hts.push_back(HashTable());
+      ctx->ht_by_name[s.name] = idx;
+    }
+    HashTable& H = ctx->hts[idx];
+    H = shape;
+    H.id = idx;
+    H.name = s.name;
+    H.valid = true;
+    if (ht_id) *ht_id = idx;
+    return GPL_OK;
+  }
+  if ((st = check_dev(ctx))) return st;
+  // (re)allocate the destination table
+  int idx;
+  auto it = ctx->ht_by_name.find(s.name);
+  if (it == ctx->ht_by_name.end()) {
+    idx = (int)ctx->hts.size();
+    ctx->hts.push_back(HashTable());
+    ctx->hts[idx].id = idx;
+    ctx->ht_by_name[s.name] = idx;
+  } else {
+    idx = it->second;
+  }
+  HashTable& H = ctx->hts[idx];
+  const int sb = shape.kind == HT_SET32 ? 4 : shape.kind == HT_MAP32 ? 8 : 16;
+  if (!H.slots || H.cap_slots * (H.kind == HT_SET32 ? 4 : H.kind == HT_MAP32 ? 8 : 16) < shape.cap_slots * sb) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (H.slots) cudaFree(H.slots);
+    H.slots = nullptr;
+    cudaError_t e = cudaMalloc(&H.slots, (size_t)shape.cap_slots * sb);
+    if (e != cudaSuccess) {
+      H.valid = false;
+      return fail(ctx, GPL_E_NOMEM, std::string("hash table allocation: ") + cudaGetErrorString(e));
+    }
+    H.cap_slots = shape.cap_slots;
+  } else {
+    H.cap_slots = H.cap_slots * (H.kind == HT_SET32 ? 4 : H.kind == HT_MAP32 ? 8 : 16) / sb;
+  }
+  if (!H.hdr) {
+    CK(cudaMalloc(&H.hdr, sizeof(HTHeader)));
+    CK(launch_header_init(H.hdr, ctx->stream));
+  }
+  H.name = s.name;
+  H.kind = shape.kind;
+  H.hash = shape.hash;
+  H.key_arity = shape.key_arity;
+  H.has_payload = shape.has_payload;
+  H.pay_min = shape.pay_min;
+  H.pay_max = shape.pay_max;
+  H.src_table = shape.src_table;
+  H.src_version = shape.src_version;
+  d.slots = H.slots;
+  d.hdr = H.hdr;
+  d.cap_slots = H.cap_slots;
+  d.err = err_ptr(ctx);
+  HTHeader known{};
+  if (trivial) {
+    const Table& T = ctx->tables[s.table];
+    long long kmin = 0, kmax = 0;
+    if (H.key_arity == 1) {
+      const Column* kc = T.find(s.key[0]);
+      kmin = (long long)(uint32_t)kc->vmin;
+      kmax = (long long)(uint32_t)kc->vmax;
+      if (kc->vmin < 0) { kmin = 0; kmax = 0xFFFFFFFFll; }  // negative keys: whole unsigned range
+    }
+    known = trivial_header(T.nrows, kmin, kmax, H.cap_slots, d.load_pct);
+  }
+  CK(launch_build(d, trivial, known, ctx->sms, ctx->stream));
+  H.valid = true;
+  if (ht_id) *ht_id = H.id;
+  return GPL_OK;
+}
+
+static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows, PipeDesc* d, LowerInfo* li,
+                              Config* cfg, Segment* seg) {
+  std::string err;
+  if (!parse_segment(text, seg, &err)) return fail(ctx, GPL_E_PLAN, err);
+  if (seg->is_build) return fail(ctx, GPL_E_PLAN, "expected a probe segment ('run TABLE')");
+  gpl_status st = lower_probe(ctx, *seg, choose_split(ctx, *seg), d, li, &err);
+  if (st) return fail(ctx, st, err);
+  auto lit = ctx->lambda.find(seg->text);
+  if (lit != ctx->lambda.end()) li->lambda = lit->second;
+  for (int i = 0; i < d->nht; i++) {
+    for (auto& h : ctx->hts)
+      if (h.slots == d->ht[i].slots)
+        li->ht_bytes[i] = h.cap_slots * (h.kind == HT_SET32 ? 4 : h.kind == HT_MAP32 ? 8 : 16) / 2;
+  }
+  if (tile_rows < 0) return fail(ctx, GPL_E_ARG, "tile_rows must be >= 0");
+  if (!choose_config(ctx, *d, *li, d->nrows, tile_rows, cfg, &err)) return fail(ctx, GPL_E_ARG, err);
+  apply_config(d, *li, *cfg);
+  return GPL_OK;
+}
+
+static gpl_status ensure_partials(gpl_ctx* ctx, size_t bytes) {
+  if (ctx->partials_cap < bytes) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ctx->d_partials) cudaFree(ctx->d_partials);
+    ctx->d_partials = nullptr;
+    ctx->partials_cap = 0;
+    cudaError_t e = cudaMalloc(&ctx->d_partials, bytes);
+    if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("partials: ") + cudaGetErrorString(e));
+    ctx->partials_cap = bytes;
+  }
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows) {
+  if (!ctx || !probe_segment) return GPL_E_ARG;
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  PipeDesc d;
+  LowerInfo li;
+  Config cfg;
+  Segment seg;
+  if ((st = prepare_run(ctx, probe_segment, tile_rows, &d, &li, &cfg, &seg))) return st;
+  const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
+  if ((st = ensure_partials(ctx, pbytes))) return st;
+  d.partials = ctx->d_partials;
+  d.tile_counter = ctx->d_scratch;
+  d.op_pass = op_pass_ptr(ctx);
+  d.err = err_ptr(ctx);
+  CK(cudaMemsetAsync(ctx->d_partials, 0, pbytes, ctx->stream));
+  CK(cudaMemsetAsync(ctx->d_scratch, 0, (1 + MAXOPS) * sizeof(unsigned long long), ctx->stream));
+  CK(cudaEventRecord(ctx->ev0, ctx->stream));
+  CK(launch_pipeline(d, cfg.grid, ctx->stream));
+  CK(cudaEventRecord(ctx->ev1, ctx->stream));
+  LastRun& L = ctx->last;
+  L.valid = true;
+  L.kbe = false;
+  L.text = seg.text;
+  L.desc = d;
+  L.li = li;
+  L.timed = true;
+  gpl_stats& S = L.stats;
+  S = gpl_stats{};
+  S.rows_scanned = d.nrows;
+  S.tile_rows_used = d.tile_rows;
+  S.stage_rows = d.stage_rows;
+  S.ring_depth = d.depth;
+  S.consumer_warps = d.nwarps;
+  S.grid = cfg.grid;
+  S.n_ops = li.nops;
+  S.probe_split = d.nsprobe;
+  S.predicted_ms = cfg.pred_ms;
+  S.bytes_scanned = (double)d.nrows * li.bytes_per_row;
+  S.agg_mode = d.agg_mode;
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
+  if (!ctx || !probe_segment) return GPL_E_ARG;
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  PipeDesc d;
+  LowerInfo li;
+  Config cfg;
+  Segment seg;
+  if ((st = prepare_run(ctx, probe_segment, 0, &d, &li, &cfg, &seg))) return st;
+  const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
+  if ((st = ensure_partials(ctx, pbytes))) return st;
+  d.partials = ctx->d_partials;
+  d.tile_counter = ctx->d_scratch;
+  d.op_pass = op_pass_ptr(ctx);
+  d.err = err_ptr(ctx);
+  CK(cudaMemsetAsync(ctx->d_partials, 0, pbytes, ctx->stream));
+  CK(cudaMemsetAsync(ctx->d_scratch, 0, (1 + MAXOPS) * sizeof(unsigned long long), ctx->stream));
+  double inter = 0;
+  CK(cudaEventRecord(ctx->ev0, ctx->stream));
+  CK(run_kbe(d, ctx->sms, ctx->stream, &inter));
+  CK(cudaEventRecord(ctx->ev1, ctx->stream));
+  LastRun& L = ctx->last;
+  L.valid = true;
+  L.kbe = true;
+  L.text = seg.text;
+  L.desc = d;
+  L.li = li;
+  L.timed = true;
+  gpl_stats& S = L.stats;
+  S = gpl_stats{};
+  S.rows_scanned = d.nrows;
+  S.n_ops = li.nops;
+  S.probe_split = -1;
+  S.bytes_scanned = (double)d.nrows * li.bytes_per_row;
+  S.agg_mode = AGG_GLOBAL;
+  S.kbe = 1;
+  S.intermediate_bytes = inter;
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_sync(gpl_ctx* ctx) {
+  if (!ctx) return GPL_E_ARG;
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  CK(cudaStreamSynchronize(ctx->stream));
+  return take_device_errors(ctx);
+}
+
+GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
+  if (!ctx || !out) return GPL_E_ARG;
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run to fetch");
+  const LowerInfo& li = ctx->last.li;
+  std::vector<unsigned long long> part((size_t)li.ngroups_total * li.nagg * 2);
+  unsigned long long ops[MAXOPS];
+  CK(cudaMemcpyAsync(part.data(), ctx->d_partials, part.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaMemcpyAsync(ops, op_pass_ptr(ctx), sizeof(ops), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  gpl_stats& S = ctx->last.stats;
+  if (ctx->last.timed) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1) == cudaSuccess) S.kernel_ms = ms;
+  }
+  for (int i = 0; i < MAXOPS && i < 16; i++) S.op_pass[i] = (int64_t)ops[i];
+  // λ cache for the model / split choice (cumulative pass fraction after each op)
+  if (!ctx->last.kbe && S.rows_scanned > 0) {
+    std::vector<double> lam;
+    for (int i = 0; i < li.nops; i++) lam.push_back((double)ops[i] / (double)S.rows_scanned);
+    ctx->lambda[ctx->last.text] = lam;
+  }
+  if ((st = take_device_errors(ctx))) {
+    out->stats = S;
+    return st;
+  }
+  out->stats = S;
+  return decode(ctx, part.data(), out);
+}
+
+GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_device, size_t cap_bytes, size_t* nbytes) {
+  if (!ctx || !nbytes) return GPL_E_ARG;
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run");
+  const size_t b = (size_t)ctx->last.li.ngroups_total * ctx->last.li.nagg * 16;
+  *nbytes = b;
+  if (cap_bytes < b || !dst) return fail(ctx, GPL_E_CAPACITY, "partials buffer too small");
+  CK(cudaMemcpyAsync(dst, ctx->d_partials, b, dst_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                     ctx->stream));
+  if (!dst_on_device) CK(cudaStreamSynchronize(ctx->stream));
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_decode_partials(gpl_ctx* ctx, const void* host_partials, size_t nbytes, gpl_result* out) {
+  if (!ctx || !host_partials || !out) return GPL_E_ARG;
+  if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run (the plan of the last run defines the layout)");
+  const size_t b = (size_t)ctx->last.li.ngroups_total * ctx->last.li.nagg * 16;
+  if (nbytes != b) return fail(ctx, GPL_E_ARG, "partials size does not match the last run's plan");
+  out->stats = ctx->last.stats;
+  return decode(ctx, (const unsigned long long*)host_partials, out);
+}
+
+GPL_API gpl_status gpl_merge_partials(const void* gathered, int32_t nranks, size_t nbytes_each, void* out) {
+  if (!gathered || !out || nranks < 1 || nbytes_each % 16) return GPL_E_ARG;
+  const size_t n = nbytes_each / 16;
+  const unsigned long long* in = (const unsigned long long*)gathered;
+  unsigned long long* o = (unsigned long long*)out;
+  for (size_t i = 0; i < n; i++) {
+    unsigned __int128 acc = 0;
+    for (int r = 0; r < nranks; r++) {  // fixed order: rank 0, 1, ...
+      const unsigned long long* p = in + (size_t)r * n * 2 + 2 * i;
+      acc += ((unsigned __int128)p[1] << 64) | p[0];
+    }
+    o[2 * i] = (unsigned long long)acc;
+    o[2 * i + 1] = (unsigned long long)(acc >> 64);
+  }
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t n_rows, gpl_model_report* out) {
+  if (!ctx || !probe_segment || !out) return GPL_E_ARG;
+  ctx->err.clear();
+  Segment s;
+  std::string err;
+  if (!parse_segment(probe_segment, &s, &err)) return fail(ctx, GPL_E_PLAN, err);
+  PipeDesc d;
+  LowerInfo li;
+  gpl_status st = lower_probe(ctx, s, choose_split(ctx, s), &d, &li, &err);
+  if (st) return fail(ctx, st, err);
+  auto lit = ctx->lambda.find(s.text);
+  if (lit != ctx->lambda.end()) li.lambda = lit->second;
+  for (int i = 0; i < d.nht; i++)
+    for (auto& h : ctx->hts)
+      if (h.slots == d.ht[i].slots) li.ht_bytes[i] = h.cap_slots * (h.kind == HT_SET32 ? 4 : h.kind == HT_MAP32 ? 8 : 16) / 2;
+  Config c;
+  const int64_t N = n_rows > 0 ? n_rows : d.nrows;
+  if (!choose_config(ctx, d, li, N, 0, &c, &err)) return fail(ctx, GPL_E_ARG, err);
+  out->tile_rows = c.tile_rows;
+  out->stage_rows = c.stage_rows;
+  out->ring_depth = c.depth;
+  out->consumer_warps = c.warps;
+  out->grid = c.grid;
+  out->predicted_ms = c.pred_ms;
+  out->t_stream_ms = c.t_stream_ms;
+  out->t_probe_ms = c.t_probe_ms;
+  out->t_tail_ms = c.t_tail_ms;
+  out->t_launch_ms = c.t_launch_ms;
+  out->bw_gbs = c.bw_gbs;
+  out->smem_bytes = c.smem;
+  out->feasible = c.feasible;
+  return GPL_OK;
+}

@@ -1,0 +1,158 @@
+// common.h — POD descriptors shared by the host lowering (plan.cpp) and the
+// sm_100a kernels (build.cu, pipeline.cu, kbe.cu). No torch, no CUDA types.
+#pragma once
+#include <cstdint>
+
+namespace gpl {
+
+constexpr int MAXC = 8;      // staged / scanned columns per segment
+constexpr int MAXF = 4;      // filters
+constexpr int MAXP = 4;      // probes
+constexpr int MAXR = 3;      // where-residuals
+constexpr int MAXG = 3;      // group-by dimensions
+constexpr int MAXA = 4;      // aggregates (agg 0 = COUNT)
+constexpr int MAXQ = 12;     // survivor-queue fields
+constexpr int MAXHT = 8;     // hash tables referenced by one segment
+constexpr int MAXTERM = 2;   // value = term +/- term
+constexpr int MAXFACT = 3;   // factors per term
+constexpr int MAXOPS = 16;   // op_pass counters
+constexpr int QCAP = 64;     // survivor-queue entries per warp (>= 2 packets)
+
+constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;
+constexpr unsigned long long EMPTY64 = 0xFFFFFFFFFFFFFFFFull;
+
+// Device error bits (latched, returned at fetch/sync).
+enum : uint32_t { ERR_DOMAIN = 1u, ERR_DUPKEY = 2u, ERR_RESERVED_KEY = 4u, ERR_CAPACITY = 8u };
+
+// ---- filters: x passes RANGE iff lo <= x <= hi; MASK iff 0 <= x < 64 and bit x of mask; NE iff x != lo
+enum : int32_t { F_RANGE = 0, F_MASK = 1, F_NE = 2 };
+struct Filt {
+  int32_t kind, ref;  // ref: stage column (pipeline) / scanned column (build) / field (residual)
+  int64_t lo, hi;
+  uint64_t mask;
+};
+
+// ---- hash tables (open addressing, linear probing, power-of-two slots)
+enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2 };  // 4 B {key}, 8 B {key,payload}, 16 B {key64,payload64}
+enum : int32_t { H_MULT = 0, H_ORDERED = 1 };
+
+// Device-resident header, written by the build's count and size kernels and
+// read by every probing kernel's prologue (sizing is exact and on-device).
+struct HTHeader {
+  unsigned long long count;  // rows that reached the insert step
+  long long kmin, kmax;      // inserted key range (ordered hash)
+  unsigned long long mult;   // ordered hash: slot = ((key-kmin)*mult) >> 32
+  uint32_t log2, mask;       // nslots = mask + 1 = 1 << log2
+  // count-pass accumulators; the count kernel's last block publishes them
+  // into the fields above and resets them (so no per-build init launch).
+  unsigned long long acc_count;
+  long long acc_kmin, acc_kmax;
+  uint32_t done, pad;
+};
+
+struct HTRef {
+  const void* slots;
+  const HTHeader* hdr;
+  int32_t kind, hash;
+};
+
+// ---- probes
+enum : int32_t { P_INNER = 0, P_SEMI = 1, P_MARK = 2 };
+struct Probe {
+  int32_t ht;         // index into the segment's HTRef table
+  int32_t kind;
+  int32_t k1, k2;     // key refs (k2 = -1: single int32 key; else composite (k1<<32)|k2)
+  int32_t out;        // ref receiving payload (INNER on MAP) or flag (MARK); -1 none
+};
+
+// ---- residual predicates on queue fields
+enum : int32_t { R_EQ = 0, R_PAIRS = 1, R_RANGE = 2, R_MASK = 3 };
+struct Resid {
+  int32_t kind, a, b, npairs;
+  int32_t pa[4], pb[4];
+  int64_t lo, hi;
+  uint64_t mask;
+};
+
+// ---- group-by: gid = sum_d (t(v_d) - lo_d) * stride_d, t = identity or year
+enum : int32_t { G_ID = 0, G_YEAR = 1 };
+struct GroupDim {
+  int32_t field, transform;
+  int32_t lo, size, stride, pad;
+};
+
+// ---- value expression: sum over terms of sign * prod(a + b * x_field)
+struct Factor {
+  int32_t field;  // -1: constant a
+  int32_t b;      // +1 / -1
+  int64_t a;
+};
+struct Term {
+  int32_t sign, nfact;
+  Factor f[MAXFACT];
+};
+
+// ---- aggregates
+enum : int32_t { A_COUNT = 0, A_SUM = 1, A_SUMIF = 2, A_SUMIFEQ = 3 };
+struct Agg {
+  int32_t kind, field;
+  int64_t c;
+};
+enum : int32_t { AGG_REG = 0, AGG_SMEM = 1, AGG_GLOBAL = 2 };
+
+// ---- survivor-queue push: field <- stage column or stage-phase probe slot
+enum : int32_t { PUSH_COL = 0, PUSH_SREG = 1 };
+struct Push {
+  int32_t kind, src;
+};
+
+// Descriptor of the fused probe-segment pipeline (kernel parameter, by value).
+struct PipeDesc {
+  // staging (A3)
+  long long nrows;
+  const char* col[MAXC];
+  int32_t colw[MAXC];
+  int32_t coloff[MAXC];  // byte offset of column c inside one ring slot
+  int32_t ncols, slot_bytes;
+  // schedule (A2)
+  long long tile_rows;
+  int32_t stage_rows, depth, nwarps, flush_each_tile;
+  // stage phase (A4 + first probes)
+  int32_t nfilt, nsprobe, nprobe, npush;
+  Filt filt[MAXF];
+  Probe probe[MAXP];     // [0, nsprobe): keys are stage columns; [nsprobe, nprobe): keys are fields
+  Push push[MAXQ];       // push[i] fills queue field i
+  int32_t nfield, nresid, ngroup, ngroups_total;
+  Resid resid[MAXR];
+  GroupDim gdim[MAXG];
+  int32_t nterm, nagg, agg_mode, nht;
+  Term term[MAXTERM];
+  Agg agg[MAXA];
+  HTRef ht[MAXHT];
+  // smem layout
+  int32_t off_queue, off_agg, off_ring, smem_bytes;
+  // outputs
+  unsigned long long* partials;      // [ngroups_total][nagg] x (lo, hi)
+  unsigned long long* tile_counter;  // zeroed before launch
+  unsigned long long* op_pass;       // [MAXOPS]
+  unsigned int* err;
+};
+
+// Descriptor of one build segment (hash_build kernels).
+enum : int32_t { PAY_NONE = 0, PAY_COL = 1, PAY_SLOT = 2, PAY_YEARCOL = 3 };
+struct BuildDesc {
+  long long nrows;
+  const char* col[MAXC];
+  int32_t colw[MAXC];
+  int32_t ncols, nfilt, nprobe, k1, k2, pay_kind, pay_ref, nht;
+  Filt filt[MAXF];
+  Probe probe[MAXP];  // inner/semi probes into earlier tables; out = slot register 0..MAXP-1
+  HTRef src[MAXHT];
+  void* slots;        // destination table
+  HTHeader* hdr;
+  long long cap_slots;
+  int32_t kind, hash, load_pct, pad;
+  unsigned int* err;
+};
+
+}  // namespace gpl

@@ -1,0 +1,37 @@
+// costmodel.h — A9: tile-size / pipeline-shape selection, the B200
+// re-derivation of the paper's analytical model (§4, Eqs 1-9,
+// P:205-315) — see costmodel.cpp for the term-by-term mapping.
+#pragma once
+#include <string>
+
+#include "ctx.h"
+
+namespace gpl {
+
+struct Config {
+  int64_t tile_rows = 0;
+  int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1, grid = 0, smem = 0;
+  double pred_ms = 0, t_stream_ms = 0, t_probe_ms = 0, t_tail_ms = 0, t_launch_ms = 0, bw_gbs = 0;
+  bool feasible = false;
+};
+
+// Shared-memory bytes of a configuration (Eq 2 feasibility input).
+int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps);
+
+// Predicted time (ms) of one configuration (Eqs 3-9 analog).
+Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t nrows, int64_t tile_rows,
+               int stage_rows, int depth, int warps, int ctas_per_sm);
+
+// Search the feasible space (Δ, stage rows, depth, consumer warps), honouring
+// options and a requested tile_rows (> 0 fixes Δ). Returns false if nothing fits.
+bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t nrows, int64_t tile_req,
+                   Config* out, std::string* err);
+
+// Fill the schedule and shared-memory layout fields of d from c.
+void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c);
+
+// Probes run before the survivor queue, from the previous run's pass
+// fractions (the paper profiles the first tile) or a heuristic.
+int choose_split(const gpl_ctx* ctx, const Segment& s);
+
+}  // namespace gpl

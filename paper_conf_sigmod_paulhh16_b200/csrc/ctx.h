@@ -1,0 +1,109 @@
+// ctx.h — the opaque gpl_ctx: column store (A0), hash tables (A1), run state.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "common.h"
+#include "gpl.h"
+#include "plan.h"
+
+namespace gpl {
+
+struct Column {
+  std::string name;
+  int type = 0, scale = 0, width = 4;
+  char* dev = nullptr;   // device base (owned or borrowed)
+  bool owned = false;
+  int64_t cap_rows = 0;
+  int64_t vmin = 0, vmax = 0;
+  std::vector<char> host;  // host-only context storage
+};
+
+struct Table {
+  std::string name;
+  int64_t nrows = 0;
+  uint64_t version = 0;
+  std::vector<Column> cols;
+  const Column* find(const std::string& n) const {
+    for (auto& c : cols)
+      if (c.name == n) return &c;
+    return nullptr;
+  }
+};
+
+struct HashTable {
+  std::string name;
+  int32_t id = -1;
+  int kind = HT_SET32, hash = H_MULT, key_arity = 1;
+  bool has_payload = false;
+  int64_t pay_min = 1, pay_max = 1;  // payload value range (validator)
+  void* slots = nullptr;
+  HTHeader* hdr = nullptr;
+  int64_t cap_slots = 0;
+  std::string src_table;
+  uint64_t src_version = 0;
+  bool valid = false;
+};
+
+// Host-side facts produced by lowering a probe segment.
+struct LowerInfo {
+  int ngroups_total = 1, nagg = 1, nops = 0, ngroup_dims = 0;
+  int glo[MAXG] = {0, 0, 0}, gsize[MAXG] = {1, 1, 1}, gstride[MAXG] = {1, 1, 1};
+  int bytes_per_row = 0;
+  long double maxabs = 0;  // bound on |value| per row
+  std::vector<std::string> op_names;
+  std::vector<int64_t> ht_bytes;  // slot bytes of each probed table
+  std::vector<int> probe_ht;      // probe index -> d.ht index
+  int nprobe = 0, nfilt = 0;
+  bool has_groups = false;
+  std::vector<double> lambda;     // cumulative pass fraction after each op (previous run)
+};
+
+struct LastRun {
+  bool valid = false;
+  std::string text;
+  PipeDesc desc{};
+  LowerInfo li;
+  gpl_stats stats{};
+  bool timed = false;
+  bool kbe = false;
+};
+
+struct Options {
+  int64_t stage_rows = -1, ring_depth = -1, consumer_warps = -1, ctas_per_sm = -1, probe_split = -2,
+          hash_load_pct = -1;
+  double hbm_gbs = -1;
+};
+
+}  // namespace gpl
+
+struct gpl_ctx {
+  int device = -1;
+  bool host_only = true;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int sms = 148, smem_optin = 232448, l2_bytes = 126 * 1024 * 1024;
+  double hbm_gbs = 6556.5;  // measured copy BW of this pool's B200s; gpl_set_option("hbm_gbs")
+  std::map<std::string, gpl::Table> tables;
+  uint64_t next_version = 1;
+  std::vector<gpl::HashTable> hts;
+  std::map<std::string, int> ht_by_name;
+  std::string err;
+  // device scratch: [0] tile counter, [1..MAXOPS] op_pass, [MAXOPS+1] error bits
+  unsigned long long* d_scratch = nullptr;
+  unsigned long long* d_partials = nullptr;
+  size_t partials_cap = 0;
+  long long* d_minmax = nullptr;
+  size_t minmax_cap = 0;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  gpl::LastRun last;
+  gpl::Options opt;
+  std::map<std::string, std::vector<double>> lambda;  // plan text -> per-op pass fraction (A9 "profile the first tile")
+  // KBE scratch (gpl_run_plan_kbe)
+  void* kbe_buf = nullptr;
+  size_t kbe_cap = 0;
+};

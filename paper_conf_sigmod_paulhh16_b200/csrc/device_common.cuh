@@ -1,0 +1,157 @@
+// device_common.cuh — device helpers shared by the build, pipeline and KBE
+// kernels: hash-table addressing/probing, exact int128 accumulation, PTX
+// wrappers for mbarrier / bulk-async copies / L2 cache policies (sm_90+, used
+// here for sm_100a).
+#pragma once
+#include <cstdint>
+
+#include "common.h"
+
+namespace gpl {
+
+// ---------------------------------------------------------------- hash tables
+// Per-kernel copy of a table's parameters (from HTRef + its device header).
+struct HTP {
+  const void* slots;
+  unsigned long long kmin, mult;
+  uint32_t mask, shift;
+  int32_t kind, hash;
+};
+
+__device__ __forceinline__ HTP load_htp(const HTRef& r) {
+  HTP p;
+  p.slots = r.slots;
+  p.kind = r.kind;
+  p.hash = r.hash;
+  const HTHeader* h = r.hdr;
+  p.mask = h->mask;
+  const uint32_t log2 = h->log2;
+  p.shift = (r.kind == HT_MAP64 ? 64u : 32u) - log2;
+  p.kmin = (unsigned long long)h->kmin;
+  p.mult = h->mult;
+  return p;
+}
+
+// Home slot. MULT: Fibonacci (multiplicative) hashing on the high bits.
+// ORDERED: monotone range scaling, so keys arriving in order (lineitem is
+// clustered by orderkey) touch consecutive slots.
+__device__ __forceinline__ uint32_t ht_home(const HTP& h, unsigned long long key) {
+  if (h.hash == H_ORDERED) return (uint32_t)(((key - h.kmin) * h.mult) >> 32) & h.mask;
+  if (h.kind == HT_MAP64) return (uint32_t)((key * 0x9E3779B97F4A7C15ull) >> h.shift);
+  return ((uint32_t)key * 0x9E3779B1u) >> h.shift;
+}
+
+// Linear probing. Returns true on hit; MAP kinds also return the payload.
+__device__ __forceinline__ bool ht_probe(const HTP& h, unsigned long long key, long long* payload) {
+  uint32_t i = ht_home(h, key);
+  if (h.kind == HT_MAP32) {
+    if ((uint32_t)key == EMPTY32) return false;
+    const unsigned long long* s = (const unsigned long long*)h.slots;
+    for (;;) {
+      const unsigned long long v = __ldg(s + i);
+      const uint32_t k = (uint32_t)v;
+      if (k == (uint32_t)key) { *payload = (long long)(int32_t)(uint32_t)(v >> 32); return true; }
+      if (k == EMPTY32) return false;
+      i = (i + 1) & h.mask;
+    }
+  } else if (h.kind == HT_SET32) {
+    if ((uint32_t)key == EMPTY32) return false;
+    const uint32_t* s = (const uint32_t*)h.slots;
+    for (;;) {
+      const uint32_t k = __ldg(s + i);
+      if (k == (uint32_t)key) { *payload = 1; return true; }
+      if (k == EMPTY32) return false;
+      i = (i + 1) & h.mask;
+    }
+  } else {
+    if (key == EMPTY64) return false;
+    const ulonglong2* s = (const ulonglong2*)h.slots;
+    for (;;) {
+      const ulonglong2 v = __ldg(s + i);
+      if (v.x == key) { *payload = (long long)v.y; return true; }
+      if (v.x == EMPTY64) return false;
+      i = (i + 1) & h.mask;
+    }
+  }
+}
+
+// ------------------------------------------------------------ exact int128
+// p[0] = low word, p[1] = high word (two's complement). Adds a signed int64.
+// Correct under concurrency: the low word wraps exactly once per carry seen
+// by the atomic that caused it.
+__device__ __forceinline__ void atomic_add_i128(unsigned long long* p, long long v) {
+  const unsigned long long lo = (unsigned long long)v;
+  const unsigned long long old = atomicAdd(p, lo);
+  const unsigned long long carry = (old + lo) < old ? 1ull : 0ull;
+  const unsigned long long hi = (v < 0 ? ~0ull : 0ull) + carry;
+  if (hi) atomicAdd(p + 1, hi);
+}
+
+__device__ __forceinline__ long long warp_sum_i64(long long v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// ------------------------------------------------------------- PTX wrappers
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(unsigned long long* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "GPL_WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra GPL_WAIT_%=;\n"
+      "}\n" ::"r"(smem_addr(bar)),
+      "r"(parity)
+      : "memory");
+}
+// 1-D bulk async copy global -> shared (TMA engine), completes on `bar` by
+// transaction bytes; L2 cache hint `policy`.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, unsigned long long* bar,
+                                         unsigned long long policy) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar)), "l"(policy)
+      : "memory");
+}
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+  unsigned long long p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+// Typed column read (4- or 8-byte column) widened to int64.
+__device__ __forceinline__ long long ld_col_global(const char* base, int w, long long row) {
+  return w == 4 ? (long long)__ldg((const int*)base + row) : __ldg((const long long*)base + row);
+}
+
+__device__ __forceinline__ bool filt_pass(const Filt& f, long long x) {
+  if (f.kind == F_RANGE) return x >= f.lo && x <= f.hi;
+  if (f.kind == F_MASK) return (unsigned long long)x < 64ull && ((f.mask >> x) & 1ull);
+  return x != f.lo;
+}
+
+}  // namespace gpl

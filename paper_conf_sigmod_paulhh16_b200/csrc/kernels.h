@@ -1,0 +1,29 @@
+// kernels.h — host launchers of the sm_100a kernels (implemented in *.cu).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "common.h"
+
+namespace gpl {
+
+// A1 build segment. `trivial` (no filter, no probe): every row is inserted,
+// so the host passes the exact header (count, key range, size) and the count
+// pass is skipped. Otherwise: count pass (+ on-device sizing) -> clear -> insert.
+cudaError_t launch_build(const BuildDesc& d, bool trivial, const HTHeader& known, int num_sms,
+                         cudaStream_t s);
+
+// Initialise a freshly allocated header (accumulators in their identity state).
+cudaError_t launch_header_init(HTHeader* hdr, cudaStream_t s);
+
+// A2-A8 fused persistent pipeline. d.smem_bytes of dynamic shared memory.
+cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s);
+
+// Column min/max (int32 or int64 column, n rows) -> out[0] = min, out[1] = max.
+cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s);
+
+// KBE baseline: kernel-at-a-time with materialisation. Returns the
+// bytes of intermediates written to HBM in *inter_bytes (host-side count).
+struct KbeBuffers;
+cudaError_t run_kbe(const PipeDesc& d, int num_sms, cudaStream_t s, double* inter_bytes);
+
+}  // namespace gpl

@@ -1,0 +1,458 @@
+// lower.cpp — semantic validation of parsed segments and lowering to the
+// device descriptors (BuildDesc / PipeDesc). Host only.
+#include "lower.h"
+
+#include <algorithm>
+#include <cmath>
+#include <map>
+#include <set>
+
+namespace gpl {
+namespace {
+
+bool is_int32(const Column& c) { return c.width == 4; }
+
+struct Range {
+  long double lo, hi;
+};
+Range mul(Range a, Range b) {
+  long double c[4] = {a.lo * b.lo, a.lo * b.hi, a.hi * b.lo, a.hi * b.hi};
+  return {*std::min_element(c, c + 4), *std::max_element(c, c + 4)};
+}
+
+}  // namespace
+
+int64_t next_pow2(int64_t x) {
+  int64_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+HTHeader trivial_header(int64_t count, long long kmin, long long kmax, int64_t cap_slots, int load_pct) {
+  HTHeader h{};
+  uint64_t need = ((uint64_t)count * 100ull + (uint64_t)load_pct - 1) / (uint64_t)load_pct;
+  uint32_t log2 = 4;
+  while ((1ull << log2) < need) log2++;
+  while ((1ll << log2) > cap_slots && log2 > 4) log2--;
+  uint64_t nslots = 1ull << log2;
+  if (count == 0) kmin = kmax = 0;
+  uint64_t range = (uint64_t)(kmax - kmin) + 1ull;
+  h.count = (unsigned long long)count;
+  h.kmin = kmin;
+  h.kmax = kmax;
+  h.mult = (nslots << 32) / range;
+  h.log2 = log2;
+  h.mask = (uint32_t)(nslots - 1);
+  h.acc_count = 0;
+  h.acc_kmin = INT64_MAX;
+  h.acc_kmax = INT64_MIN;
+  h.done = 0;
+  return h;
+}
+
+gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* shape, bool* trivial,
+                       std::string* err) {
+  *d = BuildDesc{};
+  auto tit = ctx->tables.find(s.table);
+  if (tit == ctx->tables.end()) { *err = "unknown table '" + s.table + "'"; return GPL_E_STATE; }
+  const Table& T = tit->second;
+  std::vector<const Column*> cols;
+  std::map<std::string, int> cidx;
+  std::map<std::string, int> slot_of;  // slot name -> probe index
+  for (size_t p = 0; p < s.probes.size(); p++)
+    if (!s.probes[p].out.empty()) {
+      if (T.find(s.probes[p].out)) { *err = "slot '" + s.probes[p].out + "' shadows a column"; return GPL_E_PLAN; }
+      if (slot_of.count(s.probes[p].out)) { *err = "slot '" + s.probes[p].out + "' defined twice"; return GPL_E_PLAN; }
+      slot_of[s.probes[p].out] = (int)p;
+    }
+  auto col = [&](const std::string& n, int* out) -> gpl_status {
+    auto it = cidx.find(n);
+    if (it != cidx.end()) { *out = it->second; return GPL_OK; }
+    const Column* c = T.find(n);
+    if (!c) { *err = "unknown column '" + n + "' in table " + T.name; return GPL_E_STATE; }
+    if ((int)cols.size() >= MAXC) { *err = "too many columns"; return GPL_E_PLAN; }
+    cidx[n] = (int)cols.size();
+    cols.push_back(c);
+    *out = cidx[n];
+    return GPL_OK;
+  };
+  gpl_status st;
+  d->nfilt = (int)s.filters.size();
+  for (int f = 0; f < d->nfilt; f++) {
+    const FilterIR& F = s.filters[f];
+    int ci;
+    if ((st = col(F.col, &ci))) return st;
+    d->filt[f] = Filt{F.kind, ci, F.lo, F.hi, F.mask};
+  }
+  std::map<int, int> ht_slot;  // ht id -> index in d->src
+  d->nprobe = (int)s.probes.size();
+  std::vector<const HashTable*> src_ht(d->nprobe);
+  for (int p = 0; p < d->nprobe; p++) {
+    const ProbeIR& P = s.probes[p];
+    auto hit = ctx->ht_by_name.find(P.ht);
+    if (hit == ctx->ht_by_name.end()) { *err = "unknown hash table '" + P.ht + "'"; return GPL_E_STATE; }
+    const HashTable& H = ctx->hts[hit->second];
+    if (!H.valid) { *err = "hash table '" + P.ht + "' is stale (its table was reloaded)"; return GPL_E_STATE; }
+    if (P.kind == P_MARK) { *err = "'mark' is not allowed in a build segment"; return GPL_E_PLAN; }
+    if ((int)P.keys.size() != H.key_arity) { *err = "key arity mismatch probing " + P.ht; return GPL_E_PLAN; }
+    if (!P.out.empty() && !H.has_payload) { *err = P.ht + " has no payload to bind to '" + P.out + "'"; return GPL_E_PLAN; }
+    int k1, k2 = -1;
+    if ((st = col(P.keys[0], &k1))) return st;
+    if (P.keys.size() == 2 && (st = col(P.keys[1], &k2))) return st;
+    if (!is_int32(*cols[k1]) || (k2 >= 0 && !is_int32(*cols[k2]))) { *err = "probe keys must be 32-bit columns"; return GPL_E_PLAN; }
+    if (!ht_slot.count(H.id)) {
+      int i = (int)ht_slot.size();
+      ht_slot[H.id] = i;
+      d->src[i] = HTRef{H.slots, H.hdr, H.kind, H.hash};
+    }
+    d->probe[p] = Probe{ht_slot[H.id], P.kind, k1, k2, p};
+    src_ht[p] = &H;
+  }
+  d->nht = (int)ht_slot.size();
+  if (s.key.size() > 2) { *err = "at most 2 key columns"; return GPL_E_PLAN; }
+  if ((st = col(s.key[0], &d->k1))) return st;
+  d->k2 = -1;
+  if (s.key.size() == 2 && (st = col(s.key[1], &d->k2))) return st;
+  if (!is_int32(*cols[d->k1]) || (d->k2 >= 0 && !is_int32(*cols[d->k2]))) { *err = "build keys must be 32-bit columns"; return GPL_E_PLAN; }
+  shape->key_arity = (int)s.key.size();
+  shape->has_payload = s.payload.kind != RefIR::CONST;
+  shape->pay_min = shape->pay_max = 1;
+  d->pay_kind = PAY_NONE;
+  if (shape->has_payload) {
+    if (s.payload.kind == RefIR::YEARCOL) {
+      if ((st = col(s.payload.name, &d->pay_ref))) return st;
+      if (!is_int32(*cols[d->pay_ref])) { *err = "year() needs a 32-bit date column"; return GPL_E_PLAN; }
+      d->pay_kind = PAY_YEARCOL;
+      shape->pay_min = cols[d->pay_ref]->vmin / 10000;
+      shape->pay_max = cols[d->pay_ref]->vmax / 10000;
+    } else if (slot_of.count(s.payload.name)) {
+      int p = slot_of[s.payload.name];
+      d->pay_kind = PAY_SLOT;
+      d->pay_ref = p;
+      shape->pay_min = src_ht[p]->pay_min;
+      shape->pay_max = src_ht[p]->pay_max;
+    } else {
+      if ((st = col(s.payload.name, &d->pay_ref))) return st;
+      d->pay_kind = PAY_COL;
+      shape->pay_min = cols[d->pay_ref]->vmin;
+      shape->pay_max = cols[d->pay_ref]->vmax;
+    }
+  }
+  if (shape->key_arity == 2) shape->kind = HT_MAP64;
+  else shape->kind = shape->has_payload ? HT_MAP32 : HT_SET32;
+  if (shape->kind == HT_MAP32 && (shape->pay_min < INT32_MIN || shape->pay_max > INT32_MAX)) {
+    *err = "payload range does not fit the 32-bit payload of a single-key table";
+    return GPL_E_OVERFLOW;
+  }
+  shape->hash = shape->kind == HT_MAP64 ? H_MULT : s.hash;
+  int load = ctx->opt.hash_load_pct > 0 ? (int)ctx->opt.hash_load_pct : s.load_pct;
+  d->ncols = (int)cols.size();
+  for (int c = 0; c < d->ncols; c++) {
+    d->col[c] = cols[c]->dev;
+    d->colw[c] = cols[c]->width;
+  }
+  d->nrows = T.nrows;
+  d->kind = shape->kind;
+  d->hash = shape->hash;
+  d->load_pct = load;
+  d->cap_slots = std::max<int64_t>(16, next_pow2((T.nrows * 100 + load - 1) / load));
+  shape->cap_slots = d->cap_slots;
+  shape->src_table = T.name;
+  shape->src_version = T.version;
+  *trivial = s.filters.empty() && s.probes.empty();
+  return GPL_OK;
+}
+
+gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, LowerInfo* li, std::string* err) {
+  *d = PipeDesc{};
+  *li = LowerInfo{};
+  if (s.is_build) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
+  auto tit = ctx->tables.find(s.table);
+  if (tit == ctx->tables.end()) { *err = "unknown table '" + s.table + "'"; return GPL_E_STATE; }
+  const Table& T = tit->second;
+  const int np = (int)s.probes.size();
+
+  // slots
+  std::map<std::string, int> slot_of;
+  for (int p = 0; p < np; p++)
+    if (!s.probes[p].out.empty()) {
+      const std::string& o = s.probes[p].out;
+      if (T.find(o)) { *err = "slot '" + o + "' shadows a column"; return GPL_E_PLAN; }
+      if (slot_of.count(o)) { *err = "slot '" + o + "' defined twice"; return GPL_E_PLAN; }
+      slot_of[o] = p;
+    }
+  // hash tables
+  std::vector<const HashTable*> pht(np);
+  std::map<int, int> ht_slot;
+  for (int p = 0; p < np; p++) {
+    const ProbeIR& P = s.probes[p];
+    auto hit = ctx->ht_by_name.find(P.ht);
+    if (hit == ctx->ht_by_name.end()) { *err = "unknown hash table '" + P.ht + "'"; return GPL_E_STATE; }
+    const HashTable& H = ctx->hts[hit->second];
+    if (!H.valid) { *err = "hash table '" + P.ht + "' is stale (its table was reloaded)"; return GPL_E_STATE; }
+    if ((int)P.keys.size() != H.key_arity) { *err = "key arity mismatch probing " + P.ht; return GPL_E_PLAN; }
+    if (P.kind == P_INNER && !P.out.empty() && !H.has_payload) {
+      *err = P.ht + " has no payload to bind to '" + P.out + "' (use semi or mark)";
+      return GPL_E_PLAN;
+    }
+    pht[p] = &H;
+    if (!ht_slot.count(H.id)) {
+      int i = (int)ht_slot.size();
+      if (i >= MAXHT) { *err = "too many hash tables"; return GPL_E_PLAN; }
+      ht_slot[H.id] = i;
+      d->ht[i] = HTRef{H.slots, H.hdr, H.kind, H.hash};
+      li->ht_bytes.push_back(((int64_t)1 << 20));  // refined by the model from the header at run time
+    }
+    li->probe_ht.push_back(ht_slot[H.id]);
+  }
+  d->nht = (int)ht_slot.size();
+
+  // staged columns
+  std::vector<const Column*> cols;
+  std::map<std::string, int> cidx;
+  auto stage = [&](const std::string& n, int* out) -> gpl_status {
+    auto it = cidx.find(n);
+    if (it != cidx.end()) { *out = it->second; return GPL_OK; }
+    const Column* c = T.find(n);
+    if (!c) { *err = "unknown column or slot '" + n + "'"; return GPL_E_STATE; }
+    if ((int)cols.size() >= MAXC) { *err = "too many columns (max 8)"; return GPL_E_PLAN; }
+    cidx[n] = (int)cols.size();
+    cols.push_back(c);
+    *out = cidx[n];
+    return GPL_OK;
+  };
+  gpl_status st;
+  int tmp;
+  for (auto& f : s.filters)
+    if ((st = stage(f.col, &tmp))) return st;
+  for (auto& p : s.probes)
+    for (auto& k : p.keys) {
+      if (slot_of.count(k)) { *err = "probe keys must be columns"; return GPL_E_PLAN; }
+      if ((st = stage(k, &tmp))) return st;
+      if (!is_int32(*cols[tmp])) { *err = "probe key '" + k + "' must be a 32-bit column"; return GPL_E_PLAN; }
+    }
+  for (auto& g : s.groups)
+    if (!slot_of.count(g.ref.name)) {
+      if ((st = stage(g.ref.name, &tmp))) return st;
+      if (g.ref.kind == RefIR::YEARCOL && !is_int32(*cols[tmp])) { *err = "year() needs a 32-bit date column"; return GPL_E_PLAN; }
+    } else if (g.ref.kind == RefIR::YEARCOL) {
+      *err = "year() takes a column";
+      return GPL_E_PLAN;
+    }
+  for (auto& t : s.value)
+    for (auto& f : t.f)
+      if (f.x.kind != RefIR::CONST && !slot_of.count(f.x.name))
+        if ((st = stage(f.x.name, &tmp))) return st;
+  for (auto& w : s.wheres) {
+    if (!slot_of.count(w.a) || (w.kind == R_EQ || w.kind == R_PAIRS ? !slot_of.count(w.b) : false)) {
+      *err = "where refers to an unknown slot";
+      return GPL_E_PLAN;
+    }
+  }
+  for (auto& a : s.aggs)
+    if (a.kind >= A_SUMIF && !slot_of.count(a.slot)) { *err = "agg condition refers to unknown slot '" + a.slot + "'"; return GPL_E_PLAN; }
+
+  // split (probes run before the survivor queue)
+  int sp = split;
+  if (sp < 0 && s.split_hint >= -1) sp = s.split_hint;
+  if (sp < 0) sp = s.filters.empty() ? std::min(1, np) : 0;
+  sp = std::min(sp, np);
+
+  // queue fields: columns used in the queue phase, then stage-probe slots, then queue-probe slots
+  std::vector<std::string> qcols;
+  auto need_col = [&](const std::string& n) {
+    if (std::find(qcols.begin(), qcols.end(), n) == qcols.end()) qcols.push_back(n);
+  };
+  for (int p = sp; p < np; p++)
+    for (auto& k : s.probes[p].keys) need_col(k);
+  for (auto& g : s.groups)
+    if (!slot_of.count(g.ref.name)) need_col(g.ref.name);
+  for (auto& t : s.value)
+    for (auto& f : t.f)
+      if (f.x.kind != RefIR::CONST && !slot_of.count(f.x.name)) need_col(f.x.name);
+  std::set<std::string> used_slots;
+  for (auto& w : s.wheres) {
+    used_slots.insert(w.a);
+    if (w.kind == R_EQ || w.kind == R_PAIRS) used_slots.insert(w.b);
+  }
+  for (auto& g : s.groups)
+    if (slot_of.count(g.ref.name)) used_slots.insert(g.ref.name);
+  for (auto& t : s.value)
+    for (auto& f : t.f)
+      if (f.x.kind != RefIR::CONST && slot_of.count(f.x.name)) used_slots.insert(f.x.name);
+  for (auto& a : s.aggs)
+    if (a.kind >= A_SUMIF) used_slots.insert(a.slot);
+
+  std::map<std::string, int> field;
+  int nf = 0;
+  for (auto& c : qcols) {
+    d->push[nf] = Push{PUSH_COL, cidx[c]};
+    field[c] = nf++;
+  }
+  for (int p = 0; p < sp; p++) {
+    const std::string& o = s.probes[p].out;
+    if (!o.empty() && used_slots.count(o)) {
+      if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+      d->push[nf] = Push{PUSH_SREG, p};
+      field[o] = nf++;
+    }
+  }
+  d->npush = nf;
+  for (int p = sp; p < np; p++) {
+    const std::string& o = s.probes[p].out;
+    if (!o.empty() && used_slots.count(o)) {
+      if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+      field[o] = nf++;
+    }
+  }
+  if (nf > MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+  d->nfield = std::max(nf, 1);
+
+  // slot value ranges (validator)
+  auto slot_range = [&](const std::string& n) -> Range {
+    int p = slot_of[n];
+    if (s.probes[p].kind == P_MARK) return {0, 1};
+    return {(long double)pht[p]->pay_min, (long double)pht[p]->pay_max};
+  };
+  auto ref_range = [&](const std::string& n) -> Range {
+    if (slot_of.count(n)) return slot_range(n);
+    const Column* c = cols[cidx[n]];
+    return {(long double)c->vmin, (long double)c->vmax};
+  };
+
+  // filters (stage columns)
+  d->nfilt = (int)s.filters.size();
+  for (int f = 0; f < d->nfilt; f++) {
+    const FilterIR& F = s.filters[f];
+    d->filt[f] = Filt{F.kind, cidx[F.col], F.lo, F.hi, F.mask};
+    li->op_names.push_back("filter " + F.col);
+  }
+  // probes
+  d->nprobe = np;
+  d->nsprobe = sp;
+  for (int p = 0; p < np; p++) {
+    const ProbeIR& P = s.probes[p];
+    Probe& D = d->probe[p];
+    D.ht = li->probe_ht[p];
+    D.kind = P.kind;
+    if (p < sp) {
+      D.k1 = cidx[P.keys[0]];
+      D.k2 = P.keys.size() == 2 ? cidx[P.keys[1]] : -1;
+      D.out = -1;
+    } else {
+      D.k1 = field[P.keys[0]];
+      D.k2 = P.keys.size() == 2 ? field[P.keys[1]] : -1;
+      D.out = (!P.out.empty() && field.count(P.out)) ? field[P.out] : -1;
+    }
+    li->op_names.push_back(std::string(P.kind == P_INNER ? "probe " : P.kind == P_SEMI ? "semi " : "mark ") + P.ht);
+  }
+  // where residuals
+  d->nresid = (int)s.wheres.size();
+  for (int r = 0; r < d->nresid; r++) {
+    const WhereIR& W = s.wheres[r];
+    Resid& R = d->resid[r];
+    R = Resid{};
+    R.kind = W.kind;
+    R.a = field[W.a];
+    R.b = (W.kind == R_EQ || W.kind == R_PAIRS) ? field[W.b] : -1;
+    R.npairs = (int)W.pairs.size();
+    for (int i = 0; i < R.npairs; i++) {
+      R.pa[i] = (int32_t)W.pairs[i].first;
+      R.pb[i] = (int32_t)W.pairs[i].second;
+    }
+    R.lo = W.lo;
+    R.hi = W.hi;
+    R.mask = W.mask;
+    li->op_names.push_back("where " + W.a);
+  }
+  // group-by
+  d->ngroup = (int)s.groups.size();
+  int64_t G = 1;
+  for (int g = d->ngroup - 1; g >= 0; g--) {
+    const GroupIR& Gi = s.groups[g];
+    GroupDim& D = d->gdim[g];
+    D.field = field[Gi.ref.name];
+    D.transform = Gi.ref.kind == RefIR::YEARCOL ? G_YEAR : G_ID;
+    D.lo = (int32_t)Gi.lo;
+    D.size = (int32_t)(Gi.hi - Gi.lo);
+    D.stride = (int32_t)G;
+    G *= D.size;
+    if (G > (1 << 16)) { *err = "group domain too large (max 65536 groups)"; return GPL_E_PLAN; }
+    li->glo[g] = D.lo;
+    li->gsize[g] = D.size;
+    li->gstride[g] = D.stride;
+  }
+  d->ngroups_total = (int)G;
+  li->ngroups_total = (int)G;
+  li->ngroup_dims = d->ngroup;
+  li->has_groups = d->ngroup > 0;
+  // value
+  d->nterm = (int)s.value.size();
+  Range vr{0, 0};
+  for (int t = 0; t < d->nterm; t++) {
+    const TermIR& Ti = s.value[t];
+    Term& D = d->term[t];
+    D.sign = Ti.sign;
+    D.nfact = (int)Ti.f.size();
+    Range tr{1, 1};
+    for (int f = 0; f < D.nfact; f++) {
+      const FactorIR& F = Ti.f[f];
+      Factor& X = D.f[f];
+      X.a = F.a;
+      X.b = F.b;
+      Range fr;
+      if (F.x.kind == RefIR::CONST) {
+        X.field = -1;
+        X.b = 0;
+        fr = {(long double)F.a, (long double)F.a};
+      } else {
+        X.field = field[F.x.name];
+        Range xr = ref_range(F.x.name);
+        long double e1 = F.a + F.b * xr.lo, e2 = F.a + F.b * xr.hi;
+        fr = {std::min(e1, e2), std::max(e1, e2)};
+      }
+      tr = mul(tr, fr);
+    }
+    if (Ti.sign < 0) tr = {-tr.hi, -tr.lo};
+    vr = {vr.lo + tr.lo, vr.hi + tr.hi};
+  }
+  li->maxabs = std::max(std::fabs((double)vr.lo), std::fabs((double)vr.hi));
+  if (li->maxabs >= 4.0e18L) {
+    *err = "value expression may exceed exact int64 arithmetic per row (bound " + std::to_string((double)li->maxabs) + ")";
+    return GPL_E_OVERFLOW;
+  }
+  // aggregates (agg 0 = COUNT)
+  d->nagg = (int)s.aggs.size();
+  for (int a = 0; a < d->nagg; a++) {
+    const AggIR& A = s.aggs[a];
+    d->agg[a] = Agg{A.kind, A.kind >= A_SUMIF ? field[A.slot] : -1, A.c};
+  }
+  li->nagg = d->nagg;
+  // staged columns
+  d->ncols = (int)cols.size();
+  int bpr = 0;
+  for (int c = 0; c < d->ncols; c++) {
+    d->col[c] = cols[c]->dev;
+    d->colw[c] = cols[c]->width;
+    bpr += cols[c]->width;
+  }
+  li->bytes_per_row = bpr;
+  d->nrows = T.nrows;
+  li->nfilt = d->nfilt;
+  li->nprobe = np;
+  li->nops = d->nfilt + np + d->nresid;
+  // aggregation mode (exactness): per-row |value| <= maxabs, so any int64
+  // accumulator covering <= R rows is exact when R * maxabs < 2^62.
+  const long double lim = 4.6e18L;
+  const long double total = (long double)std::max<int64_t>(T.nrows, 1) * std::max<long double>(li->maxabs, 1);
+  if (d->ngroups_total == 1) {
+    d->agg_mode = AGG_REG;
+    d->flush_each_tile = total >= lim ? 1 : 0;
+  } else {
+    d->agg_mode = (total < lim && (int64_t)d->ngroups_total * d->nagg * 8 <= 48 * 1024) ? AGG_SMEM : AGG_GLOBAL;
+    d->flush_each_tile = 0;
+  }
+  return GPL_OK;
+}
+
+}  // namespace gpl

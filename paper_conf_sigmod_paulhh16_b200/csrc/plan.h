@@ -1,0 +1,87 @@
+// plan.h — plan-segment IR and parser (host).
+//
+// A query is a sequence of segments, each ending at a blocking kernel
+// (§3.1, segmentation after [23]); here:
+//   build segments: scan -> filter* -> probe* -> insert   (ends at hash build)
+//   probe segment : scan -> filter* -> probe* -> where* -> group-by aggregate
+// Grammar (one statement per line, '#' comments): DESIGN.md §4.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace gpl {
+
+struct RefIR {
+  enum Kind { COL, SLOT, YEARCOL, CONST } kind = CONST;
+  std::string name;  // column or slot name
+  int64_t c = 0;
+};
+
+struct FilterIR {
+  std::string col;
+  int kind = 0;  // F_RANGE / F_MASK / F_NE
+  int64_t lo = INT64_MIN, hi = INT64_MAX;
+  uint64_t mask = 0;
+};
+
+struct ProbeIR {
+  std::string ht;
+  int kind = 0;                   // P_INNER / P_SEMI / P_MARK
+  std::vector<std::string> keys;  // 1 or 2 columns
+  std::string out;                // slot name ("" none)
+};
+
+struct WhereIR {
+  int kind = 0;  // R_EQ / R_PAIRS / R_RANGE / R_MASK
+  std::string a, b;
+  std::vector<std::pair<int64_t, int64_t>> pairs;
+  int64_t lo = INT64_MIN, hi = INT64_MAX;
+  uint64_t mask = 0;
+};
+
+struct GroupIR {
+  RefIR ref;
+  int64_t lo = 0, hi = 0;  // domain [lo, hi)
+};
+
+struct FactorIR {
+  RefIR x;   // CONST => constant a
+  int64_t a = 0;
+  int b = 1;
+};
+struct TermIR {
+  int sign = 1;
+  std::vector<FactorIR> f;
+};
+
+struct AggIR {
+  int kind = 0;  // A_COUNT / A_SUM / A_SUMIF / A_SUMIFEQ
+  std::string slot;
+  int64_t c = 0;
+};
+
+struct Segment {
+  bool is_build = false;
+  std::string name;   // build: hash table name
+  std::string table;  // scanned table
+  std::vector<FilterIR> filters;
+  std::vector<ProbeIR> probes;
+  // build
+  std::vector<std::string> key;
+  RefIR payload;  // CONST kind => none
+  int hash = 0;   // H_MULT / H_ORDERED
+  int load_pct = 50;
+  // probe segment
+  std::vector<WhereIR> wheres;
+  std::vector<GroupIR> groups;
+  std::vector<TermIR> value;
+  std::vector<AggIR> aggs;  // agg 0 is always COUNT
+  int split_hint = -2;      // -2: auto
+  std::string text;
+};
+
+// Parse one segment. Returns false with a message (line number included).
+bool parse_segment(const std::string& text, Segment* out, std::string* err);
+
+}  // namespace gpl

@@ -1,0 +1,183 @@
+"""Query driver: the paper's five TPC-H plans plus Listing 1, as plan texts.
+
+A query is an ordered list of segments (§3.1): build segments
+ending at a blocking hash build, then one pipelined probe segment.
+Plans are hand-written (the Selinger optimizer is out of scope); string
+predicates are constant-folded to dictionary codes from the loaded catalog
+here, which is the job of a plan generator. The oracle resolves the same
+names by string comparison independently.
+
+Everything that computes runs inside libgpl.so; this module only fills plan
+templates, calls the C ABI in segment order, and finalises results on the
+host (decode keys, ratios, ORDER BY: SURVEY §8(a) A10).
+"""
+from __future__ import annotations
+
+import os
+
+from .gpl import GPL_DATE32, GPL_DEC64, GPL_DICT32, GPL_I32, Context, Result
+
+PLAN_DIR = os.path.join(os.path.dirname(os.path.abspath(__file__)), "plans")
+
+# column types of the TPC-H-shaped tables (decimals: scaled int64, scale 100)
+SCHEMA = {
+    "region": {"r_regionkey": GPL_I32, "r_name": GPL_DICT32},
+    "nation": {"n_nationkey": GPL_I32, "n_name": GPL_DICT32, "n_regionkey": GPL_I32},
+    "supplier": {"s_suppkey": GPL_I32, "s_nationkey": GPL_I32},
+    "customer": {"c_custkey": GPL_I32, "c_nationkey": GPL_I32},
+    "part": {"p_partkey": GPL_I32, "p_type": GPL_DICT32, "p_retailprice": GPL_DEC64},
+    "partsupp": {"ps_partkey": GPL_I32, "ps_suppkey": GPL_I32, "ps_supplycost": GPL_DEC64},
+    "orders": {"o_orderkey": GPL_I32, "o_custkey": GPL_I32, "o_orderdate": GPL_DATE32},
+    "lineitem": {"l_orderkey": GPL_I32, "l_partkey": GPL_I32, "l_suppkey": GPL_I32, "l_quantity": GPL_DEC64,
+                 "l_extendedprice": GPL_DEC64, "l_discount": GPL_DEC64, "l_tax": GPL_DEC64,
+                 "l_shipdate": GPL_DATE32},
+}
+
+# Query literals exactly as printed in the Listings (dates as yyyymmdd).
+DEFAULT_PARAMS = {
+    "L1": (19881101,),
+    "Q5": (19940101, 19950101),   # P:603-604, [lo, hi)
+    "Q7": (19950101, 19961231),   # P:626-627, between (inclusive)
+    "Q8": (19950101, 19961231),   # P:650-651, between (inclusive)
+    "Q9": (1000,),                # P:677, p_partKey < 1000
+    "Q14": (19950901, 19951001),  # P:688-689, [lo, hi)
+}
+QUERIES = ["L1", "Q5", "Q7", "Q8", "Q9", "Q14"]
+# fact-table (lineitem) columns each probe segment stages, for reporting
+FACT_COLUMNS = {
+    "L1": ["l_shipdate", "l_extendedprice", "l_discount", "l_tax"],
+    "Q5": ["l_suppkey", "l_orderkey", "l_extendedprice", "l_discount"],
+    "Q7": ["l_shipdate", "l_suppkey", "l_orderkey", "l_extendedprice", "l_discount"],
+    "Q8": ["l_partkey", "l_orderkey", "l_suppkey", "l_extendedprice", "l_discount"],
+    "Q9": ["l_partkey", "l_suppkey", "l_orderkey", "l_extendedprice", "l_discount", "l_quantity"],
+    "Q14": ["l_shipdate", "l_partkey", "l_extendedprice", "l_discount"],
+}
+# tables each query reads
+TABLES = {
+    "L1": ["lineitem"],
+    "Q5": ["customer", "orders", "supplier", "lineitem", "nation", "region"],
+    "Q7": ["supplier", "customer", "orders", "lineitem", "nation"],
+    "Q8": ["part", "customer", "orders", "supplier", "lineitem", "nation", "region"],
+    "Q9": ["part", "partsupp", "supplier", "orders", "lineitem", "nation"],
+    "Q14": ["part", "lineitem"],
+}
+
+
+def _nations_of_region(catalog, region_name):
+    reg = catalog.tables["region"]
+    rk = [int(k) for k, c in zip(reg["r_regionkey"], reg["r_name"]) if catalog.r_name[int(c)] == region_name]
+    nat = catalog.tables["nation"]
+    return [int(k) for k, r in zip(nat["n_nationkey"], nat["n_regionkey"]) if int(r) in rk]
+
+
+def _nation_key(catalog, name):
+    nat = catalog.tables["nation"]
+    for k, c in zip(nat["n_nationkey"], nat["n_name"]):
+        if catalog.n_name[int(c)] == name:
+            return int(k)
+    raise KeyError(name)
+
+
+def plan_params(query: str, catalog, params=None) -> dict:
+    """Template values: Listing literals + names constant-folded via the catalog."""
+    p = tuple(params) if params is not None else DEFAULT_PARAMS[query]
+    if query == "L1":
+        return {"date_le": p[0]}
+    if query == "Q5":
+        return {"asia": ",".join(map(str, _nations_of_region(catalog, "ASIA"))), "od_lo": p[0],
+                "od_hi_incl": p[1] - 1}
+    if query == "Q7":
+        n1, n2 = _nation_key(catalog, "FRANCE"), _nation_key(catalog, "GERMANY")
+        return {"n1": n1, "n2": n2, "nlo": min(n1, n2), "nhi": max(n1, n2) + 1, "sd_lo": p[0], "sd_hi": p[1],
+                "ylo": p[0] // 10000, "yhi": p[1] // 10000 + 1}
+    if query == "Q8":
+        return {"eas": catalog.p_type.index("ECONOMY ANODIZED STEEL"),
+                "america": ",".join(map(str, _nations_of_region(catalog, "AMERICA"))),
+                "brazil": _nation_key(catalog, "BRAZIL"), "od_lo": p[0], "od_hi": p[1],
+                "ylo": p[0] // 10000, "yhi": p[1] // 10000 + 1}
+    if query == "Q9":
+        return {"p_bound": p[0]}
+    if query == "Q14":
+        promo = [i for i, s in enumerate(catalog.p_type) if s.startswith("PROMO")]
+        lo, hi = (min(promo), max(promo)) if promo else (1, 0)
+        if promo and promo != list(range(lo, hi + 1)):
+            raise ValueError("p_type dictionary must be sorted (PROMO% as one code range)")
+        return {"promo_lo": lo, "promo_hi": hi, "sd_lo": p[0], "sd_hi_incl": p[1] - 1}
+    raise KeyError(query)
+
+
+def plan_text(query: str, catalog, params=None) -> str:
+    with open(os.path.join(PLAN_DIR, query.lower() + ".plan")) as f:
+        return f.read().format(**plan_params(query, catalog, params))
+
+
+def segments(text: str) -> list:
+    """Split a plan into segments at 'build NAME' / 'run TABLE' lines."""
+    segs, cur = [], []
+    for line in text.splitlines():
+        head = line.strip().split()
+        if head and head[0] in ("build", "run") and any(x.strip() and not x.strip().startswith("#") for x in cur):
+            segs.append("\n".join(cur))
+            cur = []
+        cur.append(line)
+    if any(x.strip() and not x.strip().startswith("#") for x in cur):
+        segs.append("\n".join(cur))
+    return segs
+
+
+def load_database(ctx: Context, db, tables=None, borrow=False):
+    """Load tables (dict of column arrays / tensors) into the context's column store."""
+    for t in tables or db.tables.keys():
+        if t not in db.tables:
+            continue
+        cols = db.tables[t]
+        ctx.load_columns(t, cols, types={c: SCHEMA[t][c] for c in cols if c in SCHEMA.get(t, {})}, borrow=borrow)
+
+
+def run_segments(ctx: Context, text: str, tile_rows: int = 0, kbe: bool = False):
+    """Enqueue every segment in order (asynchronous)."""
+    segs = segments(text)
+    for s in segs[:-1]:
+        ctx.build_hash(s)
+    if kbe:
+        ctx.run_plan_kbe(segs[-1])
+    else:
+        ctx.run_plan(segs[-1], tile_rows)
+
+
+def decode_keys(query: str, result: Result, catalog) -> Result:
+    """Nation-valued group keys (nation keys) -> n_name dictionary codes, as SQL outputs n_name."""
+    nat = catalog.tables.get("nation")
+    if nat is None or query not in ("Q5", "Q7", "Q9"):
+        return result
+    name_of = {int(k): int(c) for k, c in zip(nat["n_nationkey"], nat["n_name"])}
+    dims = {"Q5": (0,), "Q7": (0, 1), "Q9": (0,)}[query]
+    keys = [tuple(name_of[v] if i in dims else v for i, v in enumerate(k)) for k in result.keys]
+    order = sorted(range(len(keys)), key=lambda i: keys[i])
+    return Result([keys[i] for i in order], [result.aggs[i] for i in order], result.stats)
+
+
+def run_query(ctx: Context, query: str, catalog, params=None, tile_rows: int = 0, kbe: bool = False) -> Result:
+    run_segments(ctx, plan_text(query, catalog, params), tile_rows, kbe)
+    return decode_keys(query, ctx.fetch_result(), catalog)
+
+
+def finalize(query: str, result: Result, catalog) -> list:
+    """A10: host ratios and ORDER BY of the Listing (ties per DESIGN.md reading R8)."""
+    rows = []
+    for k, a in zip(result.keys, result.aggs):
+        r = {"key": k, "count": a[0], "sums": a[1:]}
+        if query == "Q14":
+            r["promo_revenue"] = None if a[2] == 0 else 100.0 * a[1] / a[2]
+        if query == "Q8":
+            r["mkt_share"] = None if a[2] == 0 else a[1] / a[2]
+        rows.append(r)
+    if query == "Q5":
+        rows.sort(key=lambda r: (-r["sums"][0], r["key"]))
+    elif query == "Q7":
+        rows.sort(key=lambda r: (r["key"][2], r["key"][0], r["key"][1]))
+    elif query == "Q9":
+        rows.sort(key=lambda r: (-r["key"][1], catalog.n_name[r["key"][0]]))
+    else:
+        rows.sort(key=lambda r: r["key"])
+    return rows

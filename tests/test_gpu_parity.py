@@ -1,0 +1,170 @@
+"""CUDA path (libgpl.so, through the C ABI) vs the CPU oracle — bit-exact.
+
+Every integer the pipeline produces (group keys, COUNT(*), int128 SUMs,
+per-operator pass counts) must equal the oracle's on the same seeded inputs.
+Sizes span many stages/tiles plus ragged tails; edge cases cover empty and
+one-row inputs, every schedule knob (tile_rows, stage rows, ring depth,
+consumer warps, probe split), device error latching, and partition
+additivity of the raw partials (the multi-GPU merge path).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import tpchgen
+from golden_db import build_db, expected_keys_as_codes, load
+from paper_conf_sigmod_paulhh16_b200 import gpl, queries
+
+pytestmark = pytest.mark.gpu
+
+QUERIES = queries.QUERIES
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    c = gpl.Context(0)
+    yield c
+    c.close()
+
+
+def _gpu(ctx, db, q, params=None, tile_rows=0, tables=None):
+    queries.load_database(ctx, db, tables or queries.TABLES[q])
+    return queries.run_query(ctx, q, db, params, tile_rows)
+
+
+def _params(q):
+    return (19981101,) if q == "L1" else None
+
+
+@pytest.mark.parametrize("sf,seed", [(0.01, 20160626), (0.01, 3), (0.2, 11)])
+@pytest.mark.parametrize("q", QUERIES)
+def test_parity_small(ctx, q, sf, seed):
+    db = tpchgen.generate(sf, seed=seed)
+    r = _gpu(ctx, db, q, _params(q))
+    o = oracle.run(q, db, _params(q))
+    assert r.keys == o.keys and r.aggs == o.aggs
+    assert sum(a[0] for a in r.aggs) == (r.stats["op_pass"][-1] if r.stats["op_pass"] else db.nrows("lineitem"))
+
+
+def test_listing1_literal_empty(ctx):
+    db = tpchgen.generate(0.01, seed=tpchgen.DEFAULT_SEED)
+    r = _gpu(ctx, db, "L1")
+    assert r.keys == [()] and r.aggs == [[0, 0]]
+
+
+@pytest.mark.parametrize("q", QUERIES)
+def test_parity_sf1(ctx, q):
+    db = tpchgen.generate(1.0, seed=tpchgen.DEFAULT_SEED)
+    r = _gpu(ctx, db, q, _params(q))
+    o = oracle.run(q, db, _params(q))
+    assert r.keys == o.keys and r.aggs == o.aggs
+
+
+@pytest.mark.parametrize("fname", ["w1_listing1.json", "w2_q14.json", "w3_q5.json", "w4_q9.json"])
+def test_worked_examples(ctx, fname):
+    fx = load(fname)
+    db = build_db(fx)
+    r = _gpu(ctx, db, fx["query"], fx["params"], tables=list(db.tables))
+    assert r.keys == expected_keys_as_codes(fx, db)
+    assert r.aggs == fx["expected"]["aggs"]
+
+
+@pytest.mark.parametrize("n", [0, 1, 31, 32, 33, 1000, 4097, 65537])
+def test_ragged_and_empty(ctx, n):
+    db = tpchgen.generate(0.02, seed=5)
+    db.tables["lineitem"] = {c: v[:n].copy() for c, v in db.tables["lineitem"].items()}
+    for q in ("L1", "Q5", "Q9", "Q14"):
+        r = _gpu(ctx, db, q, _params(q))
+        o = oracle.run(q, db, _params(q))
+        assert r.keys == o.keys and r.aggs == o.aggs, (q, n)
+
+
+def test_schedule_invariance(ctx):
+    db = tpchgen.generate(0.1, seed=8)
+    expect = {q: oracle.run(q, db, _params(q)) for q in ("Q5", "Q7", "Q14", "L1")}
+    knobs = [dict(stage_rows=32, ring_depth=2, consumer_warps=1), dict(stage_rows=256, ring_depth=3, consumer_warps=4),
+             dict(stage_rows=1024, ring_depth=4, consumer_warps=8), dict(stage_rows=2048, ring_depth=2, consumer_warps=16), dict(stage_rows=4096, ring_depth=2, consumer_warps=2),
+             dict(probe_split=0), dict(probe_split=1), dict(probe_split=2), dict(probe_split=-1)]
+    try:
+        for k in knobs:
+            for key, v in k.items():
+                ctx.set_option(key, v)
+            for q, o in expect.items():
+                for tile in (0, 1, 5000, 1 << 20):
+                    r = _gpu(ctx, db, q, _params(q), tile_rows=tile)
+                    assert r.keys == o.keys and r.aggs == o.aggs, (q, k, tile)
+            for key in k:
+                ctx.set_option(key, -1 if key != "probe_split" else -2)
+    finally:
+        for key in ("stage_rows", "ring_depth", "consumer_warps"):
+            ctx.set_option(key, -1)
+        ctx.set_option("probe_split", -2)
+
+
+def test_op_pass_counts(ctx):
+    db = tpchgen.generate(0.05, seed=2)
+    r = _gpu(ctx, db, "Q14")
+    li = db.tables["lineitem"]
+    m = (li["l_shipdate"] >= 19950901) & (li["l_shipdate"] < 19951001)
+    assert r.stats["op_pass"] == [int(m.sum()), int(m.sum())]  # filter, mark (keeps rows)
+    assert r.stats["rows_scanned"] == db.nrows("lineitem")
+
+
+def test_duplicate_key_detected(ctx):
+    db = tpchgen.generate(0.01, seed=1)
+    cust = db.tables["customer"]
+    cust["c_custkey"] = cust["c_custkey"].copy()
+    cust["c_custkey"][1] = cust["c_custkey"][0]
+    cust["c_nationkey"] = np.full_like(cust["c_nationkey"], 8)
+    queries.load_database(ctx, db, queries.TABLES["Q5"])
+    queries.run_segments(ctx, queries.plan_text("Q5", db))
+    with pytest.raises(gpl.GplError) as e:
+        ctx.fetch_result()
+    assert e.value.status == gpl.GPL_E_DUPKEY
+    ctx.sync()  # error was consumed
+
+
+def test_group_domain_violation(ctx):
+    db = tpchgen.generate(0.01, seed=1)
+    text = queries.plan_text("Q5", db).replace("group s_nat 0 25", "group s_nat 0 10")
+    queries.load_database(ctx, db, queries.TABLES["Q5"])
+    queries.run_segments(ctx, text)
+    with pytest.raises(gpl.GplError) as e:
+        ctx.fetch_result()
+    assert e.value.status == gpl.GPL_E_DOMAIN
+
+
+@pytest.mark.parametrize("q", ["Q5", "Q9", "L1"])
+def test_partition_additivity_via_partials(ctx, q):
+    """Shard lineitem+orders by order range (the multi-GPU layout), run each
+    shard, merge the raw int128 partials with gpl_merge_partials: must equal
+    the oracle on the whole database (SURVEY §8(c) invariant 3)."""
+    sf, R = 0.05, 3
+    whole = tpchgen.generate(sf, seed=13)
+    parts = []
+    for r in range(R):
+        shard = tpchgen.generate(sf, seed=13, rank=r, world=R)
+        _gpu(ctx, shard, q, _params(q))
+        parts.append(ctx.fetch_partials())
+    merged = gpl.merge_partials(np.concatenate(parts), R)
+    res = queries.decode_keys(q, ctx.decode_partials(merged), whole)
+    o = oracle.run(q, whole, _params(q))
+    assert res.keys == o.keys and res.aggs == o.aggs
+
+
+def test_int128_totals(ctx):
+    """Listing 1 at scale 1e6 with values chosen so the total exceeds int64."""
+    n = 200_000
+    db = tpchgen.generate(0.01, seed=1)
+    db.tables["lineitem"] = {
+        "l_shipdate": np.full(n, 19950101, np.int32),
+        "l_extendedprice": np.full(n, 10_499_990_000, np.int64),  # ~1.05e10 cents
+        "l_discount": np.zeros(n, np.int64),
+        "l_tax": np.full(n, 8, np.int64),
+        "l_orderkey": np.zeros(n, np.int32), "l_partkey": np.zeros(n, np.int32),
+        "l_suppkey": np.zeros(n, np.int32), "l_quantity": np.zeros(n, np.int64),
+    }
+    r = _gpu(ctx, db, "L1", (19981101,))
+    expect = n * 10_499_990_000 * 100 * 108
+    assert expect > 2**63
+    assert r.aggs == [[n, expect]]

@@ -1,0 +1,101 @@
+"""Host-side logic without a GPU: the C ABI loads and exports every symbol of
+include/gpl.h; plan texts parse and validate against loaded tables (host-only
+context, device -1); the A9 model answers; the int128 partial merge is exact."""
+import re
+
+import numpy as np
+import pytest
+
+import tpchgen
+from paper_conf_sigmod_paulhh16_b200 import gpl, queries
+
+
+def test_library_exports_every_header_symbol():
+    lib = gpl.load_library()
+    header = open("include/gpl.h").read()
+    declared = set(re.findall(r"\b(gpl_[a-z_]+)\s*\(", header)) - {"gpl_status"}
+    assert declared == set(gpl.EXPORTED)
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert "sm_100a" in gpl.version()
+
+
+@pytest.fixture(scope="module")
+def host_ctx():
+    db = tpchgen.generate(0.01, seed=1)
+    ctx = gpl.Context(device=-1)
+    queries.load_database(ctx, db)
+    return ctx, db
+
+
+@pytest.mark.parametrize("q", queries.QUERIES)
+def test_plans_validate(host_ctx, q):
+    ctx, db = host_ctx
+    segs = queries.segments(queries.plan_text(q, db))
+    # a host-only context validates build segments and registers their shapes
+    for s in segs[:-1]:
+        ctx.check_plan(s)
+        ctx.build_hash(s)
+    ctx.check_plan(segs[-1])
+    with pytest.raises(gpl.GplError) as e:
+        ctx.run_plan(segs[-1])
+    assert e.value.status == gpl.GPL_E_NODEV
+
+
+def test_plan_errors(host_ctx):
+    ctx, _ = host_ctx
+    bad = {
+        "run lineitem\nfilter l_shipdate >< 3": gpl.GPL_E_PLAN,
+        "run nosuchtable\nagg count": gpl.GPL_E_STATE,
+        "run lineitem\nfilter nosuchcol <= 3": gpl.GPL_E_STATE,
+        "run lineitem\nprobe HT_X l_partkey -> x": gpl.GPL_E_STATE,
+        "build H\nscan part\nkey p_partkey\nwhere a == b": gpl.GPL_E_PLAN,
+        "run lineitem\nagg sum": gpl.GPL_E_PLAN,
+        "frobnicate": gpl.GPL_E_PLAN,
+        "build H\nscan part": gpl.GPL_E_PLAN,
+        "run lineitem\nfilter l_partkey in {64}": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup l_partkey 5 5": gpl.GPL_E_PLAN,
+        "run lineitem\nvalue l_extendedprice * l_extendedprice * l_extendedprice\nagg sum": gpl.GPL_E_OVERFLOW,
+    }
+    for text, status in bad.items():
+        with pytest.raises(gpl.GplError) as e:
+            ctx.check_plan(text)
+        assert e.value.status == status, (text, e.value)
+    ctx.check_plan("run lineitem\nfilter l_shipdate between 19950101 and 19951231\n"
+                   "group year(l_shipdate) 1995 1996\nvalue l_extendedprice * (100 - l_discount)\nagg sum")
+
+
+def test_segments_split():
+    text = "# c\nbuild A\nscan t\nkey k\n\nbuild B\nscan t\nkey k\nrun t\nagg count\n"
+    segs = queries.segments(text)
+    assert len(segs) == 3 and segs[2].strip().startswith("run t")
+
+
+def test_model_report(host_ctx):
+    ctx, db = host_ctx
+    seg = queries.segments(queries.plan_text("L1", db, (19981101,)))[-1]
+    m = ctx.choose_tile_rows(seg, 6_000_000)
+    assert m["feasible"] and m["tile_rows"] % m["stage_rows"] == 0
+    assert m["predicted_ms"] > 6_000_000 * 28 / 8e12 * 1e3  # above the bandwidth floor
+    m100 = ctx.choose_tile_rows(seg, 600_000_000)
+    assert m100["predicted_ms"] > 50 * m["predicted_ms"]
+
+
+def test_merge_partials_exact():
+    rng = np.random.default_rng(0)
+    nr, n = 5, 7
+    vals = [[int(x) for x in rng.integers(-2**62, 2**62, n)] for _ in range(nr)]
+    vals[0][0] = 2**62 - 1
+    vals[1][0] = 2**62 - 1  # carries into the high word
+    buf = np.zeros((nr, n, 2), dtype=np.uint64)
+    for r in range(nr):
+        for i in range(n):
+            u = vals[r][i] & ((1 << 128) - 1)
+            buf[r, i, 0] = u & ((1 << 64) - 1)
+            buf[r, i, 1] = u >> 64
+    out = gpl.merge_partials(buf.reshape(-1), nr).reshape(n, 2)
+    for i in range(n):
+        got = (int(out[i, 1]) << 64) | int(out[i, 0])
+        if got >= 1 << 127:
+            got -= 1 << 128
+        assert got == sum(v[i] for v in vals)
