@@ -1,0 +1,359 @@
+#!/usr/bin/env python
+"""bench.py — TPC-H-shaped query throughput of the fused GPL pipeline on B200.
+
+One "step" = one pass of the whole hot path over the workload: every build
+segment (A1, hash builds), the fused probe segment (A2-A8, tile size from the
+A9 model), and the result fetch (A10: partials D2H + decode; for N > 1 also
+the NCCL all-gather merge). Inputs are resident in HBM before timing (value);
+`e2e` repeats the step through the C ABI from pinned HOST buffers with the
+H2D copies inside the timed region.
+
+Default workload = BASELINE.json configs[1]: TPC-H SF 1, Q5, one B200.
+Multi-GPU (torchrun): weak scaling, each rank holds an SF-per-GPU shard of
+lineitem+orders (order-key range) and replicated dimension tables.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--query Q5] [--sf 1]
+  python bench.py --impl reference ...   # the CPU oracle on the same workload
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "TPC-H query ms and fact rows/s at SF 1/10/100; HBM GB/s vs peak at 1/2/4/8 B200"
+UNIT = "fact rows/s"
+CONFIG_NAMES = {
+    ("Q14", 0.01): "configs[0]: TPC-H SF 0.01 Q14-style lineitem-part filter + SUM, 1 GPU",
+    ("Q5", 1.0): "configs[1]: TPC-H SF 1 Q5-style 6-table join + group-by on 1xB200",
+    ("Q9", 10.0): "configs[2]: TPC-H SF 10 Q9-style join-heavy aggregate",
+}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    FIELDS = "clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown," \
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                v = [x.strip() for x in out.stdout.strip().split(",")]
+                if len(v) == 6:
+                    self.samples.append(v)
+            except Exception:
+                pass
+            self._stop.wait(0.1)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for s in self.samples for n, v in zip(names, s[2:]) if v.lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def kernel_launches(segs):
+    """Kernels of ours per step: each build = count+clear+insert (2 if trivial), +1 pipeline."""
+    n = 1
+    for s in segs[:-1]:
+        body = [ln.split()[0] for ln in s.splitlines() if ln.strip() and not ln.strip().startswith("#")]
+        n += 2 if not any(k in ("filter", "probe", "semi") for k in body) else 3
+    return n
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, on the same workload."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    import tpchgen
+    from paper_conf_sigmod_paulhh16_b200 import queries
+    sf = args.sf
+    db = tpchgen.generate(sf, seed=args.seed, tables=queries.TABLES[args.query] + ["region", "nation"])
+    n = db.nrows("lineitem")
+    # bounded sample: the full workload if one evaluation fits ~6 s, else a lineitem prefix
+    _, t1 = oracle.timed_run(args.query, db, None, (0, min(n, 200_000)))
+    est = t1 * n / max(1, min(n, 200_000))
+    rows = n if est <= 6.0 else max(1, int(n * 6.0 / est))
+    for _ in range(args.warmup):
+        oracle.run(args.query, db, None, (0, rows))
+    times = []
+    for _ in range(args.steps):
+        _, t = oracle.timed_run(args.query, db, None, (0, rows))
+        times.append(t)
+    ms = 1e3 * statistics.mean(times)
+    value = rows / (ms / 1e3)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": workload_config(args, n, None),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": f"{args.query} over lineitem rows [0, {rows}) of SF {sf} (full dimension tables)"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def workload_config(args, rows_per_gpu, tile_rows):
+    return {"workload": CONFIG_NAMES.get((args.query, args.sf), f"TPC-H SF {args.sf} {args.query}"),
+            "query": args.query, "sf_per_gpu": args.sf, "lineitem_rows_per_gpu": rows_per_gpu,
+            "seed": args.seed, "parallelism": f"dp{args.gpus}" if args.gpus > 1 else "single",
+            "l2": "flushed before every step (write of 2x L2)", "tile_rows": tile_rows or "A9 cost model"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="gpl", choices=["gpl", "reference"])
+    ap.add_argument("--query", default="Q5")
+    ap.add_argument("--sf", type=float, default=1.0)
+    ap.add_argument("--seed", type=int, default=20160626)
+    ap.add_argument("--tile-rows", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import tpchgen
+    from paper_conf_sigmod_paulhh16_b200 import gpl, queries
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    args.gpus = world if world > 1 else args.gpus
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream()
+
+    q = args.query
+    tables = sorted(set(queries.TABLES[q]) | {"region", "nation"})
+    t0 = time.time()
+    db = tpchgen.generate(args.sf * world, seed=args.seed, rank=rank, world=world, tables=tables)
+    log(f"[rank {rank}] generated SF {args.sf * world} shard in {time.time() - t0:.1f}s: "
+        f"{db.nrows('lineitem')} lineitem rows")
+
+    # device-resident columns (padded to 64 rows, borrowed by the library)
+    class DevDB:
+        pass
+    ddb = DevDB()
+    ddb.tables = {}
+    for t, cols in db.tables.items():
+        ddb.tables[t] = {}
+        for c, a in cols.items():
+            n = len(a)
+            buf = torch.zeros(max(64, (n + 63) // 64 * 64), dtype=torch.int32 if a.dtype == np.int32 else torch.int64,
+                              device=dev)
+            if n:
+                buf[:n].copy_(torch.from_numpy(a))
+            v = buf[:n]
+            v._gpl_capacity_rows = buf.numel()
+            ddb.tables[t][c] = v
+    ctx = gpl.Context(local, stream=stream)
+    queries.load_database(ctx, ddb, borrow=True)
+    text = queries.plan_text(q, db)
+    segs = queries.segments(text)
+    n_local = db.nrows("lineitem")
+    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size, dtype=torch.uint8, device=dev)
+
+    part_dev = gathered = None
+
+    def step():
+        for s in segs[:-1]:
+            ctx.build_hash(s)
+        ctx.run_plan(segs[-1], args.tile_rows)
+        if world > 1:
+            nonlocal part_dev, gathered
+            nb = ctx.partials_nbytes()
+            if part_dev is None:
+                part_dev = torch.empty(nb // 8, dtype=torch.int64, device=dev)
+                gathered = torch.empty(world * nb // 8, dtype=torch.int64, device=dev)
+            ctx.fetch_partials(out=part_dev)
+            dist.all_gather_into_tensor(gathered, part_dev)
+            host = gathered.cpu().numpy()
+            res = ctx.decode_partials(gpl.merge_partials(host, world))
+            ctx.sync()
+        else:
+            res = ctx.fetch_result()
+        return res
+
+    for _ in range(args.warmup):
+        res = step()
+    res0 = ctx.fetch_result() if world == 1 else res
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    step_ms, kern_ms = [], []
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    wall0 = time.time()
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            flush.zero_()
+            ev0.record(stream)
+            res = step()
+            ev1.record(stream)
+            ev1.synchronize()
+            step_ms.append(ev0.elapsed_time(ev1))
+            kern_ms.append(res.stats["kernel_ms"])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    wall = time.time() - wall0
+    total_ms = sum(step_ms)
+    kernel_avg = statistics.mean(kern_ms)
+    stats = res0.stats
+    if world > 1:
+        t = torch.tensor([total_ms, kernel_avg], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms, kernel_avg = float(t[0]), float(t[1])
+        rows_all = torch.tensor([n_local], dtype=torch.int64, device=dev)
+        dist.all_reduce(rows_all)
+        rows_total = int(rows_all[0])
+    else:
+        rows_total = n_local
+    ms_per_step = total_ms / args.steps
+    value = rows_total / (ms_per_step / 1e3)
+
+    # e2e: same step through the C ABI from pinned host buffers (H2D inside the timed region)
+    e2e = None
+    if not args.no_e2e:
+        pinned = {t: {c: torch.from_numpy(a).pin_memory() for c, a in cols.items()} for t, cols in db.tables.items()}
+        h2d = sum(v.numel() * v.element_size() for cols in pinned.values() for v in cols.values())
+        ctx2 = gpl.Context(local, stream=stream)
+
+        def e2e_step():
+            queries.load_database(ctx2, type("H", (), {"tables": pinned})(), borrow=False)
+            for s in segs[:-1]:
+                ctx2.build_hash(s)
+            ctx2.run_plan(segs[-1], args.tile_rows)
+            return ctx2.fetch_result()
+        for _ in range(2):
+            e2e_step()
+        e_ms = []
+        for _ in range(max(3, args.steps // 4)):
+            flush.zero_()
+            ev0.record(stream)
+            r2 = e2e_step()
+            ev1.record(stream)
+            ev1.synchronize()
+            e_ms.append(ev0.elapsed_time(ev1))
+        assert r2.aggs == res0.aggs and r2.keys == res0.keys
+        ncols = sum(len(c) for c in pinned.values())
+        d2h = len(res0.aggs) * 0 + ctx2.partials_nbytes() + 16 * 8 + 4 + 16 * ncols
+        e_ms_v = statistics.mean(e_ms)
+        if world > 1:
+            t = torch.tensor([e_ms_v], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms_v = float(t[0])
+        e2e = {"value": rows_total / (e_ms_v / 1e3), "unit": UNIT, "ms_per_step": e_ms_v,
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)}
+        ctx2.close()
+
+    peak, peak_kind = measured_peak()
+    bytes_per_launch = stats["bytes_scanned"]
+    achieved = bytes_per_launch / (kernel_avg / 1e3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(prof):
+        try:
+            with open(prof) as f:
+                traffic = json.load(f).get(f"{q}@{args.sf}")
+        except Exception:
+            traffic = None
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        _, t1 = oracle.timed_run(q, db, None, (0, min(n_local, 200_000)))
+        est = t1 * n_local / max(1, min(n_local, 200_000))
+        rows = n_local if est <= 15.0 else max(1, int(n_local * 15.0 / est))
+        _, tc = oracle.timed_run(q, db, None, (0, rows))
+        cpu = {"value": rows / tc, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"{q} over lineitem rows [0, {rows}) of SF {args.sf} (full dimension tables), one evaluation"}
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world if world > 1 else 1,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+        "data": "synthetic (in-repo TPC-H-shaped generator, seed %d)" % args.seed,
+        "config": workload_config(args, n_local, stats["tile_rows_used"]),
+        "query_ms": ms_per_step, "kernel_ms": kernel_avg,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                     "kernel": "pipeline_kernel (fused scan-filter-probe-aggregate)",
+                     "bytes_per_launch": bytes_per_launch},
+        "gpu_launches": kernel_launches(segs) * args.steps,
+        "e2e": e2e,
+        "cpu_baseline": cpu,
+        "clocks": clk.summary(),
+        "wall_s_timed_region": wall,
+        "pipeline": {k: stats[k] for k in ("tile_rows_used", "stage_rows", "ring_depth", "consumer_warps", "grid",
+                                           "probe_split", "predicted_ms", "agg_mode")},
+        "op_pass": stats["op_pass"],
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

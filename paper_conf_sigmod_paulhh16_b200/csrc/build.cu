@@ -174,8 +174,8 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
   __shared__ HTP src[MAXHT];
   __shared__ HTP dst;
   if (threadIdx.x < d.nht) src[threadIdx.x] = load_htp(d.src[threadIdx.x]);
-  if (threadIdx.x == 0) {
-    HTRef r;
+  if (threadIdx.x == 0 && d.kind != HT_DIRECT) {
+    HTRef r{};
     r.slots = d.slots;
     r.hdr = d.hdr;
     r.kind = d.kind;
@@ -188,6 +188,32 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
     unsigned long long key;
     long long pay;
     if (!build_row(d, src, row, &key, &pay)) continue;
+    if (d.kind == HT_DIRECT) {
+      const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key - d.kmin);
+      if (idx >= d.nslots) { atomicOr(d.err, ERR_CAPACITY); continue; }
+      if (d.width == 0) {
+        const uint32_t bit = 1u << (idx & 31);
+        if (atomicOr((uint32_t*)d.slots + (idx >> 5), bit) & bit) atomicOr(d.err, ERR_DUPKEY);
+      } else {
+        const uint32_t v = (uint32_t)(pay - d.pay_base + 1);
+        if (d.width == 4) {
+          if (atomicCAS((uint32_t*)d.slots + idx, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
+        } else {
+          const unsigned long long byte = idx * (unsigned long long)d.width;
+          uint32_t* w = (uint32_t*)((char*)d.slots + (byte & ~3ull));
+          const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
+          const uint32_t m = (d.width == 1 ? 0xFFu : 0xFFFFu) << sh;
+          uint32_t old = *((volatile uint32_t*)w);
+          for (;;) {
+            if (old & m) { atomicOr(d.err, ERR_DUPKEY); break; }
+            const uint32_t got = atomicCAS(w, old, old | (v << sh));
+            if (got == old) break;
+            old = got;
+          }
+        }
+      }
+      continue;
+    }
     uint32_t i = ht_home(dst, key);
     if (d.kind == HT_MAP32) {
       if ((uint32_t)key == EMPTY32) { atomicOr(d.err, ERR_RESERVED_KEY); continue; }
@@ -255,6 +281,12 @@ cudaError_t launch_build(const BuildDesc& d, bool trivial, const HTHeader& known
   long long work = d.nrows > 0 ? d.nrows : 1;
   int grid = (int)std::min<long long>((work + kThreads - 1) / kThreads, (long long)num_sms * 8);
   if (grid < 1) grid = 1;
+  if (d.kind == HT_DIRECT) {  // host-sized: clear + insert, no count pass
+    cudaError_t e = cudaMemsetAsync(d.slots, 0, direct_bytes(d.width, d.nslots), s);
+    if (e != cudaSuccess) return e;
+    if (d.nrows > 0) build_insert_kernel<<<grid, kThreads, 0, s>>>(d);
+    return cudaGetLastError();
+  }
   if (!trivial) build_count_kernel<<<grid, kThreads, 0, s>>>(d);
   long long clear_blocks = std::min<long long>((d.cap_slots * 16 / 16 + kThreads - 1) / kThreads, (long long)num_sms * 8);
   if (trivial) {

@@ -181,7 +181,7 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   Options& o = ctx->opt;
   int64_t v = value;
   if (k == "stage_rows") {
-    if (v >= 0 && (v % 32 || v < 32 || v > 8192)) return fail(ctx, GPL_E_ARG, "stage_rows: multiple of 32 in [32, 8192]");
+    if (v >= 0 && (v % 128 || v < 128 || v > 8192)) return fail(ctx, GPL_E_ARG, "stage_rows: multiple of 128 in [128, 8192]");
     o.stage_rows = v;
   } else if (k == "ring_depth") {
     if (v >= 0 && (v < 2 || v > 8)) return fail(ctx, GPL_E_ARG, "ring_depth in [2, 8]");
@@ -370,20 +370,24 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
     idx = it->second;
   }
   HashTable& H = ctx->hts[idx];
-  const int sb = shape.kind == HT_SET32 ? 4 : shape.kind == HT_MAP32 ? 8 : 16;
-  if (!H.slots || H.cap_slots * (H.kind == HT_SET32 ? 4 : H.kind == HT_MAP32 ? 8 : 16) < shape.cap_slots * sb) {
+  const size_t need = std::max<size_t>(shape.bytes(), 16);
+  if (!H.slots || H.alloc_bytes < need) {
     CK(cudaStreamSynchronize(ctx->stream));
     if (H.slots) cudaFree(H.slots);
     H.slots = nullptr;
-    cudaError_t e = cudaMalloc(&H.slots, (size_t)shape.cap_slots * sb);
+    H.alloc_bytes = 0;
+    cudaError_t e = cudaMalloc(&H.slots, need);
     if (e != cudaSuccess) {
       H.valid = false;
       return fail(ctx, GPL_E_NOMEM, std::string("hash table allocation: ") + cudaGetErrorString(e));
     }
-    H.cap_slots = shape.cap_slots;
-  } else {
-    H.cap_slots = H.cap_slots * (H.kind == HT_SET32 ? 4 : H.kind == HT_MAP32 ? 8 : 16) / sb;
+    H.alloc_bytes = need;
   }
+  H.cap_slots = shape.cap_slots;
+  H.width = shape.width;
+  H.dkmin = shape.dkmin;
+  H.dnslots = shape.dnslots;
+  H.pay_base = shape.pay_base;
   if (!H.hdr) {
     CK(cudaMalloc(&H.hdr, sizeof(HTHeader)));
     CK(launch_header_init(H.hdr, ctx->stream));
@@ -431,7 +435,7 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
   for (int i = 0; i < d->nht; i++) {
     for (auto& h : ctx->hts)
       if (h.slots == d->ht[i].slots)
-        li->ht_bytes[i] = h.cap_slots * (h.kind == HT_SET32 ? 4 : h.kind == HT_MAP32 ? 8 : 16) / 2;
+        li->ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
   }
   if (tile_rows < 0) return fail(ctx, GPL_E_ARG, "tile_rows must be >= 0");
   if (!choose_config(ctx, *d, *li, d->nrows, tile_rows, cfg, &err)) return fail(ctx, GPL_E_ARG, err);
@@ -596,7 +600,12 @@ GPL_API gpl_status gpl_decode_partials(gpl_ctx* ctx, const void* host_partials, 
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run (the plan of the last run defines the layout)");
   const size_t b = (size_t)ctx->last.li.ngroups_total * ctx->last.li.nagg * 16;
   if (nbytes != b) return fail(ctx, GPL_E_ARG, "partials size does not match the last run's plan");
-  out->stats = ctx->last.stats;
+  gpl_stats& S = ctx->last.stats;
+  if (ctx->last.timed && !ctx->host_only && cudaEventQuery(ctx->ev1) == cudaSuccess) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1) == cudaSuccess) S.kernel_ms = ms;
+  }
+  out->stats = S;
   return decode(ctx, (const unsigned long long*)host_partials, out);
 }
 
@@ -631,7 +640,7 @@ GPL_API gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment,
   if (lit != ctx->lambda.end()) li.lambda = lit->second;
   for (int i = 0; i < d.nht; i++)
     for (auto& h : ctx->hts)
-      if (h.slots == d.ht[i].slots) li.ht_bytes[i] = h.cap_slots * (h.kind == HT_SET32 ? 4 : h.kind == HT_MAP32 ? 8 : 16) / 2;
+      if (h.slots == d.ht[i].slots) li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
   Config c;
   const int64_t N = n_rows > 0 ? n_rows : d.nrows;
   if (!choose_config(ctx, d, li, N, 0, &c, &err)) return fail(ctx, GPL_E_ARG, err);

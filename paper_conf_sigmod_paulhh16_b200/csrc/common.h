@@ -16,7 +16,9 @@ constexpr int MAXHT = 8;     // hash tables referenced by one segment
 constexpr int MAXTERM = 2;   // value = term +/- term
 constexpr int MAXFACT = 3;   // factors per term
 constexpr int MAXOPS = 16;   // op_pass counters
-constexpr int QCAP = 64;     // survivor-queue entries per warp (>= 2 packets)
+constexpr int RPL = 4;       // rows per lane per consumer iteration (128-row warp packets)
+constexpr int MAXSP = 2;     // probes that may run in the stage phase (register slots)
+constexpr int QCAP = 256;    // survivor-queue entries per warp (>= 127 + 128)
 
 constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;
 constexpr unsigned long long EMPTY64 = 0xFFFFFFFFFFFFFFFFull;
@@ -33,7 +35,12 @@ struct Filt {
 };
 
 // ---- hash tables (open addressing, linear probing, power-of-two slots)
-enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2 };  // 4 B {key}, 8 B {key,payload}, 16 B {key64,payload64}
+// Hashed kinds: open addressing, linear probing, power-of-two slots:
+//   SET32 4 B {key}, MAP32 8 B {key, payload}, MAP64 16 B {key64, payload64}.
+// DIRECT: direct-addressed array over a dense key domain [kmin, kmin+nslots)
+//   (a collision-free perfect hash): width 0 = bitmap set, else 1/2/4-byte
+//   cells holding payload - pay_base + 1 (0 = empty).
+enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2, HT_DIRECT = 3 };
 enum : int32_t { H_MULT = 0, H_ORDERED = 1 };
 
 // Device-resident header, written by the build's count and size kernels and
@@ -54,6 +61,11 @@ struct HTRef {
   const void* slots;
   const HTHeader* hdr;
   int32_t kind, hash;
+  // DIRECT only (host-decided): key base, cell count, payload base, cell width
+  long long kmin;
+  unsigned long long nslots;
+  long long pay_base;
+  int32_t width, pad;
 };
 
 // ---- probes
@@ -100,11 +112,14 @@ struct Agg {
 };
 enum : int32_t { AGG_REG = 0, AGG_SMEM = 1, AGG_GLOBAL = 2 };
 
-// ---- survivor-queue push: field <- stage column or stage-phase probe slot
-enum : int32_t { PUSH_COL = 0, PUSH_SREG = 1 };
+// ---- survivor-queue push: field <- stage column, stage-phase probe slot, or
+// a value term computed in the stage phase (expression pushdown)
+enum : int32_t { PUSH_COL = 0, PUSH_SREG = 1, PUSH_TERM = 2 };
 struct Push {
   int32_t kind, src;
 };
+// Stage-phase factor refs: >= 0 stage column, -1 constant, <= -2 stage slot (-(p+2)).
+constexpr int32_t SREF_CONST = -1;
 
 // Descriptor of the fused probe-segment pipeline (kernel parameter, by value).
 struct PipeDesc {
@@ -122,6 +137,11 @@ struct PipeDesc {
   Filt filt[MAXF];
   Probe probe[MAXP];     // [0, nsprobe): keys are stage columns; [nsprobe, nprobe): keys are fields
   Push push[MAXQ];       // push[i] fills queue field i
+  int32_t qoff[MAXQ];    // byte offset of field f's array in a warp's queue (QCAP entries)
+  int32_t qw[MAXQ];      // field width in bytes (4 or 8)
+  int32_t qbytes;        // bytes of one warp's queue
+  int32_t term_field[MAXTERM];  // >= 0: term t was computed in the stage phase into this field
+  Term sterm[MAXTERM];          // stage-phase form of pushed-down terms (stage refs)
   int32_t nfield, nresid, ngroup, ngroups_total;
   Resid resid[MAXR];
   GroupDim gdim[MAXG];
@@ -151,7 +171,9 @@ struct BuildDesc {
   void* slots;        // destination table
   HTHeader* hdr;
   long long cap_slots;
-  int32_t kind, hash, load_pct, pad;
+  int32_t kind, hash, load_pct, width;  // width: DIRECT cell bytes (0 = bitmap)
+  long long kmin, pay_base;             // DIRECT key / payload bases
+  unsigned long long nslots;            // DIRECT cells
   unsigned int* err;
 };
 

@@ -41,7 +41,7 @@ int align128(int x) { return (x + 127) & ~127; }
 }  // namespace
 
 int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps) {
-  int q = warps * d.nfield * QCAP * 8;
+  int q = warps * d.qbytes;
   int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   int slot = 0;
   for (int c = 0; c < d.ncols; c++) slot += align128(stage_rows * d.colw[c]);
@@ -54,7 +54,7 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->depth = c.depth;
   d->nwarps = c.warps;
   d->off_queue = kFixed;
-  d->off_agg = align128(kFixed + c.warps * d->nfield * QCAP * 8);
+  d->off_agg = align128(kFixed + c.warps * d->qbytes);
   int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   d->off_ring = d->off_agg + align128(agg);
   int off = 0;
@@ -81,7 +81,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.bw_gbs = B / 1e9;
   const double b = std::max(1, li.bytes_per_row);
   const double f_sm = 1.9e9;
-  const double B_sm = 3.0 * B / ctx->sms;  // one SM's TMA/L2 fill cap
+  const double B_sm = 1.6 * B / ctx->sms;  // one SM's TMA/L2 fill cap
   N = std::max<int64_t>(N, 1);
 
   // λ: fraction of rows reaching each operator (previous run, else defaults)
@@ -100,21 +100,22 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
     double cr = std::min(1.0, L2_eff / std::max(ht, 1.0));
     probe_bytes += reach[li.nfilt + p] * N * 32.0 * (1.0 - cr);
   }
-  // Eq 4 analog: warp-instructions per 32-row packet
-  const double packets = (double)N / 32.0;
-  double stage_cost = 24 + 8.0 * d.nfilt + 30.0 * d.nsprobe + 6.0 * d.npush;
-  double qfrac = reach.size() > (size_t)(li.nfilt + d.nsprobe) ? reach[li.nfilt + d.nsprobe] : 1.0;
-  double queue_cost = 40 + 45.0 * (d.nprobe - d.nsprobe) + 10.0 * d.nresid + 12.0 * d.nterm + 8.0 * d.nagg;
-  const double issue = 4.0 * f_sm * ctx->sms * 0.6 * std::min(1.0, W / 8.0);
-  const double t_cons = packets * (stage_cost + qfrac * queue_cost) / issue;
+  // Eq 4 analog: warp-instructions per 128-row warp packet (4 rows per lane)
+  const double qfrac = reach.size() > (size_t)(li.nfilt + d.nsprobe) ? reach[li.nfilt + d.nsprobe] : 1.0;
+  const double stage_cost = 40 + 12.0 * d.nfilt + 60.0 * d.nsprobe + 14.0 * d.npush * std::min(1.0, 8 * qfrac);
+  const double queue_cost = 60 + 90.0 * (d.nprobe - d.nsprobe) + 25.0 * d.nresid + 40.0 * d.nterm + 12.0 * d.nagg;
+  const double instr_per_row = (stage_cost + qfrac * queue_cost) / 128.0;
+  const double issue_sm = 4.0 * f_sm * 0.5 * std::min(1.0, W / 6.0);  // warp-instr/s one SM sustains
+  const double R_cons = issue_sm / instr_per_row * b * k;              // bytes/s one SM's consumers absorb
+  const double t_cons = (double)N * instr_per_row / (issue_sm * ctx->sms);
 
   // Eq 3 analog: waves of Δ-row tiles over G persistent CTAs, with the last wave's tail
   const int64_t tiles = (N + tile - 1) / tile;
   const int64_t G = c.grid;
   const int64_t waves = (tiles + G - 1) / G;
   const int64_t last = tiles - (waves - 1) * G;
-  const double rate_full = std::min(B_sm, B / (double)std::min<int64_t>(G, tiles));
-  const double rate_last = std::min(B_sm, B / (double)last);
+  const double rate_full = std::min(std::min(B_sm, R_cons / k), B / (double)std::min<int64_t>(G, tiles));
+  const double rate_last = std::min(std::min(B_sm, R_cons / k), B / (double)last);
   const double t_tile = tile * b / rate_full;
   const double last_rows = (double)(N - (tiles - 1) * tile);
   const double t_last = (last == 1 ? last_rows : (double)tile) * b / rate_last;
@@ -145,7 +146,7 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
   Config best;
   bool found = false;
   for (int S : Ss) {
-    if (S % 32 || S < 32 || S > 8192) { *err = "stage_rows must be a multiple of 32 in [32, 8192]"; return false; }
+    if (S % 128 || S < 128 || S > 8192) { *err = "stage_rows must be a multiple of 128 in [128, 8192]"; return false; }
     std::vector<int64_t> tiles;
     if (tile_req > 0) {
       tiles.push_back((tile_req + S - 1) / S * S);

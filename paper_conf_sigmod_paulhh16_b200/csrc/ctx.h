@@ -42,8 +42,18 @@ struct HashTable {
   bool has_payload = false;
   int64_t pay_min = 1, pay_max = 1;  // payload value range (validator)
   void* slots = nullptr;
+  size_t alloc_bytes = 0;
   HTHeader* hdr = nullptr;
   int64_t cap_slots = 0;
+  // DIRECT tables (kind == HT_DIRECT)
+  int width = 0;
+  long long dkmin = 0, pay_base = 0;
+  unsigned long long dnslots = 0;
+  size_t bytes() const {
+    if (kind == HT_DIRECT) return width == 0 ? (dnslots + 31) / 32 * 4 : (dnslots * width + 3) / 4 * 4;
+    return (size_t)cap_slots * (kind == HT_SET32 ? 4 : kind == HT_MAP32 ? 8 : 16);
+  }
+  HTRef ref() const { return HTRef{slots, hdr, kind, hash, dkmin, dnslots, pay_base, width, 0}; }
   std::string src_table;
   uint64_t src_version = 0;
   bool valid = false;

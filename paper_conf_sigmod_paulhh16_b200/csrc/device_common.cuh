@@ -13,9 +13,11 @@ namespace gpl {
 // Per-kernel copy of a table's parameters (from HTRef + its device header).
 struct HTP {
   const void* slots;
-  unsigned long long kmin, mult;
+  unsigned long long kmin, mult;  // hashed: ordered-hash base/multiplier; DIRECT: key base
+  unsigned long long nslots;      // DIRECT cells
+  long long pay_base;             // DIRECT payload base
   uint32_t mask, shift;
-  int32_t kind, hash;
+  int32_t kind, hash, width, pad;
 };
 
 __device__ __forceinline__ HTP load_htp(const HTRef& r) {
@@ -23,13 +25,43 @@ __device__ __forceinline__ HTP load_htp(const HTRef& r) {
   p.slots = r.slots;
   p.kind = r.kind;
   p.hash = r.hash;
+  p.width = r.width;
+  p.pad = 0;
+  if (r.kind == HT_DIRECT) {
+    p.kmin = (unsigned long long)r.kmin;
+    p.nslots = r.nslots;
+    p.pay_base = r.pay_base;
+    p.mult = 0;
+    p.mask = 0;
+    p.shift = 0;
+    return p;
+  }
   const HTHeader* h = r.hdr;
   p.mask = h->mask;
   const uint32_t log2 = h->log2;
   p.shift = (r.kind == HT_MAP64 ? 64u : 32u) - log2;
   p.kmin = (unsigned long long)h->kmin;
   p.mult = h->mult;
+  p.nslots = 0;
+  p.pay_base = 0;
   return p;
+}
+
+// DIRECT probe: one load, no chain. key is the int32 key zero-extended.
+__device__ __forceinline__ bool direct_probe(const HTP& h, unsigned long long key, long long* payload) {
+  const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key - (long long)h.kmin);
+  if (idx >= h.nslots) return false;
+  if (h.width == 0) {
+    const uint32_t w = __ldg((const uint32_t*)h.slots + (idx >> 5));
+    *payload = 1;
+    return (w >> (idx & 31)) & 1u;
+  }
+  uint32_t v;
+  if (h.width == 1) v = __ldg((const unsigned char*)h.slots + idx);
+  else if (h.width == 2) v = __ldg((const unsigned short*)h.slots + idx);
+  else v = __ldg((const uint32_t*)h.slots + idx);
+  *payload = (long long)v - 1 + h.pay_base;
+  return v != 0;
 }
 
 // Home slot. MULT: Fibonacci (multiplicative) hashing on the high bits.
@@ -43,6 +75,7 @@ __device__ __forceinline__ uint32_t ht_home(const HTP& h, unsigned long long key
 
 // Linear probing. Returns true on hit; MAP kinds also return the payload.
 __device__ __forceinline__ bool ht_probe(const HTP& h, unsigned long long key, long long* payload) {
+  if (h.kind == HT_DIRECT) return direct_probe(h, key, payload);
   uint32_t i = ht_home(h, key);
   if (h.kind == HT_MAP32) {
     if ((uint32_t)key == EMPTY32) return false;
@@ -71,6 +104,104 @@ __device__ __forceinline__ bool ht_probe(const HTP& h, unsigned long long key, l
       if (v.x == key) { *payload = (long long)v.y; return true; }
       if (v.x == EMPTY64) return false;
       i = (i + 1) & h.mask;
+    }
+  }
+}
+
+// Probe R keys of one lane with their loads in flight together (ILP): each
+// round issues one slot load per still-active row, then resolves them.
+template <int R>
+__device__ __forceinline__ void ht_probe_n(const HTP& h, const unsigned long long (&key)[R], const bool (&act)[R],
+                                           bool (&hit)[R], long long (&pay)[R]) {
+  if (h.kind == HT_DIRECT) {  // one load per row; dispatch on the cell width once
+    unsigned long long idx[R];
+    bool in[R];
+#pragma unroll
+    for (int j = 0; j < R; j++) {
+      idx[j] = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
+      in[j] = act[j] && idx[j] < h.nslots;
+    }
+    uint32_t v[R];
+    if (h.width == 0) {
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = in[j] ? (__ldg((const uint32_t*)h.slots + (idx[j] >> 5)) >> (idx[j] & 31)) & 1u : 0u;
+#pragma unroll
+      for (int j = 0; j < R; j++) { hit[j] = v[j] != 0; pay[j] = 1; }
+      return;
+    }
+    if (h.width == 1) {
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = in[j] ? (uint32_t)__ldg((const unsigned char*)h.slots + idx[j]) : 0u;
+    } else if (h.width == 2) {
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = in[j] ? (uint32_t)__ldg((const unsigned short*)h.slots + idx[j]) : 0u;
+    } else {
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = in[j] ? __ldg((const uint32_t*)h.slots + idx[j]) : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < R; j++) {
+      hit[j] = v[j] != 0;
+      pay[j] = (long long)v[j] - 1 + h.pay_base;
+    }
+    return;
+  }
+  uint32_t pos[R];
+  bool live[R];
+  bool any = false;
+#pragma unroll
+  for (int j = 0; j < R; j++) {
+    hit[j] = false;
+    pay[j] = 0;
+    live[j] = act[j] && (h.kind == HT_MAP64 ? key[j] != EMPTY64 : (uint32_t)key[j] != EMPTY32);
+    pos[j] = ht_home(h, key[j]);
+    any |= live[j];
+  }
+  if (h.kind == HT_MAP32) {
+    const unsigned long long* s = (const unsigned long long*)h.slots;
+    while (any) {
+      unsigned long long v[R];
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = live[j] ? __ldg(s + pos[j]) : 0ull;
+      any = false;
+#pragma unroll
+      for (int j = 0; j < R; j++) {
+        if (!live[j]) continue;
+        const uint32_t k = (uint32_t)v[j];
+        if (k == (uint32_t)key[j]) { hit[j] = true; pay[j] = (long long)(int32_t)(uint32_t)(v[j] >> 32); live[j] = false; }
+        else if (k == EMPTY32) live[j] = false;
+        else { pos[j] = (pos[j] + 1) & h.mask; any = true; }
+      }
+    }
+  } else if (h.kind == HT_SET32) {
+    const uint32_t* s = (const uint32_t*)h.slots;
+    while (any) {
+      uint32_t v[R];
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = live[j] ? __ldg(s + pos[j]) : 0u;
+      any = false;
+#pragma unroll
+      for (int j = 0; j < R; j++) {
+        if (!live[j]) continue;
+        if (v[j] == (uint32_t)key[j]) { hit[j] = true; pay[j] = 1; live[j] = false; }
+        else if (v[j] == EMPTY32) live[j] = false;
+        else { pos[j] = (pos[j] + 1) & h.mask; any = true; }
+      }
+    }
+  } else {
+    const ulonglong2* s = (const ulonglong2*)h.slots;
+    while (any) {
+      ulonglong2 v[R];
+#pragma unroll
+      for (int j = 0; j < R; j++) v[j] = live[j] ? __ldg(s + pos[j]) : make_ulonglong2(0ull, 0ull);
+      any = false;
+#pragma unroll
+      for (int j = 0; j < R; j++) {
+        if (!live[j]) continue;
+        if (v[j].x == key[j]) { hit[j] = true; pay[j] = (long long)v[j].y; live[j] = false; }
+        else if (v[j].x == EMPTY64) live[j] = false;
+        else { pos[j] = (pos[j] + 1) & h.mask; any = true; }
+      }
     }
   }
 }

@@ -6,6 +6,11 @@
 
 namespace gpl {
 
+// Bytes of a DIRECT table (bitmap when width == 0), 4-byte granular.
+inline unsigned long long direct_bytes(int width, unsigned long long nslots) {
+  return width == 0 ? (nslots + 31) / 32 * 4 : (nslots * (unsigned long long)width + 3) / 4 * 4;
+}
+
 // A1 build segment. `trivial` (no filter, no probe): every row is inserted,
 // so the host passes the exact header (count, key range, size) and the count
 // pass is skipped. Otherwise: count pass (+ on-device sizing) -> clear -> insert.

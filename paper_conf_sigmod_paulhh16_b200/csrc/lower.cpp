@@ -103,7 +103,7 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
     if (!ht_slot.count(H.id)) {
       int i = (int)ht_slot.size();
       ht_slot[H.id] = i;
-      d->src[i] = HTRef{H.slots, H.hdr, H.kind, H.hash};
+      d->src[i] = H.ref();
     }
     d->probe[p] = Probe{ht_slot[H.id], P.kind, k1, k2, p};
     src_ht[p] = &H;
@@ -138,14 +138,42 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
       shape->pay_max = cols[d->pay_ref]->vmax;
     }
   }
+  int load = ctx->opt.hash_load_pct > 0 ? (int)ctx->opt.hash_load_pct : s.load_pct;
   if (shape->key_arity == 2) shape->kind = HT_MAP64;
   else shape->kind = shape->has_payload ? HT_MAP32 : HT_SET32;
   if (shape->kind == HT_MAP32 && (shape->pay_min < INT32_MIN || shape->pay_max > INT32_MAX)) {
     *err = "payload range does not fit the 32-bit payload of a single-key table";
     return GPL_E_OVERFLOW;
   }
-  shape->hash = shape->kind == HT_MAP64 ? H_MULT : s.hash;
-  int load = ctx->opt.hash_load_pct > 0 ? (int)ctx->opt.hash_load_pct : s.load_pct;
+  shape->hash = shape->kind == HT_MAP64 ? H_MULT : std::max(s.hash, 0);
+  // DIRECT (collision-free) addressing over a dense key domain: single int32
+  // key, domain [min, max] of the key column, cells just wide enough for the
+  // payload range. Chosen when its size is modest or within 2x of the hashed
+  // table's upper-bound size (explicit 'hash mult|ordered' keeps hashing).
+  if (shape->key_arity == 1 && (s.hash == -1 || s.hash == 2)) {
+    const Column* kc = cols[d->k1];
+    const long long kmin = T.nrows ? kc->vmin : 0, kmax = T.nrows ? kc->vmax : 0;
+    const unsigned long long range = (unsigned long long)(kmax - kmin) + 1ull;
+    int width = -1;
+    if (!shape->has_payload) width = 0;
+    else {
+      const unsigned long long prange = (unsigned long long)(shape->pay_max - shape->pay_min) + 2ull;
+      width = prange <= 0xFFull ? 1 : prange <= 0xFFFFull ? 2 : prange <= 0xFFFFFFFFull ? 4 : -1;
+    }
+    if (width >= 0 && range <= (1ull << 31)) {
+      const unsigned long long dbytes = width == 0 ? (range + 31) / 32 * 4 : range * width;
+      const unsigned long long hbytes = (unsigned long long)std::max<int64_t>(16, next_pow2((T.nrows * 100 + load - 1) / load)) *
+                                        (shape->has_payload ? 8ull : 4ull);
+      if (s.hash == 2 || dbytes <= (64ull << 20) || dbytes <= 2 * hbytes) {
+        shape->kind = HT_DIRECT;
+        shape->width = width;
+        shape->dkmin = kmin;
+        shape->dnslots = range;
+        shape->pay_base = shape->has_payload ? shape->pay_min : 0;
+      }
+    }
+    if (s.hash == 2 && shape->kind != HT_DIRECT) { *err = "'hash direct' needs a single key and a bounded payload range"; return GPL_E_PLAN; }
+  }
   d->ncols = (int)cols.size();
   for (int c = 0; c < d->ncols; c++) {
     d->col[c] = cols[c]->dev;
@@ -155,6 +183,10 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
   d->kind = shape->kind;
   d->hash = shape->hash;
   d->load_pct = load;
+  d->width = shape->width;
+  d->kmin = shape->dkmin;
+  d->nslots = shape->dnslots;
+  d->pay_base = shape->pay_base;
   d->cap_slots = std::max<int64_t>(16, next_pow2((T.nrows * 100 + load - 1) / load));
   shape->cap_slots = d->cap_slots;
   shape->src_table = T.name;
@@ -200,8 +232,8 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
       int i = (int)ht_slot.size();
       if (i >= MAXHT) { *err = "too many hash tables"; return GPL_E_PLAN; }
       ht_slot[H.id] = i;
-      d->ht[i] = HTRef{H.slots, H.hdr, H.kind, H.hash};
-      li->ht_bytes.push_back(((int64_t)1 << 20));  // refined by the model from the header at run time
+      d->ht[i] = H.ref();
+      li->ht_bytes.push_back((int64_t)(H.kind == HT_DIRECT ? H.bytes() : H.bytes() / 2));
     }
     li->probe_ht.push_back(ht_slot[H.id]);
   }
@@ -256,9 +288,22 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   int sp = split;
   if (sp < 0 && s.split_hint >= -1) sp = s.split_hint;
   if (sp < 0) sp = s.filters.empty() ? std::min(1, np) : 0;
-  sp = std::min(sp, np);
+  sp = std::min(std::min(sp, np), MAXSP);
 
-  // queue fields: columns used in the queue phase, then stage-probe slots, then queue-probe slots
+  // Expression pushdown: a value term whose factors are all columns, constants
+  // or stage-phase slots is computed before the queue and carried as one field.
+  auto stage_avail = [&](const std::string& n) {
+    return !slot_of.count(n) || slot_of[n] < sp;
+  };
+  std::vector<bool> term_push(s.value.size(), false);
+  for (size_t t = 0; t < s.value.size(); t++) {
+    bool ok = true;
+    for (auto& f : s.value[t].f)
+      if (f.x.kind != RefIR::CONST && !stage_avail(f.x.name)) ok = false;
+    term_push[t] = ok;
+  }
+  // queue fields: columns used in the queue phase, stage-probe slots, pushed
+  // terms, then queue-probe slots (written in the queue phase)
   std::vector<std::string> qcols;
   auto need_col = [&](const std::string& n) {
     if (std::find(qcols.begin(), qcols.end(), n) == qcols.end()) qcols.push_back(n);
@@ -267,9 +312,10 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     for (auto& k : s.probes[p].keys) need_col(k);
   for (auto& g : s.groups)
     if (!slot_of.count(g.ref.name)) need_col(g.ref.name);
-  for (auto& t : s.value)
-    for (auto& f : t.f)
-      if (f.x.kind != RefIR::CONST && !slot_of.count(f.x.name)) need_col(f.x.name);
+  for (size_t t = 0; t < s.value.size(); t++)
+    if (!term_push[t])
+      for (auto& f : s.value[t].f)
+        if (f.x.kind != RefIR::CONST && !slot_of.count(f.x.name)) need_col(f.x.name);
   std::set<std::string> used_slots;
   for (auto& w : s.wheres) {
     used_slots.insert(w.a);
@@ -277,16 +323,20 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   }
   for (auto& g : s.groups)
     if (slot_of.count(g.ref.name)) used_slots.insert(g.ref.name);
-  for (auto& t : s.value)
-    for (auto& f : t.f)
-      if (f.x.kind != RefIR::CONST && slot_of.count(f.x.name)) used_slots.insert(f.x.name);
+  for (size_t t = 0; t < s.value.size(); t++)
+    if (!term_push[t])
+      for (auto& f : s.value[t].f)
+        if (f.x.kind != RefIR::CONST && slot_of.count(f.x.name)) used_slots.insert(f.x.name);
   for (auto& a : s.aggs)
     if (a.kind >= A_SUMIF) used_slots.insert(a.slot);
 
+  auto slot_width = [&](int p) { return (s.probes[p].kind != P_MARK && pht[p]->kind == HT_MAP64) ? 8 : 4; };
   std::map<std::string, int> field;
+  std::vector<int> fw;
   int nf = 0;
   for (auto& c : qcols) {
     d->push[nf] = Push{PUSH_COL, cidx[c]};
+    fw.push_back(cols[cidx[c]]->width);
     field[c] = nf++;
   }
   for (int p = 0; p < sp; p++) {
@@ -294,19 +344,39 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     if (!o.empty() && used_slots.count(o)) {
       if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
       d->push[nf] = Push{PUSH_SREG, p};
+      fw.push_back(slot_width(p));
       field[o] = nf++;
     }
   }
+  for (int t = 0; t < MAXTERM; t++) d->term_field[t] = -1;
+  for (size_t t = 0; t < s.value.size(); t++)
+    if (term_push[t]) {
+      if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+      d->push[nf] = Push{PUSH_TERM, (int)t};
+      d->term_field[t] = nf;
+      fw.push_back(8);
+      nf++;
+    }
   d->npush = nf;
   for (int p = sp; p < np; p++) {
     const std::string& o = s.probes[p].out;
     if (!o.empty() && used_slots.count(o)) {
       if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+      fw.push_back(slot_width(p));
       field[o] = nf++;
     }
   }
   if (nf > MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
   d->nfield = std::max(nf, 1);
+  {
+    int off = 0;
+    for (int f = 0; f < nf; f++) {
+      d->qoff[f] = off;
+      d->qw[f] = fw[f];
+      off += fw[f] * QCAP;
+    }
+    d->qbytes = std::max(off, 16);
+  }
 
   // slot value ranges (validator)
   auto slot_range = [&](const std::string& n) -> Range {
@@ -392,21 +462,29 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   for (int t = 0; t < d->nterm; t++) {
     const TermIR& Ti = s.value[t];
     Term& D = d->term[t];
-    D.sign = Ti.sign;
-    D.nfact = (int)Ti.f.size();
+    Term& SD = d->sterm[t];
+    D.sign = SD.sign = Ti.sign;
+    D.nfact = SD.nfact = (int)Ti.f.size();
     Range tr{1, 1};
     for (int f = 0; f < D.nfact; f++) {
       const FactorIR& F = Ti.f[f];
       Factor& X = D.f[f];
-      X.a = F.a;
-      X.b = F.b;
+      Factor& SX = SD.f[f];
+      X.a = SX.a = F.a;
+      X.b = SX.b = F.b;
       Range fr;
       if (F.x.kind == RefIR::CONST) {
-        X.field = -1;
-        X.b = 0;
+        X.field = SX.field = SREF_CONST;
+        X.b = SX.b = 0;
         fr = {(long double)F.a, (long double)F.a};
       } else {
-        X.field = field[F.x.name];
+        if (term_push[t]) {
+          X.field = -1;
+          SX.field = slot_of.count(F.x.name) ? -(slot_of[F.x.name] + 2) : cidx[F.x.name];
+        } else {
+          X.field = field[F.x.name];
+          SX.field = SREF_CONST;
+        }
         Range xr = ref_range(F.x.name);
         long double e1 = F.a + F.b * xr.lo, e2 = F.a + F.b * xr.hi;
         fr = {std::min(e1, e2), std::max(e1, e2)};

@@ -8,20 +8,25 @@
 //   producer warp (lane 0)                     consumer warps (W per CTA)
 //   ----------------------                     -------------------------------------------
 //   claim tile t = atomicAdd(counter)   A2     wait full[slot]
-//   for each stage of the tile:                for each 32-row packet of the stage:
-//     wait empty[slot]                           filters (selection = map only)  A4
-//     cp.async.bulk every column       A3        stage-phase probes (first `nsprobe`)     A5
-//       (TMA engine, L2 evict_first)             ballot/popc compaction -> warp queue     A8
-//     arrive.expect_tx full[slot]                whenever >= 32 survivors are queued:
+//   for each stage of the tile:                for each 128-row packet of the stage
+//     wait empty[slot]                         (4 consecutive rows per lane):
+//     cp.async.bulk every column       A3        filters (selection = map only)  A4
+//       (TMA engine, L2 evict_first)             stage-phase probes (first `nsprobe`)     A5
+//     arrive.expect_tx full[slot]                value terms computable here (pushdown)
+//                                                ballot/popc compaction -> warp queue     A8
+//                                                whenever >= 128 survivors are queued:
 //                                                  remaining probes, where, group-by,   A5-A7
 //                                                  exact int64 aggregation
 //                                              arrive empty[slot]
 //
 // The ring of `depth` stages replaces the paper's "number of channels" n and
-// a 32-row warp packet replaces its packet size p. Survivors travel
-// through per-warp shared-memory queues carrying their values, so no
-// operator writes an intermediate to HBM; the only global writes
-// are the few-KB aggregate partials (int128) and counters.
+// the warp packet replaces its packet size p. Survivors travel
+// through per-warp shared-memory queues carrying their values, so no operator
+// writes an intermediate to HBM; the only global writes are the
+// few-KB aggregate partials (int128) and counters.
+//
+// All shared-memory accesses use integer offsets into the one __shared__
+// array so they compile to plain LDS/STS (no generic-address conversion).
 #include <climits>
 
 #include "device_common.cuh"
@@ -29,6 +34,8 @@
 
 namespace gpl {
 namespace {
+
+extern __shared__ __align__(128) unsigned char g_smem[];
 
 constexpr int kMaxWarps = 17;  // 16 consumers + 1 producer
 constexpr int kMaxThreads = kMaxWarps * 32;
@@ -40,6 +47,12 @@ constexpr int kOffHdr = 128;      // int4[kMaxDepth]
 constexpr int kOffHtp = 256;      // HTP[MAXHT]
 constexpr int kOffCnt = 1024;     // unsigned long long[kMaxWarps][MAXOPS]
 static_assert(kOffHtp + MAXHT * sizeof(HTP) <= kOffCnt, "HTP region overflow");
+static_assert(kOffCnt + kMaxWarps * MAXOPS * 8 <= 4096, "fixed region overflow");
+
+template <class T>
+__device__ __forceinline__ T& S(uint32_t off) {
+  return *reinterpret_cast<T*>(g_smem + off);
+}
 
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
@@ -47,113 +60,140 @@ __device__ __forceinline__ unsigned lanemask_lt() {
   return m;
 }
 
-__device__ __forceinline__ long long ld_stage(const PipeDesc& d, const char* sb, int c, int r) {
-  const char* p = sb + d.coloff[c];
-  return d.colw[c] == 4 ? (long long)((const int*)p)[r] : ((const long long*)p)[r];
+// RPL consecutive rows (r0 % 4 == 0) of one staged column, widened to int64.
+__device__ __forceinline__ void ld_rows(uint32_t a, int w, long long (&x)[RPL]) {
+  if (w == 4) {
+    const int4 v = S<int4>(a);
+    x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
+  } else {
+    const longlong2 u = S<longlong2>(a);
+    const longlong2 v = S<longlong2>(a + 16);
+    x[0] = u.x; x[1] = u.y; x[2] = v.x; x[3] = v.y;
+  }
 }
 
-__device__ __forceinline__ long long sel4(const long long (&s)[MAXP], int i) {
-  long long v = s[0];
+__device__ __forceinline__ long long qget(const PipeDesc& d, uint32_t qb, int f, int i) {
+  const uint32_t a = qb + d.qoff[f];
+  return d.qw[f] == 4 ? (long long)S<int>(a + i * 4) : S<long long>(a + i * 8);
+}
+__device__ __forceinline__ void qput(const PipeDesc& d, uint32_t qb, int f, int i, long long v) {
+  const uint32_t a = qb + d.qoff[f];
+  if (d.qw[f] == 4) S<int>(a + i * 4) = (int)v;
+  else S<long long>(a + i * 8) = v;
+}
+
+__device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
+  return (unsigned)p[0] + (unsigned)p[1] + (unsigned)p[2] + (unsigned)p[3];
+}
+__device__ __forceinline__ bool any4(const bool (&p)[RPL]) { return p[0] | p[1] | p[2] | p[3]; }
+
+// Queue phase on up to RPL*32 queued survivors starting at qhead: lane `lane`
+// owns entries qhead + j*32 + lane (j < RPL) that are < n. Remaining probes,
+// where residuals, group-by and the exact aggregation (A5-A7).
+__device__ __noinline__ void drain(const PipeDesc& d, uint32_t qb, int qhead, int n, unsigned long long* cnt,
+                                   long long* acc, int lane) {
+  const HTP* htp = &S<HTP>(kOffHtp);
+  int idx[RPL];
+  bool p[RPL];
 #pragma unroll
-  for (int k = 1; k < MAXP; k++) v = (i == k) ? s[k] : v;
-  return v;
-}
-
-// Queue phase on one packet of up to 32 queued survivors: lane `lane` owns
-// queue entry `idx` (valid iff `pass`). Runs the remaining probes, the where
-// residuals, the group-by and the aggregation (A5-A7).
-__device__ __forceinline__ void drain(const PipeDesc& d, const HTP* htp, long long* q, int idx, bool pass,
-                                      unsigned long long* cnt, long long (&acc)[MAXA], unsigned long long* stab,
-                                      int lane) {
+  for (int j = 0; j < RPL; j++) {
+    const int e = j * 32 + lane;
+    idx[j] = (qhead + e) & (QCAP - 1);
+    p[j] = e < n;
+  }
   int op = d.nfilt + d.nsprobe;
-  for (int p = d.nsprobe; p < d.nprobe; p++, op++) {
-    const Probe& P = d.probe[p];
-    if (__any_sync(0xffffffffu, pass)) {
-      if (pass) {
-        unsigned long long k = (uint32_t)q[P.k1 * QCAP + idx];
-        if (P.k2 >= 0) k = (k << 32) | (uint32_t)q[P.k2 * QCAP + idx];
-        long long v = 0;
-        const bool hit = ht_probe(htp[P.ht], k, &v);
+  for (int pi = d.nsprobe; pi < d.nprobe; pi++, op++) {
+    const Probe P = d.probe[pi];
+    if (__any_sync(0xffffffffu, any4(p))) {
+      unsigned long long k[RPL];
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
+        k[j] = (uint32_t)qget(d, qb, P.k1, idx[j]);
+        if (P.k2 >= 0) k[j] = (k[j] << 32) | (uint32_t)qget(d, qb, P.k2, idx[j]);
+      }
+      bool hit[RPL];
+      long long v[RPL];
+      ht_probe_n<RPL>(htp[P.ht], k, p, hit, v);
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
         if (P.kind == P_MARK) {
-          q[P.out * QCAP + idx] = hit ? 1 : 0;
+          if (p[j] && P.out >= 0) qput(d, qb, P.out, idx[j], hit[j] ? 1 : 0);
         } else {
-          pass = hit;
-          if (hit && P.out >= 0) q[P.out * QCAP + idx] = v;
+          if (hit[j] && P.out >= 0) qput(d, qb, P.out, idx[j], v[j]);
+          p[j] = hit[j];
         }
       }
     }
-    const unsigned m = __ballot_sync(0xffffffffu, pass);
-    if (lane == 0) cnt[op] += __popc(m);
+    const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+    if (lane == 0) cnt[op] += c;
   }
   for (int r = 0; r < d.nresid; r++, op++) {
     const Resid& R = d.resid[r];
-    if (pass) {
-      const long long a = q[R.a * QCAP + idx];
-      if (R.kind == R_EQ) {
-        pass = a == q[R.b * QCAP + idx];
-      } else if (R.kind == R_PAIRS) {
-        const long long b = q[R.b * QCAP + idx];
+    const int kind = R.kind, fa = R.a, fb = R.b;
+#pragma unroll
+    for (int j = 0; j < RPL; j++) {
+      if (!p[j]) continue;
+      const long long a = qget(d, qb, fa, idx[j]);
+      if (kind == R_EQ) {
+        p[j] = a == qget(d, qb, fb, idx[j]);
+      } else if (kind == R_PAIRS) {
+        const long long b = qget(d, qb, fb, idx[j]);
         bool ok = false;
         for (int i = 0; i < R.npairs; i++) ok |= (a == R.pa[i]) & (b == R.pb[i]);
-        pass = ok;
-      } else if (R.kind == R_RANGE) {
-        pass = a >= R.lo && a <= R.hi;
+        p[j] = ok;
+      } else if (kind == R_RANGE) {
+        p[j] = a >= R.lo && a <= R.hi;
       } else {
-        pass = (unsigned long long)a < 64ull && ((R.mask >> a) & 1ull);
+        p[j] = (unsigned long long)a < 64ull && ((R.mask >> a) & 1ull);
       }
     }
-    const unsigned m = __ballot_sync(0xffffffffu, pass);
-    if (lane == 0) cnt[op] += __popc(m);
+    const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+    if (lane == 0) cnt[op] += c;
   }
-  if (!__any_sync(0xffffffffu, pass)) return;
-  int gid = 0;
-  if (pass) {
+  if (!__any_sync(0xffffffffu, any4(p))) return;
+  unsigned long long* stab = &S<unsigned long long>(d.off_agg);
+#pragma unroll
+  for (int j = 0; j < RPL; j++) {
+    if (!p[j]) continue;
+    int gid = 0;
+    bool ok = true;
     for (int g = 0; g < d.ngroup; g++) {
       const GroupDim& G = d.gdim[g];
-      long long v = q[G.field * QCAP + idx];
+      long long v = qget(d, qb, G.field, idx[j]);
       if (G.transform == G_YEAR) v = (int)v / 10000;
       const long long o = v - G.lo;
-      if ((unsigned long long)o >= (unsigned long long)G.size) {
-        atomicOr(d.err, ERR_DOMAIN);
-        pass = false;
-      }
+      if ((unsigned long long)o >= (unsigned long long)G.size) ok = false;
       gid += (int)o * G.stride;
     }
-  }
-  long long val = 0;
-  for (int t = 0; t < d.nterm; t++) {
-    const Term& T = d.term[t];
-    long long prod = T.sign;
-    for (int f = 0; f < T.nfact; f++) {
-      const Factor& F = T.f[f];
-      const long long x = F.field < 0 ? F.a : F.a + (long long)F.b * q[F.field * QCAP + idx];
-      prod *= x;
+    if (!ok) {
+      atomicOr(d.err, ERR_DOMAIN);
+      continue;
     }
-    val += prod;
-  }
-  if (!pass) return;
-  if (d.agg_mode == AGG_REG) {
-#pragma unroll
-    for (int a = 0; a < MAXA; a++) {
-      if (a < d.nagg) {
-        const Agg& A = d.agg[a];
-        long long c = 1;
-        if (A.kind == A_SUM) c = val;
-        else if (A.kind == A_SUMIF) c = q[A.field * QCAP + idx] != 0 ? val : 0;
-        else if (A.kind == A_SUMIFEQ) c = q[A.field * QCAP + idx] == A.c ? val : 0;
-        acc[a] += c;
+    long long val = 0;
+    for (int t = 0; t < d.nterm; t++) {
+      if (d.term_field[t] >= 0) {
+        val += qget(d, qb, d.term_field[t], idx[j]);
+        continue;
       }
+      const Term& T = d.term[t];
+      long long prod = T.sign;
+      for (int f = 0; f < T.nfact; f++) {
+        const Factor& F = T.f[f];
+        prod *= F.field < 0 ? F.a : F.a + (long long)F.b * qget(d, qb, F.field, idx[j]);
+      }
+      val += prod;
     }
-  } else {
     for (int a = 0; a < d.nagg; a++) {
       const Agg& A = d.agg[a];
       long long c = 1;
       if (A.kind == A_SUM) c = val;
-      else if (A.kind == A_SUMIF) c = q[A.field * QCAP + idx] != 0 ? val : 0;
-      else if (A.kind == A_SUMIFEQ) c = q[A.field * QCAP + idx] == A.c ? val : 0;
-      if (c == 0) continue;
-      if (d.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * d.nagg + a], (unsigned long long)c);
-      else atomic_add_i128(d.partials + 2 * (gid * d.nagg + a), c);
+      else if (A.kind == A_SUMIF) c = qget(d, qb, A.field, idx[j]) != 0 ? val : 0;
+      else if (A.kind == A_SUMIFEQ) c = qget(d, qb, A.field, idx[j]) == A.c ? val : 0;
+      if (d.agg_mode == AGG_REG) acc[a] += c;
+      else if (c != 0) {
+        if (d.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * d.nagg + a], (unsigned long long)c);
+        else atomic_add_i128(d.partials + 2 * (gid * d.nagg + a), c);
+      }
     }
   }
 }
@@ -170,14 +210,12 @@ __device__ __forceinline__ void flush_reg(const PipeDesc& d, long long (&acc)[MA
 }
 
 __global__ void __launch_bounds__(kMaxThreads, 1) pipeline_kernel(const __grid_constant__ PipeDesc d) {
-  extern __shared__ __align__(128) unsigned char smem[];
-  unsigned long long* full = (unsigned long long*)(smem + kOffFull);
-  unsigned long long* empty = (unsigned long long*)(smem + kOffEmpty);
-  int4* hdr = (int4*)(smem + kOffHdr);
-  HTP* htp = (HTP*)(smem + kOffHtp);
-  unsigned long long* cnt_all = (unsigned long long*)(smem + kOffCnt);
-  unsigned long long* stab = (unsigned long long*)(smem + d.off_agg);
-  char* ring = (char*)(smem + d.off_ring);
+  unsigned long long* full = &S<unsigned long long>(kOffFull);
+  unsigned long long* empty = &S<unsigned long long>(kOffEmpty);
+  int4* hdr = &S<int4>(kOffHdr);
+  HTP* htp = &S<HTP>(kOffHtp);
+  unsigned long long* cnt_all = &S<unsigned long long>(kOffCnt);
+  unsigned long long* stab = &S<unsigned long long>(d.off_agg);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int W = d.nwarps;
@@ -213,7 +251,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) pipeline_kernel(const __grid_c
           uint32_t bytes = 0;
           for (int c = 0; c < d.ncols; c++) bytes += ((uint32_t)n * d.colw[c] + 15u) & ~15u;
           mbar_arrive_expect_tx(&full[slot], bytes);
-          char* dst = ring + (size_t)slot * d.slot_bytes;
+          unsigned char* dst = g_smem + d.off_ring + (size_t)slot * d.slot_bytes;
           for (int c = 0; c < d.ncols; c++)
             bulk_g2s(dst + d.coloff[c], d.col[c] + row * d.colw[c], ((uint32_t)n * d.colw[c] + 15u) & ~15u,
                      &full[slot], pol);
@@ -229,67 +267,124 @@ __global__ void __launch_bounds__(kMaxThreads, 1) pipeline_kernel(const __grid_c
 
   // -------------------------------------------------------------- consumers
   unsigned long long* cnt = cnt_all + warp * MAXOPS;
-  long long* q = (long long*)(smem + d.off_queue) + (size_t)warp * d.nfield * QCAP;
+  const uint32_t qb = (uint32_t)d.off_queue + (uint32_t)warp * (uint32_t)d.qbytes;
   long long acc[MAXA] = {0, 0, 0, 0};
   int qhead = 0, qcount = 0;
   uint32_t slot = 0, phase = 0;
+  const int nfilt = d.nfilt, nsprobe = d.nsprobe, npush = d.npush;
   for (;;) {
     mbar_wait(&full[slot], phase);
     const int4 h = hdr[slot];
     const int n = h.z;
     if (n < 0) break;
-    const char* sb = ring + (size_t)slot * d.slot_bytes;
-    const int npk = (n + 31) >> 5;
-    for (int pk = warp; pk < npk; pk += W) {
-      const int r = (pk << 5) + lane;
-      bool pass = r < n;
-      for (int f = 0; f < d.nfilt; f++) {
-        const Filt& F = d.filt[f];
-        if (pass) pass = filt_pass(F, ld_stage(d, sb, F.ref, r));
-        const unsigned m = __ballot_sync(0xffffffffu, pass);
-        if (lane == 0) cnt[f] += __popc(m);
-      }
-      long long sreg[MAXP] = {0, 0, 0, 0};
+    const uint32_t sb = (uint32_t)d.off_ring + slot * (uint32_t)d.slot_bytes;
+    const int nit = (n + 127) >> 7;
+    for (int it = warp; it < nit; it += W) {
+      const int r0 = (it << 7) + (lane << 2);
+      bool p[RPL];
 #pragma unroll
-      for (int p = 0; p < MAXP; p++) {
-        if (p < d.nsprobe) {
-          const Probe& P = d.probe[p];
-          if (__any_sync(0xffffffffu, pass)) {
-            if (pass) {
-              unsigned long long k = (uint32_t)ld_stage(d, sb, P.k1, r);
-              if (P.k2 >= 0) k = (k << 32) | (uint32_t)ld_stage(d, sb, P.k2, r);
-              long long v = 0;
-              const bool hit = ht_probe(htp[P.ht], k, &v);
+      for (int j = 0; j < RPL; j++) p[j] = r0 + j < n;
+      // A4 selection: predicates on staged columns, 4 rows per lane
+      for (int f = 0; f < nfilt; f++) {
+        const Filt F = d.filt[f];
+        long long x[RPL];
+        ld_rows(sb + d.coloff[F.ref] + r0 * d.colw[F.ref], d.colw[F.ref], x);
+#pragma unroll
+        for (int j = 0; j < RPL; j++) p[j] = p[j] && filt_pass(F, x[j]);
+        const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+        if (lane == 0) cnt[f] += c;
+      }
+      // A5 stage-phase probes (keys from the stage; loads of the 4 rows in flight together)
+      long long sreg[MAXSP][RPL];
+#pragma unroll
+      for (int sp = 0; sp < MAXSP; sp++) {
+#pragma unroll
+        for (int j = 0; j < RPL; j++) sreg[sp][j] = 0;
+        if (sp < nsprobe) {
+          const Probe P = d.probe[sp];
+          if (__any_sync(0xffffffffu, any4(p))) {
+            long long k1[RPL];
+            ld_rows(sb + d.coloff[P.k1] + r0 * d.colw[P.k1], d.colw[P.k1], k1);
+            unsigned long long k[RPL];
+#pragma unroll
+            for (int j = 0; j < RPL; j++) k[j] = (uint32_t)k1[j];
+            if (P.k2 >= 0) {
+              long long k2[RPL];
+              ld_rows(sb + d.coloff[P.k2] + r0 * d.colw[P.k2], d.colw[P.k2], k2);
+#pragma unroll
+              for (int j = 0; j < RPL; j++) k[j] = (k[j] << 32) | (uint32_t)k2[j];
+            }
+            bool hit[RPL];
+            long long v[RPL];
+            ht_probe_n<RPL>(htp[P.ht], k, p, hit, v);
+#pragma unroll
+            for (int j = 0; j < RPL; j++) {
               if (P.kind == P_MARK) {
-                sreg[p] = hit ? 1 : 0;
+                sreg[sp][j] = hit[j] ? 1 : 0;
               } else {
-                pass = hit;
-                sreg[p] = v;
+                sreg[sp][j] = v[j];
+                p[j] = hit[j];
               }
             }
           }
-          const unsigned m = __ballot_sync(0xffffffffu, pass);
-          if (lane == 0) cnt[d.nfilt + p] += __popc(m);
+          const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+          if (lane == 0) cnt[nfilt + sp] += c;
         }
       }
-      const unsigned mask = __ballot_sync(0xffffffffu, pass);
-      if (mask) {
-        if (pass) {
-          const int idx = (qhead + qcount + __popc(mask & lanemask_lt())) & (QCAP - 1);
-          for (int e = 0; e < d.npush; e++) {
-            const Push& E = d.push[e];
-            const long long v = E.kind == PUSH_COL ? ld_stage(d, sb, E.src, r) : sel4(sreg, E.src);
-            q[e * QCAP + idx] = v;
+      // A8 compaction into the warp's survivor queue (the on-chip channel)
+      int base = qcount;
+      int pos[RPL];
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
+        const unsigned m = __ballot_sync(0xffffffffu, p[j]);
+        pos[j] = (qhead + base + __popc(m & lanemask_lt())) & (QCAP - 1);
+        base += __popc(m);
+      }
+      if (base == qcount) continue;
+      for (int e = 0; e < npush; e++) {
+        const Push E = d.push[e];
+        const uint32_t qa = qb + d.qoff[e];
+        const int qw = d.qw[e];
+        long long v[RPL];
+        if (E.kind == PUSH_COL) {
+          ld_rows(sb + d.coloff[E.src] + r0 * d.colw[E.src], d.colw[E.src], v);
+        } else if (E.kind == PUSH_SREG) {
+#pragma unroll
+          for (int j = 0; j < RPL; j++) v[j] = E.src == 0 ? sreg[0][j] : sreg[1][j];
+        } else {  // pushed-down value term: sign * prod(a + b * x)
+          const Term& T = d.sterm[E.src];
+#pragma unroll
+          for (int j = 0; j < RPL; j++) v[j] = T.sign;
+          for (int f = 0; f < T.nfact; f++) {
+            const Factor F = T.f[f];
+            long long x[RPL];
+            if (F.field >= 0) {
+              ld_rows(sb + d.coloff[F.field] + r0 * d.colw[F.field], d.colw[F.field], x);
+            } else {
+#pragma unroll
+              for (int j = 0; j < RPL; j++) x[j] = F.field == SREF_CONST ? 0 : (F.field == -2 ? sreg[0][j] : sreg[1][j]);
+            }
+#pragma unroll
+            for (int j = 0; j < RPL; j++) v[j] *= F.a + (long long)F.b * x[j];
           }
         }
-        qcount += __popc(mask);
-        if (qcount >= 32) {
-          __syncwarp();
-          drain(d, htp, q, (qhead + lane) & (QCAP - 1), true, cnt, acc, stab, lane);
-          __syncwarp();
-          qhead = (qhead + 32) & (QCAP - 1);
-          qcount -= 32;
+        if (qw == 4) {
+#pragma unroll
+          for (int j = 0; j < RPL; j++)
+            if (p[j]) S<int>(qa + pos[j] * 4) = (int)v[j];
+        } else {
+#pragma unroll
+          for (int j = 0; j < RPL; j++)
+            if (p[j]) S<long long>(qa + pos[j] * 8) = v[j];
         }
+      }
+      qcount = base;
+      if (qcount >= RPL * 32) {
+        __syncwarp();
+        drain(d, qb, qhead, RPL * 32, cnt, acc, lane);
+        __syncwarp();
+        qhead = (qhead + RPL * 32) & (QCAP - 1);
+        qcount -= RPL * 32;
       }
     }
     __syncwarp();
@@ -299,7 +394,7 @@ __global__ void __launch_bounds__(kMaxThreads, 1) pipeline_kernel(const __grid_c
   }
   if (qcount > 0) {
     __syncwarp();
-    drain(d, htp, q, (qhead + lane) & (QCAP - 1), lane < qcount, cnt, acc, stab, lane);
+    drain(d, qb, qhead, qcount, cnt, acc, lane);
   }
   __syncwarp();
   if (d.agg_mode == AGG_REG) flush_reg(d, acc, lane);
@@ -326,12 +421,13 @@ cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     configured = d.smem_bytes;
   }
-  if (d.nwarps + 1 > kMaxWarps || d.depth > kMaxDepth) return cudaErrorInvalidValue;
+  if (d.nwarps + 1 > kMaxWarps || d.depth > kMaxDepth || d.nsprobe > MAXSP || d.stage_rows % 128)
+    return cudaErrorInvalidValue;
   pipeline_kernel<<<grid, (d.nwarps + 1) * 32, d.smem_bytes, s>>>(d);
   return cudaGetLastError();
 }
 
-int pipeline_fixed_smem() { return kOffCnt + kMaxWarps * MAXOPS * 8; }
+int pipeline_fixed_smem() { return 4096; }
 int pipeline_max_consumer_warps() { return kMaxWarps - 1; }
 
 }  // namespace gpl

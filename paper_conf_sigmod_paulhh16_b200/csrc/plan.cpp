@@ -278,10 +278,12 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
         if (!seg->is_build) throw ParseError{"'payload' only in build segments"};
         seg->payload = parse_ref(c);
       } else if (kw == "hash") {
-        std::string h = expect_id(c, "mult|ordered");
+        std::string h = expect_id(c, "auto|direct|mult|ordered");
         if (h == "mult") seg->hash = H_MULT;
         else if (h == "ordered") seg->hash = H_ORDERED;
-        else throw ParseError{"hash must be 'mult' or 'ordered'"};
+        else if (h == "direct") seg->hash = 2;
+        else if (h == "auto") seg->hash = -1;
+        else throw ParseError{"hash must be auto, direct, mult or ordered"};
       } else if (kw == "load") {
         seg->load_pct = (int)expect_int(c, "percent");
         if (seg->load_pct < 10 || seg->load_pct > 90) throw ParseError{"load must be in [10, 90]"};

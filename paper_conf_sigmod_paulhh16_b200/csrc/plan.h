@@ -70,7 +70,7 @@ struct Segment {
   // build
   std::vector<std::string> key;
   RefIR payload;  // CONST kind => none
-  int hash = 0;   // H_MULT / H_ORDERED
+  int hash = -1;  // -1 auto, H_MULT, H_ORDERED, 2 = direct
   int load_pct = 50;
   // probe segment
   std::vector<WhereIR> wheres;

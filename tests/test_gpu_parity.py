@@ -82,8 +82,8 @@ def test_ragged_and_empty(ctx, n):
 def test_schedule_invariance(ctx):
     db = tpchgen.generate(0.1, seed=8)
     expect = {q: oracle.run(q, db, _params(q)) for q in ("Q5", "Q7", "Q14", "L1")}
-    knobs = [dict(stage_rows=32, ring_depth=2, consumer_warps=1), dict(stage_rows=256, ring_depth=3, consumer_warps=4),
-             dict(stage_rows=1024, ring_depth=4, consumer_warps=8), dict(stage_rows=2048, ring_depth=2, consumer_warps=16), dict(stage_rows=4096, ring_depth=2, consumer_warps=2),
+    knobs = [dict(stage_rows=128, ring_depth=2, consumer_warps=1), dict(stage_rows=256, ring_depth=3, consumer_warps=4),
+             dict(stage_rows=1024, ring_depth=4, consumer_warps=8), dict(stage_rows=2048, ring_depth=2, consumer_warps=12), dict(stage_rows=3072, ring_depth=2, consumer_warps=2),
              dict(probe_split=0), dict(probe_split=1), dict(probe_split=2), dict(probe_split=-1)]
     try:
         for k in knobs:
