@@ -40,7 +40,16 @@ $(OBJDIR)/%.cpp.o: $(CSRC)/%.cpp $(HDRS)
 	@mkdir -p $(OBJDIR)
 	$(CXX) $(CXXFLAGS) -c $< -o $@
 
-$(LIBGPL): $(CU_OBJS) $(CPP_OBJS)
+JIT_HDRS := $(CSRC)/common.h $(CSRC)/device_common.cuh $(CSRC)/pipeline_body.cuh
+
+$(OBJDIR)/jit_sources.cpp: $(JIT_HDRS) tools/embed_sources.py
+	@mkdir -p $(OBJDIR)
+	python3 tools/embed_sources.py $@ $(JIT_HDRS)
+
+$(OBJDIR)/jit_sources.o: $(OBJDIR)/jit_sources.cpp
+	$(CXX) $(CXXFLAGS) -c $< -o $@
+
+$(LIBGPL): $(CU_OBJS) $(CPP_OBJS) $(OBJDIR)/jit_sources.o
 	@mkdir -p $(PKG)/lib
 	$(NVCC) $(ARCH) -shared -o $@ $^ -cudart static -lpthread -ldl -lrt
 

@@ -87,6 +87,8 @@ typedef struct {
   double bytes_scanned;        /* algorithmic bytes: rows x bytes/row of staged columns           */
   int32_t agg_mode;            /* 0 registers (1 group), 1 smem table, 2 global int128 atomics   */
   int32_t kbe;                 /* 1 if produced by gpl_run_plan_kbe                               */
+  int32_t jit;                 /* 1 if the plan-specialised (NVRTC) kernel ran, 0 the generic one */
+  int32_t reserved;
   double intermediate_bytes;   /* bytes of operator outputs materialised in HBM (fused path: 0)   */
 } gpl_stats;
 
@@ -196,12 +198,22 @@ gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t
                                 gpl_model_report* out);
 
 /* Tuning knobs (tests / sweeps): "stage_rows", "ring_depth",
- * "consumer_warps", "ctas_per_sm", "probe_split" (-1 = auto), "hash_load_pct".
+ * "consumer_warps", "ctas_per_sm", "probe_split" (-1 = auto), "hash_load_pct",
+ * "jit" (1 = plan-specialised kernels, default; 0 = generic kernel).
  * value < 0 restores automatic selection. */
 gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value);
 
 /* Validate a plan segment against the loaded tables (host only). */
 gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment);
+
+/* Compile (NVRTC, sm_100a) the plan-specialised build of the fused kernel for
+ * this probe segment and cache it, so the first gpl_run_plan does not pay the
+ * compile. The shape depends on the loaded tables, hash tables, options and
+ * the A9 configuration for tile_rows. On a host-only context it compiles
+ * without loading (a build check). GPL_E_STATE if NVRTC is unavailable or
+ * the compile fails (message in gpl_last_error); gpl_run_plan then uses the
+ * generic precompiled kernel. Disable with gpl_set_option("jit", 0). */
+gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows);
 
 /* Message of the last failed call on ctx (ctx-owned, valid until the next
  * call). gpl_last_error(NULL) reports gpl_create failures. */

@@ -197,6 +197,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "hash_load_pct") {
     if (v >= 0 && (v < 10 || v > 90)) return fail(ctx, GPL_E_ARG, "hash_load_pct in [10, 90]");
     o.hash_load_pct = v;
+  } else if (k == "jit") {
+    o.jit = v != 0 ? 1 : 0;
   } else if (k == "hbm_mbs") {
     o.hbm_gbs = v > 0 ? v / 1000.0 : -1;
   } else {
@@ -474,8 +476,9 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   d.err = err_ptr(ctx);
   CK(cudaMemsetAsync(ctx->d_partials, 0, pbytes, ctx->stream));
   CK(cudaMemsetAsync(ctx->d_scratch, 0, (1 + MAXOPS) * sizeof(unsigned long long), ctx->stream));
+  std::string jerr;
   CK(cudaEventRecord(ctx->ev0, ctx->stream));
-  CK(launch_pipeline(d, cfg.grid, ctx->stream));
+  CK(launch_pipeline(d, cfg.grid, ctx->stream, ctx->opt.jit != 0, &jerr));
   CK(cudaEventRecord(ctx->ev1, ctx->stream));
   LastRun& L = ctx->last;
   L.valid = true;
@@ -497,6 +500,22 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   S.predicted_ms = cfg.pred_ms;
   S.bytes_scanned = (double)d.nrows * li.bytes_per_row;
   S.agg_mode = d.agg_mode;
+  S.jit = (ctx->opt.jit != 0 && jerr.empty()) ? 1 : 0;
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows) {
+  if (!ctx || !probe_segment) return GPL_E_ARG;
+  ctx->err.clear();
+  PipeDesc d;
+  LowerInfo li;
+  Config cfg;
+  Segment seg;
+  gpl_status st;
+  if ((st = prepare_run(ctx, probe_segment, tile_rows, &d, &li, &cfg, &seg))) return st;
+  std::string err;
+  if (!ctx->host_only && (st = check_dev(ctx))) return st;
+  if (!jit_prepare(d, !ctx->host_only, &err)) return fail(ctx, GPL_E_STATE, err);
   return GPL_OK;
 }
 

@@ -1,7 +1,14 @@
 // common.h — POD descriptors shared by the host lowering (plan.cpp) and the
 // sm_100a kernels (build.cu, pipeline.cu, kbe.cu). No torch, no CUDA types.
 #pragma once
+#ifndef __CUDACC_RTC__
 #include <cstdint>
+#else  // NVRTC (plan-specialised JIT kernels): no host headers
+typedef int int32_t;
+typedef unsigned int uint32_t;
+typedef long long int64_t;
+typedef unsigned long long uint64_t;
+#endif
 
 namespace gpl {
 

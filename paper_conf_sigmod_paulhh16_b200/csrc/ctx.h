@@ -86,6 +86,7 @@ struct LastRun {
 struct Options {
   int64_t stage_rows = -1, ring_depth = -1, consumer_warps = -1, ctas_per_sm = -1, probe_split = -2,
           hash_load_pct = -1;
+  int64_t jit = 1;
   double hbm_gbs = -1;
 };
 

@@ -3,7 +3,9 @@
 // wrappers for mbarrier / bulk-async copies / L2 cache policies (sm_90+, used
 // here for sm_100a).
 #pragma once
+#ifndef __CUDACC_RTC__
 #include <cstdint>
+#endif
 
 #include "common.h"
 
@@ -110,10 +112,13 @@ __device__ __forceinline__ bool ht_probe(const HTP& h, unsigned long long key, l
 
 // Probe R keys of one lane with their loads in flight together (ILP): each
 // round issues one slot load per still-active row, then resolves them.
+// `kind` and `width` are passed separately so that a plan-specialised (JIT)
+// kernel sees them as compile-time constants.
 template <int R>
-__device__ __forceinline__ void ht_probe_n(const HTP& h, const unsigned long long (&key)[R], const bool (&act)[R],
-                                           bool (&hit)[R], long long (&pay)[R]) {
-  if (h.kind == HT_DIRECT) {  // one load per row; dispatch on the cell width once
+__device__ __forceinline__ void ht_probe_n(const HTP& h, const int kind, const int width,
+                                           const unsigned long long (&key)[R], const bool (&act)[R], bool (&hit)[R],
+                                           long long (&pay)[R]) {
+  if (kind == HT_DIRECT) {  // one load per row; dispatch on the cell width once
     unsigned long long idx[R];
     bool in[R];
 #pragma unroll
@@ -122,17 +127,17 @@ __device__ __forceinline__ void ht_probe_n(const HTP& h, const unsigned long lon
       in[j] = act[j] && idx[j] < h.nslots;
     }
     uint32_t v[R];
-    if (h.width == 0) {
+    if (width == 0) {
 #pragma unroll
       for (int j = 0; j < R; j++) v[j] = in[j] ? (__ldg((const uint32_t*)h.slots + (idx[j] >> 5)) >> (idx[j] & 31)) & 1u : 0u;
 #pragma unroll
       for (int j = 0; j < R; j++) { hit[j] = v[j] != 0; pay[j] = 1; }
       return;
     }
-    if (h.width == 1) {
+    if (width == 1) {
 #pragma unroll
       for (int j = 0; j < R; j++) v[j] = in[j] ? (uint32_t)__ldg((const unsigned char*)h.slots + idx[j]) : 0u;
-    } else if (h.width == 2) {
+    } else if (width == 2) {
 #pragma unroll
       for (int j = 0; j < R; j++) v[j] = in[j] ? (uint32_t)__ldg((const unsigned short*)h.slots + idx[j]) : 0u;
     } else {
@@ -153,11 +158,11 @@ __device__ __forceinline__ void ht_probe_n(const HTP& h, const unsigned long lon
   for (int j = 0; j < R; j++) {
     hit[j] = false;
     pay[j] = 0;
-    live[j] = act[j] && (h.kind == HT_MAP64 ? key[j] != EMPTY64 : (uint32_t)key[j] != EMPTY32);
+    live[j] = act[j] && (kind == HT_MAP64 ? key[j] != EMPTY64 : (uint32_t)key[j] != EMPTY32);
     pos[j] = ht_home(h, key[j]);
     any |= live[j];
   }
-  if (h.kind == HT_MAP32) {
+  if (kind == HT_MAP32) {
     const unsigned long long* s = (const unsigned long long*)h.slots;
     while (any) {
       unsigned long long v[R];
@@ -173,7 +178,7 @@ __device__ __forceinline__ void ht_probe_n(const HTP& h, const unsigned long lon
         else { pos[j] = (pos[j] + 1) & h.mask; any = true; }
       }
     }
-  } else if (h.kind == HT_SET32) {
+  } else if (kind == HT_SET32) {
     const uint32_t* s = (const uint32_t*)h.slots;
     while (any) {
       uint32_t v[R];

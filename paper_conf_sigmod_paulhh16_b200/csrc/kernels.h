@@ -2,6 +2,8 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <string>
+
 #include "common.h"
 
 namespace gpl {
@@ -21,7 +23,14 @@ cudaError_t launch_build(const BuildDesc& d, bool trivial, const HTHeader& known
 cudaError_t launch_header_init(HTHeader* hdr, cudaStream_t s);
 
 // A2-A8 fused persistent pipeline. d.smem_bytes of dynamic shared memory.
-cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s);
+// use_jit: launch the plan-specialised NVRTC build of the kernel (compiled and
+// cached on first use of a shape); falls back to the generic build when NVRTC
+// is unavailable (reason in *jit_err).
+cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s, bool use_jit, std::string* jit_err);
+
+// JIT: compile (and, when load is true, load) the specialised kernel for d's
+// shape. Returns false with a message when NVRTC is unavailable or fails.
+bool jit_prepare(const PipeDesc& d, bool load, std::string* err);
 
 // Column min/max (int32 or int64 column, n rows) -> out[0] = min, out[1] = max.
 cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s);

@@ -1,433 +1,41 @@
-// pipeline.cu — A2-A8: the fused, warp-specialised, persistent probe-segment
-// kernel for sm_100a.
-//
-// GPL's segment = concurrently running kernels connected by channels, fed one
-// tile at a time (§3.1, §3.3, §3.4,
-// P:191-203 §3.5). The B200 re-expression is ONE kernel per segment:
-//
-//   producer warp (lane 0)                     consumer warps (W per CTA)
-//   ----------------------                     -------------------------------------------
-//   claim tile t = atomicAdd(counter)   A2     wait full[slot]
-//   for each stage of the tile:                for each 128-row packet of the stage
-//     wait empty[slot]                         (4 consecutive rows per lane):
-//     cp.async.bulk every column       A3        filters (selection = map only)  A4
-//       (TMA engine, L2 evict_first)             stage-phase probes (first `nsprobe`)     A5
-//     arrive.expect_tx full[slot]                value terms computable here (pushdown)
-//                                                ballot/popc compaction -> warp queue     A8
-//                                                whenever >= 128 survivors are queued:
-//                                                  remaining probes, where, group-by,   A5-A7
-//                                                  exact int64 aggregation
-//                                              arrive empty[slot]
-//
-// The ring of `depth` stages replaces the paper's "number of channels" n and
-// the warp packet replaces its packet size p. Survivors travel
-// through per-warp shared-memory queues carrying their values, so no operator
-// writes an intermediate to HBM; the only global writes are the
-// few-KB aggregate partials (int128) and counters.
-//
-// All shared-memory accesses use integer offsets into the one __shared__
-// array so they compile to plain LDS/STS (no generic-address conversion).
-#include <climits>
-
-#include "device_common.cuh"
+// pipeline.cu — generic (precompiled) instantiation of the fused probe-segment
+// kernel (pipeline_body.cuh) and its launcher. The launcher prefers the
+// plan-specialised NVRTC build of the same body (jit.cpp) when available.
 #include "kernels.h"
+#include "pipeline_body.cuh"
 
 namespace gpl {
 namespace {
 
-extern __shared__ __align__(128) unsigned char g_smem[];
-
-constexpr int kMaxWarps = 17;  // 16 consumers + 1 producer
-constexpr int kMaxThreads = kMaxWarps * 32;
-constexpr int kMaxDepth = 8;
-// fixed shared-memory region (see PipeDesc.off_*):
-constexpr int kOffFull = 0;       // unsigned long long[kMaxDepth]
-constexpr int kOffEmpty = 64;     // unsigned long long[kMaxDepth]
-constexpr int kOffHdr = 128;      // int4[kMaxDepth]
-constexpr int kOffHtp = 256;      // HTP[MAXHT]
-constexpr int kOffCnt = 1024;     // unsigned long long[kMaxWarps][MAXOPS]
-static_assert(kOffHtp + MAXHT * sizeof(HTP) <= kOffCnt, "HTP region overflow");
-static_assert(kOffCnt + kMaxWarps * MAXOPS * 8 <= 4096, "fixed region overflow");
-
-template <class T>
-__device__ __forceinline__ T& S(uint32_t off) {
-  return *reinterpret_cast<T*>(g_smem + off);
-}
-
-__device__ __forceinline__ unsigned lanemask_lt() {
-  unsigned m;
-  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
-  return m;
-}
-
-// RPL consecutive rows (r0 % 4 == 0) of one staged column, widened to int64.
-__device__ __forceinline__ void ld_rows(uint32_t a, int w, long long (&x)[RPL]) {
-  if (w == 4) {
-    const int4 v = S<int4>(a);
-    x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
-  } else {
-    const longlong2 u = S<longlong2>(a);
-    const longlong2 v = S<longlong2>(a + 16);
-    x[0] = u.x; x[1] = u.y; x[2] = v.x; x[3] = v.y;
-  }
-}
-
-__device__ __forceinline__ long long qget(const PipeDesc& d, uint32_t qb, int f, int i) {
-  const uint32_t a = qb + d.qoff[f];
-  return d.qw[f] == 4 ? (long long)S<int>(a + i * 4) : S<long long>(a + i * 8);
-}
-__device__ __forceinline__ void qput(const PipeDesc& d, uint32_t qb, int f, int i, long long v) {
-  const uint32_t a = qb + d.qoff[f];
-  if (d.qw[f] == 4) S<int>(a + i * 4) = (int)v;
-  else S<long long>(a + i * 8) = v;
-}
-
-__device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
-  return (unsigned)p[0] + (unsigned)p[1] + (unsigned)p[2] + (unsigned)p[3];
-}
-__device__ __forceinline__ bool any4(const bool (&p)[RPL]) { return p[0] | p[1] | p[2] | p[3]; }
-
-// Queue phase on up to RPL*32 queued survivors starting at qhead: lane `lane`
-// owns entries qhead + j*32 + lane (j < RPL) that are < n. Remaining probes,
-// where residuals, group-by and the exact aggregation (A5-A7).
-__device__ __noinline__ void drain(const PipeDesc& d, uint32_t qb, int qhead, int n, unsigned long long* cnt,
-                                   long long* acc, int lane) {
-  const HTP* htp = &S<HTP>(kOffHtp);
-  int idx[RPL];
-  bool p[RPL];
-#pragma unroll
-  for (int j = 0; j < RPL; j++) {
-    const int e = j * 32 + lane;
-    idx[j] = (qhead + e) & (QCAP - 1);
-    p[j] = e < n;
-  }
-  int op = d.nfilt + d.nsprobe;
-  for (int pi = d.nsprobe; pi < d.nprobe; pi++, op++) {
-    const Probe P = d.probe[pi];
-    if (__any_sync(0xffffffffu, any4(p))) {
-      unsigned long long k[RPL];
-#pragma unroll
-      for (int j = 0; j < RPL; j++) {
-        k[j] = (uint32_t)qget(d, qb, P.k1, idx[j]);
-        if (P.k2 >= 0) k[j] = (k[j] << 32) | (uint32_t)qget(d, qb, P.k2, idx[j]);
-      }
-      bool hit[RPL];
-      long long v[RPL];
-      ht_probe_n<RPL>(htp[P.ht], k, p, hit, v);
-#pragma unroll
-      for (int j = 0; j < RPL; j++) {
-        if (P.kind == P_MARK) {
-          if (p[j] && P.out >= 0) qput(d, qb, P.out, idx[j], hit[j] ? 1 : 0);
-        } else {
-          if (hit[j] && P.out >= 0) qput(d, qb, P.out, idx[j], v[j]);
-          p[j] = hit[j];
-        }
-      }
-    }
-    const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
-    if (lane == 0) cnt[op] += c;
-  }
-  for (int r = 0; r < d.nresid; r++, op++) {
-    const Resid& R = d.resid[r];
-    const int kind = R.kind, fa = R.a, fb = R.b;
-#pragma unroll
-    for (int j = 0; j < RPL; j++) {
-      if (!p[j]) continue;
-      const long long a = qget(d, qb, fa, idx[j]);
-      if (kind == R_EQ) {
-        p[j] = a == qget(d, qb, fb, idx[j]);
-      } else if (kind == R_PAIRS) {
-        const long long b = qget(d, qb, fb, idx[j]);
-        bool ok = false;
-        for (int i = 0; i < R.npairs; i++) ok |= (a == R.pa[i]) & (b == R.pb[i]);
-        p[j] = ok;
-      } else if (kind == R_RANGE) {
-        p[j] = a >= R.lo && a <= R.hi;
-      } else {
-        p[j] = (unsigned long long)a < 64ull && ((R.mask >> a) & 1ull);
-      }
-    }
-    const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
-    if (lane == 0) cnt[op] += c;
-  }
-  if (!__any_sync(0xffffffffu, any4(p))) return;
-  unsigned long long* stab = &S<unsigned long long>(d.off_agg);
-#pragma unroll
-  for (int j = 0; j < RPL; j++) {
-    if (!p[j]) continue;
-    int gid = 0;
-    bool ok = true;
-    for (int g = 0; g < d.ngroup; g++) {
-      const GroupDim& G = d.gdim[g];
-      long long v = qget(d, qb, G.field, idx[j]);
-      if (G.transform == G_YEAR) v = (int)v / 10000;
-      const long long o = v - G.lo;
-      if ((unsigned long long)o >= (unsigned long long)G.size) ok = false;
-      gid += (int)o * G.stride;
-    }
-    if (!ok) {
-      atomicOr(d.err, ERR_DOMAIN);
-      continue;
-    }
-    long long val = 0;
-    for (int t = 0; t < d.nterm; t++) {
-      if (d.term_field[t] >= 0) {
-        val += qget(d, qb, d.term_field[t], idx[j]);
-        continue;
-      }
-      const Term& T = d.term[t];
-      long long prod = T.sign;
-      for (int f = 0; f < T.nfact; f++) {
-        const Factor& F = T.f[f];
-        prod *= F.field < 0 ? F.a : F.a + (long long)F.b * qget(d, qb, F.field, idx[j]);
-      }
-      val += prod;
-    }
-    for (int a = 0; a < d.nagg; a++) {
-      const Agg& A = d.agg[a];
-      long long c = 1;
-      if (A.kind == A_SUM) c = val;
-      else if (A.kind == A_SUMIF) c = qget(d, qb, A.field, idx[j]) != 0 ? val : 0;
-      else if (A.kind == A_SUMIFEQ) c = qget(d, qb, A.field, idx[j]) == A.c ? val : 0;
-      if (d.agg_mode == AGG_REG) acc[a] += c;
-      else if (c != 0) {
-        if (d.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * d.nagg + a], (unsigned long long)c);
-        else atomic_add_i128(d.partials + 2 * (gid * d.nagg + a), c);
-      }
-    }
-  }
-}
-
-__device__ __forceinline__ void flush_reg(const PipeDesc& d, long long (&acc)[MAXA], int lane) {
-#pragma unroll
-  for (int a = 0; a < MAXA; a++) {
-    if (a < d.nagg) {
-      const long long s = warp_sum_i64(acc[a]);
-      if (lane == 0 && s != 0) atomic_add_i128(d.partials + 2 * a, s);
-      acc[a] = 0;
-    }
-  }
-}
-
-__global__ void __launch_bounds__(kMaxThreads, 1) pipeline_kernel(const __grid_constant__ PipeDesc d) {
-  unsigned long long* full = &S<unsigned long long>(kOffFull);
-  unsigned long long* empty = &S<unsigned long long>(kOffEmpty);
-  int4* hdr = &S<int4>(kOffHdr);
-  HTP* htp = &S<HTP>(kOffHtp);
-  unsigned long long* cnt_all = &S<unsigned long long>(kOffCnt);
-  unsigned long long* stab = &S<unsigned long long>(d.off_agg);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int W = d.nwarps;
-
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < d.depth; i++) {
-      mbar_init(&full[i], 1);
-      mbar_init(&empty[i], (uint32_t)W);
-    }
-    fence_mbar_init();
-  }
-  if (threadIdx.x < d.nht) htp[threadIdx.x] = load_htp(d.ht[threadIdx.x]);
-  for (int i = threadIdx.x; i < kMaxWarps * MAXOPS; i += blockDim.x) cnt_all[i] = 0;
-  if (d.agg_mode == AGG_SMEM)
-    for (int i = threadIdx.x; i < d.ngroups_total * d.nagg; i += blockDim.x) stab[i] = 0;
-  __syncthreads();
-
-  if (warp == W) {
-    // ------------------------------------------------------------ producer
-    if (lane == 0) {
-      const unsigned long long pol = policy_evict_first();
-      uint32_t slot = 0, phase = 0;
-      for (;;) {
-        const unsigned long long t = atomicAdd(d.tile_counter, 1ull);
-        const long long r0 = (long long)t * d.tile_rows;
-        if (r0 >= d.nrows) break;
-        const long long rn = min(d.tile_rows, d.nrows - r0);
-        for (long long s0 = 0; s0 < rn; s0 += d.stage_rows) {
-          const int n = (int)min((long long)d.stage_rows, rn - s0);
-          mbar_wait(&empty[slot], phase ^ 1u);
-          const long long row = r0 + s0;
-          hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, (s0 + d.stage_rows >= rn) ? 1 : 0);
-          uint32_t bytes = 0;
-          for (int c = 0; c < d.ncols; c++) bytes += ((uint32_t)n * d.colw[c] + 15u) & ~15u;
-          mbar_arrive_expect_tx(&full[slot], bytes);
-          unsigned char* dst = g_smem + d.off_ring + (size_t)slot * d.slot_bytes;
-          for (int c = 0; c < d.ncols; c++)
-            bulk_g2s(dst + d.coloff[c], d.col[c] + row * d.colw[c], ((uint32_t)n * d.colw[c] + 15u) & ~15u,
-                     &full[slot], pol);
-          if (++slot == (uint32_t)d.depth) { slot = 0; phase ^= 1u; }
-        }
-      }
-      mbar_wait(&empty[slot], phase ^ 1u);
-      hdr[slot] = make_int4(0, 0, -1, 0);
-      mbar_arrive(&full[slot]);
-    }
-    return;
-  }
-
-  // -------------------------------------------------------------- consumers
-  unsigned long long* cnt = cnt_all + warp * MAXOPS;
-  const uint32_t qb = (uint32_t)d.off_queue + (uint32_t)warp * (uint32_t)d.qbytes;
-  long long acc[MAXA] = {0, 0, 0, 0};
-  int qhead = 0, qcount = 0;
-  uint32_t slot = 0, phase = 0;
-  const int nfilt = d.nfilt, nsprobe = d.nsprobe, npush = d.npush;
-  for (;;) {
-    mbar_wait(&full[slot], phase);
-    const int4 h = hdr[slot];
-    const int n = h.z;
-    if (n < 0) break;
-    const uint32_t sb = (uint32_t)d.off_ring + slot * (uint32_t)d.slot_bytes;
-    const int nit = (n + 127) >> 7;
-    for (int it = warp; it < nit; it += W) {
-      const int r0 = (it << 7) + (lane << 2);
-      bool p[RPL];
-#pragma unroll
-      for (int j = 0; j < RPL; j++) p[j] = r0 + j < n;
-      // A4 selection: predicates on staged columns, 4 rows per lane
-      for (int f = 0; f < nfilt; f++) {
-        const Filt F = d.filt[f];
-        long long x[RPL];
-        ld_rows(sb + d.coloff[F.ref] + r0 * d.colw[F.ref], d.colw[F.ref], x);
-#pragma unroll
-        for (int j = 0; j < RPL; j++) p[j] = p[j] && filt_pass(F, x[j]);
-        const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
-        if (lane == 0) cnt[f] += c;
-      }
-      // A5 stage-phase probes (keys from the stage; loads of the 4 rows in flight together)
-      long long sreg[MAXSP][RPL];
-#pragma unroll
-      for (int sp = 0; sp < MAXSP; sp++) {
-#pragma unroll
-        for (int j = 0; j < RPL; j++) sreg[sp][j] = 0;
-        if (sp < nsprobe) {
-          const Probe P = d.probe[sp];
-          if (__any_sync(0xffffffffu, any4(p))) {
-            long long k1[RPL];
-            ld_rows(sb + d.coloff[P.k1] + r0 * d.colw[P.k1], d.colw[P.k1], k1);
-            unsigned long long k[RPL];
-#pragma unroll
-            for (int j = 0; j < RPL; j++) k[j] = (uint32_t)k1[j];
-            if (P.k2 >= 0) {
-              long long k2[RPL];
-              ld_rows(sb + d.coloff[P.k2] + r0 * d.colw[P.k2], d.colw[P.k2], k2);
-#pragma unroll
-              for (int j = 0; j < RPL; j++) k[j] = (k[j] << 32) | (uint32_t)k2[j];
-            }
-            bool hit[RPL];
-            long long v[RPL];
-            ht_probe_n<RPL>(htp[P.ht], k, p, hit, v);
-#pragma unroll
-            for (int j = 0; j < RPL; j++) {
-              if (P.kind == P_MARK) {
-                sreg[sp][j] = hit[j] ? 1 : 0;
-              } else {
-                sreg[sp][j] = v[j];
-                p[j] = hit[j];
-              }
-            }
-          }
-          const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
-          if (lane == 0) cnt[nfilt + sp] += c;
-        }
-      }
-      // A8 compaction into the warp's survivor queue (the on-chip channel)
-      int base = qcount;
-      int pos[RPL];
-#pragma unroll
-      for (int j = 0; j < RPL; j++) {
-        const unsigned m = __ballot_sync(0xffffffffu, p[j]);
-        pos[j] = (qhead + base + __popc(m & lanemask_lt())) & (QCAP - 1);
-        base += __popc(m);
-      }
-      if (base == qcount) continue;
-      for (int e = 0; e < npush; e++) {
-        const Push E = d.push[e];
-        const uint32_t qa = qb + d.qoff[e];
-        const int qw = d.qw[e];
-        long long v[RPL];
-        if (E.kind == PUSH_COL) {
-          ld_rows(sb + d.coloff[E.src] + r0 * d.colw[E.src], d.colw[E.src], v);
-        } else if (E.kind == PUSH_SREG) {
-#pragma unroll
-          for (int j = 0; j < RPL; j++) v[j] = E.src == 0 ? sreg[0][j] : sreg[1][j];
-        } else {  // pushed-down value term: sign * prod(a + b * x)
-          const Term& T = d.sterm[E.src];
-#pragma unroll
-          for (int j = 0; j < RPL; j++) v[j] = T.sign;
-          for (int f = 0; f < T.nfact; f++) {
-            const Factor F = T.f[f];
-            long long x[RPL];
-            if (F.field >= 0) {
-              ld_rows(sb + d.coloff[F.field] + r0 * d.colw[F.field], d.colw[F.field], x);
-            } else {
-#pragma unroll
-              for (int j = 0; j < RPL; j++) x[j] = F.field == SREF_CONST ? 0 : (F.field == -2 ? sreg[0][j] : sreg[1][j]);
-            }
-#pragma unroll
-            for (int j = 0; j < RPL; j++) v[j] *= F.a + (long long)F.b * x[j];
-          }
-        }
-        if (qw == 4) {
-#pragma unroll
-          for (int j = 0; j < RPL; j++)
-            if (p[j]) S<int>(qa + pos[j] * 4) = (int)v[j];
-        } else {
-#pragma unroll
-          for (int j = 0; j < RPL; j++)
-            if (p[j]) S<long long>(qa + pos[j] * 8) = v[j];
-        }
-      }
-      qcount = base;
-      if (qcount >= RPL * 32) {
-        __syncwarp();
-        drain(d, qb, qhead, RPL * 32, cnt, acc, lane);
-        __syncwarp();
-        qhead = (qhead + RPL * 32) & (QCAP - 1);
-        qcount -= RPL * 32;
-      }
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[slot]);
-    if (d.flush_each_tile && h.w) flush_reg(d, acc, lane);
-    if (++slot == (uint32_t)d.depth) { slot = 0; phase ^= 1u; }
-  }
-  if (qcount > 0) {
-    __syncwarp();
-    drain(d, qb, qhead, qcount, cnt, acc, lane);
-  }
-  __syncwarp();
-  if (d.agg_mode == AGG_REG) flush_reg(d, acc, lane);
-  if (lane == 0) {
-    const int nops = d.nfilt + d.nprobe + d.nresid;
-    for (int o = 0; o < nops; o++)
-      if (cnt[o]) atomicAdd(d.op_pass + o, cnt[o]);
-  }
-  if (d.agg_mode == AGG_SMEM) {
-    named_bar_sync(1, (uint32_t)W * 32u);
-    for (int i = threadIdx.x; i < d.ngroups_total * d.nagg; i += W * 32) {
-      const long long v = (long long)stab[i];
-      if (v != 0) atomic_add_i128(d.partials + 2 * i, v);
-    }
-  }
+__global__ void __launch_bounds__(pipe::kMaxThreads, 1) pipeline_kernel(const __grid_constant__ PipeDesc d) {
+  pipe::pipeline_body(d);
 }
 
 }  // namespace
 
-cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s) {
-  static int configured = 0;
-  if (d.smem_bytes > configured) {
-    cudaError_t e = cudaFuncSetAttribute(pipeline_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, d.smem_bytes);
-    if (e != cudaSuccess) return e;
-    configured = d.smem_bytes;
-  }
-  if (d.nwarps + 1 > kMaxWarps || d.depth > kMaxDepth || d.nsprobe > MAXSP || d.stage_rows % 128)
+// jit.cpp: plan-specialised kernel for this descriptor's shape (nullptr if
+// NVRTC is unavailable or disabled).
+const void* jit_pipeline_kernel(const PipeDesc& d, std::string* err);
+
+cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s, bool use_jit, std::string* jit_err) {
+  if (d.nwarps + 1 > pipe::kMaxWarps || d.depth > pipe::kMaxDepth || d.nsprobe > MAXSP || d.stage_rows % 128)
     return cudaErrorInvalidValue;
-  pipeline_kernel<<<grid, (d.nwarps + 1) * 32, d.smem_bytes, s>>>(d);
-  return cudaGetLastError();
+  const void* fn = nullptr;
+  if (use_jit) fn = jit_pipeline_kernel(d, jit_err);
+  if (!fn) {
+    static int configured = 0;
+    fn = (const void*)pipeline_kernel;
+    if (d.smem_bytes > configured) {
+      cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, d.smem_bytes);
+      if (e != cudaSuccess) return e;
+      configured = d.smem_bytes;
+    }
+  }
+  void* args[] = {(void*)&d};
+  return cudaLaunchKernel(fn, dim3(grid), dim3((d.nwarps + 1) * 32), args, (size_t)d.smem_bytes, s);
 }
 
 int pipeline_fixed_smem() { return 4096; }
-int pipeline_max_consumer_warps() { return kMaxWarps - 1; }
+int pipeline_max_consumer_warps() { return pipe::kMaxWarps - 1; }
 
 }  // namespace gpl

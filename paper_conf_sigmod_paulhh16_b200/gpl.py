@@ -28,7 +28,7 @@ GPL_COPY, GPL_BORROW = 0, 1
 EXPORTED = ["gpl_create", "gpl_destroy", "gpl_load_columns", "gpl_build_hash", "gpl_run_plan",
             "gpl_run_plan_kbe", "gpl_fetch_result", "gpl_fetch_partials", "gpl_decode_partials",
             "gpl_merge_partials", "gpl_sync", "gpl_choose_tile_rows", "gpl_set_option",
-            "gpl_check_plan", "gpl_last_error", "gpl_version"]
+            "gpl_check_plan", "gpl_compile_plan", "gpl_last_error", "gpl_version"]
 
 
 class GplError(RuntimeError):
@@ -51,7 +51,7 @@ class _Stats(ctypes.Structure):
                 ("probe_split", ctypes.c_int32), ("op_pass", ctypes.c_int64 * 16),
                 ("kernel_ms", ctypes.c_double), ("predicted_ms", ctypes.c_double),
                 ("bytes_scanned", ctypes.c_double), ("agg_mode", ctypes.c_int32), ("kbe", ctypes.c_int32),
-                ("intermediate_bytes", ctypes.c_double)]
+                ("jit", ctypes.c_int32), ("reserved", ctypes.c_int32), ("intermediate_bytes", ctypes.c_double)]
 
 
 class _Result(ctypes.Structure):
@@ -96,6 +96,7 @@ def load_library():
         "gpl_choose_tile_rows": ([P, ctypes.c_char_p, I64, ctypes.POINTER(_Model)], I32),
         "gpl_set_option": ([P, ctypes.c_char_p, I64], I32),
         "gpl_check_plan": ([P, ctypes.c_char_p], I32),
+        "gpl_compile_plan": ([P, ctypes.c_char_p, I64], I32),
         "gpl_last_error": ([P], ctypes.c_char_p),
         "gpl_version": ([], ctypes.c_char_p),
     }
@@ -228,6 +229,10 @@ class Context:
 
     def check_plan(self, segment: str):
         self._check(self._lib.gpl_check_plan(self._h, segment.encode()))
+
+    def compile_plan(self, segment: str, tile_rows: int = 0):
+        """Warm the plan-specialised kernel cache (NVRTC) for this probe segment."""
+        self._check(self._lib.gpl_compile_plan(self._h, segment.encode(), int(tile_rows)))
 
     def sync(self):
         self._check(self._lib.gpl_sync(self._h))

@@ -20,9 +20,12 @@ pytestmark = pytest.mark.gpu
 QUERIES = queries.QUERIES
 
 
-@pytest.fixture(scope="module")
-def ctx():
+@pytest.fixture(scope="module", params=[1, 0], ids=["jit", "generic"])
+def ctx(request):
+    """Both builds of the fused kernel: plan-specialised (NVRTC) and generic."""
     c = gpl.Context(0)
+    c.set_option("jit", request.param)
+    c.jit = request.param
     yield c
     c.close()
 
@@ -43,6 +46,7 @@ def test_parity_small(ctx, q, sf, seed):
     r = _gpu(ctx, db, q, _params(q))
     o = oracle.run(q, db, _params(q))
     assert r.keys == o.keys and r.aggs == o.aggs
+    assert r.stats["jit"] == ctx.jit
     assert sum(a[0] for a in r.aggs) == (r.stats["op_pass"][-1] if r.stats["op_pass"] else db.nrows("lineitem"))
 
 

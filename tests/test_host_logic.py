@@ -99,3 +99,20 @@ def test_merge_partials_exact():
         if got >= 1 << 127:
             got -= 1 << 128
         assert got == sum(v[i] for v in vals)
+
+
+def test_jit_compiles_every_plan():
+    """NVRTC builds the plan-specialised kernel of every paper query (no GPU needed)."""
+    db = tpchgen.generate(0.01, seed=1)
+    ctx = gpl.Context(device=-1)
+    queries.load_database(ctx, db)
+    for q in queries.QUERIES:
+        segs = queries.segments(queries.plan_text(q, db, (19981101,) if q == "L1" else None))
+        for s in segs[:-1]:
+            ctx.build_hash(s)
+        try:
+            ctx.compile_plan(segs[-1])
+        except gpl.GplError as e:
+            if "NVRTC unavailable" in str(e):
+                pytest.skip(str(e))
+            raise
