@@ -1,0 +1,162 @@
+"""Paper experiments re-run on B200 (bench.py --sweep / --kbe).
+
+config 2 (tile sweep, §5.2 Figs 12-13, Eq 10): the fused kernel's
+  measured time T(Δ) for Δ = 2^9..2^22 rows next to the A9 model's estimate
+  for the same Δ; reports Eq 10 relative error |T_meas - T_est| / T_meas per
+  point and the model's argmin vs the measured argmin. Results must be
+  identical at every Δ (checked).
+config 5 (fused vs KBE, §2.2 Obs 1 / §5.3.2 Figs 3, 16-18): Q14 with shipdate
+  windows giving ~1-100% selectivity, Q5 and Q9-wide at SF 10: kernel/step
+  latency of the fused pipeline and of the kernel-at-a-time materialising
+  baseline, and the intermediate bytes materialised, normalised to input.
+
+Both print one JSON line and write the full table to --out.
+"""
+from __future__ import annotations
+
+import json
+import math
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+
+def _setup(q, sf, seed, tables=None):
+    import numpy as np  # noqa: F401
+    import torch
+
+    import tpchgen
+    from paper_conf_sigmod_paulhh16_b200 import gpl, queries
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_stream(torch.cuda.Stream(device=dev))  # a real stream shared with libgpl
+    stream = torch.cuda.current_stream()
+    db = tpchgen.generate(sf, seed=seed, tables=tables or sorted(set(queries.TABLES[q]) | {"region", "nation"}))
+
+    class D:
+        pass
+    ddb = D()
+    ddb.tables = {t: {c: torch.from_numpy(a).to(dev) for c, a in cols.items()} for t, cols in db.tables.items()}
+    ctx = gpl.Context(0, stream=stream)
+    queries.load_database(ctx, ddb)
+    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size, dtype=torch.uint8, device=dev)
+    return db, ctx, flush, stream
+
+
+def tile_sweep(q="Q5", sf=1.0, seed=20160626, reps=5, out=None):
+    import torch
+
+    from paper_conf_sigmod_paulhh16_b200 import queries
+    db, ctx, flush, stream = _setup(q, sf, seed)
+    segs = queries.segments(queries.plan_text(q, db))
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+
+    def measure(tile):
+        ts, r = [], None
+        for i in range(reps + 2):
+            for s in segs[:-1]:
+                ctx.build_hash(s)
+            flush.zero_()
+            ctx.run_plan(segs[-1], tile)
+            r = ctx.fetch_result()
+            if i >= 2:
+                ts.append(r.stats["kernel_ms"])
+        return statistics.median(ts), r
+
+    t_auto, r_auto = measure(0)
+    ref = (r_auto.keys, r_auto.aggs)
+    rows = []
+    for e in range(9, 23):
+        tile = 1 << e
+        t, r = measure(tile)
+        assert (r.keys, r.aggs) == ref, "result changed with tile_rows"
+        est = r.stats["predicted_ms"]
+        rows.append({"tile_rows": r.stats["tile_rows_used"], "tile_bytes": r.stats["tile_rows_used"] * r.stats["bytes_scanned"] / max(1, r.stats["rows_scanned"]),
+                     "measured_ms": t, "predicted_ms": est, "rel_error": abs(t - est) / t,
+                     "stage_rows": r.stats["stage_rows"], "ring_depth": r.stats["ring_depth"],
+                     "consumer_warps": r.stats["consumer_warps"]})
+    best_meas = min(rows, key=lambda x: x["measured_ms"])
+    best_pred = min(rows, key=lambda x: (x["predicted_ms"], -x["tile_rows"]))
+    summary = {"experiment": "tile_sweep (config 2)", "query": q, "sf": sf,
+               "auto": {"tile_rows": r_auto.stats["tile_rows_used"], "measured_ms": t_auto,
+                        "predicted_ms": r_auto.stats["predicted_ms"]},
+               "measured_argmin_tile_rows": best_meas["tile_rows"], "measured_min_ms": best_meas["measured_ms"],
+               "model_argmin_tile_rows": best_pred["tile_rows"],
+               "model_pick_vs_best": t_auto / best_meas["measured_ms"],
+               "mean_rel_error": statistics.mean(x["rel_error"] for x in rows),
+               "results_identical_across_tiles": True, "points": rows}
+    if out:
+        with open(out, "w") as f:
+            json.dump(summary, f, indent=1)
+    return summary
+
+
+def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
+    import numpy as np
+    import torch
+
+    import tpchgen
+    from paper_conf_sigmod_paulhh16_b200 import queries
+    tables = ["part", "partsupp", "supplier", "customer", "orders", "lineitem", "nation", "region"]
+    db, ctx, flush, stream = _setup("Q9", sf, seed, tables)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sd = np.sort(db.tables["lineitem"]["l_shipdate"][:: max(1, db.nrows("lineitem") // 200000)])
+    cases = []
+    for pct in (1, 5, 10, 25, 50, 75, 100):  # Q14 selectivity sweep (Fig 3/18)
+        lo = 19920101
+        hi = 19990101 if pct == 100 else int(sd[min(len(sd) - 1, int(len(sd) * pct / 100))])
+        cases.append((f"Q14 sel~{pct}%", "Q14", (lo, hi)))
+    cases.append(("Q5", "Q5", None))
+    n_part = tpchgen.sizes(sf)["part"]
+    cases.append(("Q9-wide", "Q9", (math.ceil(0.054 * n_part),)))  # reading R5: ~%green% share
+    rows = []
+    for name, q, params in cases:
+        segs = queries.segments(queries.plan_text(q, db, params))
+
+        def timed(kbe):
+            ts, r = [], None
+            for i in range(reps + 1):
+                for s in segs[:-1]:
+                    ctx.build_hash(s)
+                flush.zero_()
+                ev0.record(stream)
+                if kbe:
+                    ctx.run_plan_kbe(segs[-1])
+                else:
+                    ctx.run_plan(segs[-1])
+                ev1.record(stream)
+                r = ctx.fetch_result()
+                if i >= 1:
+                    ts.append(ev0.elapsed_time(ev1))
+            return statistics.median(ts), r
+        tf, rf = timed(False)
+        tk, rk = timed(True)
+        assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs), name
+        inp = rf.stats["bytes_scanned"]
+        ops = rf.stats["op_pass"]
+        sel = (ops[0] / rf.stats["rows_scanned"]) if q == "Q14" and ops else None
+        rows.append({"case": name, "selectivity": sel, "input_bytes": inp,
+                     "fused_ms": tf, "kbe_ms": tk, "speedup": tk / tf,
+                     "fused_intermediate_bytes": rf.stats["intermediate_bytes"],
+                     "kbe_intermediate_bytes": rk.stats["intermediate_bytes"],
+                     "kbe_intermediate_over_input": rk.stats["intermediate_bytes"] / inp,
+                     "fused_kernel_ms": rf.stats["kernel_ms"]})
+    summary = {"experiment": "fused vs KBE (config 5)", "sf": sf, "points": rows,
+               "paper_context": "AMD A10: KBE intermediates 1.38x input at 100% Q14 selectivity vs 0.22x for GPL "
+                                "(P:402); GPL up to 48% faster than KBE (P:384)"}
+    if out:
+        with open(out, "w") as f:
+            json.dump(summary, f, indent=1)
+    return summary
+
+
+if __name__ == "__main__":
+    which = sys.argv[1] if len(sys.argv) > 1 else "sweep"
+    if which == "sweep":
+        s = tile_sweep(out=os.path.join(ROOT, "gpurun_out", "sweep_config2.json"))
+    else:
+        s = kbe_compare(out=os.path.join(ROOT, "gpurun_out", "kbe_config5.json"))
+    s.pop("points", None)
+    print(json.dumps(s))

@@ -158,9 +158,23 @@ gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32_t* ht_i
  * GPL_E_OVERFLOW (value bound not provably exact). */
 gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows);
 
+/* Whole query in one call: `plan` holds the build segments followed by the
+ * probe segment (split at 'build NAME' / 'run TABLE' lines); equivalent to
+ * gpl_build_hash for each build segment then gpl_run_plan. Once every segment
+ * is prepared and profiled, the sequence (hash builds + fused kernel) is
+ * recorded as a CUDA graph and later calls replay it with a single
+ * cudaGraphLaunch while the tables, hash tables and options are unchanged
+ * (any change falls back to the per-segment path and re-records). Fetch with
+ * gpl_fetch_result. Errors: as gpl_build_hash / gpl_run_plan. */
+gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_rows);
+
 /* Same plan, executed kernel-at-a-time with every operator's output
- * materialised in HBM: the paper's KBE baseline (§2.2, Fig 7). Same
- * result contract; stats.op_pass holds the same counts. For comparison only. */
+ * materialised in HBM: the paper's KBE baseline (§2.2, Fig 7): per
+ * operator a map kernel, a prefix sum and a scatter, the host reading each
+ * output cardinality to size the next buffers (so this call synchronises).
+ * Same result contract (bit-identical results); stats.kbe = 1 and
+ * stats.intermediate_bytes = bytes materialised between operators (flags,
+ * positions, payload and compacted columns). For comparison only (config 5). */
 gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment);
 
 /* Synchronise the stream and return the last run's result (host decode of

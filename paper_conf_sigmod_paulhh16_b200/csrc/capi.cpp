@@ -45,10 +45,19 @@ int type_width(int t) {
   }
 }
 
-constexpr int kScratchWords = MAXOPS + 4;  // [0] tile counter, [1..MAXOPS] op_pass, [MAXOPS+1] err bits
+// Device scratch, one allocation so a run's outputs come back in ONE D2H copy:
+//   word 0          error bits (u32), latched until fetched
+//   word 1          tile counter (zeroed per run)
+//   words 2..17     op_pass[MAXOPS]  (zeroed per run)
+//   words 18..      int128 partials [groups][aggs] (zeroed per run)
+constexpr int kScratchHead = 2 + MAXOPS;
+constexpr size_t kMaxPartialBytes = (size_t)(1 << 16) * MAXA * 16;
+constexpr size_t kScratchBytes = kScratchHead * 8 + kMaxPartialBytes;
 
-unsigned long long* op_pass_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 1; }
-unsigned int* err_ptr(gpl_ctx* ctx) { return (unsigned int*)(ctx->d_scratch + MAXOPS + 1); }
+unsigned int* err_ptr(gpl_ctx* ctx) { return (unsigned int*)ctx->d_scratch; }
+unsigned long long* counter_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 1; }
+unsigned long long* op_pass_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 2; }
+unsigned long long* partials_ptr(gpl_ctx* ctx) { return ctx->d_scratch + kScratchHead; }
 
 gpl_status check_dev(gpl_ctx* ctx) {
   if (!ctx) return GPL_E_ARG;
@@ -145,8 +154,10 @@ GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
     if ((e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking)) != cudaSuccess) return bad(e, "stream");
     ctx->own_stream = true;
   }
-  if ((e = cudaMalloc(&ctx->d_scratch, kScratchWords * sizeof(unsigned long long))) != cudaSuccess) return bad(e, "scratch");
-  if ((e = cudaMemset(ctx->d_scratch, 0, kScratchWords * sizeof(unsigned long long))) != cudaSuccess) return bad(e, "scratch");
+  if ((e = cudaMalloc(&ctx->d_scratch, kScratchBytes)) != cudaSuccess) return bad(e, "scratch");
+  if ((e = cudaMemset(ctx->d_scratch, 0, kScratchBytes)) != cudaSuccess) return bad(e, "scratch");
+  if ((e = cudaMallocHost(&ctx->h_stage, kScratchBytes)) != cudaSuccess) return bad(e, "pinned staging");
+  ctx->h_stage_cap = kScratchBytes;
   if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
   if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
   *out = ctx;
@@ -165,7 +176,8 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
       if (h.hdr) cudaFree(h.hdr);
     }
     if (ctx->d_scratch) cudaFree(ctx->d_scratch);
-    if (ctx->d_partials) cudaFree(ctx->d_partials);
+    for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
+    if (ctx->h_stage) cudaFreeHost(ctx->h_stage);
     if (ctx->d_minmax) cudaFree(ctx->d_minmax);
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
@@ -204,6 +216,7 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else {
     return fail(ctx, GPL_E_ARG, "unknown option '" + k + "'");
   }
+  ctx->opt_version++;
   return GPL_OK;
 }
 
@@ -277,17 +290,33 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
         c.cap_rows = cap;
       } else {
         const int64_t rows = std::max<int64_t>(64, (nrows + 63) / 64 * 64);
-        cudaError_t e = cudaMalloc(&c.dev, (size_t)rows * c.width);
-        if (e != cudaSuccess) {
-          cleanup();
-          return fail(ctx, GPL_E_NOMEM, std::string("cudaMalloc for column ") + c.name + ": " + cudaGetErrorString(e));
+        // reloading a table: reuse the old owned buffer of the same column when
+        // it is large enough (stream order keeps earlier readers safe)
+        Column* reuse = nullptr;
+        auto oldt = ctx->tables.find(t.name);
+        if (oldt != ctx->tables.end())
+          for (auto& oc : oldt->second.cols)
+            if (oc.name == c.name && oc.owned && oc.dev && oc.width == c.width && oc.cap_rows >= rows) reuse = &oc;
+        if (reuse) {
+          c.dev = reuse->dev;
+          c.cap_rows = reuse->cap_rows;
+          reuse->dev = nullptr;
+          reuse->owned = false;
+        } else {
+          cudaError_t e = cudaMalloc(&c.dev, (size_t)rows * c.width);
+          if (e != cudaSuccess) {
+            cleanup();
+            return fail(ctx, GPL_E_NOMEM, std::string("cudaMalloc for column ") + c.name + ": " + cudaGetErrorString(e));
+          }
+          c.cap_rows = rows;
         }
         c.owned = true;
-        c.cap_rows = rows;
+        const int64_t cap_rows = c.cap_rows;
         t.cols.push_back(c);  // owned from here on (cleanup frees it)
         if (nrows > 0)
           CK(cudaMemcpyAsync(c.dev, cols[i].data, (size_t)nrows * c.width, cudaMemcpyDefault, ctx->stream));
-        CK(cudaMemsetAsync(c.dev + (size_t)nrows * c.width, 0, (size_t)(rows - nrows) * c.width, ctx->stream));
+        CK(cudaMemsetAsync(c.dev + (size_t)nrows * c.width, 0, (size_t)(std::min(cap_rows, rows + 64) - nrows) * c.width,
+                           ctx->stream));
         t.cols.pop_back();
       }
       t.cols.push_back(c);
@@ -303,7 +332,9 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
   }
   auto old = ctx->tables.find(t.name);
   if (old != ctx->tables.end()) {
-    if (!ctx->host_only) cudaStreamSynchronize(ctx->stream);
+    bool any_owned = false;
+    for (auto& c : old->second.cols) any_owned |= c.owned && c.dev;
+    if (!ctx->host_only && any_owned) cudaStreamSynchronize(ctx->stream);
     for (auto& c : old->second.cols) free_column(ctx, c);
     for (auto& h : ctx->hts)
       if (h.src_table == t.name) h.valid = false;
@@ -332,9 +363,66 @@ GPL_API gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment) {
   return st ? fail(ctx, st, err) : GPL_OK;
 }
 
+// A prepared build is reusable while its scanned table, its destination and
+// source hash tables and the options are unchanged.
+static bool build_cache_valid(gpl_ctx* ctx, const PreparedBuild& P) {
+  auto ti = ctx->tables.find(P.table);
+  bool ok = ti != ctx->tables.end() && ti->second.version == P.table_version && P.opt_version == ctx->opt_version &&
+            P.ht_index >= 0 && P.ht_index < (int)ctx->hts.size();
+  if (ok) {
+    const HTRef r = ctx->hts[P.ht_index].ref();
+    ok = std::memcmp(&r, &P.dest_ref, sizeof(HTRef)) == 0;
+  }
+  for (size_t i = 0; ok && i < P.src_ids.size(); i++) {
+    const HashTable& Hs = ctx->hts[P.src_ids[i]];
+    const HTRef r = Hs.ref();
+    ok = Hs.valid && std::memcmp(&r, &P.desc.src[i], sizeof(HTRef)) == 0;
+  }
+  return ok;
+}
+
+static bool run_cache_valid(gpl_ctx* ctx, const PreparedRun& P) {
+  auto lam = ctx->lambda.find(P.text);
+  const size_t lambda_n = lam == ctx->lambda.end() ? 0 : lam->second.size();
+  auto ti = ctx->tables.find(P.li.table);
+  bool ok = ti != ctx->tables.end() && ti->second.version == P.table_version && P.opt_version == ctx->opt_version &&
+            P.lambda_n == lambda_n;
+  for (int i = 0; ok && i < P.desc.nht; i++) {
+    const HashTable& H = ctx->hts[P.li.ht_ids[i]];
+    const HTRef r = H.ref();
+    ok = H.valid && std::memcmp(&r, &P.desc.ht[i], sizeof(HTRef)) == 0;
+  }
+  return ok;
+}
+
+// Events around the fused kernel; inside a graph capture they must be
+// external so the replayed graph still reports the kernel time.
+static cudaError_t record_event(gpl_ctx* ctx, cudaEvent_t ev) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(ctx->stream, &cs);
+  if (cs == cudaStreamCaptureStatusActive) return cudaEventRecordWithFlags(ev, ctx->stream, cudaEventRecordExternal);
+  return cudaEventRecord(ev, ctx->stream);
+}
+
 GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32_t* ht_id) {
   if (!ctx || !build_segment) return GPL_E_ARG;
   ctx->err.clear();
+  // fast path: the same segment over unchanged tables / hash tables / options
+  if (!ctx->host_only) {
+    auto ci = ctx->build_cache.find(build_segment);
+    if (ci != ctx->build_cache.end()) {
+      const PreparedBuild& P = ci->second;
+      if (build_cache_valid(ctx, P)) {
+        gpl_status st = check_dev(ctx);
+        if (st) return st;
+        CK(launch_build(P.desc, P.trivial, P.known, ctx->sms, ctx->stream));
+        ctx->hts[P.ht_index].valid = true;
+        if (ht_id) *ht_id = P.ht_index;
+        return GPL_OK;
+      }
+      ctx->build_cache.erase(ci);
+    }
+  }
   Segment s;
   std::string err;
   if (!parse_segment(build_segment, &s, &err)) return fail(ctx, GPL_E_PLAN, err);
@@ -422,15 +510,35 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
   CK(launch_build(d, trivial, known, ctx->sms, ctx->stream));
   H.valid = true;
   if (ht_id) *ht_id = H.id;
+  // invalidate prepared builds/runs that referenced this table's old shape
+  PreparedBuild P;
+  P.desc = d;
+  P.shape = shape;
+  P.trivial = trivial;
+  P.known = known;
+  P.ht_index = H.id;
+  P.dest_ref = H.ref();
+  P.name = s.name;
+  P.table = s.table;
+  P.table_version = ctx->tables[s.table].version;
+  P.opt_version = ctx->opt_version;
+  for (int i = 0; i < d.nht; i++)
+    for (auto& h : ctx->hts)
+      if (h.slots == d.src[i].slots && h.slots) {
+        P.src_ids.push_back(h.id);
+        break;
+      }
+  if ((int)P.src_ids.size() == d.nht) ctx->build_cache[build_segment] = P;
   return GPL_OK;
 }
 
 static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows, PipeDesc* d, LowerInfo* li,
-                              Config* cfg, Segment* seg) {
+                              Config* cfg, Segment* seg, int force_split = -2) {
   std::string err;
   if (!parse_segment(text, seg, &err)) return fail(ctx, GPL_E_PLAN, err);
   if (seg->is_build) return fail(ctx, GPL_E_PLAN, "expected a probe segment ('run TABLE')");
-  gpl_status st = lower_probe(ctx, *seg, choose_split(ctx, *seg), d, li, &err);
+  if (force_split >= 0) seg->split_hint = force_split;
+  gpl_status st = lower_probe(ctx, *seg, force_split >= 0 ? force_split : choose_split(ctx, *seg), d, li, &err);
   if (st) return fail(ctx, st, err);
   auto lit = ctx->lambda.find(seg->text);
   if (lit != ctx->lambda.end()) li->lambda = lit->second;
@@ -445,16 +553,47 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
   return GPL_OK;
 }
 
-static gpl_status ensure_partials(gpl_ctx* ctx, size_t bytes) {
-  if (ctx->partials_cap < bytes) {
-    CK(cudaStreamSynchronize(ctx->stream));
-    if (ctx->d_partials) cudaFree(ctx->d_partials);
-    ctx->d_partials = nullptr;
-    ctx->partials_cap = 0;
-    cudaError_t e = cudaMalloc(&ctx->d_partials, bytes);
-    if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("partials: ") + cudaGetErrorString(e));
-    ctx->partials_cap = bytes;
+// Prepared (parsed, lowered, configured, kernel-resolved) probe segment,
+// cached by text + tile_rows and revalidated against the scanned table's
+// version, the referenced hash tables, the options and the λ profile.
+static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_rows, PreparedRun** out) {
+  const std::string key = std::string(text) + "\x1f" + std::to_string(tile_rows);
+  auto lam = ctx->lambda.find(text);
+  const size_t lambda_n = lam == ctx->lambda.end() ? 0 : lam->second.size();
+  auto it = ctx->run_cache.find(key);
+  if (it != ctx->run_cache.end()) {
+    PreparedRun& P = it->second;
+    if (run_cache_valid(ctx, P)) {
+      *out = &P;
+      return GPL_OK;
+    }
+    ctx->run_cache.erase(it);
   }
+  PipeDesc d;
+  LowerInfo li;
+  Config cfg;
+  Segment seg;
+  gpl_status st;
+  if ((st = prepare_run(ctx, text, tile_rows, &d, &li, &cfg, &seg))) return st;
+  PreparedRun P;
+  li.table = seg.table;
+  d.partials = partials_ptr(ctx);
+  d.tile_counter = counter_ptr(ctx);
+  d.op_pass = op_pass_ptr(ctx);
+  d.err = err_ptr(ctx);
+  P.desc = d;
+  P.li = li;
+  P.grid = cfg.grid;
+  P.pred_ms = cfg.pred_ms;
+  P.text = seg.text;
+  P.table_version = ctx->tables[seg.table].version;
+  P.opt_version = ctx->opt_version;
+  P.lambda_n = lambda_n;
+  std::string jerr;
+  P.fn = resolve_pipeline_fn(d, ctx->opt.jit != 0, &jerr);
+  P.jit = ctx->opt.jit != 0 && jerr.empty();
+  if (!P.fn) return fail(ctx, GPL_E_CUDA, "cannot configure the pipeline kernel");
+  *out = &(ctx->run_cache[key] = P);
   return GPL_OK;
 }
 
@@ -463,27 +602,21 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
-  PipeDesc d;
-  LowerInfo li;
-  Config cfg;
-  Segment seg;
-  if ((st = prepare_run(ctx, probe_segment, tile_rows, &d, &li, &cfg, &seg))) return st;
+  if (tile_rows < 0) return fail(ctx, GPL_E_ARG, "tile_rows must be >= 0");
+  PreparedRun* P = nullptr;
+  if ((st = get_prepared_run(ctx, probe_segment, tile_rows, &P))) return st;
+  const PipeDesc& d = P->desc;
+  const LowerInfo& li = P->li;
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
-  if ((st = ensure_partials(ctx, pbytes))) return st;
-  d.partials = ctx->d_partials;
-  d.tile_counter = ctx->d_scratch;
-  d.op_pass = op_pass_ptr(ctx);
-  d.err = err_ptr(ctx);
-  CK(cudaMemsetAsync(ctx->d_partials, 0, pbytes, ctx->stream));
-  CK(cudaMemsetAsync(ctx->d_scratch, 0, (1 + MAXOPS) * sizeof(unsigned long long), ctx->stream));
-  std::string jerr;
-  CK(cudaEventRecord(ctx->ev0, ctx->stream));
-  CK(launch_pipeline(d, cfg.grid, ctx->stream, ctx->opt.jit != 0, &jerr));
-  CK(cudaEventRecord(ctx->ev1, ctx->stream));
+  // one memset: tile counter, op_pass and the partials are contiguous
+  CK(cudaMemsetAsync(counter_ptr(ctx), 0, (1 + MAXOPS) * sizeof(unsigned long long) + pbytes, ctx->stream));
+  CK(record_event(ctx, ctx->ev0));
+  CK(launch_pipeline_fn(P->fn, d, P->grid, ctx->stream));
+  CK(record_event(ctx, ctx->ev1));
   LastRun& L = ctx->last;
   L.valid = true;
   L.kbe = false;
-  L.text = seg.text;
+  L.text = P->text;
   L.desc = d;
   L.li = li;
   L.timed = true;
@@ -494,13 +627,115 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   S.stage_rows = d.stage_rows;
   S.ring_depth = d.depth;
   S.consumer_warps = d.nwarps;
-  S.grid = cfg.grid;
+  S.grid = P->grid;
   S.n_ops = li.nops;
   S.probe_split = d.nsprobe;
-  S.predicted_ms = cfg.pred_ms;
+  S.predicted_ms = P->pred_ms;
   S.bytes_scanned = (double)d.nrows * li.bytes_per_row;
   S.agg_mode = d.agg_mode;
-  S.jit = (ctx->opt.jit != 0 && jerr.empty()) ? 1 : 0;
+  S.jit = P->jit ? 1 : 0;
+  return GPL_OK;
+}
+
+// Split a whole plan into its segments at 'build NAME' / 'run TABLE' lines.
+static std::vector<std::string> split_segments(const std::string& plan) {
+  std::vector<std::string> segs;
+  std::string cur;
+  bool cur_has_head = false;
+  size_t i = 0;
+  while (i <= plan.size()) {
+    size_t j = plan.find('\n', i);
+    if (j == std::string::npos) j = plan.size();
+    const std::string line = plan.substr(i, j - i);
+    size_t k = line.find_first_not_of(" \t\r");
+    const std::string head = k == std::string::npos ? "" : line.substr(k, line.find_first_of(" \t\r#", k) - k);
+    if ((head == "build" || head == "run") && cur_has_head) {
+      segs.push_back(cur);
+      cur.clear();
+    }
+    if (head == "build" || head == "run") cur_has_head = true;
+    cur += line + "\n";
+    i = j + 1;
+  }
+  if (cur_has_head) segs.push_back(cur);
+  return segs;
+}
+
+GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_rows) {
+  if (!ctx || !plan) return GPL_E_ARG;
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  const std::vector<std::string> segs = split_segments(plan);
+  if (segs.empty()) return fail(ctx, GPL_E_PLAN, "plan has no segment");
+  const std::string key = std::string(plan) + "\x1f" + std::to_string(tile_rows);
+  const std::string run_key = segs.back() + "\x1f" + std::to_string(tile_rows);
+  // are all segments prepared and still valid?
+  auto all_valid = [&]() {
+    for (size_t i = 0; i + 1 < segs.size(); i++) {
+      auto b = ctx->build_cache.find(segs[i]);
+      if (b == ctx->build_cache.end() || !build_cache_valid(ctx, b->second)) return false;
+    }
+    auto r = ctx->run_cache.find(run_key);
+    return r != ctx->run_cache.end() && run_cache_valid(ctx, r->second) && ctx->lambda.count(r->second.text);
+  };
+  auto eager = [&]() -> gpl_status {
+    for (size_t i = 0; i + 1 < segs.size(); i++) {
+      gpl_status s2 = gpl_build_hash(ctx, segs[i].c_str(), nullptr);
+      if (s2) return s2;
+    }
+    return gpl_run_plan(ctx, segs.back().c_str(), tile_rows);
+  };
+  auto g = ctx->graphs.find(key);
+  if (g != ctx->graphs.end()) {
+    if (all_valid()) {
+      CK(cudaGraphLaunch(g->second, ctx->stream));
+      // the run's bookkeeping is the cached plan's
+      const PreparedRun& P = ctx->run_cache[run_key];
+      LastRun& L = ctx->last;
+      L.valid = true;
+      L.kbe = false;
+      L.text = P.text;
+      L.desc = P.desc;
+      L.li = P.li;
+      L.timed = true;
+      gpl_stats& S = L.stats;
+      S = gpl_stats{};
+      S.rows_scanned = P.desc.nrows;
+      S.tile_rows_used = P.desc.tile_rows;
+      S.stage_rows = P.desc.stage_rows;
+      S.ring_depth = P.desc.depth;
+      S.consumer_warps = P.desc.nwarps;
+      S.grid = P.grid;
+      S.n_ops = P.li.nops;
+      S.probe_split = P.desc.nsprobe;
+      S.predicted_ms = P.pred_ms;
+      S.bytes_scanned = (double)P.desc.nrows * P.li.bytes_per_row;
+      S.agg_mode = P.desc.agg_mode;
+      S.jit = P.jit ? 1 : 0;
+      return GPL_OK;
+    }
+    cudaGraphExecDestroy(g->second);
+    ctx->graphs.erase(g);
+  }
+  // run eagerly (refreshes the prepared caches); once everything is prepared
+  // and profiled, record the same sequence as a graph for the next call
+  if ((st = eager())) return st;
+  if (all_valid()) {
+    const LastRun saved = ctx->last;
+    cudaGraph_t graph = nullptr;
+    bool ok = cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+    gpl_status cst = ok ? eager() : GPL_E_CUDA;
+    cudaError_t ce = cudaStreamEndCapture(ctx->stream, &graph);
+    ctx->last = saved;
+    cudaGraphExec_t exec = nullptr;
+    if (ok && cst == GPL_OK && ce == cudaSuccess && graph &&
+        cudaGraphInstantiate(&exec, graph, 0) == cudaSuccess)
+      ctx->graphs[key] = exec;
+    if (graph) cudaGraphDestroy(graph);
+    cudaGetLastError();  // a failed capture only means no graph; the eager run above stands
+    ctx->err.clear();
+  }
   return GPL_OK;
 }
 
@@ -528,18 +763,27 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   LowerInfo li;
   Config cfg;
   Segment seg;
-  if ((st = prepare_run(ctx, probe_segment, 0, &d, &li, &cfg, &seg))) return st;
+  // every probe reads its keys from materialised columns: lower with no stage-phase probe
+  if ((st = prepare_run(ctx, probe_segment, 0, &d, &li, &cfg, &seg, 0))) return st;
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
-  if ((st = ensure_partials(ctx, pbytes))) return st;
-  d.partials = ctx->d_partials;
-  d.tile_counter = ctx->d_scratch;
+  d.partials = partials_ptr(ctx);
+  d.tile_counter = counter_ptr(ctx);
   d.op_pass = op_pass_ptr(ctx);
   d.err = err_ptr(ctx);
-  CK(cudaMemsetAsync(ctx->d_partials, 0, pbytes, ctx->stream));
-  CK(cudaMemsetAsync(ctx->d_scratch, 0, (1 + MAXOPS) * sizeof(unsigned long long), ctx->stream));
+  CK(cudaMemsetAsync(counter_ptr(ctx), 0, (1 + MAXOPS) * sizeof(unsigned long long) + pbytes, ctx->stream));
   double inter = 0;
+  const size_t need = kbe_pool_bytes(d);
+  if (ctx->kbe_cap < need) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
+    ctx->kbe_buf = nullptr;
+    ctx->kbe_cap = 0;
+    cudaError_t e = cudaMalloc(&ctx->kbe_buf, need);
+    if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("KBE buffers: ") + cudaGetErrorString(e));
+    ctx->kbe_cap = need;
+  }
   CK(cudaEventRecord(ctx->ev0, ctx->stream));
-  CK(run_kbe(d, ctx->sms, ctx->stream, &inter));
+  CK(run_kbe(d, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &inter));
   CK(cudaEventRecord(ctx->ev1, ctx->stream));
   LastRun& L = ctx->last;
   L.valid = true;
@@ -575,11 +819,14 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   if (st) return st;
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run to fetch");
   const LowerInfo& li = ctx->last.li;
-  std::vector<unsigned long long> part((size_t)li.ngroups_total * li.nagg * 2);
-  unsigned long long ops[MAXOPS];
-  CK(cudaMemcpyAsync(part.data(), ctx->d_partials, part.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  CK(cudaMemcpyAsync(ops, op_pass_ptr(ctx), sizeof(ops), cudaMemcpyDeviceToHost, ctx->stream));
+  // one D2H: error bits, counter, op_pass and partials are contiguous
+  const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
+  CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
+  const unsigned long long* hs = (const unsigned long long*)ctx->h_stage;
+  const unsigned int bits = (unsigned int)hs[0];
+  const unsigned long long* ops = hs + 2;
+  const unsigned long long* part = hs + kScratchHead;
   gpl_stats& S = ctx->last.stats;
   if (ctx->last.timed) {
     float ms = 0;
@@ -587,17 +834,17 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   }
   for (int i = 0; i < MAXOPS && i < 16; i++) S.op_pass[i] = (int64_t)ops[i];
   // λ cache for the model / split choice (cumulative pass fraction after each op)
-  if (!ctx->last.kbe && S.rows_scanned > 0) {
+  // (recorded once per plan text: the first run profiles the plan)
+  if (!ctx->last.kbe && S.rows_scanned > 0 && !ctx->lambda.count(ctx->last.text)) {
     std::vector<double> lam;
     for (int i = 0; i < li.nops; i++) lam.push_back((double)ops[i] / (double)S.rows_scanned);
     ctx->lambda[ctx->last.text] = lam;
   }
-  if ((st = take_device_errors(ctx))) {
-    out->stats = S;
-    return st;
-  }
   out->stats = S;
-  return decode(ctx, part.data(), out);
+  if (bits) {
+    if ((st = take_device_errors(ctx))) return st;
+  }
+  return decode(ctx, part, out);
 }
 
 GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_device, size_t cap_bytes, size_t* nbytes) {
@@ -608,7 +855,7 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
   const size_t b = (size_t)ctx->last.li.ngroups_total * ctx->last.li.nagg * 16;
   *nbytes = b;
   if (cap_bytes < b || !dst) return fail(ctx, GPL_E_CAPACITY, "partials buffer too small");
-  CK(cudaMemcpyAsync(dst, ctx->d_partials, b, dst_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+  CK(cudaMemcpyAsync(dst, partials_ptr(ctx), b, dst_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
                      ctx->stream));
   if (!dst_on_device) CK(cudaStreamSynchronize(ctx->stream));
   return GPL_OK;

@@ -68,6 +68,8 @@ struct LowerInfo {
   std::vector<std::string> op_names;
   std::vector<int64_t> ht_bytes;  // slot bytes of each probed table
   std::vector<int> probe_ht;      // probe index -> d.ht index
+  std::vector<int> ht_ids;        // d.ht index -> ctx hash-table id
+  std::string table;              // scanned (fact) table
   int nprobe = 0, nfilt = 0;
   bool has_groups = false;
   std::vector<double> lambda;     // cumulative pass fraction after each op (previous run)
@@ -81,6 +83,30 @@ struct LastRun {
   gpl_stats stats{};
   bool timed = false;
   bool kbe = false;
+};
+
+struct PreparedRun {
+  PipeDesc desc{};
+  LowerInfo li;
+  int grid = 0;
+  double pred_ms = 0;
+  const void* fn = nullptr;  // kernel to launch (JIT or generic)
+  bool jit = false;
+  uint64_t table_version = 0, opt_version = 0;
+  size_t lambda_n = 0;
+  std::string text;
+};
+
+struct PreparedBuild {
+  BuildDesc desc{};
+  HashTable shape;
+  bool trivial = false;
+  HTHeader known{};
+  int ht_index = -1;
+  HTRef dest_ref{};
+  std::string name, table;
+  uint64_t table_version = 0, opt_version = 0;
+  std::vector<int> src_ids;
 };
 
 struct Options {
@@ -113,7 +139,16 @@ struct gpl_ctx {
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   gpl::LastRun last;
   gpl::Options opt;
+  uint64_t opt_version = 1;  // bumped by gpl_set_option (invalidates prepared plans)
   std::map<std::string, std::vector<double>> lambda;  // plan text -> per-op pass fraction (A9 "profile the first tile")
+  // prepared-plan caches (keyed by segment text [+ tile_rows]); validated on
+  // every use against table versions, hash-table refs and options
+  std::map<std::string, gpl::PreparedRun> run_cache;
+  std::map<std::string, gpl::PreparedBuild> build_cache;
+  // gpl_run_query: whole-query CUDA graphs (builds + fused run), keyed by plan text + tile_rows
+  std::map<std::string, cudaGraphExec_t> graphs;
+  void* h_stage = nullptr;  // pinned host staging for one packed D2H of results
+  size_t h_stage_cap = 0;
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;
   size_t kbe_cap = 0;

@@ -28,6 +28,10 @@ cudaError_t launch_header_init(HTHeader* hdr, cudaStream_t s);
 // is unavailable (reason in *jit_err).
 cudaError_t launch_pipeline(const PipeDesc& d, int grid, cudaStream_t s, bool use_jit, std::string* jit_err);
 
+// Resolve once (JIT or generic, dynamic-smem attribute set), then launch many times.
+const void* resolve_pipeline_fn(const PipeDesc& d, bool use_jit, std::string* jit_err);
+cudaError_t launch_pipeline_fn(const void* fn, const PipeDesc& d, int grid, cudaStream_t s);
+
 // JIT: compile (and, when load is true, load) the specialised kernel for d's
 // shape. Returns false with a message when NVRTC is unavailable or fails.
 bool jit_prepare(const PipeDesc& d, bool load, std::string* err);
@@ -37,7 +41,8 @@ cudaError_t launch_minmax(const void* col, int width, long long n, long long* ou
 
 // KBE baseline: kernel-at-a-time with materialisation. Returns the
 // bytes of intermediates written to HBM in *inter_bytes (host-side count).
-struct KbeBuffers;
-cudaError_t run_kbe(const PipeDesc& d, int num_sms, cudaStream_t s, double* inter_bytes);
+// `pool` must hold kbe_pool_bytes(d) bytes (per-context, reused).
+size_t kbe_pool_bytes(const PipeDesc& d);
+cudaError_t run_kbe(const PipeDesc& d, int num_sms, cudaStream_t s, void* pool, size_t pool_bytes, double* inter_bytes);
 
 }  // namespace gpl

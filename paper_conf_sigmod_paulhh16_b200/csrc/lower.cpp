@@ -234,6 +234,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
       ht_slot[H.id] = i;
       d->ht[i] = H.ref();
       li->ht_bytes.push_back((int64_t)(H.kind == HT_DIRECT ? H.bytes() : H.bytes() / 2));
+      li->ht_ids.push_back(H.id);
     }
     li->probe_ht.push_back(ht_slot[H.id]);
   }

@@ -28,7 +28,7 @@ GPL_COPY, GPL_BORROW = 0, 1
 EXPORTED = ["gpl_create", "gpl_destroy", "gpl_load_columns", "gpl_build_hash", "gpl_run_plan",
             "gpl_run_plan_kbe", "gpl_fetch_result", "gpl_fetch_partials", "gpl_decode_partials",
             "gpl_merge_partials", "gpl_sync", "gpl_choose_tile_rows", "gpl_set_option",
-            "gpl_check_plan", "gpl_compile_plan", "gpl_last_error", "gpl_version"]
+            "gpl_check_plan", "gpl_compile_plan", "gpl_run_query", "gpl_last_error", "gpl_version"]
 
 
 class GplError(RuntimeError):
@@ -97,6 +97,7 @@ def load_library():
         "gpl_set_option": ([P, ctypes.c_char_p, I64], I32),
         "gpl_check_plan": ([P, ctypes.c_char_p], I32),
         "gpl_compile_plan": ([P, ctypes.c_char_p, I64], I32),
+        "gpl_run_query": ([P, ctypes.c_char_p, I64], I32),
         "gpl_last_error": ([P], ctypes.c_char_p),
         "gpl_version": ([], ctypes.c_char_p),
     }
@@ -154,6 +155,9 @@ class Context:
         self._h = ctypes.c_void_p()
         if stream is not None and not isinstance(stream, int):
             stream = stream.cuda_stream
+            if stream == 0:
+                raise ValueError("pass a non-default CUDA stream (torch.cuda.Stream()): the legacy default "
+                                 "stream would make libgpl create its own unsynchronised stream")
         st = self._lib.gpl_create(device, ctypes.c_void_p(stream or 0), ctypes.byref(self._h))
         if st:
             raise GplError(st, self._lib.gpl_last_error(None).decode())
@@ -223,6 +227,10 @@ class Context:
 
     def run_plan(self, segment: str, tile_rows: int = 0):
         self._check(self._lib.gpl_run_plan(self._h, segment.encode(), int(tile_rows)))
+
+    def run_query(self, plan: str, tile_rows: int = 0):
+        """All segments of a plan (builds then the probe segment); replays a CUDA graph once warm."""
+        self._check(self._lib.gpl_run_query(self._h, plan.encode(), int(tile_rows)))
 
     def run_plan_kbe(self, segment: str):
         self._check(self._lib.gpl_run_plan_kbe(self._h, segment.encode()))

@@ -158,7 +158,11 @@ def decode_keys(query: str, result: Result, catalog) -> Result:
 
 
 def run_query(ctx: Context, query: str, catalog, params=None, tile_rows: int = 0, kbe: bool = False) -> Result:
-    run_segments(ctx, plan_text(query, catalog, params), tile_rows, kbe)
+    text = plan_text(query, catalog, params)
+    if kbe:
+        run_segments(ctx, text, tile_rows, kbe=True)
+    else:
+        ctx.run_query(text, tile_rows)  # graph-replayed once the plan is warm
     return decode_keys(query, ctx.fetch_result(), catalog)
 
 

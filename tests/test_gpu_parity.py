@@ -172,3 +172,34 @@ def test_int128_totals(ctx):
     expect = n * 10_499_990_000 * 100 * 108
     assert expect > 2**63
     assert r.aggs == [[n, expect]]
+
+
+@pytest.mark.parametrize("q", QUERIES)
+def test_kbe_baseline_bit_identical(ctx, q):
+    """The KBE baseline (map -> prefix sum -> scatter per operator) computes the
+    same exact result and materialises intermediates the fused path does not."""
+    db = tpchgen.generate(0.05, seed=21)
+    queries.load_database(ctx, db, queries.TABLES[q])
+    r = queries.run_query(ctx, q, db, _params(q), kbe=True)
+    o = oracle.run(q, db, _params(q))
+    assert r.keys == o.keys and r.aggs == o.aggs
+    assert r.stats["kbe"] == 1 and r.stats["intermediate_bytes"] > 0
+    f = queries.run_query(ctx, q, db, _params(q))
+    assert f.stats["intermediate_bytes"] == 0 and f.aggs == r.aggs
+
+
+def test_query_graph_replay_and_invalidation(ctx):
+    """gpl_run_query records builds + fused kernel as a CUDA graph once warm;
+    replays must stay exact, and reloading a table must re-plan, not replay."""
+    db = tpchgen.generate(0.05, seed=31)
+    o = oracle.run("Q5", db)
+    queries.load_database(ctx, db, queries.TABLES["Q5"])
+    for _ in range(4):
+        r = queries.run_query(ctx, "Q5", db)
+        assert r.keys == o.keys and r.aggs == o.aggs
+    db2 = tpchgen.generate(0.05, seed=32)
+    queries.load_database(ctx, db2, queries.TABLES["Q5"])
+    o2 = oracle.run("Q5", db2)
+    for _ in range(3):
+        r = queries.run_query(ctx, "Q5", db2)
+        assert r.keys == o2.keys and r.aggs == o2.aggs
