@@ -23,41 +23,69 @@ namespace {
 
 constexpr int kThreads = 256;
 
-__device__ __forceinline__ long long sel_slot(const long long (&s)[MAXP], int i) {
-  long long v = s[0];
+// Evaluate BR build rows at once (rows row0 + j*stride): filters, probes into
+// earlier tables (a miss drops the row: inner / semi join), key and payload.
+// Every
+// column load and hash probe of the BR rows is issued before any is needed,
+// so one thread keeps BR independent memory round trips in flight.
+#ifndef GPL_BUILD_BR
+#define GPL_BUILD_BR 1
+#endif
+constexpr int BR = GPL_BUILD_BR;
+__device__ __forceinline__ void build_rows(const BuildDesc& d, const HTP* src, long long row0, long long stride,
+                                           bool (&ok)[BR], unsigned long long (&key)[BR], long long (&pay)[BR]) {
 #pragma unroll
-  for (int k = 1; k < MAXP; k++) v = (i == k) ? s[k] : v;
-  return v;
-}
-
-// Evaluate one build row: filters, probes into earlier tables, key and payload.
-__device__ __forceinline__ bool build_row(const BuildDesc& d, const HTP* src, long long row,
-                                          unsigned long long* key, long long* payload) {
+  for (int j = 0; j < BR; j++) ok[j] = row0 + j * stride < d.nrows;
   for (int f = 0; f < d.nfilt; f++) {
     const Filt& F = d.filt[f];
-    if (!filt_pass(F, ld_col_global(d.col[F.ref], d.colw[F.ref], row))) return false;
+    long long x[BR];
+#pragma unroll
+    for (int j = 0; j < BR; j++) x[j] = ok[j] ? ld_col_global(d.col[F.ref], d.colw[F.ref], row0 + j * stride) : 0;
+#pragma unroll
+    for (int j = 0; j < BR; j++) ok[j] = ok[j] && filt_pass(F, x[j]);
   }
-  long long slot[MAXP] = {0, 0, 0, 0};
+  long long slot[MAXP][BR];
 #pragma unroll
   for (int p = 0; p < MAXP; p++) {
+#pragma unroll
+    for (int j = 0; j < BR; j++) slot[p][j] = 0;
     if (p < d.nprobe) {
       const Probe& P = d.probe[p];
-      unsigned long long k = (uint32_t)ld_col_global(d.col[P.k1], d.colw[P.k1], row);
-      if (P.k2 >= 0) k = (k << 32) | (uint32_t)ld_col_global(d.col[P.k2], d.colw[P.k2], row);
-      long long v = 0;
-      if (!ht_probe(src[P.ht], k, &v)) return false;  // inner / semi: a miss drops the row
-      slot[p] = v;
+      unsigned long long k[BR];
+#pragma unroll
+      for (int j = 0; j < BR; j++) {
+        k[j] = ok[j] ? (uint32_t)ld_col_global(d.col[P.k1], d.colw[P.k1], row0 + j * stride) : 0u;
+        if (P.k2 >= 0 && ok[j]) k[j] = (k[j] << 32) | (uint32_t)ld_col_global(d.col[P.k2], d.colw[P.k2], row0 + j * stride);
+      }
+      bool hit[BR];
+      long long v[BR];
+      const HTP& H = src[P.ht];
+      ht_probe_n<BR>(H, H.kind, H.width, k, ok, hit, v);
+#pragma unroll
+      for (int j = 0; j < BR; j++) {
+        ok[j] = ok[j] && hit[j];  // inner / semi: a miss drops the row
+        slot[p][j] = v[j];
+      }
     }
   }
-  unsigned long long k = (uint32_t)ld_col_global(d.col[d.k1], d.colw[d.k1], row);
-  if (d.k2 >= 0) k = (k << 32) | (uint32_t)ld_col_global(d.col[d.k2], d.colw[d.k2], row);
-  *key = k;
-  long long pay = 0;
-  if (d.pay_kind == PAY_COL) pay = ld_col_global(d.col[d.pay_ref], d.colw[d.pay_ref], row);
-  else if (d.pay_kind == PAY_SLOT) pay = sel_slot(slot, d.pay_ref);
-  else if (d.pay_kind == PAY_YEARCOL) pay = (int)ld_col_global(d.col[d.pay_ref], d.colw[d.pay_ref], row) / 10000;
-  *payload = pay;
-  return true;
+#pragma unroll
+  for (int j = 0; j < BR; j++) {
+    const long long row = row0 + j * stride;
+    key[j] = 0;
+    pay[j] = 0;
+    if (!ok[j]) continue;
+    unsigned long long k = (uint32_t)ld_col_global(d.col[d.k1], d.colw[d.k1], row);
+    if (d.k2 >= 0) k = (k << 32) | (uint32_t)ld_col_global(d.col[d.k2], d.colw[d.k2], row);
+    key[j] = k;
+    if (d.pay_kind == PAY_COL) pay[j] = ld_col_global(d.col[d.pay_ref], d.colw[d.pay_ref], row);
+    else if (d.pay_kind == PAY_YEARCOL) pay[j] = (int)ld_col_global(d.col[d.pay_ref], d.colw[d.pay_ref], row) / 10000;
+    else if (d.pay_kind == PAY_SLOT) {
+      long long s = slot[0][j];
+#pragma unroll
+      for (int p = 1; p < MAXP; p++) s = d.pay_ref == p ? slot[p][j] : s;
+      pay[j] = s;
+    }
+  }
 }
 
 __device__ __forceinline__ void finalize_header(HTHeader* h, unsigned long long count, long long kmin,
@@ -99,14 +127,18 @@ __global__ void __launch_bounds__(kThreads) build_count_kernel(const __grid_cons
   unsigned long long cnt = 0;
   long long mn = LLONG_MAX, mx = LLONG_MIN;
   const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long row = (long long)blockIdx.x * blockDim.x + threadIdx.x; row < d.nrows; row += stride) {
-    unsigned long long k;
-    long long pay;
-    if (build_row(d, src, row, &k, &pay)) {
-      cnt++;
-      mn = min(mn, (long long)k);
-      mx = max(mx, (long long)k);
-    }
+  for (long long row = (long long)blockIdx.x * blockDim.x + threadIdx.x; row < d.nrows; row += stride * BR) {
+    bool ok[BR];
+    unsigned long long k[BR];
+    long long pay[BR];
+    build_rows(d, src, row, stride, ok, k, pay);
+#pragma unroll
+    for (int j = 0; j < BR; j++)
+      if (ok[j]) {
+        cnt++;
+        mn = min(mn, (long long)k[j]);
+        mx = max(mx, (long long)k[j]);
+      }
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
@@ -184,18 +216,26 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
   }
   __syncthreads();
   const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long row = (long long)blockIdx.x * blockDim.x + threadIdx.x; row < d.nrows; row += stride) {
-    unsigned long long key;
-    long long pay;
-    if (!build_row(d, src, row, &key, &pay)) continue;
-    if (d.kind == HT_DIRECT) {
-      const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key - d.kmin);
+  for (long long row0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; row0 < d.nrows; row0 += stride * BR) {
+   bool okv[BR];
+   unsigned long long keyv[BR];
+   long long payv[BR];
+   build_rows(d, src, row0, stride, okv, keyv, payv);
+   if (d.kind == HT_DIRECT) {
+    // one atomic per row, all BR in flight: bitmap / 32-bit cells by
+    // atomicOr / atomicCAS; 1- and 2-byte cells by atomicOr into their word
+    // (cells start at 0 = empty, so OR sets exactly the cell; a non-zero old
+    // cell means a duplicate key)
+#pragma unroll
+    for (int j = 0; j < BR; j++) {
+      if (!okv[j]) continue;
+      const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)keyv[j] - d.kmin);
       if (idx >= d.nslots) { atomicOr(d.err, ERR_CAPACITY); continue; }
       if (d.width == 0) {
         const uint32_t bit = 1u << (idx & 31);
         if (atomicOr((uint32_t*)d.slots + (idx >> 5), bit) & bit) atomicOr(d.err, ERR_DUPKEY);
       } else {
-        const uint32_t v = (uint32_t)(pay - d.pay_base + 1);
+        const uint32_t v = (uint32_t)(payv[j] - d.pay_base + 1);
         if (d.width == 4) {
           if (atomicCAS((uint32_t*)d.slots + idx, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
         } else {
@@ -203,17 +243,16 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
           uint32_t* w = (uint32_t*)((char*)d.slots + (byte & ~3ull));
           const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
           const uint32_t m = (d.width == 1 ? 0xFFu : 0xFFFFu) << sh;
-          uint32_t old = *((volatile uint32_t*)w);
-          for (;;) {
-            if (old & m) { atomicOr(d.err, ERR_DUPKEY); break; }
-            const uint32_t got = atomicCAS(w, old, old | (v << sh));
-            if (got == old) break;
-            old = got;
-          }
+          if (atomicOr(w, v << sh) & m) atomicOr(d.err, ERR_DUPKEY);
         }
       }
-      continue;
     }
+    continue;
+   }
+   for (int j = 0; j < BR; j++) {
+    if (!okv[j]) continue;
+    const unsigned long long key = keyv[j];
+    const long long pay = payv[j];
     uint32_t i = ht_home(dst, key);
     if (d.kind == HT_MAP32) {
       if ((uint32_t)key == EMPTY32) { atomicOr(d.err, ERR_RESERVED_KEY); continue; }
@@ -244,6 +283,7 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
         i = (i + 1) & dst.mask;
       }
     }
+   }
   }
 }
 
