@@ -176,10 +176,19 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     args.gpus = world if world > 1 else args.gpus
+    ndev = torch.cuda.device_count()
+    local = local % ndev
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    # NCCL over NVLink/NVSwitch when every rank has its own GPU; gloo (CPU
+    # tensors) only to exercise the multi-rank path on a box with fewer GPUs
+    backend = "nccl" if world <= ndev else "gloo"
+    cdev = dev if backend == "nccl" else torch.device("cpu")
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     torch.cuda.set_stream(torch.cuda.Stream(device=dev))  # a real stream shared with libgpl
     stream = torch.cuda.current_stream()
 
@@ -221,9 +230,12 @@ def main():
             nonlocal part_dev, gathered
             nb = ctx.partials_nbytes()
             if part_dev is None:
-                part_dev = torch.empty(nb // 8, dtype=torch.int64, device=dev)
-                gathered = torch.empty(world * nb // 8, dtype=torch.int64, device=dev)
-            ctx.fetch_partials(out=part_dev)
+                part_dev = torch.empty(nb // 8, dtype=torch.int64, device=cdev)
+                gathered = torch.empty(world * nb // 8, dtype=torch.int64, device=cdev)
+            if backend == "nccl":
+                ctx.fetch_partials(out=part_dev)  # device-to-device copy on the ctx stream
+            else:
+                part_dev.copy_(torch.from_numpy(ctx.fetch_partials().view(np.int64)))
             dist.all_gather_into_tensor(gathered, part_dev)
             host = gathered.cpu().numpy()
             res = ctx.decode_partials(gpl.merge_partials(host, world))
@@ -258,10 +270,10 @@ def main():
     kernel_avg = statistics.mean(kern_ms)
     stats = res0.stats
     if world > 1:
-        t = torch.tensor([total_ms, kernel_avg], dtype=torch.float64, device=dev)
+        t = torch.tensor([total_ms, kernel_avg], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms, kernel_avg = float(t[0]), float(t[1])
-        rows_all = torch.tensor([n_local], dtype=torch.int64, device=dev)
+        rows_all = torch.tensor([n_local], dtype=torch.int64, device=cdev)
         dist.all_reduce(rows_all)
         rows_total = int(rows_all[0])
     else:
@@ -279,7 +291,12 @@ def main():
         def e2e_step():
             queries.load_database(ctx2, type("H", (), {"tables": pinned})(), borrow=False)
             ctx2.run_query(text, args.tile_rows)
-            return ctx2.fetch_result()
+            if world == 1:
+                return ctx2.fetch_result()
+            host = ctx2.fetch_partials()  # D2H of this rank's int128 partials
+            g = torch.empty(world * host.size, dtype=torch.int64, device=cdev)
+            dist.all_gather_into_tensor(g, torch.from_numpy(host.view(np.int64)).to(cdev))
+            return ctx2.decode_partials(gpl.merge_partials(g.cpu().numpy(), world))
         for _ in range(2):
             e2e_step()
         e_ms = []
@@ -292,10 +309,10 @@ def main():
             e_ms.append(ev0.elapsed_time(ev1))
         assert r2.aggs == res0.aggs and r2.keys == res0.keys
         ncols = sum(len(c) for c in pinned.values())
-        d2h = len(res0.aggs) * 0 + ctx2.partials_nbytes() + 16 * 8 + 4 + 16 * ncols
+        d2h = ctx2.partials_nbytes() + 16 * 8 + 4 + 16 * ncols  # partials + counters + errors + column min/max
         e_ms_v = statistics.mean(e_ms)
         if world > 1:
-            t = torch.tensor([e_ms_v], dtype=torch.float64, device=dev)
+            t = torch.tensor([e_ms_v], dtype=torch.float64, device=cdev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_ms_v = float(t[0])
         e2e = {"value": rows_total / (e_ms_v / 1e3), "unit": UNIT, "ms_per_step": e_ms_v,
@@ -343,6 +360,8 @@ def main():
         "pipeline": {k: stats[k] for k in ("tile_rows_used", "stage_rows", "ring_depth", "consumer_warps", "grid",
                                            "probe_split", "predicted_ms", "agg_mode")},
         "op_pass": stats["op_pass"],
+        "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
+        "jit": stats.get("jit"),
     }
     if rank == 0:
         print(json.dumps(line), flush=True)
