@@ -159,6 +159,7 @@ def main():
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-autotune", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -244,6 +245,11 @@ def main():
             res = ctx.fetch_result()
         return res
 
+    # calibrate the pipeline shape on the device (model shortlist, measured; untimed)
+    tuned = None
+    if not args.no_autotune and args.tile_rows == 0:
+        tuned = ctx.autotune(text)
+        log(f"[rank {rank}] autotune: {tuned}")
     for _ in range(args.warmup):
         res = step()
     res0 = ctx.fetch_result() if world == 1 else res
@@ -362,6 +368,8 @@ def main():
         "op_pass": stats["op_pass"],
         "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
         "jit": stats.get("jit"),
+        "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm")}
+                     if tuned else None),
     }
     if rank == 0:
         print(json.dumps(line), flush=True)

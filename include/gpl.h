@@ -112,6 +112,9 @@ typedef struct {
   double bw_gbs;               /* effective HBM bandwidth the model used                           */
   int32_t smem_bytes;
   int32_t feasible;
+  int32_t ctas_per_sm;
+  int32_t candidates;          /* gpl_autotune: shapes measured                                    */
+  double measured_ms;          /* gpl_autotune: median kernel time of the chosen shape            */
 } gpl_model_report;
 
 /* Create a context on CUDA device `device` enqueuing on `cuda_stream` (a
@@ -210,6 +213,16 @@ gpl_status gpl_sync(gpl_ctx* ctx);
  * Fills the chosen configuration and its predicted time. */
 gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t n_rows,
                                 gpl_model_report* out);
+
+/* Calibrate the pipeline shape of a query by measurement (the paper profiles
+ * the first tile and then searches its model): runs the plan's
+ * build segments, takes the A9 model's best configuration for every
+ * (CTAs per SM, stage rows) shape (at most max_candidates), times each on the
+ * device with L2 flushed (median of 3), and pins the fastest for this probe
+ * segment; later gpl_run_plan / gpl_run_query calls with tile_rows = 0 use
+ * it until gpl_set_option is called. Synchronises. out (optional) receives
+ * the chosen shape, its model estimate and its measured time. */
+gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_candidates, gpl_model_report* out);
 
 /* Tuning knobs (tests / sweeps): "stage_rows", "ring_depth",
  * "consumer_warps", "ctas_per_sm", "probe_split" (-1 = auto), "hash_load_pct",

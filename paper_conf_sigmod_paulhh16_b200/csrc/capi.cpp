@@ -217,6 +217,7 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
     return fail(ctx, GPL_E_ARG, "unknown option '" + k + "'");
   }
   ctx->opt_version++;
+  ctx->tuned.clear();
   return GPL_OK;
 }
 
@@ -548,7 +549,14 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
         li->ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
   }
   if (tile_rows < 0) return fail(ctx, GPL_E_ARG, "tile_rows must be >= 0");
-  if (!choose_config(ctx, *d, *li, d->nrows, tile_rows, cfg, &err)) return fail(ctx, GPL_E_ARG, err);
+  auto tu = tile_rows == 0 ? ctx->tuned.find(seg->text) : ctx->tuned.end();
+  if (tu != ctx->tuned.end()) {  // shape pinned by gpl_autotune
+    const TunedShape& t = tu->second;
+    *cfg = predict(ctx, *d, *li, std::max<int64_t>(d->nrows, 1), t.tile_rows, t.stage_rows, t.depth, t.warps,
+                   t.ctas_per_sm);
+  } else if (!choose_config(ctx, *d, *li, d->nrows, tile_rows, cfg, &err)) {
+    return fail(ctx, GPL_E_ARG, err);
+  }
   apply_config(d, *li, *cfg);
   return GPL_OK;
 }
@@ -739,6 +747,107 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
   return GPL_OK;
 }
 
+GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_candidates, gpl_model_report* out) {
+  if (!ctx || !plan) return GPL_E_ARG;
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  const std::vector<std::string> segs = split_segments(plan);
+  if (segs.empty()) return fail(ctx, GPL_E_PLAN, "plan has no segment");
+  for (size_t i = 0; i + 1 < segs.size(); i++)
+    if ((st = gpl_build_hash(ctx, segs[i].c_str(), nullptr))) return st;
+  const std::string& probe = segs.back();
+  // one eager run profiles λ (the split and the model depend on it)
+  if ((st = gpl_run_plan(ctx, probe.c_str(), 0))) return st;
+  gpl_result tmp{};
+  tmp.cap_groups = 0;
+  gpl_fetch_result(ctx, &tmp);  // records λ; capacity errors are irrelevant here
+  ctx->err.clear();
+  // the model's shortlist
+  Segment seg;
+  std::string err;
+  if (!parse_segment(probe, &seg, &err)) return fail(ctx, GPL_E_PLAN, err);
+  PipeDesc d;
+  LowerInfo li;
+  if ((st = lower_probe(ctx, seg, choose_split(ctx, seg), &d, &li, &err))) return fail(ctx, st, err);
+  auto lit = ctx->lambda.find(seg.text);
+  if (lit != ctx->lambda.end()) li.lambda = lit->second;
+  for (int i = 0; i < d.nht; i++) {
+    const HashTable& h = ctx->hts[li.ht_ids[i]];
+    li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+  }
+  Config best_model;
+  std::vector<Config> cands;
+  ctx->tuned.erase(seg.text);
+  if (!choose_config(ctx, d, li, d.nrows, 0, &best_model, &err, &cands)) return fail(ctx, GPL_E_ARG, err);
+  if (max_candidates > 0 && (int)cands.size() > max_candidates) cands.resize(max_candidates);
+  // L2 flush buffer (2x L2) so every timing starts cold, as the bench does
+  void* flush = nullptr;
+  const size_t fbytes = (size_t)2 * ctx->l2_bytes;
+  CK(cudaMalloc(&flush, fbytes));
+  double best_ms = 1e300;
+  TunedShape best;
+  int tried = 0;
+  for (const Config& c : cands) {
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm};
+    ctx->tuned[seg.text] = t;
+    ctx->run_cache.erase(probe + "\x1f" + std::to_string(0));
+    std::vector<float> ms;
+    for (int rep = 0; rep < 4; rep++) {
+      if (cudaMemsetAsync(flush, rep, fbytes, ctx->stream) != cudaSuccess) break;
+      if ((st = gpl_run_plan(ctx, probe.c_str(), 0))) break;
+      if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) break;
+      float m = 0;
+      cudaEventElapsedTime(&m, ctx->ev0, ctx->ev1);
+      if (rep > 0) ms.push_back(m);
+    }
+    if (st) {  // a candidate that cannot run (resources) is skipped
+      st = GPL_OK;
+      ctx->err.clear();
+      continue;
+    }
+    if (ms.size() < 3) continue;
+    std::sort(ms.begin(), ms.end());
+    tried++;
+    if (ms[1] < best_ms) {
+      best_ms = ms[1];
+      best = t;
+    }
+  }
+  cudaFree(flush);
+  take_device_errors(ctx);
+  if (tried == 0) {
+    ctx->tuned.erase(seg.text);
+    return fail(ctx, GPL_E_CUDA, "no candidate configuration could run");
+  }
+  ctx->tuned[seg.text] = best;
+  ctx->run_cache.erase(probe + "\x1f" + std::to_string(0));
+  for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
+  ctx->graphs.clear();
+  if (out) {
+    const Config c = predict(ctx, d, li, std::max<int64_t>(d.nrows, 1), best.tile_rows, best.stage_rows, best.depth,
+                             best.warps, best.ctas_per_sm);
+    *out = gpl_model_report{};
+    out->tile_rows = c.tile_rows;
+    out->stage_rows = c.stage_rows;
+    out->ring_depth = c.depth;
+    out->consumer_warps = c.warps;
+    out->grid = c.grid;
+    out->predicted_ms = c.pred_ms;
+    out->t_stream_ms = c.t_stream_ms;
+    out->t_probe_ms = c.t_probe_ms;
+    out->t_tail_ms = c.t_tail_ms;
+    out->t_launch_ms = c.t_launch_ms;
+    out->bw_gbs = c.bw_gbs;
+    out->smem_bytes = c.smem;
+    out->feasible = c.feasible;
+    out->ctas_per_sm = c.ctas_per_sm;
+    out->candidates = tried;
+    out->measured_ms = best_ms;
+  }
+  return GPL_OK;
+}
+
 GPL_API gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows) {
   if (!ctx || !probe_segment) return GPL_E_ARG;
   ctx->err.clear();
@@ -923,5 +1032,6 @@ GPL_API gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment,
   out->bw_gbs = c.bw_gbs;
   out->smem_bytes = c.smem;
   out->feasible = c.feasible;
+  out->ctas_per_sm = c.ctas_per_sm;
   return GPL_OK;
 }

@@ -26,6 +26,8 @@ constexpr int MAXOPS = 16;   // op_pass counters
 constexpr int RPL = 4;       // rows per lane per consumer iteration (128-row warp packets)
 constexpr int MAXSP = 2;     // probes that may run in the stage phase (register slots)
 constexpr int QCAP = 256;    // survivor-queue entries per warp (>= 127 + 128)
+constexpr int kSmemTableMax = 32 * 1024;     // DIRECT tables up to this size are staged in smem
+constexpr int kSmemTablesTotal = 48 * 1024;  // ... up to this total per CTA
 
 constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;
 constexpr unsigned long long EMPTY64 = 0xFFFFFFFFFFFFFFFFull;
@@ -156,6 +158,10 @@ struct PipeDesc {
   Term term[MAXTERM];
   Agg agg[MAXA];
   HTRef ht[MAXHT];
+  // small DIRECT tables copied into shared memory at kernel start (-1: global)
+  int32_t ht_smem_off[MAXHT];
+  int32_t ht_smem_bytes[MAXHT];
+  int32_t smem_tables_bytes;
   // smem layout
   int32_t off_queue, off_agg, off_ring, smem_bytes;
   // outputs

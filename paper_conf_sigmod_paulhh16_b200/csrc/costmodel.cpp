@@ -29,6 +29,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <map>
 
 namespace gpl {
 
@@ -45,7 +46,7 @@ int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth
   int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   int slot = 0;
   for (int c = 0; c < d.ncols; c++) slot += align128(stage_rows * d.colw[c]);
-  return align128(kFixed + q) + align128(agg) + depth * slot;
+  return align128(kFixed + q) + align128(agg) + align128(d.smem_tables_bytes) + depth * slot;
 }
 
 void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
@@ -56,7 +57,10 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->off_queue = kFixed;
   d->off_agg = align128(kFixed + c.warps * d->qbytes);
   int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
-  d->off_ring = d->off_agg + align128(agg);
+  const int off_tables = d->off_agg + align128(agg);
+  for (int i = 0; i < d->nht; i++)
+    if (d->ht_smem_off[i] >= 0) d->ht_smem_off[i] += off_tables;  // relative -> absolute
+  d->off_ring = off_tables + align128(d->smem_tables_bytes);
   int off = 0;
   for (int i = 0; i < d->ncols; i++) {
     d->coloff[i] = off;
@@ -76,7 +80,11 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.ctas_per_sm = k;
   c.grid = ctx->sms * k;
   c.smem = smem_bytes(d, li, S, depth, W);
-  c.feasible = c.smem * k <= ctx->smem_optin && W >= 1 && W <= pipeline_max_consumer_warps() && depth >= 2;
+  // Eq 2 analog: shared memory (228 KB per SM, 1 KB reserved per CTA),
+  // threads and registers (<= 80 per thread assumed) of k resident CTAs
+  c.feasible = c.smem <= ctx->smem_optin && k * (c.smem + 1024) <= 228 * 1024 && W >= 1 &&
+               W <= pipeline_max_consumer_warps() && depth >= 2 && k * (W + 1) * 32 <= 2048 &&
+               k * (W + 1) * 32 * 80 <= 65536;
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
   const double b = std::max(1, li.bytes_per_row);
@@ -104,18 +112,29 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   const double qfrac = reach.size() > (size_t)(li.nfilt + d.nsprobe) ? reach[li.nfilt + d.nsprobe] : 1.0;
   const double stage_cost = 40 + 12.0 * d.nfilt + 60.0 * d.nsprobe + 14.0 * d.npush * std::min(1.0, 8 * qfrac);
   const double queue_cost = 60 + 90.0 * (d.nprobe - d.nsprobe) + 25.0 * d.nresid + 40.0 * d.nterm + 12.0 * d.nagg;
-  const double instr_per_row = (stage_cost + qfrac * queue_cost) / 128.0;
-  const double issue_sm = 4.0 * f_sm * 0.5 * std::min(1.0, W / 6.0);  // warp-instr/s one SM sustains
-  const double R_cons = issue_sm / instr_per_row * b * k;              // bytes/s one SM's consumers absorb
-  const double t_cons = (double)N * instr_per_row / (issue_sm * ctx->sms);
+  const double instr_iter = stage_cost + qfrac * queue_cost;  // per warp per 128 rows
+  // Latency of the probes on a warp iteration's critical path, by where the
+  // table lives: staged in smem, small enough for L1, L2-resident, or HBM.
+  auto lat = [&](int t) {
+    if (d.ht_smem_off[t] >= 0) return 40.0;
+    const double bytes = li.ht_bytes.empty() ? 1e6 : (double)li.ht_bytes[t];
+    return bytes <= 64e3 ? 80.0 : bytes <= L2_eff ? 500.0 : 1000.0;
+  };
+  double lat_stage = 0, lat_queue = 0;
+  for (int p = 0; p < li.nprobe; p++) (p < d.nsprobe ? lat_stage : lat_queue) += lat(li.probe_ht[p]);
+  const double crit = 150.0 + lat_stage + qfrac * lat_queue + instr_iter;  // cycles per warp iteration
+  const double w_eff = (double)std::min(W, S / 128) * k;                   // warps with work per stage
+  const double rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 / crit);  // per SM
+  const double R_cons = rows_cyc * f_sm * b;                                // bytes/s one SM's consumers absorb
+  const double t_cons = (double)N / (rows_cyc * f_sm * ctx->sms);
 
   // Eq 3 analog: waves of Δ-row tiles over G persistent CTAs, with the last wave's tail
   const int64_t tiles = (N + tile - 1) / tile;
   const int64_t G = c.grid;
   const int64_t waves = (tiles + G - 1) / G;
   const int64_t last = tiles - (waves - 1) * G;
-  const double rate_full = std::min(std::min(B_sm, R_cons / k), B / (double)std::min<int64_t>(G, tiles));
-  const double rate_last = std::min(std::min(B_sm, R_cons / k), B / (double)last);
+  const double rate_full = std::min(std::min(B_sm, R_cons) / k, B / (double)std::min<int64_t>(G, tiles));
+  const double rate_last = std::min(std::min(B_sm, R_cons) / k, B / (double)last);
   const double t_tile = tile * b / rate_full;
   const double last_rows = (double)(N - (tiles - 1) * tile);
   const double t_last = (last == 1 ? last_rows : (double)tile) * b / rate_last;
@@ -137,12 +156,13 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
 }
 
 bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t N, int64_t tile_req,
-                   Config* out, std::string* err) {
+                   Config* out, std::string* err, std::vector<Config>* shortlist) {
+  std::map<std::pair<int, int>, Config> per_shape;  // best predicted per (CTAs/SM, stage rows)
   const Options& o = ctx->opt;
   std::vector<int> Ss = o.stage_rows > 0 ? std::vector<int>{(int)o.stage_rows} : std::vector<int>{512, 1024, 2048, 4096};
   std::vector<int> Ds = o.ring_depth > 0 ? std::vector<int>{(int)o.ring_depth} : std::vector<int>{2, 3, 4, 6};
   std::vector<int> Ws = o.consumer_warps > 0 ? std::vector<int>{(int)o.consumer_warps} : std::vector<int>{4, 8, 12, 16};
-  int k = o.ctas_per_sm > 0 ? (int)o.ctas_per_sm : 1;
+  std::vector<int> Ks = o.ctas_per_sm > 0 ? std::vector<int>{(int)o.ctas_per_sm} : std::vector<int>{1, 2};
   Config best;
   bool found = false;
   for (int S : Ss) {
@@ -156,12 +176,18 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
         if (t >= N) break;
       }
     }
+    for (int k : Ks)
     for (int D : Ds)
       for (int W : Ws)
         for (int64_t t : tiles) {
           if (d.flush_each_tile && (long double)(t + QCAP) * std::max<long double>(li.maxabs, 1) >= 4.6e18L) continue;
           Config c = predict(ctx, d, li, N, t, S, D, W, k);
           if (!c.feasible) continue;
+          {
+            auto key = std::make_pair(k, S);
+            auto it = per_shape.find(key);
+            if (it == per_shape.end() || c.pred_ms < it->second.pred_ms) per_shape[key] = c;
+          }
           if (!found || c.pred_ms < best.pred_ms * (1 - 1e-9) ||
               (std::fabs(c.pred_ms - best.pred_ms) <= best.pred_ms * 1e-9 && c.tile_rows > best.tile_rows)) {
             best = c;
@@ -174,6 +200,11 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
     return false;
   }
   *out = best;
+  if (shortlist) {
+    shortlist->clear();
+    for (auto& kv : per_shape) shortlist->push_back(kv.second);
+    std::sort(shortlist->begin(), shortlist->end(), [](const Config& a, const Config& b) { return a.pred_ms < b.pred_ms; });
+  }
   return true;
 }
 

@@ -3,6 +3,7 @@
 // P:205-315) — see costmodel.cpp for the term-by-term mapping.
 #pragma once
 #include <string>
+#include <vector>
 
 #include "ctx.h"
 
@@ -24,8 +25,10 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
 
 // Search the feasible space (Δ, stage rows, depth, consumer warps), honouring
 // options and a requested tile_rows (> 0 fixes Δ). Returns false if nothing fits.
+// shortlist (optional): the best predicted configuration for every
+// (CTAs per SM, stage rows) shape, best first — the candidates gpl_autotune measures.
 bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t nrows, int64_t tile_req,
-                   Config* out, std::string* err);
+                   Config* out, std::string* err, std::vector<Config>* shortlist = nullptr);
 
 // Fill the schedule and shared-memory layout fields of d from c.
 void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c);

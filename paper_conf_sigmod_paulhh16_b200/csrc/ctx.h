@@ -109,6 +109,12 @@ struct PreparedBuild {
   std::vector<int> src_ids;
 };
 
+// gpl_autotune's pinned pipeline shape for one probe segment
+struct TunedShape {
+  int64_t tile_rows = 0;
+  int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1;
+};
+
 struct Options {
   int64_t stage_rows = -1, ring_depth = -1, consumer_warps = -1, ctas_per_sm = -1, probe_split = -2,
           hash_load_pct = -1;
@@ -147,6 +153,7 @@ struct gpl_ctx {
   std::map<std::string, gpl::PreparedBuild> build_cache;
   // gpl_run_query: whole-query CUDA graphs (builds + fused run), keyed by plan text + tile_rows
   std::map<std::string, cudaGraphExec_t> graphs;
+  std::map<std::string, gpl::TunedShape> tuned;  // probe segment text -> measured-best shape
   void* h_stage = nullptr;  // pinned host staging for one packed D2H of results
   size_t h_stage_cap = 0;
   // KBE scratch (gpl_run_plan_kbe)

@@ -157,7 +157,10 @@ std::string shape_source(const PipeDesc& d) {
     o << "  k.agg[" << a << "] = gpl::Agg{" << d.agg[a].kind << ", " << d.agg[a].field << ", " << i64(d.agg[a].c) << "};\n";
   for (int h = 0; h < d.nht; h++)
     o << "  k.ht[" << h << "].kind = " << d.ht[h].kind << "; k.ht[" << h << "].hash = " << d.ht[h].hash << "; k.ht[" << h
-      << "].width = " << d.ht[h].width << ";\n";
+      << "].width = " << d.ht[h].width << "; k.ht_smem_off[" << h << "] = " << d.ht_smem_off[h] << "; k.ht_smem_bytes["
+      << h << "] = " << d.ht_smem_bytes[h] << ";\n";
+  for (int h = d.nht; h < MAXHT; h++) o << "  k.ht_smem_off[" << h << "] = -1;\n";
+  I("smem_tables_bytes", d.smem_tables_bytes);
   I("off_queue", d.off_queue);
   I("off_agg", d.off_agg);
   I("off_ring", d.off_ring);

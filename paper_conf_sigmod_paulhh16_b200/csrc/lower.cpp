@@ -239,6 +239,22 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     li->probe_ht.push_back(ht_slot[H.id]);
   }
   d->nht = (int)ht_slot.size();
+  // small DIRECT tables live in shared memory for the kernel's lifetime
+  // (offsets relative to the tables region; apply_config makes them absolute)
+  {
+    int off = 0;
+    for (int i = 0; i < MAXHT; i++) d->ht_smem_off[i] = -1, d->ht_smem_bytes[i] = 0;
+    for (int i = 0; i < d->nht; i++) {
+      const HashTable& H = ctx->hts[li->ht_ids[i]];
+      const int b = (int)((H.bytes() + 15) / 16 * 16);
+      if (H.kind == HT_DIRECT && b <= kSmemTableMax && off + b <= kSmemTablesTotal) {
+        d->ht_smem_off[i] = off;
+        d->ht_smem_bytes[i] = b;
+        off += b;
+      }
+    }
+    d->smem_tables_bytes = off;
+  }
 
   // staged columns
   std::vector<const Column*> cols;

@@ -100,6 +100,35 @@ __device__ __forceinline__ void qput(const PipeDesc& K, uint32_t qb, int f, int 
   else S<long long>(a + i * 8) = v;
 }
 
+// Probe RPL rows of one lane in table t: small DIRECT tables were staged in
+// shared memory by the prologue (LDS, no L1/L2 round trip); the rest go to
+// global memory (ht_probe_n: all RPL loads in flight).
+__device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP* htp, int t, const unsigned long long (&key)[RPL],
+                                           const bool (&act)[RPL], bool (&hit)[RPL], long long (&pay)[RPL]) {
+  const int kind = K.ht[t].kind, width = K.ht[t].width, so = K.ht_smem_off[t];
+  if (kind == HT_DIRECT && so >= 0) {
+    const HTP& h = htp[t];
+    uint32_t v[RPL];
+#pragma unroll
+    for (int j = 0; j < RPL; j++) {
+      const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
+      const bool in = act[j] && idx < h.nslots;
+      const uint32_t i = (uint32_t)idx;
+      if (width == 0) v[j] = in ? (S<uint32_t>(so + (i >> 5) * 4) >> (i & 31)) & 1u : 0u;
+      else if (width == 1) v[j] = in ? (uint32_t)S<unsigned char>(so + i) : 0u;
+      else if (width == 2) v[j] = in ? (uint32_t)S<unsigned short>(so + i * 2) : 0u;
+      else v[j] = in ? S<uint32_t>(so + i * 4) : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < RPL; j++) {
+      hit[j] = v[j] != 0;
+      pay[j] = width == 0 ? 1 : (long long)v[j] - 1 + h.pay_base;
+    }
+    return;
+  }
+  ht_probe_n<RPL>(htp[t], kind, width, key, act, hit, pay);
+}
+
 __device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
   return (unsigned)p[0] + (unsigned)p[1] + (unsigned)p[2] + (unsigned)p[3];
 }
@@ -133,7 +162,7 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
       }
       bool hit[RPL];
       long long v[RPL];
-      ht_probe_n<RPL>(htp[P.ht], K.ht[P.ht].kind, K.ht[P.ht].width, k, p, hit, v);
+      probe_rows(K, htp, P.ht, k, p, hit, v);
 #pragma unroll
       for (int j = 0; j < RPL; j++) {
         if (P.kind == P_MARK) {
@@ -256,6 +285,14 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     fence_mbar_init();
   }
   if (threadIdx.x < K.nht) htp[threadIdx.x] = load_htp(d.ht[threadIdx.x]);
+  GPL_UNROLL
+  for (int t = 0; t < K.nht; t++) {  // stage small DIRECT tables into shared memory
+    if (K.ht_smem_off[t] >= 0) {
+      const uint4* src = (const uint4*)d.ht[t].slots;
+      for (int j = threadIdx.x; j < K.ht_smem_bytes[t] / 16; j += blockDim.x)
+        S<uint4>(K.ht_smem_off[t] + j * 16) = __ldg(src + j);
+    }
+  }
   for (int i = threadIdx.x; i < kMaxWarps * MAXOPS; i += blockDim.x) cnt_all[i] = 0;
   if (K.agg_mode == AGG_SMEM)
     for (int i = threadIdx.x; i < K.ngroups_total * K.nagg; i += blockDim.x) stab[i] = 0;
@@ -346,7 +383,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             }
             bool hit[RPL];
             long long v[RPL];
-            ht_probe_n<RPL>(htp[P.ht], K.ht[P.ht].kind, K.ht[P.ht].width, k, p, hit, v);
+            probe_rows(K, htp, P.ht, k, p, hit, v);
 #pragma unroll
             for (int j = 0; j < RPL; j++) {
               if (P.kind == P_MARK) {

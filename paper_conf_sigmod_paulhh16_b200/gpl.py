@@ -28,7 +28,8 @@ GPL_COPY, GPL_BORROW = 0, 1
 EXPORTED = ["gpl_create", "gpl_destroy", "gpl_load_columns", "gpl_build_hash", "gpl_run_plan",
             "gpl_run_plan_kbe", "gpl_fetch_result", "gpl_fetch_partials", "gpl_decode_partials",
             "gpl_merge_partials", "gpl_sync", "gpl_choose_tile_rows", "gpl_set_option",
-            "gpl_check_plan", "gpl_compile_plan", "gpl_run_query", "gpl_last_error", "gpl_version"]
+            "gpl_check_plan", "gpl_compile_plan", "gpl_run_query", "gpl_autotune", "gpl_last_error",
+            "gpl_version"]
 
 
 class GplError(RuntimeError):
@@ -65,7 +66,8 @@ class _Model(ctypes.Structure):
                 ("consumer_warps", ctypes.c_int32), ("grid", ctypes.c_int32), ("predicted_ms", ctypes.c_double),
                 ("t_stream_ms", ctypes.c_double), ("t_probe_ms", ctypes.c_double), ("t_tail_ms", ctypes.c_double),
                 ("t_launch_ms", ctypes.c_double), ("bw_gbs", ctypes.c_double), ("smem_bytes", ctypes.c_int32),
-                ("feasible", ctypes.c_int32)]
+                ("feasible", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32), ("candidates", ctypes.c_int32),
+                ("measured_ms", ctypes.c_double)]
 
 
 _lib = None
@@ -98,6 +100,7 @@ def load_library():
         "gpl_check_plan": ([P, ctypes.c_char_p], I32),
         "gpl_compile_plan": ([P, ctypes.c_char_p, I64], I32),
         "gpl_run_query": ([P, ctypes.c_char_p, I64], I32),
+        "gpl_autotune": ([P, ctypes.c_char_p, I32, ctypes.POINTER(_Model)], I32),
         "gpl_last_error": ([P], ctypes.c_char_p),
         "gpl_version": ([], ctypes.c_char_p),
     }
@@ -231,6 +234,12 @@ class Context:
     def run_query(self, plan: str, tile_rows: int = 0):
         """All segments of a plan (builds then the probe segment); replays a CUDA graph once warm."""
         self._check(self._lib.gpl_run_query(self._h, plan.encode(), int(tile_rows)))
+
+    def autotune(self, plan: str, max_candidates: int = 0) -> dict:
+        """Measure the model's shortlist of pipeline shapes for this query and pin the fastest."""
+        m = _Model()
+        self._check(self._lib.gpl_autotune(self._h, plan.encode(), int(max_candidates), ctypes.byref(m)))
+        return {k: getattr(m, k) for k, _ in _Model._fields_}
 
     def run_plan_kbe(self, segment: str):
         self._check(self._lib.gpl_run_plan_kbe(self._h, segment.encode()))

@@ -203,3 +203,18 @@ def test_query_graph_replay_and_invalidation(ctx):
     for _ in range(3):
         r = queries.run_query(ctx, "Q5", db2)
         assert r.keys == o2.keys and r.aggs == o2.aggs
+
+
+def test_autotune_pins_a_measured_shape(ctx):
+    """gpl_autotune measures the model's shortlist and pins the fastest shape;
+    the pinned shape must keep results exact."""
+    db = tpchgen.generate(0.1, seed=41)
+    queries.load_database(ctx, db, queries.TABLES["Q7"])
+    m = ctx.autotune(queries.plan_text("Q7", db))
+    assert m["candidates"] >= 1 and m["measured_ms"] > 0
+    r = queries.run_query(ctx, "Q7", db)
+    o = oracle.run("Q7", db)
+    assert r.keys == o.keys and r.aggs == o.aggs
+    assert (r.stats["stage_rows"], r.stats["ring_depth"], r.stats["consumer_warps"]) == \
+        (m["stage_rows"], m["ring_depth"], m["consumer_warps"])
+    ctx.set_option("stage_rows", -1)  # any option change un-pins
