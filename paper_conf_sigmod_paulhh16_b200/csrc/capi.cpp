@@ -461,7 +461,8 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
     idx = it->second;
   }
   HashTable& H = ctx->hts[idx];
-  const size_t need = std::max<size_t>(shape.bytes(), 16);
+  // rounded to 256 B: kernels stage small tables with 16-B vector loads
+  const size_t need = (std::max<size_t>(shape.bytes(), 16) + 255) / 256 * 256;
   if (!H.slots || H.alloc_bytes < need) {
     CK(cudaStreamSynchronize(ctx->stream));
     if (H.slots) cudaFree(H.slots);
