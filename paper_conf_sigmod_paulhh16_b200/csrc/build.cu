@@ -23,24 +23,43 @@ namespace {
 
 constexpr int kThreads = 256;
 
-// Evaluate BR build rows at once (rows row0 + j*stride): filters, probes into
-// earlier tables (a miss drops the row: inner / semi join), key and payload.
-// Every
-// column load and hash probe of the BR rows is issued before any is needed,
-// so one thread keeps BR independent memory round trips in flight.
+// Evaluate BR consecutive build rows at once (row0 % BR == 0): filters,
+// probes into earlier tables (a miss drops the row: inner / semi join), key
+// and payload. The filter columns are read with one 16-B vector load per
+// BR = 4 rows and every probe of the BR rows is issued before any is needed,
+// so one thread keeps BR independent memory round trips in flight (the build
+// is latency-bound otherwise). Rows past nrows read the zero padding of the
+// column store (64-row padded copies; borrowed columns hold >= 4-row multiples).
+// Measured on B200 (Q5 SF1 builds): BR = 1 with one row per thread is faster
+// than BR = 4 (5.4/19.7/5.0 us vs 9.0/25.6/8.7 us): the per-row chains are
+// predicated control flow that does not overlap, and fewer threads are
+// resident. Kept selectable for experiments.
 #ifndef GPL_BUILD_BR
 #define GPL_BUILD_BR 1
 #endif
 constexpr int BR = GPL_BUILD_BR;
+__device__ __forceinline__ void ld4_global(const char* col, int w, long long row0, long long (&x)[BR]) {
+  if (BR != 4) {
+#pragma unroll
+    for (int j = 0; j < BR; j++) x[j] = ld_col_global(col, w, row0 + j);
+  } else if (w == 4) {
+    const int4 v = __ldg((const int4*)col + (row0 >> 2));
+    x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
+  } else {
+    const longlong2 a = __ldg((const longlong2*)col + (row0 >> 1));
+    const longlong2 b = __ldg((const longlong2*)col + (row0 >> 1) + 1);
+    x[0] = a.x; x[1] = a.y; x[2] = b.x; x[3] = b.y;
+  }
+}
 __device__ __forceinline__ void build_rows(const BuildDesc& d, const HTP* src, long long row0, long long stride,
                                            bool (&ok)[BR], unsigned long long (&key)[BR], long long (&pay)[BR]) {
+  (void)stride;
 #pragma unroll
-  for (int j = 0; j < BR; j++) ok[j] = row0 + j * stride < d.nrows;
+  for (int j = 0; j < BR; j++) ok[j] = row0 + j < d.nrows;
   for (int f = 0; f < d.nfilt; f++) {
     const Filt& F = d.filt[f];
     long long x[BR];
-#pragma unroll
-    for (int j = 0; j < BR; j++) x[j] = ok[j] ? ld_col_global(d.col[F.ref], d.colw[F.ref], row0 + j * stride) : 0;
+    ld4_global(d.col[F.ref], d.colw[F.ref], row0, x);
 #pragma unroll
     for (int j = 0; j < BR; j++) ok[j] = ok[j] && filt_pass(F, x[j]);
   }
@@ -54,8 +73,8 @@ __device__ __forceinline__ void build_rows(const BuildDesc& d, const HTP* src, l
       unsigned long long k[BR];
 #pragma unroll
       for (int j = 0; j < BR; j++) {
-        k[j] = ok[j] ? (uint32_t)ld_col_global(d.col[P.k1], d.colw[P.k1], row0 + j * stride) : 0u;
-        if (P.k2 >= 0 && ok[j]) k[j] = (k[j] << 32) | (uint32_t)ld_col_global(d.col[P.k2], d.colw[P.k2], row0 + j * stride);
+        k[j] = ok[j] ? (uint32_t)ld_col_global(d.col[P.k1], d.colw[P.k1], row0 + j) : 0u;
+        if (P.k2 >= 0 && ok[j]) k[j] = (k[j] << 32) | (uint32_t)ld_col_global(d.col[P.k2], d.colw[P.k2], row0 + j);
       }
       bool hit[BR];
       long long v[BR];
@@ -70,7 +89,7 @@ __device__ __forceinline__ void build_rows(const BuildDesc& d, const HTP* src, l
   }
 #pragma unroll
   for (int j = 0; j < BR; j++) {
-    const long long row = row0 + j * stride;
+    const long long row = row0 + j;
     key[j] = 0;
     pay[j] = 0;
     if (!ok[j]) continue;
@@ -127,7 +146,7 @@ __global__ void __launch_bounds__(kThreads) build_count_kernel(const __grid_cons
   unsigned long long cnt = 0;
   long long mn = LLONG_MAX, mx = LLONG_MIN;
   const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long row = (long long)blockIdx.x * blockDim.x + threadIdx.x; row < d.nrows; row += stride * BR) {
+  for (long long row = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * BR; row < d.nrows; row += stride * BR) {
     bool ok[BR];
     unsigned long long k[BR];
     long long pay[BR];
@@ -216,7 +235,7 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
   }
   __syncthreads();
   const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long row0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; row0 < d.nrows; row0 += stride * BR) {
+  for (long long row0 = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * BR; row0 < d.nrows; row0 += stride * BR) {
    bool okv[BR];
    unsigned long long keyv[BR];
    long long payv[BR];
@@ -319,7 +338,7 @@ cudaError_t launch_header_init(HTHeader* hdr, cudaStream_t s) {
 
 cudaError_t launch_build(const BuildDesc& d, bool trivial, const HTHeader& known, int num_sms, cudaStream_t s) {
   long long work = d.nrows > 0 ? d.nrows : 1;
-  int grid = (int)std::min<long long>((work + kThreads - 1) / kThreads, (long long)num_sms * 8);
+  int grid = (int)std::min<long long>((work + kThreads * BR - 1) / (kThreads * BR), (long long)num_sms * 8);
   if (grid < 1) grid = 1;
   if (d.kind == HT_DIRECT) {  // host-sized: clear + insert, no count pass
     cudaError_t e = cudaMemsetAsync(d.slots, 0, direct_bytes(d.width, d.nslots), s);

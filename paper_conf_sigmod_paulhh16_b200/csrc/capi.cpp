@@ -87,7 +87,7 @@ gpl_status take_device_errors(gpl_ctx* ctx) {
 }
 
 gpl_status decode(gpl_ctx* ctx, const unsigned long long* part, gpl_result* out) {
-  const LowerInfo& li = ctx->last.li;
+  const LowerInfo& li = ctx->last.run->li;
   const int G = li.ngroups_total, A = li.nagg;
   out->n_keys = li.ngroup_dims;
   out->n_aggs = A;
@@ -571,7 +571,7 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
   const size_t lambda_n = lam == ctx->lambda.end() ? 0 : lam->second.size();
   auto it = ctx->run_cache.find(key);
   if (it != ctx->run_cache.end()) {
-    PreparedRun& P = it->second;
+    PreparedRun& P = *it->second;
     if (run_cache_valid(ctx, P)) {
       *out = &P;
       return GPL_OK;
@@ -602,7 +602,9 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
   P.fn = resolve_pipeline_fn(d, ctx->opt.jit != 0, &jerr);
   P.jit = ctx->opt.jit != 0 && jerr.empty();
   if (!P.fn) return fail(ctx, GPL_E_CUDA, "cannot configure the pipeline kernel");
-  *out = &(ctx->run_cache[key] = P);
+  auto sp = std::make_shared<PreparedRun>(P);
+  ctx->run_cache[key] = sp;
+  *out = sp.get();
   return GPL_OK;
 }
 
@@ -625,9 +627,7 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   LastRun& L = ctx->last;
   L.valid = true;
   L.kbe = false;
-  L.text = P->text;
-  L.desc = d;
-  L.li = li;
+  L.run = ctx->run_cache[std::string(probe_segment) + "\x1f" + std::to_string(tile_rows)];
   L.timed = true;
   gpl_stats& S = L.stats;
   S = gpl_stats{};
@@ -675,7 +675,9 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
-  const std::vector<std::string> segs = split_segments(plan);
+  auto ps = ctx->plan_segs.find(plan);
+  if (ps == ctx->plan_segs.end()) ps = ctx->plan_segs.emplace(plan, split_segments(plan)).first;
+  const std::vector<std::string>& segs = ps->second;
   if (segs.empty()) return fail(ctx, GPL_E_PLAN, "plan has no segment");
   const std::string key = std::string(plan) + "\x1f" + std::to_string(tile_rows);
   const std::string run_key = segs.back() + "\x1f" + std::to_string(tile_rows);
@@ -686,7 +688,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       if (b == ctx->build_cache.end() || !build_cache_valid(ctx, b->second)) return false;
     }
     auto r = ctx->run_cache.find(run_key);
-    return r != ctx->run_cache.end() && run_cache_valid(ctx, r->second) && ctx->lambda.count(r->second.text);
+    return r != ctx->run_cache.end() && run_cache_valid(ctx, *r->second) && ctx->lambda.count(r->second->text);
   };
   auto eager = [&]() -> gpl_status {
     for (size_t i = 0; i + 1 < segs.size(); i++) {
@@ -700,13 +702,12 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     if (all_valid()) {
       CK(cudaGraphLaunch(g->second, ctx->stream));
       // the run's bookkeeping is the cached plan's
-      const PreparedRun& P = ctx->run_cache[run_key];
+      const std::shared_ptr<PreparedRun>& PP = ctx->run_cache[run_key];
+      const PreparedRun& P = *PP;
       LastRun& L = ctx->last;
       L.valid = true;
       L.kbe = false;
-      L.text = P.text;
-      L.desc = P.desc;
-      L.li = P.li;
+      L.run = PP;
       L.timed = true;
       gpl_stats& S = L.stats;
       S = gpl_stats{};
@@ -898,9 +899,13 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   LastRun& L = ctx->last;
   L.valid = true;
   L.kbe = true;
-  L.text = seg.text;
-  L.desc = d;
-  L.li = li;
+  {
+    auto kr = std::make_shared<PreparedRun>();
+    kr->desc = d;
+    kr->li = li;
+    kr->text = seg.text;
+    L.run = kr;
+  }
   L.timed = true;
   gpl_stats& S = L.stats;
   S = gpl_stats{};
@@ -928,7 +933,7 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   gpl_status st = check_dev(ctx);
   if (st) return st;
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run to fetch");
-  const LowerInfo& li = ctx->last.li;
+  const LowerInfo& li = ctx->last.run->li;
   // one D2H: error bits, counter, op_pass and partials are contiguous
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
   CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
@@ -945,10 +950,10 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   for (int i = 0; i < MAXOPS && i < 16; i++) S.op_pass[i] = (int64_t)ops[i];
   // λ cache for the model / split choice (cumulative pass fraction after each op)
   // (recorded once per plan text: the first run profiles the plan)
-  if (!ctx->last.kbe && S.rows_scanned > 0 && !ctx->lambda.count(ctx->last.text)) {
+  if (!ctx->last.kbe && S.rows_scanned > 0 && !ctx->lambda.count(ctx->last.run->text)) {
     std::vector<double> lam;
     for (int i = 0; i < li.nops; i++) lam.push_back((double)ops[i] / (double)S.rows_scanned);
-    ctx->lambda[ctx->last.text] = lam;
+    ctx->lambda[ctx->last.run->text] = lam;
   }
   out->stats = S;
   if (bits) {
@@ -962,7 +967,7 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
   gpl_status st = check_dev(ctx);
   if (st) return st;
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run");
-  const size_t b = (size_t)ctx->last.li.ngroups_total * ctx->last.li.nagg * 16;
+  const size_t b = (size_t)ctx->last.run->li.ngroups_total * ctx->last.run->li.nagg * 16;
   *nbytes = b;
   if (cap_bytes < b || !dst) return fail(ctx, GPL_E_CAPACITY, "partials buffer too small");
   CK(cudaMemcpyAsync(dst, partials_ptr(ctx), b, dst_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
@@ -974,7 +979,7 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
 GPL_API gpl_status gpl_decode_partials(gpl_ctx* ctx, const void* host_partials, size_t nbytes, gpl_result* out) {
   if (!ctx || !host_partials || !out) return GPL_E_ARG;
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run (the plan of the last run defines the layout)");
-  const size_t b = (size_t)ctx->last.li.ngroups_total * ctx->last.li.nagg * 16;
+  const size_t b = (size_t)ctx->last.run->li.ngroups_total * ctx->last.run->li.nagg * 16;
   if (nbytes != b) return fail(ctx, GPL_E_ARG, "partials size does not match the last run's plan");
   gpl_stats& S = ctx->last.stats;
   if (ctx->last.timed && !ctx->host_only && cudaEventQuery(ctx->ev1) == cudaSuccess) {

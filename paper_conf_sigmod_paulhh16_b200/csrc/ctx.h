@@ -4,6 +4,7 @@
 
 #include <cstdint>
 #include <map>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -75,11 +76,12 @@ struct LowerInfo {
   std::vector<double> lambda;     // cumulative pass fraction after each op (previous run)
 };
 
+struct PreparedRun;
+
+// The last run: a shared reference to its prepared plan (no per-run copies)
 struct LastRun {
   bool valid = false;
-  std::string text;
-  PipeDesc desc{};
-  LowerInfo li;
+  std::shared_ptr<const PreparedRun> run;
   gpl_stats stats{};
   bool timed = false;
   bool kbe = false;
@@ -149,11 +151,12 @@ struct gpl_ctx {
   std::map<std::string, std::vector<double>> lambda;  // plan text -> per-op pass fraction (A9 "profile the first tile")
   // prepared-plan caches (keyed by segment text [+ tile_rows]); validated on
   // every use against table versions, hash-table refs and options
-  std::map<std::string, gpl::PreparedRun> run_cache;
+  std::map<std::string, std::shared_ptr<gpl::PreparedRun>> run_cache;
   std::map<std::string, gpl::PreparedBuild> build_cache;
   // gpl_run_query: whole-query CUDA graphs (builds + fused run), keyed by plan text + tile_rows
   std::map<std::string, cudaGraphExec_t> graphs;
   std::map<std::string, gpl::TunedShape> tuned;  // probe segment text -> measured-best shape
+  std::map<std::string, std::vector<std::string>> plan_segs;  // gpl_run_query: plan text -> segments
   void* h_stage = nullptr;  // pinned host staging for one packed D2H of results
   size_t h_stage_cap = 0;
   // KBE scratch (gpl_run_plan_kbe)

@@ -254,18 +254,30 @@ class Context:
     def sync(self):
         self._check(self._lib.gpl_sync(self._h))
 
-    def _result(self, fn, cap=4096) -> Result:
-        keys = np.zeros(cap * 4, dtype=np.int32)
-        aggs = np.zeros(cap * 8 * 2, dtype=np.int64)
-        r = _Result()
-        r.cap_groups = cap
+    def _result(self, fn) -> Result:
+        # result buffers are reused across calls (grown on GPL_E_CAPACITY)
+        if not hasattr(self, "_rbuf"):
+            self._rcap = 256
+            self._rbuf = (np.zeros(self._rcap * 4, dtype=np.int32), np.zeros(self._rcap * 8 * 2, dtype=np.int64),
+                          _Result())
+        keys, aggs, r = self._rbuf
+        r.cap_groups = self._rcap
         r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data
-        self._check(fn(ctypes.byref(r)))
-        nk, na = r.n_keys, r.n_aggs
-        out_k, out_a = [], []
-        for i in range(r.n_groups):
-            out_k.append(tuple(int(x) for x in keys[i * nk:(i + 1) * nk]))
-            out_a.append([_i128(aggs[(i * na + j) * 2], aggs[(i * na + j) * 2 + 1]) for j in range(na)])
+        st = fn(ctypes.byref(r))
+        if st == GPL_E_CAPACITY and r.n_groups > self._rcap:
+            self._rcap = r.n_groups
+            self._rbuf = (np.zeros(self._rcap * 4, dtype=np.int32), np.zeros(self._rcap * 8 * 2, dtype=np.int64),
+                          _Result())
+            keys, aggs, r = self._rbuf
+            r.cap_groups = self._rcap
+            r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data
+            st = fn(ctypes.byref(r))
+        self._check(st)
+        nk, na, ng = r.n_keys, r.n_aggs, r.n_groups
+        kl = keys[:ng * nk].tolist()
+        al = aggs[:ng * na * 2].tolist()
+        out_k = [tuple(kl[i * nk:(i + 1) * nk]) for i in range(ng)]
+        out_a = [[_i128(al[(i * na + j) * 2], al[(i * na + j) * 2 + 1]) for j in range(na)] for i in range(ng)]
         return Result(out_k, out_a, _stats_dict(r.stats))
 
     def fetch_result(self) -> Result:

@@ -34,3 +34,20 @@ for it in range(3):
     dev_ms = [evs[i].elapsed_time(evs[i + 1]) for i in range(len(evs) - 1)]
     print(f"iter {it}: host total {tot*1e3:.3f} ms; host per call (ms) {[round(h*1e3,3) for h in hs]}; "
           f"device per segment (ms) {[round(x,3) for x in dev_ms]}; kernel {r.stats['kernel_ms']:.3f}")
+# host-only overheads with the GPU idle
+torch.cuda.synchronize()
+import timeit
+n = 200
+t = timeit.timeit(lambda: ctx.fetch_result(), number=n) / n
+print(f"fetch_result with idle GPU: {t*1e6:.1f} us")
+t = timeit.timeit(lambda: ctx._lib.gpl_sync(ctx._h), number=n) / n
+print(f"gpl_sync (idle): {t*1e6:.1f} us")
+text = queries.plan_text(q, db)
+ctx.run_query(text); ctx.fetch_result(); ctx.run_query(text); ctx.fetch_result()
+torch.cuda.synchronize()
+t0 = time.perf_counter(); ctx.run_query(text); t1 = time.perf_counter(); r = ctx.fetch_result(); t2 = time.perf_counter()
+print(f"run_query (graph replay) host {1e6*(t1-t0):.1f} us; fetch (incl. wait) {1e6*(t2-t1):.1f} us; kernel {r.stats['kernel_ms']*1e3:.1f} us")
+evs = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+for i in range(3):
+    evs[0].record(); ctx.run_query(text); evs[1].record(); r = ctx.fetch_result(); evs[2].record(); torch.cuda.synchronize()
+    print(f"device: graph {evs[0].elapsed_time(evs[1])*1e3:.1f} us, to-fetch-end {evs[1].elapsed_time(evs[2])*1e3:.1f} us")
