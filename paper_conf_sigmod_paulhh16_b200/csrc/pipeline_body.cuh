@@ -103,21 +103,25 @@ __device__ __forceinline__ void qput(const PipeDesc& K, uint32_t qb, int f, int 
 // Probe RPL rows of one lane in table t: small DIRECT tables were staged in
 // shared memory by the prologue (LDS, no L1/L2 round trip); the rest go to
 // global memory (ht_probe_n: all RPL loads in flight).
-__device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP* htp, int t, const unsigned long long (&key)[RPL],
+__device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int t, const unsigned long long (&key)[RPL],
                                            const bool (&act)[RPL], bool (&hit)[RPL], long long (&pay)[RPL]) {
   const int kind = K.ht[t].kind, width = K.ht[t].width, so = K.ht_smem_off[t];
   if (kind == HT_DIRECT && so >= 0) {
-    const HTP& h = htp[t];
+    // branch-free: the cell index is clamped into the table and the loaded
+    // value masked, so the 4 shared-memory loads issue back to back
+    const uint32_t last = (uint32_t)(h.nslots - 1);
     uint32_t v[RPL];
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
       const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
       const bool in = act[j] && idx < h.nslots;
-      const uint32_t i = (uint32_t)idx;
-      if (width == 0) v[j] = in ? (S<uint32_t>(so + (i >> 5) * 4) >> (i & 31)) & 1u : 0u;
-      else if (width == 1) v[j] = in ? (uint32_t)S<unsigned char>(so + i) : 0u;
-      else if (width == 2) v[j] = in ? (uint32_t)S<unsigned short>(so + i * 2) : 0u;
-      else v[j] = in ? S<uint32_t>(so + i * 4) : 0u;
+      const uint32_t i = in ? (uint32_t)idx : last;
+      uint32_t x;
+      if (width == 0) x = (S<uint32_t>(so + (i >> 5) * 4) >> (i & 31)) & 1u;
+      else if (width == 1) x = (uint32_t)S<unsigned char>(so + i);
+      else if (width == 2) x = (uint32_t)S<unsigned short>(so + i * 2);
+      else x = S<uint32_t>(so + i * 4);
+      v[j] = in ? x : 0u;
     }
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
@@ -126,7 +130,7 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP* htp, in
     }
     return;
   }
-  ht_probe_n<RPL>(htp[t], kind, width, key, act, hit, pay);
+  ht_probe_n<RPL>(h, kind, width, key, act, hit, pay);
 }
 
 __device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
@@ -162,7 +166,7 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
       }
       bool hit[RPL];
       long long v[RPL];
-      probe_rows(K, htp, P.ht, k, p, hit, v);
+      probe_rows(K, htp[P.ht], P.ht, k, p, hit, v);
 #pragma unroll
       for (int j = 0; j < RPL; j++) {
         if (P.kind == P_MARK) {
@@ -338,6 +342,17 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   long long acc[MAXA] = {0, 0, 0, 0};
   int qhead = 0, qcount = 0;
   uint32_t slot = 0, phase = 0;
+#ifdef GPL_JIT
+  // stage-phase probe tables' parameters live in registers for the kernel's
+  // lifetime (the specialised kernel has registers to spare; the generic one
+  // reads them from shared memory)
+  HTP hsp[MAXSP];
+#pragma unroll
+  for (int sp = 0; sp < MAXSP; sp++) hsp[sp] = htp[sp < K.nsprobe ? K.probe[sp].ht : 0];
+#define GPL_SP_HTP(sp) hsp[sp]
+#else
+#define GPL_SP_HTP(sp) htp[K.probe[sp].ht]
+#endif
   for (;;) {
     mbar_wait(&full[slot], phase);
     const int4 h = hdr[slot];
@@ -383,7 +398,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             }
             bool hit[RPL];
             long long v[RPL];
-            probe_rows(K, htp, P.ht, k, p, hit, v);
+            probe_rows(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v);
 #pragma unroll
             for (int j = 0; j < RPL; j++) {
               if (P.kind == P_MARK) {
