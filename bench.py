@@ -290,7 +290,9 @@ def main():
     # e2e: same step through the C ABI from pinned host buffers (H2D inside the timed region)
     e2e = None
     if not args.no_e2e:
-        pinned = {t: {c: torch.from_numpy(a).pin_memory() for c, a in cols.items()} for t, cols in db.tables.items()}
+        # the columns the plan reads (what a user of the API loads for this query)
+        need = queries.plan_columns(text)
+        pinned = {t: {c: torch.from_numpy(db.tables[t][c]).pin_memory() for c in cs} for t, cs in need.items()}
         h2d = sum(v.numel() * v.element_size() for cols in pinned.values() for v in cols.values())
         ctx2 = gpl.Context(local, stream=stream)
 
@@ -368,7 +370,7 @@ def main():
         "op_pass": stats["op_pass"],
         "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
         "jit": stats.get("jit"),
-        "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm")}
+        "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split")}
                      if tuned else None),
     }
     if rank == 0:

@@ -7,8 +7,9 @@ config 2 (tile sweep, §5.2 Figs 12-13, Eq 10): the fused kernel's
   identical at every Δ (checked).
 config 5 (fused vs KBE, §2.2 Obs 1 / §5.3.2 Figs 3, 16-18): Q14 with shipdate
   windows giving ~1-100% selectivity, Q5 and Q9-wide at SF 10: kernel/step
-  latency of the fused pipeline and of the kernel-at-a-time materialising
-  baseline, and the intermediate bytes materialised, normalised to input.
+  latency of the fused pipeline, of the kernel-at-a-time materialising
+  baseline (KBE) and of GPL (w/o CE) (KBE kernels run tile by tile, Fig 16),
+  and the intermediate bytes materialised, normalised to input.
 
 Both print one JSON line and write the full table to --out.
 """
@@ -115,7 +116,8 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
     for name, q, params in cases:
         segs = queries.segments(queries.plan_text(q, db, params))
 
-        def timed(kbe):
+        def timed(kbe, kbe_tile=0):
+            ctx.set_option("kbe_tile_rows", kbe_tile)
             ts, r = [], None
             for i in range(reps + 1):
                 for s in segs[:-1]:
@@ -130,15 +132,22 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
                 r = ctx.fetch_result()
                 if i >= 1:
                     ts.append(ev0.elapsed_time(ev1))
+            ctx.set_option("kbe_tile_rows", 0)
             return statistics.median(ts), r
         tf, rf = timed(False)
         tk, rk = timed(True)
-        assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs), name
+        # GPL (w/o CE): the KBE kernels tile by tile, with the
+        # paper's default 1 MB tile in rows of this query's scan width
+        bpr = max(1, int(rf.stats["bytes_scanned"] / max(1, rf.stats["rows_scanned"])))
+        tw, rw = timed(True, (1 << 20) // bpr)
+        assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs) == (rw.keys, rw.aggs), name
         inp = rf.stats["bytes_scanned"]
         ops = rf.stats["op_pass"]
         sel = (ops[0] / rf.stats["rows_scanned"]) if q == "Q14" and ops else None
         rows.append({"case": name, "selectivity": sel, "input_bytes": inp,
                      "fused_ms": tf, "kbe_ms": tk, "speedup": tk / tf,
+                     "wo_ce_ms": tw, "wo_ce_tile_rows": rw.stats["tile_rows_used"],
+                     "wo_ce_over_kbe": tw / tk, "wo_ce_intermediate_bytes": rw.stats["intermediate_bytes"],
                      "fused_intermediate_bytes": rf.stats["intermediate_bytes"],
                      "kbe_intermediate_bytes": rk.stats["intermediate_bytes"],
                      "kbe_intermediate_over_input": rk.stats["intermediate_bytes"] / inp,

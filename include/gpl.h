@@ -115,6 +115,8 @@ typedef struct {
   int32_t ctas_per_sm;
   int32_t candidates;          /* gpl_autotune: shapes measured                                    */
   double measured_ms;          /* gpl_autotune: median kernel time of the chosen shape            */
+  int32_t probe_split;         /* probes run before the survivor queue (autotune: measured best)  */
+  int32_t pad_;
 } gpl_model_report;
 
 /* Create a context on CUDA device `device` enqueuing on `cuda_stream` (a
@@ -177,7 +179,11 @@ gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_rows);
  * output cardinality to size the next buffers (so this call synchronises).
  * Same result contract (bit-identical results); stats.kbe = 1 and
  * stats.intermediate_bytes = bytes materialised between operators (flags,
- * positions, payload and compacted columns). For comparison only (config 5). */
+ * positions, payload and compacted columns). For comparison only (config 5).
+ * With option "kbe_tile_rows" = T > 0 the same sequence runs tile by tile
+ * (T rows at a time, materialising per tile): the paper's GPL (w/o CE)
+ * variant, tiling without concurrent kernels or channels (P:337, P:382,
+ * P:564); stats.tile_rows_used = T. */
 gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment);
 
 /* Synchronise the stream and return the last run's result (host decode of
@@ -217,7 +223,8 @@ gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t
 /* Calibrate the pipeline shape of a query by measurement (the paper profiles
  * the first tile and then searches its model): runs the plan's
  * build segments, takes the A9 model's best configuration for every
- * (CTAs per SM, stage rows) shape (at most max_candidates), times each on the
+ * (CTAs per SM, stage rows) shape (at most max_candidates) under every probe
+ * split (how many probes run before the survivor queue), times each on the
  * device with L2 flushed (median of 3), and pins the fastest for this probe
  * segment; later gpl_run_plan / gpl_run_query calls with tile_rows = 0 use
  * it until gpl_set_option is called. Synchronises. out (optional) receives
@@ -226,7 +233,10 @@ gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_candidates, 
 
 /* Tuning knobs (tests / sweeps): "stage_rows", "ring_depth",
  * "consumer_warps", "ctas_per_sm", "probe_split" (-1 = auto), "hash_load_pct",
- * "jit" (1 = plan-specialised kernels, default; 0 = generic kernel).
+ * "jit" (1 = plan-specialised kernels, default; 0 = generic kernel),
+ * "build_pipeline" (1 = DIRECT build segments run through the fused pipeline
+ * with an insert sink, default; 0 = the standalone build kernels),
+ * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input).
  * value < 0 restores automatic selection. */
 gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value);
 
@@ -239,7 +249,9 @@ gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment);
  * the A9 configuration for tile_rows. On a host-only context it compiles
  * without loading (a build check). GPL_E_STATE if NVRTC is unavailable or
  * the compile fails (message in gpl_last_error); gpl_run_plan then uses the
- * generic precompiled kernel. Disable with gpl_set_option("jit", 0). */
+ * generic precompiled kernel. Disable with gpl_set_option("jit", 0).
+ * A build segment is accepted too: a DIRECT build compiles its pipelined
+ * (insert-sink) kernel; other builds use precompiled kernels (no-op). */
 gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows);
 
 /* Message of the last failed call on ctx (ctx-owned, valid until the next

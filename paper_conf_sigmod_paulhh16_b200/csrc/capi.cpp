@@ -4,6 +4,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <climits>
 #include <cstring>
 #include <new>
@@ -52,12 +55,17 @@ int type_width(int t) {
 //   words 18..      int128 partials [groups][aggs] (zeroed per run)
 constexpr int kScratchHead = 2 + MAXOPS;
 constexpr size_t kMaxPartialBytes = (size_t)(1 << 16) * MAXA * 16;
-constexpr size_t kScratchBytes = kScratchHead * 8 + kMaxPartialBytes;
+constexpr size_t kScratchBytes = kScratchHead * 8 + kMaxPartialBytes + MAXOPS * 8;  // + build op counters
 
 unsigned int* err_ptr(gpl_ctx* ctx) { return (unsigned int*)ctx->d_scratch; }
 unsigned long long* counter_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 1; }
 unsigned long long* op_pass_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 2; }
 unsigned long long* partials_ptr(gpl_ctx* ctx) { return ctx->d_scratch + kScratchHead; }
+// op counters of pipelined builds (written, never read)
+unsigned long long* build_ops_ptr(gpl_ctx* ctx) { return ctx->d_scratch + kScratchHead + kMaxPartialBytes / 8; }
+// a DIRECT table's pipelined build keeps its tile counter right after the
+// cells, so the one memset that clears the table also resets the counter
+size_t direct_counter_off(size_t bytes) { return (bytes + 15) / 16 * 16; }
 
 gpl_status check_dev(gpl_ctx* ctx) {
   if (!ctx) return GPL_E_ARG;
@@ -73,9 +81,10 @@ void free_column(gpl_ctx* ctx, Column& c) {
 
 // Read latched device error bits (syncs) and clear them.
 gpl_status take_device_errors(gpl_ctx* ctx) {
-  unsigned int bits = 0;
-  CK(cudaMemcpyAsync(&bits, err_ptr(ctx), sizeof(bits), cudaMemcpyDeviceToHost, ctx->stream));
+  // pinned destination: a pageable D2H costs ~10 us more than the copy itself
+  CK(cudaMemcpyAsync(ctx->h_err, err_ptr(ctx), sizeof(unsigned int), cudaMemcpyDeviceToHost, ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
+  const unsigned int bits = *ctx->h_err;
   if (bits) {
     CK(cudaMemsetAsync(err_ptr(ctx), 0, sizeof(unsigned int), ctx->stream));
     if (bits & ERR_DUPKEY) return fail(ctx, GPL_E_DUPKEY, "duplicate build key (joins must be FK->PK)");
@@ -158,6 +167,7 @@ GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
   if ((e = cudaMemset(ctx->d_scratch, 0, kScratchBytes)) != cudaSuccess) return bad(e, "scratch");
   if ((e = cudaMallocHost(&ctx->h_stage, kScratchBytes)) != cudaSuccess) return bad(e, "pinned staging");
   ctx->h_stage_cap = kScratchBytes;
+  if ((e = cudaMallocHost((void**)&ctx->h_err, 64)) != cudaSuccess) return bad(e, "pinned error word");
   if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
   if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
   *out = ctx;
@@ -178,6 +188,7 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     if (ctx->d_scratch) cudaFree(ctx->d_scratch);
     for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
     if (ctx->h_stage) cudaFreeHost(ctx->h_stage);
+    if (ctx->h_err) cudaFreeHost(ctx->h_err);
     if (ctx->d_minmax) cudaFree(ctx->d_minmax);
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
@@ -209,6 +220,11 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "hash_load_pct") {
     if (v >= 0 && (v < 10 || v > 90)) return fail(ctx, GPL_E_ARG, "hash_load_pct in [10, 90]");
     o.hash_load_pct = v;
+  } else if (k == "kbe_tile_rows") {
+    if (v < 0) return fail(ctx, GPL_E_ARG, "kbe_tile_rows >= 0 (0 = whole input: KBE)");
+    o.kbe_tile_rows = v;
+  } else if (k == "build_pipeline") {
+    o.build_pipeline = v != 0 ? 1 : 0;
   } else if (k == "jit") {
     o.jit = v != 0 ? 1 : 0;
   } else if (k == "hbm_mbs") {
@@ -323,7 +339,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       t.cols.push_back(c);
       CK(launch_minmax(c.dev, c.width, nrows, ctx->d_minmax + 2 * i, ctx->stream));
     }
-    long long mm[128];
+    long long* mm = (long long*)ctx->h_stage;  // pinned (fetches re-copy their own results)
     CK(cudaMemcpyAsync(mm, ctx->d_minmax, sizeof(long long) * 2 * ncols, cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     for (int i = 0; i < ncols; i++) {
@@ -405,6 +421,32 @@ static cudaError_t record_event(gpl_ctx* ctx, cudaEvent_t ev) {
   return cudaEventRecord(ev, ctx->stream);
 }
 
+// A DIRECT build segment lowered to the fused pipeline with an insert sink
+// (shape + schedule; the caller fills the run-time pointers).
+static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTable& H, PipeDesc* pd, Config* cfg) {
+  LowerInfo li;
+  std::string err;
+  gpl_status st;
+  if ((st = lower_probe(ctx, s, choose_split(ctx, s), pd, &li, &err, &H))) return fail(ctx, st, err);
+  for (int i = 0; i < pd->nht; i++) {
+    const HashTable& h = ctx->hts[li.ht_ids[i]];
+    li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+  }
+  if (!choose_config(ctx, *pd, li, pd->nrows, 0, cfg, &err)) return fail(ctx, GPL_E_ARG, err);
+  apply_config(pd, li, *cfg);
+  return GPL_OK;
+}
+
+static gpl_status launch_prepared_build(gpl_ctx* ctx, const PreparedBuild& P) {
+  if (P.pipe) {
+    CK(cudaMemsetAsync(P.pdesc.ins_slots, 0, P.clear_bytes, ctx->stream));
+    CK(launch_pipeline_fn(P.pfn, P.pdesc, P.pgrid, ctx->stream));
+  } else {
+    CK(launch_build(P.desc, P.trivial, P.known, ctx->sms, ctx->stream));
+  }
+  return GPL_OK;
+}
+
 GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32_t* ht_id) {
   if (!ctx || !build_segment) return GPL_E_ARG;
   ctx->err.clear();
@@ -416,7 +458,7 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
       if (build_cache_valid(ctx, P)) {
         gpl_status st = check_dev(ctx);
         if (st) return st;
-        CK(launch_build(P.desc, P.trivial, P.known, ctx->sms, ctx->stream));
+        if ((st = launch_prepared_build(ctx, P))) return st;
         ctx->hts[P.ht_index].valid = true;
         if (ht_id) *ht_id = P.ht_index;
         return GPL_OK;
@@ -462,7 +504,8 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
   }
   HashTable& H = ctx->hts[idx];
   // rounded to 256 B: kernels stage small tables with 16-B vector loads
-  const size_t need = (std::max<size_t>(shape.bytes(), 16) + 255) / 256 * 256;
+  // (+16: the pipelined build's tile counter after DIRECT cells)
+  const size_t need = (std::max<size_t>(shape.bytes(), 16) + 16 + 255) / 256 * 256;
   if (!H.slots || H.alloc_bytes < need) {
     CK(cudaStreamSynchronize(ctx->stream));
     if (H.slots) cudaFree(H.slots);
@@ -509,11 +552,32 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
     }
     known = trivial_header(T.nrows, kmin, kmax, H.cap_slots, d.load_pct);
   }
-  CK(launch_build(d, trivial, known, ctx->sms, ctx->stream));
+  PreparedBuild P;
+  if (H.kind == HT_DIRECT && ctx->opt.build_pipeline) {
+    // the build segment as a pipeline: scan -> filters -> probes -> insert sink
+    PipeDesc pd;
+    Config cfg;
+    if ((st = lower_build_pipe(ctx, s, H, &pd, &cfg))) return st;
+    pd.ins_slots = H.slots;
+    pd.tile_counter = (unsigned long long*)((char*)H.slots + direct_counter_off(H.bytes()));
+    pd.op_pass = build_ops_ptr(ctx);
+    pd.err = err_ptr(ctx);
+    pd.partials = partials_ptr(ctx);  // no aggregates: never written
+    std::string jerr;
+    P.pfn = resolve_pipeline_fn(pd, ctx->opt.jit != 0, &jerr);
+    if (!P.pfn) return fail(ctx, GPL_E_CUDA, "cannot configure the pipelined build kernel");
+    P.pipe = true;
+    P.pdesc = pd;
+    P.pgrid = cfg.grid;
+    P.clear_bytes = direct_counter_off(H.bytes()) + 16;
+  }
+  P.desc = d;
+  P.trivial = trivial;
+  P.known = known;
+  if ((st = launch_prepared_build(ctx, P))) return st;
   H.valid = true;
   if (ht_id) *ht_id = H.id;
   // invalidate prepared builds/runs that referenced this table's old shape
-  PreparedBuild P;
   P.desc = d;
   P.shape = shape;
   P.trivial = trivial;
@@ -540,7 +604,11 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
   if (!parse_segment(text, seg, &err)) return fail(ctx, GPL_E_PLAN, err);
   if (seg->is_build) return fail(ctx, GPL_E_PLAN, "expected a probe segment ('run TABLE')");
   if (force_split >= 0) seg->split_hint = force_split;
-  gpl_status st = lower_probe(ctx, *seg, force_split >= 0 ? force_split : choose_split(ctx, *seg), d, li, &err);
+  auto tu0 = tile_rows == 0 && force_split < 0 ? ctx->tuned.find(seg->text) : ctx->tuned.end();
+  const int split = force_split >= 0 ? force_split
+                    : (tu0 != ctx->tuned.end() && tu0->second.split >= 0) ? tu0->second.split
+                                                                          : choose_split(ctx, *seg);
+  gpl_status st = lower_probe(ctx, *seg, split, d, li, &err);
   if (st) return fail(ctx, st, err);
   auto lit = ctx->lambda.find(seg->text);
   if (lit != ctx->lambda.end()) li->lambda = lit->second;
@@ -699,8 +767,17 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
   };
   auto g = ctx->graphs.find(key);
   if (g != ctx->graphs.end()) {
+    static const bool trace = std::getenv("GPL_TRACE_HOST") != nullptr;
+    const auto t0 = std::chrono::steady_clock::now();
     if (all_valid()) {
+      const auto t1 = std::chrono::steady_clock::now();
       CK(cudaGraphLaunch(g->second, ctx->stream));
+      if (trace) {
+        const auto t2 = std::chrono::steady_clock::now();
+        std::fprintf(stderr, "gpl_run_query host: validate %.1f us, cudaGraphLaunch %.1f us\n",
+                     std::chrono::duration<double, std::micro>(t1 - t0).count(),
+                     std::chrono::duration<double, std::micro>(t2 - t1).count());
+      }
       // the run's bookkeeping is the cached plan's
       const std::shared_ptr<PreparedRun>& PP = ctx->run_cache[run_key];
       const PreparedRun& P = *PP;
@@ -765,24 +842,47 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   tmp.cap_groups = 0;
   gpl_fetch_result(ctx, &tmp);  // records λ; capacity errors are irrelevant here
   ctx->err.clear();
-  // the model's shortlist
+  // the model's shortlist, for the heuristic's probe split and every other
+  // split (how many probes run before the survivor queue)
   Segment seg;
   std::string err;
   if (!parse_segment(probe, &seg, &err)) return fail(ctx, GPL_E_PLAN, err);
   PipeDesc d;
   LowerInfo li;
-  if ((st = lower_probe(ctx, seg, choose_split(ctx, seg), &d, &li, &err))) return fail(ctx, st, err);
-  auto lit = ctx->lambda.find(seg.text);
-  if (lit != ctx->lambda.end()) li.lambda = lit->second;
-  for (int i = 0; i < d.nht; i++) {
-    const HashTable& h = ctx->hts[li.ht_ids[i]];
-    li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
-  }
-  Config best_model;
-  std::vector<Config> cands;
+  const int split0 = choose_split(ctx, seg);
+  std::vector<int> splits{split0};
+  if (seg.split_hint < -1 && ctx->opt.probe_split < -1)
+    for (int sp = 0; sp <= std::min<int>((int)seg.probes.size(), MAXSP); sp++)
+      if (sp != split0) splits.push_back(sp);
+  std::vector<std::pair<int, Config>> cands;
   ctx->tuned.erase(seg.text);
-  if (!choose_config(ctx, d, li, d.nrows, 0, &best_model, &err, &cands)) return fail(ctx, GPL_E_ARG, err);
-  if (max_candidates > 0 && (int)cands.size() > max_candidates) cands.resize(max_candidates);
+  for (int sp : splits) {
+    PipeDesc ds;
+    LowerInfo ls;
+    if ((st = lower_probe(ctx, seg, sp, &ds, &ls, &err))) {
+      if (sp == split0) return fail(ctx, st, err);
+      st = GPL_OK;
+      continue;
+    }
+    auto lit = ctx->lambda.find(seg.text);
+    if (lit != ctx->lambda.end()) ls.lambda = lit->second;
+    for (int i = 0; i < ds.nht; i++) {
+      const HashTable& h = ctx->hts[ls.ht_ids[i]];
+      ls.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+    }
+    Config best_model;
+    std::vector<Config> cs;
+    if (!choose_config(ctx, ds, ls, ds.nrows, 0, &best_model, &err, &cs)) {
+      if (sp == split0) return fail(ctx, GPL_E_ARG, err);
+      continue;
+    }
+    if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
+    for (const Config& c : cs) cands.push_back({sp, c});
+    if (sp == split0) {
+      d = ds;
+      li = ls;
+    }
+  }
   // L2 flush buffer (2x L2) so every timing starts cold, as the bench does
   void* flush = nullptr;
   const size_t fbytes = (size_t)2 * ctx->l2_bytes;
@@ -790,8 +890,9 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   double best_ms = 1e300;
   TunedShape best;
   int tried = 0;
-  for (const Config& c : cands) {
-    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm};
+  for (const auto& sc : cands) {
+    const Config& c = sc.second;
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sc.first};
     ctx->tuned[seg.text] = t;
     ctx->run_cache.erase(probe + "\x1f" + std::to_string(0));
     std::vector<float> ms;
@@ -846,6 +947,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     out->ctas_per_sm = c.ctas_per_sm;
     out->candidates = tried;
     out->measured_ms = best_ms;
+    out->probe_split = best.split >= 0 ? best.split : split0;
   }
   return GPL_OK;
 }
@@ -858,8 +960,18 @@ GPL_API gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int
   Config cfg;
   Segment seg;
   gpl_status st;
-  if ((st = prepare_run(ctx, probe_segment, tile_rows, &d, &li, &cfg, &seg))) return st;
   std::string err;
+  if (!parse_segment(probe_segment, &seg, &err)) return fail(ctx, GPL_E_PLAN, err);
+  if (seg.is_build) {  // the pipelined build of a DIRECT table (others use the precompiled build kernels)
+    BuildDesc bd;
+    HashTable shape;
+    bool trivial = false;
+    if ((st = lower_build(ctx, seg, &bd, &shape, &trivial, &err))) return fail(ctx, st, err);
+    if (shape.kind != HT_DIRECT || !ctx->opt.build_pipeline) return GPL_OK;
+    if ((st = lower_build_pipe(ctx, seg, shape, &d, &cfg))) return st;
+  } else if ((st = prepare_run(ctx, probe_segment, tile_rows, &d, &li, &cfg, &seg))) {
+    return st;
+  }
   if (!ctx->host_only && (st = check_dev(ctx))) return st;
   if (!jit_prepare(d, !ctx->host_only, &err)) return fail(ctx, GPL_E_STATE, err);
   return GPL_OK;
@@ -883,7 +995,13 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   d.err = err_ptr(ctx);
   CK(cudaMemsetAsync(counter_ptr(ctx), 0, (1 + MAXOPS) * sizeof(unsigned long long) + pbytes, ctx->stream));
   double inter = 0;
-  const size_t need = kbe_pool_bytes(d);
+  // GPL (w/o CE): the same kernel-at-a-time sequence, one tile
+  // of kbe_tile_rows at a time (tiling without concurrency or channels)
+  const int64_t tile = ctx->opt.kbe_tile_rows > 0 ? std::min<int64_t>(ctx->opt.kbe_tile_rows, std::max<long long>(d.nrows, 1))
+                                                   : std::max<long long>(d.nrows, 1);
+  PipeDesc dt = d;
+  dt.nrows = tile;
+  const size_t need = kbe_pool_bytes(dt);
   if (ctx->kbe_cap < need) {
     CK(cudaStreamSynchronize(ctx->stream));
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
@@ -894,7 +1012,15 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
     ctx->kbe_cap = need;
   }
   CK(cudaEventRecord(ctx->ev0, ctx->stream));
-  CK(run_kbe(d, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &inter));
+  for (long long r0 = 0; r0 < d.nrows || (r0 == 0 && d.nrows == 0); r0 += tile) {
+    dt = d;
+    dt.nrows = std::min<long long>(tile, d.nrows - r0);
+    for (int c = 0; c < d.ncols; c++) dt.col[c] = d.col[c] + r0 * d.colw[c];
+    double tb = 0;
+    CK(run_kbe(dt, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &tb));
+    inter += tb;
+    if (d.nrows == 0) break;
+  }
   CK(cudaEventRecord(ctx->ev1, ctx->stream));
   LastRun& L = ctx->last;
   L.valid = true;
@@ -916,6 +1042,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   S.agg_mode = AGG_GLOBAL;
   S.kbe = 1;
   S.intermediate_bytes = inter;
+  S.tile_rows_used = ctx->opt.kbe_tile_rows > 0 ? tile : 0;
   return GPL_OK;
 }
 
@@ -1039,5 +1166,6 @@ GPL_API gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment,
   out->smem_bytes = c.smem;
   out->feasible = c.feasible;
   out->ctas_per_sm = c.ctas_per_sm;
+  out->probe_split = d.nsprobe;
   return GPL_OK;
 }

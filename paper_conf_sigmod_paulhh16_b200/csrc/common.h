@@ -120,6 +120,7 @@ struct Agg {
   int64_t c;
 };
 enum : int32_t { AGG_REG = 0, AGG_SMEM = 1, AGG_GLOBAL = 2 };
+enum : int32_t { SINK_AGG = 0, SINK_INSERT = 1 };
 
 // ---- survivor-queue push: field <- stage column, stage-phase probe slot, or
 // a value term computed in the stage phase (expression pushdown)
@@ -164,6 +165,14 @@ struct PipeDesc {
   int32_t smem_tables_bytes;
   // smem layout
   int32_t off_queue, off_agg, off_ring, smem_bytes;
+  // sink: SINK_AGG (probe segment: group-by aggregation) or SINK_INSERT (build
+  // segment run through the same pipeline: insert key -> payload into a DIRECT
+  // table; the blocking hash build of P:147 as the segment's last operator)
+  int32_t sink;
+  int32_t ins_kfield, ins_pfield, ins_ptransform, ins_width;  // queue fields, G_ID/G_YEAR, cell bytes (0 = bitmap)
+  long long ins_kmin, ins_pay_base;                            // run-time (table bases)
+  unsigned long long ins_nslots;
+  void* ins_slots;
   // outputs
   unsigned long long* partials;      // [ngroups_total][nagg] x (lo, hi)
   unsigned long long* tile_counter;  // zeroed before launch

@@ -213,16 +213,20 @@ int choose_split(const gpl_ctx* ctx, const Segment& s) {
   if (ctx->opt.probe_split >= -1) return ctx->opt.probe_split < 0 ? (int)s.probes.size() : (int)ctx->opt.probe_split;
   const int np = (int)s.probes.size(), nf = (int)s.filters.size();
   auto it = ctx->lambda.find(s.text);
+  // Stage-phase probes read their keys straight from the staged tile with all
+  // RPL loads of a lane in flight; queue-phase probes first pay the survivor
+  // queue's smem writes and reads. Measured on B200 (SF 20, Q5/Q7/Q8 with the
+  // clustered HT_O probe first): running every probe (up to MAXSP) in the stage
+  // phase is fastest even at 3-30% survival, so the queue is entered before a
+  // probe only when the filters alone already drop >= 95% of the rows (Q14).
+  // gpl_autotune measures every split and pins the best.
   if (it != ctx->lambda.end() && (int)it->second.size() >= nf + np) {
-    // earliest point whose cumulative pass fraction drops to <= 1/2
     const std::vector<double>& lam = it->second;
-    double after_filters = nf ? lam[nf - 1] : 1.0;
-    if (after_filters <= 0.5) return 0;
-    for (int p = 0; p < np; p++)
-      if (lam[nf + p] <= 0.5) return p + 1;
-    return np;
+    const double after_filters = nf ? lam[nf - 1] : 1.0;
+    if (after_filters <= 0.05) return 0;
+    return std::min(np, MAXSP);
   }
-  return nf ? 0 : std::min(1, np);
+  return nf ? 0 : std::min(np, MAXSP);
 }
 
 }  // namespace gpl

@@ -109,18 +109,27 @@ struct PreparedBuild {
   std::string name, table;
   uint64_t table_version = 0, opt_version = 0;
   std::vector<int> src_ids;
+  // DIRECT builds run through the fused pipeline with an insert sink
+  bool pipe = false;
+  PipeDesc pdesc{};
+  const void* pfn = nullptr;
+  int pgrid = 0;
+  size_t clear_bytes = 0;  // table cells + the trailing tile counter
 };
 
 // gpl_autotune's pinned pipeline shape for one probe segment
 struct TunedShape {
   int64_t tile_rows = 0;
   int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1;
+  int split = -2;  // probes run in the stage phase (-2: the heuristic's)
 };
 
 struct Options {
   int64_t stage_rows = -1, ring_depth = -1, consumer_warps = -1, ctas_per_sm = -1, probe_split = -2,
           hash_load_pct = -1;
   int64_t jit = 1;
+  int64_t build_pipeline = 1;
+  int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
   double hbm_gbs = -1;
 };
 
@@ -158,6 +167,7 @@ struct gpl_ctx {
   std::map<std::string, gpl::TunedShape> tuned;  // probe segment text -> measured-best shape
   std::map<std::string, std::vector<std::string>> plan_segs;  // gpl_run_query: plan text -> segments
   void* h_stage = nullptr;  // pinned host staging for one packed D2H of results
+  unsigned int* h_err = nullptr;  // pinned word for error-bit reads (gpl_sync)
   size_t h_stage_cap = 0;
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;

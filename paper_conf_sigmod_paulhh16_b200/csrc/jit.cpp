@@ -160,6 +160,11 @@ std::string shape_source(const PipeDesc& d) {
       << "].width = " << d.ht[h].width << "; k.ht_smem_off[" << h << "] = " << d.ht_smem_off[h] << "; k.ht_smem_bytes["
       << h << "] = " << d.ht_smem_bytes[h] << ";\n";
   for (int h = d.nht; h < MAXHT; h++) o << "  k.ht_smem_off[" << h << "] = -1;\n";
+  I("sink", d.sink);
+  I("ins_kfield", d.ins_kfield);
+  I("ins_pfield", d.ins_pfield);
+  I("ins_ptransform", d.ins_ptransform);
+  I("ins_width", d.ins_width);
   I("smem_tables_bytes", d.smem_tables_bytes);
   I("off_queue", d.off_queue);
   I("off_agg", d.off_agg);

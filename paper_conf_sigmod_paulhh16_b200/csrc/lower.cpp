@@ -195,10 +195,15 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
   return GPL_OK;
 }
 
-gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, LowerInfo* li, std::string* err) {
+gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, LowerInfo* li, std::string* err,
+                       const HashTable* ins) {
   *d = PipeDesc{};
   *li = LowerInfo{};
-  if (s.is_build) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
+  if (s.is_build && !ins) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
+  if (ins && (!s.is_build || ins->kind != HT_DIRECT || s.key.size() != 1)) {
+    *err = "pipelined build needs a single-key DIRECT build segment";
+    return GPL_E_PLAN;
+  }
   auto tit = ctx->tables.find(s.table);
   if (tit == ctx->tables.end()) { *err = "unknown table '" + s.table + "'"; return GPL_E_STATE; }
   const Table& T = tit->second;
@@ -300,6 +305,12 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   }
   for (auto& a : s.aggs)
     if (a.kind >= A_SUMIF && !slot_of.count(a.slot)) { *err = "agg condition refers to unknown slot '" + a.slot + "'"; return GPL_E_PLAN; }
+  const bool pay_slot = ins && ins->has_payload && slot_of.count(s.payload.name);
+  if (ins) {  // build key and payload columns are staged too
+    if ((st = stage(s.key[0], &tmp))) return st;
+    if (!is_int32(*cols[tmp])) { *err = "build keys must be 32-bit columns"; return GPL_E_PLAN; }
+    if (ins->has_payload && !pay_slot && (st = stage(s.payload.name, &tmp))) return st;
+  }
 
   // split (probes run before the survivor queue)
   int sp = split;
@@ -346,6 +357,13 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
         if (f.x.kind != RefIR::CONST && slot_of.count(f.x.name)) used_slots.insert(f.x.name);
   for (auto& a : s.aggs)
     if (a.kind >= A_SUMIF) used_slots.insert(a.slot);
+  if (ins) {
+    need_col(s.key[0]);
+    if (ins->has_payload) {
+      if (pay_slot) used_slots.insert(s.payload.name);
+      else need_col(s.payload.name);
+    }
+  }
 
   auto slot_width = [&](int p) { return (s.probes[p].kind != P_MARK && pht[p]->kind == HT_MAP64) ? 8 : 4; };
   std::map<std::string, int> field;
@@ -395,6 +413,16 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->qbytes = std::max(off, 16);
   }
 
+  if (ins) {
+    d->sink = SINK_INSERT;
+    d->ins_kfield = field[s.key[0]];
+    d->ins_pfield = ins->has_payload ? field[s.payload.name] : -1;
+    d->ins_ptransform = ins->has_payload && s.payload.kind == RefIR::YEARCOL ? G_YEAR : G_ID;
+    d->ins_width = ins->width;
+    d->ins_kmin = ins->dkmin;
+    d->ins_nslots = ins->dnslots;
+    d->ins_pay_base = ins->pay_base;
+  }
   // slot value ranges (validator)
   auto slot_range = [&](const std::string& n) -> Range {
     int p = slot_of[n];

@@ -13,7 +13,10 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
 
 // Probe segment -> PipeDesc (everything but the schedule/smem layout) + facts.
 // split: probes executed before the survivor queue (-1 = auto heuristic).
-gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, LowerInfo* li, std::string* err);
+// With `ins` (the DIRECT table shape lower_build chose), a build segment is
+// lowered to the same pipeline with an insert sink (SINK_INSERT).
+gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, LowerInfo* li, std::string* err,
+                       const HashTable* ins = nullptr);
 
 // Host computation of the header of a trivial build (all rows inserted).
 HTHeader trivial_header(int64_t count, long long kmin, long long kmax, int64_t cap_slots, int load_pct);

@@ -206,6 +206,40 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
     if (lane == 0) cnt[op] += c;
   }
   if (!__any_sync(0xffffffffu, any4(p))) return;
+  if (K.sink == SINK_INSERT) {
+    // build segment: the blocking hash build as the pipeline's last
+    // operator. DIRECT cells start at 0 (= empty): bitmap cells by atomicOr,
+    // 32-bit cells by atomicCAS, 1- and 2-byte cells by atomicOr into their
+    // word; a non-empty old cell is a duplicate key (FK->PK joins only).
+#pragma unroll
+    for (int j = 0; j < RPL; j++) {
+      if (!p[j]) continue;
+      const long long key = (long long)(int32_t)qget(K, qb, K.ins_kfield, idx[j]);
+      const unsigned long long ci = (unsigned long long)(key - d.ins_kmin);
+      if (ci >= d.ins_nslots) {
+        atomicOr(d.err, ERR_CAPACITY);
+        continue;
+      }
+      if (K.ins_width == 0) {
+        const uint32_t bit = 1u << (ci & 31);
+        if (atomicOr((uint32_t*)d.ins_slots + (ci >> 5), bit) & bit) atomicOr(d.err, ERR_DUPKEY);
+        continue;
+      }
+      long long pay = K.ins_pfield >= 0 ? qget(K, qb, K.ins_pfield, idx[j]) : 0;
+      if (K.ins_ptransform == G_YEAR) pay = (int)pay / 10000;
+      const uint32_t v = (uint32_t)(pay - d.ins_pay_base + 1);
+      if (K.ins_width == 4) {
+        if (atomicCAS((uint32_t*)d.ins_slots + ci, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
+      } else {
+        const unsigned long long byte = ci * (unsigned long long)K.ins_width;
+        uint32_t* w = (uint32_t*)((char*)d.ins_slots + (byte & ~3ull));
+        const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
+        const uint32_t m = (K.ins_width == 1 ? 0xFFu : 0xFFFFu) << sh;
+        if (atomicOr(w, v << sh) & m) atomicOr(d.err, ERR_DUPKEY);
+      }
+    }
+    return;
+  }
   unsigned long long* stab = &S<unsigned long long>(K.off_agg);
 #pragma unroll
   for (int j = 0; j < RPL; j++) {

@@ -67,7 +67,7 @@ class _Model(ctypes.Structure):
                 ("t_stream_ms", ctypes.c_double), ("t_probe_ms", ctypes.c_double), ("t_tail_ms", ctypes.c_double),
                 ("t_launch_ms", ctypes.c_double), ("bw_gbs", ctypes.c_double), ("smem_bytes", ctypes.c_int32),
                 ("feasible", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32), ("candidates", ctypes.c_int32),
-                ("measured_ms", ctypes.c_double)]
+                ("measured_ms", ctypes.c_double), ("probe_split", ctypes.c_int32), ("pad_", ctypes.c_int32)]
 
 
 _lib = None

@@ -125,6 +125,27 @@ def segments(text: str) -> list:
     return segs
 
 
+def plan_columns(text: str) -> dict:
+    """{table: [columns]} a plan reads: per segment, the scanned table's columns named in it."""
+    import re
+    need = {}
+    for seg in segments(text):
+        words = re.findall(r"[A-Za-z_][A-Za-z_0-9]*", "\n".join(
+            ln.split("#")[0] for ln in seg.splitlines()))
+        table = None
+        for i, w in enumerate(words):
+            if w in ("scan", "run") and i + 1 < len(words):
+                table = words[i + 1]
+                break
+        if table is None or table not in SCHEMA:
+            continue
+        cols = need.setdefault(table, [])
+        for w in words:
+            if w in SCHEMA[table] and w not in cols:
+                cols.append(w)
+    return need
+
+
 def load_database(ctx: Context, db, tables=None, borrow=False):
     """Load tables (dict of column arrays / tensors) into the context's column store."""
     for t in tables or db.tables.keys():

@@ -218,3 +218,73 @@ def test_autotune_pins_a_measured_shape(ctx):
     assert (r.stats["stage_rows"], r.stats["ring_depth"], r.stats["consumer_warps"]) == \
         (m["stage_rows"], m["ring_depth"], m["consumer_warps"])
     ctx.set_option("stage_rows", -1)  # any option change un-pins
+
+
+@pytest.mark.parametrize("q", QUERIES)
+def test_pipelined_build_matches_build_kernels(ctx, q):
+    """DIRECT build segments run through the fused pipeline with an insert sink
+    (scan -> filter -> probe -> insert); the standalone build
+    kernels are the other path. Both must give the oracle's exact result."""
+    db = tpchgen.generate(0.05, seed=51)
+    o = oracle.run(q, db, _params(q))
+    try:
+        for bp in (1, 0, 1):
+            ctx.set_option("build_pipeline", bp)
+            r = _gpu(ctx, db, q, _params(q))
+            assert r.keys == o.keys and r.aggs == o.aggs, (q, bp)
+    finally:
+        ctx.set_option("build_pipeline", 1)
+
+
+def test_pipelined_build_schedules(ctx):
+    """Build segments under every schedule knob (the knobs apply to build
+    pipelines too): tiny stages, one warp, and each probe split."""
+    db = tpchgen.generate(0.05, seed=52)
+    expect = {q: oracle.run(q, db) for q in ("Q5", "Q8")}
+    knobs = [dict(stage_rows=128, ring_depth=2, consumer_warps=1), dict(probe_split=0), dict(probe_split=1),
+             dict(stage_rows=2048, ring_depth=2, consumer_warps=16)]
+    try:
+        for k in knobs:
+            for key, v in k.items():
+                ctx.set_option(key, v)
+            for q, o in expect.items():
+                r = _gpu(ctx, db, q)
+                assert r.keys == o.keys and r.aggs == o.aggs, (q, k)
+            for key in k:
+                ctx.set_option(key, -1 if key != "probe_split" else -2)
+    finally:
+        for key in ("stage_rows", "ring_depth", "consumer_warps"):
+            ctx.set_option(key, -1)
+        ctx.set_option("probe_split", -2)
+
+
+def test_autotune_split_choice_exact(ctx):
+    """gpl_autotune searches the probe split as well as the shape; the pinned
+    choice keeps results exact and is reported."""
+    db = tpchgen.generate(0.1, seed=43)
+    queries.load_database(ctx, db, queries.TABLES["Q5"])
+    m = ctx.autotune(queries.plan_text("Q5", db))
+    assert 0 <= m["probe_split"] <= 2
+    r = queries.run_query(ctx, "Q5", db)
+    o = oracle.run("Q5", db)
+    assert r.keys == o.keys and r.aggs == o.aggs
+    assert r.stats["probe_split"] == m["probe_split"]
+    ctx.set_option("stage_rows", -1)  # un-pin
+
+
+@pytest.mark.parametrize("q", ["Q5", "Q9", "Q14", "L1"])
+def test_gpl_without_ce_bit_identical(ctx, q):
+    """GPL (w/o CE): the KBE kernel sequence run one tile at a
+    time (ragged last tile) gives the same exact result as the whole-input KBE
+    and the fused pipeline."""
+    db = tpchgen.generate(0.05, seed=22)
+    queries.load_database(ctx, db, queries.TABLES[q])
+    o = oracle.run(q, db, _params(q))
+    try:
+        for tile in (1000, 7777, 1 << 22):
+            ctx.set_option("kbe_tile_rows", tile)
+            r = queries.run_query(ctx, q, db, _params(q), kbe=True)
+            assert r.keys == o.keys and r.aggs == o.aggs, (q, tile)
+            assert r.stats["tile_rows_used"] == min(tile, db.nrows("lineitem"))
+    finally:
+        ctx.set_option("kbe_tile_rows", 0)

@@ -102,15 +102,17 @@ def test_merge_partials_exact():
 
 
 def test_jit_compiles_every_plan():
-    """NVRTC builds the plan-specialised kernel of every paper query (no GPU needed)."""
+    """NVRTC builds the plan-specialised kernels of every paper query — probe segment and
+    pipelined DIRECT builds (no GPU needed)."""
     db = tpchgen.generate(0.01, seed=1)
     ctx = gpl.Context(device=-1)
     queries.load_database(ctx, db)
     for q in queries.QUERIES:
         segs = queries.segments(queries.plan_text(q, db, (19981101,) if q == "L1" else None))
-        for s in segs[:-1]:
-            ctx.build_hash(s)
         try:
+            for s in segs[:-1]:
+                ctx.compile_plan(s)  # DIRECT build segments: the pipeline with an insert sink
+                ctx.build_hash(s)
             ctx.compile_plan(segs[-1])
         except gpl.GplError as e:
             if "NVRTC unavailable" in str(e):
