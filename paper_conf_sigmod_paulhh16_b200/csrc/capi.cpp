@@ -53,6 +53,8 @@ int type_width(int t) {
 //   word 1          tile counter (zeroed per run)
 //   words 2..17     op_pass[MAXOPS]  (zeroed per run)
 //   words 18..      int128 partials [groups][aggs] (zeroed per run)
+// After a fused run a one-CTA kernel copies words [0, head + partials) into
+// mapped pinned host memory (h_stage), so fetching needs no D2H copy node.
 constexpr int kScratchHead = 2 + MAXOPS;
 constexpr size_t kMaxPartialBytes = (size_t)(1 << 16) * MAXA * 16;
 constexpr size_t kScratchBytes = kScratchHead * 8 + kMaxPartialBytes + MAXOPS * 8;  // + build op counters
@@ -60,6 +62,10 @@ constexpr size_t kScratchBytes = kScratchHead * 8 + kMaxPartialBytes + MAXOPS * 
 unsigned int* err_ptr(gpl_ctx* ctx) { return (unsigned int*)ctx->d_scratch; }
 unsigned long long* counter_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 1; }
 unsigned long long* op_pass_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 2; }
+// bytes of the per-run zeroed region (tile counter .. partials)
+size_t run_clear_bytes(size_t pbytes) { return (1 + MAXOPS) * sizeof(unsigned long long) + pbytes; }
+// words the result copy-out moves (error bits, counters, partials)
+int result_words(size_t pbytes) { return kScratchHead + (int)(pbytes / 8); }
 unsigned long long* partials_ptr(gpl_ctx* ctx) { return ctx->d_scratch + kScratchHead; }
 // op counters of pipelined builds (written, never read)
 unsigned long long* build_ops_ptr(gpl_ctx* ctx) { return ctx->d_scratch + kScratchHead + kMaxPartialBytes / 8; }
@@ -167,7 +173,11 @@ GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
   if ((e = cudaMemset(ctx->d_scratch, 0, kScratchBytes)) != cudaSuccess) return bad(e, "scratch");
   if ((e = cudaMallocHost(&ctx->h_stage, kScratchBytes)) != cudaSuccess) return bad(e, "pinned staging");
   ctx->h_stage_cap = kScratchBytes;
+  if ((e = cudaHostGetDevicePointer((void**)&ctx->h_stage_dev, ctx->h_stage, 0)) != cudaSuccess)
+    return bad(e, "mapped staging");
   if ((e = cudaMallocHost((void**)&ctx->h_err, 64)) != cudaSuccess) return bad(e, "pinned error word");
+  if ((e = cudaMallocHost((void**)&ctx->h_minmax, 64 * 2 * sizeof(long long))) != cudaSuccess)
+    return bad(e, "pinned min/max");
   if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
   if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
   *out = ctx;
@@ -189,6 +199,7 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
     if (ctx->h_stage) cudaFreeHost(ctx->h_stage);
     if (ctx->h_err) cudaFreeHost(ctx->h_err);
+    if (ctx->h_minmax) cudaFreeHost(ctx->h_minmax);
     if (ctx->d_minmax) cudaFree(ctx->d_minmax);
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
@@ -215,6 +226,9 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "ctas_per_sm") {
     if (v >= 0 && (v < 1 || v > 4)) return fail(ctx, GPL_E_ARG, "ctas_per_sm in [1, 4]");
     o.ctas_per_sm = v;
+  } else if (k == "packets") {
+    if (v >= 0 && v != 1 && v != 2) return fail(ctx, GPL_E_ARG, "packets: 1 or 2");
+    o.packets = v;
   } else if (k == "probe_split") {
     o.probe_split = v < -1 ? -2 : v;  // -1 = after every probe, >= 0 = count, < -1 auto
   } else if (k == "hash_load_pct") {
@@ -339,7 +353,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       t.cols.push_back(c);
       CK(launch_minmax(c.dev, c.width, nrows, ctx->d_minmax + 2 * i, ctx->stream));
     }
-    long long* mm = (long long*)ctx->h_stage;  // pinned (fetches re-copy their own results)
+    long long* mm = ctx->h_minmax;  // pinned (h_stage holds the last run's copied-out results)
     CK(cudaMemcpyAsync(mm, ctx->d_minmax, sizeof(long long) * 2 * ncols, cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     for (int i = 0; i < ncols; i++) {
@@ -427,7 +441,12 @@ static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTab
   LowerInfo li;
   std::string err;
   gpl_status st;
-  if ((st = lower_probe(ctx, s, choose_split(ctx, s), pd, &li, &err, &H))) return fail(ctx, st, err);
+  // every probe in the stage phase by default: the insert then runs straight
+  // from the staged tile, with no survivor queue (the probe_split option
+  // still applies, e.g. for tests of the queue path)
+  const int split = ctx->opt.probe_split >= -1 || s.split_hint >= -1 ? choose_split(ctx, s)
+                                                                      : std::min<int>((int)s.probes.size(), MAXSP);
+  if ((st = lower_probe(ctx, s, split, pd, &li, &err, &H))) return fail(ctx, st, err);
   for (int i = 0; i < pd->nht; i++) {
     const HashTable& h = ctx->hts[li.ht_ids[i]];
     li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
@@ -622,7 +641,7 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
   if (tu != ctx->tuned.end()) {  // shape pinned by gpl_autotune
     const TunedShape& t = tu->second;
     *cfg = predict(ctx, *d, *li, std::max<int64_t>(d->nrows, 1), t.tile_rows, t.stage_rows, t.depth, t.warps,
-                   t.ctas_per_sm);
+                   t.ctas_per_sm, t.npack);
   } else if (!choose_config(ctx, *d, *li, d->nrows, tile_rows, cfg, &err)) {
     return fail(ctx, GPL_E_ARG, err);
   }
@@ -688,13 +707,15 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   const LowerInfo& li = P->li;
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
   // one memset: tile counter, op_pass and the partials are contiguous
-  CK(cudaMemsetAsync(counter_ptr(ctx), 0, (1 + MAXOPS) * sizeof(unsigned long long) + pbytes, ctx->stream));
+  CK(cudaMemsetAsync(counter_ptr(ctx), 0, run_clear_bytes(pbytes), ctx->stream));
   CK(record_event(ctx, ctx->ev0));
   CK(launch_pipeline_fn(P->fn, d, P->grid, ctx->stream));
   CK(record_event(ctx, ctx->ev1));
+  CK(launch_copyout(ctx->d_scratch, ctx->h_stage_dev, result_words(pbytes), ctx->stream));
   LastRun& L = ctx->last;
   L.valid = true;
   L.kbe = false;
+  L.copied_out = true;
   L.run = ctx->run_cache[std::string(probe_segment) + "\x1f" + std::to_string(tile_rows)];
   L.timed = true;
   gpl_stats& S = L.stats;
@@ -784,6 +805,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       LastRun& L = ctx->last;
       L.valid = true;
       L.kbe = false;
+      L.copied_out = true;
       L.run = PP;
       L.timed = true;
       gpl_stats& S = L.stats;
@@ -807,12 +829,45 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
   }
   // run eagerly (refreshes the prepared caches); once everything is prepared
   // and profiled, record the same sequence as a graph for the next call
+  // the recorded sequence: ONE clear kernel for every DIRECT table of a
+  // pipelined build (cells + tile counter) and the run's counters/partials,
+  // then the build pipelines (other builds: their own kernels) and the fused run
+  auto fused_sequence = [&]() -> gpl_status {
+    ClearList L{};
+    auto add = [&](void* p, size_t b) {
+      if (L.n < 16) {
+        L.ptr[L.n] = p;
+        L.bytes[L.n] = b;
+      }
+      L.n++;
+    };
+    std::vector<const PreparedBuild*> builds;
+    for (size_t i = 0; i + 1 < segs.size(); i++) {
+      const PreparedBuild& B = ctx->build_cache.at(segs[i]);
+      builds.push_back(&B);
+      if (B.pipe) add(B.pdesc.ins_slots, B.clear_bytes);
+    }
+    const PreparedRun& R = *ctx->run_cache.at(run_key);
+    add(counter_ptr(ctx), run_clear_bytes((size_t)R.li.ngroups_total * R.li.nagg * 16));
+    if (L.n > 16) return eager();
+    CK(launch_clear(L, ctx->sms, ctx->stream));
+    for (const PreparedBuild* B : builds) {
+      if (B->pipe) CK(launch_pipeline_fn(B->pfn, B->pdesc, B->pgrid, ctx->stream));
+      else CK(launch_build(B->desc, B->trivial, B->known, ctx->sms, ctx->stream));
+    }
+    CK(record_event(ctx, ctx->ev0));
+    CK(launch_pipeline_fn(R.fn, R.desc, R.grid, ctx->stream));
+    CK(record_event(ctx, ctx->ev1));
+    CK(launch_copyout(ctx->d_scratch, ctx->h_stage_dev,
+                      result_words((size_t)R.li.ngroups_total * R.li.nagg * 16), ctx->stream));
+    return GPL_OK;
+  };
   if ((st = eager())) return st;
   if (all_valid()) {
     const LastRun saved = ctx->last;
     cudaGraph_t graph = nullptr;
     bool ok = cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
-    gpl_status cst = ok ? eager() : GPL_E_CUDA;
+    gpl_status cst = ok ? fused_sequence() : GPL_E_CUDA;
     cudaError_t ce = cudaStreamEndCapture(ctx->stream, &graph);
     ctx->last = saved;
     cudaGraphExec_t exec = nullptr;
@@ -892,7 +947,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   int tried = 0;
   for (const auto& sc : cands) {
     const Config& c = sc.second;
-    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sc.first};
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sc.first, c.npack};
     ctx->tuned[seg.text] = t;
     ctx->run_cache.erase(probe + "\x1f" + std::to_string(0));
     std::vector<float> ms;
@@ -929,7 +984,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   ctx->graphs.clear();
   if (out) {
     const Config c = predict(ctx, d, li, std::max<int64_t>(d.nrows, 1), best.tile_rows, best.stage_rows, best.depth,
-                             best.warps, best.ctas_per_sm);
+                             best.warps, best.ctas_per_sm, best.npack);
     *out = gpl_model_report{};
     out->tile_rows = c.tile_rows;
     out->stage_rows = c.stage_rows;
@@ -993,7 +1048,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   d.tile_counter = counter_ptr(ctx);
   d.op_pass = op_pass_ptr(ctx);
   d.err = err_ptr(ctx);
-  CK(cudaMemsetAsync(counter_ptr(ctx), 0, (1 + MAXOPS) * sizeof(unsigned long long) + pbytes, ctx->stream));
+  CK(cudaMemsetAsync(counter_ptr(ctx), 0, run_clear_bytes(pbytes), ctx->stream));
   double inter = 0;
   // GPL (w/o CE): the same kernel-at-a-time sequence, one tile
   // of kbe_tile_rows at a time (tiling without concurrency or channels)
@@ -1025,6 +1080,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   LastRun& L = ctx->last;
   L.valid = true;
   L.kbe = true;
+  L.copied_out = false;
   {
     auto kr = std::make_shared<PreparedRun>();
     kr->desc = d;
@@ -1063,7 +1119,9 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   const LowerInfo& li = ctx->last.run->li;
   // one D2H: error bits, counter, op_pass and partials are contiguous
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
-  CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
+  // fused runs: the copy-out kernel already wrote the results to h_stage
+  if (!ctx->last.copied_out)
+    CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
   const unsigned long long* hs = (const unsigned long long*)ctx->h_stage;
   const unsigned int bits = (unsigned int)hs[0];

@@ -142,6 +142,7 @@ struct PipeDesc {
   // schedule (A2)
   long long tile_rows;
   int32_t stage_rows, depth, nwarps, flush_each_tile;
+  int32_t npack;  // 128-row packets per consumer iteration (1 or 2: stage-phase probes of both in flight)
   // stage phase (A4 + first probes)
   int32_t nfilt, nsprobe, nprobe, npush;
   Filt filt[MAXF];
@@ -170,6 +171,9 @@ struct PipeDesc {
   // table; the blocking hash build of P:147 as the segment's last operator)
   int32_t sink;
   int32_t ins_kfield, ins_pfield, ins_ptransform, ins_width;  // queue fields, G_ID/G_YEAR, cell bytes (0 = bitmap)
+  // stage-phase insert (every probe in the stage phase): key / payload stage
+  // columns, or the payload's stage-probe slot; ins_kcol < 0: insert from the queue
+  int32_t ins_kcol, ins_pcol, ins_psreg, ins_pad;
   long long ins_kmin, ins_pay_base;                            // run-time (table bases)
   unsigned long long ins_nslots;
   void* ins_slots;

@@ -30,6 +30,7 @@
 #include <algorithm>
 #include <cmath>
 #include <map>
+#include <tuple>
 
 namespace gpl {
 
@@ -54,6 +55,7 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->stage_rows = c.stage_rows;
   d->depth = c.depth;
   d->nwarps = c.warps;
+  d->npack = c.npack;
   d->off_queue = kFixed;
   d->off_agg = align128(kFixed + c.warps * d->qbytes);
   int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
@@ -71,8 +73,9 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
 }
 
 Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t N, int64_t tile,
-               int S, int depth, int W, int k) {
+               int S, int depth, int W, int k, int npack) {
   Config c;
+  c.npack = npack;
   c.tile_rows = tile;
   c.stage_rows = S;
   c.depth = depth;
@@ -84,7 +87,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // threads and registers (<= 80 per thread assumed) of k resident CTAs
   c.feasible = c.smem <= ctx->smem_optin && k * (c.smem + 1024) <= 228 * 1024 && W >= 1 &&
                W <= pipeline_max_consumer_warps() && depth >= 2 && k * (W + 1) * 32 <= 2048 &&
-               k * (W + 1) * 32 * 80 <= 65536;
+               k * (W + 1) * 32 * (npack == 2 ? 112 : 80) <= 65536 && (npack == 1 || npack == 2);
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
   const double b = std::max(1, li.bytes_per_row);
@@ -118,13 +121,17 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   auto lat = [&](int t) {
     if (d.ht_smem_off[t] >= 0) return 40.0;
     const double bytes = li.ht_bytes.empty() ? 1e6 : (double)li.ht_bytes[t];
-    return bytes <= 64e3 ? 80.0 : bytes <= L2_eff ? 500.0 : 1000.0;
+    // calibrated on B200 (Q5 SF 1, ncu: a stage-phase L2 probe keeps a warp
+    // ~1500 cycles per packet; two dies, so half the L2 is far)
+    return bytes <= 64e3 ? 80.0 : bytes <= L2_eff ? 1200.0 : 2000.0;
   };
   double lat_stage = 0, lat_queue = 0;
   for (int p = 0; p < li.nprobe; p++) (p < d.nsprobe ? lat_stage : lat_queue) += lat(li.probe_ht[p]);
-  const double crit = 150.0 + lat_stage + qfrac * lat_queue + instr_iter;  // cycles per warp iteration
-  const double w_eff = (double)std::min(W, S / 128) * k;                   // warps with work per stage
-  const double rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 / crit);  // per SM
+  // cycles per warp iteration of `npack` packets: the stage-phase probe
+  // latency is paid once per iteration (all npack*4 loads of a lane in flight)
+  const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);
+  const double w_eff = (double)std::min(W, S / (128 * npack)) * k;          // warps with work per stage
+  const double rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 * npack / crit);  // per SM
   const double R_cons = rows_cyc * f_sm * b;                                // bytes/s one SM's consumers absorb
   const double t_cons = (double)N / (rows_cyc * f_sm * ctx->sms);
 
@@ -157,12 +164,13 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
 
 bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t N, int64_t tile_req,
                    Config* out, std::string* err, std::vector<Config>* shortlist) {
-  std::map<std::pair<int, int>, Config> per_shape;  // best predicted per (CTAs/SM, stage rows)
+  std::map<std::tuple<int, int, int>, Config> per_shape;  // best predicted per (CTAs/SM, stage rows, packets)
   const Options& o = ctx->opt;
   std::vector<int> Ss = o.stage_rows > 0 ? std::vector<int>{(int)o.stage_rows} : std::vector<int>{512, 1024, 2048, 4096};
   std::vector<int> Ds = o.ring_depth > 0 ? std::vector<int>{(int)o.ring_depth} : std::vector<int>{2, 3, 4, 6};
   std::vector<int> Ws = o.consumer_warps > 0 ? std::vector<int>{(int)o.consumer_warps} : std::vector<int>{4, 8, 12, 16};
   std::vector<int> Ks = o.ctas_per_sm > 0 ? std::vector<int>{(int)o.ctas_per_sm} : std::vector<int>{1, 2};
+  std::vector<int> Ps = o.packets > 0 ? std::vector<int>{(int)o.packets} : std::vector<int>{1, 2};
   Config best;
   bool found = false;
   for (int S : Ss) {
@@ -177,14 +185,15 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
       }
     }
     for (int k : Ks)
+    for (int np : Ps)
     for (int D : Ds)
       for (int W : Ws)
         for (int64_t t : tiles) {
           if (d.flush_each_tile && (long double)(t + QCAP) * std::max<long double>(li.maxabs, 1) >= 4.6e18L) continue;
-          Config c = predict(ctx, d, li, N, t, S, D, W, k);
+          Config c = predict(ctx, d, li, N, t, S, D, W, k, np);
           if (!c.feasible) continue;
           {
-            auto key = std::make_pair(k, S);
+            auto key = std::make_tuple(k, S, np);
             auto it = per_shape.find(key);
             if (it == per_shape.end() || c.pred_ms < it->second.pred_ms) per_shape[key] = c;
           }

@@ -85,6 +85,7 @@ struct LastRun {
   gpl_stats stats{};
   bool timed = false;
   bool kbe = false;
+  bool copied_out = false;  // the run's results were copied to h_stage by the copy-out kernel
 };
 
 struct PreparedRun {
@@ -122,11 +123,12 @@ struct TunedShape {
   int64_t tile_rows = 0;
   int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1;
   int split = -2;  // probes run in the stage phase (-2: the heuristic's)
+  int npack = 1;
 };
 
 struct Options {
   int64_t stage_rows = -1, ring_depth = -1, consumer_warps = -1, ctas_per_sm = -1, probe_split = -2,
-          hash_load_pct = -1;
+          hash_load_pct = -1, packets = -1;
   int64_t jit = 1;
   int64_t build_pipeline = 1;
   int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
@@ -168,6 +170,8 @@ struct gpl_ctx {
   std::map<std::string, std::vector<std::string>> plan_segs;  // gpl_run_query: plan text -> segments
   void* h_stage = nullptr;  // pinned host staging for one packed D2H of results
   unsigned int* h_err = nullptr;  // pinned word for error-bit reads (gpl_sync)
+  long long* h_minmax = nullptr;  // pinned column min/max of a load (64 columns)
+  unsigned long long* h_stage_dev = nullptr;  // device alias of h_stage (the fused kernel's result copy-out)
   size_t h_stage_cap = 0;
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;

@@ -15,6 +15,8 @@
 #include <dlfcn.h>
 
 #include <climits>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -101,6 +103,7 @@ std::string shape_source(const PipeDesc& d) {
   I("stage_rows", d.stage_rows);
   I("depth", d.depth);
   I("nwarps", d.nwarps);
+  I("npack", d.npack);
   I("flush_each_tile", d.flush_each_tile);
   I("nfilt", d.nfilt);
   I("nsprobe", d.nsprobe);
@@ -165,6 +168,9 @@ std::string shape_source(const PipeDesc& d) {
   I("ins_pfield", d.ins_pfield);
   I("ins_ptransform", d.ins_ptransform);
   I("ins_width", d.ins_width);
+  I("ins_kcol", d.ins_kcol);
+  I("ins_pcol", d.ins_pcol);
+  I("ins_psreg", d.ins_psreg);
   I("smem_tables_bytes", d.smem_tables_bytes);
   I("off_queue", d.off_queue);
   I("off_agg", d.off_agg);
@@ -208,6 +214,14 @@ bool compile(const std::string& src, std::vector<char>* cubin, std::string* err)
   cubin->resize(cs);
   n.cubin(prog, cubin->data());
   n.destroy(&prog);
+  if (const char* dir = std::getenv("GPL_JIT_DUMP")) {  // diagnostics: cuobjdump / nvdisasm the plan kernels
+    static int seq = 0;
+    const std::string fn = std::string(dir) + "/gpl_jit_" + std::to_string(seq++) + ".cubin";
+    if (FILE* f = std::fopen(fn.c_str(), "wb")) {
+      std::fwrite(cubin->data(), 1, cubin->size(), f);
+      std::fclose(f);
+    }
+  }
   return cs > 0;
 }
 

@@ -36,6 +36,18 @@ cudaError_t launch_pipeline_fn(const void* fn, const PipeDesc& d, int grid, cuda
 // shape. Returns false with a message when NVRTC is unavailable or fails.
 bool jit_prepare(const PipeDesc& d, bool load, std::string* err);
 
+// Zero up to 16 device ranges (8-byte granular sizes) in one kernel launch.
+struct ClearList {
+  void* ptr[16];
+  unsigned long long bytes[16];
+  int n;
+};
+cudaError_t launch_clear(const ClearList& L, int num_sms, cudaStream_t s);
+
+// Copy `words` 8-byte words of device memory to mapped pinned host memory
+// (one CTA; programmatic dependent launch after the fused run).
+cudaError_t launch_copyout(const unsigned long long* src, unsigned long long* host_dst, int words, cudaStream_t s);
+
 // Column min/max (int32 or int64 column, n rows) -> out[0] = min, out[1] = max.
 cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s);
 

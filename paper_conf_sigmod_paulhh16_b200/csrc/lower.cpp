@@ -422,6 +422,14 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->ins_kmin = ins->dkmin;
     d->ins_nslots = ins->dnslots;
     d->ins_pay_base = ins->pay_base;
+    d->ins_kcol = d->ins_pcol = d->ins_psreg = -1;
+    if (sp == np && s.wheres.empty()) {  // every probe in the stage phase: insert from the staged tile
+      d->ins_kcol = cidx[s.key[0]];
+      if (ins->has_payload) {
+        if (pay_slot) d->ins_psreg = slot_of[s.payload.name];
+        else d->ins_pcol = cidx[s.payload.name];
+      }
+    }
   }
   // slot value ranges (validator)
   auto slot_range = [&](const std::string& n) -> Range {

@@ -103,16 +103,17 @@ __device__ __forceinline__ void qput(const PipeDesc& K, uint32_t qb, int f, int 
 // Probe RPL rows of one lane in table t: small DIRECT tables were staged in
 // shared memory by the prologue (LDS, no L1/L2 round trip); the rest go to
 // global memory (ht_probe_n: all RPL loads in flight).
-__device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int t, const unsigned long long (&key)[RPL],
-                                           const bool (&act)[RPL], bool (&hit)[RPL], long long (&pay)[RPL]) {
+template <int N>
+__device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int t, const unsigned long long (&key)[N],
+                                           const bool (&act)[N], bool (&hit)[N], long long (&pay)[N]) {
   const int kind = K.ht[t].kind, width = K.ht[t].width, so = K.ht_smem_off[t];
   if (kind == HT_DIRECT && so >= 0) {
     // branch-free: the cell index is clamped into the table and the loaded
     // value masked, so the 4 shared-memory loads issue back to back
     const uint32_t last = (uint32_t)(h.nslots - 1);
-    uint32_t v[RPL];
+    uint32_t v[N];
 #pragma unroll
-    for (int j = 0; j < RPL; j++) {
+    for (int j = 0; j < N; j++) {
       const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
       const bool in = act[j] && idx < h.nslots;
       const uint32_t i = in ? (uint32_t)idx : last;
@@ -124,19 +125,67 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int 
       v[j] = in ? x : 0u;
     }
 #pragma unroll
-    for (int j = 0; j < RPL; j++) {
+    for (int j = 0; j < N; j++) {
       hit[j] = v[j] != 0;
       pay[j] = width == 0 ? 1 : (long long)v[j] - 1 + h.pay_base;
     }
     return;
   }
-  ht_probe_n<RPL>(h, kind, width, key, act, hit, pay);
+  ht_probe_n<N>(h, kind, width, key, act, hit, pay);
 }
 
 __device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
   return (unsigned)p[0] + (unsigned)p[1] + (unsigned)p[2] + (unsigned)p[3];
 }
 __device__ __forceinline__ bool any4(const bool (&p)[RPL]) { return p[0] | p[1] | p[2] | p[3]; }
+// rows per lane of one consumer iteration: up to two packets in the
+// plan-specialised kernel; the generic kernel keeps one (register budget)
+#ifdef GPL_JIT
+constexpr int NR = 2 * RPL;
+#else
+constexpr int NR = RPL;
+#endif
+constexpr int NPMAX = NR / RPL;
+__device__ __forceinline__ unsigned count_n(const bool (&p)[NR]) {
+  unsigned c = 0;
+#pragma unroll
+  for (int j = 0; j < NR; j++) c += (unsigned)p[j];
+  return c;
+}
+__device__ __forceinline__ bool any_n(const bool (&p)[NR]) {
+  bool a = false;
+#pragma unroll
+  for (int j = 0; j < NR; j++) a |= p[j];
+  return a;
+}
+
+// Build segments: the blocking hash build as the pipeline's last
+// operator. DIRECT cells start at 0 (= empty): bitmap cells by atomicOr,
+// 32-bit cells by atomicCAS, 1- and 2-byte cells by atomicOr into their word;
+// a non-empty old cell is a duplicate key (FK->PK joins only).
+__device__ __forceinline__ void insert_cell(const PipeDesc& d, const PipeDesc& K, long long key, long long pay) {
+  const unsigned long long ci = (unsigned long long)((long long)(int32_t)key - d.ins_kmin);
+  if (ci >= d.ins_nslots) {
+    atomicOr(d.err, ERR_CAPACITY);
+    return;
+  }
+  if (K.ins_width == 0) {
+    const uint32_t bit = 1u << (ci & 31);
+    if (atomicOr((uint32_t*)d.ins_slots + (ci >> 5), bit) & bit) atomicOr(d.err, ERR_DUPKEY);
+    return;
+  }
+  if (K.ins_ptransform == G_YEAR) pay = (int)pay / 10000;
+  const uint32_t v = (uint32_t)(pay - d.ins_pay_base + 1);
+  if (K.ins_width == 4) {
+    if (atomicCAS((uint32_t*)d.ins_slots + ci, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
+  } else {
+    const unsigned long long byte = ci * (unsigned long long)K.ins_width;
+    uint32_t* w = (uint32_t*)((char*)d.ins_slots + (byte & ~3ull));
+    const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
+    const uint32_t m = (K.ins_width == 1 ? 0xFFu : 0xFFFFu) << sh;
+    if (atomicOr(w, v << sh) & m) atomicOr(d.err, ERR_DUPKEY);
+  }
+}
 
 // Queue phase on up to RPL*32 queued survivors starting at qhead: lane `lane`
 // owns entries qhead + j*32 + lane (j < RPL) that are < n. Remaining probes,
@@ -166,7 +215,7 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
       }
       bool hit[RPL];
       long long v[RPL];
-      probe_rows(K, htp[P.ht], P.ht, k, p, hit, v);
+      probe_rows<RPL>(K, htp[P.ht], P.ht, k, p, hit, v);
 #pragma unroll
       for (int j = 0; j < RPL; j++) {
         if (P.kind == P_MARK) {
@@ -207,36 +256,10 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
   }
   if (!__any_sync(0xffffffffu, any4(p))) return;
   if (K.sink == SINK_INSERT) {
-    // build segment: the blocking hash build as the pipeline's last
-    // operator. DIRECT cells start at 0 (= empty): bitmap cells by atomicOr,
-    // 32-bit cells by atomicCAS, 1- and 2-byte cells by atomicOr into their
-    // word; a non-empty old cell is a duplicate key (FK->PK joins only).
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
       if (!p[j]) continue;
-      const long long key = (long long)(int32_t)qget(K, qb, K.ins_kfield, idx[j]);
-      const unsigned long long ci = (unsigned long long)(key - d.ins_kmin);
-      if (ci >= d.ins_nslots) {
-        atomicOr(d.err, ERR_CAPACITY);
-        continue;
-      }
-      if (K.ins_width == 0) {
-        const uint32_t bit = 1u << (ci & 31);
-        if (atomicOr((uint32_t*)d.ins_slots + (ci >> 5), bit) & bit) atomicOr(d.err, ERR_DUPKEY);
-        continue;
-      }
-      long long pay = K.ins_pfield >= 0 ? qget(K, qb, K.ins_pfield, idx[j]) : 0;
-      if (K.ins_ptransform == G_YEAR) pay = (int)pay / 10000;
-      const uint32_t v = (uint32_t)(pay - d.ins_pay_base + 1);
-      if (K.ins_width == 4) {
-        if (atomicCAS((uint32_t*)d.ins_slots + ci, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
-      } else {
-        const unsigned long long byte = ci * (unsigned long long)K.ins_width;
-        uint32_t* w = (uint32_t*)((char*)d.ins_slots + (byte & ~3ull));
-        const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
-        const uint32_t m = (K.ins_width == 1 ? 0xFFu : 0xFFFFu) << sh;
-        if (atomicOr(w, v << sh) & m) atomicOr(d.err, ERR_DUPKEY);
-      }
+      insert_cell(d, K, qget(K, qb, K.ins_kfield, idx[j]), K.ins_pfield >= 0 ? qget(K, qb, K.ins_pfield, idx[j]) : 0);
     }
     return;
   }
@@ -322,6 +345,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     }
     fence_mbar_init();
   }
+  // (PDL) everything above overlaps the previous kernel's tail; tables,
+  // counters and columns it may write are read only after this wait
+  grid_dep_wait();
+  grid_dep_launch_dependents();
   if (threadIdx.x < K.nht) htp[threadIdx.x] = load_htp(d.ht[threadIdx.x]);
   GPL_UNROLL
   for (int t = 0; t < K.nht; t++) {  // stage small DIRECT tables into shared memory
@@ -341,10 +368,14 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     if (lane == 0) {
       const unsigned long long pol = policy_evict_first();
       uint32_t slot = 0, phase = 0;
+      // the next tile is claimed before the current one's copies are issued,
+      // so the claim's global-atomic round trip overlaps them (with small
+      // tiles it would otherwise bound the producer: one claim per stage)
+      unsigned long long t = atomicAdd(d.tile_counter, 1ull);
       for (;;) {
-        const unsigned long long t = atomicAdd(d.tile_counter, 1ull);
         const long long r0 = (long long)t * d.tile_rows;
         if (r0 >= d.nrows) break;
+        const unsigned long long t_next = atomicAdd(d.tile_counter, 1ull);
         const long long rn = min(d.tile_rows, d.nrows - r0);
         for (long long s0 = 0; s0 < rn; s0 += K.stage_rows) {
           const int n = (int)min((long long)K.stage_rows, rn - s0);
@@ -362,6 +393,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
                      &full[slot], pol);
           if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
         }
+        t = t_next;
       }
       mbar_wait(&empty[slot], phase ^ 1u);
       hdr[slot] = make_int4(0, 0, -1, 0);
@@ -394,47 +426,74 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     if (n < 0) break;
     const uint32_t sb = (uint32_t)K.off_ring + slot * (uint32_t)K.slot_bytes;
     const int nit = (n + 127) >> 7;
-    for (int it = warp; it < nit; it += W) {
-      const int r0 = (it << 7) + (lane << 2);
-      bool p[RPL];
+    bool released = false;
+    // Each iteration takes npk (1 or 2) of the warp's 128-row packets,
+    // it0 and it0 + W: their filters and stage-phase probes run in lockstep so
+    // a lane keeps up to NR = 8 independent probe loads in flight (the
+    // stage-phase probe latency is a warp's critical path); compaction and the
+    // queue then proceed packet by packet.
+    const int npk = K.npack < NPMAX ? K.npack : NPMAX;
+    for (int it0 = warp; it0 < nit; it0 += npk * W) {
+      int r0q[NPMAX];
+      bool live[NPMAX];
 #pragma unroll
-      for (int j = 0; j < RPL; j++) p[j] = r0 + j < n;
-      // A4 selection: predicates on staged columns, 4 rows per lane
+      for (int q = 0; q < NPMAX; q++) {
+        r0q[q] = ((it0 + q * W) << 7) + (lane << 2);
+        live[q] = q < npk && it0 + q * W < nit;
+      }
+      bool p[NR];
+#pragma unroll
+      for (int q = 0; q < NPMAX; q++)
+#pragma unroll
+        for (int j = 0; j < RPL; j++) p[q * RPL + j] = live[q] && r0q[q] + j < n;
+      // A4 selection: predicates on staged columns, 4 rows per lane per packet
       GPL_UNROLL
       for (int f = 0; f < K.nfilt; f++) {
         const Filt& F = K.filt[f];
-        long long x[RPL];
-        ld_rows(sb + K.coloff[F.ref] + r0 * K.colw[F.ref], K.colw[F.ref], x);
 #pragma unroll
-        for (int j = 0; j < RPL; j++) p[j] = p[j] && filt_pass(F, x[j]);
-        const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+        for (int q = 0; q < NPMAX; q++) {
+          if (q >= npk) break;
+          long long x[RPL];
+          ld_rows(sb + K.coloff[F.ref] + r0q[q] * K.colw[F.ref], K.colw[F.ref], x);
+#pragma unroll
+          for (int j = 0; j < RPL; j++) p[q * RPL + j] = p[q * RPL + j] && filt_pass(F, x[j]);
+        }
+        const unsigned c = __reduce_add_sync(0xffffffffu, count_n(p));
         if (lane == 0) cnt[f] += c;
       }
-      // A5 stage-phase probes (keys from the stage; loads of the 4 rows in flight together)
-      long long sreg[MAXSP][RPL];
+      // A5 stage-phase probes (keys from the stage; all NR loads in flight together)
+      long long sreg[MAXSP][NR];
 #pragma unroll
       for (int sp = 0; sp < MAXSP; sp++) {
 #pragma unroll
-        for (int j = 0; j < RPL; j++) sreg[sp][j] = 0;
+        for (int j = 0; j < NR; j++) sreg[sp][j] = 0;
         if (sp < K.nsprobe) {
           const Probe& P = K.probe[sp];
-          if (__any_sync(0xffffffffu, any4(p))) {
-            long long k1[RPL];
-            ld_rows(sb + K.coloff[P.k1] + r0 * K.colw[P.k1], K.colw[P.k1], k1);
-            unsigned long long k[RPL];
+          if (__any_sync(0xffffffffu, any_n(p))) {
+            unsigned long long k[NR];
 #pragma unroll
-            for (int j = 0; j < RPL; j++) k[j] = (uint32_t)k1[j];
-            if (P.k2 >= 0) {
-              long long k2[RPL];
-              ld_rows(sb + K.coloff[P.k2] + r0 * K.colw[P.k2], K.colw[P.k2], k2);
+            for (int q = 0; q < NPMAX; q++) {
+              long long k1[RPL];
+              if (q < npk) {
+                ld_rows(sb + K.coloff[P.k1] + r0q[q] * K.colw[P.k1], K.colw[P.k1], k1);
+              } else {
 #pragma unroll
-              for (int j = 0; j < RPL; j++) k[j] = (k[j] << 32) | (uint32_t)k2[j];
+                for (int j = 0; j < RPL; j++) k1[j] = 0;
+              }
+#pragma unroll
+              for (int j = 0; j < RPL; j++) k[q * RPL + j] = (uint32_t)k1[j];
+              if (P.k2 >= 0 && q < npk) {
+                long long k2[RPL];
+                ld_rows(sb + K.coloff[P.k2] + r0q[q] * K.colw[P.k2], K.colw[P.k2], k2);
+#pragma unroll
+                for (int j = 0; j < RPL; j++) k[q * RPL + j] = (k[q * RPL + j] << 32) | (uint32_t)k2[j];
+              }
             }
-            bool hit[RPL];
-            long long v[RPL];
-            probe_rows(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v);
+            bool hit[NR];
+            long long v[NR];
+            probe_rows<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v);
 #pragma unroll
-            for (int j = 0; j < RPL; j++) {
+            for (int j = 0; j < NR; j++) {
               if (P.kind == P_MARK) {
                 sreg[sp][j] = hit[j] ? 1 : 0;
               } else {
@@ -443,69 +502,111 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
               }
             }
           }
-          const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+          const unsigned c = __reduce_add_sync(0xffffffffu, count_n(p));
           if (lane == 0) cnt[K.nfilt + sp] += c;
         }
       }
-      // A8 compaction into the warp's survivor queue (the on-chip channel)
-      int base = qcount;
-      int pos[RPL];
+      if (K.sink == SINK_INSERT && K.ins_kcol >= 0) {
+        // build segment with every probe in the stage phase: insert straight
+        // from the staged tile (no survivor queue)
 #pragma unroll
-      for (int j = 0; j < RPL; j++) {
-        const unsigned m = __ballot_sync(0xffffffffu, p[j]);
-        pos[j] = (qhead + base + __popc(m & lanemask_lt())) & (QCAP - 1);
-        base += __popc(m);
-      }
-      if (base == qcount) continue;
-      GPL_UNROLL
-      for (int e = 0; e < K.npush; e++) {
-        const Push& E = K.push[e];
-        const uint32_t qa = qb + K.qoff[e];
-        long long v[RPL];
-        if (E.kind == PUSH_COL) {
-          ld_rows(sb + K.coloff[E.src] + r0 * K.colw[E.src], K.colw[E.src], v);
-        } else if (E.kind == PUSH_SREG) {
+        for (int q = 0; q < NPMAX; q++) {
+          if (!live[q]) break;
+          long long kx[RPL], px[RPL];
+          ld_rows(sb + K.coloff[K.ins_kcol] + r0q[q] * K.colw[K.ins_kcol], K.colw[K.ins_kcol], kx);
+          if (K.ins_pcol >= 0) {
+            ld_rows(sb + K.coloff[K.ins_pcol] + r0q[q] * K.colw[K.ins_pcol], K.colw[K.ins_pcol], px);
+          } else {
 #pragma unroll
-          for (int j = 0; j < RPL; j++) v[j] = E.src == 0 ? sreg[0][j] : sreg[1][j];
-        } else {  // pushed-down value term: sign * prod(a + b * x)
-          const Term& T = K.sterm[E.src];
+            for (int j = 0; j < RPL; j++) px[j] = K.ins_psreg == 0 ? sreg[0][q * RPL + j] : K.ins_psreg == 1 ? sreg[1][q * RPL + j] : 0;
+          }
 #pragma unroll
-          for (int j = 0; j < RPL; j++) v[j] = T.sign;
-          GPL_UNROLL
-          for (int f = 0; f < T.nfact; f++) {
-            const Factor& F = T.f[f];
-            long long x[RPL];
-            if (F.field >= 0) {
-              ld_rows(sb + K.coloff[F.field] + r0 * K.colw[F.field], K.colw[F.field], x);
-            } else {
-#pragma unroll
-              for (int j = 0; j < RPL; j++) x[j] = F.field == SREF_CONST ? 0 : (F.field == -2 ? sreg[0][j] : sreg[1][j]);
-            }
-#pragma unroll
-            for (int j = 0; j < RPL; j++) v[j] *= F.a + (long long)F.b * x[j];
+          for (int j = 0; j < RPL; j++)
+            if (p[q * RPL + j]) insert_cell(d, K, kx[j], px[j]);
+          if (it0 + q * W + W >= nit) {
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[slot]);
+            released = true;
           }
         }
-        if (K.qw[e] == 4) {
+        continue;
+      }
+      // A8 compaction into the warp's survivor queue (the on-chip channel), packet by packet
 #pragma unroll
-          for (int j = 0; j < RPL; j++)
-            if (p[j]) S<int>(qa + pos[j] * 4) = (int)v[j];
-        } else {
+      for (int q = 0; q < NPMAX; q++) {
+        if (!live[q]) break;
+        const int r0 = r0q[q];
+        int base = qcount;
+        int pos[RPL];
 #pragma unroll
-          for (int j = 0; j < RPL; j++)
-            if (p[j]) S<long long>(qa + pos[j] * 8) = v[j];
+        for (int j = 0; j < RPL; j++) {
+          const unsigned m = __ballot_sync(0xffffffffu, p[q * RPL + j]);
+          pos[j] = (qhead + base + __popc(m & lanemask_lt())) & (QCAP - 1);
+          base += __popc(m);
+        }
+        if (base != qcount) {
+          GPL_UNROLL
+          for (int e = 0; e < K.npush; e++) {
+            const Push& E = K.push[e];
+            const uint32_t qa = qb + K.qoff[e];
+            long long v[RPL];
+            if (E.kind == PUSH_COL) {
+              ld_rows(sb + K.coloff[E.src] + r0 * K.colw[E.src], K.colw[E.src], v);
+            } else if (E.kind == PUSH_SREG) {
+#pragma unroll
+              for (int j = 0; j < RPL; j++) v[j] = E.src == 0 ? sreg[0][q * RPL + j] : sreg[1][q * RPL + j];
+            } else {  // pushed-down value term: sign * prod(a + b * x)
+              const Term& T = K.sterm[E.src];
+#pragma unroll
+              for (int j = 0; j < RPL; j++) v[j] = T.sign;
+              GPL_UNROLL
+              for (int f = 0; f < T.nfact; f++) {
+                const Factor& F = T.f[f];
+                long long x[RPL];
+                if (F.field >= 0) {
+                  ld_rows(sb + K.coloff[F.field] + r0 * K.colw[F.field], K.colw[F.field], x);
+                } else {
+#pragma unroll
+                  for (int j = 0; j < RPL; j++)
+                    x[j] = F.field == SREF_CONST ? 0 : (F.field == -2 ? sreg[0][q * RPL + j] : sreg[1][q * RPL + j]);
+                }
+#pragma unroll
+                for (int j = 0; j < RPL; j++) v[j] *= F.a + (long long)F.b * x[j];
+              }
+            }
+            if (K.qw[e] == 4) {
+#pragma unroll
+              for (int j = 0; j < RPL; j++)
+                if (p[q * RPL + j]) S<int>(qa + pos[j] * 4) = (int)v[j];
+            } else {
+#pragma unroll
+              for (int j = 0; j < RPL; j++)
+                if (p[q * RPL + j]) S<long long>(qa + pos[j] * 8) = v[j];
+            }
+          }
+          qcount = base;
+        }
+        if (it0 + q * W + W >= nit) {
+          // the warp's last packet of this stage is in the queue: release the
+          // ring slot BEFORE draining (the drain reads only the queue), so the
+          // producer's next copy overlaps the drain's probe/insert latency
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&empty[slot]);
+          released = true;
+        }
+        if (qcount >= RPL * 32) {
+          __syncwarp();
+          drain(d, qb, qhead, RPL * 32, cnt, acc, lane);
+          __syncwarp();
+          qhead = (qhead + RPL * 32) & (QCAP - 1);
+          qcount -= RPL * 32;
         }
       }
-      qcount = base;
-      if (qcount >= RPL * 32) {
-        __syncwarp();
-        drain(d, qb, qhead, RPL * 32, cnt, acc, lane);
-        __syncwarp();
-        qhead = (qhead + RPL * 32) & (QCAP - 1);
-        qcount -= RPL * 32;
-      }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[slot]);
+    if (!released) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);
+    }
     if (K.flush_each_tile && h.w) flush_reg(d, acc, lane);
     if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
   }

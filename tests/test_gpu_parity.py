@@ -88,7 +88,8 @@ def test_schedule_invariance(ctx):
     expect = {q: oracle.run(q, db, _params(q)) for q in ("Q5", "Q7", "Q14", "L1")}
     knobs = [dict(stage_rows=128, ring_depth=2, consumer_warps=1), dict(stage_rows=256, ring_depth=3, consumer_warps=4),
              dict(stage_rows=1024, ring_depth=4, consumer_warps=8), dict(stage_rows=2048, ring_depth=2, consumer_warps=12), dict(stage_rows=3072, ring_depth=2, consumer_warps=2),
-             dict(probe_split=0), dict(probe_split=1), dict(probe_split=2), dict(probe_split=-1)]
+             dict(probe_split=0), dict(probe_split=1), dict(probe_split=2), dict(probe_split=-1),
+             dict(packets=2, consumer_warps=3), dict(packets=2, stage_rows=384, probe_split=2), dict(packets=1)]
     try:
         for k in knobs:
             for key, v in k.items():
@@ -100,7 +101,7 @@ def test_schedule_invariance(ctx):
             for key in k:
                 ctx.set_option(key, -1 if key != "probe_split" else -2)
     finally:
-        for key in ("stage_rows", "ring_depth", "consumer_warps"):
+        for key in ("stage_rows", "ring_depth", "consumer_warps", "packets"):
             ctx.set_option(key, -1)
         ctx.set_option("probe_split", -2)
 
@@ -288,3 +289,17 @@ def test_gpl_without_ce_bit_identical(ctx, q):
             assert r.stats["tile_rows_used"] == min(tile, db.nrows("lineitem"))
     finally:
         ctx.set_option("kbe_tile_rows", 0)
+
+
+def test_fetch_after_unrelated_load(ctx):
+    """The fused run's results are copied out to pinned host memory by the
+    run itself; loading other columns between the run and the fetch must not
+    disturb them."""
+    db = tpchgen.generate(0.05, seed=61)
+    queries.load_database(ctx, db, queries.TABLES["Q5"])
+    o = oracle.run("Q5", db)
+    for _ in range(3):  # eager, capture, graph replay
+        ctx.run_query(queries.plan_text("Q5", db))
+        ctx.load_columns("scratch_tbl", {"x": np.arange(1000, dtype=np.int32)})
+        r = queries.decode_keys("Q5", ctx.fetch_result(), db)
+        assert r.keys == o.keys and r.aggs == o.aggs

@@ -15,8 +15,12 @@ ddb = D(); ddb.tables = {t: {c: torch.from_numpy(a).to(dev) for c, a in cols.ite
 queries.load_database(ctx, ddb)
 text = queries.plan_text(q, db)
 for spec in sys.argv[3:]:
-    S, Dp, W, k = map(int, spec.split(","))
-    for key, v in (("stage_rows", S), ("ring_depth", Dp), ("consumer_warps", W), ("ctas_per_sm", k)):
+    vals = list(map(int, spec.split(",")))
+    S, Dp, W, k = vals[:4]
+    npk = vals[4] if len(vals) > 4 else -1
+    sp = vals[5] if len(vals) > 5 else -2
+    for key, v in (("stage_rows", S), ("ring_depth", Dp), ("consumer_warps", W), ("ctas_per_sm", k),
+                   ("packets", npk), ("probe_split", sp)):
         ctx.set_option(key, v)
     ts = []
     try:
@@ -26,4 +30,4 @@ for spec in sys.argv[3:]:
     except gpl.GplError as e:
         print(spec, "ERR", e); continue
     t = statistics.median(ts)
-    print(f"{q} SF{sf} S={S} D={Dp} W={W} k={k}: {t*1e3:.1f} us  {r.stats['bytes_scanned']/t/1e6:.0f} GB/s", flush=True)
+    print(f"{q} SF{sf} S={S} D={Dp} W={W} k={k} P={npk} split={r.stats['probe_split']}: {t*1e3:.1f} us  {r.stats['bytes_scanned']/t/1e6:.0f} GB/s", flush=True)
