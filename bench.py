@@ -328,7 +328,12 @@ def main():
         ctx2.close()
 
     peak, peak_kind = measured_peak()
-    bytes_per_launch = stats["bytes_scanned"]
+    # algorithmic bytes per fact row = b, every column the query
+    # reads, each read once (rows x b per launch). With late materialisation the
+    # kernel moves fewer bytes (staged columns + survivor gathers): reported as
+    # moved_bytes beside it.
+    bytes_per_launch = stats.get("bytes_full_scan") or stats["bytes_scanned"]
+    moved = stats["bytes_scanned"]
     achieved = bytes_per_launch / (kernel_avg / 1e3) / 1e9
     traffic = None
     prof = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -359,14 +364,20 @@ def main():
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                      "kernel": "pipeline_kernel (fused scan-filter-probe-aggregate)",
-                     "bytes_per_launch": bytes_per_launch},
+                     "bytes_per_launch": bytes_per_launch,
+                     "algorithmic_bytes": "lineitem rows x b (b = bytes/row of every column the plan reads, "
+                                          "SURVEY 8(d))",
+                     # late materialisation: lazy columns are gathered only for the rows that
+                     # reach their first use, so the kernel moves fewer bytes than it scans logically
+                     "moved_bytes": moved, "moved_gbs": moved / (kernel_avg / 1e3) / 1e9,
+                     "lazy_columns": stats.get("lazy_columns")},
         "gpu_launches": kernel_launches(segs) * args.steps,
         "e2e": e2e,
         "cpu_baseline": cpu,
         "clocks": clk.summary(),
         "wall_s_timed_region": wall,
-        "pipeline": {k: stats[k] for k in ("tile_rows_used", "stage_rows", "ring_depth", "consumer_warps", "grid",
-                                           "probe_split", "predicted_ms", "agg_mode")},
+        "pipeline": {k: stats.get(k) for k in ("tile_rows_used", "stage_rows", "ring_depth", "consumer_warps", "grid",
+                                               "probe_split", "predicted_ms", "agg_mode", "packets", "lazy_columns")},
         "op_pass": stats["op_pass"],
         "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
         "jit": stats.get("jit"),

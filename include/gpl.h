@@ -84,12 +84,17 @@ typedef struct {
   int64_t op_pass[16];         /* rows passing each operator in plan order (filters, probes, where) */
   double kernel_ms;            /* fused pipeline kernel time (CUDA events on the ctx stream)      */
   double predicted_ms;         /* A9 model estimate for this run                                   */
-  double bytes_scanned;        /* algorithmic bytes: rows x bytes/row of staged columns           */
+  double bytes_scanned;        /* algorithmic bytes: rows x bytes/row of TMA-staged columns +      */
+                               /* (rows reaching the first use) x width of each lazy column       */
   int32_t agg_mode;            /* 0 registers (1 group), 1 smem table, 2 global int128 atomics   */
   int32_t kbe;                 /* 1 if produced by gpl_run_plan_kbe                               */
   int32_t jit;                 /* 1 if the plan-specialised (NVRTC) kernel ran, 0 the generic one */
   int32_t reserved;
   double intermediate_bytes;   /* bytes of operator outputs materialised in HBM (fused path: 0)   */
+  double bytes_full_scan;      /* rows x bytes/row of EVERY column the plan reads (no late        */
+                               /* materialisation): the logical scan; >= bytes_scanned            */
+  int32_t lazy_columns;        /* columns gathered per surviving row instead of TMA-staged        */
+  int32_t packets;             /* 128-row packets per consumer iteration                          */
 } gpl_stats;
 
 /* Result of the last run. Arrays are CALLER-owned with capacity cap_groups. */

@@ -237,6 +237,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "kbe_tile_rows") {
     if (v < 0) return fail(ctx, GPL_E_ARG, "kbe_tile_rows >= 0 (0 = whole input: KBE)");
     o.kbe_tile_rows = v;
+  } else if (k == "lazy_columns") {
+    o.lazy_columns = v < 0 ? -1 : v > 0 ? 1 : 0;
   } else if (k == "build_pipeline") {
     o.build_pipeline = v != 0 ? 1 : 0;
   } else if (k == "jit") {
@@ -688,6 +690,13 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
   std::string jerr;
   P.fn = resolve_pipeline_fn(d, ctx->opt.jit != 0, &jerr);
   P.jit = ctx->opt.jit != 0 && jerr.empty();
+  if (std::getenv("GPL_DEBUG_DESC")) {  // diagnostics: the launch layout of each prepared run
+    std::fprintf(stderr, "prepared run: nrows %lld tile %lld S %d D %d W %d npack %d grid %d smem %d off_ring %d slot %d ncols %d split %d:",
+                 d.nrows, d.tile_rows, d.stage_rows, d.depth, d.nwarps, d.npack, P.grid, d.smem_bytes, d.off_ring,
+                 d.slot_bytes, d.ncols, d.nsprobe);
+    for (int c = 0; c < d.ncols; c++) std::fprintf(stderr, " [%d:w%d off%d lazy%d %p]", c, d.colw[c], d.coloff[c], d.lazy[c], (const void*)d.col[c]);
+    std::fprintf(stderr, " jit=%d %s\n", (int)P.jit, jerr.c_str());
+  }
   if (!P.fn) return fail(ctx, GPL_E_CUDA, "cannot configure the pipeline kernel");
   auto sp = std::make_shared<PreparedRun>(P);
   ctx->run_cache[key] = sp;
@@ -730,6 +739,9 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   S.probe_split = d.nsprobe;
   S.predicted_ms = P->pred_ms;
   S.bytes_scanned = (double)d.nrows * li.bytes_per_row;
+  S.bytes_full_scan = (double)d.nrows * li.bytes_per_row_all;
+  S.lazy_columns = (int32_t)li.lazy_w.size();
+  S.packets = d.npack;
   S.agg_mode = d.agg_mode;
   S.jit = P->jit ? 1 : 0;
   return GPL_OK;
@@ -820,6 +832,9 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       S.probe_split = P.desc.nsprobe;
       S.predicted_ms = P.pred_ms;
       S.bytes_scanned = (double)P.desc.nrows * P.li.bytes_per_row;
+      S.bytes_full_scan = (double)P.desc.nrows * P.li.bytes_per_row_all;
+      S.lazy_columns = (int32_t)P.li.lazy_w.size();
+      S.packets = P.desc.npack;
       S.agg_mode = P.desc.agg_mode;
       S.jit = P.jit ? 1 : 0;
       return GPL_OK;
@@ -910,6 +925,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     for (int sp = 0; sp <= std::min<int>((int)seg.probes.size(), MAXSP); sp++)
       if (sp != split0) splits.push_back(sp);
   std::vector<std::pair<int, Config>> cands;
+  std::vector<int> cand_split_eff;  // the split the lowering kept (late materialisation may move a probe to the queue)
   ctx->tuned.erase(seg.text);
   for (int sp : splits) {
     PipeDesc ds;
@@ -932,7 +948,10 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
       continue;
     }
     if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
-    for (const Config& c : cs) cands.push_back({sp, c});
+    for (const Config& c : cs) {
+      cands.push_back({sp, c});
+      cand_split_eff.push_back(ds.nsprobe);
+    }
     if (sp == split0) {
       d = ds;
       li = ls;
@@ -944,8 +963,10 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   CK(cudaMalloc(&flush, fbytes));
   double best_ms = 1e300;
   TunedShape best;
+  int best_eff_split = -1;
   int tried = 0;
-  for (const auto& sc : cands) {
+  for (size_t ci = 0; ci < cands.size(); ci++) {
+    const auto& sc = cands[ci];
     const Config& c = sc.second;
     TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sc.first, c.npack};
     ctx->tuned[seg.text] = t;
@@ -970,6 +991,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     if (ms[1] < best_ms) {
       best_ms = ms[1];
       best = t;
+      best_eff_split = cand_split_eff[ci];
     }
   }
   cudaFree(flush);
@@ -1002,7 +1024,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     out->ctas_per_sm = c.ctas_per_sm;
     out->candidates = tried;
     out->measured_ms = best_ms;
-    out->probe_split = best.split >= 0 ? best.split : split0;
+    out->probe_split = best_eff_split;
   }
   return GPL_OK;
 }
@@ -1041,8 +1063,14 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   LowerInfo li;
   Config cfg;
   Segment seg;
-  // every probe reads its keys from materialised columns: lower with no stage-phase probe
-  if ((st = prepare_run(ctx, probe_segment, 0, &d, &li, &cfg, &seg, 0))) return st;
+  // every probe reads its keys from materialised columns: lower with no
+  // stage-phase probe, and every column materialised by the map kernels (no
+  // late materialisation: KBE reads each column it uses in full)
+  const int64_t lazy_opt = ctx->opt.lazy_columns;
+  ctx->opt.lazy_columns = 0;
+  st = prepare_run(ctx, probe_segment, 0, &d, &li, &cfg, &seg, 0);
+  ctx->opt.lazy_columns = lazy_opt;
+  if (st) return st;
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
   d.partials = partials_ptr(ctx);
   d.tile_counter = counter_ptr(ctx);
@@ -1094,7 +1122,8 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   S.rows_scanned = d.nrows;
   S.n_ops = li.nops;
   S.probe_split = -1;
-  S.bytes_scanned = (double)d.nrows * li.bytes_per_row;
+  S.bytes_scanned = (double)d.nrows * li.bytes_per_row_all;  // KBE reads every column it uses
+  S.bytes_full_scan = S.bytes_scanned;
   S.agg_mode = AGG_GLOBAL;
   S.kbe = 1;
   S.intermediate_bytes = inter;
@@ -1133,6 +1162,14 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
     if (cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1) == cudaSuccess) S.kernel_ms = ms;
   }
   for (int i = 0; i < MAXOPS && i < 16; i++) S.op_pass[i] = (int64_t)ops[i];
+  if (!ctx->last.kbe) {  // lazy columns: the rows that reached their first use were gathered
+    double b = (double)S.rows_scanned * li.bytes_per_row;
+    for (size_t i = 0; i < li.lazy_w.size(); i++) {
+      const int op = li.lazy_reach[i];
+      b += (double)li.lazy_w[i] * (op >= 0 && op < MAXOPS ? (double)ops[op] : (double)S.rows_scanned);
+    }
+    S.bytes_scanned = b;
+  }
   // λ cache for the model / split choice (cumulative pass fraction after each op)
   // (recorded once per plan text: the first run profiles the plan)
   if (!ctx->last.kbe && S.rows_scanned > 0 && !ctx->lambda.count(ctx->last.run->text)) {

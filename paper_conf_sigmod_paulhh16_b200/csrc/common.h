@@ -124,7 +124,7 @@ enum : int32_t { SINK_AGG = 0, SINK_INSERT = 1 };
 
 // ---- survivor-queue push: field <- stage column, stage-phase probe slot, or
 // a value term computed in the stage phase (expression pushdown)
-enum : int32_t { PUSH_COL = 0, PUSH_SREG = 1, PUSH_TERM = 2 };
+enum : int32_t { PUSH_COL = 0, PUSH_SREG = 1, PUSH_TERM = 2, PUSH_ROWID = 3 };
 struct Push {
   int32_t kind, src;
 };
@@ -137,7 +137,11 @@ struct PipeDesc {
   long long nrows;
   const char* col[MAXC];
   int32_t colw[MAXC];
-  int32_t coloff[MAXC];  // byte offset of column c inside one ring slot
+  int32_t coloff[MAXC];  // byte offset of column c inside one ring slot (-1: lazy)
+  // late materialisation (the paper's k_reduce fetches
+  // LINEITEM only for satisfied tuples): a lazy column is not staged by
+  // TMA; its values are gathered from HBM for the rows that reach its first use
+  int32_t lazy[MAXC];
   int32_t ncols, slot_bytes;
   // schedule (A2)
   long long tile_rows;
@@ -151,6 +155,8 @@ struct PipeDesc {
   int32_t qoff[MAXQ];    // byte offset of field f's array in a warp's queue (QCAP entries)
   int32_t qw[MAXQ];      // field width in bytes (4 or 8)
   int32_t qbytes;        // bytes of one warp's queue
+  int32_t qlazy[MAXQ];   // >= 0: field f is lazy column qlazy[f], gathered by the drain via the row id
+  int32_t rowid_field;   // queue field holding the row id (-1: no lazy column)
   int32_t term_field[MAXTERM];  // >= 0: term t was computed in the stage phase into this field
   Term sterm[MAXTERM];          // stage-phase form of pushed-down terms (stage refs)
   int32_t nfield, nresid, ngroup, ngroups_total;

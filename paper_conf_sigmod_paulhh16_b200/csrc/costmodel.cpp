@@ -46,7 +46,8 @@ int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth
   int q = warps * d.qbytes;
   int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   int slot = 0;
-  for (int c = 0; c < d.ncols; c++) slot += align128(stage_rows * d.colw[c]);
+  for (int c = 0; c < d.ncols; c++)
+    if (!d.lazy[c]) slot += align128(stage_rows * d.colw[c]);
   return align128(kFixed + q) + align128(agg) + align128(d.smem_tables_bytes) + depth * slot;
 }
 
@@ -65,6 +66,10 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->off_ring = off_tables + align128(d->smem_tables_bytes);
   int off = 0;
   for (int i = 0; i < d->ncols; i++) {
+    if (d->lazy[i]) {  // gathered per surviving row, not staged
+      d->coloff[i] = -1;
+      continue;
+    }
     d->coloff[i] = off;
     off += align128(c.stage_rows * d->colw[i]);
   }
@@ -90,7 +95,13 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
                k * (W + 1) * 32 * (npack == 2 ? 112 : 80) <= 65536 && (npack == 1 || npack == 2);
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
-  const double b = std::max(1, li.bytes_per_row);
+  // bytes per row: staged columns, plus one 32-B sector per surviving row of
+  // each lazy (gathered) column
+  double b = std::max(1, li.bytes_per_row);
+  for (size_t i = 0; i < li.lazy_reach.size(); i++) {
+    const int op = li.lazy_reach[i];
+    b += 32.0 * (op >= 0 && op < (int)li.lambda.size() ? li.lambda[op] : 0.05);
+  }
   const double f_sm = 1.9e9;
   const double B_sm = 1.6 * B / ctx->sms;  // one SM's TMA/L2 fill cap
   N = std::max<int64_t>(N, 1);
@@ -127,6 +138,8 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   };
   double lat_stage = 0, lat_queue = 0;
   for (int p = 0; p < li.nprobe; p++) (p < d.nsprobe ? lat_stage : lat_queue) += lat(li.probe_ht[p]);
+  // lazy columns: one HBM gather round trip per drain (per 128 queued rows)
+  if (!li.lazy_reach.empty()) lat_queue += 2000.0;
   // cycles per warp iteration of `npack` packets: the stage-phase probe
   // latency is paid once per iteration (all npack*4 loads of a lane in flight)
   const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);

@@ -64,7 +64,10 @@ struct HashTable {
 struct LowerInfo {
   int ngroups_total = 1, nagg = 1, nops = 0, ngroup_dims = 0;
   int glo[MAXG] = {0, 0, 0}, gsize[MAXG] = {1, 1, 1}, gstride[MAXG] = {1, 1, 1};
-  int bytes_per_row = 0;
+  int bytes_per_row = 0;        // TMA-staged (eager) column bytes per row
+  int bytes_per_row_all = 0;    // every column the segment reads
+  std::vector<int> lazy_w;      // width of each lazy column
+  std::vector<int> lazy_reach;  // op whose pass count = rows reaching the column (-1: all rows)
   long double maxabs = 0;  // bound on |value| per row
   std::vector<std::string> op_names;
   std::vector<int64_t> ht_bytes;  // slot bytes of each probed table
@@ -130,6 +133,7 @@ struct Options {
   int64_t stage_rows = -1, ring_depth = -1, consumer_warps = -1, ctas_per_sm = -1, probe_split = -2,
           hash_load_pct = -1, packets = -1;
   int64_t jit = 1;
+  int64_t lazy_columns = -1;   // late materialisation: -1 auto (from λ), 0 off, 1 every eligible column
   int64_t build_pipeline = 1;
   int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
   double hbm_gbs = -1;

@@ -99,7 +99,9 @@ std::string shape_source(const PipeDesc& d) {
   o << "namespace gpl_jit {\n__host__ __device__ constexpr gpl::PipeDesc make_shape() {\n  gpl::PipeDesc k{};\n";
   I("ncols", d.ncols);
   I("slot_bytes", d.slot_bytes);
-  for (int c = 0; c < d.ncols; c++) o << "  k.colw[" << c << "] = " << d.colw[c] << "; k.coloff[" << c << "] = " << d.coloff[c] << ";\n";
+  for (int c = 0; c < d.ncols; c++)
+    o << "  k.colw[" << c << "] = " << d.colw[c] << "; k.coloff[" << c << "] = " << d.coloff[c] << "; k.lazy[" << c
+      << "] = " << d.lazy[c] << ";\n";
   I("stage_rows", d.stage_rows);
   I("depth", d.depth);
   I("nwarps", d.nwarps);
@@ -123,6 +125,8 @@ std::string shape_source(const PipeDesc& d) {
     o << " k.qoff[" << e << "] = " << d.qoff[e] << "; k.qw[" << e << "] = " << d.qw[e] << ";\n";
   }
   I("qbytes", d.qbytes);
+  I("rowid_field", d.rowid_field);
+  for (int f = 0; f < MAXQ; f++) o << "  k.qlazy[" << f << "] = " << d.qlazy[f] << ";\n";
   auto term = [&](const char* arr, int t, const Term& T) {
     o << "  k." << arr << "[" << t << "].sign = " << T.sign << "; k." << arr << "[" << t << "].nfact = " << T.nfact << ";\n";
     for (int f = 0; f < T.nfact; f++)
@@ -219,6 +223,10 @@ bool compile(const std::string& src, std::vector<char>* cubin, std::string* err)
     const std::string fn = std::string(dir) + "/gpl_jit_" + std::to_string(seq++) + ".cubin";
     if (FILE* f = std::fopen(fn.c_str(), "wb")) {
       std::fwrite(cubin->data(), 1, cubin->size(), f);
+      std::fclose(f);
+    }
+    if (FILE* f = std::fopen((fn + ".cu").c_str(), "wb")) {
+      std::fwrite(src.data(), 1, src.size(), f);
       std::fclose(f);
     }
   }

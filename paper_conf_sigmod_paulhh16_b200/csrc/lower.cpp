@@ -318,10 +318,62 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   if (sp < 0) sp = s.filters.empty() ? std::min(1, np) : 0;
   sp = std::min(std::min(sp, np), MAXSP);
 
+  // Late materialisation (the paper's k_reduce fetches
+  // LINEITEM only for the satisfied tuples). A column used only after
+  // selective operators is *lazy*: not TMA-staged; the survivor queue carries
+  // the row id and the drain gathers the column from HBM for its (up to) 128
+  // queued rows at once. It pays one 32-B sector per surviving row instead of
+  // its width per scanned row, so it is chosen when (rows reaching the queue /
+  // rows) * 64 <= width, from the previous run's pass fractions λ. In auto mode
+  // a stage-phase probe whose key column qualifies moves to the queue phase.
+  std::set<std::string> lazy;
+  const int nf0 = (int)s.filters.size();
+  if (!ins && ctx->opt.lazy_columns != 0 && T.nrows < (1ll << 31)) {
+    auto lit = ctx->lambda.find(s.text);
+    const std::vector<double>* lam =
+        lit != ctx->lambda.end() && (int)lit->second.size() >= nf0 + np ? &lit->second : nullptr;
+    const bool force = ctx->opt.lazy_columns > 0;
+    std::set<std::string> filter_cols;
+    for (auto& f : s.filters) filter_cols.insert(f.col);
+    auto worthy = [&](const std::string& c, int op) {
+      if (filter_cols.count(c) || op < 0) return false;
+      if (force) return true;
+      return lam && (*lam)[op] * 64.0 <= (double)cols[cidx[c]]->width;
+    };
+    if (!force)
+      for (int p = 0; p < sp; p++) {
+        bool moved = false;
+        for (auto& k : s.probes[p].keys) moved |= worthy(k, nf0 + p - 1);
+        if (moved) {
+          sp = p;
+          break;
+        }
+      }
+    std::set<std::string> stage_cols;  // read in the stage phase (filters, stage-probe keys)
+    for (auto& f : s.filters) stage_cols.insert(f.col);
+    for (int p = 0; p < sp; p++)
+      for (auto& k : s.probes[p].keys) stage_cols.insert(k);
+    const int qop = nf0 + sp - 1;  // the rows reaching the queue passed this op
+    auto consider = [&](const std::string& c) {
+      if (!slot_of.count(c) && !stage_cols.count(c) && worthy(c, qop)) lazy.insert(c);
+    };
+    for (int p = sp; p < np; p++)
+      for (auto& k : s.probes[p].keys) consider(k);
+    for (auto& g : s.groups) consider(g.ref.name);
+    for (auto& t : s.value)
+      for (auto& f : t.f)
+        if (f.x.kind != RefIR::CONST) consider(f.x.name);
+    for (auto& c : lazy) {
+      li->lazy_w.push_back(cols[cidx[c]]->width);
+      li->lazy_reach.push_back(qop);
+    }
+  }
+
   // Expression pushdown: a value term whose factors are all columns, constants
-  // or stage-phase slots is computed before the queue and carried as one field.
+  // or stage-phase slots is computed before the queue and carried as one field
+  // (not when a factor is a lazy column: the drain computes it after the gather).
   auto stage_avail = [&](const std::string& n) {
-    return !slot_of.count(n) || slot_of[n] < sp;
+    return !lazy.count(n) && (!slot_of.count(n) || slot_of[n] < sp);
   };
   std::vector<bool> term_push(s.value.size(), false);
   for (size_t t = 0; t < s.value.size(); t++) {
@@ -369,7 +421,10 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   std::map<std::string, int> field;
   std::vector<int> fw;
   int nf = 0;
+  for (int f = 0; f < MAXQ; f++) d->qlazy[f] = -1;
+  d->rowid_field = -1;
   for (auto& c : qcols) {
+    if (lazy.count(c)) continue;
     d->push[nf] = Push{PUSH_COL, cidx[c]};
     fw.push_back(cols[cidx[c]]->width);
     field[c] = nf++;
@@ -392,7 +447,20 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
       fw.push_back(8);
       nf++;
     }
+  if (!lazy.empty()) {  // the row id the drain gathers lazy columns by
+    if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+    d->push[nf] = Push{PUSH_ROWID, 0};
+    fw.push_back(4);
+    d->rowid_field = nf++;
+  }
   d->npush = nf;
+  for (auto& c : qcols) {  // lazy columns: queue fields filled by the drain's gather
+    if (!lazy.count(c)) continue;
+    if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
+    d->qlazy[nf] = cidx[c];
+    fw.push_back(cols[cidx[c]]->width);
+    field[c] = nf++;
+  }
   for (int p = sp; p < np; p++) {
     const std::string& o = s.probes[p].out;
     if (!o.empty() && used_slots.count(o)) {
@@ -561,13 +629,18 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   li->nagg = d->nagg;
   // staged columns
   d->ncols = (int)cols.size();
-  int bpr = 0;
+  int bpr = 0, bpr_all = 0;
   for (int c = 0; c < d->ncols; c++) {
     d->col[c] = cols[c]->dev;
     d->colw[c] = cols[c]->width;
-    bpr += cols[c]->width;
+    d->lazy[c] = 0;
+    bpr_all += cols[c]->width;
   }
+  for (auto& c : lazy) d->lazy[cidx[c]] = 1;
+  for (int c = 0; c < d->ncols; c++)
+    if (!d->lazy[c]) bpr += cols[c]->width;
   li->bytes_per_row = bpr;
+  li->bytes_per_row_all = bpr_all;
   d->nrows = T.nrows;
   li->nfilt = d->nfilt;
   li->nprobe = np;

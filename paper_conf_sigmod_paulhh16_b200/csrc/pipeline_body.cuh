@@ -90,6 +90,18 @@ __device__ __forceinline__ void ld_rows(uint32_t a, int w, long long (&x)[RPL]) 
   }
 }
 
+// RPL rows of column c for one lane: from the staged tile, or — for a lazy
+// (late-materialised) column — gathered from HBM for the active rows only.
+__device__ __forceinline__ void ld_col(const PipeDesc& d, const PipeDesc& K, int c, uint32_t sb, int r0,
+                                       long long rowbase, const bool* act, long long (&x)[RPL]) {
+  if (K.lazy[c]) {
+#pragma unroll
+    for (int j = 0; j < RPL; j++) x[j] = act[j] ? ld_col_global(d.col[c], K.colw[c], rowbase + r0 + j) : 0;
+  } else {
+    ld_rows(sb + K.coloff[c] + r0 * K.colw[c], K.colw[c], x);
+  }
+}
+
 __device__ __forceinline__ long long qget(const PipeDesc& K, uint32_t qb, int f, int i) {
   const uint32_t a = qb + K.qoff[f];
   return K.qw[f] == 4 ? (long long)S<int>(a + i * 4) : S<long long>(a + i * 8);
@@ -201,6 +213,24 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
     const int e = j * 32 + lane;
     idx[j] = (qhead + e) & (QCAP - 1);
     p[j] = e < n;
+  }
+  if (K.rowid_field >= 0) {
+    // late materialisation: gather the lazy columns of the queued rows (all
+    // loads of a lane in flight together: one HBM round trip per drain)
+    uint32_t row[RPL];
+#pragma unroll
+    for (int j = 0; j < RPL; j++) row[j] = (uint32_t)qget(K, qb, K.rowid_field, idx[j]);
+    GPL_UNROLL
+    for (int f = 0; f < K.nfield; f++) {
+      const int c = K.qlazy[f];
+      if (c < 0) continue;
+      long long v[RPL];
+#pragma unroll
+      for (int j = 0; j < RPL; j++) v[j] = p[j] ? ld_col_global(d.col[c], K.colw[c], (long long)row[j]) : 0;
+#pragma unroll
+      for (int j = 0; j < RPL; j++)
+        if (p[j]) qput(K, qb, f, idx[j], v[j]);
+    }
   }
   GPL_UNROLL
   for (int pi = K.nsprobe; pi < K.nprobe; pi++) {
@@ -384,13 +414,15 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, (s0 + K.stage_rows >= rn) ? 1 : 0);
           uint32_t bytes = 0;
           GPL_UNROLL
-          for (int c = 0; c < K.ncols; c++) bytes += ((uint32_t)n * K.colw[c] + 15u) & ~15u;
+          for (int c = 0; c < K.ncols; c++)
+            if (!K.lazy[c]) bytes += ((uint32_t)n * K.colw[c] + 15u) & ~15u;
           mbar_arrive_expect_tx(&full[slot], bytes);
           unsigned char* dst = g_smem + K.off_ring + (unsigned long long)slot * K.slot_bytes;
           GPL_UNROLL
           for (int c = 0; c < K.ncols; c++)
-            bulk_g2s(dst + K.coloff[c], d.col[c] + row * K.colw[c], ((uint32_t)n * K.colw[c] + 15u) & ~15u,
-                     &full[slot], pol);
+            if (!K.lazy[c])
+              bulk_g2s(dst + K.coloff[c], d.col[c] + row * K.colw[c], ((uint32_t)n * K.colw[c] + 15u) & ~15u,
+                       &full[slot], pol);
           if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
         }
         t = t_next;
@@ -425,6 +457,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     const int n = h.z;
     if (n < 0) break;
     const uint32_t sb = (uint32_t)K.off_ring + slot * (uint32_t)K.slot_bytes;
+    const long long rowbase = ((long long)h.y << 32) | (long long)(uint32_t)h.x;  // lazy-column gathers
     const int nit = (n + 127) >> 7;
     bool released = false;
     // Each iteration takes npk (1 or 2) of the warp's 128-row packets,
@@ -452,7 +485,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         const Filt& F = K.filt[f];
 #pragma unroll
         for (int q = 0; q < NPMAX; q++) {
-          if (q >= npk) break;
+          if (!live[q]) continue;  // (a packet past the stage must not be read: smem bounds)
           long long x[RPL];
           ld_rows(sb + K.coloff[F.ref] + r0q[q] * K.colw[F.ref], K.colw[F.ref], x);
 #pragma unroll
@@ -474,17 +507,17 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
             for (int q = 0; q < NPMAX; q++) {
               long long k1[RPL];
-              if (q < npk) {
-                ld_rows(sb + K.coloff[P.k1] + r0q[q] * K.colw[P.k1], K.colw[P.k1], k1);
+              if (live[q]) {
+                ld_col(d, K, P.k1, sb, r0q[q], rowbase, p + q * RPL, k1);
               } else {
 #pragma unroll
                 for (int j = 0; j < RPL; j++) k1[j] = 0;
               }
 #pragma unroll
               for (int j = 0; j < RPL; j++) k[q * RPL + j] = (uint32_t)k1[j];
-              if (P.k2 >= 0 && q < npk) {
+              if (P.k2 >= 0 && live[q]) {
                 long long k2[RPL];
-                ld_rows(sb + K.coloff[P.k2] + r0q[q] * K.colw[P.k2], K.colw[P.k2], k2);
+                ld_col(d, K, P.k2, sb, r0q[q], rowbase, p + q * RPL, k2);
 #pragma unroll
                 for (int j = 0; j < RPL; j++) k[q * RPL + j] = (k[q * RPL + j] << 32) | (uint32_t)k2[j];
               }
@@ -551,7 +584,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             const uint32_t qa = qb + K.qoff[e];
             long long v[RPL];
             if (E.kind == PUSH_COL) {
-              ld_rows(sb + K.coloff[E.src] + r0 * K.colw[E.src], K.colw[E.src], v);
+              ld_col(d, K, E.src, sb, r0, rowbase, p + q * RPL, v);
+            } else if (E.kind == PUSH_ROWID) {  // for the drain's lazy-column gather
+#pragma unroll
+              for (int j = 0; j < RPL; j++) v[j] = rowbase + r0 + j;
             } else if (E.kind == PUSH_SREG) {
 #pragma unroll
               for (int j = 0; j < RPL; j++) v[j] = E.src == 0 ? sreg[0][q * RPL + j] : sreg[1][q * RPL + j];
@@ -564,7 +600,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
                 const Factor& F = T.f[f];
                 long long x[RPL];
                 if (F.field >= 0) {
-                  ld_rows(sb + K.coloff[F.field] + r0 * K.colw[F.field], K.colw[F.field], x);
+                  ld_col(d, K, F.field, sb, r0, rowbase, p + q * RPL, x);
                 } else {
 #pragma unroll
                   for (int j = 0; j < RPL; j++)

@@ -52,7 +52,8 @@ class _Stats(ctypes.Structure):
                 ("probe_split", ctypes.c_int32), ("op_pass", ctypes.c_int64 * 16),
                 ("kernel_ms", ctypes.c_double), ("predicted_ms", ctypes.c_double),
                 ("bytes_scanned", ctypes.c_double), ("agg_mode", ctypes.c_int32), ("kbe", ctypes.c_int32),
-                ("jit", ctypes.c_int32), ("reserved", ctypes.c_int32), ("intermediate_bytes", ctypes.c_double)]
+                ("jit", ctypes.c_int32), ("reserved", ctypes.c_int32), ("intermediate_bytes", ctypes.c_double),
+                ("bytes_full_scan", ctypes.c_double), ("lazy_columns", ctypes.c_int32), ("packets", ctypes.c_int32)]
 
 
 class _Result(ctypes.Structure):

@@ -113,7 +113,12 @@ def test_jit_compiles_every_plan():
             for s in segs[:-1]:
                 ctx.compile_plan(s)  # DIRECT build segments: the pipeline with an insert sink
                 ctx.build_hash(s)
-            ctx.compile_plan(segs[-1])
+            for lazy, packets in ((0, 1), (1, 2), (1, 1)):  # staged / late-materialised columns
+                ctx.set_option("lazy_columns", lazy)
+                ctx.set_option("packets", packets)
+                ctx.compile_plan(segs[-1])
+            ctx.set_option("lazy_columns", -1)
+            ctx.set_option("packets", -1)
         except gpl.GplError as e:
             if "NVRTC unavailable" in str(e):
                 pytest.skip(str(e))
