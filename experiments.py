@@ -141,13 +141,14 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
         bpr = max(1, int(rf.stats["bytes_scanned"] / max(1, rf.stats["rows_scanned"])))
         tw, rw = timed(True, (1 << 20) // bpr)
         assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs) == (rw.keys, rw.aggs), name
-        inp = rf.stats["bytes_scanned"]
+        inp = rf.stats.get("bytes_full_scan") or rf.stats["bytes_scanned"]  # the input: every column read, once
         ops = rf.stats["op_pass"]
         sel = (ops[0] / rf.stats["rows_scanned"]) if q == "Q14" and ops else None
         rows.append({"case": name, "selectivity": sel, "input_bytes": inp,
                      "fused_ms": tf, "kbe_ms": tk, "speedup": tk / tf,
                      "wo_ce_ms": tw, "wo_ce_tile_rows": rw.stats["tile_rows_used"],
                      "wo_ce_over_kbe": tw / tk, "wo_ce_intermediate_bytes": rw.stats["intermediate_bytes"],
+                     "fused_moved_bytes": rf.stats["bytes_scanned"], "fused_lazy_columns": rf.stats.get("lazy_columns"),
                      "fused_intermediate_bytes": rf.stats["intermediate_bytes"],
                      "kbe_intermediate_bytes": rk.stats["intermediate_bytes"],
                      "kbe_intermediate_over_input": rk.stats["intermediate_bytes"] / inp,
