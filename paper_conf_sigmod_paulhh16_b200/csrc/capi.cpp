@@ -301,8 +301,18 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       CK(cudaMalloc(&ctx->d_minmax, 64 * 2 * sizeof(long long)));
       ctx->minmax_cap = 64;
     }
-    auto cleanup = [&]() {
-      for (auto& c : t.cols) free_column(ctx, c);
+    auto cleanup = [&]() {  // a failed reload hands reused buffers back to the old table
+      auto oldt = ctx->tables.find(t.name);
+      for (auto& c : t.cols) {
+        bool given_back = false;
+        if (oldt != ctx->tables.end())
+          for (auto& oc : oldt->second.cols)
+            if (oc.dev == c.dev && c.owned && !oc.owned) {
+              oc.owned = true;
+              given_back = true;
+            }
+        if (!given_back) free_column(ctx, c);
+      }
     };
     for (int i = 0; i < ncols; i++) {
       Column c;
@@ -333,8 +343,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
         if (reuse) {
           c.dev = reuse->dev;
           c.cap_rows = reuse->cap_rows;
-          reuse->dev = nullptr;
-          reuse->owned = false;
+          reuse->owned = false;  // ownership moves to the new column (dev kept for the same-shape check)
         } else {
           cudaError_t e = cudaMalloc(&c.dev, (size_t)rows * c.width);
           if (e != cudaSuccess) {
@@ -365,6 +374,18 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
   }
   auto old = ctx->tables.find(t.name);
   if (old != ctx->tables.end()) {
+    // A reload into the same buffers with the same rows and value ranges keeps
+    // the table's version: prepared plans and query graphs depend only on
+    // those (hash tables built from it are still marked stale until rebuilt).
+    const Table& o = old->second;
+    bool same = o.nrows == t.nrows && o.cols.size() == t.cols.size();
+    for (size_t i = 0; same && i < t.cols.size(); i++) {
+      const Column& a = o.cols[i];
+      const Column& b = t.cols[i];
+      same = a.name == b.name && a.type == b.type && a.width == b.width && a.dev == b.dev && a.vmin == b.vmin &&
+             a.vmax == b.vmax && a.cap_rows == b.cap_rows;
+    }
+    if (same && !ctx->host_only) t.version = o.version;
     bool any_owned = false;
     for (auto& c : old->second.cols) any_owned |= c.owned && c.dev;
     if (!ctx->host_only && any_owned) cudaStreamSynchronize(ctx->stream);
@@ -398,7 +419,10 @@ GPL_API gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment) {
 
 // A prepared build is reusable while its scanned table, its destination and
 // source hash tables and the options are unchanged.
-static bool build_cache_valid(gpl_ctx* ctx, const PreparedBuild& P) {
+// `rebuilt`: hash tables that the same query rebuilds before this segment
+// runs (a whole-query graph replays every build), so their staleness after a
+// same-shape table reload does not matter.
+static bool build_cache_valid(gpl_ctx* ctx, const PreparedBuild& P, const std::set<int>* rebuilt = nullptr) {
   auto ti = ctx->tables.find(P.table);
   bool ok = ti != ctx->tables.end() && ti->second.version == P.table_version && P.opt_version == ctx->opt_version &&
             P.ht_index >= 0 && P.ht_index < (int)ctx->hts.size();
@@ -409,12 +433,12 @@ static bool build_cache_valid(gpl_ctx* ctx, const PreparedBuild& P) {
   for (size_t i = 0; ok && i < P.src_ids.size(); i++) {
     const HashTable& Hs = ctx->hts[P.src_ids[i]];
     const HTRef r = Hs.ref();
-    ok = Hs.valid && std::memcmp(&r, &P.desc.src[i], sizeof(HTRef)) == 0;
+    ok = (Hs.valid || (rebuilt && rebuilt->count(Hs.id))) && std::memcmp(&r, &P.desc.src[i], sizeof(HTRef)) == 0;
   }
   return ok;
 }
 
-static bool run_cache_valid(gpl_ctx* ctx, const PreparedRun& P) {
+static bool run_cache_valid(gpl_ctx* ctx, const PreparedRun& P, const std::set<int>* rebuilt = nullptr) {
   auto lam = ctx->lambda.find(P.text);
   const size_t lambda_n = lam == ctx->lambda.end() ? 0 : lam->second.size();
   auto ti = ctx->tables.find(P.li.table);
@@ -423,7 +447,7 @@ static bool run_cache_valid(gpl_ctx* ctx, const PreparedRun& P) {
   for (int i = 0; ok && i < P.desc.nht; i++) {
     const HashTable& H = ctx->hts[P.li.ht_ids[i]];
     const HTRef r = H.ref();
-    ok = H.valid && std::memcmp(&r, &P.desc.ht[i], sizeof(HTRef)) == 0;
+    ok = (H.valid || (rebuilt && rebuilt->count(H.id))) && std::memcmp(&r, &P.desc.ht[i], sizeof(HTRef)) == 0;
   }
   return ok;
 }
@@ -783,13 +807,16 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
   const std::string key = std::string(plan) + "\x1f" + std::to_string(tile_rows);
   const std::string run_key = segs.back() + "\x1f" + std::to_string(tile_rows);
   // are all segments prepared and still valid?
+  std::set<int> rebuilt;  // tables this query's build segments (re)build, in order
   auto all_valid = [&]() {
+    rebuilt.clear();
     for (size_t i = 0; i + 1 < segs.size(); i++) {
       auto b = ctx->build_cache.find(segs[i]);
-      if (b == ctx->build_cache.end() || !build_cache_valid(ctx, b->second)) return false;
+      if (b == ctx->build_cache.end() || !build_cache_valid(ctx, b->second, &rebuilt)) return false;
+      rebuilt.insert(b->second.ht_index);
     }
     auto r = ctx->run_cache.find(run_key);
-    return r != ctx->run_cache.end() && run_cache_valid(ctx, *r->second) && ctx->lambda.count(r->second->text);
+    return r != ctx->run_cache.end() && run_cache_valid(ctx, *r->second, &rebuilt) && ctx->lambda.count(r->second->text);
   };
   auto eager = [&]() -> gpl_status {
     for (size_t i = 0; i + 1 < segs.size(); i++) {
@@ -805,6 +832,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     if (all_valid()) {
       const auto t1 = std::chrono::steady_clock::now();
       CK(cudaGraphLaunch(g->second, ctx->stream));
+      for (int h : rebuilt) ctx->hts[h].valid = true;  // the replay rebuilt them
       if (trace) {
         const auto t2 = std::chrono::steady_clock::now();
         std::fprintf(stderr, "gpl_run_query host: validate %.1f us, cudaGraphLaunch %.1f us\n",

@@ -172,31 +172,52 @@ __device__ __forceinline__ bool any_n(const bool (&p)[NR]) {
 }
 
 // Build segments: the blocking hash build as the pipeline's last
-// operator. DIRECT cells start at 0 (= empty): bitmap cells by atomicOr,
-// 32-bit cells by atomicCAS, 1- and 2-byte cells by atomicOr into their word;
-// a non-empty old cell is a duplicate key (FK->PK joins only).
-__device__ __forceinline__ void insert_cell(const PipeDesc& d, const PipeDesc& K, long long key, long long pay) {
-  const unsigned long long ci = (unsigned long long)((long long)(int32_t)key - d.ins_kmin);
-  if (ci >= d.ins_nslots) {
-    atomicOr(d.err, ERR_CAPACITY);
-    return;
+// operator, N rows of a lane at a time. DIRECT cells start at 0 (= empty):
+// bitmap cells by atomicOr, 32-bit cells by atomicCAS, 1- and 2-byte cells by
+// atomicOr into their word; a non-empty old cell is a duplicate key (FK->PK
+// joins only). All N atomics are issued before any old value is examined, so
+// their round trips overlap (one latency per call, not N).
+template <int N>
+__device__ __forceinline__ void insert_cells(const PipeDesc& d, const PipeDesc& K, const long long (&key)[N],
+                                             const long long (&pay)[N], const bool (&act)[N]) {
+  bool in[N];
+  unsigned long long ci[N];
+  bool bad = false;
+#pragma unroll
+  for (int j = 0; j < N; j++) {
+    ci[j] = (unsigned long long)((long long)(int32_t)key[j] - d.ins_kmin);
+    in[j] = act[j] && ci[j] < d.ins_nslots;
+    bad |= act[j] && !in[j];
   }
-  if (K.ins_width == 0) {
-    const uint32_t bit = 1u << (ci & 31);
-    if (atomicOr((uint32_t*)d.ins_slots + (ci >> 5), bit) & bit) atomicOr(d.err, ERR_DUPKEY);
-    return;
+  if (bad) atomicOr(d.err, ERR_CAPACITY);
+  uint32_t old[N], m[N];
+#pragma unroll
+  for (int j = 0; j < N; j++) {
+    old[j] = 0;
+    m[j] = 0;
+    if (!in[j]) continue;
+    if (K.ins_width == 0) {
+      m[j] = 1u << (ci[j] & 31);
+      old[j] = atomicOr((uint32_t*)d.ins_slots + (ci[j] >> 5), m[j]);
+      continue;
+    }
+    long long pv = pay[j];
+    if (K.ins_ptransform == G_YEAR) pv = (int)pv / 10000;
+    const uint32_t v = (uint32_t)(pv - d.ins_pay_base + 1);
+    if (K.ins_width == 4) {
+      m[j] = 0xFFFFFFFFu;
+      old[j] = atomicCAS((uint32_t*)d.ins_slots + ci[j], 0u, v);
+    } else {
+      const unsigned long long byte = ci[j] * (unsigned long long)K.ins_width;
+      const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
+      m[j] = (K.ins_width == 1 ? 0xFFu : 0xFFFFu) << sh;
+      old[j] = atomicOr((uint32_t*)((char*)d.ins_slots + (byte & ~3ull)), v << sh);
+    }
   }
-  if (K.ins_ptransform == G_YEAR) pay = (int)pay / 10000;
-  const uint32_t v = (uint32_t)(pay - d.ins_pay_base + 1);
-  if (K.ins_width == 4) {
-    if (atomicCAS((uint32_t*)d.ins_slots + ci, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
-  } else {
-    const unsigned long long byte = ci * (unsigned long long)K.ins_width;
-    uint32_t* w = (uint32_t*)((char*)d.ins_slots + (byte & ~3ull));
-    const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
-    const uint32_t m = (K.ins_width == 1 ? 0xFFu : 0xFFFFu) << sh;
-    if (atomicOr(w, v << sh) & m) atomicOr(d.err, ERR_DUPKEY);
-  }
+  bool dup = false;
+#pragma unroll
+  for (int j = 0; j < N; j++) dup |= (old[j] & m[j]) != 0u;
+  if (dup) atomicOr(d.err, ERR_DUPKEY);
 }
 
 // Queue phase on up to RPL*32 queued survivors starting at qhead: lane `lane`
@@ -286,11 +307,13 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
   }
   if (!__any_sync(0xffffffffu, any4(p))) return;
   if (K.sink == SINK_INSERT) {
+    long long kx[RPL], px[RPL];
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
-      if (!p[j]) continue;
-      insert_cell(d, K, qget(K, qb, K.ins_kfield, idx[j]), K.ins_pfield >= 0 ? qget(K, qb, K.ins_pfield, idx[j]) : 0);
+      kx[j] = qget(K, qb, K.ins_kfield, idx[j]);
+      px[j] = K.ins_pfield >= 0 ? qget(K, qb, K.ins_pfield, idx[j]) : 0;
     }
+    insert_cells<RPL>(d, K, kx, px, p);
     return;
   }
   unsigned long long* stab = &S<unsigned long long>(K.off_agg);
@@ -541,27 +564,34 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
       }
       if (K.sink == SINK_INSERT && K.ins_kcol >= 0) {
         // build segment with every probe in the stage phase: insert straight
-        // from the staged tile (no survivor queue)
+        // from the staged tile (no survivor queue), all rows' atomics in flight
+        long long kx[NR], px[NR];
 #pragma unroll
         for (int q = 0; q < NPMAX; q++) {
-          if (!live[q]) break;
-          long long kx[RPL], px[RPL];
-          ld_rows(sb + K.coloff[K.ins_kcol] + r0q[q] * K.colw[K.ins_kcol], K.colw[K.ins_kcol], kx);
-          if (K.ins_pcol >= 0) {
-            ld_rows(sb + K.coloff[K.ins_pcol] + r0q[q] * K.colw[K.ins_pcol], K.colw[K.ins_pcol], px);
+          long long k4[RPL], p4[RPL];
+          if (live[q]) {
+            ld_rows(sb + K.coloff[K.ins_kcol] + r0q[q] * K.colw[K.ins_kcol], K.colw[K.ins_kcol], k4);
+            if (K.ins_pcol >= 0) ld_rows(sb + K.coloff[K.ins_pcol] + r0q[q] * K.colw[K.ins_pcol], K.colw[K.ins_pcol], p4);
           } else {
 #pragma unroll
-            for (int j = 0; j < RPL; j++) px[j] = K.ins_psreg == 0 ? sreg[0][q * RPL + j] : K.ins_psreg == 1 ? sreg[1][q * RPL + j] : 0;
+            for (int j = 0; j < RPL; j++) k4[j] = p4[j] = 0;
           }
 #pragma unroll
-          for (int j = 0; j < RPL; j++)
-            if (p[q * RPL + j]) insert_cell(d, K, kx[j], px[j]);
-          if (it0 + q * W + W >= nit) {
+          for (int j = 0; j < RPL; j++) {
+            kx[q * RPL + j] = k4[j];
+            px[q * RPL + j] = K.ins_pcol >= 0 ? p4[j]
+                              : K.ins_psreg == 0 ? sreg[0][q * RPL + j] : K.ins_psreg == 1 ? sreg[1][q * RPL + j] : 0;
+          }
+        }
+        // the ring slot is no longer read: release it before the atomics' round trip
+#pragma unroll
+        for (int q = 0; q < NPMAX; q++)
+          if (live[q] && it0 + q * W + W >= nit) {
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[slot]);
             released = true;
           }
-        }
+        insert_cells<NR>(d, K, kx, px, p);
         continue;
       }
       // A8 compaction into the warp's survivor queue (the on-chip channel), packet by packet
