@@ -309,15 +309,19 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
 __global__ void minmax_init_kernel(long long* out) {
   out[0] = LLONG_MAX;
   out[1] = LLONG_MIN;
+  out[2] = 0;  // descents: rows i with v[i] > v[i+1]
 }
 
 __global__ void __launch_bounds__(kThreads) minmax_kernel(const char* col, int w, long long n, long long* out) {
   long long mn = LLONG_MAX, mx = LLONG_MIN;
+  unsigned long long desc = 0;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     const long long v = ld_col_global(col, w, i);
     mn = min(mn, v);
     mx = max(mx, v);
+    if (i + 1 < n && v > ld_col_global(col, w, i + 1)) desc++;
   }
+  if (desc) atomicAdd((unsigned long long*)&out[2], desc);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));

@@ -176,7 +176,7 @@ GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
   if ((e = cudaHostGetDevicePointer((void**)&ctx->h_stage_dev, ctx->h_stage, 0)) != cudaSuccess)
     return bad(e, "mapped staging");
   if ((e = cudaMallocHost((void**)&ctx->h_err, 64)) != cudaSuccess) return bad(e, "pinned error word");
-  if ((e = cudaMallocHost((void**)&ctx->h_minmax, 64 * 2 * sizeof(long long))) != cudaSuccess)
+  if ((e = cudaMallocHost((void**)&ctx->h_minmax, 64 * 3 * sizeof(long long))) != cudaSuccess)
     return bad(e, "pinned min/max");
   if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
   if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
@@ -239,6 +239,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
     o.kbe_tile_rows = v;
   } else if (k == "lazy_columns") {
     o.lazy_columns = v < 0 ? -1 : v > 0 ? 1 : 0;
+  } else if (k == "clustered") {
+    o.clustered = v != 0 ? 1 : 0;
   } else if (k == "build_pipeline") {
     o.build_pipeline = v != 0 ? 1 : 0;
   } else if (k == "jit") {
@@ -283,10 +285,14 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       c.host.assign((const char*)cols[i].data, (const char*)cols[i].data + nrows * c.width);
       c.vmin = LLONG_MAX;
       c.vmax = LLONG_MIN;
+      c.sorted = true;
+      long long prev = LLONG_MIN;
       for (int64_t r = 0; r < nrows; r++) {
         long long v = c.width == 4 ? (long long)((const int32_t*)c.host.data())[r] : ((const int64_t*)c.host.data())[r];
         c.vmin = std::min<long long>(c.vmin, v);
         c.vmax = std::max<long long>(c.vmax, v);
+        c.sorted = c.sorted && v >= prev;
+        prev = v;
       }
       if (nrows == 0) c.vmin = c.vmax = 0;
       t.cols.push_back(std::move(c));
@@ -298,7 +304,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       if (ctx->d_minmax) cudaFree(ctx->d_minmax);
       ctx->d_minmax = nullptr;
       ctx->minmax_cap = 0;
-      CK(cudaMalloc(&ctx->d_minmax, 64 * 2 * sizeof(long long)));
+      CK(cudaMalloc(&ctx->d_minmax, 64 * 3 * sizeof(long long)));
       ctx->minmax_cap = 64;
     }
     auto cleanup = [&]() {  // a failed reload hands reused buffers back to the old table
@@ -362,14 +368,15 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
         t.cols.pop_back();
       }
       t.cols.push_back(c);
-      CK(launch_minmax(c.dev, c.width, nrows, ctx->d_minmax + 2 * i, ctx->stream));
+      CK(launch_minmax(c.dev, c.width, nrows, ctx->d_minmax + 3 * i, ctx->stream));
     }
     long long* mm = ctx->h_minmax;  // pinned (h_stage holds the last run's copied-out results)
-    CK(cudaMemcpyAsync(mm, ctx->d_minmax, sizeof(long long) * 2 * ncols, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(mm, ctx->d_minmax, sizeof(long long) * 3 * ncols, cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     for (int i = 0; i < ncols; i++) {
-      t.cols[i].vmin = nrows ? mm[2 * i] : 0;
-      t.cols[i].vmax = nrows ? mm[2 * i + 1] : 0;
+      t.cols[i].vmin = nrows ? mm[3 * i] : 0;
+      t.cols[i].vmax = nrows ? mm[3 * i + 1] : 0;
+      t.cols[i].sorted = mm[3 * i + 2] == 0;  // no descent between consecutive rows
     }
   }
   auto old = ctx->tables.find(t.name);
@@ -383,7 +390,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       const Column& a = o.cols[i];
       const Column& b = t.cols[i];
       same = a.name == b.name && a.type == b.type && a.width == b.width && a.dev == b.dev && a.vmin == b.vmin &&
-             a.vmax == b.vmax && a.cap_rows == b.cap_rows;
+             a.vmax == b.vmax && a.cap_rows == b.cap_rows && a.sorted == b.sorted;
     }
     if (same && !ctx->host_only) t.version = o.version;
     bool any_owned = false;

@@ -156,6 +156,11 @@ struct PipeDesc {
   int32_t qw[MAXQ];      // field width in bytes (4 or 8)
   int32_t qbytes;        // bytes of one warp's queue
   int32_t qlazy[MAXQ];   // >= 0: field f is lazy column qlazy[f], gathered by the drain via the row id
+  // clustered probe: stage probe cl_probe reads a DIRECT table by a key column
+  // (cl_col) sorted in the fact table, so one stage's keys span a narrow cell
+  // range; the producer TMA-stages those cells (<= cl_cap bytes at slot offset
+  // cl_off) beside the columns and the probe reads shared memory
+  int32_t cl_probe, cl_col, cl_off, cl_cap;
   int32_t rowid_field;   // queue field holding the row id (-1: no lazy column)
   int32_t term_field[MAXTERM];  // >= 0: term t was computed in the stage phase into this field
   Term sterm[MAXTERM];          // stage-phase form of pushed-down terms (stage refs)

@@ -42,12 +42,22 @@ constexpr int kFixed = 4096;
 int align128(int x) { return (x + 127) & ~127; }
 }  // namespace
 
+// Cell buffer of a clustered probe per ring slot: a stage's key range spans
+// up to 4 keys per row (TPC-H order keys are 1 in 4 dense; a wider range
+// falls back to probing the table in memory).
+int cl_cap_bytes(const PipeDesc& d, int S) {
+  if (d.cl_probe < 0) return 0;
+  const int w = d.ht[d.probe[d.cl_probe].ht].width;
+  return align128((w == 0 ? (4 * S + 7) / 8 : 4 * S * w) + 32);
+}
+
 int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps) {
   int q = warps * d.qbytes;
   int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   int slot = 0;
   for (int c = 0; c < d.ncols; c++)
     if (!d.lazy[c]) slot += align128(stage_rows * d.colw[c]);
+  slot += cl_cap_bytes(d, stage_rows);
   return align128(kFixed + q) + align128(agg) + align128(d.smem_tables_bytes) + depth * slot;
 }
 
@@ -73,6 +83,9 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
     d->coloff[i] = off;
     off += align128(c.stage_rows * d->colw[i]);
   }
+  d->cl_off = off;
+  d->cl_cap = cl_cap_bytes(*d, c.stage_rows);
+  off += d->cl_cap;
   d->slot_bytes = off;
   d->smem_bytes = d->off_ring + c.depth * off;
 }
@@ -137,7 +150,8 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
     return bytes <= 64e3 ? 80.0 : bytes <= L2_eff ? 1200.0 : 2000.0;
   };
   double lat_stage = 0, lat_queue = 0;
-  for (int p = 0; p < li.nprobe; p++) (p < d.nsprobe ? lat_stage : lat_queue) += lat(li.probe_ht[p]);
+  for (int p = 0; p < li.nprobe; p++)  // a clustered probe reads its staged cells from shared memory
+    (p < d.nsprobe ? lat_stage : lat_queue) += p == d.cl_probe ? 40.0 : lat(li.probe_ht[p]);
   // lazy columns: one HBM gather round trip per drain (per 128 queued rows)
   if (!li.lazy_reach.empty()) lat_queue += 2000.0;
   // cycles per warp iteration of `npack` packets: the stage-phase probe

@@ -21,6 +21,7 @@ struct Column {
   bool owned = false;
   int64_t cap_rows = 0;
   int64_t vmin = 0, vmax = 0;
+  bool sorted = false;     // non-decreasing (e.g. lineitem.l_orderkey): enables clustered probe staging
   std::vector<char> host;  // host-only context storage
 };
 
@@ -135,6 +136,7 @@ struct Options {
   int64_t jit = 1;
   int64_t lazy_columns = -1;   // late materialisation: -1 auto (from λ), 0 off, 1 every eligible column
   int64_t build_pipeline = 1;
+  int64_t clustered = 1;       // stage the cell range of a probe keyed by a sorted column (0: probe L2/HBM)
   int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
   double hbm_gbs = -1;
 };

@@ -126,6 +126,10 @@ std::string shape_source(const PipeDesc& d) {
   }
   I("qbytes", d.qbytes);
   I("rowid_field", d.rowid_field);
+  I("cl_probe", d.cl_probe);
+  I("cl_col", d.cl_col);
+  I("cl_off", d.cl_off);
+  I("cl_cap", d.cl_cap);
   for (int f = 0; f < MAXQ; f++) o << "  k.qlazy[" << f << "] = " << d.qlazy[f] << ";\n";
   auto term = [&](const char* arr, int t, const Term& T) {
     o << "  k." << arr << "[" << t << "].sign = " << T.sign << "; k." << arr << "[" << t << "].nfact = " << T.nfact << ";\n";

@@ -49,6 +49,7 @@ cudaError_t launch_clear(const ClearList& L, int num_sms, cudaStream_t s);
 cudaError_t launch_copyout(const unsigned long long* src, unsigned long long* host_dst, int words, cudaStream_t s);
 
 // Column min/max (int32 or int64 column, n rows) -> out[0] = min, out[1] = max.
+// out[2] = number of descents (rows i with v[i] > v[i+1]): 0 means sorted.
 cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s);
 
 // KBE baseline: kernel-at-a-time with materialisation. Returns the

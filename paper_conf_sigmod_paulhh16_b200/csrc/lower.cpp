@@ -200,6 +200,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   *d = PipeDesc{};
   *li = LowerInfo{};
   if (s.is_build && !ins) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
+  d->cl_probe = d->cl_col = -1;
   if (ins && (!s.is_build || ins->kind != HT_DIRECT || s.key.size() != 1)) {
     *err = "pipelined build needs a single-key DIRECT build segment";
     return GPL_E_PLAN;
@@ -536,6 +537,19 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
       D.out = (!P.out.empty() && field.count(P.out)) ? field[P.out] : -1;
     }
     li->op_names.push_back(std::string(P.kind == P_INNER ? "probe " : P.kind == P_SEMI ? "semi " : "mark ") + P.ht);
+  }
+  // Clustered probe: the first stage-phase probe reads a DIRECT table (not
+  // already in shared memory) by one key column that is sorted in the fact
+  // table (lineitem.l_orderkey: lineitem is generated per order) -> the
+  // producer stages each stage's cell range with the columns.
+  if (!ins && sp >= 1 && ctx->opt.clustered != 0) {
+    const Probe& P0 = d->probe[0];
+    const HashTable& H0 = *pht[0];
+    if (H0.kind == HT_DIRECT && P0.k2 < 0 && cols[P0.k1]->sorted && cols[P0.k1]->width == 4 &&
+        d->ht_smem_off[P0.ht] < 0 && H0.bytes() < (1ull << 31)) {
+      d->cl_probe = 0;
+      d->cl_col = P0.k1;
+    }
   }
   // where residuals
   d->nresid = (int)s.wheres.size();

@@ -63,8 +63,10 @@ constexpr int kOffFull = 0;       // unsigned long long[kMaxDepth]
 constexpr int kOffEmpty = 64;     // unsigned long long[kMaxDepth]
 constexpr int kOffHdr = 128;      // int4[kMaxDepth]
 constexpr int kOffHtp = 256;      // HTP[MAXHT]
+constexpr int kOffHdr2 = 768;     // int4[kMaxDepth]: clustered-probe cell range (start lo, hi, bytes)
 constexpr int kOffCnt = 1024;     // unsigned long long[kMaxWarps][MAXOPS]
-static_assert(kOffHtp + MAXHT * sizeof(HTP) <= kOffCnt, "HTP region overflow");
+static_assert(kOffHtp + MAXHT * sizeof(HTP) <= kOffHdr2, "HTP region overflow");
+static_assert(kOffHdr2 + kMaxDepth * 16 <= kOffCnt, "header region overflow");
 static_assert(kOffCnt + kMaxWarps * MAXOPS * 8 <= 4096, "fixed region overflow");
 
 template <class T>
@@ -144,6 +146,39 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int 
     return;
   }
   ht_probe_n<N>(h, kind, width, key, act, hit, pay);
+}
+
+// Clustered probe (DIRECT table, key column sorted in the fact table): the
+// producer staged the cells of the stage's key range [klo, khi] at smem byte
+// `base`, starting at table byte `start`; a key outside the staged bytes (only
+// possible if the column is not sorted after all) reads the table in HBM.
+template <int N>
+__device__ __forceinline__ void probe_rows_cl(const PipeDesc& K, const HTP& h, int t, const unsigned long long (&key)[N],
+                                              const bool (&act)[N], bool (&hit)[N], long long (&pay)[N], uint32_t base,
+                                              long long start, int size) {
+  const int width = K.ht[t].width;
+#pragma unroll
+  for (int j = 0; j < N; j++) {
+    const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
+    const bool in = act[j] && idx < h.nslots;
+    const long long b = (width == 0 ? (long long)(idx >> 5) * 4 : (long long)idx * width) - start;
+    const bool staged = b >= 0 && b < size;
+    uint32_t x = 0;
+    if (in) {
+      if (width == 0) {
+        const uint32_t wd = staged ? S<uint32_t>(base + (uint32_t)b) : __ldg((const uint32_t*)h.slots + (idx >> 5));
+        x = (wd >> (idx & 31)) & 1u;
+      } else if (width == 1) {
+        x = staged ? (uint32_t)S<unsigned char>(base + (uint32_t)b) : (uint32_t)__ldg((const unsigned char*)h.slots + idx);
+      } else if (width == 2) {
+        x = staged ? (uint32_t)S<unsigned short>(base + (uint32_t)b) : (uint32_t)__ldg((const unsigned short*)h.slots + idx);
+      } else {
+        x = staged ? S<uint32_t>(base + (uint32_t)b) : __ldg((const uint32_t*)h.slots + idx);
+      }
+    }
+    hit[j] = x != 0;
+    pay[j] = width == 0 ? 1 : (long long)x - 1 + h.pay_base;
+  }
 }
 
 __device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
@@ -384,6 +419,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   unsigned long long* full = &S<unsigned long long>(kOffFull);
   unsigned long long* empty = &S<unsigned long long>(kOffEmpty);
   int4* hdr = &S<int4>(kOffHdr);
+  int4* hdr2 = &S<int4>(kOffHdr2);  // clustered probe: staged cell range per slot
   HTP* htp = &S<HTP>(kOffHtp);
   unsigned long long* cnt_all = &S<unsigned long long>(kOffCnt);
   unsigned long long* stab = &S<unsigned long long>(K.off_agg);
@@ -421,34 +457,87 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     if (lane == 0) {
       const unsigned long long pol = policy_evict_first();
       uint32_t slot = 0, phase = 0;
-      // the next tile is claimed before the current one's copies are issued,
-      // so the claim's global-atomic round trip overlaps them (with small
-      // tiles it would otherwise bound the producer: one claim per stage)
+      // Stages are visited in order; the next stage is computed (and the tile
+      // after it claimed) while the current one is issued, so the claim's
+      // global-atomic round trip and — for a clustered probe — the loads of
+      // the next stage's first/last key overlap the current stage's copies.
+      const long long S = K.stage_rows;
       unsigned long long t = atomicAdd(d.tile_counter, 1ull);
-      for (;;) {
-        const long long r0 = (long long)t * d.tile_rows;
-        if (r0 >= d.nrows) break;
-        const unsigned long long t_next = atomicAdd(d.tile_counter, 1ull);
+      unsigned long long tn = atomicAdd(d.tile_counter, 1ull);  // claim of the following tile
+      long long r0 = (long long)t * d.tile_rows, s0 = 0;
+      long long row = r0;
+      int n = r0 < d.nrows ? (int)min(S, min(d.tile_rows, d.nrows - r0)) : 0;
+      long long klo = 0, khi = 0;  // clustered probe: key range of the current stage
+      if (K.cl_probe >= 0 && n > 0) {
+        klo = ld_col_global(d.col[K.cl_col], 4, row);
+        khi = ld_col_global(d.col[K.cl_col], 4, row + n - 1);
+      }
+      while (n > 0) {
         const long long rn = min(d.tile_rows, d.nrows - r0);
-        for (long long s0 = 0; s0 < rn; s0 += K.stage_rows) {
-          const int n = (int)min((long long)K.stage_rows, rn - s0);
-          mbar_wait(&empty[slot], phase ^ 1u);
-          const long long row = r0 + s0;
-          hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, (s0 + K.stage_rows >= rn) ? 1 : 0);
-          uint32_t bytes = 0;
-          GPL_UNROLL
-          for (int c = 0; c < K.ncols; c++)
-            if (!K.lazy[c]) bytes += ((uint32_t)n * K.colw[c] + 15u) & ~15u;
-          mbar_arrive_expect_tx(&full[slot], bytes);
-          unsigned char* dst = g_smem + K.off_ring + (unsigned long long)slot * K.slot_bytes;
-          GPL_UNROLL
-          for (int c = 0; c < K.ncols; c++)
-            if (!K.lazy[c])
-              bulk_g2s(dst + K.coloff[c], d.col[c] + row * K.colw[c], ((uint32_t)n * K.colw[c] + 15u) & ~15u,
-                       &full[slot], pol);
-          if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
+        const bool last_of_tile = s0 + S >= rn;
+        // next stage (same tile, else the claimed tile)
+        long long r0n = r0, s0n = s0 + S, rown = 0;
+        int nn = 0;
+        if (!last_of_tile) {
+          rown = r0 + s0n;
+          nn = (int)min(S, rn - s0n);
+        } else {
+          r0n = (long long)tn * d.tile_rows;
+          s0n = 0;
+          if (r0n < d.nrows) {
+            rown = r0n;
+            nn = (int)min(S, min(d.tile_rows, d.nrows - r0n));
+            tn = atomicAdd(d.tile_counter, 1ull);
+          }
         }
-        t = t_next;
+        long long klo_n = 0, khi_n = 0;
+        if (K.cl_probe >= 0 && nn > 0) {
+          klo_n = ld_col_global(d.col[K.cl_col], 4, rown);
+          khi_n = ld_col_global(d.col[K.cl_col], 4, rown + nn - 1);
+        }
+        mbar_wait(&empty[slot], phase ^ 1u);
+        hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, last_of_tile ? 1 : 0);
+        uint32_t bytes = 0;
+        GPL_UNROLL
+        for (int c = 0; c < K.ncols; c++)
+          if (!K.lazy[c]) bytes += ((uint32_t)n * K.colw[c] + 15u) & ~15u;
+        // clustered probe: the table cells of [klo, khi] (16-B aligned), when
+        // they fit the slot's cell buffer; else the consumers probe HBM/L2
+        long long cl_start = 0;
+        uint32_t cl_size = 0;
+        if (K.cl_probe >= 0) {
+          const HTP& H = htp[K.probe[K.cl_probe].ht];
+          long long clo = klo - (long long)H.kmin, chi = khi - (long long)H.kmin;
+          clo = max(clo, 0ll);
+          chi = min(chi, (long long)H.nslots - 1);
+          if (clo <= chi) {
+            const int w = K.ht[K.probe[K.cl_probe].ht].width;
+            const long long blo = w == 0 ? (clo >> 5) * 4 : clo * w;
+            const long long bhi = w == 0 ? ((chi >> 5) + 1) * 4 : (chi + 1) * w;
+            cl_start = blo & ~15ll;
+            const long long sz = ((bhi + 15) & ~15ll) - cl_start;
+            if (sz <= K.cl_cap) cl_size = (uint32_t)sz;
+          }
+          hdr2[slot] = make_int4((int)(cl_start & 0xffffffff), (int)(cl_start >> 32), (int)cl_size, 0);
+          bytes += cl_size;
+        }
+        mbar_arrive_expect_tx(&full[slot], bytes);
+        unsigned char* dst = g_smem + K.off_ring + (unsigned long long)slot * K.slot_bytes;
+        GPL_UNROLL
+        for (int c = 0; c < K.ncols; c++)
+          if (!K.lazy[c])
+            bulk_g2s(dst + K.coloff[c], d.col[c] + row * K.colw[c], ((uint32_t)n * K.colw[c] + 15u) & ~15u,
+                     &full[slot], pol);
+        if (cl_size)
+          bulk_g2s(dst + K.cl_off, (const char*)htp[K.probe[K.cl_probe].ht].slots + cl_start, cl_size, &full[slot],
+                   policy_evict_last());
+        if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
+        row = rown;
+        n = nn;
+        r0 = r0n;
+        s0 = s0n;
+        klo = klo_n;
+        khi = khi_n;
       }
       mbar_wait(&empty[slot], phase ^ 1u);
       hdr[slot] = make_int4(0, 0, -1, 0);
@@ -481,6 +570,13 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     if (n < 0) break;
     const uint32_t sb = (uint32_t)K.off_ring + slot * (uint32_t)K.slot_bytes;
     const long long rowbase = ((long long)h.y << 32) | (long long)(uint32_t)h.x;  // lazy-column gathers
+    long long cl_start = 0;
+    int cl_size = 0;
+    if (K.cl_probe >= 0) {
+      const int4 h2 = hdr2[slot];
+      cl_start = ((long long)h2.y << 32) | (long long)(uint32_t)h2.x;
+      cl_size = h2.z;
+    }
     const int nit = (n + 127) >> 7;
     bool released = false;
     // Each iteration takes npk (1 or 2) of the warp's 128-row packets,
@@ -547,7 +643,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             }
             bool hit[NR];
             long long v[NR];
-            probe_rows<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v);
+            if (sp == K.cl_probe && cl_size > 0)
+              probe_rows_cl<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v, sb + (uint32_t)K.cl_off, cl_start, cl_size);
+            else
+              probe_rows<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v);
 #pragma unroll
             for (int j = 0; j < NR; j++) {
               if (P.kind == P_MARK) {

@@ -368,3 +368,32 @@ def test_same_shape_reload_replays_graph_exactly(ctx):
         for _ in range(3):
             r = queries.run_query(ctx, "Q5", cur)
             assert r.keys == o.keys and r.aggs == o.aggs
+
+
+@pytest.mark.parametrize("q", ["Q5", "Q7", "Q8"])
+def test_clustered_probe_exact(ctx, q):
+    """Clustered probe: lineitem is sorted by l_orderkey, so the first probe
+    (HT_O) of a stage reads a narrow cell range that the producer stages by TMA
+    with the columns. On, off, unsorted keys (disabled) and keys too sparse for
+    the cell buffer (per-stage fallback to HBM): all exact."""
+    db = tpchgen.generate(0.05, seed=91)
+    cases = [("sorted", db)]
+    sparse = tpchgen.generate(0.05, seed=91)
+    for t, c in (("orders", "o_orderkey"), ("lineitem", "l_orderkey")):
+        sparse.tables[t][c] = sparse.tables[t][c] * 37  # stage key span >> cell buffer
+    cases.append(("sparse", sparse))
+    shuffled = tpchgen.generate(0.05, seed=91)
+    perm = np.random.default_rng(3).permutation(shuffled.nrows("lineitem"))
+    shuffled.tables["lineitem"] = {c: v[perm].copy() for c, v in shuffled.tables["lineitem"].items()}
+    cases.append(("unsorted", shuffled))
+    try:
+        for name, cur in cases:
+            o = oracle.run(q, cur)
+            for cl in (1, 0):
+                ctx.set_option("clustered", cl)
+                for tile in (0, 7000):
+                    for _ in range(2):  # eager + λ-driven replan
+                        r = _gpu(ctx, cur, q, tile_rows=tile)
+                        assert r.keys == o.keys and r.aggs == o.aggs, (q, name, cl, tile)
+    finally:
+        ctx.set_option("clustered", 1)

@@ -17,8 +17,9 @@ queries.load_database(ctx, ddb, borrow=True)
 for q in qs:
     text = queries.plan_text(q, db)
     ref = None
-    for mode in (0, -1, 1):
+    for mode, cl in ((0, 0), (-1, 0), (-1, 1), (0, 1)):
         ctx.set_option("lazy_columns", mode)
+        ctx.set_option("clustered", cl)
         ts = []
         for i in range(7):
             flush.zero_(); ctx.run_query(text); r = ctx.fetch_result()
@@ -27,7 +28,8 @@ for q in qs:
         assert (r.keys, r.aggs) == ref
         t = statistics.median(ts)
         st = r.stats
-        print(f"{q} SF{sf} lazy={mode:2d}: kernel {t*1e3:8.1f} us  lazy_cols={st['lazy_columns']} P={st['packets']} split={st['probe_split']} "
+        print(f"{q} SF{sf} lazy={mode:2d} clustered={cl}: kernel {t*1e3:8.1f} us  lazy_cols={st['lazy_columns']} P={st['packets']} split={st['probe_split']} "
               f"bytes {st['bytes_scanned']/1e9:.3f}/{st['bytes_full_scan']/1e9:.3f} GB -> {st['bytes_scanned']/t/1e6:.0f} GB/s "
               f"(full-scan equiv {st['bytes_full_scan']/t/1e6:.0f} GB/s)", flush=True)
     ctx.set_option("lazy_columns", -1)
+    ctx.set_option("clustered", 1)
