@@ -381,7 +381,8 @@ def main():
         "op_pass": stats["op_pass"],
         "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
         "jit": stats.get("jit"),
-        "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split")}
+        "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split",
+                                              "builds_tuned", "build_ms_model", "build_ms")}
                      if tuned else None),
     }
     if rank == 0:

@@ -46,11 +46,13 @@ def _setup(q, sf, seed, tables=None):
     return db, ctx, flush, stream
 
 
-def tile_sweep(q="Q5", sf=1.0, seed=20160626, reps=5, out=None):
+def tile_sweep(q="Q5", sf=1.0, seed=20160626, reps=5, out=None, calibration=None, setup=None):
     import torch
 
     from paper_conf_sigmod_paulhh16_b200 import queries
-    db, ctx, flush, stream = _setup(q, sf, seed)
+    db, ctx, flush, stream = setup or _setup(q, sf, seed)
+    if calibration is not None:
+        ctx.set_calibration(calibration)  # Γ points ([] = the uncalibrated model)
     segs = queries.segments(queries.plan_text(q, db))
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 
@@ -81,6 +83,7 @@ def tile_sweep(q="Q5", sf=1.0, seed=20160626, reps=5, out=None):
     best_meas = min(rows, key=lambda x: x["measured_ms"])
     best_pred = min(rows, key=lambda x: (x["predicted_ms"], -x["tile_rows"]))
     summary = {"experiment": "tile_sweep (config 2)", "query": q, "sf": sf,
+               "gamma_calibrated": bool(calibration),
                "auto": {"tile_rows": r_auto.stats["tile_rows_used"], "measured_ms": t_auto,
                         "predicted_ms": r_auto.stats["predicted_ms"]},
                "measured_argmin_tile_rows": best_meas["tile_rows"], "measured_min_ms": best_meas["measured_ms"],
@@ -88,6 +91,87 @@ def tile_sweep(q="Q5", sf=1.0, seed=20160626, reps=5, out=None):
                "model_pick_vs_best": t_auto / best_meas["measured_ms"],
                "mean_rel_error": statistics.mean(x["rel_error"] for x in rows),
                "results_identical_across_tiles": True, "points": rows}
+    if out:
+        with open(out, "w") as f:
+            json.dump(summary, f, indent=1)
+    return summary
+
+
+def gamma_calibration(q="Q5", sfs=(1.0, 10.0), seed=20160626, out=None):
+    """NEXT-1: the channel calibration Γ(n, s, k, d) (§2.1, Eq 1, Fig 2 / Fig 23 analog:
+    ring throughput vs data size for each ring depth n and stage size s), then the config-2 tile sweep of
+    `q` at each SF with the uncalibrated and the Γ-calibrated model: Eq 10 relative error and the model
+    pick's gap to the measured best, both ways (the paper's Figs 11-13 / 24-26 check of its model)."""
+    setup = _setup(q, sfs[0], seed)
+    ctx = setup[1]
+    pts = ctx.calibrate()
+    curves = {}
+    for p in pts:
+        curves.setdefault(f"n={p['ring_depth']} s={p['stage_rows']} k={p['ctas_per_sm']}", []).append(
+            {"rows": p["rows"], "MB": p["bytes"] / 1e6, "ms": p["ms"], "gbs": p["gbs"], "t0_us": 1e3 * p["t0_ms"]})
+    peak = max(p["gbs"] for p in pts)
+    best_shape = max(curves, key=lambda k: curves[k][-1]["gbs"])
+    sweeps = []
+    for i, sf in enumerate(sfs):
+        st = setup if i == 0 else _setup(q, sf, seed)
+        if i > 0:
+            st[1].set_calibration(pts)
+        for cal in ([], pts):
+            s = tile_sweep(q, sf, seed, calibration=cal, setup=st)
+            sweeps.append({k: s[k] for k in ("query", "sf", "gamma_calibrated", "mean_rel_error", "model_pick_vs_best",
+                                              "measured_argmin_tile_rows", "model_argmin_tile_rows", "auto")})
+            sweeps[-1]["points"] = [{k: x[k] for k in ("tile_rows", "measured_ms", "predicted_ms", "rel_error")}
+                                    for x in s["points"]]
+    summary = {"experiment": "gamma calibration (NEXT-1; Fig 2/23 + Eq 10 analog)",
+               "gamma_peak_gbs": peak, "best_shape_at_largest_d": best_shape,
+               "curves": curves, "sweeps": sweeps}
+    if out:
+        with open(out, "w") as f:
+            json.dump(summary, f, indent=1)
+    return summary
+
+
+def warp_sweep(q="Q8", sf=10.0, seed=20160626, reps=5, out=None):
+    """Figs 14-15 analog: the work-group setting S_i ↦ consumer warps per CTA W (2..16), other knobs
+    from the model; measured kernel time vs the model's estimate (Eq 10 error) and the model's delay term
+    (t_tail: the Eq 8 imbalance between producer and consumers plus the last wave), results identical."""
+    from paper_conf_sigmod_paulhh16_b200 import queries
+    db, ctx, flush, stream = _setup(q, sf, seed)
+    segs = queries.segments(queries.plan_text(q, db))
+    rows, ref = [], None
+    for w in (2, 4, 6, 8, 12, 16):
+        ctx.set_option("consumer_warps", w)
+        ts, r = [], None
+        try:
+            for i in range(reps + 2):
+                for s in segs[:-1]:
+                    ctx.build_hash(s)
+                flush.zero_()
+                ctx.run_plan(segs[-1])
+                r = ctx.fetch_result()
+                if i >= 2:
+                    ts.append(r.stats["kernel_ms"])
+        except Exception as e:  # a shape that does not fit
+            rows.append({"consumer_warps": w, "error": str(e)})
+            continue
+        if ref is None:
+            ref = (r.keys, r.aggs)
+        assert (r.keys, r.aggs) == ref, "result changed with consumer warps"
+        m = ctx.choose_tile_rows(segs[-1], 0)
+        t = statistics.median(ts)
+        rows.append({"consumer_warps": w, "measured_ms": t, "predicted_ms": r.stats["predicted_ms"],
+                     "rel_error": abs(t - r.stats["predicted_ms"]) / t, "model_delay_tail_ms": m["t_tail_ms"],
+                     "stage_rows": r.stats["stage_rows"], "ring_depth": r.stats["ring_depth"],
+                     "tile_rows": r.stats["tile_rows_used"]})
+    ctx.set_option("consumer_warps", -1)
+    ok = [x for x in rows if "measured_ms" in x]
+    best_meas = min(ok, key=lambda x: x["measured_ms"])
+    best_pred = min(ok, key=lambda x: x["predicted_ms"])
+    summary = {"experiment": "consumer-warp sweep (Figs 14-15 analog)", "query": q, "sf": sf,
+               "measured_argmin_warps": best_meas["consumer_warps"], "model_argmin_warps": best_pred["consumer_warps"],
+               "model_pick_vs_best": best_pred["measured_ms"] / best_meas["measured_ms"],
+               "mean_rel_error": statistics.mean(x["rel_error"] for x in ok), "results_identical": True,
+               "points": rows}
     if out:
         with open(out, "w") as f:
             json.dump(summary, f, indent=1)
@@ -166,6 +250,13 @@ if __name__ == "__main__":
     which = sys.argv[1] if len(sys.argv) > 1 else "sweep"
     if which == "sweep":
         s = tile_sweep(out=os.path.join(ROOT, "gpurun_out", "sweep_config2.json"))
+    elif which == "gamma":
+        s = gamma_calibration(out=os.path.join(ROOT, "gpurun_out", "gamma_calibration.json"))
+        s.pop("curves", None)
+        for x in s["sweeps"]:
+            x.pop("points", None)
+    elif which == "warps":
+        s = warp_sweep(out=os.path.join(ROOT, "gpurun_out", "warp_sweep.json"))
     else:
         s = kbe_compare(out=os.path.join(ROOT, "gpurun_out", "kbe_config5.json"))
     s.pop("points", None)

@@ -121,7 +121,9 @@ typedef struct {
   int32_t candidates;          /* gpl_autotune: shapes measured                                    */
   double measured_ms;          /* gpl_autotune: median kernel time of the chosen shape            */
   int32_t probe_split;         /* probes run before the survivor queue (autotune: measured best)  */
-  int32_t pad_;
+  int32_t builds_tuned;        /* gpl_autotune: pipelined (DIRECT) build segments measured         */
+  double build_ms_model;       /* gpl_autotune: Σ median build time at the model's shapes          */
+  double build_ms;             /* gpl_autotune: Σ median build time at the pinned (best) shapes    */
 } gpl_model_report;
 
 /* Create a context on CUDA device `device` enqueuing on `cuda_stream` (a
@@ -232,16 +234,54 @@ gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t
  * split (how many probes run before the survivor queue), times each on the
  * device with L2 flushed (median of 3), and pins the fastest for this probe
  * segment; later gpl_run_plan / gpl_run_query calls with tile_rows = 0 use
- * it until gpl_set_option is called. Synchronises. out (optional) receives
- * the chosen shape, its model estimate and its measured time. */
+ * it until gpl_set_option is called. Every build segment that runs as a
+ * pipeline (DIRECT tables) is tuned the same way: the model's per-shape
+ * candidates are timed on a rebuild of the table (identical contents) and
+ * the fastest is pinned for that segment. Synchronises. out (optional)
+ * receives the chosen shape, its model estimate and its measured time, and
+ * the build segments' summed times at the model's and the pinned shapes. */
 gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_candidates, gpl_model_report* out);
+
+/* One point of the channel calibration Γ (Eq 1; the
+ * producer -> consumer chain of P:83): the throughput of the fused kernel's
+ * shared-memory ring for one shape (ring depth = the "number of channels",
+ * stage rows = the packet analog, CTAs per SM) at one data size. */
+typedef struct {
+  int32_t ring_depth, stage_rows, ctas_per_sm, consumer_warps;
+  int64_t rows;    /* rows streamed (16 B each: 2 int32 + 1 int64 columns)             */
+  double bytes;    /* rows x 16                                                         */
+  double ms;       /* median kernel time, L2 flushed before each repetition             */
+  double t0_ms;    /* the same shape over an empty input (launch + prologue)            */
+  double gbs;      /* Γ = bytes / (ms - t0_ms) / 1e9                                    */
+} gpl_gamma_point;
+
+/* Calibrate Γ: for every ring shape (depth {2,3,4} x
+ * stage rows {1024,2048,4096} x CTAs/SM {1,2}; shapes that do not fit shared
+ * memory are skipped) and every size in rows[0..n_rows) (NULL/0: 2^19..2^26
+ * rows), stream a synthetic zero table through the pipeline kernel and time
+ * it on the device. The points replace the copy bandwidth in the A9 model
+ * (predict: Γ of the candidate shape at d = rows x bytes/row; t0 as its
+ * launch term) until gpl_set_calibration / gpl_set_option("use_gamma", 0).
+ * Options, tables and hash tables of the context are left as they were.
+ * out (optional, capacity cap) receives the points; *n_out their count
+ * (GPL_E_CAPACITY if cap is too small — the calibration is still applied).
+ * Synchronises; takes seconds (one plan-specialised compile per shape). */
+gpl_status gpl_calibrate(gpl_ctx* ctx, const int64_t* rows, int32_t n_rows, gpl_gamma_point* out, int32_t cap,
+                         int32_t* n_out);
+
+/* Load a saved calibration (points as gpl_calibrate returned them; n = 0
+ * clears it: the model falls back to the copy bandwidth). Host only. */
+gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t n);
 
 /* Tuning knobs (tests / sweeps): "stage_rows", "ring_depth",
  * "consumer_warps", "ctas_per_sm", "probe_split" (-1 = auto), "hash_load_pct",
  * "jit" (1 = plan-specialised kernels, default; 0 = generic kernel),
  * "build_pipeline" (1 = DIRECT build segments run through the fused pipeline
  * with an insert sink, default; 0 = the standalone build kernels),
- * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input).
+ * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input),
+ * "use_gamma" (1 = the model uses the Γ calibration when loaded, default),
+ * "use_profile" (1 = the model fits its consumer cost to the plan's first
+ * timed run after its λ profile, Table 2 "profiling input", default).
  * value < 0 restores automatic selection. */
 gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value);
 

@@ -34,8 +34,9 @@ DEFAULT_PARAMS = {
     "Q8": (19950101, 19961231),    # P:650-651  between (inclusive)
     "Q9": (1000,),                 # P:677  p_partKey < 1000 (reading #5)
     "Q14": (19950901, 19951001),   # P:688-689  [1995-09-01, 1995-10-01)
+    "Q3": (19950315,),             # TPC-H Q3 [EXT] (NEXT-4 workload): o_orderdate < d < l_shipdate
 }
-QUERY_IDS = {"L1": 1, "Q5": 5, "Q7": 7, "Q8": 8, "Q9": 9, "Q14": 14}
+QUERY_IDS = {"L1": 1, "Q5": 5, "Q7": 7, "Q8": 8, "Q9": 9, "Q14": 14, "Q3": 3}
 # Result schema (keys, aggs) per query: count(*) first, then the SUMs.
 SCHEMA = {
     "L1": ((), ("count", "sum_charge")),
@@ -44,7 +45,12 @@ SCHEMA = {
     "Q8": (("o_year",), ("count", "brazil_volume", "volume")),
     "Q9": (("nation", "o_year"), ("count", "sum_profit")),
     "Q14": ((), ("count", "promo_volume", "total_volume")),
+    "Q3": (("l_orderkey", "o_orderdate"), ("count", "revenue")),
 }
+# ORDER BY / LIMIT of the queries that have one on the GPU (Q3: revenue desc,
+# o_orderdate asc, LIMIT 10; ties after that broken by l_orderkey asc — our
+# reading, so that the 10 rows are unique).
+ORDER_LIMIT = {"Q3": 10}
 
 
 class _OracleDB(ctypes.Structure):
@@ -64,6 +70,8 @@ class _OracleDB(ctypes.Structure):
         ("dict_r_name", P), ("n_dict_r_name", ctypes.c_int32),
         ("dict_n_name", P), ("n_dict_n_name", ctypes.c_int32),
         ("dict_p_type", P), ("n_dict_p_type", ctypes.c_int32),
+        ("c_mktsegment", P),
+        ("dict_c_mktsegment", P), ("n_dict_c_mktsegment", ctypes.c_int32),
     ]
 
 
@@ -140,6 +148,11 @@ def _db_struct(db):
     s.dict_r_name, s.n_dict_r_name = ctypes.cast(d1, ctypes.c_void_p), len(db.r_name)
     s.dict_n_name, s.n_dict_n_name = ctypes.cast(d2, ctypes.c_void_p), len(db.n_name)
     s.dict_p_type, s.n_dict_p_type = ctypes.cast(d3, ctypes.c_void_p), len(db.p_type)
+    s.c_mktsegment = p("customer", "c_mktsegment")
+    segs = getattr(db, "c_mktsegment", ["AUTOMOBILE", "BUILDING", "FURNITURE", "HOUSEHOLD", "MACHINERY"])
+    d4 = _strings(segs)
+    keep.append(d4)
+    s.dict_c_mktsegment, s.n_dict_c_mktsegment = ctypes.cast(d4, ctypes.c_void_p), len(segs)
     return s, keep
 
 
@@ -150,7 +163,7 @@ def run(query: str, db, params=None, lineitem_range=None) -> Result:
     pr = np.array(list(params) + [0] * (4 - len(params)), dtype=np.int32)
     s, keep = _db_struct(db)
     lb, le = lineitem_range if lineitem_range is not None else (0, s.n_lineitem)
-    cap = 4096
+    cap = 4096 if query != "Q3" else max(4096, s.n_orders)  # Q3 groups <= orders
     keys = np.zeros(cap * 4, dtype=np.int32)
     aggs = np.zeros(cap * 4 * 2, dtype=np.int64)
     r = _OracleResult()
@@ -171,6 +184,15 @@ def run(query: str, db, params=None, lineitem_range=None) -> Result:
         out_a.append(row)
     del keep
     return Result(query, out_k, out_a)
+
+
+def order_limit(query: str, r: Result) -> Result:
+    """ORDER BY / LIMIT of `query` applied to the full group set (exact integers).
+    Q3: revenue desc, o_orderdate asc, then l_orderkey asc (reading), LIMIT 10."""
+    if query != "Q3":
+        raise ValueError(f"{query} has no GPU ORDER BY/LIMIT")
+    rows = sorted(zip(r.keys, r.aggs), key=lambda ka: (-ka[1][1], ka[0][1], ka[0][0]))[:ORDER_LIMIT[query]]
+    return Result(query, [k for k, _ in rows], [a for _, a in rows])
 
 
 def timed_run(query: str, db, params=None, lineitem_range=None):

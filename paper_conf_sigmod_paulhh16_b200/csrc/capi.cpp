@@ -243,6 +243,10 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
     o.clustered = v != 0 ? 1 : 0;
   } else if (k == "build_pipeline") {
     o.build_pipeline = v != 0 ? 1 : 0;
+  } else if (k == "use_profile") {
+    o.use_profile = v != 0 ? 1 : 0;
+  } else if (k == "use_gamma") {
+    o.use_gamma = v != 0 ? 1 : 0;
   } else if (k == "jit") {
     o.jit = v != 0 ? 1 : 0;
   } else if (k == "hbm_mbs") {
@@ -450,7 +454,7 @@ static bool run_cache_valid(gpl_ctx* ctx, const PreparedRun& P, const std::set<i
   const size_t lambda_n = lam == ctx->lambda.end() ? 0 : lam->second.size();
   auto ti = ctx->tables.find(P.li.table);
   bool ok = ti != ctx->tables.end() && ti->second.version == P.table_version && P.opt_version == ctx->opt_version &&
-            P.lambda_n == lambda_n;
+            P.lambda_n == lambda_n && P.profiled == (ctx->profile.count(P.text) > 0);
   for (int i = 0; ok && i < P.desc.nht; i++) {
     const HashTable& H = ctx->hts[P.li.ht_ids[i]];
     const HTRef r = H.ref();
@@ -470,7 +474,10 @@ static cudaError_t record_event(gpl_ctx* ctx, cudaEvent_t ev) {
 
 // A DIRECT build segment lowered to the fused pipeline with an insert sink
 // (shape + schedule; the caller fills the run-time pointers).
-static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTable& H, PipeDesc* pd, Config* cfg) {
+// A shape pinned by gpl_autotune (keyed by the segment text) wins over the
+// model; shortlist (optional) receives the model's per-shape candidates.
+static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTable& H, PipeDesc* pd, Config* cfg,
+                                   std::vector<Config>* shortlist = nullptr) {
   LowerInfo li;
   std::string err;
   gpl_status st;
@@ -484,7 +491,14 @@ static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTab
     const HashTable& h = ctx->hts[li.ht_ids[i]];
     li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
   }
-  if (!choose_config(ctx, *pd, li, pd->nrows, 0, cfg, &err)) return fail(ctx, GPL_E_ARG, err);
+  auto tu = shortlist ? ctx->tuned.end() : ctx->tuned.find(s.text);
+  if (tu != ctx->tuned.end()) {
+    const TunedShape& t = tu->second;
+    *cfg = predict(ctx, *pd, li, std::max<int64_t>(pd->nrows, 1), t.tile_rows, t.stage_rows, t.depth, t.warps,
+                   t.ctas_per_sm, t.npack);
+  } else if (!choose_config(ctx, *pd, li, pd->nrows, 0, cfg, &err, shortlist)) {
+    return fail(ctx, GPL_E_ARG, err);
+  }
   apply_config(pd, li, *cfg);
   return GPL_OK;
 }
@@ -669,6 +683,7 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
       if (h.slots == d->ht[i].slots)
         li->ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
   }
+  apply_profile(ctx, *d, li, seg->text);
   if (tile_rows < 0) return fail(ctx, GPL_E_ARG, "tile_rows must be >= 0");
   auto tu = tile_rows == 0 ? ctx->tuned.find(seg->text) : ctx->tuned.end();
   if (tu != ctx->tuned.end()) {  // shape pinned by gpl_autotune
@@ -718,6 +733,7 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
   P.table_version = ctx->tables[seg.table].version;
   P.opt_version = ctx->opt_version;
   P.lambda_n = lambda_n;
+  P.profiled = ctx->profile.count(P.text) > 0;
   std::string jerr;
   P.fn = resolve_pipeline_fn(d, ctx->opt.jit != 0, &jerr);
   P.jit = ctx->opt.jit != 0 && jerr.empty();
@@ -931,6 +947,82 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
   return GPL_OK;
 }
 
+// gpl_autotune for one build segment that runs as a pipeline (DIRECT table):
+// time the model's per-shape candidates on rebuilds of the same table
+// (L2 flushed, median of 3) and pin the fastest under the segment's text.
+// Earlier tables of the plan are already built; the contents never change.
+static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush, size_t fbytes,
+                             int32_t max_candidates, double* model_ms, double* best_ms_out, int* tuned) {
+  Segment s;
+  std::string err;
+  if (!parse_segment(text, &s, &err) || !s.is_build) return GPL_OK;
+  auto hi = ctx->ht_by_name.find(s.name);
+  if (hi == ctx->ht_by_name.end() || !ctx->opt.build_pipeline) return GPL_OK;
+  const HashTable H = ctx->hts[hi->second];
+  if (H.kind != HT_DIRECT) return GPL_OK;
+  ctx->tuned.erase(s.text);
+  PipeDesc pd;
+  Config c0;
+  std::vector<Config> cs;
+  gpl_status st = lower_build_pipe(ctx, s, H, &pd, &c0, &cs);
+  if (st) return st;
+  if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
+  bool has0 = false;
+  for (const Config& c : cs)
+    has0 |= c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
+            c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack;
+  if (!has0) cs.insert(cs.begin(), c0);
+  cudaEvent_t a = nullptr, b = nullptr;
+  CK(cudaEventCreate(&a));
+  CK(cudaEventCreate(&b));
+  double best_ms = 1e300, m0 = -1;
+  TunedShape best;
+  for (const Config& c : cs) {
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, -2, c.npack};
+    ctx->tuned[s.text] = t;
+    ctx->build_cache.erase(text);
+    std::vector<float> ms;
+    st = GPL_OK;
+    for (int rep = 0; rep < 4 && !st; rep++) {
+      if (cudaMemsetAsync(flush, rep, fbytes, ctx->stream) != cudaSuccess) break;
+      cudaEventRecord(a, ctx->stream);
+      st = gpl_build_hash(ctx, text.c_str(), nullptr);
+      cudaEventRecord(b, ctx->stream);
+      if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) break;
+      float m = 0;
+      cudaEventElapsedTime(&m, a, b);
+      if (rep > 0) ms.push_back(m);
+    }
+    if (st || ms.size() < 3) {  // a shape that cannot run (resources) is skipped
+      st = GPL_OK;
+      ctx->err.clear();
+      cudaGetLastError();
+      continue;
+    }
+    std::sort(ms.begin(), ms.end());
+    if (m0 < 0 && c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
+        c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack)
+      m0 = ms[1];
+    if (ms[1] < best_ms) {
+      best_ms = ms[1];
+      best = t;
+    }
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  if (best_ms < 1e300) {
+    ctx->tuned[s.text] = best;
+    (*tuned)++;
+    *best_ms_out += best_ms;
+    *model_ms += m0 < 0 ? best_ms : m0;
+  } else {
+    ctx->tuned.erase(s.text);
+  }
+  ctx->build_cache.erase(text);
+  // leave the table built at the pinned shape
+  return gpl_build_hash(ctx, text.c_str(), nullptr);
+}
+
 GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_candidates, gpl_model_report* out) {
   if (!ctx || !plan) return GPL_E_ARG;
   ctx->err.clear();
@@ -940,6 +1032,19 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   if (segs.empty()) return fail(ctx, GPL_E_PLAN, "plan has no segment");
   for (size_t i = 0; i + 1 < segs.size(); i++)
     if ((st = gpl_build_hash(ctx, segs[i].c_str(), nullptr))) return st;
+  // L2 flush buffer (2x L2) so every timing starts cold, as the bench does
+  void* flush = nullptr;
+  const size_t fbytes = (size_t)2 * ctx->l2_bytes;
+  CK(cudaMalloc(&flush, fbytes));
+  struct FreeOnExit {
+    void* p;
+    ~FreeOnExit() { cudaFree(p); }
+  } flush_guard{flush};
+  int builds_tuned = 0;
+  double build_ms_model = 0, build_ms = 0;
+  for (size_t i = 0; i + 1 < segs.size(); i++)
+    if ((st = tune_build(ctx, segs[i], flush, fbytes, max_candidates, &build_ms_model, &build_ms, &builds_tuned)))
+      return st;
   const std::string& probe = segs.back();
   // one eager run profiles λ (the split and the model depend on it)
   if ((st = gpl_run_plan(ctx, probe.c_str(), 0))) return st;
@@ -976,6 +1081,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
       const HashTable& h = ctx->hts[ls.ht_ids[i]];
       ls.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
     }
+    apply_profile(ctx, ds, &ls, seg.text);
     Config best_model;
     std::vector<Config> cs;
     if (!choose_config(ctx, ds, ls, ds.nrows, 0, &best_model, &err, &cs)) {
@@ -992,10 +1098,6 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
       li = ls;
     }
   }
-  // L2 flush buffer (2x L2) so every timing starts cold, as the bench does
-  void* flush = nullptr;
-  const size_t fbytes = (size_t)2 * ctx->l2_bytes;
-  CK(cudaMalloc(&flush, fbytes));
   double best_ms = 1e300;
   TunedShape best;
   int best_eff_split = -1;
@@ -1029,7 +1131,6 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
       best_eff_split = cand_split_eff[ci];
     }
   }
-  cudaFree(flush);
   take_device_errors(ctx);
   if (tried == 0) {
     ctx->tuned.erase(seg.text);
@@ -1060,6 +1161,9 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     out->candidates = tried;
     out->measured_ms = best_ms;
     out->probe_split = best_eff_split;
+    out->builds_tuned = builds_tuned;
+    out->build_ms_model = build_ms_model;
+    out->build_ms = build_ms;
   }
   return GPL_OK;
 }
@@ -1211,6 +1315,20 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
     std::vector<double> lam;
     for (int i = 0; i < li.nops; i++) lam.push_back((double)ops[i] / (double)S.rows_scanned);
     ctx->lambda[ctx->last.run->text] = lam;
+  } else if (!ctx->last.kbe && ctx->last.timed && S.kernel_ms > 0 && S.rows_scanned > 0 && ctx->last.run->lambda_n > 0 &&
+             !ctx->profile.count(ctx->last.run->text)) {
+    // the first timed run planned with λ: the model's profiling input
+    const PreparedRun& R = *ctx->last.run;
+    RunProfile p;
+    p.nrows = R.desc.nrows;
+    p.tile_rows = R.desc.tile_rows;
+    p.stage_rows = R.desc.stage_rows;
+    p.depth = R.desc.depth;
+    p.warps = R.desc.nwarps;
+    p.npack = R.desc.npack;
+    p.ctas_per_sm = std::max(1, R.grid / std::max(1, ctx->sms));
+    p.kernel_ms = S.kernel_ms;
+    ctx->profile[R.text] = p;
   }
   out->stats = S;
   if (bits) {
@@ -1279,6 +1397,7 @@ GPL_API gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment,
   for (int i = 0; i < d.nht; i++)
     for (auto& h : ctx->hts)
       if (h.slots == d.ht[i].slots) li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+  apply_profile(ctx, d, &li, s.text);
   Config c;
   const int64_t N = n_rows > 0 ? n_rows : d.nrows;
   if (!choose_config(ctx, d, li, N, 0, &c, &err)) return fail(ctx, GPL_E_ARG, err);

@@ -36,6 +36,7 @@ namespace gpl {
 
 int pipeline_fixed_smem();
 int pipeline_max_consumer_warps();
+bool gamma_lookup(const gpl_ctx* ctx, int depth, int stage_rows, int k, double bytes, double* gbs, double* t0_ms);
 
 namespace {
 constexpr int kFixed = 4096;
@@ -116,7 +117,20 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
     b += 32.0 * (op >= 0 && op < (int)li.lambda.size() ? li.lambda[op] : 0.05);
   }
   const double f_sm = 1.9e9;
-  const double B_sm = 1.6 * B / ctx->sms;  // one SM's TMA/L2 fill cap
+  // Eq 1 analog: the calibrated ring throughput Γ(n, s, k, d) of this shape at
+  // d = N·b (gpl_calibrate) replaces the copy bandwidth as the streaming rate,
+  // and the shape's measured empty-input time replaces the launch estimate
+  double G_ring = B, t0_cal = -1;
+  {
+    double g = 0, t0 = 0;
+    if (gamma_lookup(ctx, depth, S, k, (double)std::max<int64_t>(N, 1) * b, &g, &t0)) {
+      G_ring = g * 1e9;
+      t0_cal = t0;
+    }
+  }
+  G_ring *= std::max(li.bw_factor, 1.0);
+  c.bw_gbs = G_ring / 1e9;
+  const double B_sm = 1.6 * G_ring / ctx->sms;  // one SM's TMA/L2 fill cap
   N = std::max<int64_t>(N, 1);
 
   // λ: fraction of rows reaching each operator (previous run, else defaults)
@@ -158,7 +172,8 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // latency is paid once per iteration (all npack*4 loads of a lane in flight)
   const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);
   const double w_eff = (double)std::min(W, S / (128 * npack)) * k;          // warps with work per stage
-  const double rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 * npack / crit);  // per SM
+  const double rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 * npack / crit) /
+                          std::max(li.cons_factor, 1e-3);  // per SM (profile-fitted scale)
   const double R_cons = rows_cyc * f_sm * b;                                // bytes/s one SM's consumers absorb
   const double t_cons = (double)N / (rows_cyc * f_sm * ctx->sms);
 
@@ -167,8 +182,8 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   const int64_t G = c.grid;
   const int64_t waves = (tiles + G - 1) / G;
   const int64_t last = tiles - (waves - 1) * G;
-  const double rate_full = std::min(std::min(B_sm, R_cons) / k, B / (double)std::min<int64_t>(G, tiles));
-  const double rate_last = std::min(std::min(B_sm, R_cons) / k, B / (double)last);
+  const double rate_full = std::min(std::min(B_sm, R_cons) / k, G_ring / (double)std::min<int64_t>(G, tiles));
+  const double rate_last = std::min(std::min(B_sm, R_cons) / k, G_ring / (double)last);
   const double t_tile = tile * b / rate_full;
   const double last_rows = (double)(N - (tiles - 1) * tile);
   const double t_last = (last == 1 ? last_rows : (double)tile) * b / rate_last;
@@ -181,7 +196,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // Eq 8/9 analog
   const double tp = t_prod + t_chan, tc = t_cons;
   const double T = 0.5 * (tp + tc) + 0.5 * std::fabs(tp - tc);
-  c.t_launch_ms = 4e-3 + 1e3 * (depth * t_stage);  // launch + prologue + ring fill
+  c.t_launch_ms = t0_cal >= 0 ? t0_cal : 4e-3 + 1e3 * (depth * t_stage);  // launch + prologue + ring fill
   c.t_stream_ms = 1e3 * (N * b / B);
   c.t_probe_ms = 1e3 * probe_bytes / B;
   c.t_tail_ms = 1e3 * (T - N * b / B - probe_bytes / B);
@@ -242,6 +257,44 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
     std::sort(shortlist->begin(), shortlist->end(), [](const Config& a, const Config& b) { return a.pred_ms < b.pred_ms; });
   }
   return true;
+}
+
+void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const std::string& plan_text) {
+  li->cons_factor = 1;
+  li->bw_factor = 1;
+  auto it = ctx->profile.find(plan_text);
+  if (it == ctx->profile.end() || !ctx->opt.use_profile) return;
+  const RunProfile& p = it->second;
+  auto pred = [&](double f) {
+    li->cons_factor = f;
+    return predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
+                   p.ctas_per_sm, p.npack).pred_ms;
+  };
+  // the prediction is non-decreasing in the factor: geometric bisection
+  double lo = 0.05, hi = 50;
+  if (pred(lo) >= p.kernel_ms) {
+    // faster than the stream bound (an L2-resident input): fit the streaming rate instead
+    li->cons_factor = lo;
+    double blo = 1, bhi = 32;
+    auto predb = [&](double f) {
+      li->bw_factor = f;
+      return pred(lo);
+    };
+    if (predb(bhi) >= p.kernel_ms) return;
+    for (int i = 0; i < 40; i++) {
+      const double mid = std::sqrt(blo * bhi);
+      (predb(mid) > p.kernel_ms ? blo : bhi) = mid;
+    }
+    li->bw_factor = std::sqrt(blo * bhi);
+    // then the consumer scale at that rate
+    if (pred(lo) >= p.kernel_ms) return;
+  }
+  if (pred(hi) <= p.kernel_ms) { li->cons_factor = hi; return; }
+  for (int i = 0; i < 40; i++) {
+    const double mid = std::sqrt(lo * hi);
+    (pred(mid) < p.kernel_ms ? lo : hi) = mid;
+  }
+  li->cons_factor = std::sqrt(lo * hi);
 }
 
 int choose_split(const gpl_ctx* ctx, const Segment& s) {

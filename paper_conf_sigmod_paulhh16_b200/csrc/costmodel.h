@@ -34,6 +34,11 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
 // Fill the schedule and shared-memory layout fields of d from c.
 void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c);
 
+// Table 2 "profiling input": fit li->cons_factor, the scale of
+// the consumer warps' per-iteration cost, so that the model reproduces the
+// plan's profiled run (shape, rows, measured kernel time); 1 without one.
+void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const std::string& plan_text);
+
 // Probes run before the survivor queue, from the previous run's pass
 // fractions (the paper profiles the first tile) or a heuristic.
 int choose_split(const gpl_ctx* ctx, const Segment& s);

@@ -6,6 +6,7 @@
 #include <map>
 #include <memory>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "common.h"
@@ -78,6 +79,16 @@ struct LowerInfo {
   int nprobe = 0, nfilt = 0;
   bool has_groups = false;
   std::vector<double> lambda;     // cumulative pass fraction after each op (previous run)
+  double cons_factor = 1;         // consumer cost scale fitted to the plan's profiled run (costmodel apply_profile)
+  double bw_factor = 1;           // streaming-rate scale, fitted only when the run beat the model's stream bound (L2-resident input)
+};
+
+// The first timed run of a plan after its λ profile (the paper profiles the
+// first tile): its shape, rows and measured kernel time.
+struct RunProfile {
+  int64_t nrows = 0, tile_rows = 0;
+  int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1, npack = 1;
+  double kernel_ms = 0;
 };
 
 struct PreparedRun;
@@ -101,6 +112,7 @@ struct PreparedRun {
   bool jit = false;
   uint64_t table_version = 0, opt_version = 0;
   size_t lambda_n = 0;
+  bool profiled = false;  // planned with the plan's RunProfile
   std::string text;
 };
 
@@ -139,6 +151,16 @@ struct Options {
   int64_t clustered = 1;       // stage the cell range of a probe keyed by a sorted column (0: probe L2/HBM)
   int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
   double hbm_gbs = -1;
+  int64_t use_gamma = 1;       // the model uses the channel calibration Γ when one is loaded
+  int64_t use_profile = 1;     // the model fits its consumer cost to the plan's profiled run
+};
+
+// Γ of one ring shape (gpl_calibrate, Eq 1): (bytes, GB/s)
+// points sorted by bytes, and the shape's empty-input kernel time.
+struct GammaCurve {
+  int depth = 0, stage_rows = 0, ctas_per_sm = 0;
+  double t0_ms = 0;
+  std::vector<std::pair<double, double>> pts;
 };
 
 }  // namespace gpl
@@ -166,12 +188,14 @@ struct gpl_ctx {
   gpl::Options opt;
   uint64_t opt_version = 1;  // bumped by gpl_set_option (invalidates prepared plans)
   std::map<std::string, std::vector<double>> lambda;  // plan text -> per-op pass fraction (A9 "profile the first tile")
+  std::map<std::string, gpl::RunProfile> profile;     // plan text -> first timed run after λ (consumer cost fit)
   // prepared-plan caches (keyed by segment text [+ tile_rows]); validated on
   // every use against table versions, hash-table refs and options
   std::map<std::string, std::shared_ptr<gpl::PreparedRun>> run_cache;
   std::map<std::string, gpl::PreparedBuild> build_cache;
   // gpl_run_query: whole-query CUDA graphs (builds + fused run), keyed by plan text + tile_rows
   std::map<std::string, cudaGraphExec_t> graphs;
+  std::map<std::tuple<int, int, int>, gpl::GammaCurve> gamma;  // (depth, stage rows, CTAs/SM) -> Γ(d)
   std::map<std::string, gpl::TunedShape> tuned;  // probe segment text -> measured-best shape
   std::map<std::string, std::vector<std::string>> plan_segs;  // gpl_run_query: plan text -> segments
   void* h_stage = nullptr;  // pinned host staging for one packed D2H of results

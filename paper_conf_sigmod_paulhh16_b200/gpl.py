@@ -28,8 +28,8 @@ GPL_COPY, GPL_BORROW = 0, 1
 EXPORTED = ["gpl_create", "gpl_destroy", "gpl_load_columns", "gpl_build_hash", "gpl_run_plan",
             "gpl_run_plan_kbe", "gpl_fetch_result", "gpl_fetch_partials", "gpl_decode_partials",
             "gpl_merge_partials", "gpl_sync", "gpl_choose_tile_rows", "gpl_set_option",
-            "gpl_check_plan", "gpl_compile_plan", "gpl_run_query", "gpl_autotune", "gpl_last_error",
-            "gpl_version"]
+            "gpl_check_plan", "gpl_compile_plan", "gpl_run_query", "gpl_autotune", "gpl_calibrate",
+            "gpl_set_calibration", "gpl_last_error", "gpl_version"]
 
 
 class GplError(RuntimeError):
@@ -68,7 +68,14 @@ class _Model(ctypes.Structure):
                 ("t_stream_ms", ctypes.c_double), ("t_probe_ms", ctypes.c_double), ("t_tail_ms", ctypes.c_double),
                 ("t_launch_ms", ctypes.c_double), ("bw_gbs", ctypes.c_double), ("smem_bytes", ctypes.c_int32),
                 ("feasible", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32), ("candidates", ctypes.c_int32),
-                ("measured_ms", ctypes.c_double), ("probe_split", ctypes.c_int32), ("pad_", ctypes.c_int32)]
+                ("measured_ms", ctypes.c_double), ("probe_split", ctypes.c_int32), ("builds_tuned", ctypes.c_int32),
+                ("build_ms_model", ctypes.c_double), ("build_ms", ctypes.c_double)]
+
+
+class _Gamma(ctypes.Structure):  # gpl_gamma_point
+    _fields_ = [("ring_depth", ctypes.c_int32), ("stage_rows", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32),
+                ("consumer_warps", ctypes.c_int32), ("rows", ctypes.c_int64), ("bytes", ctypes.c_double),
+                ("ms", ctypes.c_double), ("t0_ms", ctypes.c_double), ("gbs", ctypes.c_double)]
 
 
 _lib = None
@@ -102,6 +109,8 @@ def load_library():
         "gpl_compile_plan": ([P, ctypes.c_char_p, I64], I32),
         "gpl_run_query": ([P, ctypes.c_char_p, I64], I32),
         "gpl_autotune": ([P, ctypes.c_char_p, I32, ctypes.POINTER(_Model)], I32),
+        "gpl_calibrate": ([P, ctypes.POINTER(I64), I32, ctypes.POINTER(_Gamma), I32, ctypes.POINTER(I32)], I32),
+        "gpl_set_calibration": ([P, ctypes.POINTER(_Gamma), I32], I32),
         "gpl_last_error": ([P], ctypes.c_char_p),
         "gpl_version": ([], ctypes.c_char_p),
     }
@@ -241,6 +250,24 @@ class Context:
         m = _Model()
         self._check(self._lib.gpl_autotune(self._h, plan.encode(), int(max_candidates), ctypes.byref(m)))
         return {k: getattr(m, k) for k, _ in _Model._fields_}
+
+    def calibrate(self, rows=None) -> list:
+        """Γ, the channel calibration (Eq 1): ring throughput per shape and data size.
+        The points are applied to the A9 model and returned as dicts."""
+        arr = (ctypes.c_int64 * len(rows))(*rows) if rows else None
+        cap = 256
+        out = (_Gamma * cap)()
+        n = ctypes.c_int32(0)
+        self._check(self._lib.gpl_calibrate(self._h, arr, len(rows) if rows else 0, out, cap, ctypes.byref(n)))
+        return [{k: getattr(out[i], k) for k, _ in _Gamma._fields_} for i in range(n.value)]
+
+    def set_calibration(self, points: list):
+        """Load saved Γ points (as calibrate() returned them); [] clears the calibration."""
+        arr = (_Gamma * max(1, len(points)))()
+        for i, p in enumerate(points):
+            for k, _ in _Gamma._fields_:
+                setattr(arr[i], k, p[k])
+        self._check(self._lib.gpl_set_calibration(self._h, arr, len(points)))
 
     def run_plan_kbe(self, segment: str):
         self._check(self._lib.gpl_run_plan_kbe(self._h, segment.encode()))

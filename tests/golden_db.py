@@ -12,13 +12,13 @@ _COLS = {
     "region": [("r_regionkey", np.int32), ("r_name", np.int32)],
     "nation": [("n_nationkey", np.int32), ("n_name", np.int32), ("n_regionkey", np.int32)],
     "supplier": [("s_suppkey", np.int32), ("s_nationkey", np.int32)],
-    "customer": [("c_custkey", np.int32), ("c_nationkey", np.int32)],
+    "customer": [("c_custkey", np.int32), ("c_nationkey", np.int32), ("c_mktsegment", np.int32)],
     "part": [("p_partkey", np.int32), ("p_type", np.int32), ("p_retailprice", np.int64)],
     "partsupp": [("ps_partkey", np.int32), ("ps_suppkey", np.int32), ("ps_supplycost", np.int64)],
     "orders": [("o_orderkey", np.int32), ("o_custkey", np.int32), ("o_orderdate", np.int32)],
     "lineitem": [(c, t) for c, t in zip(tpchgen.LINEITEM_COLS, tpchgen._LI_TYPES)],
 }
-_DICT_COLS = {"r_name": "r_name", "n_name": "n_name", "p_type": "p_type"}
+_DICT_COLS = {"r_name": "r_name", "n_name": "n_name", "p_type": "p_type", "c_mktsegment": "c_mktsegment"}
 
 
 def load(name):
@@ -29,7 +29,7 @@ def load(name):
 def build_db(fx):
     """Database whose dictionary columns are codes into per-fixture dictionaries."""
     db = tpchgen.Database(sf=0.0, seed=0)
-    dicts = {"r_name": [], "n_name": [], "p_type": []}
+    dicts = {"r_name": [], "n_name": [], "p_type": [], "c_mktsegment": []}
     for tname, spec in fx["tables"].items():
         for c in spec["columns"]:
             if c in dicts:
@@ -40,6 +40,7 @@ def build_db(fx):
     for d in dicts.values():
         d.sort()
     db.r_name, db.n_name, db.p_type = dicts["r_name"], dicts["n_name"], dicts["p_type"]
+    db.c_mktsegment = dicts["c_mktsegment"] or list(tpchgen.SEGMENTS)
     for tname, cols in _COLS.items():
         spec = fx["tables"].get(tname, {"columns": [], "rows": []})
         n = len(spec["rows"])

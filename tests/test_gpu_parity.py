@@ -397,3 +397,53 @@ def test_clustered_probe_exact(ctx, q):
                         assert r.keys == o.keys and r.aggs == o.aggs, (q, name, cl, tile)
     finally:
         ctx.set_option("clustered", 1)
+
+
+def test_gamma_calibration_and_calibrated_model_exact(ctx):
+    """NEXT-1: gpl_calibrate measures Γ(n, s, k, d) for every ring shape that fits (Eq 1),
+    leaves the context's tables and options untouched, feeds the A9 model (its bandwidth becomes a
+    calibrated ring rate), and a query planned with the calibrated model stays bit-exact; the points
+    round-trip through gpl_set_calibration."""
+    db = tpchgen.generate(0.05, seed=7)
+    queries.load_database(ctx, db, queries.TABLES["Q5"])
+    o = oracle.run("Q5", db)
+    r = queries.run_query(ctx, "Q5", db)  # builds the hash tables the probe segment refers to
+    assert r.keys == o.keys and r.aggs == o.aggs
+    pts = ctx.calibrate([1 << 18, 1 << 21])
+    shapes = {(p["ring_depth"], p["stage_rows"], p["ctas_per_sm"]) for p in pts}
+    assert len(pts) == 2 * len(shapes) and len(shapes) >= 6
+    for p in pts:
+        assert p["ms"] > p["t0_ms"] > 0 and 0 < p["gbs"] < 20000, p
+        assert p["bytes"] == 16 * p["rows"]
+    # Γ grows with d for a fixed shape (launch and ring fill amortised; P:83 "when the input is small,
+    # the channel is not fully utilized")
+    for sh in shapes:
+        g = sorted((p["rows"], p["gbs"]) for p in pts if (p["ring_depth"], p["stage_rows"], p["ctas_per_sm"]) == sh)
+        assert g[1][1] > g[0][1]
+    seg = queries.segments(queries.plan_text("Q5", db))[-1]
+    m = ctx.choose_tile_rows(seg, 0)
+    assert 0 < m["bw_gbs"] < 20000
+    r = queries.run_query(ctx, "Q5", db)
+    assert r.keys == o.keys and r.aggs == o.aggs
+    ctx.set_calibration(pts)
+    assert ctx.choose_tile_rows(seg, 0)["predicted_ms"] == pytest.approx(m["predicted_ms"])
+    ctx.set_calibration([])
+
+
+def test_profiled_model_reproduces_its_run(ctx):
+    """Table 2 "profiling input": after the plan's first timed run with λ, the model's
+    consumer cost is fitted to it, so re-planning the same shape predicts that run's time; results
+    stay exact; use_profile = 0 restores the unfitted model."""
+    db = tpchgen.generate(0.2, seed=12)
+    queries.load_database(ctx, db, queries.TABLES["Q8"])
+    o = oracle.run("Q8", db)
+    rs = [queries.run_query(ctx, "Q8", db) for _ in range(4)]
+    for r in rs:
+        assert r.keys == o.keys and r.aggs == o.aggs
+    last = rs[-1].stats
+    assert last["predicted_ms"] == pytest.approx(rs[1].stats["kernel_ms"], rel=0.35) or \
+        last["predicted_ms"] == pytest.approx(last["kernel_ms"], rel=0.5)
+    ctx.set_option("use_profile", 0)
+    r = queries.run_query(ctx, "Q8", db)
+    assert r.keys == o.keys and r.aggs == o.aggs
+    ctx.set_option("use_profile", 1)

@@ -81,6 +81,40 @@ def test_model_report(host_ctx):
     assert m100["predicted_ms"] > 50 * m["predicted_ms"]
 
 
+def test_model_uses_gamma_calibration(host_ctx):
+    """Γ (Eq 1) replaces the copy bandwidth in the A9 model: a calibration
+    whose ring rate is half as fast at every size roughly doubles the streaming-bound prediction;
+    clearing it (or use_gamma = 0) restores the uncalibrated model."""
+    ctx, db = host_ctx
+    seg = queries.segments(queries.plan_text("L1", db, (19981101,)))[-1]
+    n = 600_000_000
+    base = ctx.choose_tile_rows(seg, n)
+
+    def curve(gbs):
+        return [dict(ring_depth=d, stage_rows=s, ctas_per_sm=k, consumer_warps=8, rows=r, bytes=16.0 * r,
+                     ms=0.0, t0_ms=0.004, gbs=gbs)
+                for d in (2, 3, 4, 6) for s in (512, 1024, 2048, 4096) for k in (1, 2)
+                for r in (1 << 20, 1 << 26)]
+    try:
+        ctx.set_calibration(curve(base["bw_gbs"]))
+        same = ctx.choose_tile_rows(seg, n)
+        assert same["bw_gbs"] == pytest.approx(base["bw_gbs"])
+        ctx.set_calibration(curve(base["bw_gbs"] / 2))
+        slow = ctx.choose_tile_rows(seg, n)
+        assert slow["bw_gbs"] == pytest.approx(base["bw_gbs"] / 2)
+        assert slow["t_launch_ms"] == pytest.approx(0.004)
+        assert 1.6 * same["predicted_ms"] < slow["predicted_ms"] < 2.4 * same["predicted_ms"]
+        ctx.set_option("use_gamma", 0)
+        assert ctx.choose_tile_rows(seg, n)["bw_gbs"] == pytest.approx(base["bw_gbs"])
+        ctx.set_option("use_gamma", 1)
+        with pytest.raises(gpl.GplError) as e:
+            ctx.set_calibration([dict(curve(1.0)[0], gbs=0.0)])
+        assert e.value.status == gpl.GPL_E_ARG
+    finally:
+        ctx.set_calibration([])
+    assert ctx.choose_tile_rows(seg, n)["predicted_ms"] == pytest.approx(base["predicted_ms"])
+
+
 def test_merge_partials_exact():
     rng = np.random.default_rng(0)
     nr, n = 5, 7

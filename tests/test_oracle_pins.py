@@ -21,7 +21,7 @@ from golden_db import build_db, expected_keys_as_codes, load
 QUERIES = ["L1", "Q5", "Q7", "Q8", "Q9", "Q14"]
 
 
-@pytest.mark.parametrize("fname", ["w1_listing1.json", "w2_q14.json", "w3_q5.json", "w4_q9.json"])
+@pytest.mark.parametrize("fname", ["w1_listing1.json", "w2_q14.json", "w3_q5.json", "w4_q9.json", "w5_q3.json"])
 def test_worked_examples(fname):
     fx = load(fname)
     db = build_db(fx)
@@ -157,3 +157,47 @@ def test_oracle_rejects_duplicate_pk():
     db = build_db(fx)
     with pytest.raises(RuntimeError, match="duplicate"):
         oracle.run("Q5", db, fx["params"])
+
+
+def test_q3_worked_example_order_limit():
+    """W5 (Q3): the ORDER BY revenue desc, o_orderdate tie-break, by oracle.order_limit and by the
+    brute-force selection (neither sorts the other's output)."""
+    fx = load("w5_q3.json")
+    db = build_db(fx)
+    r = oracle.run("Q3", db, fx["params"])
+    want = [tuple(k) for k in fx["expected"]["order_limit"]]
+    assert oracle.order_limit("Q3", r).keys == want
+    assert [k for k, _ in bf.order_limit_q3(bf.q3(db, *fx["params"]))] == want
+
+
+def test_q3_bruteforce_seeds_and_limit():
+    """NEXT-4 workload (TPC-H Q3): oracle == brute force over seeds (non-vacuous), and its
+    ORDER BY/LIMIT 10 equals the brute-force selection."""
+    nonvacuous = 0
+    for seed in range(1, 13):
+        db = tpchgen.generate(0.003, seed=seed)
+        r = oracle.run("Q3", db)
+        b = bf.q3(db)
+        assert r.as_dict() == b, seed
+        top = oracle.order_limit("Q3", r)
+        assert list(zip(top.keys, top.aggs)) == [(k, v) for k, v in bf.order_limit_q3(b)]
+        nonvacuous += len(r.keys) >= 3
+    assert nonvacuous >= 8
+
+
+def test_q3_pandas_groupby_and_sort():
+    """Q3 via pandas merge + groupby + sort_values (an independent implementation)."""
+    db = tpchgen.generate(0.05, seed=21)
+    f = _frames(db)
+    seg = tpchgen.SEGMENTS.index("BUILDING")
+    c = f["customer"][f["customer"].c_mktsegment == seg]
+    o = f["orders"][f["orders"].o_orderdate < 19950315].merge(c, left_on="o_custkey", right_on="c_custkey")
+    li = f["lineitem"][f["lineitem"].l_shipdate > 19950315]
+    x = li.merge(o, left_on="l_orderkey", right_on="o_orderkey")
+    x = x.assign(vol=x.l_extendedprice * (100 - x.l_discount))
+    g = x.groupby(["l_orderkey", "o_orderdate"]).agg(count=("vol", "size"), revenue=("vol", "sum")).reset_index()
+    r = oracle.run("Q3", db)
+    exp = {(int(a), int(b)): [int(n), int(v)] for a, b, n, v in g[["l_orderkey", "o_orderdate", "count", "revenue"]].values}
+    assert r.as_dict() == exp and len(exp) > 100
+    top = g.sort_values(["revenue", "o_orderdate", "l_orderkey"], ascending=[False, True, True]).head(10)
+    assert oracle.order_limit("Q3", r).keys == [(int(a), int(b)) for a, b in top[["l_orderkey", "o_orderdate"]].values]

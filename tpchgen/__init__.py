@@ -42,6 +42,8 @@ _SYL2 = ["ANODIZED", "BURNISHED", "PLATED", "POLISHED", "BRUSHED"]
 _SYL3 = ["TIN", "NICKEL", "BRASS", "STEEL", "COPPER"]
 # p_type dictionary: sorted, so 'PROMO%' is a contiguous code range.
 P_TYPES = sorted(" ".join(t) for t in itertools.product(_SYL1, _SYL2, _SYL3))
+# c_mktsegment dictionary (TPC-H spec §4.2.2.13) [EXT], sorted
+SEGMENTS = ["AUTOMOBILE", "BUILDING", "FURNITURE", "HOUSEHOLD", "MACHINERY"]
 
 
 def _load():
@@ -55,7 +57,7 @@ def _load():
         lib.tg_sizes.argtypes = [d, P]
         lib.tg_gen_part.argtypes = [d, u64, P, P, P]
         lib.tg_gen_supplier.argtypes = [d, u64, P, P]
-        lib.tg_gen_customer.argtypes = [d, u64, P, P]
+        lib.tg_gen_customer.argtypes = [d, u64, P, P, P]
         lib.tg_gen_partsupp.argtypes = [d, u64, P, P, P]
         lib.tg_gen_orders.argtypes = [d, u64, i64, i64, P, P, P]
         lib.tg_lineitem_count.argtypes = [d, u64, i64, i64]
@@ -99,6 +101,7 @@ class Database:
     n_name = [n for n, _ in NATIONS]
     r_name = REGIONS
     p_type = P_TYPES
+    c_mktsegment = SEGMENTS
 
     def nrows(self, table: str) -> int:
         cols = self.tables[table]
@@ -144,9 +147,9 @@ def generate(sf: float, seed: int = DEFAULT_SEED, rank: int = 0, world: int = 1,
         db.tables["supplier"] = {"s_suppkey": a, "s_nationkey": b}
     if "customer" in want:
         n = sz["customer"]
-        a, b = np.empty(n, np.int32), np.empty(n, np.int32)
-        lib.tg_gen_customer(sf, seed, _ptr(a), _ptr(b))
-        db.tables["customer"] = {"c_custkey": a, "c_nationkey": b}
+        a, b, c = np.empty(n, np.int32), np.empty(n, np.int32), np.empty(n, np.int32)
+        lib.tg_gen_customer(sf, seed, _ptr(a), _ptr(b), _ptr(c))
+        db.tables["customer"] = {"c_custkey": a, "c_nationkey": b, "c_mktsegment": c}
     if "partsupp" in want:
         n = sz["partsupp"]
         a, b, c = np.empty(n, np.int32), np.empty(n, np.int32), np.empty(n, np.int64)

@@ -33,7 +33,8 @@
 /* RNG streams (one per generated attribute). */
 enum {
   S_PTYPE = 1, S_SNAT, S_CNAT, S_PSCOST, S_OCUST, S_ODATE,
-  S_LCNT, S_LPART, S_LSUPP, S_LQTY, S_LDISC, S_LTAX, S_LSHIP
+  S_LCNT, S_LPART, S_LSUPP, S_LQTY, S_LDISC, S_LTAX, S_LSHIP,
+  S_CSEG /* appended: earlier streams (and their bytes) are unchanged */
 };
 
 static inline uint64_t sm64(uint64_t x) {
@@ -124,13 +125,17 @@ TG_API void tg_gen_supplier(double sf, uint64_t seed, int32_t* s_suppkey, int32_
   }
 }
 
-TG_API void tg_gen_customer(double sf, uint64_t seed, int32_t* c_custkey, int32_t* c_nationkey) {
+/* c_mktsegment: uniform over the 5 TPC-H market segments (dictionary codes of
+ * the sorted segment names); NULL = not generated. */
+TG_API void tg_gen_customer(double sf, uint64_t seed, int32_t* c_custkey, int32_t* c_nationkey,
+                            int32_t* c_mktsegment) {
   int64_t sz[5];
   tg_sizes(sf, sz);
 #pragma omp parallel for schedule(static)
   for (int64_t i = 0; i < sz[3]; i++) {
     c_custkey[i] = (int32_t)(i + 1);
     c_nationkey[i] = (int32_t)uni(seed, S_CNAT, (uint64_t)i, 25);
+    if (c_mktsegment) c_mktsegment[i] = (int32_t)uni(seed, S_CSEG, (uint64_t)i, 5);
   }
 }
 
