@@ -86,7 +86,8 @@ typedef struct {
   double predicted_ms;         /* A9 model estimate for this run                                   */
   double bytes_scanned;        /* algorithmic bytes: rows x bytes/row of TMA-staged columns +      */
                                /* (rows reaching the first use) x width of each lazy column       */
-  int32_t agg_mode;            /* 0 registers (1 group), 1 smem table, 2 global int128 atomics   */
+  int32_t agg_mode;            /* 0 registers (1 group), 1 smem table, 2 global int128 atomics,  */
+                               /* 3 hash group-by (global open-addressing table, int64 sums)      */
   int32_t kbe;                 /* 1 if produced by gpl_run_plan_kbe                               */
   int32_t jit;                 /* 1 if the plan-specialised (NVRTC) kernel ran, 0 the generic one */
   int32_t reserved;
@@ -95,15 +96,20 @@ typedef struct {
                                /* materialisation): the logical scan; >= bytes_scanned            */
   int32_t lazy_columns;        /* columns gathered per surviving row instead of TMA-staged        */
   int32_t packets;             /* 128-row packets per consumer iteration                          */
+  int64_t groups_total;        /* hash group-by: distinct groups (the result may be LIMITed)      */
+  int64_t hash_slots;          /* hash group-by: slots of the aggregation table                    */
 } gpl_stats;
 
 /* Result of the last run. Arrays are CALLER-owned with capacity cap_groups. */
 typedef struct {
   int32_t cap_groups;          /* in: rows the arrays can hold                                    */
-  int32_t n_groups;            /* out: non-empty groups (1 row when the plan has no GROUP BY)    */
+  int32_t n_groups;            /* out: non-empty groups (1 row when the plan has no GROUP BY);   */
+                               /* hash group-by with 'order'/'limit': rows in ORDER BY order,    */
+                               /* at most the limit (stats.groups_total = all distinct groups)   */
   int32_t n_keys;              /* out: group key columns                                          */
   int32_t n_aggs;              /* out: aggregates per row; agg 0 is COUNT(*)                      */
   int32_t* keys;               /* out: [cap_groups][n_keys] decoded key values, rows sorted by key */
+                               /* (hash group-by with 'order': in the plan's ORDER BY order)      */
   int64_t* aggs;               /* out: [cap_groups][n_aggs][2] int128 as (lo, hi) little-endian   */
   gpl_stats stats;             /* out */
 } gpl_result;
@@ -280,7 +286,8 @@ gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t
  * with an insert sink, default; 0 = the standalone build kernels),
  * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input),
  * "use_gamma" (1 = the model uses the Γ calibration when loaded, default),
- * "use_profile" (1 = the model fits its consumer cost to the plan's first
+ * "hash_slots_log2" (hash group-by table of 2^v slots; 0 = sized from the
+ * plan's last run, default), "use_profile" (1 = the model fits its consumer cost to the plan's first
  * timed run after its λ profile, Table 2 "profiling input", default).
  * value < 0 restores automatic selection. */
 gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value);

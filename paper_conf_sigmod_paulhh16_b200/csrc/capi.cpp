@@ -64,6 +64,20 @@ unsigned long long* counter_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 1; }
 unsigned long long* op_pass_ptr(gpl_ctx* ctx) { return ctx->d_scratch + 2; }
 // bytes of the per-run zeroed region (tile counter .. partials)
 size_t run_clear_bytes(size_t pbytes) { return (1 + MAXOPS) * sizeof(unsigned long long) + pbytes; }
+// the plan has a RunProfile taken on the current contents of its fact table
+bool profile_current(const gpl_ctx* ctx, const std::string& text, const std::string& table) {
+  auto it = ctx->profile.find(text);
+  if (it == ctx->profile.end()) return false;
+  auto ti = ctx->tables.find(table);
+  return ti != ctx->tables.end() && ti->second.version == it->second.table_version && it->second.runs >= 2;
+}
+
+// per-run result bytes after the head: dense int128 partials, or for a hash
+// group-by [distinct groups, rows out, LIMIT rows of (1 + nagg) words]
+size_t run_pbytes(const LowerInfo& li) {
+  if (li.hash_group) return ((size_t)(2 + li.limit * (1 + li.nagg)) * 8 + 15) / 16 * 16;
+  return (size_t)li.ngroups_total * li.nagg * 16;
+}
 // words the result copy-out moves (error bits, counters, partials)
 int result_words(size_t pbytes) { return kScratchHead + (int)(pbytes / 8); }
 unsigned long long* partials_ptr(gpl_ctx* ctx) { return ctx->d_scratch + kScratchHead; }
@@ -124,6 +138,54 @@ gpl_status decode(gpl_ctx* ctx, const unsigned long long* part, gpl_result* out)
       out->aggs[(r * A + a) * 2 + 1] = (int64_t)part[2 * (g * A + a) + 1];
     }
     r++;
+  }
+  return GPL_OK;
+}
+
+// Hash group-by result (NEXT-4): LIMIT rows come back with the counters in
+// ORDER BY order; without a LIMIT every group is copied from the device row
+// buffer and ordered by key on the host (as the dense decode orders gids).
+gpl_status decode_hash(gpl_ctx* ctx, const unsigned long long* part, gpl_result* out) {
+  const LowerInfo& li = ctx->last.run->li;
+  const int A = li.nagg, NK = li.ngroup_dims, W = 1 + A;
+  const uint64_t nrows = part[1];
+  out->n_keys = NK;
+  out->n_aggs = A;
+  out->n_groups = (int32_t)std::min<uint64_t>(nrows, INT32_MAX);
+  if (nrows > (uint64_t)std::max(out->cap_groups, 0)) return fail(ctx, GPL_E_CAPACITY, "result capacity too small");
+  if (nrows && (!out->aggs || !out->keys)) return fail(ctx, GPL_E_ARG, "NULL result arrays");
+  std::vector<unsigned long long> rows;
+  const unsigned long long* src = part + 2;
+  if (li.limit == 0 && nrows) {
+    rows.resize((size_t)nrows * W);
+    CK(cudaMemcpyAsync(rows.data(), ctx->last.run->hres.rows, rows.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    std::vector<size_t> ord(nrows);
+    for (size_t i = 0; i < nrows; i++) ord[i] = i;
+    auto field = [&](unsigned long long key, int k) {
+      return NK == 2 ? (int32_t)(uint32_t)(k == 0 ? key >> 32 : key) : (int32_t)(uint32_t)key;
+    };
+    std::sort(ord.begin(), ord.end(), [&](size_t a, size_t b) {
+      const unsigned long long ka = rows[a * W], kb = rows[b * W];
+      for (int k = 0; k < NK; k++)
+        if (field(ka, k) != field(kb, k)) return field(ka, k) < field(kb, k);
+      return false;
+    });
+    std::vector<unsigned long long> sorted(rows.size());
+    for (size_t i = 0; i < nrows; i++)
+      std::copy(rows.begin() + ord[i] * W, rows.begin() + (ord[i] + 1) * W, sorted.begin() + i * W);
+    rows.swap(sorted);
+    src = rows.data();
+  }
+  for (uint64_t r = 0; r < nrows; r++) {
+    const unsigned long long key = src[r * W];
+    for (int k = 0; k < NK; k++)
+      out->keys[r * NK + k] = NK == 2 ? (int32_t)(uint32_t)(k == 0 ? key >> 32 : key) : (int32_t)(uint32_t)key;
+    for (int a = 0; a < A; a++) {
+      const long long v = (long long)src[r * W + 1 + a];
+      out->aggs[(r * A + a) * 2] = v;
+      out->aggs[(r * A + a) * 2 + 1] = v < 0 ? -1 : 0;
+    }
   }
   return GPL_OK;
 }
@@ -202,6 +264,9 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     if (ctx->h_minmax) cudaFreeHost(ctx->h_minmax);
     if (ctx->d_minmax) cudaFree(ctx->d_minmax);
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
+    if (ctx->d_hagg) cudaFree(ctx->d_hagg);
+    if (ctx->d_hres) cudaFree(ctx->d_hres);
+    if (ctx->d_hcand) cudaFree(ctx->d_hcand);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
     if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
@@ -243,6 +308,9 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
     o.clustered = v != 0 ? 1 : 0;
   } else if (k == "build_pipeline") {
     o.build_pipeline = v != 0 ? 1 : 0;
+  } else if (k == "hash_slots_log2") {
+    if (v > 0 && (v < 12 || v > 34)) return fail(ctx, GPL_E_ARG, "hash_slots_log2 in [12, 34] (0 = auto)");
+    o.hash_slots_log2 = v > 0 ? v : 0;
   } else if (k == "use_profile") {
     o.use_profile = v != 0 ? 1 : 0;
   } else if (k == "use_gamma") {
@@ -454,7 +522,12 @@ static bool run_cache_valid(gpl_ctx* ctx, const PreparedRun& P, const std::set<i
   const size_t lambda_n = lam == ctx->lambda.end() ? 0 : lam->second.size();
   auto ti = ctx->tables.find(P.li.table);
   bool ok = ti != ctx->tables.end() && ti->second.version == P.table_version && P.opt_version == ctx->opt_version &&
-            P.lambda_n == lambda_n && P.profiled == (ctx->profile.count(P.text) > 0);
+            P.lambda_n == lambda_n && P.profiled == profile_current(ctx, P.text, P.li.table);
+  if (ok && P.li.hash_group) {
+    auto ge = ctx->hagg_groups.find(P.text);
+    ok = P.desc.hagg_keys == ctx->d_hagg && P.hres.rows == ctx->d_hres && P.hres.cand == ctx->d_hcand &&
+         (ge == ctx->hagg_groups.end() || 2 * ge->second.first <= P.hagg_cap || ctx->opt.hash_slots_log2 > 0);
+  }
   for (int i = 0; ok && i < P.desc.nht; i++) {
     const HashTable& H = ctx->hts[P.li.ht_ids[i]];
     const HTRef r = H.ref();
@@ -721,6 +794,66 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
   if ((st = prepare_run(ctx, text, tile_rows, &d, &li, &cfg, &seg))) return st;
   PreparedRun P;
   li.table = seg.table;
+  if (li.hash_group) {
+    // aggregation table: 2^k slots >= 2 x the distinct groups of the plan's
+    // last run (load <= 1/2), else min(rows, 2^21) groups assumed; keys then
+    // accumulators, zeroed per run. Selection scratch and the row buffer too.
+    // (groups scale with the fact rows when the table was reloaded at another size)
+    auto ge = ctx->hagg_groups.find(seg.text);
+    const uint64_t est =
+        ge != ctx->hagg_groups.end()
+            ? (uint64_t)((double)ge->second.first * std::max(1.0, (double)d.nrows / (double)std::max<int64_t>(ge->second.second, 1)))
+            : (uint64_t)std::min<int64_t>(std::max<int64_t>(d.nrows, 1), 1 << 21);
+    int lg = 12;
+    while ((1ull << lg) < 2 * est && lg < 34) lg++;
+    if (ctx->opt.hash_slots_log2 > 0) lg = (int)ctx->opt.hash_slots_log2;
+    const uint64_t cap = 1ull << lg;
+    const size_t bytes = (size_t)cap * 8 * (1 + li.nagg);
+    const size_t rbytes = (size_t)cap * 8 * (1 + li.nagg);
+    const int nblocks = hagg_select_blocks(cap, ctx->sms);
+    const size_t cbytes = (size_t)nblocks * std::max(1, li.limit) * 4;
+    auto grow = [&](void** p, size_t* have, size_t need) -> cudaError_t {
+      if (*have >= need) return cudaSuccess;
+      cudaError_t e = cudaStreamSynchronize(ctx->stream);
+      if (e != cudaSuccess) return e;
+      if (*p) cudaFree(*p);
+      *p = nullptr;
+      *have = 0;
+      e = cudaMalloc(p, need);
+      if (e == cudaSuccess) *have = need;
+      return e;
+    };
+    if (grow(&ctx->d_hagg, &ctx->hagg_alloc, bytes) != cudaSuccess ||
+        grow((void**)&ctx->d_hres, &ctx->hres_alloc, li.limit ? (size_t)li.limit * 8 * (1 + li.nagg) : rbytes) != cudaSuccess ||
+        grow((void**)&ctx->d_hcand, &ctx->hcand_alloc, cbytes) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(ctx, GPL_E_NOMEM, "hash group-by: cannot allocate a " + std::to_string(cap) + "-slot table");
+    }
+    d.hagg_keys = (unsigned long long*)ctx->d_hagg;
+    d.hagg_accs = (long long*)((char*)ctx->d_hagg + (size_t)cap * 8);
+    d.hagg_count = partials_ptr(ctx);  // result word 0: distinct groups
+    d.hagg_log2 = lg;
+    P.hagg_cap = cap;
+    P.hagg_clear = bytes;
+    HaggResultDesc& R = P.hres;
+    R.keys = d.hagg_keys;
+    R.accs = d.hagg_accs;
+    R.nslots = cap;
+    R.nagg = li.nagg;
+    R.nkeys = li.ngroup_dims;
+    R.limit = li.limit;
+    R.norder = li.norder;
+    for (int i = 0; i < 3; i++) {
+      R.ord_is_agg[i] = li.ord_is_agg[i];
+      R.ord_idx[i] = li.ord_idx[i];
+      R.ord_desc[i] = li.ord_desc[i];
+    }
+    R.cand = ctx->d_hcand;
+    R.nblocks = nblocks;
+    R.rows = ctx->d_hres;
+    R.small_out = partials_ptr(ctx);
+    R.n_out = partials_ptr(ctx) + 1;
+  }
   d.partials = partials_ptr(ctx);
   d.tile_counter = counter_ptr(ctx);
   d.op_pass = op_pass_ptr(ctx);
@@ -733,7 +866,7 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
   P.table_version = ctx->tables[seg.table].version;
   P.opt_version = ctx->opt_version;
   P.lambda_n = lambda_n;
-  P.profiled = ctx->profile.count(P.text) > 0;
+  P.profiled = profile_current(ctx, P.text, li.table);
   std::string jerr;
   P.fn = resolve_pipeline_fn(d, ctx->opt.jit != 0, &jerr);
   P.jit = ctx->opt.jit != 0 && jerr.empty();
@@ -761,12 +894,14 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   if ((st = get_prepared_run(ctx, probe_segment, tile_rows, &P))) return st;
   const PipeDesc& d = P->desc;
   const LowerInfo& li = P->li;
-  const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
+  const size_t pbytes = run_pbytes(li);
   // one memset: tile counter, op_pass and the partials are contiguous
   CK(cudaMemsetAsync(counter_ptr(ctx), 0, run_clear_bytes(pbytes), ctx->stream));
+  if (li.hash_group) CK(cudaMemsetAsync(d.hagg_keys, 0, P->hagg_clear, ctx->stream));
   CK(record_event(ctx, ctx->ev0));
   CK(launch_pipeline_fn(P->fn, d, P->grid, ctx->stream));
   CK(record_event(ctx, ctx->ev1));
+  if (li.hash_group) CK(launch_hagg_result(P->hres, d.hagg_count, ctx->sms, ctx->stream));
   CK(launch_copyout(ctx->d_scratch, ctx->h_stage_dev, result_words(pbytes), ctx->stream));
   LastRun& L = ctx->last;
   L.valid = true;
@@ -791,6 +926,7 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   S.packets = d.npack;
   S.agg_mode = d.agg_mode;
   S.jit = P->jit ? 1 : 0;
+  S.hash_slots = (int64_t)P->hagg_cap;
   return GPL_OK;
 }
 
@@ -888,6 +1024,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       S.packets = P.desc.npack;
       S.agg_mode = P.desc.agg_mode;
       S.jit = P.jit ? 1 : 0;
+      S.hash_slots = (int64_t)P.hagg_cap;
       return GPL_OK;
     }
     cudaGraphExecDestroy(g->second);
@@ -914,7 +1051,8 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       if (B.pipe) add(B.pdesc.ins_slots, B.clear_bytes);
     }
     const PreparedRun& R = *ctx->run_cache.at(run_key);
-    add(counter_ptr(ctx), run_clear_bytes((size_t)R.li.ngroups_total * R.li.nagg * 16));
+    add(counter_ptr(ctx), run_clear_bytes(run_pbytes(R.li)));
+    if (R.li.hash_group) add(R.desc.hagg_keys, R.hagg_clear);
     if (L.n > 16) return eager();
     CK(launch_clear(L, ctx->sms, ctx->stream));
     for (const PreparedBuild* B : builds) {
@@ -924,8 +1062,8 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     CK(record_event(ctx, ctx->ev0));
     CK(launch_pipeline_fn(R.fn, R.desc, R.grid, ctx->stream));
     CK(record_event(ctx, ctx->ev1));
-    CK(launch_copyout(ctx->d_scratch, ctx->h_stage_dev,
-                      result_words((size_t)R.li.ngroups_total * R.li.nagg * 16), ctx->stream));
+    if (R.li.hash_group) CK(launch_hagg_result(R.hres, R.desc.hagg_count, ctx->sms, ctx->stream));
+    CK(launch_copyout(ctx->d_scratch, ctx->h_stage_dev, result_words(run_pbytes(R.li)), ctx->stream));
     return GPL_OK;
   };
   if ((st = eager())) return st;
@@ -945,6 +1083,27 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     ctx->err.clear();
   }
   return GPL_OK;
+}
+
+// The model's per-shape candidates plus, for the `top` best predicted, the
+// other consumer-warp counts that fit (the model's W is the least certain
+// knob: the work-group sweep of P:366 / Figs 14-15 is measured, not only
+// modelled; every extra shape costs one plan-specialised compile).
+static void with_warp_variants(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t N,
+                               std::vector<Config>* cs, size_t top = 3) {
+  if (ctx->opt.consumer_warps > 0) return;
+  std::vector<Config> out;
+  for (size_t i = 0; i < cs->size(); i++) {
+    const Config& c = (*cs)[i];
+    out.push_back(c);
+    if (i >= top) continue;
+    for (int W : {4, 8, 12, 16}) {
+      if (W == c.warps) continue;
+      Config v = predict(ctx, d, li, std::max<int64_t>(N, 1), c.tile_rows, c.stage_rows, c.depth, W, c.ctas_per_sm, c.npack);
+      if (v.feasible) out.push_back(v);
+    }
+  }
+  cs->swap(out);
 }
 
 // gpl_autotune for one build segment that runs as a pipeline (DIRECT table):
@@ -967,6 +1126,20 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
   gpl_status st = lower_build_pipe(ctx, s, H, &pd, &c0, &cs);
   if (st) return st;
   if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
+  {
+    LowerInfo lb;  // the build pipeline's facts for the warp variants (as lower_build_pipe computed them)
+    PipeDesc pb;
+    std::string e2;
+    const int split = ctx->opt.probe_split >= -1 || s.split_hint >= -1 ? choose_split(ctx, s)
+                                                                        : std::min<int>((int)s.probes.size(), MAXSP);
+    if (lower_probe(ctx, s, split, &pb, &lb, &e2, &H) == GPL_OK) {
+      for (int i = 0; i < pb.nht; i++) {
+        const HashTable& h = ctx->hts[lb.ht_ids[i]];
+        lb.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+      }
+      with_warp_variants(ctx, pb, lb, pb.nrows, &cs);
+    }
+  }
   bool has0 = false;
   for (const Config& c : cs)
     has0 |= c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
@@ -1089,6 +1262,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
       continue;
     }
     if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
+    with_warp_variants(ctx, ds, ls, ds.nrows, &cs);
     for (const Config& c : cs) {
       cands.push_back({sp, c});
       cand_split_eff.push_back(ds.nsprobe);
@@ -1210,6 +1384,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   st = prepare_run(ctx, probe_segment, 0, &d, &li, &cfg, &seg, 0);
   ctx->opt.lazy_columns = lazy_opt;
   if (st) return st;
+  if (li.hash_group) return fail(ctx, GPL_E_PLAN, "the KBE baseline has no hash group-by ('group hash')");
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
   d.partials = partials_ptr(ctx);
   d.tile_counter = counter_ptr(ctx);
@@ -1286,7 +1461,7 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run to fetch");
   const LowerInfo& li = ctx->last.run->li;
   // one D2H: error bits, counter, op_pass and partials are contiguous
-  const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
+  const size_t pbytes = run_pbytes(li);
   // fused runs: the copy-out kernel already wrote the results to h_stage
   if (!ctx->last.copied_out)
     CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
@@ -1316,24 +1491,54 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
     for (int i = 0; i < li.nops; i++) lam.push_back((double)ops[i] / (double)S.rows_scanned);
     ctx->lambda[ctx->last.run->text] = lam;
   } else if (!ctx->last.kbe && ctx->last.timed && S.kernel_ms > 0 && S.rows_scanned > 0 && ctx->last.run->lambda_n > 0 &&
-             !ctx->profile.count(ctx->last.run->text)) {
-    // the first timed run planned with λ: the model's profiling input
+             !profile_current(ctx, ctx->last.run->text, ctx->last.run->li.table)) {
+    // the first two timed runs planned with λ (same shape; the faster one —
+    // the first may pay cold TLB/L2 misses after a load): the model's
+    // profiling input
     const PreparedRun& R = *ctx->last.run;
-    RunProfile p;
-    p.nrows = R.desc.nrows;
-    p.tile_rows = R.desc.tile_rows;
-    p.stage_rows = R.desc.stage_rows;
-    p.depth = R.desc.depth;
-    p.warps = R.desc.nwarps;
-    p.npack = R.desc.npack;
-    p.ctas_per_sm = std::max(1, R.grid / std::max(1, ctx->sms));
-    p.kernel_ms = S.kernel_ms;
-    ctx->profile[R.text] = p;
+    auto ti = ctx->tables.find(R.li.table);
+    const uint64_t ver = ti != ctx->tables.end() ? ti->second.version : 0;
+    auto old = ctx->profile.find(R.text);
+    if (old != ctx->profile.end() && old->second.runs == 1 && old->second.table_version == ver &&
+        old->second.tile_rows == R.desc.tile_rows && old->second.stage_rows == R.desc.stage_rows &&
+        old->second.depth == R.desc.depth && old->second.warps == R.desc.nwarps && old->second.npack == R.desc.npack) {
+      old->second.kernel_ms = std::min(old->second.kernel_ms, S.kernel_ms);
+      old->second.runs = 2;
+    } else {
+      RunProfile p;
+      p.nrows = R.desc.nrows;
+      p.tile_rows = R.desc.tile_rows;
+      p.stage_rows = R.desc.stage_rows;
+      p.depth = R.desc.depth;
+      p.warps = R.desc.nwarps;
+      p.npack = R.desc.npack;
+      p.ctas_per_sm = std::max(1, R.grid / std::max(1, ctx->sms));
+      p.kernel_ms = S.kernel_ms;
+      p.table_version = ver;
+      p.runs = 1;
+      ctx->profile[R.text] = p;
+    }
+  }
+  if (li.hash_group) {
+    // distinct groups size the next run's table (load <= 1/2); an overflow
+    // (ERR_CAPACITY) quadruples it
+    const uint64_t seen = part[0];
+    const uint64_t cap = ctx->last.run->hagg_cap;
+    auto& est = ctx->hagg_groups[ctx->last.run->text];
+    est.first = (bits & ERR_CAPACITY) ? std::max<uint64_t>(2 * cap, seen) : seen;
+    est.second = (int64_t)S.rows_scanned;
+    S.groups_total = (int64_t)seen;
   }
   out->stats = S;
   if (bits) {
-    if ((st = take_device_errors(ctx))) return st;
+    if ((st = take_device_errors(ctx))) {
+      if (li.hash_group && st == GPL_E_CAPACITY)
+        return fail(ctx, st, "hash group-by table overflowed (" + std::to_string(ctx->last.run->hagg_cap) +
+                                 " slots); the next run of the plan uses a larger table");
+      return st;
+    }
   }
+  if (li.hash_group) return decode_hash(ctx, part, out);
   return decode(ctx, part, out);
 }
 
@@ -1342,6 +1547,8 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
   gpl_status st = check_dev(ctx);
   if (st) return st;
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run");
+  if (ctx->last.run->li.hash_group)
+    return fail(ctx, GPL_E_STATE, "a hash group-by has no dense partial vector (fetch its rows with gpl_fetch_result)");
   const size_t b = (size_t)ctx->last.run->li.ngroups_total * ctx->last.run->li.nagg * 16;
   *nbytes = b;
   if (cap_bytes < b || !dst) return fail(ctx, GPL_E_CAPACITY, "partials buffer too small");
@@ -1354,6 +1561,7 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
 GPL_API gpl_status gpl_decode_partials(gpl_ctx* ctx, const void* host_partials, size_t nbytes, gpl_result* out) {
   if (!ctx || !host_partials || !out) return GPL_E_ARG;
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run (the plan of the last run defines the layout)");
+  if (ctx->last.run->li.hash_group) return fail(ctx, GPL_E_STATE, "a hash group-by has no dense partial vector");
   const size_t b = (size_t)ctx->last.run->li.ngroups_total * ctx->last.run->li.nagg * 16;
   if (nbytes != b) return fail(ctx, GPL_E_ARG, "partials size does not match the last run's plan");
   gpl_stats& S = ctx->last.stats;

@@ -119,7 +119,7 @@ struct Agg {
   int32_t kind, field;
   int64_t c;
 };
-enum : int32_t { AGG_REG = 0, AGG_SMEM = 1, AGG_GLOBAL = 2 };
+enum : int32_t { AGG_REG = 0, AGG_SMEM = 1, AGG_GLOBAL = 2, AGG_HASH = 3 };
 enum : int32_t { SINK_AGG = 0, SINK_INSERT = 1 };
 
 // ---- survivor-queue push: field <- stage column, stage-phase probe slot, or
@@ -188,11 +188,36 @@ struct PipeDesc {
   long long ins_kmin, ins_pay_base;                            // run-time (table bases)
   unsigned long long ins_nslots;
   void* ins_slots;
+  // hash group-by (AGG_HASH): open addressing, linear
+  // probing over 2^hagg_log2 slots; hagg_keys holds ~key (0 = empty, so the
+  // table clears with zeros), hagg_accs [slot][nagg] exact int64 sums;
+  // hagg_count counts distinct groups (CAS winners)
+  unsigned long long* hagg_keys;
+  long long* hagg_accs;
+  unsigned long long* hagg_count;
+  int32_t hagg_log2, hagg_pad;
   // outputs
   unsigned long long* partials;      // [ngroups_total][nagg] x (lo, hi)
   unsigned long long* tile_counter;  // zeroed before launch
   unsigned long long* op_pass;       // [MAXOPS]
   unsigned int* err;
+};
+
+// Result step of a hash group-by (blocking, after the pipeline): ORDER BY ...
+// LIMIT k selection, or compaction of every group. Rows are [key, acc 0..nagg).
+struct HaggResultDesc {
+  const unsigned long long* keys;  // ~key per slot, 0 = empty
+  const long long* accs;           // [slot][nagg]
+  unsigned long long nslots;
+  int32_t nagg, nkeys;             // key fields packed (k0 << 32 | k1) when nkeys == 2
+  int32_t limit;                   // 0: every group (compaction)
+  int32_t norder;
+  int32_t ord_is_agg[3], ord_idx[3], ord_desc[3];
+  unsigned int* cand;              // selection scratch: slot indices [nblocks * limit]
+  int32_t nblocks, pad;
+  unsigned long long* rows;        // out: n_out rows of (1 + nagg) words (device)
+  unsigned long long* small_out;   // out (limit): [n_groups, n_out, rows...] in the partials area
+  unsigned long long* n_out;       // out (compaction): row counter (zeroed per run)
 };
 
 // Descriptor of one build segment (hash_build kernels).

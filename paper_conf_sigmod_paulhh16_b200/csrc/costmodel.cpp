@@ -29,6 +29,8 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <map>
 #include <tuple>
 
@@ -265,6 +267,9 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
   auto it = ctx->profile.find(plan_text);
   if (it == ctx->profile.end() || !ctx->opt.use_profile) return;
   const RunProfile& p = it->second;
+  auto ti = ctx->tables.find(li->table.empty() ? std::string() : li->table);
+  if (ti != ctx->tables.end() && ti->second.version != p.table_version) return;  // profiled on other data
+  if (p.runs < 2) return;
   auto pred = [&](double f) {
     li->cons_factor = f;
     return predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
@@ -295,6 +300,10 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
     (pred(mid) < p.kernel_ms ? lo : hi) = mid;
   }
   li->cons_factor = std::sqrt(lo * hi);
+  if (std::getenv("GPL_DEBUG_MODEL"))
+    std::fprintf(stderr, "apply_profile: measured %.4f ms at S %d D %d W %d k %d np %d tile %lld N %lld -> cons %.3f bw %.3f pred %.4f\n",
+                 p.kernel_ms, p.stage_rows, p.depth, p.warps, p.ctas_per_sm, p.npack, (long long)p.tile_rows,
+                 (long long)p.nrows, li->cons_factor, li->bw_factor, pred(li->cons_factor));
 }
 
 int choose_split(const gpl_ctx* ctx, const Segment& s) {

@@ -80,12 +80,18 @@ struct LowerInfo {
   bool has_groups = false;
   std::vector<double> lambda;     // cumulative pass fraction after each op (previous run)
   double cons_factor = 1;         // consumer cost scale fitted to the plan's profiled run (costmodel apply_profile)
+  // hash group-by (NEXT-4): the result step's ORDER BY / LIMIT
+  bool hash_group = false;
+  int limit = 0, norder = 0;
+  int ord_is_agg[3] = {0, 0, 0}, ord_idx[3] = {0, 0, 0}, ord_desc[3] = {0, 0, 0};
   double bw_factor = 1;           // streaming-rate scale, fitted only when the run beat the model's stream bound (L2-resident input)
 };
 
 // The first timed run of a plan after its λ profile (the paper profiles the
 // first tile): its shape, rows and measured kernel time.
 struct RunProfile {
+  uint64_t table_version = 0;  // the fact table's version when profiled (a reload re-profiles)
+  int runs = 0;                // timed runs folded in (the profile is used from 2 on)
   int64_t nrows = 0, tile_rows = 0;
   int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1, npack = 1;
   double kernel_ms = 0;
@@ -113,6 +119,10 @@ struct PreparedRun {
   uint64_t table_version = 0, opt_version = 0;
   size_t lambda_n = 0;
   bool profiled = false;  // planned with the plan's RunProfile
+  // hash group-by (NEXT-4): the aggregation table's size and the result step
+  uint64_t hagg_cap = 0;
+  size_t hagg_clear = 0;  // bytes zeroed per run (keys + accumulators)
+  HaggResultDesc hres{};
   std::string text;
 };
 
@@ -153,6 +163,7 @@ struct Options {
   double hbm_gbs = -1;
   int64_t use_gamma = 1;       // the model uses the channel calibration Γ when one is loaded
   int64_t use_profile = 1;     // the model fits its consumer cost to the plan's profiled run
+  int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
 };
 
 // Γ of one ring shape (gpl_calibrate, Eq 1): (bytes, GB/s)
@@ -203,6 +214,15 @@ struct gpl_ctx {
   long long* h_minmax = nullptr;  // pinned column min/max of a load (64 columns)
   unsigned long long* h_stage_dev = nullptr;  // device alias of h_stage (the fused kernel's result copy-out)
   size_t h_stage_cap = 0;
+  // hash group-by (NEXT-4): aggregation table, result rows, selection scratch;
+  // distinct groups of each plan's last run size the next table
+  void* d_hagg = nullptr;
+  size_t hagg_alloc = 0;
+  unsigned long long* d_hres = nullptr;
+  size_t hres_alloc = 0;
+  unsigned int* d_hcand = nullptr;
+  size_t hcand_alloc = 0;
+  std::map<std::string, std::pair<uint64_t, int64_t>> hagg_groups;  // plan text -> (distinct groups, fact rows) of its last run
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;
   size_t kbe_cap = 0;

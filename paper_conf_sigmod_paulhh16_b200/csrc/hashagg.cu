@@ -1,0 +1,222 @@
+// hashagg.cu — result step of a hash group-by: the
+// blocking operator after the fused pipeline (ORDER BY is blocking).
+//
+//   * ORDER BY ... LIMIT k: a two-phase device selection. Phase A: every CTA
+//     walks its slice of the hash-aggregation table, keeps its k best groups
+//     in shared memory (bitonic sort of a 1024-entry tile whenever new
+//     candidates arrive; once k entries are held, only groups better than the
+//     current k-th are admitted) and writes their slot indices. Phase B: one
+//     CTA runs the same selection over the candidates and writes the k rows
+//     in order — to the device row buffer and to the run's result words, so
+//     the copy-out kernel brings them back with the counters (no extra D2H).
+//   * no LIMIT: every occupied slot is compacted into the row buffer (order
+//     arbitrary; the host orders by key).
+// A row is [packed key, acc 0 .. nagg-1] (8-byte words). Ordering: the plan's
+// components (aggregate or key field, asc/desc), then the full key ascending,
+// so the first k rows are unique.
+#include "kernels.h"
+#include "device_common.cuh"
+
+namespace gpl {
+namespace {
+
+constexpr int kTile = 1024;
+constexpr int kThreads = 256;
+constexpr unsigned kNone = 0xFFFFFFFFu;
+constexpr unsigned long long kSign = 1ull << 63;
+
+struct SelSmem {
+  unsigned long long w[4][kTile];  // sort words (lexicographic, ascending = better)
+  unsigned idx[kTile];             // slot index (kNone = padding)
+  unsigned long long thr[4];       // the current k-th best (admission threshold)
+  int fill, have_thr;
+};
+
+__device__ __forceinline__ int key_field(unsigned long long key, int nkeys, int i) {
+  return nkeys == 2 ? (int)(unsigned)(i == 0 ? key >> 32 : key) : (int)(unsigned)key;
+}
+
+// The sort words of slot s (order components, then the full key ascending,
+// then zeros); returns false when the slot is empty.
+__device__ __forceinline__ bool words_of(const HaggResultDesc& D, unsigned long long s, unsigned long long (&w)[4]) {
+  const unsigned long long st = __ldcg(D.keys + s);
+  if (st == 0ull) return false;
+  const unsigned long long key = ~st;
+  unsigned long long kw;  // full key ascending (signed fields)
+  if (D.nkeys == 2)
+    kw = ((unsigned long long)((unsigned)key_field(key, 2, 0) ^ 0x80000000u) << 32) |
+         (unsigned long long)((unsigned)key_field(key, 2, 1) ^ 0x80000000u);
+  else
+    kw = (unsigned long long)(long long)key_field(key, 1, 0) ^ kSign;
+#pragma unroll
+  for (int c = 0; c < 4; c++) {
+    if (c < D.norder) {
+      const long long v = D.ord_is_agg[c] ? __ldcg(D.accs + s * D.nagg + D.ord_idx[c])
+                                          : (long long)key_field(key, D.nkeys, D.ord_idx[c]);
+      const unsigned long long u = (unsigned long long)v ^ kSign;
+      w[c] = D.ord_desc[c] ? ~u : u;
+    } else {
+      w[c] = c == D.norder ? kw : 0ull;
+    }
+  }
+  return true;
+}
+
+__device__ __forceinline__ bool less4(const unsigned long long (&a)[4], const unsigned long long (&b)[4]) {
+#pragma unroll
+  for (int c = 0; c < 4; c++)
+    if (a[c] != b[c]) return a[c] < b[c];
+  return false;
+}
+
+__device__ __forceinline__ bool less_at(const SelSmem& m, int i, int j) {
+#pragma unroll
+  for (int c = 0; c < 4; c++)
+    if (m.w[c][i] != m.w[c][j]) return m.w[c][i] < m.w[c][j];
+  return m.idx[i] < m.idx[j];
+}
+
+__device__ void bitonic_sort(SelSmem& m) {
+  for (int k = 2; k <= kTile; k <<= 1)
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < kTile; i += blockDim.x) {
+        const int p = i ^ j;
+        if (p > i) {
+          const bool up = (i & k) == 0;
+          if (less_at(m, p, i) == up) {
+#pragma unroll
+            for (int c = 0; c < 4; c++) {
+              const unsigned long long t = m.w[c][i];
+              m.w[c][i] = m.w[c][p];
+              m.w[c][p] = t;
+            }
+            const unsigned t = m.idx[i];
+            m.idx[i] = m.idx[p];
+            m.idx[p] = t;
+          }
+        }
+      }
+      __syncthreads();
+    }
+}
+
+__device__ __forceinline__ void set_pad(SelSmem& m, int i) {
+#pragma unroll
+  for (int c = 0; c < 4; c++) m.w[c][i] = ~0ull;
+  m.idx[i] = kNone;
+}
+
+// Keep the k best of [input range] in m.idx[0..k) (sorted, best first).
+// from_cand: the input is D.cand[lo..hi) (slot indices, kNone = none),
+// else the hash slots [lo, hi).
+__device__ void select_k(const HaggResultDesc& D, SelSmem& m, unsigned long long lo, unsigned long long hi,
+                         bool from_cand) {
+  const int K = D.limit;
+  for (int i = threadIdx.x; i < kTile; i += blockDim.x) set_pad(m, i);
+  if (threadIdx.x == 0) {
+    m.fill = 0;
+    m.have_thr = 0;
+  }
+  __syncthreads();
+  const int batch = kTile - K;
+  for (unsigned long long base = lo; base < hi; base += (unsigned long long)batch) {
+    for (int t = threadIdx.x; t < batch; t += blockDim.x) {
+      const unsigned long long pos = base + (unsigned long long)t;
+      if (pos >= hi) break;
+      unsigned long long s = pos;
+      if (from_cand) {
+        const unsigned c = D.cand[pos];
+        if (c == kNone) continue;
+        s = c;
+      }
+      unsigned long long w[4];
+      if (!words_of(D, s, w)) continue;
+      if (m.have_thr) {
+        unsigned long long th[4] = {m.thr[0], m.thr[1], m.thr[2], m.thr[3]};
+        if (!less4(w, th)) continue;
+      }
+      const int at = K + atomicAdd(&m.fill, 1);
+#pragma unroll
+      for (int c = 0; c < 4; c++) m.w[c][at] = w[c];
+      m.idx[at] = (unsigned)s;
+    }
+    __syncthreads();
+    const int fill = m.fill;
+    if (fill > 0) {  // uniform branch
+      bitonic_sort(m);
+      // entries [K, kTile) are dropped: reset them, record the threshold
+      for (int i = K + threadIdx.x; i < kTile; i += blockDim.x) set_pad(m, i);
+      if (threadIdx.x == 0) {
+        m.fill = 0;
+        if (m.idx[K - 1] != kNone) {
+          m.have_thr = 1;
+#pragma unroll
+          for (int c = 0; c < 4; c++) m.thr[c] = m.w[c][K - 1];
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(kThreads) select_phase_a(const __grid_constant__ HaggResultDesc D) {
+  __shared__ SelSmem m;
+  const unsigned long long per = (D.nslots + gridDim.x - 1) / gridDim.x;
+  const unsigned long long lo = per * blockIdx.x, hi = min(D.nslots, lo + per);
+  select_k(D, m, lo, lo < hi ? hi : lo, false);
+  for (int i = threadIdx.x; i < D.limit; i += blockDim.x) D.cand[(unsigned long long)blockIdx.x * D.limit + i] = m.idx[i];
+}
+
+__global__ void __launch_bounds__(kThreads) select_phase_b(const __grid_constant__ HaggResultDesc D,
+                                                           const unsigned long long* hagg_count) {
+  __shared__ SelSmem m;
+  select_k(D, m, 0, (unsigned long long)D.nblocks * D.limit, true);
+  int n = 0;
+  for (int i = 0; i < D.limit; i++) n += m.idx[i] != kNone;
+  const int W = 1 + D.nagg;
+  for (int i = threadIdx.x; i < n * W; i += blockDim.x) {
+    const int r = i / W, c = i % W;
+    const unsigned long long s = m.idx[r];
+    const unsigned long long v = c == 0 ? ~__ldcg(D.keys + s) : (unsigned long long)__ldcg(D.accs + s * D.nagg + (c - 1));
+    D.rows[i] = v;
+    D.small_out[2 + i] = v;
+  }
+  if (threadIdx.x == 0) {
+    D.small_out[0] = __ldcg(hagg_count);
+    D.small_out[1] = (unsigned long long)n;
+  }
+}
+
+__global__ void __launch_bounds__(kThreads) compact_groups(const __grid_constant__ HaggResultDesc D) {
+  const int W = 1 + D.nagg;
+  for (unsigned long long s = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; s < D.nslots;
+       s += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned long long st = __ldcg(D.keys + s);
+    if (st == 0ull) continue;
+    const unsigned long long r = atomicAdd(D.n_out, 1ull);
+    D.rows[r * W] = ~st;
+    for (int a = 0; a < D.nagg; a++) D.rows[r * W + 1 + a] = (unsigned long long)__ldcg(D.accs + s * D.nagg + a);
+  }
+}
+
+}  // namespace
+
+int hagg_select_blocks(unsigned long long nslots, int num_sms) {
+  // one slice per CTA, >= 4K slots each, at most 2 CTAs per SM
+  const unsigned long long b = (nslots + 4095) / 4096;
+  return (int)(b < 1 ? 1 : b > (unsigned long long)(2 * num_sms) ? 2 * num_sms : b);
+}
+
+cudaError_t launch_hagg_result(const HaggResultDesc& D, const unsigned long long* hagg_count, int num_sms,
+                               cudaStream_t s) {
+  if (D.limit > 0) {
+    select_phase_a<<<D.nblocks, kThreads, 0, s>>>(D);
+    select_phase_b<<<1, kThreads, 0, s>>>(D, hagg_count);
+  } else {
+    const unsigned long long b = (D.nslots + kThreads - 1) / kThreads;
+    compact_groups<<<(int)(b < 1 ? 1 : b > (unsigned long long)(4 * num_sms) ? 4 * num_sms : b), kThreads, 0, s>>>(D);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace gpl

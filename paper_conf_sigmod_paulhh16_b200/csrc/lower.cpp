@@ -199,6 +199,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
                        const HashTable* ins) {
   *d = PipeDesc{};
   *li = LowerInfo{};
+  li->table = s.table;
   if (s.is_build && !ins) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
   d->cl_probe = d->cl_col = -1;
   if (ins && (!s.is_build || ins->kind != HT_DIRECT || s.key.size() != 1)) {
@@ -573,7 +574,28 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   // group-by
   d->ngroup = (int)s.groups.size();
   int64_t G = 1;
-  for (int g = d->ngroup - 1; g >= 0; g--) {
+  if (s.hash_group) {  // unbounded keys (NEXT-4): packed int32 fields, no domain
+    for (int g = 0; g < d->ngroup; g++) {
+      const GroupIR& Gi = s.groups[g];
+      GroupDim& D = d->gdim[g];
+      D.field = field[Gi.ref.name];
+      D.transform = Gi.ref.kind == RefIR::YEARCOL ? G_YEAR : G_ID;
+      D.lo = D.size = D.stride = 0;
+      if (Gi.ref.kind != RefIR::YEARCOL) {
+        const Range r = ref_range(Gi.ref.name);
+        if (r.lo < INT32_MIN || r.hi > INT32_MAX) { *err = "group hash keys must be 32-bit values"; return GPL_E_PLAN; }
+      }
+    }
+    li->hash_group = true;
+    li->limit = s.limit;
+    li->norder = (int)s.order.size();
+    for (int i = 0; i < li->norder; i++) {
+      li->ord_is_agg[i] = s.order[i].is_agg;
+      li->ord_idx[i] = s.order[i].idx;
+      li->ord_desc[i] = s.order[i].desc;
+    }
+  }
+  for (int g = s.hash_group ? -1 : d->ngroup - 1; g >= 0; g--) {
     const GroupIR& Gi = s.groups[g];
     GroupDim& D = d->gdim[g];
     D.field = field[Gi.ref.name];
@@ -663,7 +685,14 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   // accumulator covering <= R rows is exact when R * maxabs < 2^62.
   const long double lim = 4.6e18L;
   const long double total = (long double)std::max<int64_t>(T.nrows, 1) * std::max<long double>(li->maxabs, 1);
-  if (d->ngroups_total == 1) {
+  if (s.hash_group) {  // one exact int64 accumulator per group and aggregate
+    if (total >= lim) {
+      *err = "hash group-by sums are int64: rows x max|value| may exceed 2^62";
+      return GPL_E_OVERFLOW;
+    }
+    d->agg_mode = AGG_HASH;
+    d->flush_each_tile = 0;
+  } else if (d->ngroups_total == 1) {
     d->agg_mode = AGG_REG;
     d->flush_each_tile = total >= lim ? 1 : 0;
   } else {

@@ -355,10 +355,46 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
 #pragma unroll
   for (int j = 0; j < RPL; j++) {
     if (!p[j]) continue;
+    long long hslot = -1;  // AGG_HASH: the group's slot
+    if (K.agg_mode == AGG_HASH) {
+      // hash group-by over unbounded keys (NEXT-4): the packed key finds or
+      // claims its slot (open addressing, linear probing); slots hold ~key
+      unsigned long long key = 0;
+      GPL_UNROLL
+      for (int g = 0; g < K.ngroup; g++) {
+        long long v = qget(K, qb, K.gdim[g].field, idx[j]);
+        if (K.gdim[g].transform == G_YEAR) v = (int)v / 10000;
+        key = (key << 32) | (unsigned long long)(unsigned)v;
+      }
+      if (key == ~0ull) {
+        atomicOr(d.err, ERR_RESERVED_KEY);
+        continue;
+      }
+      const unsigned long long st = ~key, mask = (1ull << d.hagg_log2) - 1ull;
+      unsigned long long h = (key * 0x9E3779B97F4A7C15ull) >> (64 - d.hagg_log2);
+      for (unsigned long long step = 0; step <= mask; step++, h = (h + 1) & mask) {
+        unsigned long long cur = __ldcg(d.hagg_keys + h);
+        if (cur == 0ull) {
+          cur = atomicCAS(d.hagg_keys + h, 0ull, st);
+          if (cur == 0ull) {
+            atomicAdd(d.hagg_count, 1ull);
+            cur = st;
+          }
+        }
+        if (cur == st) {
+          hslot = (long long)h;
+          break;
+        }
+      }
+      if (hslot < 0) {  // table full: latched, the host re-runs with a larger table
+        atomicOr(d.err, ERR_CAPACITY);
+        continue;
+      }
+    }
     int gid = 0;
     bool ok = true;
     GPL_UNROLL
-    for (int g = 0; g < K.ngroup; g++) {
+    for (int g = 0; g < (K.agg_mode == AGG_HASH ? 0 : K.ngroup); g++) {
       const GroupDim& G = K.gdim[g];
       long long v = qget(K, qb, G.field, idx[j]);
       if (G.transform == G_YEAR) v = (int)v / 10000;
@@ -395,7 +431,8 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
       else if (A.kind == A_SUMIFEQ) c = qget(K, qb, A.field, idx[j]) == A.c ? val : 0;
       if (K.agg_mode == AGG_REG) acc[a] += c;
       else if (c != 0) {
-        if (K.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * K.nagg + a], (unsigned long long)c);
+        if (K.agg_mode == AGG_HASH) atomicAdd((unsigned long long*)d.hagg_accs + hslot * K.nagg + a, (unsigned long long)c);
+        else if (K.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * K.nagg + a], (unsigned long long)c);
         else atomic_add_i128(d.partials + 2 * (gid * K.nagg + a), c);
       }
     }

@@ -323,8 +323,41 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
           }
         }
         seg->wheres.push_back(w);
+      } else if (kw == "group" && c.is_id("hash")) {
+        // hash group-by over unbounded int32 keys: group hash A[, B]
+        if (seg->is_build) throw ParseError{"'group' only in the probe segment"};
+        if (!seg->groups.empty()) throw ParseError{"one 'group hash' statement, not mixed with dense groups"};
+        c.i++;
+        seg->hash_group = true;
+        do {
+          GroupIR g;
+          g.ref = parse_ref(c);
+          seg->groups.push_back(g);
+        } while (c.accept_sym(","));
+        if (seg->groups.size() > 2) throw ParseError{"group hash takes at most 2 keys"};
+      } else if (kw == "order") {
+        if (seg->is_build) throw ParseError{"'order' only in the probe segment"};
+        do {
+          OrderIR o;
+          std::string what = expect_id(c, "agg|key");
+          if (what != "agg" && what != "key") throw ParseError{"order component must be 'agg N' or 'key N'"};
+          o.is_agg = what == "agg";
+          o.idx = (int)expect_int(c, "index");
+          if (c.is_id("desc") || c.is_id("asc")) {
+            o.desc = c.is_id("desc");
+            c.i++;
+          }
+          seg->order.push_back(o);
+        } while (c.accept_sym(","));
+        if (seg->order.size() > 3) throw ParseError{"at most 3 order components"};
+      } else if (kw == "limit") {
+        if (seg->is_build) throw ParseError{"'limit' only in the probe segment"};
+        const int64_t k = expect_int(c, "row count");
+        if (k < 1 || k > 512) throw ParseError{"limit must be in [1, 512]"};
+        seg->limit = (int)k;
       } else if (kw == "group") {
         if (seg->is_build) throw ParseError{"'group' only in the probe segment"};
+        if (seg->hash_group) throw ParseError{"dense groups cannot follow 'group hash'"};
         GroupIR g;
         g.ref = parse_ref(c);
         g.lo = expect_int(c, "domain lower bound");
@@ -370,6 +403,12 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
     if ((int)seg->probes.size() > MAXP) throw ParseError{"too many probes"};
     if ((int)seg->wheres.size() > MAXR) throw ParseError{"too many where clauses"};
     if ((int)seg->groups.size() > MAXG) throw ParseError{"too many group dimensions"};
+    if ((seg->limit || !seg->order.empty()) && !seg->hash_group)
+      throw ParseError{"'order' / 'limit' need 'group hash' (dense group results are ordered on the host)"};
+    if (seg->limit && seg->order.empty()) throw ParseError{"'limit' needs an 'order' statement"};
+    for (auto& o : seg->order)
+      if (o.idx < 0 || (o.is_agg ? o.idx >= (int)seg->aggs.size() : o.idx >= (int)seg->groups.size()))
+        throw ParseError{"order component index out of range"};
     bool has_sum = false;
     for (auto& a : seg->aggs) has_sum |= a.kind != A_COUNT;
     if (has_sum && seg->value.empty()) throw ParseError{"'agg sum' needs a 'value' statement"};

@@ -42,7 +42,14 @@ struct WhereIR {
 
 struct GroupIR {
   RefIR ref;
-  int64_t lo = 0, hi = 0;  // domain [lo, hi)
+  int64_t lo = 0, hi = 0;  // domain [lo, hi) (dense group-by)
+};
+
+// ORDER BY component of a hash group-by result
+struct OrderIR {
+  bool is_agg = true;  // agg index (0 = COUNT) or group-key index
+  int idx = 0;
+  bool desc = false;
 };
 
 struct FactorIR {
@@ -77,6 +84,11 @@ struct Segment {
   std::vector<GroupIR> groups;
   std::vector<TermIR> value;
   std::vector<AggIR> aggs;  // agg 0 is always COUNT
+  // hash group-by over unbounded keys (NEXT-4): 'group hash A[, B]' (no
+  // domain), then optional 'order ...' / 'limit K' run on the device
+  bool hash_group = false;
+  std::vector<OrderIR> order;
+  int limit = 0;
   int split_hint = -2;      // -2: auto
   std::string text;
 };

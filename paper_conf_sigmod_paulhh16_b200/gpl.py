@@ -53,7 +53,8 @@ class _Stats(ctypes.Structure):
                 ("kernel_ms", ctypes.c_double), ("predicted_ms", ctypes.c_double),
                 ("bytes_scanned", ctypes.c_double), ("agg_mode", ctypes.c_int32), ("kbe", ctypes.c_int32),
                 ("jit", ctypes.c_int32), ("reserved", ctypes.c_int32), ("intermediate_bytes", ctypes.c_double),
-                ("bytes_full_scan", ctypes.c_double), ("lazy_columns", ctypes.c_int32), ("packets", ctypes.c_int32)]
+                ("bytes_full_scan", ctypes.c_double), ("lazy_columns", ctypes.c_int32), ("packets", ctypes.c_int32),
+                ("groups_total", ctypes.c_int64), ("hash_slots", ctypes.c_int64)]
 
 
 class _Result(ctypes.Structure):

@@ -437,13 +437,90 @@ def test_profiled_model_reproduces_its_run(ctx):
     db = tpchgen.generate(0.2, seed=12)
     queries.load_database(ctx, db, queries.TABLES["Q8"])
     o = oracle.run("Q8", db)
-    rs = [queries.run_query(ctx, "Q8", db) for _ in range(4)]
+    rs = [queries.run_query(ctx, "Q8", db) for _ in range(5)]
     for r in rs:
         assert r.keys == o.keys and r.aggs == o.aggs
+    # the profile is the faster of the first two timed runs with λ (runs 0-1, or 1-2 when this plan
+    # text had no λ yet); the re-planned run's estimate is close to what the kernel then takes
     last = rs[-1].stats
-    assert last["predicted_ms"] == pytest.approx(rs[1].stats["kernel_ms"], rel=0.35) or \
-        last["predicted_ms"] == pytest.approx(last["kernel_ms"], rel=0.5)
+    assert last["predicted_ms"] == pytest.approx(last["kernel_ms"], rel=0.5) or \
+        last["predicted_ms"] == pytest.approx(min(r.stats["kernel_ms"] for r in rs[:3]), rel=0.35)
     ctx.set_option("use_profile", 0)
     r = queries.run_query(ctx, "Q8", db)
     assert r.keys == o.keys and r.aggs == o.aggs
     ctx.set_option("use_profile", 1)
+
+
+# ---- hash group-by over unbounded keys + device ORDER BY/LIMIT (TPC-H Q3)
+
+def _q3_full_plan(db):
+    """Q3 without ORDER BY/LIMIT: every group, compacted on the device."""
+    return "\n".join(ln for ln in queries.plan_text("Q3", db).splitlines()
+                     if not ln.startswith(("order", "limit")))
+
+
+@pytest.mark.parametrize("sf,seed", [(0.01, 20160626), (0.2, 3), (1.0, 20160626)])
+def test_q3_hash_groupby_topk_exact(ctx, sf, seed):
+    db = tpchgen.generate(sf, seed=seed)
+    queries.load_database(ctx, db, queries.TABLES["Q3"])
+    o = oracle.run("Q3", db)
+    want = oracle.order_limit("Q3", o)
+    for _ in range(2):  # first run sizes the table from the rows, the second from the groups seen
+        r = queries.run_query(ctx, "Q3", db)
+        assert r.keys == want.keys and r.aggs == want.aggs
+        assert r.stats["groups_total"] == len(o.keys) and r.stats["agg_mode"] == 3
+        assert r.stats["hash_slots"] >= 2 * len(o.keys) or r.stats["hash_slots"] == 4096
+    # every group (no LIMIT): compaction + host key order (a table sized from another run may overflow
+    # once: the error is latched and the next run is sized from it)
+    for attempt in range(2):
+        ctx.run_query(_q3_full_plan(db))
+        try:
+            full = ctx.fetch_result()
+            break
+        except gpl.GplError as e:
+            assert e.status == gpl.GPL_E_CAPACITY and attempt == 0
+    assert full.keys == o.keys and full.aggs == o.aggs
+
+
+def test_q3_worked_example_ties(ctx):
+    fx = load("w5_q3.json")
+    db = build_db(fx)
+    queries.load_database(ctx, db, ["customer", "orders", "lineitem"])
+    r = queries.run_query(ctx, "Q3", db, fx["params"])
+    assert r.keys == [tuple(k) for k in fx["expected"]["order_limit"]]
+
+
+@pytest.mark.parametrize("n", [0, 1, 33, 4097])
+def test_q3_ragged_and_empty(ctx, n):
+    db = tpchgen.generate(0.05, seed=8)
+    db.tables["lineitem"] = {c: v[:n].copy() for c, v in db.tables["lineitem"].items()}
+    queries.load_database(ctx, db, queries.TABLES["Q3"])
+    o = oracle.run("Q3", db)
+    r = queries.run_query(ctx, "Q3", db)
+    want = oracle.order_limit("Q3", o)
+    assert r.keys == want.keys and r.aggs == want.aggs
+
+
+def test_q3_schedules_and_overflow(ctx):
+    db = tpchgen.generate(0.6, seed=4)
+    queries.load_database(ctx, db, queries.TABLES["Q3"])
+    o = oracle.run("Q3", db)
+    want = oracle.order_limit("Q3", o)
+    for opts in ({"stage_rows": 512, "ring_depth": 2, "consumer_warps": 2}, {"stage_rows": 2048, "packets": 2},
+                 {"probe_split": 0}, {"lazy_columns": 1}, {"lazy_columns": 0}):
+        for k, v in opts.items():
+            ctx.set_option(k, v)
+        for tile in (0, 4096):
+            r = queries.run_query(ctx, "Q3", db, tile_rows=tile)
+            assert r.keys == want.keys and r.aggs == want.aggs, opts
+        for k in opts:
+            ctx.set_option(k, -1)
+    # a table too small for the groups latches an overflow (never a wrong answer)
+    assert len(o.keys) > 4096
+    ctx.set_option("hash_slots_log2", 12)
+    with pytest.raises(gpl.GplError) as e:
+        queries.run_query(ctx, "Q3", db)
+    assert e.value.status == gpl.GPL_E_CAPACITY
+    ctx.set_option("hash_slots_log2", 0)
+    r = queries.run_query(ctx, "Q3", db)  # sized from the overflowed run: exact again
+    assert r.keys == want.keys and r.aggs == want.aggs
