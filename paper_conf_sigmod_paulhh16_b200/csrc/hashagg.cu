@@ -2,13 +2,14 @@
 // blocking operator after the fused pipeline (ORDER BY is blocking).
 //
 //   * ORDER BY ... LIMIT k: a two-phase device selection. Phase A: every CTA
-//     walks its slice of the hash-aggregation table, keeps its k best groups
-//     in shared memory (bitonic sort of a 1024-entry tile whenever new
-//     candidates arrive; once k entries are held, only groups better than the
-//     current k-th are admitted) and writes their slot indices. Phase B: one
-//     CTA runs the same selection over the candidates and writes the k rows
-//     in order — to the device row buffer and to the run's result words, so
-//     the copy-out kernel brings them back with the counters (no extra D2H).
+//     walks its slice of the hash-aggregation table in coalesced chunks and
+//     keeps its k best groups in a shared-memory tile: a group is admitted
+//     only if it beats the current k-th best, and the tile is bitonic-sorted
+//     only when its free room runs low (so after the first sort almost every
+//     group is rejected by one comparison). Phase B: one CTA runs the same
+//     selection over the CTAs' candidates and writes the k rows in order — to
+//     the device row buffer and to the run's result words, so the copy-out
+//     kernel brings them back with the counters (no extra D2H).
 //   * no LIMIT: every occupied slot is compacted into the row buffer (order
 //     arbitrary; the host orders by key).
 // A row is [packed key, acc 0 .. nagg-1] (8-byte words). Ordering: the plan's
@@ -20,15 +21,17 @@
 namespace gpl {
 namespace {
 
-constexpr int kTile = 1024;
 constexpr int kThreads = 256;
 constexpr unsigned kNone = 0xFFFFFFFFu;
 constexpr unsigned long long kSign = 1ull << 63;
 
+// Selection tile of T entries: the k best so far in [0, k), new candidates
+// appended after them.
+template <int T>
 struct SelSmem {
-  unsigned long long w[4][kTile];  // sort words (lexicographic, ascending = better)
-  unsigned idx[kTile];             // slot index (kNone = padding)
-  unsigned long long thr[4];       // the current k-th best (admission threshold)
+  unsigned long long w[4][T];  // sort words (lexicographic, ascending = better)
+  unsigned idx[T];             // slot index (kNone = padding)
+  unsigned long long thr[4];   // the current k-th best (admission threshold)
   int fill, have_thr;
 };
 
@@ -69,17 +72,19 @@ __device__ __forceinline__ bool less4(const unsigned long long (&a)[4], const un
   return false;
 }
 
-__device__ __forceinline__ bool less_at(const SelSmem& m, int i, int j) {
+template <int T>
+__device__ __forceinline__ bool less_at(const SelSmem<T>& m, int i, int j) {
 #pragma unroll
   for (int c = 0; c < 4; c++)
     if (m.w[c][i] != m.w[c][j]) return m.w[c][i] < m.w[c][j];
   return m.idx[i] < m.idx[j];
 }
 
-__device__ void bitonic_sort(SelSmem& m) {
-  for (int k = 2; k <= kTile; k <<= 1)
+template <int T>
+__device__ void bitonic_sort(SelSmem<T>& m) {
+  for (int k = 2; k <= T; k <<= 1)
     for (int j = k >> 1; j > 0; j >>= 1) {
-      for (int i = threadIdx.x; i < kTile; i += blockDim.x) {
+      for (int i = threadIdx.x; i < T; i += blockDim.x) {
         const int p = i ^ j;
         if (p > i) {
           const bool up = (i & k) == 0;
@@ -100,52 +105,60 @@ __device__ void bitonic_sort(SelSmem& m) {
     }
 }
 
-__device__ __forceinline__ void set_pad(SelSmem& m, int i) {
+template <int T>
+__device__ __forceinline__ void set_pad(SelSmem<T>& m, int i) {
 #pragma unroll
   for (int c = 0; c < 4; c++) m.w[c][i] = ~0ull;
   m.idx[i] = kNone;
 }
 
-// Keep the k best of [input range] in m.idx[0..k) (sorted, best first).
-// from_cand: the input is D.cand[lo..hi) (slot indices, kNone = none),
-// else the hash slots [lo, hi).
-__device__ void select_k(const HaggResultDesc& D, SelSmem& m, unsigned long long lo, unsigned long long hi,
+// Keep the k best of the input range in m.idx[0..k) (sorted, best first).
+// from_cand: the input is D.cand[lo..hi) (slot indices, kNone = none), else
+// the hash slots [lo, hi). One coalesced chunk of blockDim positions per
+// step; the tile is sorted only when its free room could not take another
+// chunk (or at the end).
+template <int T>
+__device__ void select_k(const HaggResultDesc& D, SelSmem<T>& m, unsigned long long lo, unsigned long long hi,
                          bool from_cand) {
   const int K = D.limit;
-  for (int i = threadIdx.x; i < kTile; i += blockDim.x) set_pad(m, i);
+  for (int i = threadIdx.x; i < T; i += blockDim.x) set_pad(m, i);
   if (threadIdx.x == 0) {
     m.fill = 0;
     m.have_thr = 0;
   }
   __syncthreads();
-  const int batch = kTile - K;
-  for (unsigned long long base = lo; base < hi; base += (unsigned long long)batch) {
-    for (int t = threadIdx.x; t < batch; t += blockDim.x) {
-      const unsigned long long pos = base + (unsigned long long)t;
-      if (pos >= hi) break;
+  const int room = T - K;  // >= blockDim (the launcher picks T from k)
+  for (unsigned long long base = lo; base < hi; base += blockDim.x) {
+    const unsigned long long pos = base + threadIdx.x;
+    if (pos < hi) {
       unsigned long long s = pos;
+      bool ok = true;
       if (from_cand) {
         const unsigned c = D.cand[pos];
-        if (c == kNone) continue;
+        ok = c != kNone;
         s = c;
       }
       unsigned long long w[4];
-      if (!words_of(D, s, w)) continue;
-      if (m.have_thr) {
-        unsigned long long th[4] = {m.thr[0], m.thr[1], m.thr[2], m.thr[3]};
-        if (!less4(w, th)) continue;
-      }
-      const int at = K + atomicAdd(&m.fill, 1);
+      if (ok && words_of(D, s, w)) {
+        bool admit = true;
+        if (m.have_thr) {
+          const unsigned long long th[4] = {m.thr[0], m.thr[1], m.thr[2], m.thr[3]};
+          admit = less4(w, th);
+        }
+        if (admit) {
+          const int at = K + atomicAdd(&m.fill, 1);
 #pragma unroll
-      for (int c = 0; c < 4; c++) m.w[c][at] = w[c];
-      m.idx[at] = (unsigned)s;
+          for (int c = 0; c < 4; c++) m.w[c][at] = w[c];
+          m.idx[at] = (unsigned)s;
+        }
+      }
     }
     __syncthreads();
-    const int fill = m.fill;
-    if (fill > 0) {  // uniform branch
+    const int fill = m.fill;  // uniform
+    if (fill > 0 && (fill > room - (int)blockDim.x || base + blockDim.x >= hi)) {
       bitonic_sort(m);
-      // entries [K, kTile) are dropped: reset them, record the threshold
-      for (int i = K + threadIdx.x; i < kTile; i += blockDim.x) set_pad(m, i);
+      // entries [K, T) are dropped: reset them, record the threshold
+      for (int i = K + threadIdx.x; i < T; i += blockDim.x) set_pad(m, i);
       if (threadIdx.x == 0) {
         m.fill = 0;
         if (m.idx[K - 1] != kNone) {
@@ -159,18 +172,20 @@ __device__ void select_k(const HaggResultDesc& D, SelSmem& m, unsigned long long
   }
 }
 
+template <int T>
 __global__ void __launch_bounds__(kThreads) select_phase_a(const __grid_constant__ HaggResultDesc D) {
-  __shared__ SelSmem m;
+  __shared__ SelSmem<T> m;
   const unsigned long long per = (D.nslots + gridDim.x - 1) / gridDim.x;
   const unsigned long long lo = per * blockIdx.x, hi = min(D.nslots, lo + per);
-  select_k(D, m, lo, lo < hi ? hi : lo, false);
+  select_k<T>(D, m, lo, lo < hi ? hi : lo, false);
   for (int i = threadIdx.x; i < D.limit; i += blockDim.x) D.cand[(unsigned long long)blockIdx.x * D.limit + i] = m.idx[i];
 }
 
+template <int T>
 __global__ void __launch_bounds__(kThreads) select_phase_b(const __grid_constant__ HaggResultDesc D,
                                                            const unsigned long long* hagg_count) {
-  __shared__ SelSmem m;
-  select_k(D, m, 0, (unsigned long long)D.nblocks * D.limit, true);
+  __shared__ SelSmem<T> m;
+  select_k<T>(D, m, 0, (unsigned long long)D.nblocks * D.limit, true);
   int n = 0;
   for (int i = 0; i < D.limit; i++) n += m.idx[i] != kNone;
   const int W = 1 + D.nagg;
@@ -202,16 +217,22 @@ __global__ void __launch_bounds__(kThreads) compact_groups(const __grid_constant
 }  // namespace
 
 int hagg_select_blocks(unsigned long long nslots, int num_sms) {
-  // one slice per CTA, >= 4K slots each, at most 2 CTAs per SM
-  const unsigned long long b = (nslots + 4095) / 4096;
+  // one slice per CTA, >= 1K slots each, at most 2 CTAs per SM
+  const unsigned long long b = (nslots + 1023) / 1024;
   return (int)(b < 1 ? 1 : b > (unsigned long long)(2 * num_sms) ? 2 * num_sms : b);
 }
 
 cudaError_t launch_hagg_result(const HaggResultDesc& D, const unsigned long long* hagg_count, int num_sms,
                                cudaStream_t s) {
   if (D.limit > 0) {
-    select_phase_a<<<D.nblocks, kThreads, 0, s>>>(D);
-    select_phase_b<<<1, kThreads, 0, s>>>(D, hagg_count);
+    // tile: room for the k best plus one chunk of candidates (k <= 512)
+    if (D.limit <= 512 - kThreads) {
+      select_phase_a<512><<<D.nblocks, kThreads, 0, s>>>(D);
+      select_phase_b<512><<<1, kThreads, 0, s>>>(D, hagg_count);
+    } else {
+      select_phase_a<1024><<<D.nblocks, kThreads, 0, s>>>(D);
+      select_phase_b<1024><<<1, kThreads, 0, s>>>(D, hagg_count);
+    }
   } else {
     const unsigned long long b = (D.nslots + kThreads - 1) / kThreads;
     compact_groups<<<(int)(b < 1 ? 1 : b > (unsigned long long)(4 * num_sms) ? 4 * num_sms : b), kThreads, 0, s>>>(D);

@@ -435,6 +435,7 @@ def test_profiled_model_reproduces_its_run(ctx):
     consumer cost is fitted to it, so re-planning the same shape predicts that run's time; results
     stay exact; use_profile = 0 restores the unfitted model."""
     db = tpchgen.generate(0.2, seed=12)
+    ctx.set_option("use_profile", 1)  # (also drops shapes pinned by earlier autotune tests: model-chosen runs)
     queries.load_database(ctx, db, queries.TABLES["Q8"])
     o = oracle.run("Q8", db)
     rs = [queries.run_query(ctx, "Q8", db) for _ in range(5)]

@@ -5,13 +5,14 @@ import subprocess
 import sys
 
 
-def raw(rep):
+def raw(rep, which=0):
+    """Metrics of the `which`-th kernel captured in the report."""
     out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(out.splitlines()))
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "usecond": 1, "msecond": 1e3,
              "second": 1e6}
     d = {}
-    for name, unit, val in zip(rows[0], rows[1], rows[2]):
+    for name, unit, val in zip(rows[0], rows[1], rows[2 + which]):
         if unit in scale:
             try:
                 val = str(float(val.replace(",", "")) * scale[unit])  # bytes / microseconds
@@ -37,8 +38,8 @@ def sass_counts(rep):
     return ops
 
 
-def summarise(rep, key):
-    d = raw(rep)
+def summarise(rep, key, which=0):
+    d = raw(rep, which)
     f = lambda k: float(d[k].replace(",", "")) if k in d and d[k] not in ("", "n/a") else None
     s = {
         "workload": key,
@@ -56,7 +57,7 @@ def summarise(rep, key):
                           for k in d if k.startswith("smsp__pcsamp_warps_issue_stalled_") and "not_issued" not in k
                           and f(k) and f(k) > 0},
     }
-    ops = sass_counts(rep)
+    ops = sass_counts(rep) if which == 0 else {}
     s["sass_evidence"] = {k: ops.get(k, 0) for k in ("UBLKCP", "SYNCS", "LDS", "STS", "LDG", "ATOMS", "RED", "ATOMG")}
     s["traffic_bytes"] = (s["dram_bytes_read"] or 0) + (s["dram_bytes_write"] or 0)
     return s
@@ -64,8 +65,12 @@ def summarise(rep, key):
 
 if __name__ == "__main__":
     out = sys.argv[1]
-    pairs = sys.argv[2:]
-    res = [summarise(pairs[i], pairs[i + 1]) for i in range(0, len(pairs), 2)]
+    pairs = sys.argv[2:]  # REP KEY [REP KEY ...]; KEY may end in "#n" for the n-th kernel of REP
+    res = []
+    for i in range(0, len(pairs), 2):
+        key = pairs[i + 1]
+        which = int(key.split("#")[1]) if "#" in key else 0
+        res.append(summarise(pairs[i], key, which))
     json.dump(res, open(out, "w"), indent=1)
     for r in res:
         print(json.dumps({k: r[k] for k in ("workload", "duration_us", "dram_bytes_read", "dram_bytes_write", "traffic_bytes")}))
