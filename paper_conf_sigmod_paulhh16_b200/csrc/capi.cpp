@@ -811,7 +811,7 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
     const size_t bytes = (size_t)cap * 8 * (1 + li.nagg);
     const size_t rbytes = (size_t)cap * 8 * (1 + li.nagg);
     const int nblocks = hagg_select_blocks(cap, ctx->sms);
-    const size_t cbytes = (size_t)nblocks * std::max(1, li.limit) * 4;
+    const size_t cbytes = (size_t)nblocks * std::max(1, li.limit) * 5 * 8;
     auto grow = [&](void** p, size_t* have, size_t need) -> cudaError_t {
       if (*have >= need) return cudaSuccess;
       cudaError_t e = cudaStreamSynchronize(ctx->stream);
@@ -1299,6 +1299,10 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     if (ms.size() < 3) continue;
     std::sort(ms.begin(), ms.end());
     tried++;
+    if (std::getenv("GPL_DEBUG_TUNE"))
+      std::fprintf(stderr, "autotune: split %d(eff %d) k %d S %d D %d W %d np %d tile %lld: %.4f ms (model %.4f)\n",
+                   sc.first, cand_split_eff[ci], c.ctas_per_sm, c.stage_rows, c.depth, c.warps, c.npack,
+                   (long long)c.tile_rows, ms[1], c.pred_ms);
     if (ms[1] < best_ms) {
       best_ms = ms[1];
       best = t;

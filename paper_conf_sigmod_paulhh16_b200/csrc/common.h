@@ -213,7 +213,7 @@ struct HaggResultDesc {
   int32_t limit;                   // 0: every group (compaction)
   int32_t norder;
   int32_t ord_is_agg[3], ord_idx[3], ord_desc[3];
-  unsigned int* cand;              // selection scratch: slot indices [nblocks * limit]
+  unsigned long long* cand;        // selection scratch: [nblocks * limit] x (4 sort words, slot index)
   int32_t nblocks, pad;
   unsigned long long* rows;        // out: n_out rows of (1 + nagg) words (device)
   unsigned long long* small_out;   // out (limit): [n_groups, n_out, rows...] in the partials area

@@ -220,7 +220,7 @@ struct gpl_ctx {
   size_t hagg_alloc = 0;
   unsigned long long* d_hres = nullptr;
   size_t hres_alloc = 0;
-  unsigned int* d_hcand = nullptr;
+  unsigned long long* d_hcand = nullptr;
   size_t hcand_alloc = 0;
   std::map<std::string, std::pair<uint64_t, int64_t>> hagg_groups;  // plan text -> (distinct groups, fact rows) of its last run
   // KBE scratch (gpl_run_plan_kbe)

@@ -27,12 +27,20 @@ constexpr unsigned long long kSign = 1ull << 63;
 
 // Selection tile of T entries: the k best so far in [0, k), new candidates
 // appended after them.
+constexpr int kSmallK = 32;  // k <= 32: compaction by k rounds of block arg-min, else bitonic sort
+
 template <int T>
 struct SelSmem {
   unsigned long long w[4][T];  // sort words (lexicographic, ascending = better)
-  unsigned idx[T];             // slot index (kNone = padding)
+  unsigned idx[T];             // slot index (kNone = padding / taken)
   unsigned long long thr[4];   // the current k-th best (admission threshold)
   int fill, have_thr;
+  // small-k selection: the rounds' winners and the per-warp arg-min scratch
+  unsigned long long selw[4][kSmallK];
+  unsigned selidx[kSmallK];
+  unsigned long long redw[4][kThreads / 32];
+  int redpos[kThreads / 32];
+  int nsel;
 };
 
 __device__ __forceinline__ int key_field(unsigned long long key, int nkeys, int i) {
@@ -105,6 +113,89 @@ __device__ void bitonic_sort(SelSmem<T>& m) {
     }
 }
 
+// The k best of tile entries [0, n) moved to [0, k) in order (k <= kSmallK):
+// k rounds of a block-wide arg-min (warp shuffles, then one warp over the
+// per-warp winners); a winner is marked taken (idx = kNone). Much cheaper
+// than sorting the tile when k is small.
+template <int T>
+__device__ void select_small(SelSmem<T>& m, int n, int K) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if (threadIdx.x == 0) m.nsel = 0;
+  for (int r = 0; r < K; r++) {
+    unsigned long long b[4] = {~0ull, ~0ull, ~0ull, ~0ull};
+    int bp = -1;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+      if (m.idx[i] == kNone) continue;
+      const unsigned long long x[4] = {m.w[0][i], m.w[1][i], m.w[2][i], m.w[3][i]};
+      if (bp < 0 || less4(x, b)) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) b[c] = x[c];
+        bp = i;
+      }
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      unsigned long long o[4];
+#pragma unroll
+      for (int c = 0; c < 4; c++) o[c] = __shfl_down_sync(0xffffffffu, b[c], off);
+      const int op = __shfl_down_sync(0xffffffffu, bp, off);
+      if (op >= 0 && (bp < 0 || less4(o, b))) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) b[c] = o[c];
+        bp = op;
+      }
+    }
+    if (lane == 0) {
+#pragma unroll
+      for (int c = 0; c < 4; c++) m.redw[c][warp] = b[c];
+      m.redpos[warp] = bp;
+    }
+    __syncthreads();
+    if (warp == 0) {
+      unsigned long long x[4] = {~0ull, ~0ull, ~0ull, ~0ull};
+      int xp = -1;
+      if (lane < nw) {
+#pragma unroll
+        for (int c = 0; c < 4; c++) x[c] = m.redw[c][lane];
+        xp = m.redpos[lane];
+      }
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        unsigned long long o[4];
+#pragma unroll
+        for (int c = 0; c < 4; c++) o[c] = __shfl_down_sync(0xffffffffu, x[c], off);
+        const int op = __shfl_down_sync(0xffffffffu, xp, off);
+        if (op >= 0 && (xp < 0 || less4(o, x))) {
+#pragma unroll
+          for (int c = 0; c < 4; c++) x[c] = o[c];
+          xp = op;
+        }
+      }
+      if (lane == 0 && xp >= 0) {
+        const int t = m.nsel++;
+#pragma unroll
+        for (int c = 0; c < 4; c++) m.selw[c][t] = x[c];
+        m.selidx[t] = m.idx[xp];
+        m.idx[xp] = kNone;
+      }
+    }
+    __syncthreads();
+  }
+  const int ns = m.nsel;
+  for (int i = threadIdx.x; i < T; i += blockDim.x) {
+    if (i < ns) {
+#pragma unroll
+      for (int c = 0; c < 4; c++) m.w[c][i] = m.selw[c][i];
+      m.idx[i] = m.selidx[i];
+    } else {
+#pragma unroll
+      for (int c = 0; c < 4; c++) m.w[c][i] = ~0ull;
+      m.idx[i] = kNone;
+    }
+  }
+  __syncthreads();
+}
+
 template <int T>
 __device__ __forceinline__ void set_pad(SelSmem<T>& m, int i) {
 #pragma unroll
@@ -113,8 +204,8 @@ __device__ __forceinline__ void set_pad(SelSmem<T>& m, int i) {
 }
 
 // Keep the k best of the input range in m.idx[0..k) (sorted, best first).
-// from_cand: the input is D.cand[lo..hi) (slot indices, kNone = none), else
-// the hash slots [lo, hi). One coalesced chunk of blockDim positions per
+// from_cand: the input is D.cand entries [lo..hi) (phase A's winners with
+// their sort words: 5 words each, idx kNone = none), else the hash slots. One coalesced chunk of blockDim positions per
 // step; the tile is sorted only when its free room could not take another
 // chunk (or at the end).
 template <int T>
@@ -132,14 +223,18 @@ __device__ void select_k(const HaggResultDesc& D, SelSmem<T>& m, unsigned long l
     const unsigned long long pos = base + threadIdx.x;
     if (pos < hi) {
       unsigned long long s = pos;
-      bool ok = true;
-      if (from_cand) {
-        const unsigned c = D.cand[pos];
-        ok = c != kNone;
-        s = c;
-      }
       unsigned long long w[4];
-      if (ok && words_of(D, s, w)) {
+      bool ok;
+      if (from_cand) {  // coalesced: the words travel with the candidate
+        const unsigned long long* e = D.cand + pos * 5;
+        s = e[4];
+        ok = s != kNone;
+#pragma unroll
+        for (int c = 0; c < 4; c++) w[c] = e[c];
+      } else {
+        ok = words_of(D, s, w);
+      }
+      if (ok) {
         bool admit = true;
         if (m.have_thr) {
           const unsigned long long th[4] = {m.thr[0], m.thr[1], m.thr[2], m.thr[3]};
@@ -156,9 +251,14 @@ __device__ void select_k(const HaggResultDesc& D, SelSmem<T>& m, unsigned long l
     __syncthreads();
     const int fill = m.fill;  // uniform
     if (fill > 0 && (fill > room - (int)blockDim.x || base + blockDim.x >= hi)) {
-      bitonic_sort(m);
-      // entries [K, T) are dropped: reset them, record the threshold
-      for (int i = K + threadIdx.x; i < T; i += blockDim.x) set_pad(m, i);
+      if (K <= kSmallK) {
+        select_small(m, K + fill, K);  // [0, K) best, the rest padding
+      } else {
+        bitonic_sort(m);
+        // entries [K, T) are dropped: reset them
+        for (int i = K + threadIdx.x; i < T; i += blockDim.x) set_pad(m, i);
+      }
+      // record the threshold (the k-th best)
       if (threadIdx.x == 0) {
         m.fill = 0;
         if (m.idx[K - 1] != kNone) {
@@ -178,7 +278,11 @@ __global__ void __launch_bounds__(kThreads) select_phase_a(const __grid_constant
   const unsigned long long per = (D.nslots + gridDim.x - 1) / gridDim.x;
   const unsigned long long lo = per * blockIdx.x, hi = min(D.nslots, lo + per);
   select_k<T>(D, m, lo, lo < hi ? hi : lo, false);
-  for (int i = threadIdx.x; i < D.limit; i += blockDim.x) D.cand[(unsigned long long)blockIdx.x * D.limit + i] = m.idx[i];
+  unsigned long long* out = D.cand + (unsigned long long)blockIdx.x * D.limit * 5;
+  for (int i = threadIdx.x; i < D.limit * 5; i += blockDim.x) {
+    const int e = i / 5, c = i % 5;
+    out[i] = c < 4 ? m.w[c][e] : (unsigned long long)m.idx[e];
+  }
 }
 
 template <int T>

@@ -37,7 +37,7 @@ cudaError_t launch_pipeline_fn(const void* fn, const PipeDesc& d, int grid, cuda
 bool jit_prepare(const PipeDesc& d, bool load, std::string* err);
 
 // Hash group-by result step (hashagg.cu): ORDER BY/LIMIT selection (D.limit
-// > 0; D.nblocks = hagg_select_blocks(...) CTAs, D.cand sized nblocks*limit)
+// > 0; D.nblocks = hagg_select_blocks(...) CTAs, D.cand sized nblocks*limit*5 words)
 // or compaction of every group. Plain stream order after the fused run.
 int hagg_select_blocks(unsigned long long nslots, int num_sms);
 cudaError_t launch_hagg_result(const HaggResultDesc& D, const unsigned long long* hagg_count, int num_sms,

@@ -28,7 +28,7 @@ def host_ctx():
     return ctx, db
 
 
-@pytest.mark.parametrize("q", queries.QUERIES)
+@pytest.mark.parametrize("q", queries.QUERIES + queries.EXTRA_QUERIES)
 def test_plans_validate(host_ctx, q):
     ctx, db = host_ctx
     segs = queries.segments(queries.plan_text(q, db))
@@ -56,6 +56,14 @@ def test_plan_errors(host_ctx):
         "run lineitem\nfilter l_partkey in {64}": gpl.GPL_E_PLAN,
         "run lineitem\ngroup l_partkey 5 5": gpl.GPL_E_PLAN,
         "run lineitem\nvalue l_extendedprice * l_extendedprice * l_extendedprice\nagg sum": gpl.GPL_E_OVERFLOW,
+        # hash group-by / device ORDER BY-LIMIT (NEXT-4)
+        "run lineitem\nagg count\norder agg 0 desc\nlimit 3": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup hash l_orderkey\nagg count\nlimit 3": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup hash l_orderkey\nagg count\norder agg 1 desc": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup hash l_orderkey\nagg count\norder key 0 asc\nlimit 513": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup hash l_orderkey, l_partkey, l_suppkey\nagg count": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup hash l_orderkey\ngroup l_suppkey 0 10\nagg count": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup hash l_orderkey\nvalue l_extendedprice * l_extendedprice\nagg sum": gpl.GPL_E_OVERFLOW,
     }
     for text, status in bad.items():
         with pytest.raises(gpl.GplError) as e:
@@ -141,7 +149,7 @@ def test_jit_compiles_every_plan():
     db = tpchgen.generate(0.01, seed=1)
     ctx = gpl.Context(device=-1)
     queries.load_database(ctx, db)
-    for q in queries.QUERIES:
+    for q in queries.QUERIES + queries.EXTRA_QUERIES:  # Q3: the hash group-by sink (AGG_HASH)
         segs = queries.segments(queries.plan_text(q, db, (19981101,) if q == "L1" else None))
         try:
             for s in segs[:-1]:
