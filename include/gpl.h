@@ -286,6 +286,8 @@ gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t
  * with an insert sink, default; 0 = the standalone build kernels),
  * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input),
  * "use_gamma" (1 = the model uses the Γ calibration when loaded, default),
+ * "graph_branches" (1 = gpl_run_query's graph runs build segments that do
+ * not depend on each other on two lanes, default; 0 = one chain),
  * "hash_slots_log2" (hash group-by table of 2^v slots; 0 = sized from the
  * plan's last run, default), "use_profile" (1 = the model fits its consumer cost to the plan's first
  * timed run after its λ profile, Table 2 "profiling input", default).

@@ -267,6 +267,9 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     if (ctx->d_hagg) cudaFree(ctx->d_hagg);
     if (ctx->d_hres) cudaFree(ctx->d_hres);
     if (ctx->d_hcand) cudaFree(ctx->d_hcand);
+    if (ctx->side) cudaStreamDestroy(ctx->side);
+    for (auto& e : ctx->fork_ev)
+      if (e) cudaEventDestroy(e);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
     if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
@@ -311,6 +314,12 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "hash_slots_log2") {
     if (v > 0 && (v < 12 || v > 34)) return fail(ctx, GPL_E_ARG, "hash_slots_log2 in [12, 34] (0 = auto)");
     o.hash_slots_log2 = v > 0 ? v : 0;
+  } else if (k == "graph_branches") {
+    // only how whole-query graphs are recorded: drop them, keep plans and pinned shapes
+    o.graph_branches = v != 0 ? 1 : 0;
+    for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
+    ctx->graphs.clear();
+    return GPL_OK;
   } else if (k == "use_profile") {
     o.use_profile = v != 0 ? 1 : 0;
   } else if (k == "use_gamma") {
@@ -1055,9 +1064,53 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     if (R.li.hash_group) add(R.desc.hagg_keys, R.hagg_clear);
     if (L.n > 16) return eager();
     CK(launch_clear(L, ctx->sms, ctx->stream));
-    for (const PreparedBuild* B : builds) {
-      if (B->pipe) CK(launch_pipeline_fn(B->pfn, B->pdesc, B->pgrid, ctx->stream));
-      else CK(launch_build(B->desc, B->trivial, B->known, ctx->sms, ctx->stream));
+    // Build segments form a DAG (a build depends on the tables it probes,
+    // each segment ends at its blocking build). Two capture lanes:
+    // a build runs on the lane of the builds it depends on (joining the other
+    // lane by an event when it depends on both), an independent build on the
+    // lane that has fewer; the run joins both. Small dimension builds then
+    // overlap instead of queueing behind each other.
+    auto launch_b = [&](const PreparedBuild* B, cudaStream_t st) -> gpl_status {
+      if (B->pipe) CK(launch_pipeline_fn(B->pfn, B->pdesc, B->pgrid, st));
+      else CK(launch_build(B->desc, B->trivial, B->known, ctx->sms, st));
+      return GPL_OK;
+    };
+    bool two = ctx->opt.graph_branches && builds.size() >= 2;
+    if (two && !ctx->side) {
+      two = cudaStreamCreateWithFlags(&ctx->side, cudaStreamNonBlocking) == cudaSuccess;
+      for (auto& e : ctx->fork_ev)
+        if (two && !e) two = cudaEventCreateWithFlags(&e, cudaEventDisableTiming) == cudaSuccess;
+    }
+    if (!two) {
+      for (const PreparedBuild* B : builds)
+        if (gpl_status s2 = launch_b(B, ctx->stream)) return s2;
+    } else {
+      int nev = 0;
+      auto join = [&](cudaStream_t from, cudaStream_t to) -> gpl_status {
+        if (nev >= 8) return fail(ctx, GPL_E_CUDA, "too many graph lane joins");
+        CK(cudaEventRecord(ctx->fork_ev[nev], from));
+        CK(cudaStreamWaitEvent(to, ctx->fork_ev[nev], 0));
+        nev++;
+        return GPL_OK;
+      };
+      cudaStream_t lane_st[2] = {ctx->stream, ctx->side};
+      if (gpl_status s2 = join(ctx->stream, ctx->side)) return s2;  // the side lane starts after the clear
+      std::map<int, int> lane_of;  // hash-table id -> lane that builds it
+      int count[2] = {0, 0};
+      for (const PreparedBuild* B : builds) {
+        bool dep[2] = {false, false};
+        for (int id : B->src_ids) {
+          auto it = lane_of.find(id);
+          if (it != lane_of.end()) dep[it->second] = true;
+        }
+        int ln = dep[0] ? 0 : dep[1] ? 1 : (count[1] < count[0] ? 1 : 0);
+        if (dep[0] && dep[1])
+          if (gpl_status s2 = join(lane_st[1], lane_st[0])) return s2;
+        if (gpl_status s2 = launch_b(B, lane_st[ln])) return s2;
+        lane_of[B->ht_index] = ln;
+        count[ln]++;
+      }
+      if (gpl_status s2 = join(ctx->side, ctx->stream)) return s2;  // the run waits for both lanes
     }
     CK(record_event(ctx, ctx->ev0));
     CK(launch_pipeline_fn(R.fn, R.desc, R.grid, ctx->stream));
@@ -1263,6 +1316,27 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     }
     if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
     with_warp_variants(ctx, ds, ls, ds.nrows, &cs);
+    if (ls.cons_factor != 1 || ls.bw_factor != 1) {
+      // the profile-fitted model and the plain one disagree on each shape's best
+      // depth / warps / Δ: measure both shortlists (a fitted model must never
+      // hide a configuration the plain model would have offered)
+      LowerInfo lr = ls;
+      lr.cons_factor = lr.bw_factor = 1;
+      Config b2;
+      std::vector<Config> cr;
+      if (choose_config(ctx, ds, lr, ds.nrows, 0, &b2, &err, &cr)) {
+        if (max_candidates > 0 && (int)cr.size() > max_candidates) cr.resize(max_candidates);
+        with_warp_variants(ctx, ds, lr, ds.nrows, &cr);
+        for (const Config& c : cr) {
+          bool dup = false;
+          for (const Config& x : cs)
+            dup |= x.tile_rows == c.tile_rows && x.stage_rows == c.stage_rows && x.depth == c.depth &&
+                   x.warps == c.warps && x.ctas_per_sm == c.ctas_per_sm && x.npack == c.npack;
+          if (!dup) cs.push_back(c);
+        }
+      }
+      err.clear();
+    }
     for (const Config& c : cs) {
       cands.push_back({sp, c});
       cand_split_eff.push_back(ds.nsprobe);

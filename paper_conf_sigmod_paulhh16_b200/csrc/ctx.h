@@ -164,6 +164,7 @@ struct Options {
   int64_t use_gamma = 1;       // the model uses the channel calibration Γ when one is loaded
   int64_t use_profile = 1;     // the model fits its consumer cost to the plan's profiled run
   int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
+  int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
 };
 
 // Γ of one ring shape (gpl_calibrate, Eq 1): (bytes, GB/s)
@@ -195,6 +196,10 @@ struct gpl_ctx {
   long long* d_minmax = nullptr;
   size_t minmax_cap = 0;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  // whole-query graphs: a second capture lane for build segments that do not
+  // depend on each other (fork/join events, created on first use)
+  cudaStream_t side = nullptr;
+  cudaEvent_t fork_ev[8] = {};
   gpl::LastRun last;
   gpl::Options opt;
   uint64_t opt_version = 1;  // bumped by gpl_set_option (invalidates prepared plans)

@@ -530,3 +530,20 @@ def test_q3_schedules_and_overflow(ctx):
     ctx.set_option("hash_slots_log2", 0)
     r = queries.run_query(ctx, "Q3", db)  # sized from the overflowed run: exact again
     assert r.keys == want.keys and r.aggs == want.aggs
+
+
+@pytest.mark.parametrize("q", ["Q5", "Q8", "Q9", "Q3"])
+def test_graph_branches_exact(ctx, q):
+    """Whole-query graphs with independent build segments on two capture lanes (fork/join events) give
+    the oracle's result on every replay, as the one-lane chain does."""
+    db = tpchgen.generate(0.1, seed=17)
+    queries.load_database(ctx, db, queries.TABLES[q])
+    o = oracle.run(q, db)
+    if q == "Q3":
+        o = oracle.order_limit("Q3", o)
+    for br in (1, 0, 1):
+        ctx.set_option("graph_branches", br)
+        for _ in range(3):  # eager run, capture, replays
+            r = queries.run_query(ctx, q, db)
+            assert r.keys == o.keys and r.aggs == o.aggs, (q, br)
+    ctx.set_option("graph_branches", 1)
