@@ -250,7 +250,9 @@ def main():
     if not args.no_autotune and args.tile_rows == 0:
         tuned = ctx.autotune(text)
         log(f"[rank {rank}] autotune: {tuned}")
-    for _ in range(args.warmup):
+    # warm-up: W steps; without autotune at least 6, since the first runs profile
+    # the plan (λ, then two timed runs for the model) and re-plan it once
+    for _ in range(args.warmup if tuned else max(args.warmup, 6)):
         res = step()
     res0 = ctx.fetch_result() if world == 1 else res
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
