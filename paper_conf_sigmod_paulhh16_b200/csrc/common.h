@@ -147,6 +147,7 @@ struct PipeDesc {
   long long tile_rows;
   int32_t stage_rows, depth, nwarps, flush_each_tile;
   int32_t npack;  // 128-row packets per consumer iteration (1 or 2: stage-phase probes of both in flight)
+  int32_t min_blocks;  // CTAs per SM the configuration runs (JIT: __launch_bounds__ minimum, caps registers)
   // stage phase (A4 + first probes)
   int32_t nfilt, nsprobe, nprobe, npush;
   Filt filt[MAXF];

@@ -70,6 +70,7 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->depth = c.depth;
   d->nwarps = c.warps;
   d->npack = c.npack;
+  d->min_blocks = c.ctas_per_sm;
   d->off_queue = kFixed;
   d->off_agg = align128(kFixed + c.warps * d->qbytes);
   int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
@@ -106,9 +107,13 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.smem = smem_bytes(d, li, S, depth, W);
   // Eq 2 analog: shared memory (228 KB per SM, 1 KB reserved per CTA),
   // threads and registers (<= 80 per thread assumed) of k resident CTAs
+  // registers: the generic kernel needs ~80 (112 with two packets); a
+  // plan-specialised kernel is compiled with the shape's exact launch bounds,
+  // so it fits down to 64 (80) registers per thread
+  const int regs_need = ctx->opt.jit ? (npack == 2 ? 80 : 64) : (npack == 2 ? 112 : 80);
   c.feasible = c.smem <= ctx->smem_optin && k * (c.smem + 1024) <= 228 * 1024 && W >= 1 &&
                W <= pipeline_max_consumer_warps() && depth >= 2 && k * (W + 1) * 32 <= 2048 &&
-               k * (W + 1) * 32 * (npack == 2 ? 112 : 80) <= 65536 && (npack == 1 || npack == 2);
+               k * (W + 1) * 32 * regs_need <= 65536 && (npack == 1 || npack == 2);
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
   // bytes per row: staged columns, plus one 32-B sector per surviving row of

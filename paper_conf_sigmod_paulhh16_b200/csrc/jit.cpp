@@ -106,6 +106,7 @@ std::string shape_source(const PipeDesc& d) {
   I("depth", d.depth);
   I("nwarps", d.nwarps);
   I("npack", d.npack);
+  I("min_blocks", d.min_blocks);
   I("flush_each_tile", d.flush_each_tile);
   I("nfilt", d.nfilt);
   I("nsprobe", d.nsprobe);
@@ -188,10 +189,15 @@ std::string shape_source(const PipeDesc& d) {
   return o.str();
 }
 
-std::string program_source(const std::string& shape) {
+// Launch bounds of the shape: exactly its (warps + 1) x 32 threads and its
+// CTAs per SM, so the register budget is the one the configuration can use
+// (2 CTAs of 12+1 warps -> <= 78 registers; the generic kernel assumes 1 CTA
+// of 17 warps).
+std::string program_source(const std::string& shape, int threads, int min_blocks) {
   return "#define GPL_JIT 1\n#include \"common.h\"\n" + shape +
          "#define GPL_SHAPE_OF(d) (::gpl_jit::kShape)\n#include \"pipeline_body.cuh\"\n"
-         "extern \"C\" __global__ void __launch_bounds__(gpl::pipe::kMaxThreads, 1)\n"
+         "extern \"C\" __global__ void __launch_bounds__(" + std::to_string(threads) + ", " +
+         std::to_string(min_blocks < 1 ? 1 : min_blocks) + ")\n"
          "gpl_pipeline_jit(const __grid_constant__ gpl::PipeDesc d) { gpl::pipe::pipeline_body(d); }\n";
 }
 
@@ -247,7 +253,7 @@ bool jit_prepare(const PipeDesc& d, bool load, std::string* err) {
     *err = e.err;
     return false;
   }
-  if (e.cubin.empty() && !compile(program_source(key), &e.cubin, &e.err)) {
+  if (e.cubin.empty() && !compile(program_source(key, (d.nwarps + 1) * 32, d.min_blocks), &e.cubin, &e.err)) {
     *err = e.err;
     return false;
   }
