@@ -381,7 +381,8 @@ def main():
         "clocks": clk.summary(),
         "wall_s_timed_region": wall,
         "pipeline": {k: stats.get(k) for k in ("tile_rows_used", "stage_rows", "ring_depth", "consumer_warps", "grid",
-                                               "probe_split", "predicted_ms", "agg_mode", "packets", "lazy_columns")},
+                                               "probe_split", "predicted_ms", "agg_mode", "packets", "lazy_columns",
+                                               "drain_warps")},
         "op_pass": stats["op_pass"],
         "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
         "jit": stats.get("jit"),

@@ -98,6 +98,8 @@ typedef struct {
   int32_t packets;             /* 128-row packets per consumer iteration                          */
   int64_t groups_total;        /* hash group-by: distinct groups (the result may be LIMITed)      */
   int64_t hash_slots;          /* hash group-by: slots of the aggregation table                    */
+  int32_t drain_warps;         /* of consumer_warps, those that only drain hand-off packets (NEXT-1) */
+  int32_t reserved2;
 } gpl_stats;
 
 /* Result of the last run. Arrays are CALLER-owned with capacity cap_groups. */
@@ -286,6 +288,9 @@ gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t
  * with an insert sink, default; 0 = the standalone build kernels),
  * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input),
  * "use_gamma" (1 = the model uses the Γ calibration when loaded, default),
+ * "drain_warps" (operator-specialised consumer warps, NEXT-1: of the
+ * consumer warps, this many only run the queue phase of survivor packets the
+ * others hand over; -1 = the model's choice from {0, 1, 2}, default),
  * "graph_branches" (1 = gpl_run_query's graph runs build segments that do
  * not depend on each other on two lanes, default; 0 = one chain),
  * "hash_slots_log2" (hash group-by table of 2^v slots; 0 = sized from the

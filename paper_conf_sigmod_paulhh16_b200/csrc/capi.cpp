@@ -314,6 +314,9 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "hash_slots_log2") {
     if (v > 0 && (v < 12 || v > 34)) return fail(ctx, GPL_E_ARG, "hash_slots_log2 in [12, 34] (0 = auto)");
     o.hash_slots_log2 = v > 0 ? v : 0;
+  } else if (k == "drain_warps") {
+    if (v >= 0 && v > 4) return fail(ctx, GPL_E_ARG, "drain_warps in [0, 4] (-1 = model)");
+    o.drain_warps = v < 0 ? -1 : v;
   } else if (k == "graph_branches") {
     // only how whole-query graphs are recorded: drop them, keep plans and pinned shapes
     o.graph_branches = v != 0 ? 1 : 0;
@@ -577,7 +580,7 @@ static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTab
   if (tu != ctx->tuned.end()) {
     const TunedShape& t = tu->second;
     *cfg = predict(ctx, *pd, li, std::max<int64_t>(pd->nrows, 1), t.tile_rows, t.stage_rows, t.depth, t.warps,
-                   t.ctas_per_sm, t.npack);
+                   t.ctas_per_sm, t.npack, t.ndrain);
   } else if (!choose_config(ctx, *pd, li, pd->nrows, 0, cfg, &err, shortlist)) {
     return fail(ctx, GPL_E_ARG, err);
   }
@@ -771,7 +774,7 @@ static gpl_status prepare_run(gpl_ctx* ctx, const char* text, int64_t tile_rows,
   if (tu != ctx->tuned.end()) {  // shape pinned by gpl_autotune
     const TunedShape& t = tu->second;
     *cfg = predict(ctx, *d, *li, std::max<int64_t>(d->nrows, 1), t.tile_rows, t.stage_rows, t.depth, t.warps,
-                   t.ctas_per_sm, t.npack);
+                   t.ctas_per_sm, t.npack, t.ndrain);
   } else if (!choose_config(ctx, *d, *li, d->nrows, tile_rows, cfg, &err)) {
     return fail(ctx, GPL_E_ARG, err);
   }
@@ -936,6 +939,7 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   S.agg_mode = d.agg_mode;
   S.jit = P->jit ? 1 : 0;
   S.hash_slots = (int64_t)P->hagg_cap;
+  S.drain_warps = d.ndrain;
   return GPL_OK;
 }
 
@@ -1034,6 +1038,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       S.agg_mode = P.desc.agg_mode;
       S.jit = P.jit ? 1 : 0;
       S.hash_slots = (int64_t)P.hagg_cap;
+      S.drain_warps = P.desc.ndrain;
       return GPL_OK;
     }
     cudaGraphExecDestroy(g->second);
@@ -1152,9 +1157,18 @@ static void with_warp_variants(const gpl_ctx* ctx, const PipeDesc& d, const Lowe
     if (i >= top) continue;
     for (int W : {4, 8, 12, 16}) {
       if (W == c.warps) continue;
-      Config v = predict(ctx, d, li, std::max<int64_t>(N, 1), c.tile_rows, c.stage_rows, c.depth, W, c.ctas_per_sm, c.npack);
+      Config v = predict(ctx, d, li, std::max<int64_t>(N, 1), c.tile_rows, c.stage_rows, c.depth, W, c.ctas_per_sm, c.npack,
+                         c.ndrain);
       if (v.feasible) out.push_back(v);
     }
+    // operator-specialised drain warps (NEXT-1): the same shape with 0, 1, 2 of its warps draining
+    if (ctx->opt.drain_warps < 0)
+      for (int nd : {0, 1, 2}) {
+        if (nd == c.ndrain) continue;
+        Config v = predict(ctx, d, li, std::max<int64_t>(N, 1), c.tile_rows, c.stage_rows, c.depth, c.warps,
+                           c.ctas_per_sm, c.npack, nd);
+        if (v.feasible) out.push_back(v);
+      }
   }
   cs->swap(out);
 }
@@ -1196,7 +1210,7 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
   bool has0 = false;
   for (const Config& c : cs)
     has0 |= c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
-            c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack;
+            c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack && c.ndrain == c0.ndrain;
   if (!has0) cs.insert(cs.begin(), c0);
   cudaEvent_t a = nullptr, b = nullptr;
   CK(cudaEventCreate(&a));
@@ -1204,7 +1218,7 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
   double best_ms = 1e300, m0 = -1;
   TunedShape best;
   for (const Config& c : cs) {
-    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, -2, c.npack};
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, -2, c.npack, c.ndrain};
     ctx->tuned[s.text] = t;
     ctx->build_cache.erase(text);
     std::vector<float> ms;
@@ -1227,7 +1241,7 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
     }
     std::sort(ms.begin(), ms.end());
     if (m0 < 0 && c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
-        c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack)
+        c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack && c.ndrain == c0.ndrain)
       m0 = ms[1];
     if (ms[1] < best_ms) {
       best_ms = ms[1];
@@ -1331,7 +1345,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
           bool dup = false;
           for (const Config& x : cs)
             dup |= x.tile_rows == c.tile_rows && x.stage_rows == c.stage_rows && x.depth == c.depth &&
-                   x.warps == c.warps && x.ctas_per_sm == c.ctas_per_sm && x.npack == c.npack;
+                   x.warps == c.warps && x.ctas_per_sm == c.ctas_per_sm && x.npack == c.npack && x.ndrain == c.ndrain;
           if (!dup) cs.push_back(c);
         }
       }
@@ -1353,7 +1367,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   for (size_t ci = 0; ci < cands.size(); ci++) {
     const auto& sc = cands[ci];
     const Config& c = sc.second;
-    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sc.first, c.npack};
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sc.first, c.npack, c.ndrain};
     ctx->tuned[seg.text] = t;
     ctx->run_cache.erase(probe + "\x1f" + std::to_string(0));
     std::vector<float> ms;
@@ -1374,8 +1388,8 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     std::sort(ms.begin(), ms.end());
     tried++;
     if (std::getenv("GPL_DEBUG_TUNE"))
-      std::fprintf(stderr, "autotune: split %d(eff %d) k %d S %d D %d W %d np %d tile %lld: %.4f ms (model %.4f)\n",
-                   sc.first, cand_split_eff[ci], c.ctas_per_sm, c.stage_rows, c.depth, c.warps, c.npack,
+      std::fprintf(stderr, "autotune: split %d(eff %d) k %d S %d D %d W %d dr %d np %d tile %lld: %.4f ms (model %.4f)\n",
+                   sc.first, cand_split_eff[ci], c.ctas_per_sm, c.stage_rows, c.depth, c.warps, c.ndrain, c.npack,
                    (long long)c.tile_rows, ms[1], c.pred_ms);
     if (ms[1] < best_ms) {
       best_ms = ms[1];
@@ -1394,7 +1408,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   ctx->graphs.clear();
   if (out) {
     const Config c = predict(ctx, d, li, std::max<int64_t>(d.nrows, 1), best.tile_rows, best.stage_rows, best.depth,
-                             best.warps, best.ctas_per_sm, best.npack);
+                             best.warps, best.ctas_per_sm, best.npack, best.ndrain);
     *out = gpl_model_report{};
     out->tile_rows = c.tile_rows;
     out->stage_rows = c.stage_rows;
@@ -1579,7 +1593,8 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
     auto old = ctx->profile.find(R.text);
     if (old != ctx->profile.end() && old->second.runs == 1 && old->second.table_version == ver &&
         old->second.tile_rows == R.desc.tile_rows && old->second.stage_rows == R.desc.stage_rows &&
-        old->second.depth == R.desc.depth && old->second.warps == R.desc.nwarps && old->second.npack == R.desc.npack) {
+        old->second.depth == R.desc.depth && old->second.warps == R.desc.nwarps && old->second.npack == R.desc.npack &&
+        old->second.ndrain == R.desc.ndrain) {
       old->second.kernel_ms = std::min(old->second.kernel_ms, S.kernel_ms);
       old->second.runs = 2;
     } else {
@@ -1590,6 +1605,7 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
       p.depth = R.desc.depth;
       p.warps = R.desc.nwarps;
       p.npack = R.desc.npack;
+      p.ndrain = R.desc.ndrain;
       p.ctas_per_sm = std::max(1, R.grid / std::max(1, ctx->sms));
       p.kernel_ms = S.kernel_ms;
       p.table_version = ver;

@@ -148,6 +148,12 @@ struct PipeDesc {
   int32_t stage_rows, depth, nwarps, flush_each_tile;
   int32_t npack;  // 128-row packets per consumer iteration (1 or 2: stage-phase probes of both in flight)
   int32_t min_blocks;  // CTAs per SM the configuration runs (JIT: __launch_bounds__ minimum, caps registers)
+  // operator-specialised consumer warps (the paper's
+  // per-operator kernels and work-group counts, Eq 8): the last
+  // ndrain consumer warps only drain survivor packets that the stage warps
+  // hand over through a 2*ndrain-slot shared-memory ring (0: every consumer
+  // warp drains its own queue)
+  int32_t ndrain;
   // stage phase (A4 + first probes)
   int32_t nfilt, nsprobe, nprobe, npush;
   Filt filt[MAXF];

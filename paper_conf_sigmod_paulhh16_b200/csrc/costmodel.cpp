@@ -54,8 +54,9 @@ int cl_cap_bytes(const PipeDesc& d, int S) {
   return align128((w == 0 ? (4 * S + 7) / 8 : 4 * S * w) + 32);
 }
 
-int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps) {
-  int q = warps * d.qbytes;
+int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps, int ndrain) {
+  // per-warp queues of the stage warps + the 2*ndrain hand-off slots
+  int q = (warps + ndrain) * d.qbytes;
   int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   int slot = 0;
   for (int c = 0; c < d.ncols; c++)
@@ -71,8 +72,9 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->nwarps = c.warps;
   d->npack = c.npack;
   d->min_blocks = c.ctas_per_sm;
+  d->ndrain = c.ndrain;
   d->off_queue = kFixed;
-  d->off_agg = align128(kFixed + c.warps * d->qbytes);
+  d->off_agg = align128(kFixed + (c.warps + c.ndrain) * d->qbytes);
   int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
   const int off_tables = d->off_agg + align128(agg);
   for (int i = 0; i < d->nht; i++)
@@ -95,16 +97,17 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
 }
 
 Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t N, int64_t tile,
-               int S, int depth, int W, int k, int npack) {
+               int S, int depth, int W, int k, int npack, int ndrain) {
   Config c;
   c.npack = npack;
+  c.ndrain = ndrain;
   c.tile_rows = tile;
   c.stage_rows = S;
   c.depth = depth;
   c.warps = W;
   c.ctas_per_sm = k;
   c.grid = ctx->sms * k;
-  c.smem = smem_bytes(d, li, S, depth, W);
+  c.smem = smem_bytes(d, li, S, depth, W, ndrain);
   // Eq 2 analog: shared memory (228 KB per SM, 1 KB reserved per CTA),
   // threads and registers (<= 80 per thread assumed) of k resident CTAs
   // registers: the generic kernel needs ~80 (112 with two packets); a
@@ -113,7 +116,8 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   const int regs_need = ctx->opt.jit ? (npack == 2 ? 80 : 64) : (npack == 2 ? 112 : 80);
   c.feasible = c.smem <= ctx->smem_optin && k * (c.smem + 1024) <= 228 * 1024 && W >= 1 &&
                W <= pipeline_max_consumer_warps() && depth >= 2 && k * (W + 1) * 32 <= 2048 &&
-               k * (W + 1) * 32 * regs_need <= 65536 && (npack == 1 || npack == 2);
+               k * (W + 1) * 32 * regs_need <= 65536 && (npack == 1 || npack == 2) && ndrain >= 0 &&
+               ndrain <= 4 && W - ndrain >= 1 && (ndrain == 0 || (d.npush > 0 && !(d.sink == SINK_INSERT && d.ins_kcol >= 0)));
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
   // bytes per row: staged columns, plus one 32-B sector per surviving row of
@@ -177,10 +181,25 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   if (!li.lazy_reach.empty()) lat_queue += 2000.0;
   // cycles per warp iteration of `npack` packets: the stage-phase probe
   // latency is paid once per iteration (all npack*4 loads of a lane in flight)
-  const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);
-  const double w_eff = (double)std::min(W, S / (128 * npack)) * k;          // warps with work per stage
-  const double rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 * npack / crit) /
-                          std::max(li.cons_factor, 1e-3);  // per SM (profile-fitted scale)
+  double rows_cyc;  // fact rows per cycle per SM the consumer warps sustain
+  if (ndrain == 0) {
+    const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);
+    const double w_eff = (double)std::min(W, S / (128 * npack)) * k;  // warps with work per stage
+    rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 * npack / crit);
+  } else {
+    // operator-specialised warps (NEXT-1): stage warps never block on the
+    // queue phase; drain warps absorb qfrac of the rows at one 128-row packet
+    // per (queue latency + queue work). The consumers sustain the slower of
+    // the two groups; Eq 8's delay between them is what the ring and the
+    // hand-off slots must absorb (min() below: the faster group idles).
+    const int Wsg = W - ndrain;
+    const double crit_s = 150.0 + lat_stage + npack * stage_cost;
+    const double w_eff = (double)std::min(Wsg, S / (128 * npack)) * k;
+    const double r_stage = w_eff * 128.0 * npack / crit_s;
+    const double r_drain = qfrac > 0 ? (double)ndrain * k * 128.0 / (lat_queue + queue_cost + 60.0) / qfrac : 1e30;
+    rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, std::min(r_stage, r_drain));
+  }
+  rows_cyc /= std::max(li.cons_factor, 1e-3);  // profile-fitted scale
   const double R_cons = rows_cyc * f_sm * b;                                // bytes/s one SM's consumers absorb
   const double t_cons = (double)N / (rows_cyc * f_sm * ctx->sms);
 
@@ -220,6 +239,10 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
   std::vector<int> Ws = o.consumer_warps > 0 ? std::vector<int>{(int)o.consumer_warps} : std::vector<int>{4, 8, 12, 16};
   std::vector<int> Ks = o.ctas_per_sm > 0 ? std::vector<int>{(int)o.ctas_per_sm} : std::vector<int>{1, 2};
   std::vector<int> Ps = o.packets > 0 ? std::vector<int>{(int)o.packets} : std::vector<int>{1, 2};
+  // drain warps only for a segment with a queue phase (not a stage-phase insert)
+  const bool can_drain = d.npush > 0 && !(d.sink == SINK_INSERT && d.ins_kcol >= 0);
+  std::vector<int> Dr = !can_drain ? std::vector<int>{0}
+                        : o.drain_warps >= 0 ? std::vector<int>{(int)o.drain_warps} : std::vector<int>{0, 1, 2};
   Config best;
   bool found = false;
   for (int S : Ss) {
@@ -237,9 +260,10 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
     for (int np : Ps)
     for (int D : Ds)
       for (int W : Ws)
+        for (int nd : Dr)
         for (int64_t t : tiles) {
           if (d.flush_each_tile && (long double)(t + QCAP) * std::max<long double>(li.maxabs, 1) >= 4.6e18L) continue;
-          Config c = predict(ctx, d, li, N, t, S, D, W, k, np);
+          Config c = predict(ctx, d, li, N, t, S, D, W, k, np, nd);
           if (!c.feasible) continue;
           {
             auto key = std::make_tuple(k, S, np);
@@ -278,7 +302,7 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
   auto pred = [&](double f) {
     li->cons_factor = f;
     return predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
-                   p.ctas_per_sm, p.npack).pred_ms;
+                   p.ctas_per_sm, p.npack, p.ndrain).pred_ms;
   };
   // the prediction is non-decreasing in the factor: geometric bisection
   double lo = 0.05, hi = 50;

@@ -13,16 +13,17 @@ struct Config {
   int64_t tile_rows = 0;
   int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1, grid = 0, smem = 0;
   int npack = 1;  // 128-row packets a consumer warp takes per iteration (1 or 2)
+  int ndrain = 0; // of the consumer warps, those that only drain hand-off packets (NEXT-1)
   double pred_ms = 0, t_stream_ms = 0, t_probe_ms = 0, t_tail_ms = 0, t_launch_ms = 0, bw_gbs = 0;
   bool feasible = false;
 };
 
 // Shared-memory bytes of a configuration (Eq 2 feasibility input).
-int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps);
+int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps, int ndrain = 0);
 
 // Predicted time (ms) of one configuration (Eqs 3-9 analog).
 Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t nrows, int64_t tile_rows,
-               int stage_rows, int depth, int warps, int ctas_per_sm, int npack = 1);
+               int stage_rows, int depth, int warps, int ctas_per_sm, int npack = 1, int ndrain = 0);
 
 // Search the feasible space (Δ, stage rows, depth, consumer warps), honouring
 // options and a requested tile_rows (> 0 fixes Δ). Returns false if nothing fits.

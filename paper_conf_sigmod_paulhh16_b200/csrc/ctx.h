@@ -93,7 +93,7 @@ struct RunProfile {
   uint64_t table_version = 0;  // the fact table's version when profiled (a reload re-profiles)
   int runs = 0;                // timed runs folded in (the profile is used from 2 on)
   int64_t nrows = 0, tile_rows = 0;
-  int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1, npack = 1;
+  int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1, npack = 1, ndrain = 0;
   double kernel_ms = 0;
 };
 
@@ -150,6 +150,7 @@ struct TunedShape {
   int stage_rows = 0, depth = 0, warps = 0, ctas_per_sm = 1;
   int split = -2;  // probes run in the stage phase (-2: the heuristic's)
   int npack = 1;
+  int ndrain = 0;
 };
 
 struct Options {
@@ -165,6 +166,7 @@ struct Options {
   int64_t use_profile = 1;     // the model fits its consumer cost to the plan's profiled run
   int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
   int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
+  int64_t drain_warps = -1;    // operator-specialised drain warps (NEXT-1): -1 = the model's choice
 };
 
 // Γ of one ring shape (gpl_calibrate, Eq 1): (bytes, GB/s)

@@ -107,6 +107,7 @@ std::string shape_source(const PipeDesc& d) {
   I("nwarps", d.nwarps);
   I("npack", d.npack);
   I("min_blocks", d.min_blocks);
+  I("ndrain", d.ndrain);
   I("flush_each_tile", d.flush_each_tile);
   I("nfilt", d.nfilt);
   I("nsprobe", d.nsprobe);

@@ -65,9 +65,19 @@ constexpr int kOffHdr = 128;      // int4[kMaxDepth]
 constexpr int kOffHtp = 256;      // HTP[MAXHT]
 constexpr int kOffHdr2 = 768;     // int4[kMaxDepth]: clustered-probe cell range (start lo, hi, bytes)
 constexpr int kOffCnt = 1024;     // unsigned long long[kMaxWarps][MAXOPS]
+// drain hand-off ring (ndrain > 0): a bounded multi-producer / multi-consumer
+// queue of R slots. Slot s carries a sequence number: ticket t may fill it
+// when seq == t and drain it when seq == t + 1 (then seq = t + R). Several
+// stage warps hold tickets at once, so an mbarrier's phase parity could not
+// tell ticket t from ticket t + 2R; the sequence numbers can.
+constexpr int kMaxHand = 8;
+constexpr int kOffHSeq = 3328;    // unsigned[kMaxHand]
+constexpr int kOffHHdr = 3456;    // int[kMaxHand]: entries in the packet (-1: end)
+constexpr int kOffHTick = 3488;   // unsigned[3]: producer ticket, consumer ticket, stage warps done
 static_assert(kOffHtp + MAXHT * sizeof(HTP) <= kOffHdr2, "HTP region overflow");
 static_assert(kOffHdr2 + kMaxDepth * 16 <= kOffCnt, "header region overflow");
-static_assert(kOffCnt + kMaxWarps * MAXOPS * 8 <= 4096, "fixed region overflow");
+static_assert(kOffCnt + kMaxWarps * MAXOPS * 8 <= kOffHSeq, "counter region overflow");
+static_assert(kOffHTick + 12 <= 4096, "fixed region overflow");
 
 template <class T>
 __device__ __forceinline__ T& S(uint32_t off) {
@@ -462,13 +472,17 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   unsigned long long* stab = &S<unsigned long long>(K.off_agg);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int W = K.nwarps;
+  const int W = K.nwarps;          // consumer warps (the producer is warp W)
+  const int Ws = W - K.ndrain;      // stage warps (the rest only drain hand-off packets)
+  const int R = 2 * K.ndrain;       // hand-off ring slots
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < K.depth; i++) {
       mbar_init(&full[i], 1);
-      mbar_init(&empty[i], (uint32_t)W);
+      mbar_init(&empty[i], (uint32_t)Ws);
     }
+    for (int i = 0; i < R; i++) S<unsigned>(kOffHSeq + 4 * i) = (unsigned)i;
+    S<unsigned>(kOffHTick) = S<unsigned>(kOffHTick + 4) = S<unsigned>(kOffHTick + 8) = 0u;
     fence_mbar_init();
   }
   // (PDL) everything above overlaps the previous kernel's tail; tables,
@@ -600,6 +614,61 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #else
 #define GPL_SP_HTP(sp) htp[K.probe[sp].ht]
 #endif
+  // drain hand-off ring (ndrain > 0): slot s's packet lives after the stage
+  // warps' queues, in the same field layout as a warp queue
+  const uint32_t hq0 = (uint32_t)K.off_queue + (uint32_t)Ws * (uint32_t)K.qbytes;
+  // stage warp: hand n queued survivors (from qhead) to the drain warps (n < 0: end token)
+  auto seq_wait = [&](int hs, unsigned want) {  // lane 0 spins, then the warp proceeds (acquire)
+    if (lane == 0) {
+      volatile unsigned* q = &S<unsigned>(kOffHSeq + 4 * hs);
+      while (*q != want) __nanosleep(32);
+      __threadfence_block();
+    }
+    __syncwarp();
+  };
+  auto seq_set = [&](int hs, unsigned v) {  // the warp's writes are visible before the slot moves on (release)
+    __syncwarp();
+    if (lane == 0) {
+      __threadfence_block();
+      *(volatile unsigned*)&S<unsigned>(kOffHSeq + 4 * hs) = v;
+    }
+  };
+  auto hand_off = [&](int head, int n) {
+    unsigned t = 0;
+    if (lane == 0) t = atomicAdd(&S<unsigned>(kOffHTick), 1u);
+    t = __shfl_sync(0xffffffffu, t, 0);
+    const int hs = (int)(t % (unsigned)R);
+    seq_wait(hs, t);
+    const uint32_t hb = hq0 + (uint32_t)hs * (uint32_t)K.qbytes;
+    GPL_UNROLL
+    for (int e = 0; e < K.npush; e++) {
+      const uint32_t src = qb + K.qoff[e], dst = hb + K.qoff[e];
+      for (int i = lane; i < n; i += 32) {
+        const int si = (head + i) & (QCAP - 1);
+        if (K.qw[e] == 4) S<int>(dst + i * 4) = S<int>(src + si * 4);
+        else S<long long>(dst + i * 8) = S<long long>(src + si * 8);
+      }
+    }
+    if (lane == 0) S<int>(kOffHHdr + 4 * hs) = n;
+    seq_set(hs, t + 1u);
+  };
+  if (K.ndrain > 0 && warp >= Ws) {
+    // ------------------------------------------------ drain warps (NEXT-1)
+    // the queue phase (remaining probes, residuals, aggregation / insert) of
+    // the packets the stage warps hand over, in ticket order
+    for (;;) {
+      unsigned t = 0;
+      if (lane == 0) t = atomicAdd(&S<unsigned>(kOffHTick + 4), 1u);
+      t = __shfl_sync(0xffffffffu, t, 0);
+      const int hs = (int)(t % (unsigned)R);
+      seq_wait(hs, t + 1u);
+      const int n = S<int>(kOffHHdr + 4 * hs);
+      if (n < 0) break;
+      drain(d, hq0 + (uint32_t)hs * (uint32_t)K.qbytes, 0, n, cnt, acc, lane);
+      if (K.flush_each_tile) flush_reg(d, acc, lane);
+      seq_set(hs, t + (unsigned)R);
+    }
+  } else {
   for (;;) {
     mbar_wait(&full[slot], phase);
     const int4 h = hdr[slot];
@@ -622,13 +691,13 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     // stage-phase probe latency is a warp's critical path); compaction and the
     // queue then proceed packet by packet.
     const int npk = K.npack < NPMAX ? K.npack : NPMAX;
-    for (int it0 = warp; it0 < nit; it0 += npk * W) {
+    for (int it0 = warp; it0 < nit; it0 += npk * Ws) {
       int r0q[NPMAX];
       bool live[NPMAX];
 #pragma unroll
       for (int q = 0; q < NPMAX; q++) {
-        r0q[q] = ((it0 + q * W) << 7) + (lane << 2);
-        live[q] = q < npk && it0 + q * W < nit;
+        r0q[q] = ((it0 + q * Ws) << 7) + (lane << 2);
+        live[q] = q < npk && it0 + q * Ws < nit;
       }
       bool p[NR];
 #pragma unroll
@@ -722,7 +791,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         // the ring slot is no longer read: release it before the atomics' round trip
 #pragma unroll
         for (int q = 0; q < NPMAX; q++)
-          if (live[q] && it0 + q * W + W >= nit) {
+          if (live[q] && it0 + q * Ws + Ws >= nit) {
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[slot]);
             released = true;
@@ -788,7 +857,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           }
           qcount = base;
         }
-        if (it0 + q * W + W >= nit) {
+        if (it0 + q * Ws + Ws >= nit) {
           // the warp's last packet of this stage is in the queue: release the
           // ring slot BEFORE draining (the drain reads only the queue), so the
           // producer's next copy overlaps the drain's probe/insert latency
@@ -798,7 +867,8 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         }
         if (qcount >= RPL * 32) {
           __syncwarp();
-          drain(d, qb, qhead, RPL * 32, cnt, acc, lane);
+          if (K.ndrain > 0) hand_off(qhead, RPL * 32);
+          else drain(d, qb, qhead, RPL * 32, cnt, acc, lane);
           __syncwarp();
           qhead = (qhead + RPL * 32) & (QCAP - 1);
           qcount -= RPL * 32;
@@ -814,8 +884,17 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   }
   if (qcount > 0) {
     __syncwarp();
-    drain(d, qb, qhead, qcount, cnt, acc, lane);
+    if (K.ndrain > 0) hand_off(qhead, qcount);
+    else drain(d, qb, qhead, qcount, cnt, acc, lane);
   }
+  if (K.ndrain > 0) {  // the last stage warp to finish sends one end token per drain warp
+    unsigned done = 0;
+    if (lane == 0) done = atomicAdd(&S<unsigned>(kOffHTick + 8), 1u);
+    done = __shfl_sync(0xffffffffu, done, 0);
+    if (done == (unsigned)(Ws - 1))
+      for (int e = 0; e < K.ndrain; e++) hand_off(0, -1);
+  }
+  }  // stage warps
   __syncwarp();
   if (K.agg_mode == AGG_REG) flush_reg(d, acc, lane);
   if (lane == 0) {

@@ -54,7 +54,8 @@ class _Stats(ctypes.Structure):
                 ("bytes_scanned", ctypes.c_double), ("agg_mode", ctypes.c_int32), ("kbe", ctypes.c_int32),
                 ("jit", ctypes.c_int32), ("reserved", ctypes.c_int32), ("intermediate_bytes", ctypes.c_double),
                 ("bytes_full_scan", ctypes.c_double), ("lazy_columns", ctypes.c_int32), ("packets", ctypes.c_int32),
-                ("groups_total", ctypes.c_int64), ("hash_slots", ctypes.c_int64)]
+                ("groups_total", ctypes.c_int64), ("hash_slots", ctypes.c_int64), ("drain_warps", ctypes.c_int32),
+                ("reserved2", ctypes.c_int32)]
 
 
 class _Result(ctypes.Structure):

@@ -547,3 +547,29 @@ def test_graph_branches_exact(ctx, q):
             r = queries.run_query(ctx, q, db)
             assert r.keys == o.keys and r.aggs == o.aggs, (q, br)
     ctx.set_option("graph_branches", 1)
+
+
+@pytest.mark.parametrize("q", QUERIES + ["Q3"])
+def test_drain_warps_exact(ctx, q):
+    """Operator-specialised consumer warps: with 1 or 2 of the consumer warps only
+    draining the survivor packets the stage warps hand over (shared-memory hand-off ring), every plan stays
+    bit-exact, under several schedules (tile sizes, packets, late materialisation, probe split)."""
+    db = tpchgen.generate(0.1, seed=23)
+    queries.load_database(ctx, db, queries.TABLES[q])
+    o = oracle.run(q, db, _params(q))
+    if q == "Q3":
+        o = oracle.order_limit("Q3", o)
+    try:
+        for nd, opts, tiles in ((1, {}, (0, 1024)), (2, {"consumer_warps": 6, "packets": 2}, (0,)),
+                                (1, {"lazy_columns": 0, "probe_split": 0, "consumer_warps": 2}, (0,))):
+            ctx.set_option("drain_warps", nd)
+            for k, v in opts.items():
+                ctx.set_option(k, v)
+            for tile in tiles:
+                r = queries.run_query(ctx, q, db, _params(q), tile_rows=tile)
+                assert r.keys == o.keys and r.aggs == o.aggs, (q, nd, opts, tile)
+                assert r.stats["drain_warps"] in (0, nd)  # a plan without a queue phase runs none
+            for k in opts:
+                ctx.set_option(k, -1)
+    finally:
+        ctx.set_option("drain_warps", -1)
