@@ -20,9 +20,15 @@ ctx = gpl.Context(0, stream=torch.cuda.current_stream())
 queries.load_database(ctx, ddb, borrow=True)
 text = queries.plan_text(q, db)
 flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size, dtype=torch.uint8, device=dev)
+for _ in range(3):  # λ and the model's profile first (unpinned)
+    ctx.run_query(text)
+    ctx.fetch_result()
 for name, v in (("stage_rows", S), ("ring_depth", D), ("consumer_warps", W), ("ctas_per_sm", k), ("packets", npk),
                 ("probe_split", 1)):
     ctx.set_option(name, v)
+for kv in filter(None, os.environ.get("GPL_OPTS", "").split(",")):  # e.g. lazy_columns=0,clustered=0
+    name, v = kv.split("=")
+    ctx.set_option(name, int(v))
 ts = []
 for i in range(8):
     flush.zero_()
