@@ -225,8 +225,32 @@ def main():
 
     part_dev = gathered = None
 
+    hash_plan = args.query in queries.EXTRA_QUERIES  # hash group-by (NEXT-4): rows, not dense partials
+    probe_seg = queries.segments(text)[-1]
+
+    def hash_merge(c):
+        # the group key holds l_orderkey, the shard key: the ranks' groups are
+        # disjoint, so their LIMIT rows hold the global top-k
+        local_res = c.fetch_result()  # this rank's run statistics (kernel time, counters)
+        rows = torch.from_numpy(c.fetch_groups()).to(cdev)
+        cnt = torch.tensor([rows.shape[0]], dtype=torch.int64, device=cdev)
+        cnts = torch.empty(world, dtype=torch.int64, device=cdev)
+        dist.all_gather_into_tensor(cnts, cnt)
+        mx = max(1, int(cnts.max()))
+        pad = torch.zeros((mx, rows.shape[1]), dtype=torch.int64, device=cdev)
+        pad[:rows.shape[0]] = rows
+        allr = torch.empty((world * mx, rows.shape[1]), dtype=torch.int64, device=cdev)
+        dist.all_gather_into_tensor(allr, pad)
+        allr = allr.cpu().numpy().reshape(world, mx, -1)
+        merged = c.merge_groups(probe_seg, np.concatenate([allr[r, :int(cnts[r])] for r in range(world)]))
+        stats = dict(local_res.stats)
+        stats["groups_total_merged_topk_rows"] = merged.stats["groups_total"]
+        return type(merged)(merged.keys, merged.aggs, stats)
+
     def step():
         ctx.run_query(text, args.tile_rows)  # builds + fused run; a CUDA graph replay once warm
+        if world > 1 and hash_plan:
+            return hash_merge(ctx)
         if world > 1:
             nonlocal part_dev, gathered
             nb = ctx.partials_nbytes()
@@ -303,6 +327,8 @@ def main():
             ctx2.run_query(text, args.tile_rows)
             if world == 1:
                 return ctx2.fetch_result()
+            if hash_plan:
+                return hash_merge(ctx2)
             host = ctx2.fetch_partials()  # D2H of this rank's int128 partials
             g = torch.empty(world * host.size, dtype=torch.int64, device=cdev)
             dist.all_gather_into_tensor(g, torch.from_numpy(host.view(np.int64)).to(cdev))
@@ -321,7 +347,8 @@ def main():
             e_ms.append(ev0.elapsed_time(ev1))
         assert r2.aggs == res0.aggs and r2.keys == res0.keys
         ncols = sum(len(c) for c in pinned.values())
-        d2h = ctx2.partials_nbytes() + 16 * 8 + 4 + 16 * ncols  # partials + counters + errors + column min/max
+        res_bytes = 16 + ctx2.fetch_groups().nbytes if hash_plan else ctx2.partials_nbytes()  # result rows / partials
+        d2h = res_bytes + 16 * 8 + 4 + 16 * ncols  # + counters + errors + column min/max
         e_ms_v = statistics.mean(e_ms)
         if world > 1:
             t = torch.tensor([e_ms_v], dtype=torch.float64, device=cdev)
@@ -384,7 +411,8 @@ def main():
                                                "probe_split", "predicted_ms", "agg_mode", "packets", "lazy_columns",
                                                "drain_warps")},
         "op_pass": stats["op_pass"],
-        "collective": (f"{backend} all_gather of int128 partials + fixed-order merge" if world > 1 else None),
+        "collective": ((f"{backend} all_gather of hash group-by rows + gpl_merge_groups" if hash_plan else
+                        f"{backend} all_gather of int128 partials + fixed-order merge") if world > 1 else None),
         "jit": stats.get("jit"),
         "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split",
                                               "builds_tuned", "build_ms_model", "build_ms")}

@@ -313,6 +313,23 @@ gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment);
  * (insert-sink) kernel; other builds use precompiled kernels (no-op). */
 gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows);
 
+/* Hash group-by across ranks (SURVEY §8(f) NEXT-4 with §8(e)): the rows of the
+ * last run of a 'group hash' plan — [packed key, acc 0 .. nagg-1] int64 words
+ * per row (key = k0 << 32 | k1 for two keys; *row_words = 1 + nagg) — into
+ * caller-owned host memory (cap_rows rows):
+ * the LIMIT rows in ORDER BY order, else every group. *n_rows is set even when
+ * cap_rows is too small (GPL_E_CAPACITY). Synchronises. */
+gpl_status gpl_fetch_groups(gpl_ctx* ctx, int64_t* rows, int64_t cap_rows, int64_t* n_rows, int32_t* row_words);
+
+/* Merge the rows of several ranks (concatenated gpl_fetch_groups outputs,
+ * e.g. all-gathered over NCCL): exact int128 sums per key, then the probe
+ * segment's ORDER BY / LIMIT (else key order), into `out` as gpl_fetch_result
+ * fills it (stats.groups_total = distinct merged groups). A LIMIT plan is exact
+ * when every rank ships all its groups, or when the group key contains the
+ * shard key (TPC-H Q3: l_orderkey; disjoint groups). Host only. */
+gpl_status gpl_merge_groups(gpl_ctx* ctx, const char* probe_segment, const int64_t* rows, int64_t n_rows,
+                            gpl_result* out);
+
 /* Message of the last failed call on ctx (ctx-owned, valid until the next
  * call). gpl_last_error(NULL) reports gpl_create failures. */
 const char* gpl_last_error(const gpl_ctx* ctx);

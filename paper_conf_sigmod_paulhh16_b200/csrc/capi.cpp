@@ -10,6 +10,7 @@
 #include <climits>
 #include <cstring>
 #include <new>
+#include <map>
 #include <set>
 #include <string>
 
@@ -1680,6 +1681,97 @@ GPL_API gpl_status gpl_merge_partials(const void* gathered, int32_t nranks, size
     }
     o[2 * i] = (unsigned long long)acc;
     o[2 * i + 1] = (unsigned long long)(acc >> 64);
+  }
+  return GPL_OK;
+}
+
+// Hash group-by rows of the last run (NEXT-4 multi-GPU): [packed key, acc 0 .. nagg-1] int64 words per row —
+// the LIMIT rows in ORDER BY order, else every group (device compaction order).
+GPL_API gpl_status gpl_fetch_groups(gpl_ctx* ctx, int64_t* rows, int64_t cap_rows, int64_t* n_rows,
+                                    int32_t* row_words) {
+  if (!ctx || !n_rows || cap_rows < 0 || (cap_rows > 0 && !rows)) return GPL_E_ARG;
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  if (!ctx->last.valid || !ctx->last.run || !ctx->last.run->li.hash_group)
+    return fail(ctx, GPL_E_STATE, "gpl_fetch_groups: the last run is not a hash group-by");
+  CK(cudaStreamSynchronize(ctx->stream));
+  if ((st = take_device_errors(ctx))) return st;
+  const LowerInfo& li = ctx->last.run->li;
+  const int W = 1 + li.nagg;
+  const unsigned long long* part = (const unsigned long long*)ctx->h_stage + kScratchHead;
+  const int64_t n = (int64_t)part[1];
+  *n_rows = n;
+  if (row_words) *row_words = W;
+  if (n > cap_rows) return fail(ctx, GPL_E_CAPACITY, "gpl_fetch_groups: rows capacity too small");
+  if (n == 0) return GPL_OK;
+  if (li.limit > 0) {
+    std::memcpy(rows, part + 2, (size_t)n * W * 8);
+  } else {
+    CK(cudaMemcpyAsync(rows, ctx->last.run->hres.rows, (size_t)n * W * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+  }
+  return GPL_OK;
+}
+
+// Merge hash group-by rows of several ranks (concatenated gpl_fetch_groups
+// outputs) exactly — int128 sums per key, in input order — then apply the
+// probe segment's ORDER BY / LIMIT (else key order) into `out`, as
+// gpl_fetch_result would. For a LIMIT plan every rank must ship ALL its
+// groups (run the plan without 'order'/'limit') unless the shard key is part
+// of the group key (disjoint groups: the union of the ranks' top-k rows holds
+// the global top-k).
+GPL_API gpl_status gpl_merge_groups(gpl_ctx* ctx, const char* probe_segment, const int64_t* rows, int64_t n_rows,
+                                    gpl_result* out) {
+  if (!ctx || !probe_segment || !out || n_rows < 0 || (n_rows > 0 && !rows)) return GPL_E_ARG;
+  ctx->err.clear();
+  Segment s;
+  std::string err;
+  if (!parse_segment(probe_segment, &s, &err)) return fail(ctx, GPL_E_PLAN, err);
+  if (!s.hash_group) return fail(ctx, GPL_E_PLAN, "gpl_merge_groups: the segment has no 'group hash'");
+  const int NK = (int)s.groups.size(), A = (int)s.aggs.size(), W = 1 + A;
+  auto field = [&](unsigned long long key, int k) {
+    return NK == 2 ? (int32_t)(uint32_t)(k == 0 ? key >> 32 : key) : (int32_t)(uint32_t)key;
+  };
+  std::map<unsigned long long, std::vector<__int128>> acc;
+  for (int64_t r = 0; r < n_rows; r++) {
+    const unsigned long long key = (unsigned long long)rows[r * W];
+    auto it = acc.find(key);
+    if (it == acc.end()) it = acc.emplace(key, std::vector<__int128>(A, 0)).first;
+    for (int a = 0; a < A; a++) it->second[a] += (__int128)rows[r * W + 1 + a];
+  }
+  std::vector<std::pair<unsigned long long, const std::vector<__int128>*>> v;
+  v.reserve(acc.size());
+  for (auto& kv : acc) v.push_back({kv.first, &kv.second});
+  auto key_less = [&](unsigned long long a, unsigned long long b) {
+    for (int k = 0; k < NK; k++)
+      if (field(a, k) != field(b, k)) return field(a, k) < field(b, k);
+    return false;
+  };
+  std::sort(v.begin(), v.end(), [&](const auto& x, const auto& y) {
+    for (const OrderIR& o : s.order) {
+      __int128 a = o.is_agg ? (*x.second)[o.idx] : (__int128)field(x.first, o.idx);
+      __int128 b = o.is_agg ? (*y.second)[o.idx] : (__int128)field(y.first, o.idx);
+      if (a != b) return o.desc ? a > b : a < b;
+    }
+    return key_less(x.first, y.first);
+  });
+  const int64_t n = s.limit > 0 ? std::min<int64_t>((int64_t)v.size(), s.limit) : (int64_t)v.size();
+  out->n_keys = NK;
+  out->n_aggs = A;
+  out->n_groups = (int32_t)std::min<int64_t>(n, INT32_MAX);
+  out->stats = gpl_stats{};
+  out->stats.groups_total = (int64_t)v.size();
+  out->stats.agg_mode = AGG_HASH;
+  if (n > out->cap_groups) return fail(ctx, GPL_E_CAPACITY, "result capacity too small");
+  if (n && (!out->keys || !out->aggs)) return fail(ctx, GPL_E_ARG, "NULL result arrays");
+  for (int64_t r = 0; r < n; r++) {
+    for (int k = 0; k < NK; k++) out->keys[r * NK + k] = field(v[r].first, k);
+    for (int a = 0; a < A; a++) {
+      const unsigned __int128 u = (unsigned __int128)(*v[r].second)[a];
+      out->aggs[(r * A + a) * 2] = (int64_t)(uint64_t)u;
+      out->aggs[(r * A + a) * 2 + 1] = (int64_t)(uint64_t)(u >> 64);
+    }
   }
   return GPL_OK;
 }

@@ -29,7 +29,7 @@ EXPORTED = ["gpl_create", "gpl_destroy", "gpl_load_columns", "gpl_build_hash", "
             "gpl_run_plan_kbe", "gpl_fetch_result", "gpl_fetch_partials", "gpl_decode_partials",
             "gpl_merge_partials", "gpl_sync", "gpl_choose_tile_rows", "gpl_set_option",
             "gpl_check_plan", "gpl_compile_plan", "gpl_run_query", "gpl_autotune", "gpl_calibrate",
-            "gpl_set_calibration", "gpl_last_error", "gpl_version"]
+            "gpl_set_calibration", "gpl_fetch_groups", "gpl_merge_groups", "gpl_last_error", "gpl_version"]
 
 
 class GplError(RuntimeError):
@@ -113,6 +113,8 @@ def load_library():
         "gpl_autotune": ([P, ctypes.c_char_p, I32, ctypes.POINTER(_Model)], I32),
         "gpl_calibrate": ([P, ctypes.POINTER(I64), I32, ctypes.POINTER(_Gamma), I32, ctypes.POINTER(I32)], I32),
         "gpl_set_calibration": ([P, ctypes.POINTER(_Gamma), I32], I32),
+        "gpl_fetch_groups": ([P, ctypes.POINTER(I64), I64, ctypes.POINTER(I64), ctypes.POINTER(I32)], I32),
+        "gpl_merge_groups": ([P, ctypes.c_char_p, ctypes.POINTER(I64), I64, ctypes.POINTER(_Result)], I32),
         "gpl_last_error": ([P], ctypes.c_char_p),
         "gpl_version": ([], ctypes.c_char_p),
     }
@@ -309,6 +311,25 @@ class Context:
         out_k = [tuple(kl[i * nk:(i + 1) * nk]) for i in range(ng)]
         out_a = [[_i128(al[(i * na + j) * 2], al[(i * na + j) * 2 + 1]) for j in range(na)] for i in range(ng)]
         return Result(out_k, out_a, _stats_dict(r.stats))
+
+    def fetch_groups(self) -> np.ndarray:
+        """Rows of the last hash group-by run: int64 [n, 1 + nagg] (packed key, accumulators)."""
+        n, w = ctypes.c_int64(0), ctypes.c_int32(0)
+        st = self._lib.gpl_fetch_groups(self._h, None, 0, ctypes.byref(n), ctypes.byref(w))  # size query
+        if st not in (0, GPL_E_CAPACITY):
+            self._check(st)
+        buf = np.zeros((n.value, max(1, w.value)), dtype=np.int64)
+        if n.value:
+            self._check(self._lib.gpl_fetch_groups(self._h, buf.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                                   n.value, ctypes.byref(n), ctypes.byref(w)))
+        return buf
+
+    def merge_groups(self, segment: str, rows: np.ndarray) -> Result:
+        """Exact merge of several ranks' hash group-by rows (int64 [n, 1 + nagg]) with the segment's ORDER BY/LIMIT."""
+        rows = np.ascontiguousarray(rows, dtype=np.int64)
+        nrows = rows.shape[0] if rows.ndim == 2 else 0
+        return self._result(lambda rp: self._lib.gpl_merge_groups(
+            self._h, segment.encode(), rows.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)), nrows, rp))
 
     def fetch_result(self) -> Result:
         return self._result(lambda rp: self._lib.gpl_fetch_result(self._h, rp))

@@ -573,3 +573,36 @@ def test_drain_warps_exact(ctx, q):
                 ctx.set_option(k, -1)
     finally:
         ctx.set_option("drain_warps", -1)
+
+
+def test_hash_groupby_shards_merge_exact(ctx):
+    """§8(e) layout for the hash group-by: Q3 on two order-key shards on the device, gpl_fetch_groups per
+    shard, gpl_merge_groups on the host = the oracle on the whole database (top-10 from the shards' top-10s;
+    every group from the no-LIMIT plan)."""
+    import numpy as np
+    sf, seed = 0.1, 31
+    whole = oracle.run("Q3", tpchgen.generate(sf, seed=seed))
+    top, full = [], []
+    seg = None
+    for rank in range(2):
+        shard = tpchgen.generate(sf, seed=seed, rank=rank, world=2)
+        queries.load_database(ctx, shard, queries.TABLES["Q3"])
+        text = queries.plan_text("Q3", shard)
+        seg = queries.segments(text)[-1]
+        queries.run_query(ctx, "Q3", shard)
+        top.append(ctx.fetch_groups())
+        full_text = "\n".join(ln for ln in text.splitlines() if not ln.startswith(("order", "limit")))
+        for _ in range(2):  # a table sized from the other shard may overflow once
+            ctx.run_query(full_text)
+            try:
+                ctx.fetch_result()
+                break
+            except gpl.GplError as e:
+                assert e.status == gpl.GPL_E_CAPACITY
+        full.append(ctx.fetch_groups())
+    r = ctx.merge_groups(seg, np.concatenate(top))
+    want = oracle.order_limit("Q3", whole)
+    assert r.keys == want.keys and r.aggs == want.aggs
+    full_seg = "\n".join(ln for ln in seg.splitlines() if not ln.startswith(("order", "limit")))
+    r = ctx.merge_groups(full_seg, np.concatenate(full))
+    assert r.keys == whole.keys and r.aggs == whole.aggs

@@ -88,3 +88,82 @@ def test_sharded_merge_world2(q):
         p.join(timeout=300)
     assert all(p.exitcode == 0 for p in procs)
     assert ret.get(0) and ret.get(1)
+
+
+def _q3_rows(res):
+    """oracle Q3 result -> hash group-by rows as the device emits them: [(l_orderkey << 32) | o_orderdate, count, sum]."""
+    import numpy as np
+    rows = np.zeros((len(res.keys), 3), dtype=np.int64)
+    for i, (k, a) in enumerate(zip(res.keys, res.aggs)):
+        rows[i] = [(int(k[0]) << 32) | (int(k[1]) & 0xFFFFFFFF), a[0], a[1]]
+    return rows
+
+
+def _worker_hash(rank, world, port, ret):
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    import numpy as np
+
+    import oracle
+    import tpchgen
+    from paper_conf_sigmod_paulhh16_b200 import gpl, queries
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        sf, seed = 0.05, 29
+        whole_db = tpchgen.generate(sf, seed=seed)
+        whole = oracle.run("Q3", whole_db)
+        seg = queries.segments(queries.plan_text("Q3", whole_db))[-1]
+        full_seg = "\n".join(ln for ln in seg.splitlines() if not ln.startswith(("order", "limit")))
+        ctx = gpl.Context(device=-1)
+        ok = True
+        # (1) order-key shards (§8(e) layout): groups are disjoint; each rank ships its top-10 rows only
+        shard = tpchgen.generate(sf, seed=seed, rank=rank, world=world)
+        local_top = _q3_rows(oracle.order_limit("Q3", oracle.run("Q3", shard)))
+        parts = [None] * world
+        dist.all_gather_object(parts, local_top)
+        r = ctx.merge_groups(seg, np.concatenate(parts))
+        want = oracle.order_limit("Q3", whole)
+        ok &= r.keys == want.keys and r.aggs == want.aggs
+        # (2) lineitem split NOT on order boundaries: groups overlap across ranks, every group shipped
+        n = whole_db.nrows("lineitem")
+        # cut inside a qualifying order with >= 2 qualifying lineitems, so that group has rows on both ranks
+        k = next(k for k, a in zip(whole.keys, whole.aggs) if a[0] >= 2)[0]
+        first = int(np.nonzero(whole_db.tables["lineitem"]["l_orderkey"] == k)[0][0])
+        mid = first + 1
+        while not (whole_db.tables["lineitem"]["l_shipdate"][first:mid] > 19950315).any():
+            mid += 1
+        cut = [0, mid, n][rank:rank + 2]
+        local_all = _q3_rows(oracle.run("Q3", whole_db, None, tuple(cut)))
+        parts = [None] * world
+        dist.all_gather_object(parts, local_all)
+        rows = np.concatenate(parts)
+        overlap = len({int(x) for x in parts[0][:, 0]} & {int(x) for x in parts[1][:, 0]}) if world == 2 else 0
+        r = ctx.merge_groups(seg, rows)
+        ok &= r.keys == want.keys and r.aggs == want.aggs and overlap > 0
+        r = ctx.merge_groups(full_seg, rows)
+        ok &= r.keys == whole.keys and r.aggs == whole.aggs and r.stats["groups_total"] == len(whole.keys)
+        ret[rank] = bool(ok)
+    finally:
+        dist.destroy_process_group()
+
+
+def test_hash_groupby_merge_world2():
+    """NEXT-4 across ranks (§8(e)): hash group-by rows all-gathered over gloo and merged exactly by
+    gpl_merge_groups (int128 sums per key, then ORDER BY/LIMIT) equal the oracle on the whole database —
+    for order-key shards (disjoint groups: the ranks' top-10s suffice) and for an arbitrary lineitem split
+    (overlapping groups: all groups shipped)."""
+    ctx = mp.get_context("spawn")
+    mgr = ctx.Manager()
+    ret = mgr.dict()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_hash, args=(r, 2, port, ret)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=300)
+    assert all(p.exitcode == 0 for p in procs)
+    assert ret.get(0) and ret.get(1)
