@@ -1147,7 +1147,8 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
 // The model's per-shape candidates plus, for the `top` best predicted, the
 // other consumer-warp counts that fit (the model's W is the least certain
 // knob: the work-group sweep of P:366 / Figs 14-15 is measured, not only
-// modelled; every extra shape costs one plan-specialised compile).
+// modelled; every extra shape costs one plan-specialised compile), tile
+// sizes of 1, 2 and 4 stages (same kernel) and drain-warp splits.
 static void with_warp_variants(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64_t N,
                                std::vector<Config>* cs, size_t top = 3) {
   if (ctx->opt.consumer_warps > 0) return;
@@ -1159,6 +1160,14 @@ static void with_warp_variants(const gpl_ctx* ctx, const PipeDesc& d, const Lowe
     for (int W : {4, 8, 12, 16}) {
       if (W == c.warps) continue;
       Config v = predict(ctx, d, li, std::max<int64_t>(N, 1), c.tile_rows, c.stage_rows, c.depth, W, c.ctas_per_sm, c.npack,
+                         c.ndrain);
+      if (v.feasible) out.push_back(v);
+    }
+    // scheduling granularity (Eq 3's waves / last-wave tail): the same shape at Δ = 1, 2, 4 stages
+    for (int m : {1, 2, 4}) {
+      const int64_t t = (int64_t)c.stage_rows * m;
+      if (t == c.tile_rows) continue;
+      Config v = predict(ctx, d, li, std::max<int64_t>(N, 1), t, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, c.npack,
                          c.ndrain);
       if (v.feasible) out.push_back(v);
     }
