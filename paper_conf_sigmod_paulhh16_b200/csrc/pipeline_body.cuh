@@ -84,21 +84,80 @@ __device__ __forceinline__ T& S(uint32_t off) {
   return *reinterpret_cast<T*>(g_smem + off);
 }
 
+// shared-space scalar loads at a shared-window address (see smem_base)
+__device__ __forceinline__ uint32_t lds_u32(uint32_t sa) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(sa));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds_u16(uint32_t sa) {
+  unsigned short v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(sa));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(uint32_t sa) {
+  uint32_t v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(sa));
+  return v;
+}
+
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
   return m;
 }
 
+// Shared-space loads at g_smem + a: the shared-window address of g_smem is
+// computed once per thread (smem_base) instead of being rematerialised from
+// SR_CgaCtaId for every load of the hot loop (ncu: that S2R + LEA chain was
+// the top stall of the stage phase). Volatile: never hoisted above the ring's
+// mbarrier waits (which are volatile asm too).
+__device__ __forceinline__ uint32_t smem_base() {
+  return (uint32_t)__cvta_generic_to_shared(g_smem);
+}
+__device__ __forceinline__ int4 lds_v4(uint32_t sa) {
+  int4 v;
+  asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(sa));
+  return v;
+}
+__device__ __forceinline__ longlong2 lds_v2_64(uint32_t sa) {
+  longlong2 v;
+  asm volatile("ld.shared.v2.s64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "r"(sa));
+  return v;
+}
+
 // RPL consecutive rows (r0 % 4 == 0) of one staged column, widened to int64.
 __device__ __forceinline__ void ld_rows(uint32_t a, int w, long long (&x)[RPL]) {
+  const uint32_t sa = smem_base() + a;
   if (w == 4) {
-    const int4 v = S<int4>(a);
+    const int4 v = lds_v4(sa);
     x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
   } else {
-    const longlong2 u = S<longlong2>(a);
-    const longlong2 v = S<longlong2>(a + 16);
+    const longlong2 u = lds_v2_64(sa);
+    const longlong2 v = lds_v2_64(sa + 16);
     x[0] = u.x; x[1] = u.y; x[2] = v.x; x[3] = v.y;
+  }
+}
+
+// A 4-byte filter column evaluated in 32-bit arithmetic (dates, keys, codes):
+// range as one unsigned compare of x - lo against hi - lo, bounds clamped to
+// the int32 range (an empty clamp passes nothing).
+__device__ __forceinline__ void filt_rows32(const Filt& F, uint32_t a, bool* p) {
+  const int4 v = lds_v4(smem_base() + a);
+  const int x[RPL] = {v.x, v.y, v.z, v.w};
+  if (F.kind == F_RANGE) {
+    const long long lo = F.lo < -2147483648LL ? -2147483648LL : F.lo;
+    const long long hi = F.hi > 2147483647LL ? 2147483647LL : F.hi;
+    const bool none = lo > hi;
+    const unsigned lo32 = (unsigned)(int)(none ? 0 : lo), span = (unsigned)((none ? 0 : hi) - (none ? 0 : lo));
+#pragma unroll
+    for (int j = 0; j < RPL; j++) p[j] = p[j] && !none && ((unsigned)x[j] - lo32) <= span;
+  } else if (F.kind == F_MASK) {
+#pragma unroll
+    for (int j = 0; j < RPL; j++) p[j] = p[j] && (unsigned)x[j] < 64u && ((F.mask >> x[j]) & 1ull);
+  } else {
+#pragma unroll
+    for (int j = 0; j < RPL; j++) p[j] = p[j] && (long long)x[j] != F.lo;
   }
 }
 
@@ -167,6 +226,7 @@ __device__ __forceinline__ void probe_rows_cl(const PipeDesc& K, const HTP& h, i
                                               const bool (&act)[N], bool (&hit)[N], long long (&pay)[N], uint32_t base,
                                               long long start, int size) {
   const int width = K.ht[t].width;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(g_smem) + base;
 #pragma unroll
   for (int j = 0; j < N; j++) {
     const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
@@ -176,14 +236,14 @@ __device__ __forceinline__ void probe_rows_cl(const PipeDesc& K, const HTP& h, i
     uint32_t x = 0;
     if (in) {
       if (width == 0) {
-        const uint32_t wd = staged ? S<uint32_t>(base + (uint32_t)b) : __ldg((const uint32_t*)h.slots + (idx >> 5));
+        const uint32_t wd = staged ? lds_u32(sbase + (uint32_t)b) : __ldg((const uint32_t*)h.slots + (idx >> 5));
         x = (wd >> (idx & 31)) & 1u;
       } else if (width == 1) {
-        x = staged ? (uint32_t)S<unsigned char>(base + (uint32_t)b) : (uint32_t)__ldg((const unsigned char*)h.slots + idx);
+        x = staged ? lds_u8(sbase + (uint32_t)b) : (uint32_t)__ldg((const unsigned char*)h.slots + idx);
       } else if (width == 2) {
-        x = staged ? (uint32_t)S<unsigned short>(base + (uint32_t)b) : (uint32_t)__ldg((const unsigned short*)h.slots + idx);
+        x = staged ? lds_u16(sbase + (uint32_t)b) : (uint32_t)__ldg((const unsigned short*)h.slots + idx);
       } else {
-        x = staged ? S<uint32_t>(base + (uint32_t)b) : __ldg((const uint32_t*)h.slots + idx);
+        x = staged ? lds_u32(sbase + (uint32_t)b) : __ldg((const uint32_t*)h.slots + idx);
       }
     }
     hit[j] = x != 0;
@@ -717,10 +777,14 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
         for (int q = 0; q < NPMAX; q++) {
           if (!live[q]) continue;  // (a packet past the stage must not be read: smem bounds)
-          long long x[RPL];
-          ld_rows(sb + K.coloff[F.ref] + r0q[q] * K.colw[F.ref], K.colw[F.ref], x);
+          if (K.colw[F.ref] == 4) {
+            filt_rows32(F, sb + K.coloff[F.ref] + r0q[q] * 4, p + q * RPL);
+          } else {
+            long long x[RPL];
+            ld_rows(sb + K.coloff[F.ref] + r0q[q] * K.colw[F.ref], K.colw[F.ref], x);
 #pragma unroll
-          for (int j = 0; j < RPL; j++) p[q * RPL + j] = p[q * RPL + j] && filt_pass(F, x[j]);
+            for (int j = 0; j < RPL; j++) p[q * RPL + j] = p[q * RPL + j] && filt_pass(F, x[j]);
+          }
         }
         const unsigned c = __reduce_add_sync(0xffffffffu, count_n(p));
         if (lane == 0) cnt[f] += c;
