@@ -101,6 +101,23 @@ __device__ __forceinline__ uint32_t lds_u8(uint32_t sa) {
   return v;
 }
 
+__device__ __forceinline__ long long lds_s64(uint32_t sa) {
+  long long v;
+  asm volatile("ld.shared.s64 %0, [%1];" : "=l"(v) : "r"(sa));
+  return v;
+}
+__device__ __forceinline__ int lds_s32(uint32_t sa) {
+  int v;
+  asm volatile("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(sa));
+  return v;
+}
+__device__ __forceinline__ void sts_32(uint32_t sa, int v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(sa), "r"(v));
+}
+__device__ __forceinline__ void sts_64(uint32_t sa, long long v) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(sa), "l"(v));
+}
+
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -173,14 +190,15 @@ __device__ __forceinline__ void ld_col(const PipeDesc& d, const PipeDesc& K, int
   }
 }
 
+// survivor-queue field access (shared-space loads/stores, see smem_base)
 __device__ __forceinline__ long long qget(const PipeDesc& K, uint32_t qb, int f, int i) {
-  const uint32_t a = qb + K.qoff[f];
-  return K.qw[f] == 4 ? (long long)S<int>(a + i * 4) : S<long long>(a + i * 8);
+  const uint32_t a = smem_base() + qb + K.qoff[f];
+  return K.qw[f] == 4 ? (long long)lds_s32(a + i * 4) : lds_s64(a + i * 8);
 }
 __device__ __forceinline__ void qput(const PipeDesc& K, uint32_t qb, int f, int i, long long v) {
-  const uint32_t a = qb + K.qoff[f];
-  if (K.qw[f] == 4) S<int>(a + i * 4) = (int)v;
-  else S<long long>(a + i * 8) = v;
+  const uint32_t a = smem_base() + qb + K.qoff[f];
+  if (K.qw[f] == 4) sts_32(a + i * 4, (int)v);
+  else sts_64(a + i * 8, v);
 }
 
 // Probe RPL rows of one lane in table t: small DIRECT tables were staged in
@@ -918,11 +936,11 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             if (K.qw[e] == 4) {
 #pragma unroll
               for (int j = 0; j < RPL; j++)
-                if (p[q * RPL + j]) S<int>(qa + pos[j] * 4) = (int)v[j];
+                if (p[q * RPL + j]) sts_32(smem_base() + qa + pos[j] * 4, (int)v[j]);
             } else {
 #pragma unroll
               for (int j = 0; j < RPL; j++)
-                if (p[q * RPL + j]) S<long long>(qa + pos[j] * 8) = v[j];
+                if (p[q * RPL + j]) sts_64(smem_base() + qa + pos[j] * 8, v[j]);
             }
           }
           qcount = base;
