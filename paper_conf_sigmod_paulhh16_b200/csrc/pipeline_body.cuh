@@ -212,6 +212,7 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int 
     // branch-free: the cell index is clamped into the table and the loaded
     // value masked, so the 4 shared-memory loads issue back to back
     const uint32_t last = (uint32_t)(h.nslots - 1);
+    const uint32_t sso = smem_base() + (uint32_t)so;
     uint32_t v[N];
 #pragma unroll
     for (int j = 0; j < N; j++) {
@@ -219,10 +220,10 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int 
       const bool in = act[j] && idx < h.nslots;
       const uint32_t i = in ? (uint32_t)idx : last;
       uint32_t x;
-      if (width == 0) x = (S<uint32_t>(so + (i >> 5) * 4) >> (i & 31)) & 1u;
-      else if (width == 1) x = (uint32_t)S<unsigned char>(so + i);
-      else if (width == 2) x = (uint32_t)S<unsigned short>(so + i * 2);
-      else x = S<uint32_t>(so + i * 4);
+      if (width == 0) x = (lds_u32(sso + (i >> 5) * 4) >> (i & 31)) & 1u;
+      else if (width == 1) x = lds_u8(sso + i);
+      else if (width == 2) x = lds_u16(sso + i * 2);
+      else x = lds_u32(sso + i * 4);
       v[j] = in ? x : 0u;
     }
 #pragma unroll
