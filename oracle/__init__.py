@@ -90,6 +90,9 @@ def _load():
         lib.oracle_run.argtypes = [ctypes.c_int, ctypes.POINTER(_OracleDB), ctypes.c_void_p,
                                    ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(_OracleResult)]
         lib.oracle_run.restype = ctypes.c_int
+        lib.oracle_run_mt.argtypes = [ctypes.c_int, ctypes.POINTER(_OracleDB), ctypes.c_void_p,
+                                      ctypes.c_int64, ctypes.c_int64, ctypes.c_int, ctypes.POINTER(_OracleResult)]
+        lib.oracle_run_mt.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -156,8 +159,29 @@ def _db_struct(db):
     return s, keep
 
 
-def run(query: str, db, params=None, lineitem_range=None) -> Result:
-    """Evaluate `query` ("L1", "Q5", "Q7", "Q8", "Q9", "Q14") on `db` (tpchgen.Database)."""
+def host_threads() -> int:
+    """Threads the multi-threaded oracle uses on this host: the CPUs this process may run on."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        return os.cpu_count() or 1
+
+
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def run(query: str, db, params=None, lineitem_range=None, threads: int = 1) -> Result:
+    """Evaluate `query` ("L1", "Q5", "Q7", "Q8", "Q9", "Q14", "Q3") on `db` (tpchgen.Database).
+    threads > 1: the LINEITEM rows are split into `threads` contiguous ranges whose
+    group maps are merged exactly (oracle.cpp header); the result is identical."""
     lib = _load()
     params = tuple(params) if params is not None else DEFAULT_PARAMS[query]
     pr = np.array(list(params) + [0] * (4 - len(params)), dtype=np.int32)
@@ -169,7 +193,8 @@ def run(query: str, db, params=None, lineitem_range=None) -> Result:
     r = _OracleResult()
     r.cap_rows = cap
     r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data
-    rc = lib.oracle_run(QUERY_IDS[query], ctypes.byref(s), pr.ctypes.data, lb, le, ctypes.byref(r))
+    rc = lib.oracle_run_mt(QUERY_IDS[query], ctypes.byref(s), pr.ctypes.data, lb, le, int(threads),
+                           ctypes.byref(r))
     if rc != 0:
         raise RuntimeError("oracle: " + r.err.decode())
     nk, na = r.n_keys, r.n_aggs
@@ -195,8 +220,68 @@ def order_limit(query: str, r: Result) -> Result:
     return Result(query, [k for k, _ in rows], [a for _, a in rows])
 
 
-def timed_run(query: str, db, params=None, lineitem_range=None):
-    """(Result, seconds) — wall time of one oracle evaluation (single thread)."""
+# A10 finalize of each Listing: its ORDER BY clause and its derived ratio
+# column, applied to the exact group rows (Appendix B Listings):
+#   Q5  "order by revenue desc"                             P:609  (Listing 2)
+#   Q7  "order by l_year"                                   P:629  (Listing 3)
+#   Q8  "order by o_year"; mkt_share = sum(case nation = 'BRAZIL' then volume
+#        else 0 end) / sum(volume)                          P:634-635, P:655 (Listing 4)
+#   Q9  "order by o_year desc"                              P:680  (Listing 5)
+#   Q14 promo_revenue = 100.00 * sum(case ...) / sum(...)   P:682-685 (Listing 6)
+#   Q3  revenue desc, o_orderdate, LIMIT 10                 [EXT] TPC-H Q3
+# Rows the ORDER BY leaves tied are ordered by the group key tuple ascending
+# (output codes), so the order is unique (reading R8). A ratio is
+# the IEEE double sequence C * double(num) / double(den) (reading R12); a zero
+# denominator is SQL NULL (None).
+# ORDER: list of (is_agg, index, desc); RATIO: (C, num agg, den agg).
+FINALIZE = {
+    "L1": ([], None, 0),
+    "Q5": ([(True, 1, True)], None, 0),
+    "Q7": ([(False, 2, False)], None, 0),
+    "Q8": ([(False, 0, False)], (1.0, 1, 2), 0),
+    "Q9": ([(False, 1, True)], None, 0),
+    "Q14": ([], (100.0, 1, 2), 0),
+    "Q3": ([(True, 1, True), (False, 1, False)], None, 10),
+}
+
+
+@dataclass
+class Final:
+    """A query's output rows in ORDER BY order, with the ratio column (or None)."""
+    query: str
+    keys: list
+    aggs: list
+    ratios: list
+
+
+def ratio(c: float, num: int, den: int):
+    """C * num / den as the double sequence fl(fl(C * fl(num)) / fl(den)); None when den == 0."""
+    if den == 0:
+        return None
+    return c * float(num) / float(den)
+
+
+def finalize(query: str, r: Result) -> Final:
+    """The Listing's ORDER BY (ties: group key ascending), LIMIT and ratio column on r's exact rows."""
+    order, rat, limit = FINALIZE[query]
+
+    def sort_key(ka):
+        k, a = ka
+        parts = []
+        for is_agg, idx, desc in order:
+            v = a[idx] if is_agg else k[idx]
+            parts.append(-v if desc else v)
+        return tuple(parts) + tuple(k)
+
+    rows = sorted(zip(r.keys, r.aggs), key=sort_key)
+    if limit:
+        rows = rows[:limit]
+    ratios = [ratio(rat[0], a[rat[1]], a[rat[2]]) if rat else None for _, a in rows]
+    return Final(query, [k for k, _ in rows], [a for _, a in rows], ratios)
+
+
+def timed_run(query: str, db, params=None, lineitem_range=None, threads: int = 1):
+    """(Result, seconds) — wall time of one oracle evaluation on `threads` threads."""
     t0 = time.perf_counter()
-    r = run(query, db, params, lineitem_range)
+    r = run(query, db, params, lineitem_range, threads)
     return r, time.perf_counter() - t0
