@@ -106,14 +106,21 @@ typedef struct {
 typedef struct {
   int32_t cap_groups;          /* in: rows the arrays can hold                                    */
   int32_t n_groups;            /* out: non-empty groups (1 row when the plan has no GROUP BY);   */
-                               /* hash group-by with 'order'/'limit': rows in ORDER BY order,    */
-                               /* at most the limit (stats.groups_total = all distinct groups)   */
+                               /* with 'order'/'limit' (A10): rows in ORDER BY order      */
+                               /* (ties: decoded key tuple ascending), at most the limit         */
+                               /* (hash group-by: stats.groups_total = all distinct groups)      */
   int32_t n_keys;              /* out: group key columns                                          */
   int32_t n_aggs;              /* out: aggregates per row; agg 0 is COUNT(*)                      */
-  int32_t* keys;               /* out: [cap_groups][n_keys] decoded key values, rows sorted by key */
-                               /* (hash group-by with 'order': in the plan's ORDER BY order)      */
+  int32_t* keys;               /* out: [cap_groups][n_keys] key values (after the plan's 'decode' */
+                               /* maps, e.g. nation key -> n_name code); rows sorted by key       */
+                               /* unless the plan has 'order'                                     */
   int64_t* aggs;               /* out: [cap_groups][n_aggs][2] int128 as (lo, hi) little-endian   */
   gpl_stats stats;             /* out */
+  int32_t n_ratios;            /* out: ratio columns of the plan ('ratio [C *] agg I / agg J')    */
+  int32_t reserved;
+  double* ratios;              /* out (optional, may be NULL): [cap_groups][n_ratios] C*num/den    */
+                               /* as doubles (P:634-635 mkt_share, P:682-685 promo_revenue);      */
+                               /* NaN = SQL NULL (den = 0)                                         */
 } gpl_result;
 
 /* A9 model report (gpl_choose_tile_rows). */
@@ -201,8 +208,14 @@ gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_rows);
  * P:564); stats.tile_rows_used = T. */
 gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment);
 
-/* Synchronise the stream and return the last run's result (host decode of
- * the int128 partials; empty groups dropped; ordered by key). Device error
+/* Synchronise the stream and return the last run's result: the A10 finalize
+ * step ("ORDER BY is blocking") — host decode of the
+ * int128 partials, empty groups dropped, group keys mapped through the plan's
+ * 'decode key I TABLE KEYCOL -> OUTCOL' tables, the plan's ORDER BY ('order
+ * agg I|key I [asc|desc], ...'; ties by the key tuple ascending) else key
+ * order, 'limit K', and the 'ratio [C *] agg I / agg J' columns (into
+ * out->ratios when non-NULL; den = 0 gives NaN). Errors: as below, plus
+ * GPL_E_STATE when a decode table misses a group key. Device error
  * flags latched during builds/run are returned here (GPL_E_DUPKEY,
  * GPL_E_DOMAIN, GPL_E_OVERFLOW). GPL_E_CAPACITY if out->cap_groups is too
  * small (out->n_groups then holds the needed rows). */

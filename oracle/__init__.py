@@ -188,8 +188,9 @@ def run(query: str, db, params=None, lineitem_range=None, threads: int = 1) -> R
     s, keep = _db_struct(db)
     lb, le = lineitem_range if lineitem_range is not None else (0, s.n_lineitem)
     cap = 4096 if query != "Q3" else max(4096, s.n_orders)  # Q3 groups <= orders
-    keys = np.zeros(cap * 4, dtype=np.int32)
-    aggs = np.zeros(cap * 4 * 2, dtype=np.int64)
+    nk, na = max(1, len(SCHEMA[query][0])), len(SCHEMA[query][1])
+    keys = np.zeros(cap * nk, dtype=np.int32)
+    aggs = np.zeros(cap * na * 2, dtype=np.int64)
     r = _OracleResult()
     r.cap_rows = cap
     r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data

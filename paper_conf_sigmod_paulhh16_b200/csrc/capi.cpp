@@ -10,6 +10,7 @@
 #include <climits>
 #include <cstring>
 #include <new>
+#include <limits>
 #include <map>
 #include <set>
 #include <string>
@@ -116,30 +117,122 @@ gpl_status take_device_errors(gpl_ctx* ctx) {
   return GPL_OK;
 }
 
+// A10: the key -> output map of a 'decode' statement, read from the loaded
+// table (one small D2H per table version; nation: 25 rows).
+gpl_status decode_map(gpl_ctx* ctx, const DecodeIR& dc, const std::map<int32_t, int32_t>** out) {
+  auto ti = ctx->tables.find(dc.table);
+  if (ti == ctx->tables.end()) return fail(ctx, GPL_E_STATE, "decode: table " + dc.table + " is not loaded");
+  const Table& T = ti->second;
+  const std::string id = dc.table + "." + dc.keycol + "->" + dc.outcol;
+  auto it = ctx->decode_maps.find(id);
+  if (it != ctx->decode_maps.end() && it->second.first == T.version) {
+    *out = &it->second.second;
+    return GPL_OK;
+  }
+  const Column* kc = T.find(dc.keycol);
+  const Column* oc = T.find(dc.outcol);
+  if (!kc || !oc || kc->width != 4 || oc->width != 4) return fail(ctx, GPL_E_STATE, "decode: bad columns of " + dc.table);
+  std::vector<int32_t> k(T.nrows), v(T.nrows);
+  if (T.nrows) {
+    if (ctx->host_only) {
+      std::memcpy(k.data(), kc->host.data(), T.nrows * 4);
+      std::memcpy(v.data(), oc->host.data(), T.nrows * 4);
+    } else {
+      CK(cudaMemcpyAsync(k.data(), kc->dev, T.nrows * 4, cudaMemcpyDeviceToHost, ctx->stream));
+      CK(cudaMemcpyAsync(v.data(), oc->dev, T.nrows * 4, cudaMemcpyDeviceToHost, ctx->stream));
+      CK(cudaStreamSynchronize(ctx->stream));
+    }
+  }
+  std::map<int32_t, int32_t> m;
+  for (int64_t i = 0; i < T.nrows; i++)
+    if (!m.emplace(k[i], v[i]).second)
+      return fail(ctx, GPL_E_DUPKEY, "decode: duplicate key in " + dc.table + "." + dc.keycol);
+  auto& slot = ctx->decode_maps[id];
+  slot.first = T.version;
+  slot.second.swap(m);
+  *out = &slot.second;
+  return GPL_OK;
+}
+
+// A10 ratio columns: scale * double(num) / double(den), den = 0 -> NaN (SQL
+// NULL); the IEEE sequence of reading R12, from the exact int128 sums.
+void fill_ratios(const std::vector<RatioIR>& ratios, gpl_result* out, int rows) {
+  out->n_ratios = (int32_t)ratios.size();
+  if (!out->ratios) return;
+  const int A = out->n_aggs;
+  for (int r = 0; r < rows; r++)
+    for (size_t j = 0; j < ratios.size(); j++) {
+      auto get = [&](int a) {
+        const unsigned __int128 u = ((unsigned __int128)(uint64_t)out->aggs[(r * A + a) * 2 + 1] << 64) |
+                                    (uint64_t)out->aggs[(r * A + a) * 2];
+        return (__int128)u;
+      };
+      const __int128 num = get(ratios[j].num), den = get(ratios[j].den);
+      out->ratios[r * ratios.size() + j] =
+          den == 0 ? std::numeric_limits<double>::quiet_NaN() : ratios[j].scale * (double)num / (double)den;
+    }
+}
+
+// Dense partials -> result rows (A10 finalize, "ORDER BY is blocking";
+// SURVEY §8(a) A10): drop empty groups, decode group ids to key values and
+// through the plan's 'decode' tables, ORDER BY (ties: the decoded key tuple
+// ascending, reading R8) else key order, LIMIT, ratio columns.
 gpl_status decode(gpl_ctx* ctx, const unsigned long long* part, gpl_result* out) {
   const LowerInfo& li = ctx->last.run->li;
-  const int G = li.ngroups_total, A = li.nagg;
-  out->n_keys = li.ngroup_dims;
+  const int G = li.ngroups_total, A = li.nagg, NK = li.ngroup_dims;
+  out->n_keys = NK;
   out->n_aggs = A;
-  int rows = 0;
-  for (int g = 0; g < G; g++) {
-    const bool nonempty = part[2 * (g * A)] != 0 || part[2 * (g * A) + 1] != 0;
-    if (nonempty || !li.has_groups) rows++;
-  }
-  out->n_groups = rows;
-  if (rows > out->cap_groups) return fail(ctx, GPL_E_CAPACITY, "result capacity too small");
-  if (rows && (!out->aggs || (li.ngroup_dims && !out->keys))) return fail(ctx, GPL_E_ARG, "NULL result arrays");
-  int r = 0;
+  out->n_ratios = (int32_t)li.ratios.size();
+  struct Row {
+    int32_t key[MAXG];
+    int g;
+  };
+  std::vector<Row> rows;
   for (int g = 0; g < G; g++) {
     const bool nonempty = part[2 * (g * A)] != 0 || part[2 * (g * A) + 1] != 0;
     if (!nonempty && li.has_groups) continue;
-    for (int k = 0; k < li.ngroup_dims; k++) out->keys[r * li.ngroup_dims + k] = li.glo[k] + (g / li.gstride[k]) % li.gsize[k];
-    for (int a = 0; a < A; a++) {
-      out->aggs[(r * A + a) * 2] = (int64_t)part[2 * (g * A + a)];
-      out->aggs[(r * A + a) * 2 + 1] = (int64_t)part[2 * (g * A + a) + 1];
-    }
-    r++;
+    Row r{};
+    r.g = g;
+    for (int k = 0; k < NK; k++) r.key[k] = li.glo[k] + (g / li.gstride[k]) % li.gsize[k];
+    rows.push_back(r);
   }
+  for (const DecodeIR& dc : li.decodes) {
+    const std::map<int32_t, int32_t>* m = nullptr;
+    gpl_status st = decode_map(ctx, dc, &m);
+    if (st) return st;
+    for (Row& r : rows) {
+      auto it = m->find(r.key[dc.key]);
+      if (it == m->end())
+        return fail(ctx, GPL_E_STATE, "decode: group key " + std::to_string(r.key[dc.key]) + " not in " + dc.table);
+      r.key[dc.key] = it->second;
+    }
+  }
+  auto agg = [&](const Row& r, int a) {
+    return (__int128)(((unsigned __int128)part[2 * (r.g * A + a) + 1] << 64) | part[2 * (r.g * A + a)]);
+  };
+  std::sort(rows.begin(), rows.end(), [&](const Row& x, const Row& y) {
+    for (int i = 0; i < li.norder; i++) {
+      const __int128 a = li.ord_is_agg[i] ? agg(x, li.ord_idx[i]) : (__int128)x.key[li.ord_idx[i]];
+      const __int128 b = li.ord_is_agg[i] ? agg(y, li.ord_idx[i]) : (__int128)y.key[li.ord_idx[i]];
+      if (a != b) return li.ord_desc[i] ? a > b : a < b;
+    }
+    for (int k = 0; k < NK; k++)
+      if (x.key[k] != y.key[k]) return x.key[k] < y.key[k];
+    return false;
+  });
+  if (li.limit > 0 && (int)rows.size() > li.limit) rows.resize(li.limit);
+  const int n = (int)rows.size();
+  out->n_groups = n;
+  if (n > out->cap_groups) return fail(ctx, GPL_E_CAPACITY, "result capacity too small");
+  if (n && (!out->aggs || (NK && !out->keys))) return fail(ctx, GPL_E_ARG, "NULL result arrays");
+  for (int r = 0; r < n; r++) {
+    for (int k = 0; k < NK; k++) out->keys[r * NK + k] = rows[r].key[k];
+    for (int a = 0; a < A; a++) {
+      out->aggs[(r * A + a) * 2] = (int64_t)part[2 * (rows[r].g * A + a)];
+      out->aggs[(r * A + a) * 2 + 1] = (int64_t)part[2 * (rows[r].g * A + a) + 1];
+    }
+  }
+  fill_ratios(li.ratios, out, n);
   return GPL_OK;
 }
 
@@ -152,6 +245,7 @@ gpl_status decode_hash(gpl_ctx* ctx, const unsigned long long* part, gpl_result*
   const uint64_t nrows = part[1];
   out->n_keys = NK;
   out->n_aggs = A;
+  out->n_ratios = (int32_t)li.ratios.size();
   out->n_groups = (int32_t)std::min<uint64_t>(nrows, INT32_MAX);
   if (nrows > (uint64_t)std::max(out->cap_groups, 0)) return fail(ctx, GPL_E_CAPACITY, "result capacity too small");
   if (nrows && (!out->aggs || !out->keys)) return fail(ctx, GPL_E_ARG, "NULL result arrays");
@@ -188,6 +282,7 @@ gpl_status decode_hash(gpl_ctx* ctx, const unsigned long long* part, gpl_result*
       out->aggs[(r * A + a) * 2 + 1] = v < 0 ? -1 : 0;
     }
   }
+  fill_ratios(li.ratios, out, (int)nrows);
   return GPL_OK;
 }
 
@@ -313,11 +408,15 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "build_pipeline") {
     o.build_pipeline = v != 0 ? 1 : 0;
   } else if (k == "hash_slots_log2") {
-    if (v > 0 && (v < 12 || v > 34)) return fail(ctx, GPL_E_ARG, "hash_slots_log2 in [12, 34] (0 = auto)");
+    // slot indices are 32-bit in the ORDER BY/LIMIT selection (0xFFFFFFFF = none)
+    if (v > 0 && (v < 12 || v > 31)) return fail(ctx, GPL_E_ARG, "hash_slots_log2 in [12, 31] (0 = auto)");
     o.hash_slots_log2 = v > 0 ? v : 0;
   } else if (k == "drain_warps") {
     if (v >= 0 && v > 4) return fail(ctx, GPL_E_ARG, "drain_warps in [0, 4] (-1 = model)");
     o.drain_warps = v < 0 ? -1 : v;
+  } else if (k == "agg_mode") {
+    if (v >= 0 && v != AGG_GLOBAL) return fail(ctx, GPL_E_ARG, "agg_mode: 2 (global int128 atomics) or -1 (auto)");
+    o.agg_mode = v < 0 ? -1 : v;
   } else if (k == "graph_branches") {
     // only how whole-query graphs are recorded: drop them, keep plans and pinned shapes
     o.graph_branches = v != 0 ? 1 : 0;
@@ -818,7 +917,7 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
             ? (uint64_t)((double)ge->second.first * std::max(1.0, (double)d.nrows / (double)std::max<int64_t>(ge->second.second, 1)))
             : (uint64_t)std::min<int64_t>(std::max<int64_t>(d.nrows, 1), 1 << 21);
     int lg = 12;
-    while ((1ull << lg) < 2 * est && lg < 34) lg++;
+    while ((1ull << lg) < 2 * est && lg < 31) lg++;  // 32-bit slot indices in the selection
     if (ctx->opt.hash_slots_log2 > 0) lg = (int)ctx->opt.hash_slots_log2;
     const uint64_t cap = 1ull << lg;
     const size_t bytes = (size_t)cap * 8 * (1 + li.nagg);
@@ -920,6 +1019,7 @@ GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t
   L.valid = true;
   L.kbe = false;
   L.copied_out = true;
+  L.overflowed = false;
   L.run = ctx->run_cache[std::string(probe_segment) + "\x1f" + std::to_string(tile_rows)];
   L.timed = true;
   gpl_stats& S = L.stats;
@@ -1019,6 +1119,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       L.valid = true;
       L.kbe = false;
       L.copied_out = true;
+      L.overflowed = false;
       L.run = PP;
       L.timed = true;
       gpl_stats& S = L.stats;
@@ -1525,6 +1626,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   L.valid = true;
   L.kbe = true;
   L.copied_out = false;
+  L.overflowed = false;
   {
     auto kr = std::make_shared<PreparedRun>();
     kr->desc = d;
@@ -1630,6 +1732,7 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
     const uint64_t cap = ctx->last.run->hagg_cap;
     auto& est = ctx->hagg_groups[ctx->last.run->text];
     est.first = (bits & ERR_CAPACITY) ? std::max<uint64_t>(2 * cap, seen) : seen;
+    if (bits & ERR_CAPACITY) ctx->last.overflowed = true;
     est.second = (int64_t)S.rows_scanned;
     S.groups_total = (int64_t)seen;
   }
@@ -1705,7 +1808,13 @@ GPL_API gpl_status gpl_fetch_groups(gpl_ctx* ctx, int64_t* rows, int64_t cap_row
   if (!ctx->last.valid || !ctx->last.run || !ctx->last.run->li.hash_group)
     return fail(ctx, GPL_E_STATE, "gpl_fetch_groups: the last run is not a hash group-by");
   CK(cudaStreamSynchronize(ctx->stream));
-  if ((st = take_device_errors(ctx))) return st;
+  // an overflowed aggregation table holds an incomplete group set: never
+  // returned as rows (whether or not gpl_fetch_result already took the bits)
+  const gpl_status dev_st = take_device_errors(ctx);
+  if (dev_st == GPL_E_CAPACITY || ctx->last.overflowed)
+    return fail(ctx, GPL_E_STATE, "gpl_fetch_groups: the last run's hash group-by table overflowed; run the plan "
+                                  "again (the next run is sized from this one)");
+  if (dev_st) return dev_st;
   const LowerInfo& li = ctx->last.run->li;
   const int W = 1 + li.nagg;
   const unsigned long long* part = (const unsigned long long*)ctx->h_stage + kScratchHead;
@@ -1768,6 +1877,7 @@ GPL_API gpl_status gpl_merge_groups(gpl_ctx* ctx, const char* probe_segment, con
   const int64_t n = s.limit > 0 ? std::min<int64_t>((int64_t)v.size(), s.limit) : (int64_t)v.size();
   out->n_keys = NK;
   out->n_aggs = A;
+  out->n_ratios = (int32_t)s.ratios.size();
   out->n_groups = (int32_t)std::min<int64_t>(n, INT32_MAX);
   out->stats = gpl_stats{};
   out->stats.groups_total = (int64_t)v.size();
@@ -1782,6 +1892,7 @@ GPL_API gpl_status gpl_merge_groups(gpl_ctx* ctx, const char* probe_segment, con
       out->aggs[(r * A + a) * 2 + 1] = (int64_t)(uint64_t)(u >> 64);
     }
   }
+  fill_ratios(s.ratios, out, (int)n);
   return GPL_OK;
 }
 

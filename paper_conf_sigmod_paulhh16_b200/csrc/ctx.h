@@ -84,6 +84,8 @@ struct LowerInfo {
   bool hash_group = false;
   int limit = 0, norder = 0;
   int ord_is_agg[3] = {0, 0, 0}, ord_idx[3] = {0, 0, 0}, ord_desc[3] = {0, 0, 0};
+  std::vector<DecodeIR> decodes;  // A10: group key decodes through loaded tables
+  std::vector<RatioIR> ratios;    // A10: derived ratio columns
   double bw_factor = 1;           // streaming-rate scale, fitted only when the run beat the model's stream bound (L2-resident input)
 };
 
@@ -107,6 +109,7 @@ struct LastRun {
   bool timed = false;
   bool kbe = false;
   bool copied_out = false;  // the run's results were copied to h_stage by the copy-out kernel
+  bool overflowed = false;  // hash group-by: the run's aggregation table overflowed (rows incomplete)
 };
 
 struct PreparedRun {
@@ -167,6 +170,7 @@ struct Options {
   int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
   int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
   int64_t drain_warps = -1;    // operator-specialised drain warps (NEXT-1): -1 = the model's choice
+  int64_t agg_mode = -1;       // dense group accumulators: -1 exactness-driven choice, 2 = force global int128 atomics
 };
 
 // Γ of one ring shape (gpl_calibrate, Eq 1): (bytes, GB/s)
@@ -230,6 +234,8 @@ struct gpl_ctx {
   unsigned long long* d_hcand = nullptr;
   size_t hcand_alloc = 0;
   std::map<std::string, std::pair<uint64_t, int64_t>> hagg_groups;  // plan text -> (distinct groups, fact rows) of its last run
+  // A10 key decodes: table name -> (table version, key -> output value)
+  std::map<std::string, std::pair<uint64_t, std::map<int32_t, int32_t>>> decode_maps;
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;
   size_t kbe_cap = 0;

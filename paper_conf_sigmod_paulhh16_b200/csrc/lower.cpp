@@ -587,14 +587,27 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
       }
     }
     li->hash_group = true;
-    li->limit = s.limit;
-    li->norder = (int)s.order.size();
-    for (int i = 0; i < li->norder; i++) {
-      li->ord_is_agg[i] = s.order[i].is_agg;
-      li->ord_idx[i] = s.order[i].idx;
-      li->ord_desc[i] = s.order[i].desc;
-    }
   }
+  // the result step (A10): ORDER BY / LIMIT (on the device for a hash
+  // group-by, on the host at fetch for dense groups), key decodes, ratios
+  li->limit = s.limit;
+  li->norder = (int)s.order.size();
+  for (int i = 0; i < li->norder; i++) {
+    li->ord_is_agg[i] = s.order[i].is_agg;
+    li->ord_idx[i] = s.order[i].idx;
+    li->ord_desc[i] = s.order[i].desc;
+  }
+  for (const DecodeIR& dc : s.decodes) {
+    auto dt = ctx->tables.find(dc.table);
+    if (dt == ctx->tables.end()) { *err = "decode: unknown table " + dc.table; return GPL_E_STATE; }
+    const Column* kc = dt->second.find(dc.keycol);
+    const Column* oc = dt->second.find(dc.outcol);
+    if (!kc || !oc) { *err = "decode: unknown column of " + dc.table; return GPL_E_STATE; }
+    if (kc->width != 4 || oc->width != 4) { *err = "decode: columns must be 32-bit"; return GPL_E_PLAN; }
+    if (dt->second.nrows > (1 << 20)) { *err = "decode: table larger than 2^20 rows"; return GPL_E_PLAN; }
+  }
+  li->decodes = s.decodes;
+  li->ratios = s.ratios;
   for (int g = s.hash_group ? -1 : d->ngroup - 1; g >= 0; g--) {
     const GroupIR& Gi = s.groups[g];
     GroupDim& D = d->gdim[g];
@@ -697,6 +710,12 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->flush_each_tile = total >= lim ? 1 : 0;
   } else {
     d->agg_mode = (total < lim && (int64_t)d->ngroups_total * d->nagg * 8 <= 48 * 1024) ? AGG_SMEM : AGG_GLOBAL;
+    d->flush_each_tile = 0;
+  }
+  // forced accumulator placement (tests): global int128 atomics are exact for
+  // every plan; registers / the smem table only where the bound above allows
+  if (!s.hash_group && ctx->opt.agg_mode == AGG_GLOBAL) {
+    d->agg_mode = AGG_GLOBAL;
     d->flush_each_tile = 0;
   }
   return GPL_OK;

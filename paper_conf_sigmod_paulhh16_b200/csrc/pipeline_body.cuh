@@ -460,10 +460,16 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
         continue;
       }
       const unsigned long long st = ~key, mask = (1ull << d.hagg_log2) - 1ull;
+      // an overfull table stops early instead of walking every slot: no new
+      // group is claimed past 7/8 load, and a probe gives up after 2^14
+      // steps; both latch ERR_CAPACITY and the host re-runs with a larger table
+      const unsigned long long fill_limit = mask + 1ull - ((mask + 1ull) >> 3);
+      const unsigned long long max_steps = mask < 16383ull ? mask : 16383ull;
       unsigned long long h = (key * 0x9E3779B97F4A7C15ull) >> (64 - d.hagg_log2);
-      for (unsigned long long step = 0; step <= mask; step++, h = (h + 1) & mask) {
+      for (unsigned long long step = 0; step <= max_steps; step++, h = (h + 1) & mask) {
         unsigned long long cur = __ldcg(d.hagg_keys + h);
         if (cur == 0ull) {
+          if (__ldcg(d.hagg_count) >= fill_limit) break;
           cur = atomicCAS(d.hagg_keys + h, 0ull, st);
           if (cur == 0ull) {
             atomicAdd(d.hagg_count, 1ull);

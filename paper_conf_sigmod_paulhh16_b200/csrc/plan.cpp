@@ -56,7 +56,7 @@ bool tokenize(const std::string& line, std::vector<Tok>* out, std::string* err) 
       }
     }
     if (matched) continue;
-    if (std::string("{}(),<>*-+").find(c) != std::string::npos) {
+    if (std::string("{}(),<>*-+/").find(c) != std::string::npos) {
       out->push_back({Tok::SYM, std::string(1, c)});
       i++;
       continue;
@@ -350,6 +350,31 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
           seg->order.push_back(o);
         } while (c.accept_sym(","));
         if (seg->order.size() > 3) throw ParseError{"at most 3 order components"};
+      } else if (kw == "decode") {
+        // decode key I TABLE KEYCOL -> OUTCOL (A10: e.g. nation key -> n_name)
+        if (seg->is_build) throw ParseError{"'decode' only in the probe segment"};
+        if (expect_id(c, "key") != "key") throw ParseError{"decode needs 'key N'"};
+        DecodeIR dc;
+        dc.key = (int)expect_int(c, "key index");
+        dc.table = expect_id(c, "table");
+        dc.keycol = expect_id(c, "key column");
+        expect_sym(c, "->");
+        dc.outcol = expect_id(c, "output column");
+        seg->decodes.push_back(dc);
+      } else if (kw == "ratio") {
+        // ratio [C *] agg I / agg J   (A10: Q8 mkt_share, Q14 promo_revenue)
+        if (seg->is_build) throw ParseError{"'ratio' only in the probe segment"};
+        RatioIR r;
+        if (c.t[c.i].k == Tok::INT) {
+          r.scale = (double)expect_int(c, "scale");
+          expect_sym(c, "*");
+        }
+        if (expect_id(c, "agg") != "agg") throw ParseError{"ratio operands are 'agg N'"};
+        r.num = (int)expect_int(c, "agg index");
+        expect_sym(c, "/");
+        if (expect_id(c, "agg") != "agg") throw ParseError{"ratio operands are 'agg N'"};
+        r.den = (int)expect_int(c, "agg index");
+        seg->ratios.push_back(r);
       } else if (kw == "limit") {
         if (seg->is_build) throw ParseError{"'limit' only in the probe segment"};
         const int64_t k = expect_int(c, "row count");
@@ -403,8 +428,13 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
     if ((int)seg->probes.size() > MAXP) throw ParseError{"too many probes"};
     if ((int)seg->wheres.size() > MAXR) throw ParseError{"too many where clauses"};
     if ((int)seg->groups.size() > MAXG) throw ParseError{"too many group dimensions"};
-    if ((seg->limit || !seg->order.empty()) && !seg->hash_group)
-      throw ParseError{"'order' / 'limit' need 'group hash' (dense group results are ordered on the host)"};
+    for (auto& dc : seg->decodes)
+      if (dc.key < 0 || dc.key >= (int)seg->groups.size() || seg->hash_group)
+        throw ParseError{"decode: key index out of range (dense group keys only)"};
+    if (seg->ratios.size() > 2) throw ParseError{"at most 2 ratio columns"};
+    for (auto& r : seg->ratios)
+      if (r.num < 0 || r.den < 0 || r.num >= (int)seg->aggs.size() || r.den >= (int)seg->aggs.size())
+        throw ParseError{"ratio: agg index out of range"};
     if (seg->limit && seg->order.empty()) throw ParseError{"'limit' needs an 'order' statement"};
     for (auto& o : seg->order)
       if (o.idx < 0 || (o.is_agg ? o.idx >= (int)seg->aggs.size() : o.idx >= (int)seg->groups.size()))

@@ -52,6 +52,20 @@ struct OrderIR {
   bool desc = false;
 };
 
+// A10 finalize (gpl_fetch_result): map a group key's values through a loaded
+// table, e.g. nation key -> n_name code ('decode key 0 nation n_nationkey -> n_name')
+struct DecodeIR {
+  int key = 0;
+  std::string table, keycol, outcol;
+};
+
+// A10 derived column: scale * agg[num] / agg[den] as a double (Q8 mkt_share,
+// Q14 promo_revenue); den = 0 -> NaN (SQL NULL)
+struct RatioIR {
+  double scale = 1.0;
+  int num = 0, den = 0;
+};
+
 struct FactorIR {
   RefIR x;   // CONST => constant a
   int64_t a = 0;
@@ -87,8 +101,10 @@ struct Segment {
   // hash group-by over unbounded keys (NEXT-4): 'group hash A[, B]' (no
   // domain), then optional 'order ...' / 'limit K' run on the device
   bool hash_group = false;
-  std::vector<OrderIR> order;
+  std::vector<OrderIR> order;  // dense groups: applied on the host by gpl_fetch_result (A10)
   int limit = 0;
+  std::vector<DecodeIR> decodes;  // A10: group key decodes through loaded tables
+  std::vector<RatioIR> ratios;    // A10: derived ratio columns
   int split_hint = -2;      // -2: auto
   std::string text;
 };

@@ -61,7 +61,8 @@ class _Stats(ctypes.Structure):
 class _Result(ctypes.Structure):
     _fields_ = [("cap_groups", ctypes.c_int32), ("n_groups", ctypes.c_int32), ("n_keys", ctypes.c_int32),
                 ("n_aggs", ctypes.c_int32), ("keys", ctypes.c_void_p), ("aggs", ctypes.c_void_p),
-                ("stats", _Stats)]
+                ("stats", _Stats), ("n_ratios", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("ratios", ctypes.c_void_p)]
 
 
 class _Model(ctypes.Structure):
@@ -136,12 +137,21 @@ def _i128(lo: int, hi: int) -> int:
 
 @dataclass
 class Result:
+    """Rows as gpl_fetch_result returns them: the plan's ORDER BY order (else key order),
+    decoded keys, exact int128 aggregates, ratio columns (None = SQL NULL)."""
     keys: list
     aggs: list
     stats: dict = field(default_factory=dict)
+    ratios: list = field(default_factory=list)
 
     def as_dict(self):
         return {k: a for k, a in zip(self.keys, self.aggs)}
+
+    def by_key(self) -> "Result":
+        """The same rows in group-key order (for comparisons with key-ordered results)."""
+        order = sorted(range(len(self.keys)), key=lambda i: self.keys[i])
+        return Result([self.keys[i] for i in order], [self.aggs[i] for i in order], self.stats,
+                      [self.ratios[i] for i in order] if self.ratios else [])
 
 
 def _stats_dict(s: _Stats) -> dict:
@@ -290,33 +300,39 @@ class Context:
         # result buffers are reused across calls (grown on GPL_E_CAPACITY)
         if not hasattr(self, "_rbuf"):
             self._rcap = 256
-            self._rbuf = (np.zeros(self._rcap * 4, dtype=np.int32), np.zeros(self._rcap * 8 * 2, dtype=np.int64),
-                          _Result())
-        keys, aggs, r = self._rbuf
-        r.cap_groups = self._rcap
-        r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data
+            self._rbuf = self._alloc_result(self._rcap)
+        keys, aggs, rat, r = self._rbuf
         st = fn(ctypes.byref(r))
         if st == GPL_E_CAPACITY and r.n_groups > self._rcap:
             self._rcap = r.n_groups
-            self._rbuf = (np.zeros(self._rcap * 4, dtype=np.int32), np.zeros(self._rcap * 8 * 2, dtype=np.int64),
-                          _Result())
-            keys, aggs, r = self._rbuf
-            r.cap_groups = self._rcap
-            r.keys, r.aggs = keys.ctypes.data, aggs.ctypes.data
+            self._rbuf = self._alloc_result(self._rcap)
+            keys, aggs, rat, r = self._rbuf
             st = fn(ctypes.byref(r))
         self._check(st)
-        nk, na, ng = r.n_keys, r.n_aggs, r.n_groups
+        nk, na, ng, nr = r.n_keys, r.n_aggs, r.n_groups, r.n_ratios
         kl = keys[:ng * nk].tolist()
         al = aggs[:ng * na * 2].tolist()
+        rl = rat[:ng * nr].tolist()
         out_k = [tuple(kl[i * nk:(i + 1) * nk]) for i in range(ng)]
         out_a = [[_i128(al[(i * na + j) * 2], al[(i * na + j) * 2 + 1]) for j in range(na)] for i in range(ng)]
-        return Result(out_k, out_a, _stats_dict(r.stats))
+        nul = [None if x != x else x for x in rl]  # NaN = SQL NULL
+        out_r = (nul if nr == 1 else [tuple(nul[i * nr:(i + 1) * nr]) for i in range(ng)]) if nr else []
+        return Result(out_k, out_a, _stats_dict(r.stats), out_r)
+
+    @staticmethod
+    def _alloc_result(cap):
+        keys, aggs, rat = (np.zeros(cap * 4, dtype=np.int32), np.zeros(cap * 8 * 2, dtype=np.int64),
+                           np.zeros(cap * 2, dtype=np.float64))
+        r = _Result()
+        r.cap_groups = cap
+        r.keys, r.aggs, r.ratios = keys.ctypes.data, aggs.ctypes.data, rat.ctypes.data
+        return keys, aggs, rat, r
 
     def fetch_groups(self) -> np.ndarray:
         """Rows of the last hash group-by run: int64 [n, 1 + nagg] (packed key, accumulators)."""
         n, w = ctypes.c_int64(0), ctypes.c_int32(0)
         st = self._lib.gpl_fetch_groups(self._h, None, 0, ctypes.byref(n), ctypes.byref(w))  # size query
-        if st not in (0, GPL_E_CAPACITY):
+        if st != 0 and not (st == GPL_E_CAPACITY and n.value > 0):  # CAPACITY is a size answer only with rows
             self._check(st)
         buf = np.zeros((n.value, max(1, w.value)), dtype=np.int64)
         if n.value:

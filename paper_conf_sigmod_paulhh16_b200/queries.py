@@ -7,9 +7,10 @@ predicates are constant-folded to dictionary codes from the loaded catalog
 here, which is the job of a plan generator. The oracle resolves the same
 names by string comparison independently.
 
-Everything that computes runs inside libgpl.so; this module only fills plan
-templates, calls the C ABI in segment order, and finalises results on the
-host (decode keys, ratios, ORDER BY: SURVEY §8(a) A10).
+Everything that computes runs inside libgpl.so, including the A10 finalize
+(key decodes, ORDER BY, ratio columns: the plans' 'decode' / 'order' /
+'ratio' statements, applied by gpl_fetch_result); this module only fills plan
+templates and calls the C ABI.
 """
 from __future__ import annotations
 
@@ -147,6 +148,11 @@ def plan_columns(text: str) -> dict:
             if w in ("scan", "run") and i + 1 < len(words):
                 table = words[i + 1]
                 break
+        for ln in seg.splitlines():  # A10 'decode key I TABLE KEYCOL -> OUTCOL' reads a dimension table
+            w = re.findall(r"[A-Za-z_][A-Za-z_0-9]*", ln.split("#")[0])
+            if len(w) >= 5 and w[0] == "decode" and w[2] in SCHEMA:
+                dc = need.setdefault(w[2], [])
+                dc += [c for c in w[3:5] if c not in dc]
         if table is None or table not in SCHEMA:
             continue
         cols = need.setdefault(table, [])
@@ -176,18 +182,6 @@ def run_segments(ctx: Context, text: str, tile_rows: int = 0, kbe: bool = False)
         ctx.run_plan(segs[-1], tile_rows)
 
 
-def decode_keys(query: str, result: Result, catalog) -> Result:
-    """Nation-valued group keys (nation keys) -> n_name dictionary codes, as SQL outputs n_name."""
-    nat = catalog.tables.get("nation")
-    if nat is None or query not in ("Q5", "Q7", "Q9"):
-        return result
-    name_of = {int(k): int(c) for k, c in zip(nat["n_nationkey"], nat["n_name"])}
-    dims = {"Q5": (0,), "Q7": (0, 1), "Q9": (0,)}[query]
-    keys = [tuple(name_of[v] if i in dims else v for i, v in enumerate(k)) for k in result.keys]
-    order = sorted(range(len(keys)), key=lambda i: keys[i])
-    return Result([keys[i] for i in order], [result.aggs[i] for i in order], result.stats)
-
-
 def run_query(ctx: Context, query: str, catalog, params=None, tile_rows: int = 0, kbe: bool = False) -> Result:
     text = plan_text(query, catalog, params)
     for attempt in range(3):
@@ -196,30 +190,9 @@ def run_query(ctx: Context, query: str, catalog, params=None, tile_rows: int = 0
         else:
             ctx.run_query(text, tile_rows)  # graph-replayed once the plan is warm
         try:
-            return decode_keys(query, ctx.fetch_result(), catalog)
+            return ctx.fetch_result()  # A10 (decode, ORDER BY, ratios) runs in libgpl
         except GplError as e:
             # a hash group-by whose table overflowed: the library sized the
             # next run's table from this one, so run the plan again
             if e.status != GPL_E_CAPACITY or "hash group-by table overflowed" not in str(e) or attempt == 2:
                 raise
-
-
-def finalize(query: str, result: Result, catalog) -> list:
-    """A10: host ratios and ORDER BY of the Listing (ties per DESIGN.md reading R8)."""
-    rows = []
-    for k, a in zip(result.keys, result.aggs):
-        r = {"key": k, "count": a[0], "sums": a[1:]}
-        if query == "Q14":
-            r["promo_revenue"] = None if a[2] == 0 else 100.0 * a[1] / a[2]
-        if query == "Q8":
-            r["mkt_share"] = None if a[2] == 0 else a[1] / a[2]
-        rows.append(r)
-    if query == "Q5":
-        rows.sort(key=lambda r: (-r["sums"][0], r["key"]))
-    elif query == "Q7":
-        rows.sort(key=lambda r: (r["key"][2], r["key"][0], r["key"][1]))
-    elif query == "Q9":
-        rows.sort(key=lambda r: (-r["key"][1], catalog.n_name[r["key"][0]]))
-    else:
-        rows.sort(key=lambda r: r["key"])
-    return rows

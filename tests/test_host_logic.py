@@ -57,7 +57,14 @@ def test_plan_errors(host_ctx):
         "run lineitem\ngroup l_partkey 5 5": gpl.GPL_E_PLAN,
         "run lineitem\nvalue l_extendedprice * l_extendedprice * l_extendedprice\nagg sum": gpl.GPL_E_OVERFLOW,
         # hash group-by / device ORDER BY-LIMIT (NEXT-4)
-        "run lineitem\nagg count\norder agg 0 desc\nlimit 3": gpl.GPL_E_PLAN,
+        # A10 finalize statements
+        "run lineitem\ngroup l_suppkey 0 10\nagg count\ndecode key 1 nation n_nationkey -> n_name": gpl.GPL_E_PLAN,
+        "run lineitem\ngroup l_suppkey 0 10\nagg count\ndecode key 0 nosuch n_nationkey -> n_name": gpl.GPL_E_STATE,
+        "run lineitem\ngroup l_suppkey 0 10\nagg count\ndecode key 0 nation n_nationkey n_name": gpl.GPL_E_PLAN,
+        "run lineitem\nagg count\nratio agg 0 / agg 1": gpl.GPL_E_PLAN,
+        "run lineitem\nagg count\nratio 100 agg 0 / agg 0": gpl.GPL_E_PLAN,
+        "run lineitem\nagg count\norder agg 1 desc": gpl.GPL_E_PLAN,
+        "run lineitem\nagg count\nlimit 3": gpl.GPL_E_PLAN,
         "run lineitem\ngroup hash l_orderkey\nagg count\nlimit 3": gpl.GPL_E_PLAN,
         "run lineitem\ngroup hash l_orderkey\nagg count\norder agg 1 desc": gpl.GPL_E_PLAN,
         "run lineitem\ngroup hash l_orderkey\nagg count\norder key 0 asc\nlimit 513": gpl.GPL_E_PLAN,
@@ -71,6 +78,10 @@ def test_plan_errors(host_ctx):
         assert e.value.status == status, (text, e.value)
     ctx.check_plan("run lineitem\nfilter l_shipdate between 19950101 and 19951231\n"
                    "group year(l_shipdate) 1995 1996\nvalue l_extendedprice * (100 - l_discount)\nagg sum")
+    # dense ORDER BY / LIMIT / ratio / decode (A10, applied by gpl_fetch_result) are valid plans
+    ctx.check_plan("run lineitem\nagg count\norder agg 0 desc\nlimit 3")
+    ctx.check_plan("run lineitem\ngroup l_suppkey 0 10\nvalue l_extendedprice\nagg count\nagg sum\n"
+                   "decode key 0 nation n_nationkey -> n_name\norder agg 1 desc, key 0 asc\nratio 100 * agg 1 / agg 0")
 
 
 def test_segments_split():
