@@ -84,8 +84,9 @@ typedef struct {
   int64_t op_pass[16];         /* rows passing each operator in plan order (filters, probes, where) */
   double kernel_ms;            /* fused pipeline kernel time (CUDA events on the ctx stream)      */
   double predicted_ms;         /* A9 model estimate for this run                                   */
-  double bytes_scanned;        /* algorithmic bytes: rows x bytes/row of TMA-staged columns +      */
-                               /* (rows reaching the first use) x width of each lazy column       */
+  double bytes_scanned;        /* the fused kernel's own HBM bytes: rows x bytes/row of TMA-staged */
+                               /* columns + the clustered probe's table cells + per lazy column   */
+                               /* min(rows reaching its first use x 32 B sector, rows x width)     */
   int32_t agg_mode;            /* 0 registers (1 group), 1 smem table, 2 global int128 atomics,  */
                                /* 3 hash group-by (global open-addressing table, int64 sums)      */
   int32_t kbe;                 /* 1 if produced by gpl_run_plan_kbe                               */

@@ -1680,11 +1680,17 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
     if (cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1) == cudaSuccess) S.kernel_ms = ms;
   }
   for (int i = 0; i < MAXOPS && i < 16; i++) S.op_pass[i] = (int64_t)ops[i];
-  if (!ctx->last.kbe) {  // lazy columns: the rows that reached their first use were gathered
-    double b = (double)S.rows_scanned * li.bytes_per_row;
+  if (!ctx->last.kbe) {
+    // the kernel's own HBM bytes per launch (sector-granular):
+    // staged columns x rows + the clustered probe's table cells + for every
+    // lazy column one 32-B sector per row that reached its first use (a
+    // scattered gather moves a whole sector), at most the column's full scan
+    const double N = (double)S.rows_scanned;
+    double b = N * li.bytes_per_row + (N > 0 ? li.cl_bytes : 0.0);
     for (size_t i = 0; i < li.lazy_w.size(); i++) {
       const int op = li.lazy_reach[i];
-      b += (double)li.lazy_w[i] * (op >= 0 && op < MAXOPS ? (double)ops[op] : (double)S.rows_scanned);
+      const double reach = op >= 0 && op < MAXOPS ? (double)ops[op] : N;
+      b += std::min(reach * 32.0, N * li.lazy_w[i]);
     }
     S.bytes_scanned = b;
   }

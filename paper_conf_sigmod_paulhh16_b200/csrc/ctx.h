@@ -70,6 +70,7 @@ struct LowerInfo {
   int bytes_per_row_all = 0;    // every column the segment reads
   std::vector<int> lazy_w;      // width of each lazy column
   std::vector<int> lazy_reach;  // op whose pass count = rows reaching the column (-1: all rows)
+  double cl_bytes = 0;          // clustered probe: cell bytes of the table the producer stages with the columns
   long double maxabs = 0;  // bound on |value| per row
   std::vector<std::string> op_names;
   std::vector<int64_t> ht_bytes;  // slot bytes of each probed table

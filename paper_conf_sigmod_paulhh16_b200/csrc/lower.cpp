@@ -550,6 +550,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
         d->ht_smem_off[P0.ht] < 0 && H0.bytes() < (1ull << 31)) {
       d->cl_probe = 0;
       d->cl_col = P0.k1;
+      li->cl_bytes = (double)H0.bytes();  // the producer streams the table's cells once (bytes per launch)
     }
   }
   // where residuals
