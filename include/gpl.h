@@ -163,7 +163,15 @@ void gpl_destroy(gpl_ctx* ctx);
  *   GPL_BORROW: data must be device memory, 16-B aligned, with
  *               capacity_rows >= nrows rounded up to 4 rows; the caller keeps
  *               it alive and unchanged while any run may read it.
- * Per-column min/max are computed on load (validator bounds).
+ * Per-column min/max and sortedness are computed on the device with the load
+ * (validator bounds, clustered probes). The call does NOT synchronise: the
+ * copies and the min/max pass are enqueued on the ctx stream, and the first
+ * later call that validates, plans or runs (gpl_check_plan, gpl_build_hash,
+ * gpl_run_*, gpl_autotune, gpl_compile_plan, gpl_choose_tile_rows,
+ * gpl_fetch_result, gpl_sync) waits for all pending loads at once. So a
+ * GPL_COPY source in pinned host or device memory must stay allocated and
+ * unchanged until such a call (pageable host memory is staged by the CUDA
+ * runtime before this call returns).
  * Errors: GPL_E_ARG (type, alignment, duplicate name, nrows < 0), GPL_E_NOMEM. */
 gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nrows, int32_t ncols,
                             const gpl_column* cols, uint32_t flags);

@@ -333,7 +333,65 @@ __global__ void __launch_bounds__(kThreads) minmax_kernel(const char* col, int w
   }
 }
 
+// one table's columns at once (A0 load): blockIdx.y = column
+struct MinmaxCols {
+  const char* col[64];
+  int w[64];
+  long long* out;  // [ncols][3]
+};
+
+__global__ void minmax_init_cols_kernel(long long* out, int ncols) {
+  const int c = threadIdx.x;
+  if (c < ncols) {
+    out[3 * c] = LLONG_MAX;
+    out[3 * c + 1] = LLONG_MIN;
+    out[3 * c + 2] = 0;
+  }
+}
+
+__global__ void __launch_bounds__(kThreads) minmax_cols_kernel(MinmaxCols a, long long n) {
+  const int c = blockIdx.y;
+  const char* col = a.col[c];
+  const int w = a.w[c];
+  long long* out = a.out + 3 * c;
+  long long mn = LLONG_MAX, mx = LLONG_MIN;
+  unsigned long long desc = 0;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const long long v = ld_col_global(col, w, i);
+    mn = min(mn, v);
+    mx = max(mx, v);
+    if (i + 1 < n && v > ld_col_global(col, w, i + 1)) desc++;
+  }
+  if (desc) atomicAdd((unsigned long long*)&out[2], desc);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+    mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMin(&out[0], mn);
+    atomicMax(&out[1], mx);
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_minmax_cols(const char* const* cols, const int* widths, int ncols, long long n, long long* out,
+                               cudaStream_t s) {
+  if (ncols < 1 || ncols > 64) return cudaErrorInvalidValue;
+  minmax_init_cols_kernel<<<1, 64, 0, s>>>(out, ncols);
+  if (n > 0) {
+    MinmaxCols a;
+    for (int c = 0; c < ncols; c++) {
+      a.col[c] = cols[c];
+      a.w[c] = widths[c];
+    }
+    a.out = out;
+    const int gx = (int)std::min<long long>((n + kThreads - 1) / kThreads, std::max(1, 148 * 8 / ncols));
+    minmax_cols_kernel<<<dim3(gx, ncols), kThreads, 0, s>>>(a, n);
+  }
+  return cudaGetLastError();
+}
 
 cudaError_t launch_header_init(HTHeader* hdr, cudaStream_t s) {
   header_init_kernel<<<1, 1, 0, s>>>(hdr);

@@ -58,6 +58,7 @@ int type_width(int t) {
 // After a fused run a one-CTA kernel copies words [0, head + partials) into
 // mapped pinned host memory (h_stage), so fetching needs no D2H copy node.
 constexpr int kScratchHead = 2 + MAXOPS;
+constexpr int kMinmaxSlots = 4096;  // column slots for pending loads' min/max
 constexpr size_t kMaxPartialBytes = (size_t)(1 << 16) * MAXA * 16;
 constexpr size_t kScratchBytes = kScratchHead * 8 + kMaxPartialBytes + MAXOPS * 8;  // + build op counters
 
@@ -177,6 +178,43 @@ void fill_ratios(const std::vector<RatioIR>& ratios, gpl_result* out, int rows) 
 // SURVEY §8(a) A10): drop empty groups, decode group ids to key values and
 // through the plan's 'decode' tables, ORDER BY (ties: the decoded key tuple
 // ascending, reading R8) else key order, LIMIT, ratio columns.
+}  // namespace
+
+// Read back the min/max/sortedness of every pending load (one event wait for
+// the whole batch) and decide each reloaded table's version: unchanged shape
+// (same rows, buffers and value ranges) keeps the old version.
+gpl_status resolve_pending(gpl_ctx* ctx) {
+  if (ctx->pending.empty()) return GPL_OK;
+  CK(cudaEventSynchronize(ctx->mm_ev));
+  for (PendingLoad& pl : ctx->pending) {
+    auto it = ctx->tables.find(pl.table);
+    if (it == ctx->tables.end()) continue;
+    Table& t = it->second;
+    const long long* mm = ctx->h_minmax + 3 * pl.slot0;
+    for (int i = 0; i < pl.ncols && i < (int)t.cols.size(); i++) {
+      t.cols[i].vmin = t.nrows ? mm[3 * i] : 0;
+      t.cols[i].vmax = t.nrows ? mm[3 * i + 1] : 0;
+      t.cols[i].sorted = mm[3 * i + 2] == 0;  // no descent between consecutive rows
+    }
+    if (pl.has_old) {
+      const Table& o = pl.old_meta;
+      bool same = o.nrows == t.nrows && o.cols.size() == t.cols.size();
+      for (size_t i = 0; same && i < t.cols.size(); i++) {
+        const Column& a = o.cols[i];
+        const Column& b = t.cols[i];
+        same = a.name == b.name && a.type == b.type && a.width == b.width && a.dev == b.dev && a.vmin == b.vmin &&
+               a.vmax == b.vmax && a.cap_rows == b.cap_rows && a.sorted == b.sorted;
+      }
+      if (same) t.version = o.version;
+    }
+  }
+  ctx->pending.clear();
+  ctx->mm_next = 0;
+  return GPL_OK;
+}
+
+namespace {
+
 gpl_status decode(gpl_ctx* ctx, const unsigned long long* part, gpl_result* out) {
   const LowerInfo& li = ctx->last.run->li;
   const int G = li.ngroups_total, A = li.nagg, NK = li.ngroup_dims;
@@ -334,7 +372,7 @@ GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
   if ((e = cudaHostGetDevicePointer((void**)&ctx->h_stage_dev, ctx->h_stage, 0)) != cudaSuccess)
     return bad(e, "mapped staging");
   if ((e = cudaMallocHost((void**)&ctx->h_err, 64)) != cudaSuccess) return bad(e, "pinned error word");
-  if ((e = cudaMallocHost((void**)&ctx->h_minmax, 64 * 3 * sizeof(long long))) != cudaSuccess)
+  if ((e = cudaMallocHost((void**)&ctx->h_minmax, kMinmaxSlots * 3 * sizeof(long long))) != cudaSuccess)
     return bad(e, "pinned min/max");
   if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
   if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
@@ -368,6 +406,7 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
       if (e) cudaEventDestroy(e);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+    if (ctx->mm_ev) cudaEventDestroy(ctx->mm_ev);
     if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   }
   delete ctx;
@@ -484,13 +523,18 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
   } else {
     gpl_status st = check_dev(ctx);
     if (st) return st;
-    if (ctx->minmax_cap < (size_t)ncols) {
-      if (ctx->d_minmax) cudaFree(ctx->d_minmax);
-      ctx->d_minmax = nullptr;
-      ctx->minmax_cap = 0;
-      CK(cudaMalloc(&ctx->d_minmax, 64 * 3 * sizeof(long long)));
-      ctx->minmax_cap = 64;
+    // a reload of a table whose previous load is still pending: resolve it first
+    for (auto& pl : ctx->pending)
+      if (pl.table == t.name) {
+        if ((st = resolve_pending(ctx))) return st;
+        break;
+      }
+    if (!ctx->d_minmax) {
+      CK(cudaMalloc(&ctx->d_minmax, kMinmaxSlots * 3 * sizeof(long long)));
+      ctx->minmax_cap = kMinmaxSlots;
     }
+    if (!ctx->mm_ev) CK(cudaEventCreateWithFlags(&ctx->mm_ev, cudaEventDisableTiming));
+    if (ctx->mm_next + ncols > kMinmaxSlots && (st = resolve_pending(ctx))) return st;  // slots exhausted
     auto cleanup = [&]() {  // a failed reload hands reused buffers back to the old table
       auto oldt = ctx->tables.find(t.name);
       for (auto& c : t.cols) {
@@ -552,31 +596,47 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
         t.cols.pop_back();
       }
       t.cols.push_back(c);
-      CK(launch_minmax(c.dev, c.width, nrows, ctx->d_minmax + 3 * i, ctx->stream));
     }
-    long long* mm = ctx->h_minmax;  // pinned (h_stage holds the last run's copied-out results)
-    CK(cudaMemcpyAsync(mm, ctx->d_minmax, sizeof(long long) * 3 * ncols, cudaMemcpyDeviceToHost, ctx->stream));
-    CK(cudaStreamSynchronize(ctx->stream));
+    // per-column min/max/sortedness: one pass over the table's columns, read
+    // back into pinned slots WITHOUT synchronising (resolve_pending reads them
+    // at the first call that plans or validates)
+    const char* cp[64];
+    int cw[64];
     for (int i = 0; i < ncols; i++) {
-      t.cols[i].vmin = nrows ? mm[3 * i] : 0;
-      t.cols[i].vmax = nrows ? mm[3 * i + 1] : 0;
-      t.cols[i].sorted = mm[3 * i + 2] == 0;  // no descent between consecutive rows
+      cp[i] = t.cols[i].dev;
+      cw[i] = t.cols[i].width;
     }
+    const int slot0 = ctx->mm_next;
+    CK(launch_minmax_cols(cp, cw, ncols, nrows, ctx->d_minmax + 3 * slot0, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_minmax + 3 * slot0, ctx->d_minmax + 3 * slot0, sizeof(long long) * 3 * ncols,
+                       cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaEventRecord(ctx->mm_ev, ctx->stream));
+    ctx->mm_next += ncols;
+    PendingLoad pl;
+    pl.table = t.name;
+    pl.slot0 = slot0;
+    pl.ncols = ncols;
+    ctx->pending.push_back(std::move(pl));
   }
   auto old = ctx->tables.find(t.name);
   if (old != ctx->tables.end()) {
     // A reload into the same buffers with the same rows and value ranges keeps
-    // the table's version: prepared plans and query graphs depend only on
-    // those (hash tables built from it are still marked stale until rebuilt).
-    const Table& o = old->second;
-    bool same = o.nrows == t.nrows && o.cols.size() == t.cols.size();
-    for (size_t i = 0; same && i < t.cols.size(); i++) {
-      const Column& a = o.cols[i];
-      const Column& b = t.cols[i];
-      same = a.name == b.name && a.type == b.type && a.width == b.width && a.dev == b.dev && a.vmin == b.vmin &&
-             a.vmax == b.vmax && a.cap_rows == b.cap_rows && a.sorted == b.sorted;
+    // the table's version (decided by resolve_pending once the min/max are
+    // back): prepared plans and query graphs depend only on those (hash tables
+    // built from it are still marked stale until rebuilt).
+    if (!ctx->host_only) {
+      PendingLoad& pl = ctx->pending.back();
+      pl.has_old = true;
+      pl.old_meta.name = old->second.name;
+      pl.old_meta.nrows = old->second.nrows;
+      pl.old_meta.version = old->second.version;
+      for (const Column& oc : old->second.cols) {
+        Column m = oc;
+        m.host.clear();
+        m.owned = false;
+        pl.old_meta.cols.push_back(std::move(m));
+      }
     }
-    if (same && !ctx->host_only) t.version = o.version;
     bool any_owned = false;
     for (auto& c : old->second.cols) any_owned |= c.owned && c.dev;
     if (!ctx->host_only && any_owned) cudaStreamSynchronize(ctx->stream);
@@ -590,6 +650,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
 
 GPL_API gpl_status gpl_check_plan(gpl_ctx* ctx, const char* segment) {
   if (!ctx || !segment) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   Segment s;
   std::string err;
@@ -700,6 +761,7 @@ static gpl_status launch_prepared_build(gpl_ctx* ctx, const PreparedBuild& P) {
 
 GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32_t* ht_id) {
   if (!ctx || !build_segment) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   // fast path: the same segment over unchanged tables / hash tables / options
   if (!ctx->host_only) {
@@ -998,6 +1060,7 @@ static gpl_status get_prepared_run(gpl_ctx* ctx, const char* text, int64_t tile_
 
 GPL_API gpl_status gpl_run_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows) {
   if (!ctx || !probe_segment) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
@@ -1070,6 +1133,7 @@ static std::vector<std::string> split_segments(const std::string& plan) {
 
 GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_rows) {
   if (!ctx || !plan) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
@@ -1376,6 +1440,7 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
 
 GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_candidates, gpl_model_report* out) {
   if (!ctx || !plan) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
@@ -1547,6 +1612,7 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
 
 GPL_API gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int64_t tile_rows) {
   if (!ctx || !probe_segment) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   PipeDesc d;
   LowerInfo li;
@@ -1572,6 +1638,7 @@ GPL_API gpl_status gpl_compile_plan(gpl_ctx* ctx, const char* probe_segment, int
 
 GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   if (!ctx || !probe_segment) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
@@ -1651,6 +1718,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
 
 GPL_API gpl_status gpl_sync(gpl_ctx* ctx) {
   if (!ctx) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   gpl_status st = check_dev(ctx);
   if (st) return st;
   CK(cudaStreamSynchronize(ctx->stream));
@@ -1659,6 +1727,7 @@ GPL_API gpl_status gpl_sync(gpl_ctx* ctx) {
 
 GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
   if (!ctx || !out) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   gpl_status st = check_dev(ctx);
   if (st) return st;
@@ -1773,6 +1842,7 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
 
 GPL_API gpl_status gpl_decode_partials(gpl_ctx* ctx, const void* host_partials, size_t nbytes, gpl_result* out) {
   if (!ctx || !host_partials || !out) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run (the plan of the last run defines the layout)");
   if (ctx->last.run->li.hash_group) return fail(ctx, GPL_E_STATE, "a hash group-by has no dense partial vector");
   const size_t b = (size_t)ctx->last.run->li.ngroups_total * ctx->last.run->li.nagg * 16;
@@ -1904,6 +1974,7 @@ GPL_API gpl_status gpl_merge_groups(gpl_ctx* ctx, const char* probe_segment, con
 
 GPL_API gpl_status gpl_choose_tile_rows(gpl_ctx* ctx, const char* probe_segment, int64_t n_rows, gpl_model_report* out) {
   if (!ctx || !probe_segment || !out) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
   ctx->err.clear();
   Segment s;
   std::string err;

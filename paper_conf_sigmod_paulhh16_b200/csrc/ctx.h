@@ -148,6 +148,17 @@ struct PreparedBuild {
   size_t clear_bytes = 0;  // table cells + the trailing tile counter
 };
 
+// A0 load whose per-column min/max/sortedness are still in flight (a load
+// enqueues its copies + one min/max pass and returns without synchronising;
+// the first call that plans or validates reads them back: one synchronise per
+// batch of loads instead of one per table)
+struct PendingLoad {
+  std::string table;
+  int slot0 = 0, ncols = 0;   // column slots in ctx->d_minmax / h_minmax
+  bool has_old = false;       // the table replaced an earlier version of itself
+  Table old_meta;             // that version's shape (no data): keeps its version when the shape is unchanged
+};
+
 // gpl_autotune's pinned pipeline shape for one probe segment
 struct TunedShape {
   int64_t tile_rows = 0;
@@ -200,8 +211,11 @@ struct gpl_ctx {
   unsigned long long* d_scratch = nullptr;
   unsigned long long* d_partials = nullptr;
   size_t partials_cap = 0;
-  long long* d_minmax = nullptr;
+  long long* d_minmax = nullptr;  // [kMinmaxSlots][3] column slots of pending loads
   size_t minmax_cap = 0;
+  std::vector<gpl::PendingLoad> pending;  // loads whose min/max are not read back yet
+  int mm_next = 0;                        // next free column slot
+  cudaEvent_t mm_ev = nullptr;            // recorded after the last pending load's min/max D2H
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   // whole-query graphs: a second capture lane for build segments that do not
   // depend on each other (fork/join events, created on first use)
@@ -223,7 +237,7 @@ struct gpl_ctx {
   std::map<std::string, std::vector<std::string>> plan_segs;  // gpl_run_query: plan text -> segments
   void* h_stage = nullptr;  // pinned host staging for one packed D2H of results
   unsigned int* h_err = nullptr;  // pinned word for error-bit reads (gpl_sync)
-  long long* h_minmax = nullptr;  // pinned column min/max of a load (64 columns)
+  long long* h_minmax = nullptr;  // pinned column min/max of pending loads ([kMinmaxSlots][3])
   unsigned long long* h_stage_dev = nullptr;  // device alias of h_stage (the fused kernel's result copy-out)
   size_t h_stage_cap = 0;
   // hash group-by (NEXT-4): aggregation table, result rows, selection scratch;

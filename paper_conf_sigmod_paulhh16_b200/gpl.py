@@ -244,8 +244,9 @@ class Context:
             arr[i] = _Column(name.encode(), t, int(scales.get(name, 0)), ptr, on_dev, 0, cap)
         self._check(self._lib.gpl_load_columns(self._h, table.encode(), nrows or 0, len(columns), arr,
                                                GPL_BORROW if borrow else GPL_COPY))
-        if borrow:
-            self._keep[table] = keep  # borrowed memory must outlive the runs
+        # borrowed memory must outlive the runs; a copied source must stay alive until the
+        # next planning call waits for the (unsynchronised) load: kept until the table is reloaded
+        self._keep[table] = keep
 
     def build_hash(self, segment: str) -> int:
         hid = ctypes.c_int32(-1)
