@@ -35,8 +35,9 @@ DEFAULT_PARAMS = {
     "Q9": (1000,),                 # P:677  p_partKey < 1000 (reading #5)
     "Q14": (19950901, 19951001),   # P:688-689  [1995-09-01, 1995-10-01)
     "Q3": (19950315,),             # TPC-H Q3 [EXT] (NEXT-4 workload): o_orderdate < d < l_shipdate
+    "QF": (19950901, 19951001),    # NEXT-4 fan-out workload: l_shipdate in [lo, hi)
 }
-QUERY_IDS = {"L1": 1, "Q5": 5, "Q7": 7, "Q8": 8, "Q9": 9, "Q14": 14, "Q3": 3}
+QUERY_IDS = {"L1": 1, "Q5": 5, "Q7": 7, "Q8": 8, "Q9": 9, "Q14": 14, "Q3": 3, "QF": 101}
 # Result schema (keys, aggs) per query: count(*) first, then the SUMs.
 SCHEMA = {
     "L1": ((), ("count", "sum_charge")),
@@ -46,6 +47,7 @@ SCHEMA = {
     "Q9": (("nation", "o_year"), ("count", "sum_profit")),
     "Q14": ((), ("count", "promo_volume", "total_volume")),
     "Q3": (("l_orderkey", "o_orderdate"), ("count", "revenue")),
+    "QF": (("n_name",), ("count", "revenue")),
 }
 # ORDER BY / LIMIT of the queries that have one on the GPU (Q3: revenue desc,
 # o_orderdate asc, LIMIT 10; ties after that broken by l_orderkey asc — our
@@ -243,6 +245,7 @@ FINALIZE = {
     "Q9": ([(False, 1, True)], None, 0),
     "Q14": ([], (100.0, 1, 2), 0),
     "Q3": ([(True, 1, True), (False, 1, False)], None, 10),
+    "QF": ([(True, 1, True)], None, 0),   # order by revenue desc (our workload)
 }
 
 

@@ -253,7 +253,7 @@ def test_ratio_empty_denominator_is_null():
     assert f.aggs == [[0, 0, 0]] and f.ratios == [None]
 
 
-@pytest.mark.parametrize("query", ["Q5", "Q7", "Q8", "Q9"])
+@pytest.mark.parametrize("query", ["Q5", "Q7", "Q8", "Q9", "QF"])
 def test_finalize_order_matches_bruteforce_selection(query):
     """oracle.finalize's sort == the brute-force repeated selection of bruteforce.order_by, on the
     brute-force evaluator's own groups (tiny SF, several seeds) and on the oracle's groups at
@@ -271,3 +271,47 @@ def test_finalize_order_matches_bruteforce_selection(query):
     if query == "Q8":
         for a, x in zip(f.aggs, f.ratios):
             assert 0.0 <= x <= 1.0 and x == float(a[1]) / float(a[2])
+
+
+# --- NEXT-4 fan-out workload QF (non-unique-key join) --------------------------
+
+def test_qf_worked_example():
+    fx = load("w8_qf_fanout.json")
+    db = build_db(fx)
+    r = oracle.run("QF", db, fx["params"])
+    assert r.keys == expected_keys_as_codes(fx, db) and r.aggs == fx["expected"]["aggs"]
+    f = oracle.finalize("QF", r)
+    assert f.keys == [tuple(db.n_name.index(v) for v in k) for k in fx["expected"]["order"]]
+
+
+def test_qf_bruteforce_seeds():
+    """QF == the brute-force nested loop (which fans out naturally: every partsupp row of the part
+    is a binding) over seeds; the fan-out is real: count = 4 x the window rows when every supplier
+    exists."""
+    nonvacuous = 0
+    for seed in range(1, 11):
+        db = tpchgen.generate(0.002, seed=seed)
+        r = oracle.run("QF", db)
+        b = _bf_as_codes("QF", bf.qf(db), db)
+        assert r.as_dict() == b, seed
+        li = db.tables["lineitem"]
+        m = int(((li["l_shipdate"] >= 19950901) & (li["l_shipdate"] < 19951001)).sum())
+        assert sum(a[0] for a in r.aggs) == 4 * m  # tpchgen: 4 partsupp rows per part, suppliers all exist
+        nonvacuous += m > 0
+    assert nonvacuous >= 8
+
+
+def test_qf_pandas_merge_and_threads():
+    """QF via pandas merge (a non-unique merge fans out) + groupby; the T-thread oracle equals it."""
+    db = tpchgen.generate(0.05, seed=27)
+    f = _frames(db)
+    li = f["lineitem"]
+    li = li[(li.l_shipdate >= 19950901) & (li.l_shipdate < 19951001)]
+    x = (li.merge(f["partsupp"], left_on="l_partkey", right_on="ps_partkey")
+         .merge(f["supplier"], left_on="ps_suppkey", right_on="s_suppkey")
+         .merge(f["nation"], left_on="s_nationkey", right_on="n_nationkey"))
+    x = x.assign(vol=x.l_extendedprice * (100 - x.l_discount))
+    g = x.groupby("n_name").agg(count=("vol", "size"), revenue=("vol", "sum"))
+    exp = {(int(k),): [int(r["count"]), int(r["revenue"])] for k, r in g.iterrows()}
+    assert oracle.run("QF", db).as_dict() == exp and len(exp) == 25
+    assert oracle.run("QF", db, threads=5).as_dict() == exp
