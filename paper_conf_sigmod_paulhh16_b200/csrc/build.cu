@@ -13,7 +13,10 @@
 // last block computes nslots = next_pow2(count * 100 / load_pct) and the
 // ordered-hash multiplier. The clear and insert kernels read the header, so
 // the whole build is asynchronous (no host round trip).
+#include <algorithm>
 #include <climits>
+
+#include <cub/cub.cuh>
 
 #include "device_common.cuh"
 #include "kernels.h"
@@ -374,7 +377,79 @@ __global__ void __launch_bounds__(kThreads) minmax_cols_kernel(MinmaxCols a, lon
   }
 }
 
+// MULTI tables (NEXT-4 fan-out joins, non-unique build key): CSR build.
+// Count pass: per-key match counts (a key outside the declared domain latches
+// ERR_CAPACITY; the domain comes from the key column's min/max, so it cannot
+// happen unless the column changed under a borrowed pointer).
+__global__ void __launch_bounds__(kThreads) multi_count_kernel(const __grid_constant__ BuildDesc d) {
+  __shared__ HTP src[MAXHT];
+  if (threadIdx.x < d.nht) src[threadIdx.x] = load_htp(d.src[threadIdx.x]);
+  __syncthreads();
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long row = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * BR; row < d.nrows; row += stride * BR) {
+    bool ok[BR];
+    unsigned long long k[BR];
+    long long pay[BR];
+    build_rows(d, src, row, stride, ok, k, pay);
+#pragma unroll
+    for (int j = 0; j < BR; j++) {
+      if (!ok[j]) continue;
+      const unsigned long long ix = (unsigned long long)((long long)(int32_t)(uint32_t)k[j] - d.kmin);
+      if (ix >= d.nslots) atomicOr(d.err, ERR_CAPACITY);
+      else atomicAdd(d.cursor + ix, 1u);
+    }
+  }
+}
+
+// Scatter pass: each qualifying row takes the next position of its key's
+// range (the order inside a key's range is arbitrary: a join output is a set)
+__global__ void __launch_bounds__(kThreads) multi_scatter_kernel(const __grid_constant__ BuildDesc d) {
+  __shared__ HTP src[MAXHT];
+  if (threadIdx.x < d.nht) src[threadIdx.x] = load_htp(d.src[threadIdx.x]);
+  __syncthreads();
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long row = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * BR; row < d.nrows; row += stride * BR) {
+    bool ok[BR];
+    unsigned long long k[BR];
+    long long pay[BR];
+    build_rows(d, src, row, stride, ok, k, pay);
+#pragma unroll
+    for (int j = 0; j < BR; j++) {
+      if (!ok[j]) continue;
+      const unsigned long long ix = (unsigned long long)((long long)(int32_t)(uint32_t)k[j] - d.kmin);
+      if (ix >= d.nslots) continue;
+      const unsigned pos = atomicAdd(d.cursor + ix, 1u);
+      ((int*)d.pay)[pos] = (int)pay[j];
+    }
+  }
+}
+
 }  // namespace
+
+size_t multi_scan_tmp_bytes(unsigned long long nslots) {
+  size_t tmp = 0;
+  cub::DeviceScan::ExclusiveSum(nullptr, tmp, (unsigned*)nullptr, (unsigned*)nullptr, (int)(nslots + 1));
+  return tmp;
+}
+
+// MULTI build: counts -> exclusive scan into the offsets (slots) -> cursors =
+// offsets -> scatter. Five stream-ordered steps, no host round trip.
+static cudaError_t launch_build_multi(const BuildDesc& d, int num_sms, cudaStream_t s) {
+  const size_t nb = (size_t)(d.nslots + 1) * 4;
+  cudaError_t e = cudaMemsetAsync(d.cursor, 0, nb, s);
+  if (e != cudaSuccess) return e;
+  long long work = d.nrows > 0 ? d.nrows : 1;
+  int grid = (int)std::min<long long>((work + kThreads * BR - 1) / (kThreads * BR), (long long)num_sms * 8);
+  if (grid < 1) grid = 1;
+  if (d.nrows > 0) multi_count_kernel<<<grid, kThreads, 0, s>>>(d);
+  size_t tmp = (size_t)d.scan_tmp_bytes;
+  e = cub::DeviceScan::ExclusiveSum(d.scan_tmp, tmp, d.cursor, (unsigned*)d.slots, (int)(d.nslots + 1), s);
+  if (e != cudaSuccess) return e;
+  e = cudaMemcpyAsync(d.cursor, d.slots, (size_t)d.nslots * 4, cudaMemcpyDeviceToDevice, s);
+  if (e != cudaSuccess) return e;
+  if (d.nrows > 0) multi_scatter_kernel<<<grid, kThreads, 0, s>>>(d);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_minmax_cols(const char* const* cols, const int* widths, int ncols, long long n, long long* out,
                                cudaStream_t s) {
@@ -402,6 +477,7 @@ cudaError_t launch_build(const BuildDesc& d, bool trivial, const HTHeader& known
   long long work = d.nrows > 0 ? d.nrows : 1;
   int grid = (int)std::min<long long>((work + kThreads * BR - 1) / (kThreads * BR), (long long)num_sms * 8);
   if (grid < 1) grid = 1;
+  if (d.kind == HT_MULTI) return launch_build_multi(d, num_sms, s);
   if (d.kind == HT_DIRECT) {  // host-sized: clear + insert, no count pass
     cudaError_t e = cudaMemsetAsync(d.slots, 0, direct_bytes(d.width, d.nslots), s);
     if (e != cudaSuccess) return e;

@@ -390,6 +390,8 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     for (auto& h : ctx->hts) {
       if (h.slots) cudaFree(h.slots);
       if (h.hdr) cudaFree(h.hdr);
+      if (h.pay) cudaFree(h.pay);
+      if (h.aux) cudaFree(h.aux);
     }
     if (ctx->d_scratch) cudaFree(ctx->d_scratch);
     for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
@@ -836,6 +838,33 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
   H.dkmin = shape.dkmin;
   H.dnslots = shape.dnslots;
   H.pay_base = shape.pay_base;
+  if (shape.kind == HT_MULTI) {
+    // fan-out table (NEXT-4): int32 payload per qualifying row (at most the
+    // table's rows) + scratch for the per-key counts/cursors and the scan
+    const size_t pneed = (std::max<size_t>((size_t)ctx->tables[s.table].nrows, 4) * 4 + 255) / 256 * 256;
+    const size_t cbytes = ((size_t)(shape.dnslots + 1) * 4 + 255) / 256 * 256;
+    const size_t tbytes = multi_scan_tmp_bytes(shape.dnslots);
+    const size_t aneed = cbytes + tbytes + 256;
+    auto grow = [&](void** ptr, size_t* have, size_t want) -> gpl_status {
+      if (*have >= want) return GPL_OK;
+      CK(cudaStreamSynchronize(ctx->stream));
+      if (*ptr) cudaFree(*ptr);
+      *ptr = nullptr;
+      *have = 0;
+      cudaError_t e = cudaMalloc(ptr, want);
+      if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("multi table allocation: ") + cudaGetErrorString(e));
+      *have = want;
+      return GPL_OK;
+    };
+    if ((st = grow(&H.pay, &H.pay_alloc, pneed)) || (st = grow(&H.aux, &H.aux_alloc, aneed))) {
+      H.valid = false;
+      return st;
+    }
+    d.pay = H.pay;
+    d.cursor = (unsigned int*)H.aux;
+    d.scan_tmp = (char*)H.aux + cbytes;
+    d.scan_tmp_bytes = tbytes;
+  }
   if (!H.hdr) {
     CK(cudaMalloc(&H.hdr, sizeof(HTHeader)));
     CK(launch_header_init(H.hdr, ctx->stream));
@@ -1655,6 +1684,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   ctx->opt.lazy_columns = lazy_opt;
   if (st) return st;
   if (li.hash_group) return fail(ctx, GPL_E_PLAN, "the KBE baseline has no hash group-by ('group hash')");
+  if (d.fan_probe >= 0) return fail(ctx, GPL_E_PLAN, "the KBE baseline has no fan-out join (a 'multi' table)");
   const size_t pbytes = (size_t)li.ngroups_total * li.nagg * 16;
   d.partials = partials_ptr(ctx);
   d.tile_counter = counter_ptr(ctx);

@@ -49,7 +49,10 @@ struct Filt {
 // DIRECT: direct-addressed array over a dense key domain [kmin, kmin+nslots)
 //   (a collision-free perfect hash): width 0 = bitmap set, else 1/2/4-byte
 //   cells holding payload - pay_base + 1 (0 = empty).
-enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2, HT_DIRECT = 3 };
+// MULTI (non-unique build keys): CSR over a dense key
+//   domain — slots = uint32 offsets[nslots + 1], pay = int32 payload[count];
+//   key k's matches are pay[off[k - kmin] .. off[k - kmin + 1]) (fan-out join).
+enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2, HT_DIRECT = 3, HT_MULTI = 4 };
 enum : int32_t { H_MULT = 0, H_ORDERED = 1 };
 
 // Device-resident header, written by the build's count and size kernels and
@@ -75,6 +78,7 @@ struct HTRef {
   unsigned long long nslots;
   long long pay_base;
   int32_t width, pad;
+  const void* pay;  // MULTI: the payload array (slots = offsets)
 };
 
 // ---- probes
@@ -169,6 +173,9 @@ struct PipeDesc {
   // cl_off) beside the columns and the probe reads shared memory
   int32_t cl_probe, cl_col, cl_off, cl_cap;
   int32_t rowid_field;   // queue field holding the row id (-1: no lazy column)
+  // fan-out probe (NEXT-4): queue-phase probe into a MULTI table; every match
+  // of a row continues through the remaining operators (-1: none)
+  int32_t fan_probe, fan_pad;
   int32_t term_field[MAXTERM];  // >= 0: term t was computed in the stage phase into this field
   Term sterm[MAXTERM];          // stage-phase form of pushed-down terms (stage refs)
   int32_t nfield, nresid, ngroup, ngroups_total;
@@ -239,6 +246,10 @@ struct BuildDesc {
   HTRef src[MAXHT];
   void* slots;        // destination table
   HTHeader* hdr;
+  void* pay;          // MULTI: payload array
+  unsigned int* cursor;  // MULTI: per-key counts, then scatter cursors [nslots + 1]
+  void* scan_tmp;        // MULTI: device scan scratch
+  unsigned long long scan_tmp_bytes;
   long long cap_slots;
   int32_t kind, hash, load_pct, width;  // width: DIRECT cell bytes (0 = bitmap)
   long long kmin, pay_base;             // DIRECT key / payload bases

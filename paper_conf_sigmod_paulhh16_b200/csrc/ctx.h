@@ -52,11 +52,17 @@ struct HashTable {
   int width = 0;
   long long dkmin = 0, pay_base = 0;
   unsigned long long dnslots = 0;
+  // MULTI (fan-out): payload array and scan/scatter scratch
+  void* pay = nullptr;
+  size_t pay_alloc = 0;
+  void* aux = nullptr;
+  size_t aux_alloc = 0;
   size_t bytes() const {
+    if (kind == HT_MULTI) return (dnslots + 1) * 4;
     if (kind == HT_DIRECT) return width == 0 ? (dnslots + 31) / 32 * 4 : (dnslots * width + 3) / 4 * 4;
     return (size_t)cap_slots * (kind == HT_SET32 ? 4 : kind == HT_MAP32 ? 8 : 16);
   }
-  HTRef ref() const { return HTRef{slots, hdr, kind, hash, dkmin, dnslots, pay_base, width, 0}; }
+  HTRef ref() const { return HTRef{slots, hdr, kind, hash, dkmin, dnslots, pay_base, width, 0, pay}; }
   std::string src_table;
   uint64_t src_version = 0;
   bool valid = false;

@@ -20,6 +20,7 @@ struct HTP {
   long long pay_base;             // DIRECT payload base
   uint32_t mask, shift;
   int32_t kind, hash, width, pad;
+  const void* pay;                // MULTI payload array
 };
 
 __device__ __forceinline__ HTP load_htp(const HTRef& r) {
@@ -29,7 +30,8 @@ __device__ __forceinline__ HTP load_htp(const HTRef& r) {
   p.hash = r.hash;
   p.width = r.width;
   p.pad = 0;
-  if (r.kind == HT_DIRECT) {
+  p.pay = r.pay;
+  if (r.kind == HT_DIRECT || r.kind == HT_MULTI) {
     p.kmin = (unsigned long long)r.kmin;
     p.nslots = r.nslots;
     p.pay_base = r.pay_base;

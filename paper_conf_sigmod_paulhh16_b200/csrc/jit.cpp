@@ -132,6 +132,7 @@ std::string shape_source(const PipeDesc& d) {
   I("cl_col", d.cl_col);
   I("cl_off", d.cl_off);
   I("cl_cap", d.cl_cap);
+  I("fan_probe", d.fan_probe);
   for (int f = 0; f < MAXQ; f++) o << "  k.qlazy[" << f << "] = " << d.qlazy[f] << ";\n";
   auto term = [&](const char* arr, int t, const Term& T) {
     o << "  k." << arr << "[" << t << "].sign = " << T.sign << "; k." << arr << "[" << t << "].nfact = " << T.nfact << ";\n";

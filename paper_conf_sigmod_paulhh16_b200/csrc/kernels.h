@@ -58,6 +58,8 @@ cudaError_t launch_copyout(const unsigned long long* src, unsigned long long* ho
 // Column min/max (int32 or int64 column, n rows) -> out[0] = min, out[1] = max.
 // out[2] = number of descents (rows i with v[i] > v[i+1]): 0 means sorted.
 cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s);
+// device scan scratch of a MULTI (fan-out) build over nslots keys
+size_t multi_scan_tmp_bytes(unsigned long long nslots);
 // per-column {min, max, descents} of one table's columns in two launches (A0 load)
 cudaError_t launch_minmax_cols(const char* const* cols, const int* widths, int ncols, long long n, long long* out,
                                cudaStream_t s);

@@ -94,6 +94,7 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
     const HashTable& H = ctx->hts[hit->second];
     if (!H.valid) { *err = "hash table '" + P.ht + "' is stale (its table was reloaded)"; return GPL_E_STATE; }
     if (P.kind == P_MARK) { *err = "'mark' is not allowed in a build segment"; return GPL_E_PLAN; }
+    if (H.kind == HT_MULTI) { *err = "a 'multi' table is probed by an inner 'probe' of a probe segment"; return GPL_E_PLAN; }
     if ((int)P.keys.size() != H.key_arity) { *err = "key arity mismatch probing " + P.ht; return GPL_E_PLAN; }
     if (!P.out.empty() && !H.has_payload) { *err = P.ht + " has no payload to bind to '" + P.out + "'"; return GPL_E_PLAN; }
     int k1, k2 = -1;
@@ -141,16 +142,37 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
   int load = ctx->opt.hash_load_pct > 0 ? (int)ctx->opt.hash_load_pct : s.load_pct;
   if (shape->key_arity == 2) shape->kind = HT_MAP64;
   else shape->kind = shape->has_payload ? HT_MAP32 : HT_SET32;
-  if (shape->kind == HT_MAP32 && (shape->pay_min < INT32_MIN || shape->pay_max > INT32_MAX)) {
+  if (!s.multi && shape->kind == HT_MAP32 && (shape->pay_min < INT32_MIN || shape->pay_max > INT32_MAX)) {
     *err = "payload range does not fit the 32-bit payload of a single-key table";
     return GPL_E_OVERFLOW;
   }
   shape->hash = shape->kind == HT_MAP64 ? H_MULT : std::max(s.hash, 0);
+  if (s.multi) {
+    // non-unique key (NEXT-4 fan-out join): CSR over the key column's dense
+    // domain — offsets[nslots + 1] + an int32 payload per qualifying row
+    if (shape->key_arity != 1) { *err = "'multi' tables take a single key column"; return GPL_E_PLAN; }
+    if (shape->has_payload && (shape->pay_min < INT32_MIN || shape->pay_max > INT32_MAX)) {
+      *err = "a 'multi' payload must fit 32 bits";
+      return GPL_E_OVERFLOW;
+    }
+    const Column* kc = cols[d->k1];
+    const long long kmin = T.nrows ? kc->vmin : 0, kmax = T.nrows ? kc->vmax : 0;
+    const unsigned long long range = (unsigned long long)(kmax - kmin) + 1ull;
+    if (range > (1ull << 31) || T.nrows >= (1ll << 32)) { *err = "'multi' key domain too large"; return GPL_E_PLAN; }
+    shape->kind = HT_MULTI;
+    shape->hash = 0;
+    shape->width = 4;
+    shape->dkmin = kmin;
+    shape->dnslots = range;
+    shape->pay_base = 0;
+    if (!shape->has_payload) shape->pay_min = shape->pay_max = 1;
+  }
+
   // DIRECT (collision-free) addressing over a dense key domain: single int32
   // key, domain [min, max] of the key column, cells just wide enough for the
   // payload range. Chosen when its size is modest or within 2x of the hashed
   // table's upper-bound size (explicit 'hash mult|ordered' keeps hashing).
-  if (shape->key_arity == 1 && (s.hash == -1 || s.hash == 2)) {
+  if (!s.multi && shape->key_arity == 1 && (s.hash == -1 || s.hash == 2)) {
     const Column* kc = cols[d->k1];
     const long long kmin = T.nrows ? kc->vmin : 0, kmax = T.nrows ? kc->vmax : 0;
     const unsigned long long range = (unsigned long long)(kmax - kmin) + 1ull;
@@ -202,6 +224,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   li->table = s.table;
   if (s.is_build && !ins) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
   d->cl_probe = d->cl_col = -1;
+  d->fan_probe = -1;
   if (ins && (!s.is_build || ins->kind != HT_DIRECT || s.key.size() != 1)) {
     *err = "pipelined build needs a single-key DIRECT build segment";
     return GPL_E_PLAN;
@@ -233,6 +256,11 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     if (P.kind == P_INNER && !P.out.empty() && !H.has_payload) {
       *err = P.ht + " has no payload to bind to '" + P.out + "' (use semi or mark)";
       return GPL_E_PLAN;
+    }
+    if (H.kind == HT_MULTI) {  // non-unique build key: a fan-out inner join (NEXT-4)
+      if (P.kind != P_INNER || ins) { *err = "a 'multi' table is probed by an inner 'probe' of a probe segment"; return GPL_E_PLAN; }
+      if (d->fan_probe >= 0) { *err = "at most one fan-out probe (into a 'multi' table) per segment"; return GPL_E_PLAN; }
+      d->fan_probe = p;
     }
     pht[p] = &H;
     if (!ht_slot.count(H.id)) {
@@ -281,12 +309,24 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   int tmp;
   for (auto& f : s.filters)
     if ((st = stage(f.col, &tmp))) return st;
-  for (auto& p : s.probes)
-    for (auto& k : p.keys) {
-      if (slot_of.count(k)) { *err = "probe keys must be columns"; return GPL_E_PLAN; }
+  // probes keyed by an earlier probe's slot (a chained join, e.g. partsupp ->
+  // supplier) run in the queue phase, where slots are queue fields
+  int first_queue_only = np;
+  for (int p = 0; p < np; p++)
+    for (auto& k : s.probes[p].keys) {
+      if (slot_of.count(k)) {
+        if (slot_of[k] >= p || s.probes[slot_of[k]].kind == P_MARK || pht[slot_of[k]]->kind == HT_MAP64) {
+          *err = "probe key slot '" + k + "' must be a 32-bit payload of an earlier probe";
+          return GPL_E_PLAN;
+        }
+        first_queue_only = std::min(first_queue_only, p);
+        continue;
+      }
       if ((st = stage(k, &tmp))) return st;
       if (!is_int32(*cols[tmp])) { *err = "probe key '" + k + "' must be a 32-bit column"; return GPL_E_PLAN; }
     }
+  if (d->fan_probe >= 0) first_queue_only = std::min(first_queue_only, d->fan_probe);
+  if (ins && first_queue_only < np) { *err = "a pipelined build cannot probe by a slot"; return GPL_E_PLAN; }
   for (auto& g : s.groups)
     if (!slot_of.count(g.ref.name)) {
       if ((st = stage(g.ref.name, &tmp))) return st;
@@ -318,7 +358,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   int sp = split;
   if (sp < 0 && s.split_hint >= -1) sp = s.split_hint;
   if (sp < 0) sp = s.filters.empty() ? std::min(1, np) : 0;
-  sp = std::min(std::min(sp, np), MAXSP);
+  sp = std::min(std::min(std::min(sp, np), MAXSP), first_queue_only);
 
   // Late materialisation (the paper's k_reduce fetches
   // LINEITEM only for the satisfied tuples). A column used only after
@@ -391,7 +431,8 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     if (std::find(qcols.begin(), qcols.end(), n) == qcols.end()) qcols.push_back(n);
   };
   for (int p = sp; p < np; p++)
-    for (auto& k : s.probes[p].keys) need_col(k);
+    for (auto& k : s.probes[p].keys)
+      if (!slot_of.count(k)) need_col(k);
   for (auto& g : s.groups)
     if (!slot_of.count(g.ref.name)) need_col(g.ref.name);
   for (size_t t = 0; t < s.value.size(); t++)
@@ -411,6 +452,9 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
         if (f.x.kind != RefIR::CONST && slot_of.count(f.x.name)) used_slots.insert(f.x.name);
   for (auto& a : s.aggs)
     if (a.kind >= A_SUMIF) used_slots.insert(a.slot);
+  for (auto& pr : s.probes)
+    for (auto& k : pr.keys)
+      if (slot_of.count(k)) used_slots.insert(k);
   if (ins) {
     need_col(s.key[0]);
     if (ins->has_payload) {

@@ -63,7 +63,7 @@ constexpr int kOffFull = 0;       // unsigned long long[kMaxDepth]
 constexpr int kOffEmpty = 64;     // unsigned long long[kMaxDepth]
 constexpr int kOffHdr = 128;      // int4[kMaxDepth]
 constexpr int kOffHtp = 256;      // HTP[MAXHT]
-constexpr int kOffHdr2 = 768;     // int4[kMaxDepth]: clustered-probe cell range (start lo, hi, bytes)
+constexpr int kOffHdr2 = 896;     // int4[kMaxDepth]: clustered-probe cell range (start lo, hi, bytes)
 constexpr int kOffCnt = 1024;     // unsigned long long[kMaxWarps][MAXOPS]
 // drain hand-off ring (ndrain > 0): a bounded multi-producer / multi-consumer
 // queue of R slots. Slot s carries a sequence number: ticket t may fill it
@@ -347,6 +347,11 @@ __device__ __forceinline__ void insert_cells(const PipeDesc& d, const PipeDesc& 
 // Queue phase on up to RPL*32 queued survivors starting at qhead: lane `lane`
 // owns entries qhead + j*32 + lane (j < RPL) that are < n. Remaining probes,
 // where residuals, group-by and the exact aggregation (A5-A7).
+// A fan-out probe (NEXT-4: inner join on a non-unique build key, MULTI table)
+// expands each row into its matches: the warp loops over the match index m
+// (up to the warp's largest match count); match m of every row writes its
+// payload into the row's queue field and continues through the remaining
+// probes, residuals and the sink, so no expanded row is ever materialised.
 __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead, int n, unsigned long long* cnt,
                                        long long* acc, int lane) {
   const PipeDesc& K = GPL_SHAPE_OF(d);
@@ -377,8 +382,9 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
         if (p[j]) qput(K, qb, f, idx[j], v[j]);
     }
   }
+  auto run_probes = [&](int lo, int hi, bool (&p)[RPL]) {
   GPL_UNROLL
-  for (int pi = K.nsprobe; pi < K.nprobe; pi++) {
+  for (int pi = lo; pi < hi; pi++) {
     const int op = K.nfilt + pi;
     const Probe& P = K.probe[pi];
     if (__any_sync(0xffffffffu, any4(p))) {
@@ -404,6 +410,8 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
     const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
     if (lane == 0) cnt[op] += c;
   }
+  };
+  auto tail = [&](bool (&p)[RPL]) {
   GPL_UNROLL
   for (int r = 0; r < K.nresid; r++) {
     const int op = K.nfilt + K.nprobe + r;
@@ -530,6 +538,44 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
         else if (K.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * K.nagg + a], (unsigned long long)c);
         else atomic_add_i128(d.partials + 2 * (gid * K.nagg + a), c);
       }
+    }
+  }
+  };
+  if (K.fan_probe < 0) {
+    run_probes(K.nsprobe, K.nprobe, p);
+    tail(p);
+    return;
+  }
+  run_probes(K.nsprobe, K.fan_probe, p);
+  {
+    const Probe& P = K.probe[K.fan_probe];
+    const HTP& h = htp[P.ht];
+    const uint32_t* off = (const uint32_t*)h.slots;
+    uint32_t beg[RPL], end[RPL];
+    int mx = 0;
+    unsigned tot = 0;
+#pragma unroll
+    for (int j = 0; j < RPL; j++) {
+      const unsigned long long ix =
+          (unsigned long long)((long long)(int32_t)(uint32_t)qget(K, qb, P.k1, idx[j]) - (long long)h.kmin);
+      const bool in = p[j] && ix < h.nslots;
+      beg[j] = in ? __ldg(off + ix) : 0u;
+      end[j] = in ? __ldg(off + ix + 1) : 0u;
+      mx = max(mx, (int)(end[j] - beg[j]));
+      tot += end[j] - beg[j];
+    }
+    mx = __reduce_max_sync(0xffffffffu, (unsigned)mx);
+    const unsigned c = __reduce_add_sync(0xffffffffu, tot);  // output rows of the join
+    if (lane == 0) cnt[K.nfilt + K.fan_probe] += c;
+    for (int m = 0; m < mx; m++) {
+      bool q[RPL];
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
+        q[j] = beg[j] + (uint32_t)m < end[j];
+        if (q[j] && P.out >= 0) qput(K, qb, P.out, idx[j], (long long)__ldg((const int*)h.pay + beg[j] + m));
+      }
+      run_probes(K.fan_probe + 1, K.nprobe, q);
+      tail(q);
     }
   }
 }

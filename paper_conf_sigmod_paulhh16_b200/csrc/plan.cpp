@@ -284,6 +284,9 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
         else if (h == "direct") seg->hash = 2;
         else if (h == "auto") seg->hash = -1;
         else throw ParseError{"hash must be auto, direct, mult or ordered"};
+      } else if (kw == "multi") {  // non-unique key: every match joins (NEXT-4 fan-out)
+        if (!seg->is_build) throw ParseError{"'multi' only in build segments"};
+        seg->multi = true;
       } else if (kw == "load") {
         seg->load_pct = (int)expect_int(c, "percent");
         if (seg->load_pct < 10 || seg->load_pct > 90) throw ParseError{"load must be in [10, 90]"};

@@ -92,6 +92,7 @@ struct Segment {
   std::vector<std::string> key;
   RefIR payload;  // CONST kind => none
   int hash = -1;  // -1 auto, H_MULT, H_ORDERED, 2 = direct
+  bool multi = false;  // 'multi': the key is not unique; probes join every match (NEXT-4 fan-out)
   int load_pct = 50;
   // probe segment
   std::vector<WhereIR> wheres;

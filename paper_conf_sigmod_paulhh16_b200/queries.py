@@ -43,13 +43,14 @@ DEFAULT_PARAMS = {
     "Q9": (1000,),                # P:677, p_partKey < 1000
     "Q14": (19950901, 19951001),  # P:688-689, [lo, hi)
     "Q3": (19950315,),            # TPC-H Q3 [EXT]: o_orderdate < d, l_shipdate > d
+    "QF": (19950901, 19951001),   # NEXT-4 fan-out workload: l_shipdate in [lo, hi)
 }
 # the paper's queries (Listings 1-6)
 QUERIES = ["L1", "Q5", "Q7", "Q8", "Q9", "Q14"]
 # SURVEY §8(f) NEXT-4 workloads beyond the paper's FK->PK star joins with
 # declared group domains: TPC-H Q3 (hash group-by over unbounded keys + device
-# ORDER BY/LIMIT)
-EXTRA_QUERIES = ["Q3"]
+# ORDER BY/LIMIT) and QF (a fan-out join on the non-unique ps_partkey)
+EXTRA_QUERIES = ["Q3", "QF"]
 # fact-table (lineitem) columns each probe segment stages, for reporting
 FACT_COLUMNS = {
     "L1": ["l_shipdate", "l_extendedprice", "l_discount", "l_tax"],
@@ -59,6 +60,7 @@ FACT_COLUMNS = {
     "Q9": ["l_partkey", "l_suppkey", "l_orderkey", "l_extendedprice", "l_discount", "l_quantity"],
     "Q14": ["l_shipdate", "l_partkey", "l_extendedprice", "l_discount"],
     "Q3": ["l_shipdate", "l_orderkey", "l_extendedprice", "l_discount"],
+    "QF": ["l_shipdate", "l_partkey", "l_extendedprice", "l_discount"],
 }
 # tables each query reads
 TABLES = {
@@ -69,6 +71,7 @@ TABLES = {
     "Q9": ["part", "partsupp", "supplier", "orders", "lineitem", "nation"],
     "Q14": ["part", "lineitem"],
     "Q3": ["customer", "orders", "lineitem"],
+    "QF": ["partsupp", "supplier", "lineitem", "nation"],
 }
 
 
@@ -108,6 +111,8 @@ def plan_params(query: str, catalog, params=None) -> dict:
         return {"p_bound": p[0]}
     if query == "Q3":
         return {"building": list(catalog.c_mktsegment).index("BUILDING"), "date": p[0]}
+    if query == "QF":
+        return {"sd_lo": p[0], "sd_hi_incl": p[1] - 1}
     if query == "Q14":
         promo = [i for i, s in enumerate(catalog.p_type) if s.startswith("PROMO")]
         lo, hi = (min(promo), max(promo)) if promo else (1, 0)

@@ -663,3 +663,58 @@ def test_hash_groupby_shards_merge_exact(ctx):
     full_seg = "\n".join(ln for ln in seg.splitlines() if not ln.startswith(("order", "limit")))
     r = ctx.merge_groups(full_seg, np.concatenate(full))
     assert r.keys == whole.keys and r.aggs == whole.aggs
+
+
+# ---- fan-out join on a non-unique key (QF: lineitem x every partsupp row of the part)
+
+@pytest.mark.parametrize("sf,seed", [(0.01, 20160626), (0.2, 5), (1.0, 20160626)])
+def test_qf_fanout_exact(ctx, sf, seed):
+    db = tpchgen.generate(sf, seed=seed)
+    r = _gpu(ctx, db, "QF")
+    o = _oracle("QF", db)
+    assert r.keys == o.keys and r.aggs == o.aggs
+    li = db.tables["lineitem"]
+    window = int(((li["l_shipdate"] >= 19950901) & (li["l_shipdate"] < 19951001)).sum())
+    assert sum(a[0] for a in r.aggs) == 4 * window  # every lineitem joins its part's 4 suppliers
+    assert r.stats["op_pass"][:2] == [window, 4 * window]  # filter, then the fan-out probe's output rows
+
+
+def test_qf_worked_example(ctx):
+    fx = load("w8_qf_fanout.json")
+    db = build_db(fx)
+    r = _gpu(ctx, db, "QF", fx["params"], tables=list(db.tables))
+    assert r.keys == [tuple(db.n_name.index(v) for v in k) for k in fx["expected"]["order"]]
+    assert r.by_key().aggs == fx["expected"]["aggs"]
+
+
+@pytest.mark.parametrize("n", [0, 1, 33, 4097])
+def test_qf_ragged_and_empty(ctx, n):
+    db = tpchgen.generate(0.05, seed=9)
+    db.tables["lineitem"] = {c: v[:n].copy() for c, v in db.tables["lineitem"].items()}
+    # a wide window so the few rows survive
+    r = _gpu(ctx, db, "QF", (19920101, 19990101))
+    o = _oracle("QF", db, (19920101, 19990101))
+    assert r.keys == o.keys and r.aggs == o.aggs
+
+
+def test_qf_schedules_drains_and_kbe_rejects(ctx):
+    db = tpchgen.generate(0.1, seed=14)
+    params = (19950101, 19960101)  # ~15% of the rows survive the window
+    o = _oracle("QF", db, params)
+    knobs = [dict(stage_rows=256, ring_depth=2, consumer_warps=1), dict(packets=2, consumer_warps=6),
+             dict(lazy_columns=0), dict(lazy_columns=1), dict(drain_warps=1), dict(drain_warps=2, consumer_warps=6)]
+    try:
+        for k in knobs:
+            for key, v in k.items():
+                ctx.set_option(key, v)
+            for tile in (0, 3000):
+                r = _gpu(ctx, db, "QF", params, tile_rows=tile)
+                assert r.keys == o.keys and r.aggs == o.aggs, (k, tile)
+            for key in k:
+                ctx.set_option(key, -1)
+    finally:
+        for key in ("stage_rows", "ring_depth", "consumer_warps", "packets", "lazy_columns", "drain_warps"):
+            ctx.set_option(key, -1)
+    with pytest.raises(gpl.GplError) as e:
+        queries.run_query(ctx, "QF", db, params, kbe=True)
+    assert e.value.status == gpl.GPL_E_PLAN
