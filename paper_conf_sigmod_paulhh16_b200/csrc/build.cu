@@ -424,7 +424,31 @@ __global__ void __launch_bounds__(kThreads) multi_scatter_kernel(const __grid_co
   }
 }
 
+// Row range [lower_bound(lo), upper_bound(hi)) of a non-decreasing column.
+__global__ void sorted_bounds_kernel(const char* col, int w, long long n, long long lo, long long hi, long long* out) {
+  long long a = 0, b = n;  // first row with v >= lo
+  while (a < b) {
+    const long long m = (a + b) / 2;
+    if (ld_col_global(col, w, m) < lo) a = m + 1;
+    else b = m;
+  }
+  out[0] = a;
+  b = n;  // first row with v > hi (from the lower bound on)
+  while (a < b) {
+    const long long m = (a + b) / 2;
+    if (ld_col_global(col, w, m) <= hi) a = m + 1;
+    else b = m;
+  }
+  out[1] = a;
+}
+
 }  // namespace
+
+cudaError_t launch_sorted_bounds(const void* col, int w, long long n, long long lo, long long hi, long long* out,
+                                 cudaStream_t s) {
+  sorted_bounds_kernel<<<1, 1, 0, s>>>((const char*)col, w, n, lo, hi, out);
+  return cudaGetLastError();
+}
 
 size_t multi_scan_tmp_bytes(unsigned long long nslots) {
   size_t tmp = 0;

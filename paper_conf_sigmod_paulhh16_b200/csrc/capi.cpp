@@ -290,24 +290,24 @@ gpl_status decode_hash(gpl_ctx* ctx, const unsigned long long* part, gpl_result*
   std::vector<unsigned long long> rows;
   const unsigned long long* src = part + 2;
   if (li.limit == 0 && nrows) {
+    // every group: the full ORDER BY (else key order) as a device sort of the
+    // compacted rows (ORDER BY is blocking), then one D2H
+    const size_t tb = sort_hagg_tmp_bytes(nrows);
+    const size_t need = tb + ((size_t)nrows * W * 8 + 255) / 256 * 256;
+    if (ctx->sort_alloc < need) {
+      CK(cudaStreamSynchronize(ctx->stream));
+      if (ctx->d_sort) cudaFree(ctx->d_sort);
+      ctx->d_sort = nullptr;
+      ctx->sort_alloc = 0;
+      cudaError_t e = cudaMalloc(&ctx->d_sort, need);
+      if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("sort buffers: ") + cudaGetErrorString(e));
+      ctx->sort_alloc = need;
+    }
+    unsigned long long* sorted = (unsigned long long*)((char*)ctx->d_sort + tb);
+    CK(sort_hagg_rows(ctx->last.run->hres, ctx->last.run->hres.rows, nrows, sorted, ctx->d_sort, ctx->sms, ctx->stream));
     rows.resize((size_t)nrows * W);
-    CK(cudaMemcpyAsync(rows.data(), ctx->last.run->hres.rows, rows.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(rows.data(), sorted, rows.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
-    std::vector<size_t> ord(nrows);
-    for (size_t i = 0; i < nrows; i++) ord[i] = i;
-    auto field = [&](unsigned long long key, int k) {
-      return NK == 2 ? (int32_t)(uint32_t)(k == 0 ? key >> 32 : key) : (int32_t)(uint32_t)key;
-    };
-    std::sort(ord.begin(), ord.end(), [&](size_t a, size_t b) {
-      const unsigned long long ka = rows[a * W], kb = rows[b * W];
-      for (int k = 0; k < NK; k++)
-        if (field(ka, k) != field(kb, k)) return field(ka, k) < field(kb, k);
-      return false;
-    });
-    std::vector<unsigned long long> sorted(rows.size());
-    for (size_t i = 0; i < nrows; i++)
-      std::copy(rows.begin() + ord[i] * W, rows.begin() + (ord[i] + 1) * W, sorted.begin() + i * W);
-    rows.swap(sorted);
     src = rows.data();
   }
   for (uint64_t r = 0; r < nrows; r++) {
@@ -399,10 +399,12 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     if (ctx->h_err) cudaFreeHost(ctx->h_err);
     if (ctx->h_minmax) cudaFreeHost(ctx->h_minmax);
     if (ctx->d_minmax) cudaFree(ctx->d_minmax);
+    if (ctx->d_bounds) cudaFree(ctx->d_bounds);
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
     if (ctx->d_hagg) cudaFree(ctx->d_hagg);
     if (ctx->d_hres) cudaFree(ctx->d_hres);
     if (ctx->d_hcand) cudaFree(ctx->d_hcand);
+    if (ctx->d_sort) cudaFree(ctx->d_sort);
     if (ctx->side) cudaStreamDestroy(ctx->side);
     for (auto& e : ctx->fork_ev)
       if (e) cudaEventDestroy(e);
@@ -455,6 +457,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "drain_warps") {
     if (v >= 0 && v > 4) return fail(ctx, GPL_E_ARG, "drain_warps in [0, 4] (-1 = model)");
     o.drain_warps = v < 0 ? -1 : v;
+  } else if (k == "zone_restrict") {
+    o.zone_restrict = v != 0 ? 1 : 0;
   } else if (k == "agg_mode") {
     if (v >= 0 && v != AGG_GLOBAL) return fail(ctx, GPL_E_ARG, "agg_mode: 2 (global int128 atomics) or -1 (auto)");
     o.agg_mode = v < 0 ? -1 : v;

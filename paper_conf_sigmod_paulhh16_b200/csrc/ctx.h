@@ -188,6 +188,7 @@ struct Options {
   int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
   int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
   int64_t drain_warps = -1;    // operator-specialised drain warps (NEXT-1): -1 = the model's choice
+  int64_t zone_restrict = 1;   // scan only the row range of range filters on sorted columns
   int64_t agg_mode = -1;       // dense group accumulators: -1 exactness-driven choice, 2 = force global int128 atomics
 };
 
@@ -217,6 +218,7 @@ struct gpl_ctx {
   unsigned long long* d_scratch = nullptr;
   unsigned long long* d_partials = nullptr;
   size_t partials_cap = 0;
+  long long* d_bounds = nullptr;  // zone restriction: binary-search result (2 rows)
   long long* d_minmax = nullptr;  // [kMinmaxSlots][3] column slots of pending loads
   size_t minmax_cap = 0;
   std::vector<gpl::PendingLoad> pending;  // loads whose min/max are not read back yet
@@ -254,6 +256,8 @@ struct gpl_ctx {
   size_t hres_alloc = 0;
   unsigned long long* d_hcand = nullptr;
   size_t hcand_alloc = 0;
+  void* d_sort = nullptr;  // full device sort (ORDER BY without LIMIT): scratch + sorted rows
+  size_t sort_alloc = 0;
   std::map<std::string, std::pair<uint64_t, int64_t>> hagg_groups;  // plan text -> (distinct groups, fact rows) of its last run
   // A10 key decodes: table name -> (table version, key -> output value)
   std::map<std::string, std::pair<uint64_t, std::map<int32_t, int32_t>>> decode_maps;

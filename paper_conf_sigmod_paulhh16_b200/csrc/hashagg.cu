@@ -10,11 +10,18 @@
 //     selection over the CTAs' candidates and writes the k rows in order — to
 //     the device row buffer and to the run's result words, so the copy-out
 //     kernel brings them back with the counters (no extra D2H).
-//   * no LIMIT: every occupied slot is compacted into the row buffer (order
-//     arbitrary; the host orders by key).
+//   * no LIMIT: every occupied slot is compacted into the row buffer; the
+//     full ORDER BY (else key order) is then a device sort of the compacted
+//     rows at fetch (sort_hagg_rows: one stable LSD radix-sort pass per sort
+//     word, least significant word first, then a gather): a blocking full
+//     sort on the GPU, no host sort.
 // A row is [packed key, acc 0 .. nagg-1] (8-byte words). Ordering: the plan's
 // components (aggregate or key field, asc/desc), then the full key ascending,
 // so the first k rows are unique.
+#include <algorithm>
+
+#include <cub/cub.cuh>
+
 #include "kernels.h"
 #include "device_common.cuh"
 
@@ -318,7 +325,103 @@ __global__ void __launch_bounds__(kThreads) compact_groups(const __grid_constant
   }
 }
 
+// ---- full device sort of compacted rows (ORDER BY without LIMIT)
+
+// Sort word c of the rows in permutation order (the same words as words_of,
+// read from a compacted row [key, acc...] instead of a table slot).
+__global__ void __launch_bounds__(kThreads) sort_word_kernel(const __grid_constant__ HaggResultDesc D,
+                                                              const unsigned long long* rows, const unsigned* perm,
+                                                              unsigned long long n, int c, unsigned long long* out) {
+  const int W = 1 + D.nagg;
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned r = perm ? perm[i] : (unsigned)i;
+    const unsigned long long key = rows[(unsigned long long)r * W];
+    unsigned long long w;
+    if (c < D.norder) {
+      const long long v = D.ord_is_agg[c] ? (long long)rows[(unsigned long long)r * W + 1 + D.ord_idx[c]]
+                                          : (long long)key_field(key, D.nkeys, D.ord_idx[c]);
+      const unsigned long long u = (unsigned long long)v ^ kSign;
+      w = D.ord_desc[c] ? ~u : u;
+    } else if (D.nkeys == 2) {
+      w = ((unsigned long long)((unsigned)key_field(key, 2, 0) ^ 0x80000000u) << 32) |
+          (unsigned long long)((unsigned)key_field(key, 2, 1) ^ 0x80000000u);
+    } else {
+      w = (unsigned long long)(long long)key_field(key, 1, 0) ^ kSign;
+    }
+    out[i] = w;
+  }
+}
+
+__global__ void __launch_bounds__(kThreads) iota_kernel(unsigned* p, unsigned long long n) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    p[i] = (unsigned)i;
+}
+
+__global__ void __launch_bounds__(kThreads) gather_rows_kernel(const unsigned long long* rows, const unsigned* perm,
+                                                                unsigned long long n, int W, unsigned long long* out) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n * (unsigned long long)W;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const unsigned long long r = i / (unsigned long long)W, w = i % (unsigned long long)W;
+    out[i] = rows[(unsigned long long)perm[r] * W + w];
+  }
+}
+
+struct SortTmp {
+  unsigned long long *ka, *kb;
+  unsigned *pa, *pb;
+  void* cub;
+  size_t cub_bytes;
+};
+
+SortTmp carve(void* tmp, unsigned long long n) {
+  SortTmp t;
+  char* p = (char*)tmp;
+  auto take = [&](size_t b) {
+    char* q = p;
+    p += (b + 255) / 256 * 256;
+    return q;
+  };
+  t.ka = (unsigned long long*)take(n * 8);
+  t.kb = (unsigned long long*)take(n * 8);
+  t.pa = (unsigned*)take(n * 4);
+  t.pb = (unsigned*)take(n * 4);
+  t.cub_bytes = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, t.cub_bytes, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
+                                  (unsigned*)nullptr, (unsigned*)nullptr, (int)n);
+  t.cub = take(t.cub_bytes);
+  return t;
+}
+
 }  // namespace
+
+size_t sort_hagg_tmp_bytes(unsigned long long n) {
+  auto r = [](size_t b) { return (b + 255) / 256 * 256; };
+  size_t cb = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, cb, (unsigned long long*)nullptr, (unsigned long long*)nullptr,
+                                  (unsigned*)nullptr, (unsigned*)nullptr, (int)n);
+  return 2 * r(n * 8) + 2 * r(n * 4) + r(cb);
+}
+
+cudaError_t sort_hagg_rows(const HaggResultDesc& D, const unsigned long long* rows, unsigned long long n,
+                           unsigned long long* out, void* tmp, int num_sms, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  SortTmp t = carve(tmp, n);
+  const int grid = (int)std::min<unsigned long long>((n + kThreads - 1) / kThreads, (unsigned long long)num_sms * 8);
+  iota_kernel<<<grid, kThreads, 0, s>>>(t.pa, n);
+  // least significant word first: the full key, then the ORDER BY components from last to first;
+  // each pass is a stable radix sort of (word, row) pairs
+  for (int c = D.norder; c >= 0; c--) {
+    sort_word_kernel<<<grid, kThreads, 0, s>>>(D, rows, t.pa, n, c, t.ka);
+    size_t cb = t.cub_bytes;
+    cudaError_t e = cub::DeviceRadixSort::SortPairs(t.cub, cb, t.ka, t.kb, t.pa, t.pb, (int)n, 0, 64, s);
+    if (e != cudaSuccess) return e;
+    std::swap(t.pa, t.pb);
+  }
+  gather_rows_kernel<<<grid, kThreads, 0, s>>>(rows, t.pa, n, 1 + D.nagg, out);
+  return cudaGetLastError();
+}
 
 int hagg_select_blocks(unsigned long long nslots, int num_sms) {
   // one slice per CTA, >= 1K slots each, at most 2 CTAs per SM

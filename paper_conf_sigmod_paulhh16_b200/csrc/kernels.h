@@ -40,6 +40,12 @@ bool jit_prepare(const PipeDesc& d, bool load, std::string* err);
 // > 0; D.nblocks = hagg_select_blocks(...) CTAs, D.cand sized nblocks*limit*5 words)
 // or compaction of every group. Plain stream order after the fused run.
 int hagg_select_blocks(unsigned long long nslots, int num_sms);
+// Full device sort of n compacted rows (ORDER BY without LIMIT, else key
+// order) into `out`: stable LSD radix passes over the sort words + a gather.
+// tmp: sort_hagg_tmp_bytes(n) bytes.
+size_t sort_hagg_tmp_bytes(unsigned long long n);
+cudaError_t sort_hagg_rows(const HaggResultDesc& D, const unsigned long long* rows, unsigned long long n,
+                           unsigned long long* out, void* tmp, int num_sms, cudaStream_t s);
 cudaError_t launch_hagg_result(const HaggResultDesc& D, const unsigned long long* hagg_count, int num_sms,
                                cudaStream_t s);
 
@@ -58,6 +64,9 @@ cudaError_t launch_copyout(const unsigned long long* src, unsigned long long* ho
 // Column min/max (int32 or int64 column, n rows) -> out[0] = min, out[1] = max.
 // out[2] = number of descents (rows i with v[i] > v[i+1]): 0 means sorted.
 cudaError_t launch_minmax(const void* col, int width, long long n, long long* out, cudaStream_t s);
+// [lower_bound(lo), upper_bound(hi)) of a sorted column (one thread; out[2] device)
+cudaError_t launch_sorted_bounds(const void* col, int w, long long n, long long lo, long long hi, long long* out,
+                                 cudaStream_t s);
 // device scan scratch of a MULTI (fan-out) build over nslots keys
 size_t multi_scan_tmp_bytes(unsigned long long nslots);
 // per-column {min, max, descents} of one table's columns in two launches (A0 load)

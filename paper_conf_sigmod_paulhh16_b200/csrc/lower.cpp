@@ -2,6 +2,8 @@
 // device descriptors (BuildDesc / PipeDesc). Host only.
 #include "lower.h"
 
+#include "kernels.h"
+
 #include <algorithm>
 #include <cmath>
 #include <map>
@@ -18,6 +20,50 @@ struct Range {
 Range mul(Range a, Range b) {
   long double c[4] = {a.lo * b.lo, a.lo * b.hi, a.hi * b.lo, a.hi * b.hi};
   return {*std::min_element(c, c + 4), *std::max_element(c, c + 4)};
+}
+
+// Zone restriction (SURVEY §7 "zone maps for build scans"): a range filter on
+// a column that is sorted (non-decreasing, recorded at load: partsupp by
+// ps_partkey, part by p_partkey, orders by o_orderkey, lineitem by l_orderkey)
+// selects one contiguous row range, so only that range is scanned. The bounds
+// are two binary searches (device, one small synchronous read-back at plan
+// preparation; host-only contexts search their host copy). Filters still run
+// on every scanned row, so the result does not depend on the restriction.
+gpl_status sorted_range(gpl_ctx* ctx, const Table& T, const std::vector<FilterIR>& filters, int64_t* r0, int64_t* r1,
+                        std::string* err) {
+  *r0 = 0;
+  *r1 = T.nrows;
+  if (ctx->opt.zone_restrict == 0) return GPL_OK;
+  for (const FilterIR& F : filters) {
+    const Column* c = T.find(F.col);
+    if (!c || !c->sorted || F.kind != F_RANGE || T.nrows == 0) continue;
+    if (F.lo <= c->vmin && F.hi >= c->vmax) continue;  // passes every row
+    long long b[2] = {0, T.nrows};
+    if (ctx->host_only) {
+      auto v = [&](int64_t i) {
+        return c->width == 4 ? (long long)((const int32_t*)c->host.data())[i] : ((const int64_t*)c->host.data())[i];
+      };
+      int64_t a = 0, e = T.nrows;
+      while (a < e) { const int64_t m = (a + e) / 2; if (v(m) < F.lo) a = m + 1; else e = m; }
+      b[0] = a;
+      e = T.nrows;
+      while (a < e) { const int64_t m = (a + e) / 2; if (v(m) <= F.hi) a = m + 1; else e = m; }
+      b[1] = a;
+    } else {
+      if (!ctx->d_bounds) {
+        if (cudaMalloc(&ctx->d_bounds, 16) != cudaSuccess) { *err = "bounds scratch"; return GPL_E_NOMEM; }
+      }
+      cudaError_t e = launch_sorted_bounds(c->dev, c->width, T.nrows, F.lo, F.hi, ctx->d_bounds, ctx->stream);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(b, ctx->d_bounds, 16, cudaMemcpyDeviceToHost, ctx->stream);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+      if (e != cudaSuccess) { *err = std::string("zone bounds: ") + cudaGetErrorString(e); return GPL_E_CUDA; }
+    }
+    *r0 = std::max<int64_t>(*r0, b[0]);
+    *r1 = std::min<int64_t>(*r1, b[1]);
+  }
+  *r0 &= ~(int64_t)3;  // 4-row aligned: 16-B aligned TMA sources for every column width
+  if (*r1 < *r0) *r1 = *r0;
+  return GPL_OK;
 }
 
 }  // namespace
@@ -202,6 +248,12 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
     d->colw[c] = cols[c]->width;
   }
   d->nrows = T.nrows;
+  {  // scan only the row range the sorted filter columns allow
+    int64_t r0, r1;
+    if ((st = sorted_range(ctx, T, s.filters, &r0, &r1, err))) return st;
+    for (int c = 0; c < d->ncols; c++) d->col[c] += r0 * d->colw[c];
+    d->nrows = r1 - r0;
+  }
   d->kind = shape->kind;
   d->hash = shape->hash;
   d->load_pct = load;
@@ -736,6 +788,12 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   li->bytes_per_row = bpr;
   li->bytes_per_row_all = bpr_all;
   d->nrows = T.nrows;
+  {  // scan only the row range the sorted filter columns allow (zone restriction)
+    int64_t r0, r1;
+    if ((st = sorted_range(ctx, T, s.filters, &r0, &r1, err))) return st;
+    for (int c = 0; c < d->ncols; c++) d->col[c] += r0 * d->colw[c];
+    d->nrows = r1 - r0;
+  }
   li->nfilt = d->nfilt;
   li->nprobe = np;
   li->nops = d->nfilt + np + d->nresid;

@@ -718,3 +718,23 @@ def test_qf_schedules_drains_and_kbe_rejects(ctx):
     with pytest.raises(gpl.GplError) as e:
         queries.run_query(ctx, "QF", db, params, kbe=True)
     assert e.value.status == gpl.GPL_E_PLAN
+
+
+def test_q3_full_device_sort_order_by_without_limit(ctx):
+    """NEXT-4 full GPU sort: Q3's ORDER BY revenue desc, o_orderdate (ties: key) WITHOUT the
+    LIMIT returns every group in that order, sorted on the device (radix passes over the sort words);
+    without 'order' the rows come back in key order."""
+    db = tpchgen.generate(0.3, seed=6)
+    queries.load_database(ctx, db, queries.TABLES["Q3"])
+    o = oracle.run("Q3", db)
+    want = sorted(zip(o.keys, o.aggs), key=lambda ka: (-ka[1][1], ka[0][1], ka[0]))
+    text = "\n".join(ln for ln in queries.plan_text("Q3", db).splitlines() if not ln.startswith("limit"))
+    for attempt in range(3):  # a table sized from another run may overflow once (latched, then re-sized)
+        ctx.run_query(text)
+        try:
+            r = ctx.fetch_result()
+            break
+        except gpl.GplError as e:
+            assert e.status == gpl.GPL_E_CAPACITY and attempt < 2
+    assert len(r.keys) == len(o.keys) > 1000
+    assert list(zip(r.keys, r.aggs)) == want
