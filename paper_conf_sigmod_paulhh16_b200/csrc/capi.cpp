@@ -457,6 +457,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "drain_warps") {
     if (v >= 0 && v > 4) return fail(ctx, GPL_E_ARG, "drain_warps in [0, 4] (-1 = model)");
     o.drain_warps = v < 0 ? -1 : v;
+  } else if (k == "reg_fields") {
+    o.reg_fields = v != 0 ? 1 : 0;
   } else if (k == "zone_restrict") {
     o.zone_restrict = v != 0 ? 1 : 0;
   } else if (k == "agg_mode") {

@@ -167,11 +167,17 @@ struct PipeDesc {
   int32_t qw[MAXQ];      // field width in bytes (4 or 8)
   int32_t qbytes;        // bytes of one warp's queue
   int32_t qlazy[MAXQ];   // >= 0: field f is lazy column qlazy[f], gathered by the drain via the row id
+  int32_t qlazy_at[MAXQ];  // lazy field f is gathered right before queue probe qlazy_at[f] (nprobe: before
+                           // the group-by / value / sink), only for the rows still alive there
+  // 1: fields the drain produces (f >= npush: lazy gathers, queue-probe slots) live in registers of the
+  // plan-specialised kernel; the warp queues hold only the pushed fields (0: every field in the queue)
+  int32_t reg_fields, reg_pad;
   // clustered probe: stage probe cl_probe reads a DIRECT table by a key column
   // (cl_col) sorted in the fact table, so one stage's keys span a narrow cell
   // range; the producer TMA-stages those cells (<= cl_cap bytes at slot offset
   // cl_off) beside the columns and the probe reads shared memory
   int32_t cl_probe, cl_col, cl_off, cl_cap;
+  int32_t cl_kpr, cl_pad;  // clustered probe: staged keys per stage row (cell buffer = cl_kpr x stage rows)
   int32_t rowid_field;   // queue field holding the row id (-1: no lazy column)
   // fan-out probe (NEXT-4): queue-phase probe into a MULTI table; every match
   // of a row continues through the remaining operators (-1: none)

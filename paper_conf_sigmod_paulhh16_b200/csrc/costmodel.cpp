@@ -46,12 +46,13 @@ int align128(int x) { return (x + 127) & ~127; }
 }  // namespace
 
 // Cell buffer of a clustered probe per ring slot: a stage's key range spans
-// up to 4 keys per row (TPC-H order keys are 1 in 4 dense; a wider range
-// falls back to probing the table in memory).
+// cl_kpr keys per row (twice the column's average, set by the lowering; a
+// wider range falls back to probing the table in memory).
 int cl_cap_bytes(const PipeDesc& d, int S) {
   if (d.cl_probe < 0) return 0;
   const int w = d.ht[d.probe[d.cl_probe].ht].width;
-  return align128((w == 0 ? (4 * S + 7) / 8 : 4 * S * w) + 32);
+  const int kpr = d.cl_kpr > 0 ? d.cl_kpr : 4;
+  return align128((w == 0 ? (kpr * S + 7) / 8 : kpr * S * w) + 32);
 }
 
 int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps, int ndrain) {
@@ -234,7 +235,7 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
                    Config* out, std::string* err, std::vector<Config>* shortlist) {
   std::map<std::tuple<int, int, int>, Config> per_shape;  // best predicted per (CTAs/SM, stage rows, packets)
   const Options& o = ctx->opt;
-  std::vector<int> Ss = o.stage_rows > 0 ? std::vector<int>{(int)o.stage_rows} : std::vector<int>{512, 1024, 2048, 4096};
+  std::vector<int> Ss = o.stage_rows > 0 ? std::vector<int>{(int)o.stage_rows} : std::vector<int>{512, 1024, 2048, 4096, 8192};
   std::vector<int> Ds = o.ring_depth > 0 ? std::vector<int>{(int)o.ring_depth} : std::vector<int>{2, 3, 4, 6};
   std::vector<int> Ws = o.consumer_warps > 0 ? std::vector<int>{(int)o.consumer_warps} : std::vector<int>{4, 8, 12, 16};
   std::vector<int> Ks = o.ctas_per_sm > 0 ? std::vector<int>{(int)o.ctas_per_sm} : std::vector<int>{1, 2};

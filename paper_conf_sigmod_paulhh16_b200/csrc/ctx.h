@@ -188,6 +188,7 @@ struct Options {
   int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
   int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
   int64_t drain_warps = -1;    // operator-specialised drain warps (NEXT-1): -1 = the model's choice
+  int64_t reg_fields = 1;      // JIT kernels keep drain-produced queue fields in registers
   int64_t zone_restrict = 1;   // scan only the row range of range filters on sorted columns
   int64_t agg_mode = -1;       // dense group accumulators: -1 exactness-driven choice, 2 = force global int128 atomics
 };

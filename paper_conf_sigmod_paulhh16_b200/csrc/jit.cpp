@@ -133,7 +133,9 @@ std::string shape_source(const PipeDesc& d) {
   I("cl_off", d.cl_off);
   I("cl_cap", d.cl_cap);
   I("fan_probe", d.fan_probe);
-  for (int f = 0; f < MAXQ; f++) o << "  k.qlazy[" << f << "] = " << d.qlazy[f] << ";\n";
+  for (int f = 0; f < MAXQ; f++)
+    o << "  k.qlazy[" << f << "] = " << d.qlazy[f] << "; k.qlazy_at[" << f << "] = " << d.qlazy_at[f] << ";\n";
+  I("reg_fields", d.reg_fields);
   auto term = [&](const char* arr, int t, const Term& T) {
     o << "  k." << arr << "[" << t << "].sign = " << T.sign << "; k." << arr << "[" << t << "].nfact = " << T.nfact << ";\n";
     for (int f = 0; f < T.nfact; f++)
@@ -246,6 +248,8 @@ bool compile(const std::string& src, std::vector<char>* cubin, std::string* err)
 }
 
 }  // namespace
+
+bool jit_available() { return nvrtc().ok; }
 
 bool jit_prepare(const PipeDesc& d, bool load, std::string* err) {
   const std::string key = shape_source(d);

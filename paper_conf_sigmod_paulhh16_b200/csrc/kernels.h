@@ -35,6 +35,8 @@ cudaError_t launch_pipeline_fn(const void* fn, const PipeDesc& d, int grid, cuda
 // JIT: compile (and, when load is true, load) the specialised kernel for d's
 // shape. Returns false with a message when NVRTC is unavailable or fails.
 bool jit_prepare(const PipeDesc& d, bool load, std::string* err);
+// NVRTC can be loaded (plan-specialised kernels are possible)
+bool jit_available();
 
 // Hash group-by result step (hashagg.cu): ORDER BY/LIMIT selection (D.limit
 // > 0; D.nblocks = hagg_select_blocks(...) CTAs, D.cand sized nblocks*limit*5 words)

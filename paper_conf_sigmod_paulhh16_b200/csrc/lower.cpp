@@ -421,6 +421,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   // rows) * 64 <= width, from the previous run's pass fractions λ. In auto mode
   // a stage-phase probe whose key column qualifies moves to the queue phase.
   std::set<std::string> lazy;
+  std::map<std::string, int> lazy_at;  // lazy column -> queue probe it is gathered before (np: the tail)
   const int nf0 = (int)s.filters.size();
   if (!ins && ctx->opt.lazy_columns != 0 && T.nrows < (1ll << 31)) {
     auto lit = ctx->lambda.find(s.text);
@@ -447,19 +448,32 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     for (auto& f : s.filters) stage_cols.insert(f.col);
     for (int p = 0; p < sp; p++)
       for (auto& k : s.probes[p].keys) stage_cols.insert(k);
-    const int qop = nf0 + sp - 1;  // the rows reaching the queue passed this op
-    auto consider = [&](const std::string& c) {
-      if (!slot_of.count(c) && !stage_cols.count(c) && worthy(c, qop)) lazy.insert(c);
+    // a lazy column is gathered right before its first use in the queue phase
+    // (a queue probe's key, else the group-by / value after every probe and
+    // residual), for the rows alive there: its cost is one sector per row
+    // reaching that point (the pass count of the op before it)
+    const int nops_all = nf0 + np + (int)s.wheres.size();
+    auto reach_op = [&](int at) { return at < np ? nf0 + at - 1 : nops_all - 1; };
+    std::map<std::string, int> first_use;  // queue-phase column -> its first use point
+    auto use = [&](const std::string& c, int at) {
+      if (slot_of.count(c) || stage_cols.count(c)) return;
+      auto it = first_use.find(c);
+      if (it == first_use.end() || at < it->second) first_use[c] = at;
     };
     for (int p = sp; p < np; p++)
-      for (auto& k : s.probes[p].keys) consider(k);
-    for (auto& g : s.groups) consider(g.ref.name);
+      for (auto& k : s.probes[p].keys) use(k, p);
+    for (auto& g : s.groups) use(g.ref.name, np);
     for (auto& t : s.value)
       for (auto& f : t.f)
-        if (f.x.kind != RefIR::CONST) consider(f.x.name);
+        if (f.x.kind != RefIR::CONST) use(f.x.name, np);
+    for (auto& [c, at] : first_use)
+      if (worthy(c, reach_op(at))) {
+        lazy.insert(c);
+        lazy_at[c] = at;
+      }
     for (auto& c : lazy) {
       li->lazy_w.push_back(cols[cidx[c]]->width);
-      li->lazy_reach.push_back(qop);
+      li->lazy_reach.push_back(reach_op(lazy_at[c]));
     }
   }
 
@@ -519,7 +533,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   std::map<std::string, int> field;
   std::vector<int> fw;
   int nf = 0;
-  for (int f = 0; f < MAXQ; f++) d->qlazy[f] = -1;
+  for (int f = 0; f < MAXQ; f++) d->qlazy[f] = -1, d->qlazy_at[f] = np;
   d->rowid_field = -1;
   for (auto& c : qcols) {
     if (lazy.count(c)) continue;
@@ -556,6 +570,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     if (!lazy.count(c)) continue;
     if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
     d->qlazy[nf] = cidx[c];
+    d->qlazy_at[nf] = lazy_at.count(c) ? lazy_at[c] : np;
     fw.push_back(cols[cidx[c]]->width);
     field[c] = nf++;
   }
@@ -569,12 +584,16 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   }
   if (nf > MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
   d->nfield = std::max(nf, 1);
+  // the plan-specialised kernel keeps the fields the drain produces in
+  // registers; only the pushed fields need warp-queue space (shared memory
+  // then goes to a deeper ring / more CTAs per SM)
+  d->reg_fields = ctx->opt.jit != 0 && ctx->opt.reg_fields != 0 && jit_available() ? 1 : 0;
   {
     int off = 0;
     for (int f = 0; f < nf; f++) {
       d->qoff[f] = off;
       d->qw[f] = fw[f];
-      off += fw[f] * QCAP;
+      if (!d->reg_fields || f < d->npush) off += fw[f] * QCAP;
     }
     d->qbytes = std::max(off, 16);
   }
@@ -646,6 +665,12 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
         d->ht_smem_off[P0.ht] < 0 && H0.bytes() < (1ull << 31)) {
       d->cl_probe = 0;
       d->cl_col = P0.k1;
+      // cell buffer per slot: twice the column's average key span per row
+      // (lineitem: ~1 order key per row), 1..4 keys per row; a stage whose
+      // range is wider probes the table in memory instead (correct, slower)
+      const Column& kc = *cols[P0.k1];
+      const double kpr = T.nrows > 0 ? (double)(kc.vmax - kc.vmin + 1) / (double)T.nrows : 1.0;
+      d->cl_kpr = (int)std::min(4.0, std::max(1.0, std::ceil(2.0 * kpr)));
       li->cl_bytes = (double)H0.bytes();  // the producer streams the table's cells once (bytes per launch)
     }
   }

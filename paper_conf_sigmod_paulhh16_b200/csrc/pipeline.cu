@@ -76,6 +76,8 @@ const void* resolve_pipeline_fn(const PipeDesc& d, bool use_jit, std::string* ji
     return nullptr;
   const void* fn = nullptr;
   if (use_jit) fn = jit_pipeline_kernel(d, jit_err);
+  // a register-field layout exists only in the plan-specialised kernel: no generic fallback
+  if (!fn && d.reg_fields) return nullptr;
   if (!fn) {
     static int configured = 0;
     fn = (const void*)pipeline_kernel;

@@ -237,36 +237,34 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int 
 }
 
 // Clustered probe (DIRECT table, key column sorted in the fact table): the
-// producer staged the cells of the stage's key range [klo, khi] at smem byte
-// `base`, starting at table byte `start`; a key outside the staged bytes (only
-// possible if the column is not sorted after all) reads the table in HBM.
+// producer staged the cells of the stage's key range at smem byte `base`; they
+// cover keys [k0, k0 + ncells). The column is sorted (checked at load), so
+// every key of the stage lies in the staged range or outside the table's
+// domain: one 32-bit subtract + compare + predicated LDS per row, no 64-bit
+// index math and no global fallback (a stage whose range did not fit the slot
+// probes the table in memory instead, see the caller).
 template <int N>
 __device__ __forceinline__ void probe_rows_cl(const PipeDesc& K, const HTP& h, int t, const unsigned long long (&key)[N],
                                               const bool (&act)[N], bool (&hit)[N], long long (&pay)[N], uint32_t base,
-                                              long long start, int size) {
+                                              uint32_t k0, uint32_t ncells) {
   const int width = K.ht[t].width;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(g_smem) + base;
+  uint32_t x[N];
 #pragma unroll
   for (int j = 0; j < N; j++) {
-    const unsigned long long idx = (unsigned long long)((long long)(int32_t)(uint32_t)key[j] - (long long)h.kmin);
-    const bool in = act[j] && idx < h.nslots;
-    const long long b = (width == 0 ? (long long)(idx >> 5) * 4 : (long long)idx * width) - start;
-    const bool staged = b >= 0 && b < size;
-    uint32_t x = 0;
-    if (in) {
-      if (width == 0) {
-        const uint32_t wd = staged ? lds_u32(sbase + (uint32_t)b) : __ldg((const uint32_t*)h.slots + (idx >> 5));
-        x = (wd >> (idx & 31)) & 1u;
-      } else if (width == 1) {
-        x = staged ? lds_u8(sbase + (uint32_t)b) : (uint32_t)__ldg((const unsigned char*)h.slots + idx);
-      } else if (width == 2) {
-        x = staged ? lds_u16(sbase + (uint32_t)b) : (uint32_t)__ldg((const unsigned short*)h.slots + idx);
-      } else {
-        x = staged ? lds_u32(sbase + (uint32_t)b) : __ldg((const uint32_t*)h.slots + idx);
-      }
-    }
-    hit[j] = x != 0;
-    pay[j] = width == 0 ? 1 : (long long)x - 1 + h.pay_base;
+    const uint32_t o = (uint32_t)key[j] - k0;
+    const bool in = act[j] && o < ncells;
+    uint32_t v = 0;
+    if (width == 0) v = in ? (lds_u32(sbase + (o >> 5) * 4) >> (o & 31)) & 1u : 0u;
+    else if (width == 1) v = in ? lds_u8(sbase + o) : 0u;
+    else if (width == 2) v = in ? lds_u16(sbase + o * 2) : 0u;
+    else v = in ? lds_u32(sbase + o * 4) : 0u;
+    x[j] = v;
+  }
+#pragma unroll
+  for (int j = 0; j < N; j++) {
+    hit[j] = x[j] != 0;
+    pay[j] = width == 0 ? 1 : (long long)x[j] - 1 + h.pay_base;
   }
 }
 
@@ -364,182 +362,202 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
     idx[j] = (qhead + e) & (QCAP - 1);
     p[j] = e < n;
   }
-  if (K.rowid_field >= 0) {
-    // late materialisation: gather the lazy columns of the queued rows (all
-    // loads of a lane in flight together: one HBM round trip per drain)
-    uint32_t row[RPL];
-#pragma unroll
-    for (int j = 0; j < RPL; j++) row[j] = (uint32_t)qget(K, qb, K.rowid_field, idx[j]);
+  // Field access. Pushed fields (f < npush) live in the warp queue; the fields
+  // the drain produces itself (lazy gathers, queue-probe slots) live in
+  // registers of the plan-specialised kernel (reg_fields: f is a compile-time
+  // constant there), else in the queue as well.
+#ifdef GPL_JIT
+  long long dv[MAXQ][RPL];
+#define GPL_REGF(f) (K.reg_fields && (f) >= K.npush)
+  auto fget = [&](int f, int j) -> long long { return GPL_REGF(f) ? dv[f][j] : qget(K, qb, f, idx[j]); };
+  auto fput = [&](int f, int j, long long v) {
+    if (GPL_REGF(f)) dv[f][j] = v;
+    else qput(K, qb, f, idx[j], v);
+  };
+#undef GPL_REGF
+#else
+  auto fget = [&](int f, int j) -> long long { return qget(K, qb, f, idx[j]); };
+  auto fput = [&](int f, int j, long long v) { qput(K, qb, f, idx[j], v); };
+#endif
+  // late materialisation: a lazy column is gathered right before its first
+  // use (queue probe `at`, or nprobe = the group-by / value), for the rows
+  // still alive there; all loads of a lane in flight together
+  auto gather = [&](int at, const bool (&p)[RPL]) {
+    if (K.rowid_field < 0) return;
     GPL_UNROLL
     for (int f = 0; f < K.nfield; f++) {
       const int c = K.qlazy[f];
-      if (c < 0) continue;
+      if (c < 0 || K.qlazy_at[f] != at) continue;
       long long v[RPL];
-#pragma unroll
-      for (int j = 0; j < RPL; j++) v[j] = p[j] ? ld_col_global(d.col[c], K.colw[c], (long long)row[j]) : 0;
 #pragma unroll
       for (int j = 0; j < RPL; j++)
-        if (p[j]) qput(K, qb, f, idx[j], v[j]);
+        v[j] = p[j] ? ld_col_global(d.col[c], K.colw[c], (long long)(uint32_t)fget(K.rowid_field, j)) : 0;
+#pragma unroll
+      for (int j = 0; j < RPL; j++)
+        if (p[j]) fput(f, j, v[j]);
     }
-  }
+  };
   auto run_probes = [&](int lo, int hi, bool (&p)[RPL]) {
-  GPL_UNROLL
-  for (int pi = lo; pi < hi; pi++) {
-    const int op = K.nfilt + pi;
-    const Probe& P = K.probe[pi];
-    if (__any_sync(0xffffffffu, any4(p))) {
-      unsigned long long k[RPL];
+    GPL_UNROLL
+    for (int pi = lo; pi < hi; pi++) {
+      const int op = K.nfilt + pi;
+      const Probe& P = K.probe[pi];
+      if (__any_sync(0xffffffffu, any4(p))) {
+        gather(pi, p);
+        unsigned long long k[RPL];
 #pragma unroll
-      for (int j = 0; j < RPL; j++) {
-        k[j] = (uint32_t)qget(K, qb, P.k1, idx[j]);
-        if (P.k2 >= 0) k[j] = (k[j] << 32) | (uint32_t)qget(K, qb, P.k2, idx[j]);
-      }
-      bool hit[RPL];
-      long long v[RPL];
-      probe_rows<RPL>(K, htp[P.ht], P.ht, k, p, hit, v);
+        for (int j = 0; j < RPL; j++) {
+          k[j] = (uint32_t)fget(P.k1, j);
+          if (P.k2 >= 0) k[j] = (k[j] << 32) | (uint32_t)fget(P.k2, j);
+        }
+        bool hit[RPL];
+        long long v[RPL];
+        probe_rows<RPL>(K, htp[P.ht], P.ht, k, p, hit, v);
 #pragma unroll
-      for (int j = 0; j < RPL; j++) {
-        if (P.kind == P_MARK) {
-          if (p[j] && P.out >= 0) qput(K, qb, P.out, idx[j], hit[j] ? 1 : 0);
-        } else {
-          if (hit[j] && P.out >= 0) qput(K, qb, P.out, idx[j], v[j]);
-          p[j] = hit[j];
+        for (int j = 0; j < RPL; j++) {
+          if (P.kind == P_MARK) {
+            if (p[j] && P.out >= 0) fput(P.out, j, hit[j] ? 1 : 0);
+          } else {
+            if (hit[j] && P.out >= 0) fput(P.out, j, v[j]);
+            p[j] = hit[j];
+          }
         }
       }
+      const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+      if (lane == 0) cnt[op] += c;
     }
-    const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
-    if (lane == 0) cnt[op] += c;
-  }
   };
+  // residuals, the remaining lazy gathers, then the sink (insert or aggregate)
   auto tail = [&](bool (&p)[RPL]) {
-  GPL_UNROLL
-  for (int r = 0; r < K.nresid; r++) {
-    const int op = K.nfilt + K.nprobe + r;
-    const Resid& R = K.resid[r];
+    GPL_UNROLL
+    for (int r = 0; r < K.nresid; r++) {
+      const int op = K.nfilt + K.nprobe + r;
+      const Resid& R = K.resid[r];
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
+        if (!p[j]) continue;
+        const long long a = fget(R.a, j);
+        if (R.kind == R_EQ) {
+          p[j] = a == fget(R.b, j);
+        } else if (R.kind == R_PAIRS) {
+          const long long b = fget(R.b, j);
+          bool ok = false;
+          GPL_UNROLL
+          for (int i = 0; i < R.npairs; i++) ok |= (a == R.pa[i]) & (b == R.pb[i]);
+          p[j] = ok;
+        } else if (R.kind == R_RANGE) {
+          p[j] = a >= R.lo && a <= R.hi;
+        } else {
+          p[j] = (unsigned long long)a < 64ull && ((R.mask >> a) & 1ull);
+        }
+      }
+      const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
+      if (lane == 0) cnt[op] += c;
+    }
+    if (!__any_sync(0xffffffffu, any4(p))) return;
+    gather(K.nprobe, p);
+    if (K.sink == SINK_INSERT) {
+      long long kx[RPL], px[RPL];
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
+        kx[j] = fget(K.ins_kfield, j);
+        px[j] = K.ins_pfield >= 0 ? fget(K.ins_pfield, j) : 0;
+      }
+      insert_cells<RPL>(d, K, kx, px, p);
+      return;
+    }
+    unsigned long long* stab = &S<unsigned long long>(K.off_agg);
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
       if (!p[j]) continue;
-      const long long a = qget(K, qb, R.a, idx[j]);
-      if (R.kind == R_EQ) {
-        p[j] = a == qget(K, qb, R.b, idx[j]);
-      } else if (R.kind == R_PAIRS) {
-        const long long b = qget(K, qb, R.b, idx[j]);
-        bool ok = false;
+      long long hslot = -1;  // AGG_HASH: the group's slot
+      if (K.agg_mode == AGG_HASH) {
+        // hash group-by over unbounded keys (NEXT-4): the packed key finds or
+        // claims its slot (open addressing, linear probing); slots hold ~key
+        unsigned long long key = 0;
         GPL_UNROLL
-        for (int i = 0; i < R.npairs; i++) ok |= (a == R.pa[i]) & (b == R.pb[i]);
-        p[j] = ok;
-      } else if (R.kind == R_RANGE) {
-        p[j] = a >= R.lo && a <= R.hi;
-      } else {
-        p[j] = (unsigned long long)a < 64ull && ((R.mask >> a) & 1ull);
-      }
-    }
-    const unsigned c = __reduce_add_sync(0xffffffffu, count4(p));
-    if (lane == 0) cnt[op] += c;
-  }
-  if (!__any_sync(0xffffffffu, any4(p))) return;
-  if (K.sink == SINK_INSERT) {
-    long long kx[RPL], px[RPL];
-#pragma unroll
-    for (int j = 0; j < RPL; j++) {
-      kx[j] = qget(K, qb, K.ins_kfield, idx[j]);
-      px[j] = K.ins_pfield >= 0 ? qget(K, qb, K.ins_pfield, idx[j]) : 0;
-    }
-    insert_cells<RPL>(d, K, kx, px, p);
-    return;
-  }
-  unsigned long long* stab = &S<unsigned long long>(K.off_agg);
-#pragma unroll
-  for (int j = 0; j < RPL; j++) {
-    if (!p[j]) continue;
-    long long hslot = -1;  // AGG_HASH: the group's slot
-    if (K.agg_mode == AGG_HASH) {
-      // hash group-by over unbounded keys (NEXT-4): the packed key finds or
-      // claims its slot (open addressing, linear probing); slots hold ~key
-      unsigned long long key = 0;
-      GPL_UNROLL
-      for (int g = 0; g < K.ngroup; g++) {
-        long long v = qget(K, qb, K.gdim[g].field, idx[j]);
-        if (K.gdim[g].transform == G_YEAR) v = (int)v / 10000;
-        key = (key << 32) | (unsigned long long)(unsigned)v;
-      }
-      if (key == ~0ull) {
-        atomicOr(d.err, ERR_RESERVED_KEY);
-        continue;
-      }
-      const unsigned long long st = ~key, mask = (1ull << d.hagg_log2) - 1ull;
-      // an overfull table stops early instead of walking every slot: no new
-      // group is claimed past 7/8 load, and a probe gives up after 2^14
-      // steps; both latch ERR_CAPACITY and the host re-runs with a larger table
-      const unsigned long long fill_limit = mask + 1ull - ((mask + 1ull) >> 3);
-      const unsigned long long max_steps = mask < 16383ull ? mask : 16383ull;
-      unsigned long long h = (key * 0x9E3779B97F4A7C15ull) >> (64 - d.hagg_log2);
-      for (unsigned long long step = 0; step <= max_steps; step++, h = (h + 1) & mask) {
-        unsigned long long cur = __ldcg(d.hagg_keys + h);
-        if (cur == 0ull) {
-          if (__ldcg(d.hagg_count) >= fill_limit) break;
-          cur = atomicCAS(d.hagg_keys + h, 0ull, st);
+        for (int g = 0; g < K.ngroup; g++) {
+          long long v = fget(K.gdim[g].field, j);
+          if (K.gdim[g].transform == G_YEAR) v = (int)v / 10000;
+          key = (key << 32) | (unsigned long long)(unsigned)v;
+        }
+        if (key == ~0ull) {
+          atomicOr(d.err, ERR_RESERVED_KEY);
+          continue;
+        }
+        const unsigned long long st = ~key, mask = (1ull << d.hagg_log2) - 1ull;
+        // an overfull table stops early instead of walking every slot: no new
+        // group is claimed past 7/8 load, and a probe gives up after 2^14
+        // steps; both latch ERR_CAPACITY and the host re-runs with a larger table
+        const unsigned long long fill_limit = mask + 1ull - ((mask + 1ull) >> 3);
+        const unsigned long long max_steps = mask < 16383ull ? mask : 16383ull;
+        unsigned long long h = (key * 0x9E3779B97F4A7C15ull) >> (64 - d.hagg_log2);
+        for (unsigned long long step = 0; step <= max_steps; step++, h = (h + 1) & mask) {
+          unsigned long long cur = __ldcg(d.hagg_keys + h);
           if (cur == 0ull) {
-            atomicAdd(d.hagg_count, 1ull);
-            cur = st;
+            if (__ldcg(d.hagg_count) >= fill_limit) break;
+            cur = atomicCAS(d.hagg_keys + h, 0ull, st);
+            if (cur == 0ull) {
+              atomicAdd(d.hagg_count, 1ull);
+              cur = st;
+            }
+          }
+          if (cur == st) {
+            hslot = (long long)h;
+            break;
           }
         }
-        if (cur == st) {
-          hslot = (long long)h;
-          break;
+        if (hslot < 0) {  // table full: latched, the host re-runs with a larger table
+          atomicOr(d.err, ERR_CAPACITY);
+          continue;
         }
       }
-      if (hslot < 0) {  // table full: latched, the host re-runs with a larger table
-        atomicOr(d.err, ERR_CAPACITY);
-        continue;
-      }
-    }
-    int gid = 0;
-    bool ok = true;
-    GPL_UNROLL
-    for (int g = 0; g < (K.agg_mode == AGG_HASH ? 0 : K.ngroup); g++) {
-      const GroupDim& G = K.gdim[g];
-      long long v = qget(K, qb, G.field, idx[j]);
-      if (G.transform == G_YEAR) v = (int)v / 10000;
-      const long long o = v - G.lo;
-      if ((unsigned long long)o >= (unsigned long long)G.size) ok = false;
-      gid += (int)o * G.stride;
-    }
-    if (!ok) {
-      atomicOr(d.err, ERR_DOMAIN);
-      continue;
-    }
-    long long val = 0;
-    GPL_UNROLL
-    for (int t = 0; t < K.nterm; t++) {
-      if (K.term_field[t] >= 0) {
-        val += qget(K, qb, K.term_field[t], idx[j]);
-        continue;
-      }
-      const Term& T = K.term[t];
-      long long prod = T.sign;
+      int gid = 0;
+      bool ok = true;
       GPL_UNROLL
-      for (int f = 0; f < T.nfact; f++) {
-        const Factor& F = T.f[f];
-        prod *= F.field < 0 ? F.a : F.a + (long long)F.b * qget(K, qb, F.field, idx[j]);
+      for (int g = 0; g < (K.agg_mode == AGG_HASH ? 0 : K.ngroup); g++) {
+        const GroupDim& G = K.gdim[g];
+        long long v = fget(G.field, j);
+        if (G.transform == G_YEAR) v = (int)v / 10000;
+        const long long o = v - G.lo;
+        if ((unsigned long long)o >= (unsigned long long)G.size) ok = false;
+        gid += (int)o * G.stride;
       }
-      val += prod;
-    }
-    GPL_UNROLL
-    for (int a = 0; a < K.nagg; a++) {
-      const Agg& A = K.agg[a];
-      long long c = 1;
-      if (A.kind == A_SUM) c = val;
-      else if (A.kind == A_SUMIF) c = qget(K, qb, A.field, idx[j]) != 0 ? val : 0;
-      else if (A.kind == A_SUMIFEQ) c = qget(K, qb, A.field, idx[j]) == A.c ? val : 0;
-      if (K.agg_mode == AGG_REG) acc[a] += c;
-      else if (c != 0) {
-        if (K.agg_mode == AGG_HASH) atomicAdd((unsigned long long*)d.hagg_accs + hslot * K.nagg + a, (unsigned long long)c);
-        else if (K.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * K.nagg + a], (unsigned long long)c);
-        else atomic_add_i128(d.partials + 2 * (gid * K.nagg + a), c);
+      if (!ok) {
+        atomicOr(d.err, ERR_DOMAIN);
+        continue;
+      }
+      long long val = 0;
+      GPL_UNROLL
+      for (int t = 0; t < K.nterm; t++) {
+        if (K.term_field[t] >= 0) {
+          val += fget(K.term_field[t], j);
+          continue;
+        }
+        const Term& T = K.term[t];
+        long long prod = T.sign;
+        GPL_UNROLL
+        for (int f = 0; f < T.nfact; f++) {
+          const Factor& F = T.f[f];
+          prod *= F.field < 0 ? F.a : F.a + (long long)F.b * fget(F.field, j);
+        }
+        val += prod;
+      }
+      GPL_UNROLL
+      for (int a = 0; a < K.nagg; a++) {
+        const Agg& A = K.agg[a];
+        long long c = 1;
+        if (A.kind == A_SUM) c = val;
+        else if (A.kind == A_SUMIF) c = fget(A.field, j) != 0 ? val : 0;
+        else if (A.kind == A_SUMIFEQ) c = fget(A.field, j) == A.c ? val : 0;
+        if (K.agg_mode == AGG_REG) acc[a] += c;
+        else if (c != 0) {
+          if (K.agg_mode == AGG_HASH) atomicAdd((unsigned long long*)d.hagg_accs + hslot * K.nagg + a, (unsigned long long)c);
+          else if (K.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * K.nagg + a], (unsigned long long)c);
+          else atomic_add_i128(d.partials + 2 * (gid * K.nagg + a), c);
+        }
       }
     }
-  }
   };
   if (K.fan_probe < 0) {
     run_probes(K.nsprobe, K.nprobe, p);
@@ -551,13 +569,14 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
     const Probe& P = K.probe[K.fan_probe];
     const HTP& h = htp[P.ht];
     const uint32_t* off = (const uint32_t*)h.slots;
+    gather(K.fan_probe, p);
     uint32_t beg[RPL], end[RPL];
     int mx = 0;
     unsigned tot = 0;
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
       const unsigned long long ix =
-          (unsigned long long)((long long)(int32_t)(uint32_t)qget(K, qb, P.k1, idx[j]) - (long long)h.kmin);
+          (unsigned long long)((long long)(int32_t)(uint32_t)fget(P.k1, j) - (long long)h.kmin);
       const bool in = p[j] && ix < h.nslots;
       beg[j] = in ? __ldg(off + ix) : 0u;
       end[j] = in ? __ldg(off + ix + 1) : 0u;
@@ -572,7 +591,7 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
 #pragma unroll
       for (int j = 0; j < RPL; j++) {
         q[j] = beg[j] + (uint32_t)m < end[j];
-        if (q[j] && P.out >= 0) qput(K, qb, P.out, idx[j], (long long)__ldg((const int*)h.pay + beg[j] + m));
+        if (q[j] && P.out >= 0) fput(P.out, j, (long long)__ldg((const int*)h.pay + beg[j] + m));
       }
       run_probes(K.fan_probe + 1, K.nprobe, q);
       tail(q);
@@ -806,6 +825,9 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
       seq_set(hs, t + (unsigned)R);
     }
   } else {
+  unsigned lc[MAXF + MAXSP];  // stage-phase pass counts of this lane's rows (filters, stage probes)
+#pragma unroll
+  for (int i = 0; i < MAXF + MAXSP; i++) lc[i] = 0;
   for (;;) {
     mbar_wait(&full[slot], phase);
     const int4 h = hdr[slot];
@@ -813,12 +835,17 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     if (n < 0) break;
     const uint32_t sb = (uint32_t)K.off_ring + slot * (uint32_t)K.slot_bytes;
     const long long rowbase = ((long long)h.y << 32) | (long long)(uint32_t)h.x;  // lazy-column gathers
-    long long cl_start = 0;
+    // clustered probe: the staged cells cover keys [cl_k0, cl_k0 + cl_ncells)
+    uint32_t cl_k0 = 0, cl_ncells = 0;
     int cl_size = 0;
     if (K.cl_probe >= 0) {
       const int4 h2 = hdr2[slot];
-      cl_start = ((long long)h2.y << 32) | (long long)(uint32_t)h2.x;
+      const long long cl_start = ((long long)h2.y << 32) | (long long)(uint32_t)h2.x;
       cl_size = h2.z;
+      const int w = K.ht[K.probe[K.cl_probe].ht].width;
+      const HTP& H = GPL_SP_HTP(K.cl_probe);
+      cl_k0 = (uint32_t)((long long)H.kmin + (w == 0 ? cl_start * 8 : cl_start / (w > 0 ? w : 1)));
+      cl_ncells = w == 0 ? (uint32_t)cl_size * 8u : (uint32_t)cl_size / (uint32_t)(w > 0 ? w : 1);
     }
     const int nit = (n + 127) >> 7;
     bool released = false;
@@ -857,8 +884,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             for (int j = 0; j < RPL; j++) p[q * RPL + j] = p[q * RPL + j] && filt_pass(F, x[j]);
           }
         }
-        const unsigned c = __reduce_add_sync(0xffffffffu, count_n(p));
-        if (lane == 0) cnt[f] += c;
+        lc[f] += count_n(p);  // per-lane pass count (reduced once, after the last stage)
       }
       // A5 stage-phase probes (keys from the stage; all NR loads in flight together)
       long long sreg[MAXSP][NR];
@@ -868,7 +894,8 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         for (int j = 0; j < NR; j++) sreg[sp][j] = 0;
         if (sp < K.nsprobe) {
           const Probe& P = K.probe[sp];
-          if (__any_sync(0xffffffffu, any_n(p))) {
+          // (with no operator before it every row of a live packet is active)
+          if ((sp == 0 && K.nfilt == 0) || __any_sync(0xffffffffu, any_n(p))) {
             unsigned long long k[NR];
 #pragma unroll
             for (int q = 0; q < NPMAX; q++) {
@@ -891,7 +918,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             bool hit[NR];
             long long v[NR];
             if (sp == K.cl_probe && cl_size > 0)
-              probe_rows_cl<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v, sb + (uint32_t)K.cl_off, cl_start, cl_size);
+              probe_rows_cl<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v, sb + (uint32_t)K.cl_off, cl_k0, cl_ncells);
             else
               probe_rows<NR>(K, GPL_SP_HTP(sp), P.ht, k, p, hit, v);
 #pragma unroll
@@ -904,8 +931,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
               }
             }
           }
-          const unsigned c = __reduce_add_sync(0xffffffffu, count_n(p));
-          if (lane == 0) cnt[K.nfilt + sp] += c;
+          lc[K.nfilt + sp] += count_n(p);
         }
       }
       if (K.sink == SINK_INSERT && K.ins_kcol >= 0) {
@@ -1022,6 +1048,11 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     }
     if (K.flush_each_tile && h.w) flush_reg(d, acc, lane);
     if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
+  }
+  GPL_UNROLL
+  for (int op = 0; op < K.nfilt + K.nsprobe; op++) {
+    const unsigned c = __reduce_add_sync(0xffffffffu, lc[op]);
+    if (lane == 0) cnt[op] += c;
   }
   if (qcount > 0) {
     __syncwarp();
