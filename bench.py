@@ -166,7 +166,7 @@ def workload_config(args, rows_per_gpu, tile_rows):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="gpl", choices=["gpl", "reference"])
     ap.add_argument("--query", default="Q5")
@@ -354,7 +354,7 @@ def main():
         for _ in range(max(6, args.warmup)):
             e2e_step()
         e_ms = []
-        for _ in range(max(3, args.steps // 4)):
+        for _ in range(max(3, min(10, args.steps // 4))):
             flush.zero_()
             ev0.record(stream)
             r2 = e2e_step()
@@ -417,7 +417,8 @@ def main():
                      "logical_scan_bytes": logical,
                      "effective_gbs": logical / (kernel_avg / 1e3) / 1e9,
                      "lazy_columns": stats.get("lazy_columns")},
-        "gpu_launches": kernel_launches(segs) * args.steps,
+        # kernels per step = the kernel nodes of the replayed query graph (library count), x steps
+        "gpu_launches": (stats.get("launches") or kernel_launches(segs)) * args.steps,
         "e2e": e2e,
         "cpu_baseline": cpu,
         "clocks": clk.summary(),

@@ -100,7 +100,8 @@ typedef struct {
   int64_t groups_total;        /* hash group-by: distinct groups (the result may be LIMITed)      */
   int64_t hash_slots;          /* hash group-by: slots of the aggregation table                    */
   int32_t drain_warps;         /* of consumer_warps, those that only drain hand-off packets (NEXT-1) */
-  int32_t reserved2;
+  int32_t launches;            /* kernels one graph-replayed gpl_run_query step launched (its graph's */
+                               /* kernel nodes: clear, builds, fused run, result steps); 0 otherwise */
 } gpl_stats;
 
 /* Result of the last run. Arrays are CALLER-owned with capacity cap_groups. */

@@ -1238,6 +1238,10 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
       S.packets = P.desc.npack;
       S.agg_mode = P.desc.agg_mode;
       S.jit = P.jit ? 1 : 0;
+      {
+        auto gk = ctx->graph_kernels.find(key);
+        S.launches = gk != ctx->graph_kernels.end() ? gk->second : 0;
+      }
       S.hash_slots = (int64_t)P.hagg_cap;
       S.drain_warps = P.desc.ndrain;
       return GPL_OK;
@@ -1335,8 +1339,21 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     ctx->last = saved;
     cudaGraphExec_t exec = nullptr;
     if (ok && cst == GPL_OK && ce == cudaSuccess && graph &&
-        cudaGraphInstantiate(&exec, graph, 0) == cudaSuccess)
+        cudaGraphInstantiate(&exec, graph, 0) == cudaSuccess) {
       ctx->graphs[key] = exec;
+      // kernels one replay launches (stats.launches): the graph's kernel nodes
+      size_t nn = 0;
+      int nk = 0;
+      if (cudaGraphGetNodes(graph, nullptr, &nn) == cudaSuccess && nn) {
+        std::vector<cudaGraphNode_t> nodes(nn);
+        if (cudaGraphGetNodes(graph, nodes.data(), &nn) == cudaSuccess)
+          for (size_t i = 0; i < nn; i++) {
+            cudaGraphNodeType t;
+            if (cudaGraphNodeGetType(nodes[i], &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) nk++;
+          }
+      }
+      ctx->graph_kernels[key] = nk;
+    }
     if (graph) cudaGraphDestroy(graph);
     cudaGetLastError();  // a failed capture only means no graph; the eager run above stands
     ctx->err.clear();

@@ -241,6 +241,7 @@ struct gpl_ctx {
   std::map<std::string, gpl::PreparedBuild> build_cache;
   // gpl_run_query: whole-query CUDA graphs (builds + fused run), keyed by plan text + tile_rows
   std::map<std::string, cudaGraphExec_t> graphs;
+  std::map<std::string, int> graph_kernels;  // kernel nodes of each recorded query graph
   std::map<std::tuple<int, int, int>, gpl::GammaCurve> gamma;  // (depth, stage rows, CTAs/SM) -> Γ(d)
   std::map<std::string, gpl::TunedShape> tuned;  // probe segment text -> measured-best shape
   std::map<std::string, std::vector<std::string>> plan_segs;  // gpl_run_query: plan text -> segments

@@ -55,7 +55,7 @@ class _Stats(ctypes.Structure):
                 ("jit", ctypes.c_int32), ("reserved", ctypes.c_int32), ("intermediate_bytes", ctypes.c_double),
                 ("bytes_full_scan", ctypes.c_double), ("lazy_columns", ctypes.c_int32), ("packets", ctypes.c_int32),
                 ("groups_total", ctypes.c_int64), ("hash_slots", ctypes.c_int64), ("drain_warps", ctypes.c_int32),
-                ("reserved2", ctypes.c_int32)]
+                ("launches", ctypes.c_int32)]
 
 
 class _Result(ctypes.Structure):
