@@ -215,7 +215,10 @@ gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_rows);
  * With option "kbe_tile_rows" = T > 0 the same sequence runs tile by tile
  * (T rows at a time, materialising per tile): the paper's GPL (w/o CE)
  * variant, tiling without concurrent kernels or channels (P:337, P:382,
- * P:564); stats.tile_rows_used = T. */
+ * P:564); its buffers are sized for T rows and every operator's cardinality
+ * stays on the device (the kernels read it), so the tiles run back to back
+ * with no host round trip (one synchronise at the end for the byte count);
+ * stats.tile_rows_used = T. */
 gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment);
 
 /* Synchronise the stream and return the last run's result: the A10 finalize

@@ -400,6 +400,7 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     if (ctx->h_minmax) cudaFreeHost(ctx->h_minmax);
     if (ctx->d_minmax) cudaFree(ctx->d_minmax);
     if (ctx->d_bounds) cudaFree(ctx->d_bounds);
+    if (ctx->d_kbe_bytes) cudaFree(ctx->d_kbe_bytes);
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);
     if (ctx->d_hagg) cudaFree(ctx->d_hagg);
     if (ctx->d_hres) cudaFree(ctx->d_hres);
@@ -1731,17 +1732,28 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
     if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("KBE buffers: ") + cudaGetErrorString(e));
     ctx->kbe_cap = need;
   }
+  // GPL (w/o CE): tiles run back to back with device-side cardinalities (no
+  // host round trip per tile or operator); KBE: the host sizes each operator
+  const bool tiled = ctx->opt.kbe_tile_rows > 0;
+  if (tiled && !ctx->d_kbe_bytes) CK(cudaMalloc(&ctx->d_kbe_bytes, sizeof(unsigned long long)));
+  if (tiled) CK(cudaMemsetAsync(ctx->d_kbe_bytes, 0, sizeof(unsigned long long), ctx->stream));
   CK(cudaEventRecord(ctx->ev0, ctx->stream));
   for (long long r0 = 0; r0 < d.nrows || (r0 == 0 && d.nrows == 0); r0 += tile) {
     dt = d;
     dt.nrows = std::min<long long>(tile, d.nrows - r0);
     for (int c = 0; c < d.ncols; c++) dt.col[c] = d.col[c] + r0 * d.colw[c];
     double tb = 0;
-    CK(run_kbe(dt, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &tb));
+    CK(run_kbe(dt, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &tb, tiled ? ctx->d_kbe_bytes : nullptr));
     inter += tb;
     if (d.nrows == 0) break;
   }
   CK(cudaEventRecord(ctx->ev1, ctx->stream));
+  if (tiled) {  // the materialised bytes, read once after the run
+    unsigned long long db = 0;
+    CK(cudaMemcpyAsync(&db, ctx->d_kbe_bytes, sizeof(db), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    inter += (double)db;
+  }
   LastRun& L = ctx->last;
   L.valid = true;
   L.kbe = true;

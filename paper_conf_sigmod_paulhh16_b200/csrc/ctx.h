@@ -263,6 +263,7 @@ struct gpl_ctx {
   std::map<std::string, std::pair<uint64_t, int64_t>> hagg_groups;  // plan text -> (distinct groups, fact rows) of its last run
   // A10 key decodes: table name -> (table version, key -> output value)
   std::map<std::string, std::pair<uint64_t, std::map<int32_t, int32_t>>> decode_maps;
+  unsigned long long* d_kbe_bytes = nullptr;  // GPL (w/o CE): materialised bytes counted on the device
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;
   size_t kbe_cap = 0;

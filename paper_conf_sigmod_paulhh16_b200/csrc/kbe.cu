@@ -74,7 +74,8 @@ struct FieldSet {
 // scatter: compact every live field by flags/positions. Pushed-down terms
 // with no array yet are evaluated from the staged columns (first operator).
 __global__ void kbe_scatter(const __grid_constant__ PipeDesc d, long long n, const int* flags, const int* pos,
-                            FieldSet in, FieldSet out, int first) {
+                            FieldSet in, FieldSet out, int first, const long long* nptr) {
+  if (nptr) n = min(n, *nptr);
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     if (!flags[i]) continue;
     const long long o = pos[i];
@@ -90,7 +91,8 @@ __global__ void kbe_scatter(const __grid_constant__ PipeDesc d, long long n, con
 }
 
 __global__ void kbe_probe_map(const __grid_constant__ PipeDesc d, int pi, long long n, FieldSet fs, int* flags,
-                              char* payload, int pw) {
+                              char* payload, int pw, const long long* nptr) {
+  if (nptr) n = min(n, *nptr);
   const Probe& P = d.probe[pi];
   const HTP h = load_htp(d.ht[P.ht]);
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
@@ -103,7 +105,9 @@ __global__ void kbe_probe_map(const __grid_constant__ PipeDesc d, int pi, long l
   }
 }
 
-__global__ void kbe_resid_map(const __grid_constant__ PipeDesc d, int r, long long n, FieldSet fs, int* flags) {
+__global__ void kbe_resid_map(const __grid_constant__ PipeDesc d, int r, long long n, FieldSet fs, int* flags,
+                              const long long* nptr) {
+  if (nptr) n = min(n, *nptr);
   const Resid& R = d.resid[r];
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     const long long a = ldf(fs.ptr[R.a], fs.w[R.a], i);
@@ -119,13 +123,21 @@ __global__ void kbe_resid_map(const __grid_constant__ PipeDesc d, int r, long lo
   }
 }
 
-__global__ void kbe_total(const int* flags, const int* pos, long long n, long long* total) {
-  *total = n ? (long long)pos[n - 1] + flags[n - 1] : 0;
+// output cardinality of a compaction; device-sized mode also accumulates the
+// materialised bytes (positions + live output fields) on the device
+__global__ void kbe_total(const int* flags, const int* pos, long long n, long long* total, unsigned long long* bytes,
+                          const long long* nprev, int in_row_bytes, int out_w) {
+  const long long live_in = nprev ? *nprev : n;  // (read before *total is overwritten: same word)
+  const long long t = n ? (long long)pos[n - 1] + flags[n - 1] : 0;
+  *total = t;
+  if (bytes) *bytes += (unsigned long long)(live_in * in_row_bytes + t * (long long)out_w);
 }
 
 // aggregate over the final materialised rows: per-block shared table, then
 // exact int128 global atomics (same arithmetic as the fused pipeline)
-__global__ void kbe_aggregate(const __grid_constant__ PipeDesc d, long long n, FieldSet fs, unsigned long long* partials) {
+__global__ void kbe_aggregate(const __grid_constant__ PipeDesc d, long long n, FieldSet fs, unsigned long long* partials,
+                              const long long* nptr) {
+  if (nptr) n = min(n, *nptr);
   extern __shared__ unsigned long long tab[];
   const int G = d.ngroups_total, A = d.nagg;
   const bool use_smem = G * A <= 4096;
@@ -196,10 +208,20 @@ size_t kbe_pool_bytes(const PipeDesc& d) {
   return per_row * (size_t)(d.nrows + 64) + 4 * (tmp + 4096) + (1 << 20);
 }
 
-cudaError_t run_kbe(const PipeDesc& d, int sms, cudaStream_t s, void* pool, size_t pool_bytes, double* inter_bytes) {
+// KBE over d.nrows rows. device_bytes == nullptr: the paper's KBE — the host
+// reads every operator's output cardinality (one D2H + synchronise per
+// operator) to size the next buffers. device_bytes != nullptr: the same
+// kernel sequence with every buffer sized for d.nrows (an operator's output is
+// never larger than its input) and the cardinalities kept on the device (the
+// kernels read them): no host round trip, so GPL (w/o CE) can run tile after
+// tile asynchronously; the materialised bytes accumulate in
+// *device_bytes.
+cudaError_t run_kbe(const PipeDesc& d, int sms, cudaStream_t s, void* pool, size_t pool_bytes, double* inter_bytes,
+                    unsigned long long* device_bytes) {
   double bytes = 0;
   cudaError_t e = cudaSuccess;
   size_t used = 0;
+  const bool dev = device_bytes != nullptr;
   // bump allocation from a per-context pool (sized once by kbe_pool_bytes), so
   // the baseline pays for materialisation, not for the allocator
   auto alloc = [&](size_t b) -> char* {
@@ -214,7 +236,9 @@ cudaError_t run_kbe(const PipeDesc& d, int sms, cudaStream_t s, void* pool, size
     return p;
   };
   long long* d_total = (long long*)alloc(sizeof(long long));
-  long long n = d.nrows;
+  long long n = d.nrows;          // host: the row count (KBE) / the capacity (device-sized)
+  const long long cap = d.nrows;
+  const long long* nptr = nullptr;  // device-sized: the live row count on the device (null: n rows)
   FieldSet fs{};
   fs.n = d.nfield;
   for (int f = 0; f < d.nfield; f++) {
@@ -222,34 +246,51 @@ cudaError_t run_kbe(const PipeDesc& d, int sms, cudaStream_t s, void* pool, size
     fs.ptr[f] = (f < d.npush && d.push[f].kind == PUSH_COL) ? (char*)d.col[d.push[f].src] : nullptr;
   }
   // compact all live fields by a flags array (prefix sum + scatter); returns new n
-  auto compact = [&](int* flags, bool first) -> long long {
+  auto compact = [&](int* flags, bool first, int pay_w) -> long long {
     int* pos = (int*)alloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
     size_t tmp = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, tmp, flags, pos, (int)n, s);
     void* t = alloc(tmp);
     if (e != cudaSuccess) return 0;
-    cub::DeviceScan::ExclusiveSum(t, tmp, flags, pos, (int)n, s);
-    kbe_total<<<1, 1, 0, s>>>(flags, pos, n, d_total);
+    if (n > 0) cub::DeviceScan::ExclusiveSum(t, tmp, flags, pos, (int)n, s);
+    int out_w = 0;
+    for (int f = 0; f < fs.n; f++)
+      if (fs.ptr[f] || (first && f < d.npush && d.push[f].kind == PUSH_TERM)) out_w += fs.w[f];
     long long total = 0;
-    if (e == cudaSuccess) e = cudaMemcpyAsync(&total, d_total, sizeof(total), cudaMemcpyDeviceToHost, s);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(s);  // KBE sizes the next operator's output here
-    bytes += 4.0 * n;  // positions
+    if (dev) {
+      // the count stays on the device; buffers sized for the capacity
+      // flags + positions (8 B) + the map's payload column per live input row, then the compacted fields
+      kbe_total<<<1, 1, 0, s>>>(flags, pos, n, d_total, device_bytes, nptr, 8 + pay_w, out_w);
+      total = n;
+    } else {
+      kbe_total<<<1, 1, 0, s>>>(flags, pos, n, d_total, nullptr, nullptr, 0, 0);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&total, d_total, sizeof(total), cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);  // KBE sizes the next operator's output here
+      bytes += 4.0 * n + (double)total * out_w;  // positions + the compacted live fields (flags/payloads: the maps)
+    }
     FieldSet out = fs;
     for (int f = 0; f < fs.n; f++) {
       const bool live = fs.ptr[f] || (first && f < d.npush && d.push[f].kind == PUSH_TERM);
       out.ptr[f] = live ? alloc((size_t)(total > 0 ? total : 1) * fs.w[f]) : nullptr;
-      if (live) bytes += (double)total * fs.w[f];
     }
-    if (n > 0) kbe_scatter<<<grid_for(n, sms), kThreads, 0, s>>>(d, n, flags, pos, fs, out, first ? 1 : 0);
+    if (n > 0) kbe_scatter<<<grid_for(n, sms), kThreads, 0, s>>>(d, n, flags, pos, fs, out, first ? 1 : 0, nptr);
     fs = out;
+    if (dev) nptr = d_total;  // every later kernel reads the live count
     return total;
+  };
+  // device-sized mode: a map writes flags only for the live rows; the rest of
+  // the capacity must read as 0 for the scan
+  auto flags_for = [&]() -> int* {
+    int* f = (int*)alloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    if (dev && nptr && f && n > 0 && e == cudaSuccess) e = cudaMemsetAsync(f, 0, sizeof(int) * (size_t)n, s);
+    return f;
   };
   // selection: map -> prefix sum -> scatter
   if (d.nfilt > 0) {
-    int* flags = (int*)alloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    int* flags = flags_for();
     if (n > 0) kbe_filter_map<<<grid_for(n, sms), kThreads, 0, s>>>(d, n, flags);
-    bytes += 4.0 * n;
-    n = compact(flags, true);
+    if (!dev) bytes += 4.0 * n;
+    n = compact(flags, true, 0);
   } else {
     for (int f = 0; f < d.npush; f++)
       if (d.push[f].kind == PUSH_TERM) {  // expression materialised as a column
@@ -261,29 +302,30 @@ cudaError_t run_kbe(const PipeDesc& d, int sms, cudaStream_t s, void* pool, size
   // probes: map (flags + payload) -> prefix sum -> scatter
   for (int p = 0; p < d.nprobe && e == cudaSuccess; p++) {
     const Probe& P = d.probe[p];
-    int* flags = (int*)alloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
+    int* flags = flags_for();
     char* pay = nullptr;
     int pw = 8;
     if (P.out >= 0) {
       pw = fs.w[P.out];
       pay = alloc((size_t)(n > 0 ? n : 1) * pw);
       fs.ptr[P.out] = pay;
-      bytes += (double)n * pw;
+      if (!dev) bytes += (double)n * pw;
     }
-    if (n > 0) kbe_probe_map<<<grid_for(n, sms), kThreads, 0, s>>>(d, p, n, fs, flags, pay, pw);
-    bytes += 4.0 * n;
-    if (P.kind != P_MARK) n = compact(flags, false);
+    if (n > 0) kbe_probe_map<<<grid_for(n, sms), kThreads, 0, s>>>(d, p, n, fs, flags, pay, pw, nptr);
+    if (!dev) bytes += 4.0 * n;
+    if (P.kind != P_MARK) n = compact(flags, false, P.out >= 0 ? pw : 0);
   }
   for (int r = 0; r < d.nresid && e == cudaSuccess; r++) {
-    int* flags = (int*)alloc(sizeof(int) * (size_t)(n > 0 ? n : 1));
-    if (n > 0) kbe_resid_map<<<grid_for(n, sms), kThreads, 0, s>>>(d, r, n, fs, flags);
-    bytes += 4.0 * n;
-    n = compact(flags, false);
+    int* flags = flags_for();
+    if (n > 0) kbe_resid_map<<<grid_for(n, sms), kThreads, 0, s>>>(d, r, n, fs, flags, nptr);
+    if (!dev) bytes += 4.0 * n;
+    n = compact(flags, false, 0);
   }
   if (e == cudaSuccess && n > 0) {
     const size_t sm = (size_t)d.ngroups_total * d.nagg <= 4096 ? (size_t)d.ngroups_total * d.nagg * 8 : 0;
-    kbe_aggregate<<<grid_for(n, sms), kThreads, sm, s>>>(d, n, fs, d.partials);
+    kbe_aggregate<<<grid_for(n, sms), kThreads, sm, s>>>(d, n, fs, d.partials, nptr);
   }
+  (void)cap;
   *inter_bytes = bytes;
   if (e != cudaSuccess) return e;
   return cudaGetLastError();

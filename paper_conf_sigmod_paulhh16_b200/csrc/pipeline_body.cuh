@@ -190,6 +190,19 @@ __device__ __forceinline__ void ld_col(const PipeDesc& d, const PipeDesc& K, int
   }
 }
 
+// RPL rows of a 32-bit key column (probe keys are validated 32-bit): staged
+// (one 16-B shared load) or, for a lazy column, gathered for the active rows
+__device__ __forceinline__ void ld_key32(const PipeDesc& d, const PipeDesc& K, int c, uint32_t sb, int r0,
+                                         long long rowbase, const bool* act, uint32_t (&x)[RPL]) {
+  if (K.lazy[c]) {
+#pragma unroll
+    for (int j = 0; j < RPL; j++) x[j] = act[j] ? __ldg((const uint32_t*)d.col[c] + rowbase + r0 + j) : 0u;
+  } else {
+    const int4 v = lds_v4(smem_base() + sb + K.coloff[c] + r0 * 4);
+    x[0] = (uint32_t)v.x; x[1] = (uint32_t)v.y; x[2] = (uint32_t)v.z; x[3] = (uint32_t)v.w;
+  }
+}
+
 // survivor-queue field access (shared-space loads/stores, see smem_base)
 __device__ __forceinline__ long long qget(const PipeDesc& K, uint32_t qb, int f, int i) {
   const uint32_t a = smem_base() + qb + K.qoff[f];
@@ -828,6 +841,9 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   unsigned lc[MAXF + MAXSP];  // stage-phase pass counts of this lane's rows (filters, stage probes)
 #pragma unroll
   for (int i = 0; i < MAXF + MAXSP; i++) lc[i] = 0;
+  // rows this warp queued = the pass count of the last stage-phase operator
+  const bool kQueueCounts = !(K.sink == SINK_INSERT && K.ins_kcol >= 0);
+  unsigned long long queued = 0;
   for (;;) {
     mbar_wait(&full[slot], phase);
     const int4 h = hdr[slot];
@@ -861,7 +877,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
       for (int q = 0; q < NPMAX; q++) {
         r0q[q] = ((it0 + q * Ws) << 7) + (lane << 2);
-        live[q] = q < npk && it0 + q * Ws < nit;
+        live[q] = q == 0 || (q < npk && it0 + q * Ws < nit);  // (packet 0: the loop condition)
       }
       bool p[NR];
 #pragma unroll
@@ -884,7 +900,9 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             for (int j = 0; j < RPL; j++) p[q * RPL + j] = p[q * RPL + j] && filt_pass(F, x[j]);
           }
         }
-        lc[f] += count_n(p);  // per-lane pass count (reduced once, after the last stage)
+        // per-lane pass count, reduced once after the last stage (the last stage-phase
+        // operator is counted by the compaction instead: its survivors are the queued rows)
+        if (!(kQueueCounts && K.nsprobe == 0 && f == K.nfilt - 1)) lc[f] += count_n(p);
       }
       // A5 stage-phase probes (keys from the stage; all NR loads in flight together)
       long long sreg[MAXSP][NR];
@@ -899,20 +917,20 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             unsigned long long k[NR];
 #pragma unroll
             for (int q = 0; q < NPMAX; q++) {
-              long long k1[RPL];
+              uint32_t k1[RPL];
               if (live[q]) {
-                ld_col(d, K, P.k1, sb, r0q[q], rowbase, p + q * RPL, k1);
+                ld_key32(d, K, P.k1, sb, r0q[q], rowbase, p + q * RPL, k1);
               } else {
 #pragma unroll
-                for (int j = 0; j < RPL; j++) k1[j] = 0;
+                for (int j = 0; j < RPL; j++) k1[j] = 0u;
               }
 #pragma unroll
-              for (int j = 0; j < RPL; j++) k[q * RPL + j] = (uint32_t)k1[j];
+              for (int j = 0; j < RPL; j++) k[q * RPL + j] = k1[j];
               if (P.k2 >= 0 && live[q]) {
-                long long k2[RPL];
-                ld_col(d, K, P.k2, sb, r0q[q], rowbase, p + q * RPL, k2);
+                uint32_t k2[RPL];
+                ld_key32(d, K, P.k2, sb, r0q[q], rowbase, p + q * RPL, k2);
 #pragma unroll
-                for (int j = 0; j < RPL; j++) k[q * RPL + j] = (k[q * RPL + j] << 32) | (uint32_t)k2[j];
+                for (int j = 0; j < RPL; j++) k[q * RPL + j] = (k[q * RPL + j] << 32) | k2[j];
               }
             }
             bool hit[NR];
@@ -931,7 +949,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
               }
             }
           }
-          lc[K.nfilt + sp] += count_n(p);
+          if (!(kQueueCounts && sp == K.nsprobe - 1)) lc[K.nfilt + sp] += count_n(p);
         }
       }
       if (K.sink == SINK_INSERT && K.ins_kcol >= 0) {
@@ -979,6 +997,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           pos[j] = (qhead + base + __popc(m & lanemask_lt())) & (QCAP - 1);
           base += __popc(m);
         }
+        queued += (unsigned)(base - qcount);
         if (base != qcount) {
           GPL_UNROLL
           for (int e = 0; e < K.npush; e++) {
@@ -1051,6 +1070,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   }
   GPL_UNROLL
   for (int op = 0; op < K.nfilt + K.nsprobe; op++) {
+    if (kQueueCounts && op == K.nfilt + K.nsprobe - 1) {
+      if (lane == 0) cnt[op] += queued;
+      continue;
+    }
     const unsigned c = __reduce_add_sync(0xffffffffu, lc[op]);
     if (lane == 0) cnt[op] += c;
   }

@@ -740,3 +740,24 @@ def test_q3_full_device_sort_order_by_without_limit(ctx):
             assert e.status == gpl.GPL_E_CAPACITY and attempt < 2
     assert len(r.keys) == len(o.keys) > 1000
     assert list(zip(r.keys, r.aggs)) == want
+
+
+# ---- BASELINE config 3: SF 10 Q9, the paper-literal bound and the Q9-wide reading (R5)
+
+@pytest.fixture(scope="module")
+def db_sf10():
+    return tpchgen.generate(10.0, seed=tpchgen.DEFAULT_SEED)
+
+
+@pytest.mark.parametrize("bound", ["literal", "wide"])
+def test_config3_sf10_q9_exact(ctx, db_sf10, bound):
+    """Q9 at SF 10 (60M lineitem rows) bit-exact vs the multi-threaded oracle over the whole database,
+    in the Listing's ORDER BY order: p_partkey < 1000 (literal) and the large-intermediate
+    Q9-wide bound ceil(0.054 |part|) (reading R5)."""
+    db = db_sf10
+    nparts = db.nrows("part")
+    params = (1000,) if bound == "literal" else (-(-54 * nparts // 1000),)
+    r = _gpu(ctx, db, "Q9", params)
+    o = oracle.finalize("Q9", oracle.run("Q9", db, params, threads=oracle.host_threads()))
+    assert r.keys == o.keys and r.aggs == o.aggs
+    assert len(r.keys) == 175 and sum(a[0] for a in r.aggs) > (20_000 if bound == "literal" else 1_000_000)
