@@ -224,7 +224,9 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
         # paper's default 1 MB tile in rows of this query's scan width
         bpr = max(1, int(rf.stats["bytes_scanned"] / max(1, rf.stats["rows_scanned"])))
         tw, rw = timed(True, (1 << 20) // bpr)
-        assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs) == (rw.keys, rw.aggs), name
+        # ... and with the paper's largest swept tile, 16 MB: fewer, larger tiles
+        tw16, rw16 = timed(True, (16 << 20) // bpr)
+        assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs) == (rw.keys, rw.aggs) == (rw16.keys, rw16.aggs), name
         inp = rf.stats.get("bytes_full_scan") or rf.stats["bytes_scanned"]  # the input: every column read, once
         ops = rf.stats["op_pass"]
         sel = (ops[0] / rf.stats["rows_scanned"]) if q == "Q14" and ops else None
@@ -232,6 +234,8 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
                      "fused_ms": tf, "kbe_ms": tk, "speedup": tk / tf,
                      "wo_ce_ms": tw, "wo_ce_tile_rows": rw.stats["tile_rows_used"],
                      "wo_ce_over_kbe": tw / tk, "wo_ce_intermediate_bytes": rw.stats["intermediate_bytes"],
+                     "wo_ce_16mb_ms": tw16, "wo_ce_16mb_tile_rows": rw16.stats["tile_rows_used"],
+                     "wo_ce_16mb_over_kbe": tw16 / tk,
                      "fused_moved_bytes": rf.stats["bytes_scanned"], "fused_lazy_columns": rf.stats.get("lazy_columns"),
                      "fused_intermediate_bytes": rf.stats["intermediate_bytes"],
                      "kbe_intermediate_bytes": rk.stats["intermediate_bytes"],
@@ -240,6 +244,105 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
     summary = {"experiment": "fused vs KBE (config 5)", "sf": sf, "points": rows,
                "paper_context": "AMD A10: KBE intermediates 1.38x input at 100% Q14 selectivity vs 0.22x for GPL "
                                 "(P:402); GPL up to 48% faster than KBE (P:384)"}
+    if out:
+        with open(out, "w") as f:
+            json.dump(summary, f, indent=1)
+    return summary
+
+
+def knob_sweep(q="Q5", sf=1.0, seed=20160626, reps=3, out=None, setup=None):
+    """Config 2 over the channel knobs (PAPER.md Figs 12-13; Eq 10): stage rows s in
+    {512, 1024, 2048} (the packet analog), ring depth n in {2, 3, 4} (the number of channels) and
+    Δ = 2^9 .. 2^22 rows (at least one stage), every other knob from the A9 model. Measured kernel time
+    vs the model's estimate for the same configuration (Eq 10 relative error), the model's argmin vs the
+    measured argmin, and bit-identical results at every point."""
+    from paper_conf_sigmod_paulhh16_b200 import queries
+    db, ctx, flush, stream = setup or _setup(q, sf, seed)
+    segs = queries.segments(queries.plan_text(q, db))
+    for _ in range(4):  # λ profile + the model's profiling input (the paper profiles the first tile, P:323)
+        ctx.run_query(queries.plan_text(q, db))
+        ctx.fetch_result()
+    rows, ref = [], None
+    try:
+        for S in (512, 1024, 2048):
+            for n in (2, 3, 4):
+                ctx.set_option("stage_rows", S)
+                ctx.set_option("ring_depth", n)
+                for e in range(9, 23):
+                    tile = 1 << e
+                    if tile < S:
+                        continue
+                    ts, r = [], None
+                    for i in range(reps + 1):
+                        for sg in segs[:-1]:
+                            ctx.build_hash(sg)
+                        flush.zero_()
+                        ctx.run_plan(segs[-1], tile)
+                        r = ctx.fetch_result()
+                        if i >= 1:
+                            ts.append(r.stats["kernel_ms"])
+                    if ref is None:
+                        ref = (r.keys, r.aggs)
+                    assert (r.keys, r.aggs) == ref, "result changed with the knobs"
+                    t = statistics.median(ts)
+                    est = r.stats["predicted_ms"]
+                    rows.append({"stage_rows": S, "ring_depth": n, "tile_rows": r.stats["tile_rows_used"],
+                                 "consumer_warps": r.stats["consumer_warps"], "measured_ms": t, "predicted_ms": est,
+                                 "rel_error": abs(t - est) / t})
+    finally:
+        ctx.set_option("stage_rows", -1)
+        ctx.set_option("ring_depth", -1)
+    best_meas = min(rows, key=lambda x: x["measured_ms"])
+    best_pred = min(rows, key=lambda x: (x["predicted_ms"], -x["tile_rows"]))
+    summary = {"experiment": "knob sweep (config 2: s x n x Δ)", "query": q, "sf": sf, "points_measured": len(rows),
+               "mean_rel_error": statistics.mean(x["rel_error"] for x in rows),
+               "median_rel_error": statistics.median(x["rel_error"] for x in rows),
+               "measured_best": best_meas, "model_pick": best_pred,
+               "model_pick_vs_best": best_pred["measured_ms"] / best_meas["measured_ms"],
+               "results_identical": True, "points": rows}
+    if out:
+        with open(out, "w") as f:
+            json.dump(summary, f, indent=1)
+    return summary
+
+
+def model_vs_autotune(qs=("Q5", "Q7", "Q8", "Q9", "Q14"), sf=100.0, seed=20160626, reps=5, out=None):
+    """A9 without autotune (config 4): the shape the re-derived model picks on its own (after the
+    λ profile and the profiled run) vs the shape gpl_autotune measures best; kernel times
+    (median of reps, L2 flushed), the model's Eq 10 error for its own pick, identical results."""
+    from paper_conf_sigmod_paulhh16_b200 import queries
+    tables = sorted({t for q in qs for t in queries.TABLES[q]} | {"region", "nation"})
+    db, ctx, flush, stream = _setup(qs[0], sf, seed, tables)
+    rows = []
+    for q in qs:
+        text = queries.plan_text(q, db)
+
+        def timed():
+            ts, r = [], None
+            for i in range(reps + 1):
+                flush.zero_()
+                ctx.run_query(text)
+                r = ctx.fetch_result()
+                if i >= 1:
+                    ts.append(r.stats["kernel_ms"])
+            return statistics.median(ts), r
+        for _ in range(6):  # λ, then the profiled runs; the model re-plans with its fitted costs
+            ctx.run_query(text)
+            ctx.fetch_result()
+        tm, rm = timed()
+        m = ctx.autotune(text)
+        ta, ra = timed()
+        assert (rm.keys, rm.aggs) == (ra.keys, ra.aggs), q
+        shape = lambda r: {k: r.stats[k] for k in ("stage_rows", "ring_depth", "consumer_warps", "grid",  # noqa: E731
+                                                    "tile_rows_used", "probe_split", "packets")}
+        rows.append({"query": q, "model_ms": tm, "model_predicted_ms": rm.stats["predicted_ms"],
+                     "model_rel_error": abs(tm - rm.stats["predicted_ms"]) / tm, "autotune_ms": ta,
+                     "model_over_autotune": tm / ta, "candidates_measured": m["candidates"],
+                     "model_shape": shape(rm), "autotune_shape": shape(ra)})
+        ctx.set_option("stage_rows", -1)  # un-pin for the next query
+    summary = {"experiment": "A9 model pick vs autotune (config 4)", "sf": sf, "points": rows,
+               "max_model_over_autotune": max(x["model_over_autotune"] for x in rows),
+               "mean_model_rel_error": statistics.mean(x["model_rel_error"] for x in rows)}
     if out:
         with open(out, "w") as f:
             json.dump(summary, f, indent=1)
@@ -257,6 +360,10 @@ if __name__ == "__main__":
             x.pop("points", None)
     elif which == "warps":
         s = warp_sweep(out=os.path.join(ROOT, "gpurun_out", "warp_sweep.json"))
+    elif which == "knobs":
+        s = knob_sweep(out=os.path.join(ROOT, "gpurun_out", "knob_sweep_config2.json"))
+    elif which == "model":
+        s = model_vs_autotune(out=os.path.join(ROOT, "gpurun_out", "model_vs_autotune_sf100.json"))
     else:
         s = kbe_compare(out=os.path.join(ROOT, "gpurun_out", "kbe_config5.json"))
     s.pop("points", None)

@@ -340,15 +340,16 @@ __global__ void __launch_bounds__(kThreads) minmax_kernel(const char* col, int w
 struct MinmaxCols {
   const char* col[64];
   int w[64];
-  long long* out;  // [ncols][3]
+  long long* out;  // [ncols][4]: min, max, descents, equal neighbours
 };
 
 __global__ void minmax_init_cols_kernel(long long* out, int ncols) {
   const int c = threadIdx.x;
   if (c < ncols) {
-    out[3 * c] = LLONG_MAX;
-    out[3 * c + 1] = LLONG_MIN;
-    out[3 * c + 2] = 0;
+    out[4 * c] = LLONG_MAX;
+    out[4 * c + 1] = LLONG_MIN;
+    out[4 * c + 2] = 0;
+    out[4 * c + 3] = 0;
   }
 }
 
@@ -356,16 +357,21 @@ __global__ void __launch_bounds__(kThreads) minmax_cols_kernel(MinmaxCols a, lon
   const int c = blockIdx.y;
   const char* col = a.col[c];
   const int w = a.w[c];
-  long long* out = a.out + 3 * c;
+  long long* out = a.out + 4 * c;
   long long mn = LLONG_MAX, mx = LLONG_MIN;
-  unsigned long long desc = 0;
+  unsigned long long desc = 0, eq = 0;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     const long long v = ld_col_global(col, w, i);
     mn = min(mn, v);
     mx = max(mx, v);
-    if (i + 1 < n && v > ld_col_global(col, w, i + 1)) desc++;
+    if (i + 1 < n) {
+      const long long u = ld_col_global(col, w, i + 1);
+      desc += v > u;
+      eq += v == u;
+    }
   }
   if (desc) atomicAdd((unsigned long long*)&out[2], desc);
+  if (eq) atomicAdd((unsigned long long*)&out[3], eq);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));

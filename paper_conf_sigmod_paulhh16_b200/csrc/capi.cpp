@@ -190,11 +190,12 @@ gpl_status resolve_pending(gpl_ctx* ctx) {
     auto it = ctx->tables.find(pl.table);
     if (it == ctx->tables.end()) continue;
     Table& t = it->second;
-    const long long* mm = ctx->h_minmax + 3 * pl.slot0;
+    const long long* mm = ctx->h_minmax + 4 * pl.slot0;
     for (int i = 0; i < pl.ncols && i < (int)t.cols.size(); i++) {
-      t.cols[i].vmin = t.nrows ? mm[3 * i] : 0;
-      t.cols[i].vmax = t.nrows ? mm[3 * i + 1] : 0;
-      t.cols[i].sorted = mm[3 * i + 2] == 0;  // no descent between consecutive rows
+      t.cols[i].vmin = t.nrows ? mm[4 * i] : 0;
+      t.cols[i].vmax = t.nrows ? mm[4 * i + 1] : 0;
+      t.cols[i].sorted = mm[4 * i + 2] == 0;                        // no descent between consecutive rows
+      t.cols[i].strict = t.cols[i].sorted && mm[4 * i + 3] == 0;   // ... and no two equal consecutive rows
     }
     if (pl.has_old) {
       const Table& o = pl.old_meta;
@@ -203,7 +204,7 @@ gpl_status resolve_pending(gpl_ctx* ctx) {
         const Column& a = o.cols[i];
         const Column& b = t.cols[i];
         same = a.name == b.name && a.type == b.type && a.width == b.width && a.dev == b.dev && a.vmin == b.vmin &&
-               a.vmax == b.vmax && a.cap_rows == b.cap_rows && a.sorted == b.sorted;
+               a.vmax == b.vmax && a.cap_rows == b.cap_rows && a.sorted == b.sorted && a.strict == b.strict;
       }
       if (same) t.version = o.version;
     }
@@ -372,7 +373,7 @@ GPL_API gpl_status gpl_create(int device, void* cuda_stream, gpl_ctx** out) {
   if ((e = cudaHostGetDevicePointer((void**)&ctx->h_stage_dev, ctx->h_stage, 0)) != cudaSuccess)
     return bad(e, "mapped staging");
   if ((e = cudaMallocHost((void**)&ctx->h_err, 64)) != cudaSuccess) return bad(e, "pinned error word");
-  if ((e = cudaMallocHost((void**)&ctx->h_minmax, kMinmaxSlots * 3 * sizeof(long long))) != cudaSuccess)
+  if ((e = cudaMallocHost((void**)&ctx->h_minmax, kMinmaxSlots * 4 * sizeof(long long))) != cudaSuccess)
     return bad(e, "pinned min/max");
   if ((e = cudaEventCreate(&ctx->ev0)) != cudaSuccess) return bad(e, "event");
   if ((e = cudaEventCreate(&ctx->ev1)) != cudaSuccess) return bad(e, "event");
@@ -458,6 +459,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "drain_warps") {
     if (v >= 0 && v > 4) return fail(ctx, GPL_E_ARG, "drain_warps in [0, 4] (-1 = model)");
     o.drain_warps = v < 0 ? -1 : v;
+  } else if (k == "dense_build") {
+    o.dense_build = v != 0 ? 1 : 0;
   } else if (k == "reg_fields") {
     o.reg_fields = v != 0 ? 1 : 0;
   } else if (k == "zone_restrict") {
@@ -518,12 +521,14 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       c.vmin = LLONG_MAX;
       c.vmax = LLONG_MIN;
       c.sorted = true;
+      c.strict = true;
       long long prev = LLONG_MIN;
       for (int64_t r = 0; r < nrows; r++) {
         long long v = c.width == 4 ? (long long)((const int32_t*)c.host.data())[r] : ((const int64_t*)c.host.data())[r];
         c.vmin = std::min<long long>(c.vmin, v);
         c.vmax = std::max<long long>(c.vmax, v);
         c.sorted = c.sorted && v >= prev;
+        c.strict = c.strict && (r == 0 || v > prev);
         prev = v;
       }
       if (nrows == 0) c.vmin = c.vmax = 0;
@@ -539,7 +544,7 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
         break;
       }
     if (!ctx->d_minmax) {
-      CK(cudaMalloc(&ctx->d_minmax, kMinmaxSlots * 3 * sizeof(long long)));
+      CK(cudaMalloc(&ctx->d_minmax, kMinmaxSlots * 4 * sizeof(long long)));
       ctx->minmax_cap = kMinmaxSlots;
     }
     if (!ctx->mm_ev) CK(cudaEventCreateWithFlags(&ctx->mm_ev, cudaEventDisableTiming));
@@ -616,8 +621,8 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       cw[i] = t.cols[i].width;
     }
     const int slot0 = ctx->mm_next;
-    CK(launch_minmax_cols(cp, cw, ncols, nrows, ctx->d_minmax + 3 * slot0, ctx->stream));
-    CK(cudaMemcpyAsync(ctx->h_minmax + 3 * slot0, ctx->d_minmax + 3 * slot0, sizeof(long long) * 3 * ncols,
+    CK(launch_minmax_cols(cp, cw, ncols, nrows, ctx->d_minmax + 4 * slot0, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_minmax + 4 * slot0, ctx->d_minmax + 4 * slot0, sizeof(long long) * 4 * ncols,
                        cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaEventRecord(ctx->mm_ev, ctx->stream));
     ctx->mm_next += ncols;
@@ -760,7 +765,7 @@ static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTab
 
 static gpl_status launch_prepared_build(gpl_ctx* ctx, const PreparedBuild& P) {
   if (P.pipe) {
-    CK(cudaMemsetAsync(P.pdesc.ins_slots, 0, P.clear_bytes, ctx->stream));
+    CK(cudaMemsetAsync((char*)P.pdesc.ins_slots + P.clear_off, 0, P.clear_bytes, ctx->stream));
     CK(launch_pipeline_fn(P.pfn, P.pdesc, P.pgrid, ctx->stream));
   } else {
     CK(launch_build(P.desc, P.trivial, P.known, ctx->sms, ctx->stream));
@@ -919,6 +924,11 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
     P.pdesc = pd;
     P.pgrid = cfg.grid;
     P.clear_bytes = direct_counter_off(H.bytes()) + 16;
+    P.clear_off = 0;
+    if (pd.ins_dense) {  // the build writes every cell: clear only its tile counter
+      P.clear_off = direct_counter_off(H.bytes());
+      P.clear_bytes = 16;
+    }
   }
   P.desc = d;
   P.trivial = trivial;
@@ -1268,7 +1278,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     for (size_t i = 0; i + 1 < segs.size(); i++) {
       const PreparedBuild& B = ctx->build_cache.at(segs[i]);
       builds.push_back(&B);
-      if (B.pipe) add(B.pdesc.ins_slots, B.clear_bytes);
+      if (B.pipe) add((char*)B.pdesc.ins_slots + B.clear_off, B.clear_bytes);
     }
     const PreparedRun& R = *ctx->run_cache.at(run_key);
     add(counter_ptr(ctx), run_clear_bytes(run_pbytes(R.li)));

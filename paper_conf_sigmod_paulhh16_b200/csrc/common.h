@@ -204,7 +204,10 @@ struct PipeDesc {
   int32_t ins_kfield, ins_pfield, ins_ptransform, ins_width;  // queue fields, G_ID/G_YEAR, cell bytes (0 = bitmap)
   // stage-phase insert (every probe in the stage phase): key / payload stage
   // columns, or the payload's stage-probe slot; ins_kcol < 0: insert from the queue
-  int32_t ins_kcol, ins_pcol, ins_psreg, ins_pad;
+  // ins_dense (clustered build): the key column is sorted and the domain is its [min, max], so each
+  // packet writes its whole cell range — its rows' cells (0 when a row fails) and the key gaps between
+  // them — with plain stores: no atomics and no clear pass (P:147's blocking build, B200 form)
+  int32_t ins_kcol, ins_pcol, ins_psreg, ins_dense;
   long long ins_kmin, ins_pay_base;                            // run-time (table bases)
   unsigned long long ins_nslots;
   void* ins_slots;

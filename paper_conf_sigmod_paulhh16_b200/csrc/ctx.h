@@ -23,6 +23,7 @@ struct Column {
   int64_t cap_rows = 0;
   int64_t vmin = 0, vmax = 0;
   bool sorted = false;     // non-decreasing (e.g. lineitem.l_orderkey): enables clustered probe staging
+  bool strict = false;     // strictly increasing (a primary key in key order, e.g. orders.o_orderkey): dense builds
   std::vector<char> host;  // host-only context storage
 };
 
@@ -152,6 +153,7 @@ struct PreparedBuild {
   const void* pfn = nullptr;
   int pgrid = 0;
   size_t clear_bytes = 0;  // table cells + the trailing tile counter
+  size_t clear_off = 0;    // dense builds: only the tile counter (the build writes every cell)
 };
 
 // A0 load whose per-column min/max/sortedness are still in flight (a load
@@ -188,6 +190,7 @@ struct Options {
   int64_t hash_slots_log2 = 0; // hash group-by table size (tests): 0 = from the last run's distinct groups
   int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
   int64_t drain_warps = -1;    // operator-specialised drain warps (NEXT-1): -1 = the model's choice
+  int64_t dense_build = 1;     // sorted-key DIRECT builds write their cell ranges densely (no clear, no atomics)
   int64_t reg_fields = 1;      // JIT kernels keep drain-produced queue fields in registers
   int64_t zone_restrict = 1;   // scan only the row range of range filters on sorted columns
   int64_t agg_mode = -1;       // dense group accumulators: -1 exactness-driven choice, 2 = force global int128 atomics

@@ -182,6 +182,7 @@ std::string shape_source(const PipeDesc& d) {
   I("ins_ptransform", d.ins_ptransform);
   I("ins_width", d.ins_width);
   I("ins_kcol", d.ins_kcol);
+  I("ins_dense", d.ins_dense);
   I("ins_pcol", d.ins_pcol);
   I("ins_psreg", d.ins_psreg);
   I("smem_tables_bytes", d.smem_tables_bytes);

@@ -220,7 +220,16 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
   // table's upper-bound size (explicit 'hash mult|ordered' keeps hashing).
   if (!s.multi && shape->key_arity == 1 && (s.hash == -1 || s.hash == 2)) {
     const Column* kc = cols[d->k1];
-    const long long kmin = T.nrows ? kc->vmin : 0, kmax = T.nrows ? kc->vmax : 0;
+    long long kmin = T.nrows ? kc->vmin : 0, kmax = T.nrows ? kc->vmax : 0;
+    // a range filter on the key column itself bounds the inserted keys: the
+    // domain shrinks to it (Q9: p_partkey < 1000 -> a 1000-bit set instead of
+    // one bit per part), so the table can live in shared memory
+    for (const FilterIR& F : s.filters)
+      if (F.col == s.key[0] && F.kind == F_RANGE && T.nrows) {
+        kmin = std::max<long long>(kmin, F.lo);
+        kmax = std::min<long long>(kmax, F.hi);
+      }
+    if (kmax < kmin) kmax = kmin;
     const unsigned long long range = (unsigned long long)(kmax - kmin) + 1ull;
     int width = -1;
     if (!shape->has_payload) width = 0;
@@ -818,6 +827,16 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     if ((st = sorted_range(ctx, T, s.filters, &r0, &r1, err))) return st;
     for (int c = 0; c < d->ncols; c++) d->col[c] += r0 * d->colw[c];
     d->nrows = r1 - r0;
+    // clustered (dense) build: a DIRECT build whose key column is sorted and
+    // fully scanned, with the domain exactly [min, max] of that column, writes
+    // every cell of the domain exactly once (rows' cells + the gaps)
+    d->ins_dense = 0;
+    if (ins && d->ins_kcol >= 0 && ins->kind == HT_DIRECT && ins->width >= 1 && ctx->opt.dense_build != 0 &&
+        T.nrows > 0 && r0 == 0 && r1 == T.nrows) {
+      const Column& kc = *cols[d->ins_kcol];
+      // strictly increasing: no duplicate key can exist, each row owns one cell
+      if (kc.strict && ins->dkmin == kc.vmin && ins->dkmin + (long long)ins->dnslots - 1 == kc.vmax) d->ins_dense = 1;
+    }
   }
   li->nfilt = d->nfilt;
   li->nprobe = np;

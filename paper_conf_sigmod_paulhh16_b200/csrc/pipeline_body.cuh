@@ -715,6 +715,12 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           klo_n = __ldg(kcol + rown);
           khi_n = __ldg(kcol + rown + nn - 1);
         }
+        // dense build: the first key after this stage in ROW order (the next
+        // stage's, possibly another CTA's), or one past the domain at the end
+        int knext = 0;
+        if (K.ins_dense)
+          knext = row + n < d.nrows ? __ldg((const int*)d.col[K.ins_kcol] + row + n)
+                                    : (int)(d.ins_kmin + (long long)d.ins_nslots);
         mbar_wait(&empty[slot], phase ^ 1u);
         hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, last_of_tile ? 1 : 0);
         uint32_t bytes = 0;
@@ -738,8 +744,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             const long long sz = ((bhi + 15) & ~15ll) - cl_start;
             if (sz <= K.cl_cap) cl_size = (uint32_t)sz;
           }
-          hdr2[slot] = make_int4((int)(cl_start & 0xffffffff), (int)(cl_start >> 32), (int)cl_size, 0);
+          hdr2[slot] = make_int4((int)(cl_start & 0xffffffff), (int)(cl_start >> 32), (int)cl_size, knext);
           bytes += cl_size;
+        } else if (K.ins_dense) {
+          hdr2[slot] = make_int4(0, 0, 0, knext);
         }
         mbar_arrive_expect_tx(&full[slot], bytes);
         unsigned char* dst = g_smem + K.off_ring + (unsigned long long)slot * K.slot_bytes;
@@ -851,6 +859,8 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     if (n < 0) break;
     const uint32_t sb = (uint32_t)K.off_ring + slot * (uint32_t)K.slot_bytes;
     const long long rowbase = ((long long)h.y << 32) | (long long)(uint32_t)h.x;  // lazy-column gathers
+    // dense build: the first key after this stage in row order
+    const int ins_knext = K.ins_dense ? hdr2[slot].w : 0;
     // clustered probe: the staged cells cover keys [cl_k0, cl_k0 + cl_ncells)
     uint32_t cl_k0 = 0, cl_ncells = 0;
     int cl_size = 0;
@@ -973,6 +983,47 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
                               : K.ins_psreg == 0 ? sreg[0][q * RPL + j] : K.ins_psreg == 1 ? sreg[1][q * RPL + j] : 0;
           }
         }
+        if (K.ins_dense) {
+          // clustered (dense) build: the packet owns the cells from its first
+          // row's key to the next packet's first key (the next stage's, at a
+          // stage end); it zero-fills that range (aligned 16-B stores, byte
+          // stores at the edges it shares with its neighbours) and then writes
+          // the cells of its qualifying rows. The key column is strictly
+          // increasing (checked at load), so no key repeats and every cell of
+          // the domain is written exactly once per build: no atomics, no clear
+          // pass, no duplicate check.
+#pragma unroll
+          for (int q = 0; q < NPMAX; q++) {
+            if (!live[q]) continue;
+            const int pb = (it0 + q * Ws) << 7;  // the packet's first row in the stage
+            const uint32_t kcol_sa = smem_base() + sb + (uint32_t)K.coloff[K.ins_kcol];
+            const int first = lds_s32(kcol_sa + (uint32_t)pb * 4u);
+            const int next = pb + 128 < n ? lds_s32(kcol_sa + (uint32_t)(pb + 128) * 4u) : ins_knext;
+            const int w = K.ins_width;
+            char* cells = (char*)d.ins_slots;
+            const long long blo = ((long long)first - d.ins_kmin) * w, bhi = ((long long)next - d.ins_kmin) * w;
+            const long long alo = (blo + 15) & ~15ll, ahi = bhi & ~15ll;
+            if (alo < ahi) {
+              for (long long b = alo + lane * 16; b < ahi; b += 512) *(uint4*)(cells + b) = make_uint4(0u, 0u, 0u, 0u);
+              for (long long b = blo + lane; b < alo; b += 32) cells[b] = 0;
+              for (long long b = ahi + lane; b < bhi; b += 32) cells[b] = 0;
+            } else {
+              for (long long b = blo + lane; b < bhi; b += 32) cells[b] = 0;
+            }
+            __syncwarp();  // the zero fill is ordered before the cells below (same warp)
+#pragma unroll
+            for (int j = 0; j < RPL; j++) {
+              if (!p[q * RPL + j]) continue;
+              long long pv = px[q * RPL + j];
+              if (K.ins_ptransform == G_YEAR) pv = (int)pv / 10000;
+              const uint32_t v = (uint32_t)(pv - d.ins_pay_base + 1);
+              const long long c = kx[q * RPL + j] - d.ins_kmin;
+              if (w == 1) cells[c] = (char)v;
+              else if (w == 2) ((unsigned short*)cells)[c] = (unsigned short)v;
+              else ((uint32_t*)cells)[c] = v;
+            }
+          }
+        }
         // the ring slot is no longer read: release it before the atomics' round trip
 #pragma unroll
         for (int q = 0; q < NPMAX; q++)
@@ -981,7 +1032,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
             if (lane == 0) mbar_arrive(&empty[slot]);
             released = true;
           }
-        insert_cells<NR>(d, K, kx, px, p);
+        if (!K.ins_dense) insert_cells<NR>(d, K, kx, px, p);
         continue;
       }
       // A8 compaction into the warp's survivor queue (the on-chip channel), packet by packet

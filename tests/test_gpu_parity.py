@@ -761,3 +761,44 @@ def test_config3_sf10_q9_exact(ctx, db_sf10, bound):
     o = oracle.finalize("Q9", oracle.run("Q9", db, params, threads=oracle.host_threads()))
     assert r.keys == o.keys and r.aggs == o.aggs
     assert len(r.keys) == 175 and sum(a[0] for a in r.aggs) > (20_000 if bound == "literal" else 1_000_000)
+
+
+@pytest.mark.parametrize("q", ["Q5", "Q7", "Q8", "Q9", "Q3"])
+def test_dense_clustered_build_exact(ctx, q):
+    """Clustered (dense) builds: a DIRECT build keyed by a strictly increasing column (orders by
+    o_orderkey, customer by c_custkey, supplier by s_suppkey) writes every cell of its domain with plain
+    stores (no clear, no atomics); results equal the atomic build's and the oracle's, also on a ragged
+    orders table (rows dropped: the domain and the packet ranges change) and after a duplicate key makes
+    the column non-strict (the atomic build then detects it)."""
+    db = tpchgen.generate(0.05, seed=29)
+    o = _oracle(q, db)
+    if q == "Q3":
+        o = oracle.order_limit("Q3", oracle.run("Q3", db))
+    try:
+        for dense in (1, 0, 1):
+            ctx.set_option("dense_build", dense)
+            for _ in range(2):
+                r = _gpu(ctx, db, q)
+                assert r.keys == o.keys and r.aggs == o.aggs, (q, dense)
+    finally:
+        ctx.set_option("dense_build", 1)
+    # ragged: drop every 7th order (and its lineitems stay: FK misses drop them)
+    db2 = tpchgen.generate(0.05, seed=29)
+    keep = np.arange(db2.nrows("orders")) % 7 != 3
+    db2.tables["orders"] = {c: v[keep].copy() for c, v in db2.tables["orders"].items()}
+    o2 = oracle.run(q, db2)
+    o2 = oracle.order_limit("Q3", o2) if q == "Q3" else oracle.finalize(q, o2)
+    r2 = _gpu(ctx, db2, q)
+    assert r2.keys == o2.keys and r2.aggs == o2.aggs
+    # a repeated order key: the column is sorted but not strict -> atomic build -> DUPKEY
+    db3 = tpchgen.generate(0.05, seed=29)
+    ok_ = db3.tables["orders"]["o_orderkey"].copy()
+    ok_[1000] = ok_[999]
+    db3.tables["orders"]["o_orderkey"] = ok_
+    if q == "Q9":  # (its HT_O build inserts every order)
+        queries.load_database(ctx, db3, queries.TABLES[q])
+        queries.run_segments(ctx, queries.plan_text(q, db3))
+        with pytest.raises(gpl.GplError) as e:
+            ctx.fetch_result()
+        assert e.value.status == gpl.GPL_E_DUPKEY
+        ctx.sync()
