@@ -273,7 +273,9 @@ cudaError_t run_kbe(const PipeDesc& d, int sms, cudaStream_t s, void* pool, size
       const bool live = fs.ptr[f] || (first && f < d.npush && d.push[f].kind == PUSH_TERM);
       out.ptr[f] = live ? alloc((size_t)(total > 0 ? total : 1) * fs.w[f]) : nullptr;
     }
-    if (n > 0) kbe_scatter<<<grid_for(n, sms), kThreads, 0, s>>>(d, n, flags, pos, fs, out, first ? 1 : 0, nptr);
+    // (the scatter walks the whole input capacity: flags beyond the live rows are 0, and the
+    // count word already holds this operator's OUTPUT count)
+    if (n > 0) kbe_scatter<<<grid_for(n, sms), kThreads, 0, s>>>(d, n, flags, pos, fs, out, first ? 1 : 0, nullptr);
     fs = out;
     if (dev) nptr = d_total;  // every later kernel reads the live count
     return total;
