@@ -1732,7 +1732,7 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
                                                    : std::max<long long>(d.nrows, 1);
   PipeDesc dt = d;
   dt.nrows = tile;
-  const size_t need = kbe_pool_bytes(dt);
+  const size_t need = kbe_pool_bytes(dt, ctx->opt.kbe_tile_rows > 0);
   if (ctx->kbe_cap < need) {
     CK(cudaStreamSynchronize(ctx->stream));
     if (ctx->kbe_buf) cudaFree(ctx->kbe_buf);

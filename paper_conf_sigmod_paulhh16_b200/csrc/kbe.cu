@@ -198,11 +198,15 @@ int grid_for(long long n, int sms) {
 
 }  // namespace
 
-size_t kbe_pool_bytes(const PipeDesc& d) {
+size_t kbe_pool_bytes(const PipeDesc& d, bool device_sized) {
   // upper bound: flags + positions + two generations of every field + payloads + scan temp
   size_t per_row = 8;
-  for (int f = 0; f < d.nfield; f++) per_row += 2 * (size_t)d.qw[f];
+  size_t fw = 0;
+  for (int f = 0; f < d.nfield; f++) fw += (size_t)d.qw[f];
+  per_row += 2 * fw;
   per_row += 8 * (size_t)(d.nprobe + d.nresid + d.nfilt + 2) * 2;
+  // device-sized (GPL w/o CE): every operator's outputs are allocated at the full capacity
+  if (device_sized) per_row = (size_t)(d.nprobe + d.nresid + (d.nfilt > 0 ? 1 : 0) + 1) * (24 + fw) + 16;
   size_t tmp = 0;
   cub::DeviceScan::ExclusiveSum(nullptr, tmp, (int*)nullptr, (int*)nullptr, (int)(d.nrows > 0 ? d.nrows : 1));
   return per_row * (size_t)(d.nrows + 64) + 4 * (tmp + 4096) + (1 << 20);

@@ -78,7 +78,7 @@ cudaError_t launch_minmax_cols(const char* const* cols, const int* widths, int n
 // KBE baseline: kernel-at-a-time with materialisation. Returns the
 // bytes of intermediates written to HBM in *inter_bytes (host-side count).
 // `pool` must hold kbe_pool_bytes(d) bytes (per-context, reused).
-size_t kbe_pool_bytes(const PipeDesc& d);
+size_t kbe_pool_bytes(const PipeDesc& d, bool device_sized = false);
 // device_bytes != nullptr: device-sized buffers, no host round trip (GPL w/o CE tiles); the
 // materialised bytes accumulate in *device_bytes (device memory)
 cudaError_t run_kbe(const PipeDesc& d, int num_sms, cudaStream_t s, void* pool, size_t pool_bytes, double* inter_bytes,
