@@ -448,7 +448,27 @@ __global__ void sorted_bounds_kernel(const char* col, int w, long long n, long l
   out[1] = a;
 }
 
+// partition phase: the live row count = last offset + last count
+__global__ void part_total_kernel(const unsigned* hist, const unsigned* offs, size_t n, unsigned* total) {
+  *total = n ? offs[n - 1] + hist[n - 1] : 0u;
+}
+
 }  // namespace
+
+size_t part_scan_tmp_bytes(size_t n) {
+  size_t tmp = 0;
+  cub::DeviceScan::ExclusiveSum(nullptr, tmp, (unsigned*)nullptr, (unsigned*)nullptr, (int)n);
+  return tmp;
+}
+
+cudaError_t launch_part_scan(const unsigned* hist, unsigned* offs, size_t n, unsigned* total, void* tmp, size_t tmp_bytes,
+                             cudaStream_t s) {
+  size_t tb = tmp_bytes;
+  cudaError_t e = cub::DeviceScan::ExclusiveSum(tmp, tb, hist, offs, (int)n, s);
+  if (e != cudaSuccess) return e;
+  part_total_kernel<<<1, 1, 0, s>>>(hist, offs, n, total);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_sorted_bounds(const void* col, int w, long long n, long long lo, long long hi, long long* out,
                                  cudaStream_t s) {

@@ -393,6 +393,7 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
       if (h.hdr) cudaFree(h.hdr);
       if (h.pay) cudaFree(h.pay);
       if (h.aux) cudaFree(h.aux);
+      if (h.part_buf && h.part_buf != h.slots) cudaFree(h.part_buf);
     }
     if (ctx->d_scratch) cudaFree(ctx->d_scratch);
     for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
@@ -763,13 +764,162 @@ static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTab
   return GPL_OK;
 }
 
+// partition phase: count pass, exclusive scan of the counts, scatter pass (stream order is the
+// blocking barrier before the probe segment that scans the partitioned table)
+static gpl_status launch_partition(gpl_ctx* ctx, const PreparedBuild& P, cudaStream_t st) {
+  CK(launch_pipeline_fn(P.pfn, P.pdesc, P.pgrid, st));
+  CK(launch_part_scan(P.part_hist, P.part_offs, P.part_n, P.part_total, P.scan_tmp, P.scan_bytes, st));
+  CK(launch_pipeline_fn(P.pfn2, P.pdesc2, P.pgrid, st));
+  return GPL_OK;
+}
+
 static gpl_status launch_prepared_build(gpl_ctx* ctx, const PreparedBuild& P) {
+  if (P.part) return launch_partition(ctx, P, ctx->stream);
   if (P.pipe) {
     CK(cudaMemsetAsync((char*)P.pdesc.ins_slots + P.clear_off, 0, P.clear_bytes, ctx->stream));
     CK(launch_pipeline_fn(P.pfn, P.pdesc, P.pgrid, ctx->stream));
   } else {
     CK(launch_build(P.desc, P.trivial, P.known, ctx->sms, ctx->stream));
   }
+  return GPL_OK;
+}
+
+// A partition segment ("the partition phase also can be implemented in a
+// non-blocking manner"): the scanned rows that pass its operators are range-partitioned by the key
+// over the DIRECT domain of `by` into a derived table NAME (key + source row id) grouped by
+// partition. Two pipelined passes over the source (count per (partition, CTA) in shared memory, then
+// scatter at the CTA's own offsets) around one scan of the counts: no global atomics, no host round
+// trip. A later 'run NAME' probes the big table partition by partition (each partition's slice of
+// the table stays cache-resident) and gathers any other source column through the row id.
+static gpl_status build_partition(gpl_ctx* ctx, const Segment& s, const char* text, int32_t* ht_id) {
+  gpl_status st;
+  std::string err;
+  auto ti = ctx->tables.find(s.table);
+  if (ti == ctx->tables.end()) return fail(ctx, GPL_E_STATE, "unknown table '" + s.table + "'");
+  if (ti->second.derived) return fail(ctx, GPL_E_PLAN, "partition a base table");
+  const int64_t cap = std::max<int64_t>(ti->second.nrows, 1);
+  if (cap >= (1ll << 31)) return fail(ctx, GPL_E_PLAN, "partition source larger than 2^31 rows");
+  PipeDesc pd;
+  LowerInfo li;
+  if ((st = lower_probe(ctx, s, (int)s.probes.size(), &pd, &li, &err))) return fail(ctx, st, err);
+  Config cfg;
+  if (!choose_config(ctx, pd, li, pd.nrows, 0, &cfg, &err)) return fail(ctx, GPL_E_ARG, err);
+  apply_config(&pd, li, cfg);
+  const int key_ci = pd.ins_kcol;
+  // the output's placeholder entry (owns the buffers; probes by its name are rejected)
+  int idx;
+  auto it = ctx->ht_by_name.find(s.name);
+  if (it == ctx->ht_by_name.end()) {
+    idx = (int)ctx->hts.size();
+    ctx->hts.push_back(HashTable());
+    ctx->hts[idx].id = idx;
+    ctx->ht_by_name[s.name] = idx;
+  } else {
+    idx = it->second;
+  }
+  HashTable& H = ctx->hts[idx];
+  if (H.slots && H.kind != HT_PART) return fail(ctx, GPL_E_PLAN, "'" + s.name + "' is a hash table");
+  if (ctx->host_only) {
+    H.kind = HT_PART;
+    H.name = s.name;
+    H.valid = true;
+    if (ht_id) *ht_id = idx;
+  }
+  const size_t n = (size_t)s.nparts * (size_t)cfg.grid;
+  auto r256 = [](size_t b) { return (b + 255) / 256 * 256; };
+  const size_t tmp = part_scan_tmp_bytes(n);
+  const size_t need = 2 * r256(n * 4) + 256 + r256(tmp) + 2 * r256((size_t)cap * 4);
+  if (!ctx->host_only && (!H.part_buf || H.part_alloc < need)) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (H.part_buf) cudaFree(H.part_buf);
+    H.part_buf = nullptr;
+    H.part_alloc = 0;
+    cudaError_t e = cudaMalloc(&H.part_buf, need);
+    if (e != cudaSuccess) return fail(ctx, GPL_E_NOMEM, std::string("partition buffers: ") + cudaGetErrorString(e));
+    H.part_alloc = need;
+  }
+  char* b = (char*)H.part_buf;
+  PreparedBuild P;
+  P.part = true;
+  P.part_n = n;
+  P.part_hist = (unsigned*)b;
+  P.part_offs = (unsigned*)(b + r256(n * 4));
+  P.part_total = (unsigned*)(b + 2 * r256(n * 4));
+  P.scan_tmp = b + 2 * r256(n * 4) + 256;
+  P.scan_bytes = tmp;
+  int* keys = (int*)(b + 2 * r256(n * 4) + 256 + r256(tmp));
+  int* rows = (int*)((char*)keys + r256((size_t)cap * 4));
+  pd.part_hist = P.part_hist;
+  pd.part_key_out = keys;
+  pd.part_row_out = rows;
+  pd.tile_counter = counter_ptr(ctx);  // (static tiles: never claimed)
+  pd.op_pass = build_ops_ptr(ctx);
+  pd.err = err_ptr(ctx);
+  pd.partials = partials_ptr(ctx);
+  P.pdesc = pd;
+  P.pdesc2 = pd;
+  P.pdesc2.sink = SINK_PSCATTER;
+  P.pdesc2.part_hist = P.part_offs;  // the scatter starts each (partition, CTA) at its offset
+  P.pgrid = cfg.grid;
+  // the derived table: its key column + the source row id, `cap` rows of capacity
+  const Column* kc = ti->second.find(s.key[0]);
+  Table T;
+  T.name = s.name;
+  T.nrows = cap;
+  T.derived = true;
+  T.src_table = s.table;
+  T.nrows_dev = P.part_total;
+  Column ck;
+  ck.name = s.key[0];
+  ck.type = GPL_I32;
+  ck.width = 4;
+  ck.dev = (char*)keys;
+  ck.cap_rows = cap;
+  ck.vmin = kc ? kc->vmin : 0;
+  ck.vmax = kc ? kc->vmax : 0;
+  Column cr;
+  cr.name = T.rowid_col;
+  cr.type = GPL_I32;
+  cr.width = 4;
+  cr.dev = (char*)rows;
+  cr.cap_rows = cap;
+  cr.vmin = 0;
+  cr.vmax = cap - 1;
+  T.cols = {ck, cr};
+  auto old = ctx->tables.find(s.name);
+  bool same = old != ctx->tables.end() && old->second.derived && old->second.nrows == T.nrows &&
+              old->second.cols.size() == 2 && old->second.cols[0].dev == ck.dev && old->second.cols[1].dev == cr.dev &&
+              old->second.cols[0].name == ck.name && old->second.nrows_dev == T.nrows_dev && old->second.src_table == T.src_table;
+  T.version = same ? old->second.version : ctx->next_version++;
+  ctx->tables[s.name] = T;
+  if (ctx->host_only) return GPL_OK;
+  (void)key_ci;
+  std::string jerr;
+  P.pfn = resolve_pipeline_fn(P.pdesc, ctx->opt.jit != 0, &jerr);
+  P.pfn2 = resolve_pipeline_fn(P.pdesc2, ctx->opt.jit != 0, &jerr);
+  if (!P.pfn || !P.pfn2) return fail(ctx, GPL_E_CUDA, "cannot configure the partition kernels: " + jerr);
+  if ((st = launch_partition(ctx, P, ctx->stream))) return st;
+  H.kind = HT_PART;
+  H.name = s.name;
+  H.slots = H.part_buf;
+  H.src_table = s.table;
+  H.src_version = ti->second.version;
+  H.valid = true;
+  if (ht_id) *ht_id = idx;
+  P.ht_index = idx;
+  P.dest_ref = H.ref();
+  P.name = s.name;
+  P.table = s.table;
+  P.table_version = ti->second.version;
+  P.opt_version = ctx->opt_version;
+  for (int i = 0; i < pd.nht; i++)
+    for (auto& h : ctx->hts)
+      if (h.slots == pd.ht[i].slots && h.slots) {
+        P.src_ids.push_back(h.id);
+        break;
+      }
+  // cached only when every probed table was found (as for builds)
+  if ((int)P.src_ids.size() == pd.nht) ctx->build_cache[text] = P;
   return GPL_OK;
 }
 
@@ -797,6 +947,7 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
   std::string err;
   if (!parse_segment(build_segment, &s, &err)) return fail(ctx, GPL_E_PLAN, err);
   if (!s.is_build) return fail(ctx, GPL_E_PLAN, "expected a build segment ('build NAME')");
+  if (s.is_partition) return build_partition(ctx, s, build_segment, ht_id);
   gpl_status st;
   BuildDesc d;
   HashTable shape;
@@ -1165,11 +1316,12 @@ static std::vector<std::string> split_segments(const std::string& plan) {
     const std::string line = plan.substr(i, j - i);
     size_t k = line.find_first_not_of(" \t\r");
     const std::string head = k == std::string::npos ? "" : line.substr(k, line.find_first_of(" \t\r#", k) - k);
-    if ((head == "build" || head == "run") && cur_has_head) {
+    const bool seg_head = head == "build" || head == "partition" || head == "run";
+    if (seg_head && cur_has_head) {
       segs.push_back(cur);
       cur.clear();
     }
-    if (head == "build" || head == "run") cur_has_head = true;
+    if (seg_head) cur_has_head = true;
     cur += line + "\n";
     i = j + 1;
   }
@@ -1278,7 +1430,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     for (size_t i = 0; i + 1 < segs.size(); i++) {
       const PreparedBuild& B = ctx->build_cache.at(segs[i]);
       builds.push_back(&B);
-      if (B.pipe) add((char*)B.pdesc.ins_slots + B.clear_off, B.clear_bytes);
+      if (B.pipe && !B.part) add((char*)B.pdesc.ins_slots + B.clear_off, B.clear_bytes);
     }
     const PreparedRun& R = *ctx->run_cache.at(run_key);
     add(counter_ptr(ctx), run_clear_bytes(run_pbytes(R.li)));
@@ -1292,6 +1444,7 @@ GPL_API gpl_status gpl_run_query(gpl_ctx* ctx, const char* plan, int64_t tile_ro
     // lane that has fewer; the run joins both. Small dimension builds then
     // overlap instead of queueing behind each other.
     auto launch_b = [&](const PreparedBuild* B, cudaStream_t st) -> gpl_status {
+      if (B->part) return launch_partition(ctx, *B, st);
       if (B->pipe) CK(launch_pipeline_fn(B->pfn, B->pdesc, B->pgrid, st));
       else CK(launch_build(B->desc, B->trivial, B->known, ctx->sms, st));
       return GPL_OK;

@@ -52,7 +52,9 @@ struct Filt {
 // MULTI (non-unique build keys): CSR over a dense key
 //   domain — slots = uint32 offsets[nslots + 1], pay = int32 payload[count];
 //   key k's matches are pay[off[k - kmin] .. off[k - kmin + 1]) (fan-out join).
-enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2, HT_DIRECT = 3, HT_MULTI = 4 };
+// PART: not a hash table — the output of a partition segment (a derived table), registered by name so
+//   the query's segment bookkeeping (graphs, caches) treats it like a build.
+enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2, HT_DIRECT = 3, HT_MULTI = 4, HT_PART = 5 };
 enum : int32_t { H_MULT = 0, H_ORDERED = 1 };
 
 // Device-resident header, written by the build's count and size kernels and
@@ -124,7 +126,7 @@ struct Agg {
   int64_t c;
 };
 enum : int32_t { AGG_REG = 0, AGG_SMEM = 1, AGG_GLOBAL = 2, AGG_HASH = 3 };
-enum : int32_t { SINK_AGG = 0, SINK_INSERT = 1 };
+enum : int32_t { SINK_AGG = 0, SINK_INSERT = 1, SINK_PCOUNT = 2, SINK_PSCATTER = 3 };
 
 // ---- survivor-queue push: field <- stage column, stage-phase probe slot, or
 // a value term computed in the stage phase (expression pushdown)
@@ -219,6 +221,21 @@ struct PipeDesc {
   long long* hagg_accs;
   unsigned long long* hagg_count;
   int32_t hagg_log2, hagg_pad;
+  // partition phase (NEXT-4 partitioned hash join): SINK_PCOUNT counts the rows of each
+  // (partition, CTA) in a shared-memory histogram, SINK_PSCATTER writes (key, source row id) at the
+  // CTA's own offsets (exclusive scan of the counts, partition-major), so the output is grouped by
+  // partition with no global atomics. Partition of a key: (key - part_kmin) >> part_shift; keys outside
+  // [part_kmin, part_kmin + nparts << part_shift) cannot join and are dropped. Both passes use static
+  // tiles (CTA b takes tiles b, b + grid, ...) so a CTA sees the same rows twice.
+  long long part_kmin;
+  int32_t part_shift, nparts;
+  unsigned* part_hist;   // [nparts][grid] counts, then (after the scan) offsets
+  int* part_key_out;
+  int* part_row_out;
+  int32_t static_tiles, part_pad;
+  long long part_row0;   // row id of the first scanned row (zone restriction offset)
+  // rows to scan read from the device at kernel start (a partitioned table's row count; 0: nrows)
+  const unsigned* nrows_dev;
   // outputs
   unsigned long long* partials;      // [ngroups_total][nagg] x (lo, hi)
   unsigned long long* tile_counter;  // zeroed before launch

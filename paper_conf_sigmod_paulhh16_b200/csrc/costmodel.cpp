@@ -118,7 +118,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.feasible = c.smem <= ctx->smem_optin && k * (c.smem + 1024) <= 228 * 1024 && W >= 1 &&
                W <= pipeline_max_consumer_warps() && depth >= 2 && k * (W + 1) * 32 <= 2048 &&
                k * (W + 1) * 32 * regs_need <= 65536 && (npack == 1 || npack == 2) && ndrain >= 0 &&
-               ndrain <= 4 && W - ndrain >= 1 && (ndrain == 0 || (d.npush > 0 && !(d.sink == SINK_INSERT && d.ins_kcol >= 0)));
+               ndrain <= 4 && W - ndrain >= 1 && (ndrain == 0 || (d.npush > 0 && !(d.sink != SINK_AGG && d.ins_kcol >= 0)));
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
   // bytes per row: staged columns, plus one 32-B sector per surviving row of
@@ -241,7 +241,7 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
   std::vector<int> Ks = o.ctas_per_sm > 0 ? std::vector<int>{(int)o.ctas_per_sm} : std::vector<int>{1, 2};
   std::vector<int> Ps = o.packets > 0 ? std::vector<int>{(int)o.packets} : std::vector<int>{1, 2};
   // drain warps only for a segment with a queue phase (not a stage-phase insert)
-  const bool can_drain = d.npush > 0 && !(d.sink == SINK_INSERT && d.ins_kcol >= 0);
+  const bool can_drain = d.npush > 0 && !(d.sink != SINK_AGG && d.ins_kcol >= 0);
   std::vector<int> Dr = !can_drain ? std::vector<int>{0}
                         : o.drain_warps >= 0 ? std::vector<int>{(int)o.drain_warps} : std::vector<int>{0, 1, 2};
   Config best;

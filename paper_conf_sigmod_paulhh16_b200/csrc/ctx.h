@@ -32,6 +32,12 @@ struct Table {
   int64_t nrows = 0;
   uint64_t version = 0;
   std::vector<Column> cols;
+  // a partitioned table (the output of a partition segment, NEXT-4): nrows is its
+  // capacity, the live row count is written on the device; columns of src_table are
+  // reachable through the row-id column
+  bool derived = false;
+  std::string src_table, rowid_col = "rowid";
+  const unsigned* nrows_dev = nullptr;
   const Column* find(const std::string& n) const {
     for (auto& c : cols)
       if (c.name == n) return &c;
@@ -53,6 +59,9 @@ struct HashTable {
   int width = 0;
   long long dkmin = 0, pay_base = 0;
   unsigned long long dnslots = 0;
+  // partition segment output buffers (kind == HT_PART): counts, offsets, row count, key + row id columns
+  void* part_buf = nullptr;
+  size_t part_alloc = 0;
   // MULTI (fan-out): payload array and scan/scatter scratch
   void* pay = nullptr;
   size_t pay_alloc = 0;
@@ -154,6 +163,16 @@ struct PreparedBuild {
   int pgrid = 0;
   size_t clear_bytes = 0;  // table cells + the trailing tile counter
   size_t clear_off = 0;    // dense builds: only the tile counter (the build writes every cell)
+  // partition segment (NEXT-4 partitioned hash join): count pass, scan, scatter pass
+  bool part = false;
+  PipeDesc pdesc2{};        // the scatter pass (pdesc: the count pass)
+  const void* pfn2 = nullptr;
+  unsigned* part_hist = nullptr;  // [nparts][grid] counts
+  unsigned* part_offs = nullptr;  // ... their exclusive scan
+  unsigned* part_total = nullptr;
+  void* scan_tmp = nullptr;
+  size_t scan_bytes = 0;
+  size_t part_n = 0;
 };
 
 // A0 load whose per-column min/max/sortedness are still in flight (a load

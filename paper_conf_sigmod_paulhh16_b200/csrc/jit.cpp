@@ -183,6 +183,8 @@ std::string shape_source(const PipeDesc& d) {
   I("ins_width", d.ins_width);
   I("ins_kcol", d.ins_kcol);
   I("ins_dense", d.ins_dense);
+  I("static_tiles", d.static_tiles);
+  I("nparts", d.nparts);
   I("ins_pcol", d.ins_pcol);
   I("ins_psreg", d.ins_psreg);
   I("smem_tables_bytes", d.smem_tables_bytes);

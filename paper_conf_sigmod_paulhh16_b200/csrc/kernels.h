@@ -69,6 +69,10 @@ cudaError_t launch_minmax(const void* col, int width, long long n, long long* ou
 // [lower_bound(lo), upper_bound(hi)) of a sorted column (one thread; out[2] device)
 cudaError_t launch_sorted_bounds(const void* col, int w, long long n, long long lo, long long hi, long long* out,
                                  cudaStream_t s);
+// partition phase (NEXT-4): exclusive scan of the [nparts][grid] counts into offsets + the row count
+size_t part_scan_tmp_bytes(size_t n);
+cudaError_t launch_part_scan(const unsigned* hist, unsigned* offs, size_t n, unsigned* total, void* tmp, size_t tmp_bytes,
+                             cudaStream_t s);
 // device scan scratch of a MULTI (fan-out) build over nslots keys
 size_t multi_scan_tmp_bytes(unsigned long long nslots);
 // per-column {min, max, descents} of one table's columns in two launches (A0 load)

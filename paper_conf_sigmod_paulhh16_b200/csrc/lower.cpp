@@ -141,6 +141,7 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
     if (!H.valid) { *err = "hash table '" + P.ht + "' is stale (its table was reloaded)"; return GPL_E_STATE; }
     if (P.kind == P_MARK) { *err = "'mark' is not allowed in a build segment"; return GPL_E_PLAN; }
     if (H.kind == HT_MULTI) { *err = "a 'multi' table is probed by an inner 'probe' of a probe segment"; return GPL_E_PLAN; }
+    if (H.kind == HT_PART) { *err = "'" + P.ht + "' is a partitioned table (scan it with 'run')"; return GPL_E_PLAN; }
     if ((int)P.keys.size() != H.key_arity) { *err = "key arity mismatch probing " + P.ht; return GPL_E_PLAN; }
     if (!P.out.empty() && !H.has_payload) { *err = P.ht + " has no payload to bind to '" + P.out + "'"; return GPL_E_PLAN; }
     int k1, k2 = -1;
@@ -283,7 +284,10 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   *d = PipeDesc{};
   *li = LowerInfo{};
   li->table = s.table;
-  if (s.is_build && !ins) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
+  const bool part = s.is_build && s.is_partition;  // partition phase (NEXT-4 partitioned hash join)
+  if (s.is_build && !ins && !part) { *err = "expected a probe segment ('run TABLE')"; return GPL_E_PLAN; }
+  if (part && (!s.wheres.empty() || (int)s.probes.size() > MAXSP))
+    { *err = "a partition segment takes filters and at most 2 probes"; return GPL_E_PLAN; }
   d->cl_probe = d->cl_col = -1;
   d->fan_probe = -1;
   if (ins && (!s.is_build || ins->kind != HT_DIRECT || s.key.size() != 1)) {
@@ -313,6 +317,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     if (hit == ctx->ht_by_name.end()) { *err = "unknown hash table '" + P.ht + "'"; return GPL_E_STATE; }
     const HashTable& H = ctx->hts[hit->second];
     if (!H.valid) { *err = "hash table '" + P.ht + "' is stale (its table was reloaded)"; return GPL_E_STATE; }
+    if (H.kind == HT_PART) { *err = "'" + P.ht + "' is a partitioned table (scan it with 'run')"; return GPL_E_PLAN; }
     if ((int)P.keys.size() != H.key_arity) { *err = "key arity mismatch probing " + P.ht; return GPL_E_PLAN; }
     if (P.kind == P_INNER && !P.out.empty() && !H.has_payload) {
       *err = P.ht + " has no payload to bind to '" + P.out + "' (use semi or mark)";
@@ -355,21 +360,35 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   // staged columns
   std::vector<const Column*> cols;
   std::map<std::string, int> cidx;
+  // a partitioned (derived) table holds its key and the source row id; any other
+  // column of the source table is *indirect*: gathered through the row id (lazy)
+  const Table* src = nullptr;
+  if (T.derived) {
+    auto si = ctx->tables.find(T.src_table);
+    if (si == ctx->tables.end()) { *err = "the source table of '" + T.name + "' is not loaded"; return GPL_E_STATE; }
+    src = &si->second;
+  }
+  std::set<int> ind_col;  // indices (in cols) of indirect columns
   auto stage = [&](const std::string& n, int* out) -> gpl_status {
     auto it = cidx.find(n);
     if (it != cidx.end()) { *out = it->second; return GPL_OK; }
     const Column* c = T.find(n);
+    bool ind = false;
+    if (!c && src && (c = src->find(n))) ind = true;
     if (!c) { *err = "unknown column or slot '" + n + "'"; return GPL_E_STATE; }
     if ((int)cols.size() >= MAXC) { *err = "too many columns (max 8)"; return GPL_E_PLAN; }
     cidx[n] = (int)cols.size();
+    if (ind) ind_col.insert((int)cols.size());
     cols.push_back(c);
     *out = cidx[n];
     return GPL_OK;
   };
   gpl_status st;
   int tmp;
-  for (auto& f : s.filters)
+  for (auto& f : s.filters) {
     if ((st = stage(f.col, &tmp))) return st;
+    if (ind_col.count(tmp)) { *err = "filter on '" + f.col + "': filter the source in the partition segment"; return GPL_E_PLAN; }
+  }
   // probes keyed by an earlier probe's slot (a chained join, e.g. partsupp ->
   // supplier) run in the queue phase, where slots are queue fields
   int first_queue_only = np;
@@ -385,6 +404,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
       }
       if ((st = stage(k, &tmp))) return st;
       if (!is_int32(*cols[tmp])) { *err = "probe key '" + k + "' must be a 32-bit column"; return GPL_E_PLAN; }
+      if (ind_col.count(tmp)) first_queue_only = std::min(first_queue_only, p);  // gathered in the drain
     }
   if (d->fan_probe >= 0) first_queue_only = std::min(first_queue_only, d->fan_probe);
   if (ins && first_queue_only < np) { *err = "a pipelined build cannot probe by a slot"; return GPL_E_PLAN; }
@@ -409,6 +429,10 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   for (auto& a : s.aggs)
     if (a.kind >= A_SUMIF && !slot_of.count(a.slot)) { *err = "agg condition refers to unknown slot '" + a.slot + "'"; return GPL_E_PLAN; }
   const bool pay_slot = ins && ins->has_payload && slot_of.count(s.payload.name);
+  if (part) {  // the partition key is staged
+    if ((st = stage(s.key[0], &tmp))) return st;
+    if (!is_int32(*cols[tmp])) { *err = "partition keys must be 32-bit columns"; return GPL_E_PLAN; }
+  }
   if (ins) {  // build key and payload columns are staged too
     if ((st = stage(s.key[0], &tmp))) return st;
     if (!is_int32(*cols[tmp])) { *err = "build keys must be 32-bit columns"; return GPL_E_PLAN; }
@@ -432,7 +456,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   std::set<std::string> lazy;
   std::map<std::string, int> lazy_at;  // lazy column -> queue probe it is gathered before (np: the tail)
   const int nf0 = (int)s.filters.size();
-  if (!ins && ctx->opt.lazy_columns != 0 && T.nrows < (1ll << 31)) {
+  if (!ins && !part && !T.derived && ctx->opt.lazy_columns != 0 && T.nrows < (1ll << 31)) {
     auto lit = ctx->lambda.find(s.text);
     const std::vector<double>* lam =
         lit != ctx->lambda.end() && (int)lit->second.size() >= nf0 + np ? &lit->second : nullptr;
@@ -486,6 +510,26 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     }
   }
 
+  if (src) {  // every indirect column is gathered by row id right before its first use
+    const int nops_all = nf0 + np + (int)s.wheres.size();
+    auto first = [&](const std::string& c) {
+      int at = np;
+      for (int p = sp; p < np; p++)
+        for (auto& k : s.probes[p].keys)
+          if (k == c) at = std::min(at, p);
+      return at;
+    };
+    for (int c : ind_col) {
+      std::string name;
+      for (auto& kv : cidx)
+        if (kv.second == c) name = kv.first;
+      lazy.insert(name);
+      lazy_at[name] = first(name);
+      li->lazy_w.push_back(cols[c]->width);
+      const int at = lazy_at[name];
+      li->lazy_reach.push_back(at < np ? nf0 + at - 1 : nops_all - 1);
+    }
+  }
   // Expression pushdown: a value term whose factors are all columns, constants
   // or stage-phase slots is computed before the queue and carried as one field
   // (not when a factor is a lazy column: the drain computes it after the gather).
@@ -570,7 +614,13 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     }
   if (!lazy.empty()) {  // the row id the drain gathers lazy columns by
     if (nf >= MAXQ) { *err = "too many queue fields"; return GPL_E_PLAN; }
-    d->push[nf] = Push{PUSH_ROWID, 0};
+    if (src) {  // a derived table: the source row id is a staged column
+      int rc;
+      if ((st = stage(T.rowid_col, &rc))) return st;
+      d->push[nf] = Push{PUSH_COL, rc};
+    } else {
+      d->push[nf] = Push{PUSH_ROWID, 0};
+    }
     fw.push_back(4);
     d->rowid_field = nf++;
   }
@@ -607,6 +657,23 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->qbytes = std::max(off, 16);
   }
 
+  if (part) {
+    // partition phase: every probe in the stage phase, the sink reads the staged key
+    if (sp != np) { *err = "partition segment probes must all run in the stage phase"; return GPL_E_PLAN; }
+    auto hit = ctx->ht_by_name.find(s.by_ht);
+    if (hit == ctx->ht_by_name.end()) { *err = "partition by unknown hash table '" + s.by_ht + "'"; return GPL_E_STATE; }
+    const HashTable& PH = ctx->hts[hit->second];
+    if (PH.kind != HT_DIRECT) { *err = "partition by a DIRECT (dense key domain) table"; return GPL_E_PLAN; }
+    d->sink = SINK_PCOUNT;
+    d->ins_kcol = cidx[s.key[0]];
+    d->ins_pcol = d->ins_psreg = -1;
+    d->nparts = s.nparts;
+    int sh = 0;
+    while (((unsigned long long)s.nparts << sh) < PH.dnslots) sh++;
+    d->part_shift = sh;
+    d->part_kmin = PH.dkmin;
+    d->static_tiles = 1;
+  }
   if (ins) {
     d->sink = SINK_INSERT;
     d->ins_kfield = field[s.key[0]];
@@ -822,11 +889,15 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   li->bytes_per_row = bpr;
   li->bytes_per_row_all = bpr_all;
   d->nrows = T.nrows;
+  // a partitioned (derived) table: its row count is written on the device by the partition phase
+  d->nrows_dev = T.derived ? T.nrows_dev : nullptr;
   {  // scan only the row range the sorted filter columns allow (zone restriction)
     int64_t r0, r1;
     if ((st = sorted_range(ctx, T, s.filters, &r0, &r1, err))) return st;
-    for (int c = 0; c < d->ncols; c++) d->col[c] += r0 * d->colw[c];
+    for (int c = 0; c < d->ncols; c++)
+      if (!ind_col.count(c)) d->col[c] += r0 * d->colw[c];
     d->nrows = r1 - r0;
+    d->part_row0 = r0;  // partition phase: row ids are absolute rows of the scanned table
     // clustered (dense) build: a DIRECT build whose key column is sorted and
     // fully scanned, with the domain exactly [min, max] of that column, writes
     // every cell of the domain exactly once (rows' cells + the gaps)
@@ -863,6 +934,12 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   // every plan; registers / the smem table only where the bound above allows
   if (!s.hash_group && ctx->opt.agg_mode == AGG_GLOBAL) {
     d->agg_mode = AGG_GLOBAL;
+    d->flush_each_tile = 0;
+  }
+  if (part) {  // the per-CTA partition counts / cursors live in the shared table region
+    d->agg_mode = AGG_SMEM;
+    d->ngroups_total = li->ngroups_total = (s.nparts + 1) / 2;  // u64 words holding nparts u32
+    d->nagg = li->nagg = 1;
     d->flush_each_tile = 0;
   }
   return GPL_OK;

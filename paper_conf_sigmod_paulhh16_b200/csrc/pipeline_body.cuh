@@ -662,8 +662,14 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     }
   }
   for (int i = threadIdx.x; i < kMaxWarps * MAXOPS; i += blockDim.x) cnt_all[i] = 0;
-  if (K.agg_mode == AGG_SMEM)
+  if (K.agg_mode == AGG_SMEM && K.sink == SINK_AGG)
     for (int i = threadIdx.x; i < K.ngroups_total * K.nagg; i += blockDim.x) stab[i] = 0;
+  // partition phase: per-CTA counts (zeroed) or write cursors (this CTA's offsets after the scan)
+  if (K.sink == SINK_PCOUNT || K.sink == SINK_PSCATTER) {
+    unsigned* pc = &S<unsigned>(K.off_agg);
+    for (int i = threadIdx.x; i < K.nparts; i += blockDim.x)
+      pc[i] = K.sink == SINK_PCOUNT ? 0u : d.part_hist[(size_t)i * gridDim.x + blockIdx.x];
+  }
   __syncthreads();
 
   if (warp == W) {
@@ -676,11 +682,15 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
       // global-atomic round trip and — for a clustered probe — the loads of
       // the next stage's first/last key overlap the current stage's copies.
       const long long S = K.stage_rows;
-      unsigned long long t = atomicAdd(d.tile_counter, 1ull);
-      unsigned long long tn = atomicAdd(d.tile_counter, 1ull);  // claim of the following tile
+      // rows to scan: a partitioned table's row count lives on the device
+      const long long NROWS = d.nrows_dev ? (long long)*(const volatile unsigned*)d.nrows_dev : d.nrows;
+      // tiles: claimed dynamically, or (partition phase) statically — tile b, b + grid, ... — so both
+      // passes give a CTA the same rows
+      unsigned long long t = K.static_tiles ? (unsigned long long)blockIdx.x : atomicAdd(d.tile_counter, 1ull);
+      unsigned long long tn = K.static_tiles ? t + gridDim.x : atomicAdd(d.tile_counter, 1ull);  // the following tile
       long long r0 = (long long)t * d.tile_rows, s0 = 0;
       long long row = r0;
-      int n = r0 < d.nrows ? (int)min(S, min(d.tile_rows, d.nrows - r0)) : 0;
+      int n = r0 < NROWS ? (int)min(S, min(d.tile_rows, NROWS - r0)) : 0;
       // clustered probe: key range of the current stage. The keys are int32
       // and stay raw (no conversion) until their use in the NEXT iteration,
       // after the empty-slot wait: the next stage's two HBM loads are then
@@ -693,7 +703,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         khi = __ldg(kcol + row + n - 1);
       }
       while (n > 0) {
-        const long long rn = min(d.tile_rows, d.nrows - r0);
+        const long long rn = min(d.tile_rows, NROWS - r0);
         const bool last_of_tile = s0 + S >= rn;
         // next stage (same tile, else the claimed tile)
         long long r0n = r0, s0n = s0 + S, rown = 0;
@@ -704,10 +714,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         } else {
           r0n = (long long)tn * d.tile_rows;
           s0n = 0;
-          if (r0n < d.nrows) {
+          if (r0n < NROWS) {
             rown = r0n;
-            nn = (int)min(S, min(d.tile_rows, d.nrows - r0n));
-            tn = atomicAdd(d.tile_counter, 1ull);
+            nn = (int)min(S, min(d.tile_rows, NROWS - r0n));
+            tn = K.static_tiles ? tn + gridDim.x : atomicAdd(d.tile_counter, 1ull);
           }
         }
         int klo_n = 0, khi_n = 0;
@@ -719,7 +729,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         // stage's, possibly another CTA's), or one past the domain at the end
         int knext = 0;
         if (K.ins_dense)
-          knext = row + n < d.nrows ? __ldg((const int*)d.col[K.ins_kcol] + row + n)
+          knext = row + n < NROWS ? __ldg((const int*)d.col[K.ins_kcol] + row + n)
                                     : (int)(d.ins_kmin + (long long)d.ins_nslots);
         mbar_wait(&empty[slot], phase ^ 1u);
         hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, last_of_tile ? 1 : 0);
@@ -850,7 +860,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
   for (int i = 0; i < MAXF + MAXSP; i++) lc[i] = 0;
   // rows this warp queued = the pass count of the last stage-phase operator
-  const bool kQueueCounts = !(K.sink == SINK_INSERT && K.ins_kcol >= 0);
+  const bool kQueueCounts = !(K.sink != SINK_AGG && K.ins_kcol >= 0);  // (a stage-phase sink queues nothing)
   unsigned long long queued = 0;
   for (;;) {
     mbar_wait(&full[slot], phase);
@@ -961,6 +971,38 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           }
           if (!(kQueueCounts && sp == K.nsprobe - 1)) lc[K.nfilt + sp] += count_n(p);
         }
+      }
+      if ((K.sink == SINK_PCOUNT || K.sink == SINK_PSCATTER) && K.ins_kcol >= 0) {
+        // partition phase (NEXT-4 partitioned hash join): the rows that
+        // passed the segment's operators go to their key range's partition
+        unsigned* pc = &S<unsigned>(K.off_agg);
+#pragma unroll
+        for (int q = 0; q < NPMAX; q++) {
+          if (!live[q]) continue;
+          uint32_t k4[RPL];
+          ld_key32(d, K, K.ins_kcol, sb, r0q[q], rowbase, p + q * RPL, k4);
+#pragma unroll
+          for (int j = 0; j < RPL; j++) {
+            const uint32_t pid = (uint32_t)((long long)(int32_t)k4[j] - d.part_kmin) >> K.part_shift;
+            const bool in = p[q * RPL + j] && (long long)(int32_t)k4[j] >= d.part_kmin && pid < (uint32_t)K.nparts;
+            if (!in) continue;
+            if (K.sink == SINK_PCOUNT) {
+              atomicAdd(pc + pid, 1u);
+            } else {
+              const unsigned pos = atomicAdd(pc + pid, 1u);
+              d.part_key_out[pos] = (int)k4[j];
+              d.part_row_out[pos] = (int)(d.part_row0 + rowbase + r0q[q] + j);
+            }
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < NPMAX; q++)
+          if (live[q] && it0 + q * Ws + Ws >= nit) {
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[slot]);
+            released = true;
+          }
+        continue;
       }
       if (K.sink == SINK_INSERT && K.ins_kcol >= 0) {
         // build segment with every probe in the stage phase: insert straight
@@ -1148,7 +1190,12 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     for (int o = 0; o < nops; o++)
       if (cnt[o]) atomicAdd(d.op_pass + o, cnt[o]);
   }
-  if (K.agg_mode == AGG_SMEM) {
+  if (K.sink == SINK_PCOUNT) {  // this CTA's count of every partition (partition-major for the scan)
+    named_bar_sync(1, (uint32_t)W * 32u);
+    const unsigned* pc = &S<unsigned>(K.off_agg);
+    for (int i = threadIdx.x; i < K.nparts; i += W * 32) d.part_hist[(size_t)i * gridDim.x + blockIdx.x] = pc[i];
+  }
+  if (K.agg_mode == AGG_SMEM && K.sink == SINK_AGG) {
     named_bar_sync(1, (uint32_t)W * 32u);
     for (int i = threadIdx.x; i < K.ngroups_total * K.nagg; i += W * 32) {
       const long long v = (long long)stab[i];

@@ -248,8 +248,14 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
           seg->is_build = false;
           seg->table = expect_id(c, "table name");
           expect_end(c);
+        } else if (kw == "partition") {
+          // a blocking segment like a build ("the partition phase"), with a table as output
+          seg->is_build = true;
+          seg->is_partition = true;
+          seg->name = expect_id(c, "partitioned table name");
+          expect_end(c);
         } else {
-          throw ParseError{"segment must start with 'build NAME' or 'run TABLE'"};
+          throw ParseError{"segment must start with 'build NAME', 'partition NAME' or 'run TABLE'"};
         }
         have_head = true;
         continue;
@@ -274,8 +280,18 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
       } else if (kw == "key") {
         if (!seg->is_build) throw ParseError{"'key' only in build segments"};
         seg->key = parse_keys(c);
+        if (seg->is_partition) {
+          if (expect_id(c, "by") != "by") throw ParseError{"partition key needs 'by HT'"};
+          seg->by_ht = expect_id(c, "hash table");
+          if (seg->key.size() != 1) throw ParseError{"partition key is one column"};
+        }
+      } else if (kw == "parts") {
+        if (!seg->is_partition) throw ParseError{"'parts' only in partition segments"};
+        const int64_t P = expect_int(c, "partition count");
+        if (P < 2 || P > 4096 || (P & (P - 1))) throw ParseError{"parts: a power of two in [2, 4096]"};
+        seg->nparts = (int)P;
       } else if (kw == "payload") {
-        if (!seg->is_build) throw ParseError{"'payload' only in build segments"};
+        if (!seg->is_build || seg->is_partition) throw ParseError{"'payload' only in build segments"};
         seg->payload = parse_ref(c);
       } else if (kw == "hash") {
         std::string h = expect_id(c, "auto|direct|mult|ordered");
@@ -285,7 +301,7 @@ bool parse_segment(const std::string& text, Segment* seg, std::string* err) {
         else if (h == "auto") seg->hash = -1;
         else throw ParseError{"hash must be auto, direct, mult or ordered"};
       } else if (kw == "multi") {  // non-unique key: every match joins (NEXT-4 fan-out)
-        if (!seg->is_build) throw ParseError{"'multi' only in build segments"};
+        if (!seg->is_build || seg->is_partition) throw ParseError{"'multi' only in build segments"};
         seg->multi = true;
       } else if (kw == "load") {
         seg->load_pct = (int)expect_int(c, "percent");

@@ -93,6 +93,12 @@ struct Segment {
   RefIR payload;  // CONST kind => none
   int hash = -1;  // -1 auto, H_MULT, H_ORDERED, 2 = direct
   bool multi = false;  // 'multi': the key is not unique; probes join every match (NEXT-4 fan-out)
+  // partition segment (NEXT-4 partitioned hash join): 'partition NAME' ... 'key COL by HT' ['parts P']:
+  // the scanned rows that pass its operators are range-partitioned by COL over HT's key domain into the
+  // derived table NAME (COL + rowid), grouped by partition, which a later 'run NAME' segment probes
+  bool is_partition = false;
+  std::string by_ht;
+  int nparts = 1024;
   int load_pct = 50;
   // probe segment
   std::vector<WhereIR> wheres;

@@ -44,13 +44,16 @@ DEFAULT_PARAMS = {
     "Q14": (19950901, 19951001),  # P:688-689, [lo, hi)
     "Q3": (19950315,),            # TPC-H Q3 [EXT]: o_orderdate < d, l_shipdate > d
     "QF": (19950901, 19951001),   # NEXT-4 fan-out workload: l_shipdate in [lo, hi)
+    "Q5P": (19940101, 19950101),  # Q5's literals (partitioned hash join plan)
 }
 # the paper's queries (Listings 1-6)
 QUERIES = ["L1", "Q5", "Q7", "Q8", "Q9", "Q14"]
 # SURVEY §8(f) NEXT-4 workloads beyond the paper's FK->PK star joins with
 # declared group domains: TPC-H Q3 (hash group-by over unbounded keys + device
-# ORDER BY/LIMIT) and QF (a fan-out join on the non-unique ps_partkey)
-EXTRA_QUERIES = ["Q3", "QF"]
+# ORDER BY/LIMIT), QF (a fan-out join on the non-unique ps_partkey) and Q5P
+# (Q5 with a partitioned hash join into HT_O, for a lineitem not clustered by
+# l_orderkey; same result as Q5)
+EXTRA_QUERIES = ["Q3", "QF", "Q5P"]
 # fact-table (lineitem) columns each probe segment stages, for reporting
 FACT_COLUMNS = {
     "L1": ["l_shipdate", "l_extendedprice", "l_discount", "l_tax"],
@@ -61,6 +64,7 @@ FACT_COLUMNS = {
     "Q14": ["l_shipdate", "l_partkey", "l_extendedprice", "l_discount"],
     "Q3": ["l_shipdate", "l_orderkey", "l_extendedprice", "l_discount"],
     "QF": ["l_shipdate", "l_partkey", "l_extendedprice", "l_discount"],
+    "Q5P": ["l_orderkey", "l_suppkey", "l_extendedprice", "l_discount"],
 }
 # tables each query reads
 TABLES = {
@@ -72,6 +76,7 @@ TABLES = {
     "Q14": ["part", "lineitem"],
     "Q3": ["customer", "orders", "lineitem"],
     "QF": ["partsupp", "supplier", "lineitem", "nation"],
+    "Q5P": ["customer", "orders", "supplier", "lineitem", "nation", "region"],
 }
 
 
@@ -95,7 +100,7 @@ def plan_params(query: str, catalog, params=None) -> dict:
     p = tuple(params) if params is not None else DEFAULT_PARAMS[query]
     if query == "L1":
         return {"date_le": p[0]}
-    if query == "Q5":
+    if query in ("Q5", "Q5P"):
         return {"asia": ",".join(map(str, _nations_of_region(catalog, "ASIA"))), "od_lo": p[0],
                 "od_hi_incl": p[1] - 1}
     if query == "Q7":
@@ -128,11 +133,12 @@ def plan_text(query: str, catalog, params=None) -> str:
 
 
 def segments(text: str) -> list:
-    """Split a plan into segments at 'build NAME' / 'run TABLE' lines."""
+    """Split a plan into segments at 'build NAME' / 'partition NAME' / 'run TABLE' lines."""
     segs, cur = [], []
     for line in text.splitlines():
         head = line.strip().split()
-        if head and head[0] in ("build", "run") and any(x.strip() and not x.strip().startswith("#") for x in cur):
+        if head and head[0] in ("build", "partition", "run") and any(x.strip() and not x.strip().startswith("#")
+                                                                    for x in cur):
             segs.append("\n".join(cur))
             cur = []
         cur.append(line)
@@ -150,7 +156,7 @@ def plan_columns(text: str) -> dict:
             ln.split("#")[0] for ln in seg.splitlines()))
         table = None
         for i, w in enumerate(words):
-            if w in ("scan", "run") and i + 1 < len(words):
+            if w in ("scan", "run") and i + 1 < len(words):  # (a partitioned table is not a loaded input)
                 table = words[i + 1]
                 break
         for ln in seg.splitlines():  # A10 'decode key I TABLE KEYCOL -> OUTCOL' reads a dimension table
@@ -158,7 +164,14 @@ def plan_columns(text: str) -> dict:
             if len(w) >= 5 and w[0] == "decode" and w[2] in SCHEMA:
                 dc = need.setdefault(w[2], [])
                 dc += [c for c in w[3:5] if c not in dc]
-        if table is None or table not in SCHEMA:
+        if table is not None and table not in SCHEMA:
+            # a partitioned (derived) table: its other columns are gathered from the source table
+            for w in words:
+                for t, cs in SCHEMA.items():
+                    if w in cs and w not in need.setdefault(t, []):
+                        need[t].append(w)
+            continue
+        if table is None:
             continue
         cols = need.setdefault(table, [])
         for w in words:
