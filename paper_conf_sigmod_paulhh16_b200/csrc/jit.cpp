@@ -185,6 +185,7 @@ std::string shape_source(const PipeDesc& d) {
   I("ins_dense", d.ins_dense);
   I("static_tiles", d.static_tiles);
   I("nparts", d.nparts);
+  I("part_shift", d.part_shift);
   I("ins_pcol", d.ins_pcol);
   I("ins_psreg", d.ins_psreg);
   I("smem_tables_bytes", d.smem_tables_bytes);

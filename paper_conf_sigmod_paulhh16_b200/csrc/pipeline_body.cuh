@@ -684,53 +684,78 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
       const long long S = K.stage_rows;
       // rows to scan: a partitioned table's row count lives on the device
       const long long NROWS = d.nrows_dev ? (long long)*(const volatile unsigned*)d.nrows_dev : d.nrows;
-      // tiles: claimed dynamically, or (partition phase) statically — tile b, b + grid, ... — so both
-      // passes give a CTA the same rows
-      unsigned long long t = K.static_tiles ? (unsigned long long)blockIdx.x : atomicAdd(d.tile_counter, 1ull);
-      unsigned long long tn = K.static_tiles ? t + gridDim.x : atomicAdd(d.tile_counter, 1ull);  // the following tile
-      long long r0 = (long long)t * d.tile_rows, s0 = 0;
-      long long row = r0;
-      int n = r0 < NROWS ? (int)min(S, min(d.tile_rows, NROWS - r0)) : 0;
-      // clustered probe: key range of the current stage. The keys are int32
-      // and stay raw (no conversion) until their use in the NEXT iteration,
-      // after the empty-slot wait: the next stage's two HBM loads are then
-      // waited for behind the ring instead of stalling the producer (ncu:
-      // that stall gated every stage of Q5/Q7/Q8 at SF 100)
-      const int* kcol = K.cl_probe >= 0 ? (const int*)d.col[K.cl_col] : nullptr;
-      int klo = 0, khi = 0;
-      if (K.cl_probe >= 0 && n > 0) {
-        klo = __ldg(kcol + row);
-        khi = __ldg(kcol + row + n - 1);
-      }
-      while (n > 0) {
+      // Stage cursors: A is issued now, B next, C after B. Tiles are claimed
+      // dynamically (atomicAdd), or statically for the partition phase (tile
+      // b, b + grid, ...: both passes give a CTA the same rows); `tq` is the
+      // tile claimed for after C's, so a claim's latency is hidden behind the
+      // stages still ahead. Stage keys a clustered probe or a dense build needs
+      // (first / last / next row) are loaded for B one iteration ahead, and C's
+      // are prefetched into L2 two iterations ahead, so those loads hit L2 and
+      // never stall the producer on an HBM round trip (ncu: that stall capped
+      // the producer at ~1 stage per microsecond per CTA).
+      const bool need_keys = K.cl_probe >= 0 || K.ins_dense;
+      const int* kcol = K.cl_probe >= 0 ? (const int*)d.col[K.cl_col]
+                        : K.ins_dense ? (const int*)d.col[K.ins_kcol] : nullptr;
+      auto claim = [&](unsigned long long prev) -> unsigned long long {
+        return K.static_tiles ? prev + gridDim.x : atomicAdd(d.tile_counter, 1ull);
+      };
+      auto stage_n = [&](unsigned long long tt, long long so) -> int {  // rows of stage (tile tt, offset so)
+        const long long r0 = (long long)tt * d.tile_rows;
+        if (r0 >= NROWS) return 0;
         const long long rn = min(d.tile_rows, NROWS - r0);
-        const bool last_of_tile = s0 + S >= rn;
-        // next stage (same tile, else the claimed tile)
-        long long r0n = r0, s0n = s0 + S, rown = 0;
-        int nn = 0;
-        if (!last_of_tile) {
-          rown = r0 + s0n;
-          nn = (int)min(S, rn - s0n);
+        return so < rn ? (int)min(S, rn - so) : 0;
+      };
+      unsigned long long ta = K.static_tiles ? (unsigned long long)blockIdx.x : atomicAdd(d.tile_counter, 1ull);
+      long long sa = 0;
+      unsigned long long tq = claim(ta);
+      // advance a cursor by one stage (crossing into the queued tile)
+      auto advance = [&](unsigned long long& tt, long long& so) {
+        const long long r0 = (long long)tt * d.tile_rows;
+        const long long rn = r0 < NROWS ? min(d.tile_rows, NROWS - r0) : 0;
+        if (so + S < rn) {
+          so += S;
         } else {
-          r0n = (long long)tn * d.tile_rows;
-          s0n = 0;
-          if (r0n < NROWS) {
-            rown = r0n;
-            nn = (int)min(S, min(d.tile_rows, NROWS - r0n));
-            tn = K.static_tiles ? tn + gridDim.x : atomicAdd(d.tile_counter, 1ull);
-          }
+          tt = tq;
+          so = 0;
+          tq = claim(tq);
         }
-        int klo_n = 0, khi_n = 0;
-        if (K.cl_probe >= 0 && nn > 0) {
-          klo_n = __ldg(kcol + rown);
-          khi_n = __ldg(kcol + rown + nn - 1);
-        }
-        // dense build: the first key after this stage in ROW order (the next
-        // stage's, possibly another CTA's), or one past the domain at the end
-        int knext = 0;
-        if (K.ins_dense)
-          knext = row + n < NROWS ? __ldg((const int*)d.col[K.ins_kcol] + row + n)
-                                    : (int)(d.ins_kmin + (long long)d.ins_nslots);
+      };
+      unsigned long long tb = ta, tc;
+      long long sb_ = sa, sc;
+      advance(tb, sb_);
+      tc = tb;
+      sc = sb_;
+      advance(tc, sc);
+      auto row_of = [&](unsigned long long tt, long long so) { return (long long)tt * d.tile_rows + so; };
+      // keys of A (current) and B (next)
+      int klo = 0, khi = 0, knx = 0, klo_b = 0, khi_b = 0, knx_b = 0;
+      const int kend = (int)(d.ins_kmin + (long long)d.ins_nslots);  // dense build: one past the domain
+      auto load_keys = [&](unsigned long long tt, long long so, int& lo, int& hi, int& nx) {
+        const int nn = stage_n(tt, so);
+        if (!need_keys || nn <= 0) return;
+        const long long r = row_of(tt, so);
+        lo = __ldg(kcol + r);
+        hi = __ldg(kcol + r + nn - 1);
+        if (K.ins_dense) nx = r + nn < NROWS ? __ldg(kcol + r + nn) : kend;
+      };
+      auto prefetch_keys = [&](unsigned long long tt, long long so) {
+        const int nn = stage_n(tt, so);
+        if (!need_keys || nn <= 0) return;
+        const long long r = row_of(tt, so);
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(kcol + r));
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(kcol + r + nn - 1));
+        if (K.ins_dense && r + nn < NROWS) asm volatile("prefetch.global.L2 [%0];" ::"l"(kcol + r + nn));
+      };
+      load_keys(ta, sa, klo, khi, knx);
+      load_keys(tb, sb_, klo_b, khi_b, knx_b);
+      prefetch_keys(tc, sc);
+      for (;;) {
+        const int n = stage_n(ta, sa);
+        if (n <= 0) break;
+        const long long row = row_of(ta, sa);
+        const long long rn = min(d.tile_rows, NROWS - (long long)ta * d.tile_rows);
+        const bool last_of_tile = sa + S >= rn;
+        const int knext = knx;
         mbar_wait(&empty[slot], phase ^ 1u);
         hdr[slot] = make_int4((int)(row & 0xffffffff), (int)(row >> 32), n, last_of_tile ? 1 : 0);
         uint32_t bytes = 0;
@@ -770,12 +795,18 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           bulk_g2s(dst + K.cl_off, (const char*)htp[K.probe[K.cl_probe].ht].slots + cl_start, cl_size, &full[slot],
                    policy_evict_last());
         if (++slot == (uint32_t)K.depth) { slot = 0; phase ^= 1u; }
-        row = rown;
-        n = nn;
-        r0 = r0n;
-        s0 = s0n;
-        klo = klo_n;
-        khi = khi_n;
+        // A <- B (its keys were loaded an iteration ago), B <- C (prefetched into
+        // L2 an iteration ago: load its keys now), C <- the stage after C (prefetch)
+        ta = tb;
+        sa = sb_;
+        klo = klo_b;
+        khi = khi_b;
+        knx = knx_b;
+        tb = tc;
+        sb_ = sc;
+        load_keys(tb, sb_, klo_b, khi_b, knx_b);
+        advance(tc, sc);
+        prefetch_keys(tc, sc);
       }
       mbar_wait(&empty[slot], phase ^ 1u);
       hdr[slot] = make_int4(0, 0, -1, 0);
