@@ -29,7 +29,8 @@ from paper_conf_sigmod_paulhh16_b200 import gpl, queries  # noqa: E402
 
 out = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "gpurun_out", "verify_sf100.json")
 SF = float(sys.argv[2]) if len(sys.argv) > 2 else 100.0
-QS = ["Q14", "Q5", "Q7", "Q8", "Q9", "L1", "Q3"]
+QS = ["Q14", "Q5", "Q7", "Q8", "Q9", "L1", "Q3", "QF", "Q5P"]
+ORACLE_Q = {"Q5P": "Q5"}  # Q5P is Q5 through a partitioned hash join: the same SQL result
 PARAMS = {"L1": (19981101,)}  # the non-trivial Listing 1 variant (reading R1)
 T = oracle.host_threads()
 dev = torch.device("cuda", 0)
@@ -55,9 +56,10 @@ for q in QS:
     r = queries.run_query(ctx, q, full, PARAMS.get(q))  # a sized re-run (Q3's table) / graph replay
     rec.update(groups=len(r.keys), count=sum(a[0] for a in r.aggs), kernel_ms=r.stats["kernel_ms"])
     t = time.time()
-    o = oracle.run(q, full, PARAMS.get(q), threads=T)
+    oq = ORACLE_Q.get(q, q)
+    o = oracle.run(oq, full, PARAMS.get(q), threads=T)
     rec["oracle_s"] = time.time() - t
-    f = oracle.order_limit(q, o) if q == "Q3" else oracle.finalize(q, o)
+    f = oracle.order_limit(q, o) if q == "Q3" else oracle.finalize(oq, o)
     rec["oracle_rows_compared"] = full.nrows("lineitem")
     rec["oracle_groups"] = len(o.keys)
     ok = r.keys == f.keys and r.aggs == f.aggs
@@ -71,12 +73,31 @@ for q in QS:
     rec["ratios"] = r.ratios[:10]
     print(q, rec, flush=True)
     save()
+# the partitioned hash join where it matters: lineitem rows shuffled (not clustered by l_orderkey), Q5 as
+# the plain plan (random HT_O probes) and as Q5P (partition phase + partition-ordered probes); both must equal
+# the oracle's Q5 (row order does not change the SQL result)
+import numpy as np  # noqa: E402
+rng = np.random.default_rng(7)
+perm = rng.permutation(full.nrows("lineitem"))
+full.tables["lineitem"] = {c: v[perm] for c, v in full.tables["lineitem"].items()}
+del perm
+queries.load_database(ctx, full, ["lineitem"])
+want = oracle.finalize("Q5", oracle.run("Q5", full, threads=T))
+shuf = {}
+for q in ("Q5", "Q5P"):
+    r = None
+    for _ in range(4):
+        r = queries.run_query(ctx, q, full)
+    shuf[q] = {"kernel_ms": r.stats["kernel_ms"], "parity_full": bool(r.keys == want.keys and r.aggs == want.aggs)}
+record["shuffled_lineitem_q5"] = shuf
+print("shuffled", shuf, flush=True)
+save()
 ctx.close()
 del full
 
 ctx = gpl.Context(0, stream=torch.cuda.current_stream())
 W = 4
-dense = [q for q in QS if q != "Q3"]
+dense = [q for q in QS if q not in ("Q3", "Q5P")]
 parts = {q: [] for q in dense}
 for rk in range(W):
     shard = tpchgen.generate(SF, rank=rk, world=W)
@@ -94,6 +115,7 @@ for q in dense:
     queries.run_query(ctx, q, tiny, PARAMS.get(q))
     dec = ctx.decode_partials(merged)
     record["queries"][q]["additivity_4_shards"] = bool((dec.keys, dec.aggs) == res_full[q])
-record["all_ok"] = all(v["parity_full"] and v.get("additivity_4_shards", True) for v in record["queries"].values())
+record["all_ok"] = all(v["parity_full"] and v.get("additivity_4_shards", True) for v in record["queries"].values()) and \
+    all(v["parity_full"] for v in record["shuffled_lineitem_q5"].values())
 save()
 print(json.dumps({"all_ok": record["all_ok"]}))
