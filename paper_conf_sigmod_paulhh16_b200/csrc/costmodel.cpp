@@ -228,6 +228,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.t_probe_ms = 1e3 * probe_bytes / B;
   c.t_tail_ms = 1e3 * (T - N * b / B - probe_bytes / B);
   c.pred_ms = c.t_launch_ms + 1e3 * T;
+  c.t_cons_ms = 1e3 * tc;
   return c;
 }
 
@@ -307,6 +308,26 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
   };
   // the prediction is non-decreasing in the factor: geometric bisection
   double lo = 0.05, hi = 50;
+  // A run at (or under) the stream bound does not constrain the consumer cost: the
+  // consumers are then taken to be just fast enough — their own time equals the
+  // measured time — instead of arbitrarily fast (which would make shapes whose
+  // consumers are the bound, e.g. few CTAs on a large tile, look free).
+  auto cons_only = [&](double f) {
+    li->cons_factor = f;
+    const Config c = predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
+                             p.ctas_per_sm, p.npack, p.ndrain);
+    return c.t_cons_ms + c.t_launch_ms;
+  };
+  if (pred(lo) >= p.kernel_ms * 0.98) {
+    double clo = 0.05, chi = 50;
+    if (cons_only(clo) < p.kernel_ms && cons_only(chi) > p.kernel_ms) {
+      for (int i = 0; i < 40; i++) {
+        const double mid = std::sqrt(clo * chi);
+        (cons_only(mid) < p.kernel_ms ? clo : chi) = mid;
+      }
+      lo = std::sqrt(clo * chi);
+    }
+  }
   if (pred(lo) >= p.kernel_ms) {
     // faster than the stream bound (an L2-resident input): fit the streaming rate instead
     li->cons_factor = lo;

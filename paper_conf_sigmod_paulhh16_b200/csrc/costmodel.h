@@ -15,6 +15,7 @@ struct Config {
   int npack = 1;  // 128-row packets a consumer warp takes per iteration (1 or 2)
   int ndrain = 0; // of the consumer warps, those that only drain hand-off packets (NEXT-1)
   double pred_ms = 0, t_stream_ms = 0, t_probe_ms = 0, t_tail_ms = 0, t_launch_ms = 0, bw_gbs = 0;
+  double t_cons_ms = 0;  // the consumer warps' time alone (Eq 4 analog, all waves)
   bool feasible = false;
 };
 
