@@ -1123,6 +1123,29 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         }
         queued += (unsigned)(base - qcount);
         if (base != qcount) {
+          uint32_t ra4[RPL], ra8[RPL];  // a queued row's entry: queue base + position x width
+          {
+            const uint32_t qs = smem_base() + qb;
+#pragma unroll
+            for (int j = 0; j < RPL; j++) {
+              ra4[j] = qs + (uint32_t)pos[j] * 4u;
+              ra8[j] = qs + (uint32_t)pos[j] * 8u;
+            }
+          }
+          // late materialisation: the lazy columns the drain gathers first (before its
+          // first queue probe) are prefetched into L2 as their rows are queued, so the
+          // drain's dependent gather is an L2 hit, not an HBM round trip
+          if (K.rowid_field >= 0 && K.push[K.rowid_field].kind == PUSH_ROWID) {
+            GPL_UNROLL
+            for (int f = 0; f < K.nfield; f++) {
+              const int c = K.qlazy[f];
+              if (c < 0 || K.qlazy_at[f] != K.nsprobe) continue;
+#pragma unroll
+              for (int j = 0; j < RPL; j++)
+                if (p[q * RPL + j])
+                  asm volatile("prefetch.global.L2 [%0];" ::"l"(d.col[c] + (rowbase + r0 + j) * K.colw[c]));
+            }
+          }
           GPL_UNROLL
           for (int e = 0; e < K.npush; e++) {
             const Push& E = K.push[e];
@@ -1155,14 +1178,17 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
                 for (int j = 0; j < RPL; j++) v[j] *= F.a + (long long)F.b * x[j];
               }
             }
+            // (row addresses computed once per packet; the field offset is a
+            // compile-time immediate of the store in the plan-specialised kernel)
+            (void)qa;
             if (K.qw[e] == 4) {
 #pragma unroll
               for (int j = 0; j < RPL; j++)
-                if (p[q * RPL + j]) sts_32(smem_base() + qa + pos[j] * 4, (int)v[j]);
+                if (p[q * RPL + j]) sts_32(ra4[j] + (uint32_t)K.qoff[e], (int)v[j]);
             } else {
 #pragma unroll
               for (int j = 0; j < RPL; j++)
-                if (p[q * RPL + j]) sts_64(smem_base() + qa + pos[j] * 8, v[j]);
+                if (p[q * RPL + j]) sts_64(ra8[j] + (uint32_t)K.qoff[e], v[j]);
             }
           }
           qcount = base;
