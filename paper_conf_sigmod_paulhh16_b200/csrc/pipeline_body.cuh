@@ -1115,6 +1115,10 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
         const int r0 = r0q[q];
         int base = qcount;
         int pos[RPL];
+        // a packet with no survivor (most packets of a selective stage phase:
+        // Q9's 0.005%) skips the per-row ballots with one vote
+        const bool any_q = __any_sync(0xffffffffu, p[q * RPL] | p[q * RPL + 1] | p[q * RPL + 2] | p[q * RPL + 3]);
+        if (any_q) {
 #pragma unroll
         for (int j = 0; j < RPL; j++) {
           const unsigned m = __ballot_sync(0xffffffffu, p[q * RPL + j]);
@@ -1122,6 +1126,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           base += __popc(m);
         }
         queued += (unsigned)(base - qcount);
+        }
         if (base != qcount) {
           uint32_t ra4[RPL], ra8[RPL];  // a queued row's entry: queue base + position x width
           {
