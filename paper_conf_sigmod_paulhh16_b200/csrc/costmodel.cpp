@@ -217,18 +217,11 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   const double t_stage = S * b / rate_full;
   const double t_claim = std::max(0.0, 1.5e-6 - (depth - 1) * t_stage);  // producer's claim latency not hidden by the ring
   double t_prod = (waves - 1) * (t_tile + t_claim) + t_last + probe_bytes / B;
-  // Eq 6 analog (the channel): one producer per CTA issues a stage at a time —
-  // empty-slot handshake, header, one bulk copy per staged column and the
-  // clustered cells, the full-barrier round trip — measured on B200 (SF 100,
-  // v2 kernel) at ~0.5 us + the stage's bytes at ~40 GB/s per CTA; a CTA's
-  // stages are serial in it, so with one CTA per SM it bounds the run (Q7:
-  // 1.37 us per 4096-row stage at 1 CTA/SM), with two the SM gets two streams
-  const double stage_bytes = (double)S * li.bytes_per_row + (d.cl_probe >= 0 ? (double)cl_cap_bytes(d, S) * 0.5 : 0.0);
-  const double c_stage = 0.5e-6 + stage_bytes / 40e9;
+  // Eq 6 analog (ring handoff, ~mbarrier round trip per stage per CTA)
   const double stages_per_cta = (double)N / S / std::min<int64_t>(G, tiles);
-  const double t_chan = stages_per_cta * c_stage;
+  const double t_chan = stages_per_cta * 0.3e-6 / depth;
   // Eq 8/9 analog
-  const double tp = std::max(t_prod, t_chan), tc = t_cons;
+  const double tp = t_prod + t_chan, tc = t_cons;
   const double T = 0.5 * (tp + tc) + 0.5 * std::fabs(tp - tc);
   c.t_launch_ms = t0_cal >= 0 ? t0_cal : 4e-3 + 1e3 * (depth * t_stage);  // launch + prologue + ring fill
   c.t_stream_ms = 1e3 * (N * b / B);
