@@ -386,6 +386,7 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
   if (!ctx->host_only) {
     cudaSetDevice(ctx->device);
     cudaStreamSynchronize(ctx->stream);
+    if (ctx->mm_stream) cudaStreamSynchronize(ctx->mm_stream);  // min/max passes still reading columns
     for (auto& kv : ctx->tables)
       for (auto& c : kv.second.cols) free_column(ctx, c);
     for (auto& h : ctx->hts) {
@@ -413,7 +414,11 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
       if (e) cudaEventDestroy(e);
     if (ctx->ev0) cudaEventDestroy(ctx->ev0);
     if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+    if (ctx->mm_stream) cudaStreamSynchronize(ctx->mm_stream);
     if (ctx->mm_ev) cudaEventDestroy(ctx->mm_ev);
+    for (auto& e : ctx->mm_col_ev)
+      if (e) cudaEventDestroy(e);
+    if (ctx->mm_stream) cudaStreamDestroy(ctx->mm_stream);
     if (ctx->own_stream) cudaStreamDestroy(ctx->stream);
   }
   delete ctx;
@@ -548,7 +553,11 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
       CK(cudaMalloc(&ctx->d_minmax, kMinmaxSlots * 4 * sizeof(long long)));
       ctx->minmax_cap = kMinmaxSlots;
     }
-    if (!ctx->mm_ev) CK(cudaEventCreateWithFlags(&ctx->mm_ev, cudaEventDisableTiming));
+    if (!ctx->mm_ev) {
+      CK(cudaEventCreateWithFlags(&ctx->mm_ev, cudaEventDisableTiming));
+      CK(cudaStreamCreateWithFlags(&ctx->mm_stream, cudaStreamNonBlocking));
+      for (auto& e : ctx->mm_col_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
     if (ctx->mm_next + ncols > kMinmaxSlots && (st = resolve_pending(ctx))) return st;  // slots exhausted
     auto cleanup = [&]() {  // a failed reload hands reused buffers back to the old table
       auto oldt = ctx->tables.find(t.name);
@@ -611,21 +620,21 @@ GPL_API gpl_status gpl_load_columns(gpl_ctx* ctx, const char* table, int64_t nro
         t.cols.pop_back();
       }
       t.cols.push_back(c);
-    }
-    // per-column min/max/sortedness: one pass over the table's columns, read
-    // back into pinned slots WITHOUT synchronising (resolve_pending reads them
-    // at the first call that plans or validates)
-    const char* cp[64];
-    int cw[64];
-    for (int i = 0; i < ncols; i++) {
-      cp[i] = t.cols[i].dev;
-      cw[i] = t.cols[i].width;
+      // per-column min/max/sortedness on a side stream, as soon as the column
+      // has landed: the pass overlaps the next columns' copies (the copy engine
+      // and the SMs work at once), and nothing synchronises here — the pinned
+      // slots are read by resolve_pending at the first call that plans
+      const int slot = ctx->mm_next + i;
+      CK(cudaEventRecord(ctx->mm_col_ev[i], ctx->stream));
+      CK(cudaStreamWaitEvent(ctx->mm_stream, ctx->mm_col_ev[i], 0));
+      const char* cp1 = c.dev;
+      const int cw1 = c.width;
+      CK(launch_minmax_cols(&cp1, &cw1, 1, nrows, ctx->d_minmax + 4 * slot, ctx->mm_stream));
     }
     const int slot0 = ctx->mm_next;
-    CK(launch_minmax_cols(cp, cw, ncols, nrows, ctx->d_minmax + 4 * slot0, ctx->stream));
     CK(cudaMemcpyAsync(ctx->h_minmax + 4 * slot0, ctx->d_minmax + 4 * slot0, sizeof(long long) * 4 * ncols,
-                       cudaMemcpyDeviceToHost, ctx->stream));
-    CK(cudaEventRecord(ctx->mm_ev, ctx->stream));
+                       cudaMemcpyDeviceToHost, ctx->mm_stream));
+    CK(cudaEventRecord(ctx->mm_ev, ctx->mm_stream));
     ctx->mm_next += ncols;
     PendingLoad pl;
     pl.table = t.name;

@@ -247,6 +247,8 @@ struct gpl_ctx {
   std::vector<gpl::PendingLoad> pending;  // loads whose min/max are not read back yet
   int mm_next = 0;                        // next free column slot
   cudaEvent_t mm_ev = nullptr;            // recorded after the last pending load's min/max D2H
+  cudaStream_t mm_stream = nullptr;       // the min/max passes (overlap the next columns' copies)
+  cudaEvent_t mm_col_ev[64] = {};         // "column i landed" (ctx stream -> mm_stream)
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   // whole-query graphs: a second capture lane for build segments that do not
   // depend on each other (fork/join events, created on first use)
