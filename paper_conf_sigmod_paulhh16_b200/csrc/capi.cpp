@@ -1747,7 +1747,11 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
           for (const Config& x : cs)
             dup |= x.tile_rows == c.tile_rows && x.stage_rows == c.stage_rows && x.depth == c.depth &&
                    x.warps == c.warps && x.ctas_per_sm == c.ctas_per_sm && x.npack == c.npack && x.ndrain == c.ndrain;
-          if (!dup) cs.push_back(c);
+          if (dup) continue;
+          // ranked (and reported) by the fitted model like the rest
+          Config cf = predict(ctx, ds, ls, std::max<int64_t>(ds.nrows, 1), c.tile_rows, c.stage_rows, c.depth, c.warps,
+                              c.ctas_per_sm, c.npack, c.ndrain);
+          cs.push_back(cf);
         }
       }
       err.clear();
@@ -1789,9 +1793,11 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
     std::sort(ms.begin(), ms.end());
     tried++;
     if (std::getenv("GPL_DEBUG_TUNE"))
-      std::fprintf(stderr, "autotune: split %d(eff %d) k %d S %d D %d W %d dr %d np %d tile %lld: %.4f ms (model %.4f)\n",
+      std::fprintf(stderr, "autotune: split %d(eff %d) k %d S %d D %d W %d dr %d np %d tile %lld: %.4f ms (model %.4f)"
+                   " prod %.4f cons %.4f launch %.4f r_issue %.3f r_lat %.3f\n",
                    sc.first, cand_split_eff[ci], c.ctas_per_sm, c.stage_rows, c.depth, c.warps, c.ndrain, c.npack,
-                   (long long)c.tile_rows, ms[1], c.pred_ms);
+                   (long long)c.tile_rows, ms[1], c.pred_ms, c.t_prod_ms, c.t_cons_ms, c.t_launch_ms, c.r_issue,
+                   c.r_lat);
     if (ms[1] < best_ms) {
       best_ms = ms[1];
       best = t;

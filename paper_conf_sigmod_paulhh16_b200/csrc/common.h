@@ -173,7 +173,11 @@ struct PipeDesc {
                            // the group-by / value / sink), only for the rows still alive there
   // 1: fields the drain produces (f >= npush: lazy gathers, queue-probe slots) live in registers of the
   // plan-specialised kernel; the warp queues hold only the pushed fields (0: every field in the queue)
-  int32_t reg_fields, reg_pad;
+  int32_t reg_fields;
+  // AGG_SMEM: copies of the shared-memory group table, one per lane (32) when
+  // it fits, else 1; kept as separate low / high 32-bit word arrays so a row's
+  // add is two native 32-bit shared atomics (no 64-bit CAS loop)
+  int32_t agg_lanes;
   // clustered probe: stage probe cl_probe reads a DIRECT table by a key column
   // (cl_col) sorted in the fact table, so one stage's keys span a narrow cell
   // range; the producer TMA-stages those cells (<= cl_cap bytes at slot offset

@@ -58,7 +58,7 @@ int cl_cap_bytes(const PipeDesc& d, int S) {
 int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps, int ndrain) {
   // per-warp queues of the stage warps + the 2*ndrain hand-off slots
   int q = (warps + ndrain) * d.qbytes;
-  int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
+  int agg = d.agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 * std::max(1, d.agg_lanes) : 0;
   int slot = 0;
   for (int c = 0; c < d.ncols; c++)
     if (!d.lazy[c]) slot += align128(stage_rows * d.colw[c]);
@@ -76,7 +76,7 @@ void apply_config(PipeDesc* d, const LowerInfo& li, const Config& c) {
   d->ndrain = c.ndrain;
   d->off_queue = kFixed;
   d->off_agg = align128(kFixed + (c.warps + c.ndrain) * d->qbytes);
-  int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 : 0;
+  int agg = d->agg_mode == AGG_SMEM ? li.ngroups_total * li.nagg * 8 * std::max(1, d->agg_lanes) : 0;
   const int off_tables = d->off_agg + align128(agg);
   for (int i = 0; i < d->nht; i++)
     if (d->ht_smem_off[i] >= 0) d->ht_smem_off[i] += off_tables;  // relative -> absolute
@@ -125,9 +125,10 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // each lazy (gathered) column
   double b = std::max(1, li.bytes_per_row);
   for (size_t i = 0; i < li.lazy_reach.size(); i++) {
-    const int op = li.lazy_reach[i];
+    const int op = li.lambda.empty() ? -1 : li.lazy_reach[i];
     b += 32.0 * (op >= 0 && op < (int)li.lambda.size() ? li.lambda[op] : 0.05);
   }
+  if (d.cl_probe >= 0 && N > 0) b += li.cl_bytes / (double)N;  // the clustered probe's cells, streamed once
   const double f_sm = 1.9e9;
   // Eq 1 analog: the calibrated ring throughput Γ(n, s, k, d) of this shape at
   // d = N·b (gpl_calibrate) replaces the copy bandwidth as the streaming rate,
@@ -157,6 +158,9 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   const double L2_eff = 0.5 * ctx->l2_bytes;
   double probe_bytes = 0;
   for (int p = 0; p < li.nprobe; p++) {
+    // a clustered probe reads cells the producer streams (counted in b below), a
+    // shared-memory table never misses: only the other probes pay L2 misses
+    if (p == d.cl_probe || d.ht_smem_off[li.probe_ht[p]] >= 0) continue;
     double ht = li.ht_bytes.empty() ? 1 << 20 : (double)li.ht_bytes[li.probe_ht[p]];
     double cr = std::min(1.0, L2_eff / std::max(ht, 1.0));
     probe_bytes += reach[li.nfilt + p] * N * 32.0 * (1.0 - cr);
@@ -184,23 +188,52 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // latency is paid once per iteration (all npack*4 loads of a lane in flight)
   double rows_cyc;  // fact rows per cycle per SM the consumer warps sustain
   if (ndrain == 0) {
-    const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);
+    // A warp's iteration: the probe latencies, its work, and the stage hand-off
+    // (full-barrier wait + empty arrive, ~800 cycles) shared by the packets the
+    // warp takes from one stage. A second packet per iteration overlaps less than
+    // the latency sum suggests (register-limited ILP; 1.3x fitted on the SF 100
+    // autotune candidates of Q5-Q14, profiles/r2/experiments/).
+    const double ppw = std::max(1.0, (double)S / (128.0 * npack * W));
+    const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter) + 800.0 / ppw;
     const double w_eff = (double)std::min(W, S / (128 * npack)) * k;  // warps with work per stage
-    rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, w_eff * 128.0 * npack / crit);
+    // issue cap: 4 schedulers at ~60% issue efficiency (ncu: the best Q5 shape
+    // issues on 59-63% of cycles at 126 warp-instructions per 128 rows)
+    c.r_issue = 4.0 * 0.6 * 128.0 / instr_iter;
+    c.r_lat = w_eff * 128.0 * npack / (npack == 2 ? 1.3 : 1.0) / crit;
+    // the profile fit scales the latency-bound rate only (the instruction count
+    // is the kernel's own); the two bounds combine softly (p = 2), so more
+    // latency hiding still helps near the issue cap
+    const double rl = c.r_lat / std::max(li.cons_factor, 1e-3);
+    rows_cyc = 1.0 / std::sqrt(1.0 / (c.r_issue * c.r_issue) + 1.0 / (rl * rl));
   } else {
     // operator-specialised warps (NEXT-1): stage warps never block on the
     // queue phase; drain warps absorb qfrac of the rows at one 128-row packet
-    // per (queue latency + queue work). The consumers sustain the slower of
-    // the two groups; Eq 8's delay between them is what the ring and the
-    // hand-off slots must absorb (min() below: the faster group idles).
+    // per (queue latency + queue work + hand-off). The consumers sustain the
+    // slower of the two groups; Eq 8's delay between them is what the ring and
+    // the hand-off slots must absorb (min() below: the faster group idles).
+    // Same issue cap, latency scaling and soft combination as above.
     const int Wsg = W - ndrain;
-    const double crit_s = 150.0 + lat_stage + npack * stage_cost;
+    const double ppw = std::max(1.0, (double)S / (128.0 * npack * Wsg));
+    const double crit_s = 150.0 + lat_stage + npack * stage_cost + 800.0 / ppw;
     const double w_eff = (double)std::min(Wsg, S / (128 * npack)) * k;
-    const double r_stage = w_eff * 128.0 * npack / crit_s;
-    const double r_drain = qfrac > 0 ? (double)ndrain * k * 128.0 / (lat_queue + queue_cost + 60.0) / qfrac : 1e30;
-    rows_cyc = std::min(4.0 * 0.7 * 128.0 / instr_iter, std::min(r_stage, r_drain));
+    const double r_stage = w_eff * 128.0 * npack / (npack == 2 ? 1.3 : 1.0) / crit_s;
+    const double r_drain = qfrac > 0 ? (double)ndrain * k * 128.0 / (lat_queue + queue_cost + 60.0 + 800.0) / qfrac : 1e30;
+    c.r_issue = 4.0 * 0.6 * 128.0 / instr_iter;
+    c.r_lat = std::min(r_stage, r_drain);
+    const double rl = c.r_lat / std::max(li.cons_factor, 1e-3);
+    rows_cyc = 1.0 / std::sqrt(1.0 / (c.r_issue * c.r_issue) + 1.0 / (rl * rl));
   }
-  rows_cyc /= std::max(li.cons_factor, 1e-3);  // profile-fitted scale
+  {
+    // ring refill: a released slot is refilled after the producer's load latency
+    // (~1.5 us; +1 us with a clustered probe, whose cell range needs the stage's
+    // keys first); the other D-1 slots must cover it, or every stage exposes the
+    // rest (fitted on the SF 100 autotune candidates: depth 2 loses 15-30% on
+    // Q5/Q8 and nothing on Q9)
+    const double L_ring = 1.5e-6 + (d.cl_probe >= 0 ? 1.0e-6 : 0.0);
+    const double t_st = (double)S * k / (rows_cyc * f_sm);  // one stage's consumption
+    const double expo = std::max(0.0, L_ring - (depth - 1) * t_st);
+    rows_cyc *= t_st / (t_st + expo);
+  }
   const double R_cons = rows_cyc * f_sm * b;                                // bytes/s one SM's consumers absorb
   const double t_cons = (double)N / (rows_cyc * f_sm * ctx->sms);
 
@@ -229,6 +262,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.t_tail_ms = 1e3 * (T - N * b / B - probe_bytes / B);
   c.pred_ms = c.t_launch_ms + 1e3 * T;
   c.t_cons_ms = 1e3 * tc;
+  c.t_prod_ms = 1e3 * tp;
   return c;
 }
 

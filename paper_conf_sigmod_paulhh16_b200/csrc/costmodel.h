@@ -16,6 +16,8 @@ struct Config {
   int ndrain = 0; // of the consumer warps, those that only drain hand-off packets (NEXT-1)
   double pred_ms = 0, t_stream_ms = 0, t_probe_ms = 0, t_tail_ms = 0, t_launch_ms = 0, bw_gbs = 0;
   double t_cons_ms = 0;  // the consumer warps' time alone (Eq 4 analog, all waves)
+  double t_prod_ms = 0;  // the producer's time alone (Eq 5/6 analog: stream, probe misses, ring)
+  double r_issue = 0, r_lat = 0;  // consumer rows/cycle/SM at the issue cap and the latency bound (unscaled)
   bool feasible = false;
 };
 

@@ -217,12 +217,23 @@ __device__ __forceinline__ void ht_probe_n(const HTP& h, const int kind, const i
 // p[0] = low word, p[1] = high word (two's complement). Adds a signed int64.
 // Correct under concurrency: the low word wraps exactly once per carry seen
 // by the atomic that caused it.
+// 64-bit atomics on GLOBAL memory spelled out (a generic-address atomicAdd
+// also compiles a shared-memory CAS-loop branch that never runs here).
+__device__ __forceinline__ unsigned long long gatom_add_u64(unsigned long long* p, unsigned long long v) {
+  unsigned long long old;
+  asm volatile("atom.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ void gred_add_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("red.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
 __device__ __forceinline__ void atomic_add_i128(unsigned long long* p, long long v) {
   const unsigned long long lo = (unsigned long long)v;
-  const unsigned long long old = atomicAdd(p, lo);
+  const unsigned long long old = gatom_add_u64(p, lo);
   const unsigned long long carry = (old + lo) < old ? 1ull : 0ull;
   const unsigned long long hi = (v < 0 ? ~0ull : 0ull) + carry;
-  if (hi) atomicAdd(p + 1, hi);
+  if (hi) gred_add_u64(p + 1, hi);
 }
 
 __device__ __forceinline__ long long warp_sum_i64(long long v) {

@@ -136,6 +136,7 @@ std::string shape_source(const PipeDesc& d) {
   for (int f = 0; f < MAXQ; f++)
     o << "  k.qlazy[" << f << "] = " << d.qlazy[f] << "; k.qlazy_at[" << f << "] = " << d.qlazy_at[f] << ";\n";
   I("reg_fields", d.reg_fields);
+  I("agg_lanes", d.agg_lanes);
   auto term = [&](const char* arr, int t, const Term& T) {
     o << "  k." << arr << "[" << t << "].sign = " << T.sign << "; k." << arr << "[" << t << "].nfact = " << T.nfact << ";\n";
     for (int f = 0; f < T.nfact; f++)

@@ -930,6 +930,9 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->agg_mode = (total < lim && (int64_t)d->ngroups_total * d->nagg * 8 <= 48 * 1024) ? AGG_SMEM : AGG_GLOBAL;
     d->flush_each_tile = 0;
   }
+  // lane-private copies of a small shared-memory table (<= 16 KB for all 32):
+  // lanes of a warp never collide on a word, only the same lane of other warps
+  d->agg_lanes = d->agg_mode == AGG_SMEM && (int64_t)d->ngroups_total * d->nagg * 8 * 32 <= 16 * 1024 ? 32 : 1;
   // forced accumulator placement (tests): global int128 atomics are exact for
   // every plan; registers / the smem table only where the bound above allows
   if (!s.hash_group && ctx->opt.agg_mode == AGG_GLOBAL) {
@@ -941,6 +944,7 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->ngroups_total = li->ngroups_total = (s.nparts + 1) / 2;  // u64 words holding nparts u32
     d->nagg = li->nagg = 1;
     d->flush_each_tile = 0;
+    d->agg_lanes = 1;
   }
   return GPL_OK;
 }

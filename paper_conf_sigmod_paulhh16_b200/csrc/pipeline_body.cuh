@@ -285,6 +285,16 @@ __device__ __forceinline__ unsigned count4(const bool (&p)[RPL]) {
   return (unsigned)p[0] + (unsigned)p[1] + (unsigned)p[2] + (unsigned)p[3];
 }
 __device__ __forceinline__ bool any4(const bool (&p)[RPL]) { return p[0] | p[1] | p[2] | p[3]; }
+// v added mod 2^64 to the counter whose low word is lo[i] and high word
+// lo[words + i], with two native 32-bit shared atomics: the low word's carry
+// (old + v.lo wrapped) goes into the high word. Concurrent adds are exact; the
+// words are read only after the CTA's barrier.
+__device__ __forceinline__ void smem_add_split(unsigned* lo, int words, int i, unsigned long long v) {
+  const unsigned l = (unsigned)v, h = (unsigned)(v >> 32);
+  const unsigned old = atomicAdd(lo + i, l);
+  const unsigned up = h + (unsigned)(old + l < old);
+  if (up) atomicAdd(lo + words + i, up);
+}
 // rows per lane of one consumer iteration: up to two packets in the
 // plan-specialised kernel; the generic kernel keeps one (register budget)
 #ifdef GPL_JIT
@@ -479,7 +489,75 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
       insert_cells<RPL>(d, K, kx, px, p);
       return;
     }
-    unsigned long long* stab = &S<unsigned long long>(K.off_agg);
+    // the Listings' SELECT expression of row j (exact int64, bounded by the lowering)
+    auto row_value = [&](int j) -> long long {
+      long long val = 0;
+      GPL_UNROLL
+      for (int t = 0; t < K.nterm; t++) {
+        if (K.term_field[t] >= 0) {
+          val += fget(K.term_field[t], j);
+          continue;
+        }
+        const Term& T = K.term[t];
+        long long prod = T.sign;
+        GPL_UNROLL
+        for (int f = 0; f < T.nfact; f++) {
+          const Factor& F = T.f[f];
+          prod *= F.field < 0 ? F.a : F.a + (long long)F.b * fget(F.field, j);
+        }
+        val += prod;
+      }
+      return val;
+    };
+    auto agg_contrib = [&](int a, int j, long long val) -> long long {
+      const Agg& A = K.agg[a];
+      if (A.kind == A_SUM) return val;
+      if (A.kind == A_SUMIF) return fget(A.field, j) != 0 ? val : 0;
+      if (A.kind == A_SUMIFEQ) return fget(A.field, j) == A.c ? val : 0;
+      return 1;
+    };
+    // dense group id over the GROUP BY dimensions; false outside the domain
+    auto group_id = [&](int j, int& gid) -> bool {
+      gid = 0;
+      bool ok = true;
+      GPL_UNROLL
+      for (int g = 0; g < K.ngroup; g++) {
+        const GroupDim& G = K.gdim[g];
+        long long v = fget(G.field, j);
+        if (G.transform == G_YEAR) v = (int)v / 10000;
+        const long long o = v - G.lo;
+        if ((unsigned long long)o >= (unsigned long long)G.size) ok = false;
+        gid += (int)o * G.stride;
+      }
+      return ok;
+    };
+    if (K.agg_mode == AGG_SMEM) {
+      // Shared-memory group table: sm_100 has no native 64-bit shared-memory add
+      // (atom.shared.add.u64 is a CAS loop), so each add is two native 32-bit
+      // atomics on the table's low / high word arrays (smem_add_split); with
+      // lane-private copies (agg_lanes = 32) the lanes of a warp never hit the
+      // same word, so dense groups do not serialise a warp. The
+      // copies are summed mod 2^64 at the flush (exact: the lowering bounds
+      // every partial by rows x max|value| < 4.6e18).
+      const int L = K.agg_lanes, words = K.ngroups_total * K.nagg * L;
+      unsigned* lo = &S<unsigned>(K.off_agg);
+#pragma unroll
+      for (int j = 0; j < RPL; j++) {
+        if (!p[j]) continue;
+        int gid = 0;
+        if (!group_id(j, gid)) {
+          atomicOr(d.err, ERR_DOMAIN);
+          continue;
+        }
+        const long long val = row_value(j);
+        GPL_UNROLL
+        for (int a = 0; a < K.nagg; a++) {
+          const long long c = agg_contrib(a, j, val);
+          if (c != 0) smem_add_split(lo, words, (gid * K.nagg + a) * L + (L == 32 ? lane : 0), (unsigned long long)c);
+        }
+      }
+      return;
+    }
 #pragma unroll
     for (int j = 0; j < RPL; j++) {
       if (!p[j]) continue;
@@ -511,7 +589,7 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
             if (__ldcg(d.hagg_count) >= fill_limit) break;
             cur = atomicCAS(d.hagg_keys + h, 0ull, st);
             if (cur == 0ull) {
-              atomicAdd(d.hagg_count, 1ull);
+              gred_add_u64(d.hagg_count, 1ull);
               cur = st;
             }
           }
@@ -526,47 +604,17 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
         }
       }
       int gid = 0;
-      bool ok = true;
-      GPL_UNROLL
-      for (int g = 0; g < (K.agg_mode == AGG_HASH ? 0 : K.ngroup); g++) {
-        const GroupDim& G = K.gdim[g];
-        long long v = fget(G.field, j);
-        if (G.transform == G_YEAR) v = (int)v / 10000;
-        const long long o = v - G.lo;
-        if ((unsigned long long)o >= (unsigned long long)G.size) ok = false;
-        gid += (int)o * G.stride;
-      }
-      if (!ok) {
+      if (K.agg_mode != AGG_HASH && !group_id(j, gid)) {
         atomicOr(d.err, ERR_DOMAIN);
         continue;
       }
-      long long val = 0;
-      GPL_UNROLL
-      for (int t = 0; t < K.nterm; t++) {
-        if (K.term_field[t] >= 0) {
-          val += fget(K.term_field[t], j);
-          continue;
-        }
-        const Term& T = K.term[t];
-        long long prod = T.sign;
-        GPL_UNROLL
-        for (int f = 0; f < T.nfact; f++) {
-          const Factor& F = T.f[f];
-          prod *= F.field < 0 ? F.a : F.a + (long long)F.b * fget(F.field, j);
-        }
-        val += prod;
-      }
+      const long long val = row_value(j);
       GPL_UNROLL
       for (int a = 0; a < K.nagg; a++) {
-        const Agg& A = K.agg[a];
-        long long c = 1;
-        if (A.kind == A_SUM) c = val;
-        else if (A.kind == A_SUMIF) c = fget(A.field, j) != 0 ? val : 0;
-        else if (A.kind == A_SUMIFEQ) c = fget(A.field, j) == A.c ? val : 0;
+        const long long c = agg_contrib(a, j, val);
         if (K.agg_mode == AGG_REG) acc[a] += c;
         else if (c != 0) {
-          if (K.agg_mode == AGG_HASH) atomicAdd((unsigned long long*)d.hagg_accs + hslot * K.nagg + a, (unsigned long long)c);
-          else if (K.agg_mode == AGG_SMEM) atomicAdd(&stab[gid * K.nagg + a], (unsigned long long)c);
+          if (K.agg_mode == AGG_HASH) gred_add_u64((unsigned long long*)d.hagg_accs + hslot * K.nagg + a, (unsigned long long)c);
           else atomic_add_i128(d.partials + 2 * (gid * K.nagg + a), c);
         }
       }
@@ -662,8 +710,8 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
     }
   }
   for (int i = threadIdx.x; i < kMaxWarps * MAXOPS; i += blockDim.x) cnt_all[i] = 0;
-  if (K.agg_mode == AGG_SMEM && K.sink == SINK_AGG)
-    for (int i = threadIdx.x; i < K.ngroups_total * K.nagg; i += blockDim.x) stab[i] = 0;
+  if (K.agg_mode == AGG_SMEM && K.sink == SINK_AGG)  // low + high word arrays of every copy
+    for (int i = threadIdx.x; i < K.ngroups_total * K.nagg * K.agg_lanes; i += blockDim.x) stab[i] = 0;
   // partition phase: per-CTA counts (zeroed) or write cursors (this CTA's offsets after the scan)
   if (K.sink == SINK_PCOUNT || K.sink == SINK_PSCATTER) {
     unsigned* pc = &S<unsigned>(K.off_agg);
@@ -1262,9 +1310,13 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
   }
   if (K.agg_mode == AGG_SMEM && K.sink == SINK_AGG) {
     named_bar_sync(1, (uint32_t)W * 32u);
+    const int L = K.agg_lanes, words = K.ngroups_total * K.nagg * L;
+    const unsigned* lo = &S<unsigned>(K.off_agg);
     for (int i = threadIdx.x; i < K.ngroups_total * K.nagg; i += W * 32) {
-      const long long v = (long long)stab[i];
-      if (v != 0) atomic_add_i128(d.partials + 2 * i, v);
+      unsigned long long t = 0;  // the copies' sum mod 2^64
+      for (int l = 0; l < L; l++)
+        t += (unsigned long long)lo[i * L + l] | ((unsigned long long)lo[words + i * L + l] << 32);
+      if (t != 0) atomic_add_i128(d.partials + 2 * i, (long long)t);
     }
   }
 }

@@ -854,3 +854,45 @@ def test_q5_partitioned_parts_and_schedules(ctx):
         o = oracle.finalize("Q5", oracle.run("Q5", db))
         r = _gpu(ctx, db, "Q5P")
         assert r.keys == o.keys and r.aggs == o.aggs, n
+
+
+DENSE_GROUPS_PLAN = """run lineitem
+filter l_shipdate <= {date}
+group l_discount 0 11
+value l_extendedprice * (100 - l_discount) - l_extendedprice * l_quantity * (40 + l_tax)
+agg count
+agg sum"""
+
+
+@pytest.mark.parametrize("date", [19981101, 19950101])
+def test_smem_groups_dense_warp_aggregation(ctx, date):
+    """AGG_SMEM with nearly every row surviving into 11 groups: lane-private table copies, each add
+    two 32-bit shared atomics with the low word's carry, summed mod 2^64 at the flush — exercised
+    with every row adding, negative values and per-row magnitudes above 2^32 (carries both ways).
+    Expected values: exact Python-int sums over the numpy columns (a plain definition, no shared
+    code); also equal to the forced global int128 path."""
+    db = tpchgen.generate(0.2, seed=23)
+    L = db.tables["lineitem"]
+    keep = L["l_shipdate"] <= date
+    ep, d, q, t = (L[c][keep].astype(object) for c in ("l_extendedprice", "l_discount", "l_quantity", "l_tax"))
+    vals = ep * (100 - d) - ep * q * (40 + t)
+    want = {}
+    for g, v in zip(L["l_discount"][keep].tolist(), vals.tolist()):
+        c, s = want.get(g, (0, 0))
+        want[g] = (c + 1, s + v)
+    assert max(abs(v) for v in vals.tolist()) > 2**32 and min(vals.tolist()) < 0
+    queries.load_database(ctx, db, ["lineitem"])
+    plan = DENSE_GROUPS_PLAN.format(date=date)
+    ctx.run_query(plan)
+    r = ctx.fetch_result()
+    assert r.stats["agg_mode"] == 1
+    got = {k[0]: tuple(a) for k, a in zip(r.keys, r.aggs)}
+    assert len(want) == 11
+    assert got == want
+    try:
+        ctx.set_option("agg_mode", 2)
+        ctx.run_query(plan)
+        r2 = ctx.fetch_result()
+        assert r2.stats["agg_mode"] == 2 and (r2.keys, r2.aggs) == (r.keys, r.aggs)
+    finally:
+        ctx.set_option("agg_mode", -1)

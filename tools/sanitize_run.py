@@ -2,7 +2,7 @@
 synccheck), bit-exact vs the oracle: the paper plans (clustered probe, late materialisation with
 gathers at first use, register drain fields), Q3's hash group-by (device top-k and the full device sort),
 QF's fan-out join (multi build, chained probe), operator-specialised drain warps D = 1 and 2, forced
-global int128 accumulators, and the KBE / GPL (w/o CE) baselines. Eager runs and graph replays, SF 0.02."""
+global int128 accumulators, a dense shared-memory group-by (lane-private copies), and the KBE / GPL (w/o CE) baselines. Eager runs and graph replays, SF 0.02."""
 import os
 import sys
 
@@ -70,4 +70,22 @@ for _ in range(3):
 good = list(zip(r.keys, r.aggs)) == want
 ok &= good
 print("Q3 full device sort", "exact" if good else "MISMATCH")
+# dense shared-memory group-by: lane-private table copies, every row adding (exact Python-int sums)
+L = db.tables["lineitem"]
+want = {}
+for g, ep, q_, t in zip(L["l_discount"].tolist(), L["l_extendedprice"].tolist(), L["l_quantity"].tolist(),
+                        L["l_tax"].tolist()):
+    c, v = want.get(g, (0, 0))
+    want[g] = (c + 1, v + ep * (100 - g) - ep * q_ * (40 + t))
+dense = """run lineitem
+group l_discount 0 11
+value l_extendedprice * (100 - l_discount) - l_extendedprice * l_quantity * (40 + l_tax)
+agg count
+agg sum"""
+for _ in range(3):
+    ctx.run_query(dense)
+    r = ctx.fetch_result()
+good = r.stats["agg_mode"] == 1 and {k[0]: tuple(a) for k, a in zip(r.keys, r.aggs)} == want
+ok &= good
+print("dense smem groups", "exact" if good else "MISMATCH")
 sys.exit(0 if ok else 1)
