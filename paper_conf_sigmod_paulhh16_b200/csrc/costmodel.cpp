@@ -341,54 +341,53 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
                    p.ctas_per_sm, p.npack, p.ndrain).pred_ms;
   };
   // the prediction is non-decreasing in the factor: geometric bisection
-  double lo = 0.05, hi = 50;
-  // A run at (or under) the stream bound does not constrain the consumer cost: the
-  // consumers are then taken to be just fast enough — their own time equals the
-  // measured time — instead of arbitrarily fast (which would make shapes whose
-  // consumers are the bound, e.g. few CTAs on a large tile, look free).
-  auto cons_only = [&](double f) {
-    li->cons_factor = f;
-    const Config c = predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
-                             p.ctas_per_sm, p.npack, p.ndrain);
-    return c.t_cons_ms + c.t_launch_ms;
-  };
-  if (pred(lo) >= p.kernel_ms * 0.98) {
-    double clo = 0.05, chi = 50;
-    if (cons_only(clo) < p.kernel_ms && cons_only(chi) > p.kernel_ms) {
-      for (int i = 0; i < 40; i++) {
-        const double mid = std::sqrt(clo * chi);
-        (cons_only(mid) < p.kernel_ms ? clo : chi) = mid;
-      }
-      lo = std::sqrt(clo * chi);
+  const double lo = 0.05, hi = 50;
+  auto bisect = [](double a, double b, auto&& below) {  // below(x): the prediction at x is under the target
+    for (int i = 0; i < 40; i++) {
+      const double mid = std::sqrt(a * b);
+      (below(mid) ? a : b) = mid;
     }
-  }
-  if (pred(lo) >= p.kernel_ms) {
-    // faster than the stream bound (an L2-resident input): fit the streaming rate instead
+    return std::sqrt(a * b);
+  };
+  const char* path = "consumer";
+  if (pred(hi) <= p.kernel_ms) {
+    li->cons_factor = hi;
+  } else if (pred(lo) < p.kernel_ms) {
+    // the usual case: the consumers' latency-bound rate sets the time
+    li->cons_factor = bisect(lo, hi, [&](double f) { return pred(f) < p.kernel_ms; });
+  } else {
+    // at or under the model's stream bound (an L2-resident input, or a stream
+    // model too slow for this plan): fit the streaming rate to the run, then
+    // make the consumers just fast enough — their own time equals the measured
+    // time — instead of arbitrarily fast (which would make shapes whose
+    // consumers are the bound, e.g. few CTAs on a large tile, look free)
+    path = "stream";
     li->cons_factor = lo;
-    double blo = 1, bhi = 32;
     auto predb = [&](double f) {
       li->bw_factor = f;
       return pred(lo);
     };
-    if (predb(bhi) >= p.kernel_ms) return;
-    for (int i = 0; i < 40; i++) {
-      const double mid = std::sqrt(blo * bhi);
-      (predb(mid) > p.kernel_ms ? blo : bhi) = mid;
-    }
-    li->bw_factor = std::sqrt(blo * bhi);
-    // then the consumer scale at that rate
-    if (pred(lo) >= p.kernel_ms) return;
+    li->bw_factor = predb(32) >= p.kernel_ms ? 32 : bisect(1, 32, [&](double f) { return predb(f) > p.kernel_ms; });
+    auto cons_only = [&](double f) {
+      li->cons_factor = f;
+      const Config c = predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
+                               p.ctas_per_sm, p.npack, p.ndrain);
+      return c.t_cons_ms + c.t_launch_ms;
+    };
+    li->cons_factor = cons_only(lo) >= p.kernel_ms ? lo
+                      : cons_only(hi) <= p.kernel_ms ? hi
+                      : bisect(lo, hi, [&](double f) { return cons_only(f) < p.kernel_ms; });
   }
-  if (pred(hi) <= p.kernel_ms) { li->cons_factor = hi; return; }
-  for (int i = 0; i < 40; i++) {
-    const double mid = std::sqrt(lo * hi);
-    (pred(mid) < p.kernel_ms ? lo : hi) = mid;
-  }
-  li->cons_factor = std::sqrt(lo * hi);
-  if (std::getenv("GPL_DEBUG_MODEL"))
-    std::fprintf(stderr, "apply_profile: measured %.4f ms at S %d D %d W %d k %d np %d tile %lld N %lld -> cons %.3f bw %.3f pred %.4f\n",
+  if (std::getenv("GPL_DEBUG_MODEL")) {
+    const Config c = predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
+                             p.ctas_per_sm, p.npack, p.ndrain);
+    std::fprintf(stderr,
+                 "apply_profile: measured %.4f ms at S %d D %d W %d k %d np %d tile %lld N %lld -> %s cons %.3f bw %.3f "
+                 "pred %.4f (prod %.4f cons %.4f stream %.4f probe %.4f launch %.4f)\n",
                  p.kernel_ms, p.stage_rows, p.depth, p.warps, p.ctas_per_sm, p.npack, (long long)p.tile_rows,
-                 (long long)p.nrows, li->cons_factor, li->bw_factor, pred(li->cons_factor));
+                 (long long)p.nrows, path, li->cons_factor, li->bw_factor, c.pred_ms, c.t_prod_ms, c.t_cons_ms,
+                 c.t_stream_ms, c.t_probe_ms, c.t_launch_ms);
+  }
 }
 
 int choose_split(const gpl_ctx* ctx, const Segment& s) {

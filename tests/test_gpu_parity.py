@@ -473,11 +473,8 @@ def test_gamma_calibration_and_calibrated_model_exact(ctx):
     for p in pts:
         assert p["ms"] > p["t0_ms"] > 0 and 0 < p["gbs"] < 20000, p
         assert p["bytes"] == 16 * p["rows"]
-    # Γ grows with d (launch and ring fill amortised; "when the input is small, the channel is not
-    # fully utilized"): asserted for the best shape only — per-shape curves are timing data (reported by
-    # experiments.py gamma), not a parity property
-    best = {r: max(p["gbs"] for p in pts if p["rows"] == r) for r in (1 << 18, 1 << 21)}
-    assert best[1 << 21] > best[1 << 18]
+    # how Γ grows with d ("when the input is small, the channel is not fully utilized") is timing
+    # data, reported by experiments.py gamma (profiles/), not asserted in the parity suite
     seg = queries.segments(queries.plan_text("Q5", db))[-1]
     m = ctx.choose_tile_rows(seg, 0)
     assert 0 < m["bw_gbs"] < 20000
