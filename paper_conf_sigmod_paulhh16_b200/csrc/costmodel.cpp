@@ -185,67 +185,89 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // lazy columns: one HBM gather round trip per drain (per 128 queued rows)
   if (!li.lazy_reach.empty()) lat_queue += 2000.0;
   // cycles per warp iteration of `npack` packets: the stage-phase probe
-  // latency is paid once per iteration (all npack*4 loads of a lane in flight)
-  double rows_cyc;  // fact rows per cycle per SM the consumer warps sustain
-  if (ndrain == 0) {
-    // A warp's iteration: the probe latencies, its work, and the stage hand-off
-    // (full-barrier wait + empty arrive, ~800 cycles) shared by the packets the
-    // warp takes from one stage. A second packet per iteration overlaps less than
-    // the latency sum suggests (register-limited ILP; 1.3x fitted on the SF 100
-    // autotune candidates of Q5-Q14, profiles/r2/experiments/).
-    const double ppw = std::max(1.0, (double)S / (128.0 * npack * W));
-    const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter) + 800.0 / ppw;
-    const double w_eff = (double)std::min(W, S / (128 * npack)) * k;  // warps with work per stage
-    // issue cap: 4 schedulers at ~60% issue efficiency (ncu: the best Q5 shape
-    // issues on 59-63% of cycles at 126 warp-instructions per 128 rows)
-    c.r_issue = 4.0 * 0.6 * 128.0 / instr_iter;
-    c.r_lat = w_eff * 128.0 * npack / (npack == 2 ? 1.3 : 1.0) / crit;
-    // the profile fit scales the latency-bound rate only (the instruction count
-    // is the kernel's own); the two bounds combine softly (p = 2), so more
-    // latency hiding still helps near the issue cap
-    const double rl = c.r_lat / std::max(li.cons_factor, 1e-3);
-    rows_cyc = 1.0 / std::sqrt(1.0 / (c.r_issue * c.r_issue) + 1.0 / (rl * rl));
-  } else {
-    // operator-specialised warps (NEXT-1): stage warps never block on the
-    // queue phase; drain warps absorb qfrac of the rows at one 128-row packet
-    // per (queue latency + queue work + hand-off). The consumers sustain the
-    // slower of the two groups; Eq 8's delay between them is what the ring and
-    // the hand-off slots must absorb (min() below: the faster group idles).
-    // Same issue cap, latency scaling and soft combination as above.
-    const int Wsg = W - ndrain;
-    const double ppw = std::max(1.0, (double)S / (128.0 * npack * Wsg));
-    const double crit_s = 150.0 + lat_stage + npack * stage_cost + 800.0 / ppw;
-    const double w_eff = (double)std::min(Wsg, S / (128 * npack)) * k;
-    const double r_stage = w_eff * 128.0 * npack / (npack == 2 ? 1.3 : 1.0) / crit_s;
-    const double r_drain = qfrac > 0 ? (double)ndrain * k * 128.0 / (lat_queue + queue_cost + 60.0 + 800.0) / qfrac : 1e30;
-    c.r_issue = 4.0 * 0.6 * 128.0 / instr_iter;
-    c.r_lat = std::min(r_stage, r_drain);
-    const double rl = c.r_lat / std::max(li.cons_factor, 1e-3);
-    rows_cyc = 1.0 / std::sqrt(1.0 / (c.r_issue * c.r_issue) + 1.0 / (rl * rl));
-  }
-  {
-    // ring refill: a released slot is refilled after the producer's load latency
-    // (~1.5 us; +1 us with a clustered probe, whose cell range needs the stage's
-    // keys first); the other D-1 slots must cover it, or every stage exposes the
-    // rest (fitted on the SF 100 autotune candidates: depth 2 loses 15-30% on
-    // Q5/Q8 and nothing on Q9)
-    const double L_ring = 1.5e-6 + (d.cl_probe >= 0 ? 1.0e-6 : 0.0);
-    const double t_st = (double)S * k / (rows_cyc * f_sm);  // one stage's consumption
+  // latency is paid once per iteration (all npack*4 loads of a lane in flight).
+  // cons_rate(ka): fact rows per cycle per SM the consumer warps sustain with
+  // ka CTAs of this shape active on the SM (fewer than k in a last, partial wave)
+  const double cf = std::max(li.cons_factor, 1e-3);
+  // ring refill: a released slot is refilled after the producer's load latency
+  // (~1.2 us; twice that with a clustered probe whose cells come from HBM: its
+  // cell range needs the stage's keys first); the other D-1 slots must cover
+  // it, or every stage exposes the rest (fitted on the autotune candidates:
+  // depth 2 loses 15-30% on SF 100 Q5/Q8 and nothing on Q9; SF 1 Q5, cells in
+  // L2, exposes ~1.2 us per 512-row stage at depth 2)
+  const double L_ring = 1.2e-6 + (d.cl_probe >= 0 && li.cl_bytes > L2_eff ? 1.2e-6 : 0.0);
+  auto cons_rate = [&](double ka, Config* rep) -> double {
+    double r_issue, r_lat, rl;
+    if (ndrain == 0) {
+      // A warp's iteration: the probe latencies and its work (scaled by the
+      // profile fit), plus the stage hand-off (full-barrier wait + empty arrive,
+      // ~800 cycles, not scaled) shared by the packets the warp takes from one
+      // stage. A second packet per iteration overlaps less than the latency sum
+      // suggests (register-limited ILP; 1.3x fitted on the SF 100 autotune
+      // candidates of Q5-Q14, profiles/r2/experiments/).
+      const double ppw = std::max(1.0, (double)S / (128.0 * npack * W));
+      const double crit = 150.0 + lat_stage + npack * (qfrac * lat_queue + instr_iter);
+      const double w_eff = (double)std::min(W, S / (128 * npack)) * ka;  // warps with work per stage
+      const double num = w_eff * 128.0 * npack / (npack == 2 ? 1.3 : 1.0);
+      // issue cap: 4 schedulers at 70% issue efficiency (ncu: the best Q5 / Q9
+      // shapes sustain 57-61% of the SM's issue slots while not purely
+      // issue-bound; the soft combination below keeps a shape at the cap under it)
+      r_issue = 4.0 * 0.7 * 128.0 / instr_iter;
+      r_lat = num / (crit + 800.0 / ppw);
+      rl = num / (crit * cf + 800.0 / ppw);
+    } else {
+      // operator-specialised warps (NEXT-1): stage warps never block on the
+      // queue phase; drain warps absorb qfrac of the rows at one 128-row packet
+      // per (queue latency + queue work + hand-off). The consumers sustain the
+      // slower of the two groups; Eq 8's delay between them is what the ring and
+      // the hand-off slots must absorb (min() below: the faster group idles).
+      const int Wsg = W - ndrain;
+      const double ppw = std::max(1.0, (double)S / (128.0 * npack * Wsg));
+      const double crit_s = 150.0 + lat_stage + npack * stage_cost;
+      const double w_eff = (double)std::min(Wsg, S / (128 * npack)) * ka;
+      const double num = w_eff * 128.0 * npack / (npack == 2 ? 1.3 : 1.0);
+      const double crit_d = lat_queue + queue_cost + 60.0;
+      auto drain = [&](double f) {
+        return qfrac > 0 ? (double)ndrain * ka * 128.0 / (crit_d * f + 800.0) / qfrac : 1e30;
+      };
+      r_issue = 4.0 * 0.7 * 128.0 / instr_iter;
+      r_lat = std::min(num / (crit_s + 800.0 / ppw), drain(1.0));
+      rl = std::min(num / (crit_s * cf + 800.0 / ppw), drain(cf));
+    }
+    if (rep) {
+      rep->r_issue = r_issue;
+      rep->r_lat = r_lat;
+    }
+    // the profile fit scales the latency terms only (the instruction count is
+    // the kernel's own); the two bounds combine softly (p = 2), so more latency
+    // hiding still helps near the issue cap
+    double rows = 1.0 / std::sqrt(1.0 / (r_issue * r_issue) + 1.0 / (rl * rl));
+    const double t_st = (double)S * ka / (rows * f_sm);  // one stage's consumption
     const double expo = std::max(0.0, L_ring - (depth - 1) * t_st);
-    rows_cyc *= t_st / (t_st + expo);
-  }
-  const double R_cons = rows_cyc * f_sm * b;                                // bytes/s one SM's consumers absorb
-  const double t_cons = (double)N / (rows_cyc * f_sm * ctx->sms);
+    return rows * t_st / (t_st + expo);
+  };
 
   // Eq 3 analog: waves of Δ-row tiles over G persistent CTAs, with the last wave's tail
   const int64_t tiles = (N + tile - 1) / tile;
   const int64_t G = c.grid;
   const int64_t waves = (tiles + G - 1) / G;
   const int64_t last = tiles - (waves - 1) * G;
-  const double rate_full = std::min(std::min(B_sm, R_cons) / k, G_ring / (double)std::min<int64_t>(G, tiles));
-  const double rate_last = std::min(std::min(B_sm, R_cons) / k, G_ring / (double)last);
-  const double t_tile = tile * b / rate_full;
+  // CTAs with work per SM in the full waves and in the last one
+  auto ka_of = [&](int64_t active) {
+    return std::min<double>(k, std::max<double>(1.0, (double)((active + ctx->sms - 1) / ctx->sms)));
+  };
+  const int64_t act_full = std::min<int64_t>(G, tiles);
+  const double kf = ka_of(act_full), kl = ka_of(last);
+  const double rows_cyc = cons_rate(kf, &c), rows_last = cons_rate(kl, nullptr);
+  const double R_cons = rows_cyc * f_sm * b;  // bytes/s one SM's consumers absorb
+  // per-CTA rates (bytes/s): the SM's fill cap and consumers shared by its active
+  // CTAs, the device stream shared by every active CTA
+  const double rate_full = std::min(std::min(B_sm, R_cons) / kf, G_ring / (double)act_full);
+  const double rate_last = std::min(std::min(B_sm, rows_last * f_sm * b) / kl, G_ring / (double)last);
   const double last_rows = (double)(N - (tiles - 1) * tile);
+  const double t_cons = (waves - 1) * (double)tile / (rows_cyc * f_sm / kf) +
+                        (last == 1 ? last_rows : (double)tile) / (rows_last * f_sm / kl);
+  const double t_tile = tile * b / rate_full;
   const double t_last = (last == 1 ? last_rows : (double)tile) * b / rate_last;
   const double t_stage = S * b / rate_full;
   const double t_claim = std::max(0.0, 1.5e-6 - (depth - 1) * t_stage);  // producer's claim latency not hidden by the ring

@@ -133,17 +133,23 @@ def plan_text(query: str, catalog, params=None) -> str:
 
 
 def segments(text: str) -> list:
-    """Split a plan into segments at 'build NAME' / 'partition NAME' / 'run TABLE' lines."""
-    segs, cur = [], []
-    for line in text.splitlines():
-        head = line.strip().split()
-        if head and head[0] in ("build", "partition", "run") and any(x.strip() and not x.strip().startswith("#")
-                                                                    for x in cur):
-            segs.append("\n".join(cur))
-            cur = []
-        cur.append(line)
-    if any(x.strip() and not x.strip().startswith("#") for x in cur):
-        segs.append("\n".join(cur))
+    """Split a plan into segments at 'build NAME' / 'partition NAME' / 'run TABLE' lines — the same
+    texts gpl_run_query splits a plan into (every line newline-terminated, leading comments kept with
+    the first segment, trailing ones with the segment before them), so a segment run on its own shares
+    its prepared plan, λ and profile with the whole-query run."""
+    import re
+    segs, cur, has_head = [], "", False
+    for line in text.split("\n"):
+        s = line.lstrip(" \t\r")
+        head = re.split(r"[ \t\r#]", s, maxsplit=1)[0] if s else ""
+        seg_head = head in ("build", "partition", "run")
+        if seg_head and has_head:
+            segs.append(cur)
+            cur = ""
+        has_head |= seg_head
+        cur += line + "\n"
+    if has_head:
+        segs.append(cur)
     return segs
 
 
