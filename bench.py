@@ -181,7 +181,9 @@ def workload_config(args, rows_per_gpu, tile_rows):
             "query": args.query, "sf_total": args.sf, "lineitem_rows_per_gpu": rows_per_gpu,
             "seed": args.seed, "parallelism": f"dp{args.gpus} (order-key shards)" if args.gpus > 1 else "single",
             "l2": "flushed before every step (write of 2x L2); inputs are larger than L2",
-            "tile_rows": tile_rows or "A9 cost model"}
+            "tile_rows": tile_rows or "A9 cost model",
+            "shape": "gpl_autotune (model shortlist, measured)" if getattr(args, "shape", "model") == "autotune"
+            else "A9 cost model (profiled, no search)"}
 
 
 def main():
@@ -196,7 +198,10 @@ def main():
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-autotune", action="store_true")
+    ap.add_argument("--shape", default="model", choices=["model", "autotune"],
+                    help="pipeline shape: the A9 model's own pick after the plan's profiled runs (default), or "
+                         "gpl_autotune's measured best of the model's shortlist")
+    ap.add_argument("--no-autotune", action="store_true", help="(kept for scripts: same as --shape model)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -306,9 +311,9 @@ def main():
             res = ctx.fetch_result()
         return res
 
-    # calibrate the pipeline shape on the device (model shortlist, measured; untimed)
+    # --shape autotune: measure the model's shortlist on the device (untimed); default: the model's own pick
     tuned = None
-    if not args.no_autotune and args.tile_rows == 0:
+    if args.shape == "autotune" and not args.no_autotune and args.tile_rows == 0:
         tuned = ctx.autotune(text)
         log(f"[rank {rank}] autotune: {tuned}")
     # warm-up: W steps; without autotune at least 6, since the first runs profile

@@ -6,12 +6,16 @@
 //                                           (gpl ctx hbm_gbs, the measured copy BW)
 //   Eq 2 resource constraints             -> smem_bytes() <= 227 KB/CTA, warps <= 16
 //   Eq 3 req = wg / (a_wg * a_CU)         -> waves = ceil(ceil(N/Δ) / G), G = k * #SM
-//   Eq 4 compute cost (inst * w * req)    -> t_cons: warp-instructions per packet /
-//                                           (4 schedulers * f * #SM * eff)
+//   Eq 4 compute cost (inst * w * req)    -> t_cons: per warp iteration, probe latencies +
+//                                           warp-instructions (profile-scaled) + stage
+//                                           hand-off, over the warps with work; soft-capped
+//                                           by 4 schedulers * f * #SM * 70% issue; per wave
 //   Eq 5 memory cost, cache hit ratio cr  -> t_prod: (N*b + Σ_j λ_j N 32B (1-cr_j)) / B_eff,
 //                                           cr_j = min(1, L2_eff / HT_bytes_j)
 //   Eq 6 channel cost Δλ/Γ                -> ≈0: channels are on-chip smem queues;
-//                                           kept as the per-stage ring handoff cost
+//                                           kept as the per-stage ring handoff cost and
+//                                           the ring-refill latency the n-1 other slots
+//                                           must cover
 //   Eq 7 T_K = c_K + m_K                  -> per-role times t_prod (TMA warp), t_cons
 //   Eq 8 delay |T_i r_i - T_j r_j|        -> |t_prod - t_cons| between the two roles
 //   Eq 9 T_S = (1/C) Σ T_K + delay, C = 2 -> T = ½(t_prod + t_cons) + ½|t_prod - t_cons|
@@ -23,8 +27,8 @@
 // λ (Table 2, "query optimizer") comes from the previous run's per-operator
 // pass counters — the paper profiles the first tile for the same purpose.
 // Parity of this model is UNPINNED against the paper (its numbers were in the
-// missing figures); the tile sweep (bench.py --sweep) reports Eq 10's relative
-// error per Δ and the argmin gap.
+// missing figures); experiments.py knobs / model report Eq 10's relative error
+// over the config-2 sweep and the model's pick against gpl_autotune at SF 100.
 #include "costmodel.h"
 
 #include <algorithm>
