@@ -69,28 +69,30 @@ class ClockSampler:
         self.samples = []
         self._stop = threading.Event()
         self._t = None
+        self._nvml = None
+        try:  # NVML set up before the timed region, so even a short region is sampled
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self._nvml = (pynvml, h, pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM))
+        except Exception:
+            self._nvml = None
 
-    def _run_nvml(self):
-        import pynvml
-        pynvml.nvmlInit()
-        h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
-        mx = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+    def _sample_nvml(self):
+        pynvml, h, mx = self._nvml
         bits = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20, "sw_power_cap": 0x4}
-        while not self._stop.is_set():
-            sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
-            try:
-                r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
-            except AttributeError:  # older bindings
-                r = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
-            self.samples.append([str(sm), str(mx)] + ["Active" if r & b else "Not Active" for b in bits.values()])
-            self._stop.wait(0.005)
+        sm = pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)
+        try:
+            r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+        except AttributeError:  # older bindings
+            r = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+        self.samples.append([str(sm), str(mx)] + ["Active" if r & b else "Not Active" for b in bits.values()])
 
     def _run(self):
-        try:
-            self._run_nvml()
+        if self._nvml:
+            while not self._stop.wait(0.005):
+                self._sample_nvml()
             return
-        except Exception:
-            pass
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
@@ -103,11 +105,15 @@ class ClockSampler:
             self._stop.wait(0.1)
 
     def __enter__(self):
+        if self._nvml:
+            self._sample_nvml()  # the region's first moment
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
         return self
 
     def __exit__(self, *a):
+        if self._nvml:
+            self._sample_nvml()  # the region's last moment
         self._stop.set()
         self._t.join(timeout=10)
 
