@@ -747,21 +747,27 @@ static cudaError_t record_event(gpl_ctx* ctx, cudaEvent_t ev) {
 // A shape pinned by gpl_autotune (keyed by the segment text) wins over the
 // model; shortlist (optional) receives the model's per-shape candidates.
 static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTable& H, PipeDesc* pd, Config* cfg,
-                                   std::vector<Config>* shortlist = nullptr) {
+                                   std::vector<Config>* shortlist = nullptr, int force_split = -2) {
   LowerInfo li;
   std::string err;
   gpl_status st;
-  // every probe in the stage phase by default: the insert then runs straight
-  // from the staged tile, with no survivor queue (the probe_split option
-  // still applies, e.g. for tests of the queue path)
-  const int split = ctx->opt.probe_split >= -1 || s.split_hint >= -1 ? choose_split(ctx, s)
-                                                                      : std::min<int>((int)s.probes.size(), MAXSP);
+  // Probe split: the option / plan hint, else a split pinned by gpl_autotune,
+  // else the heuristic (choose_build_split): every probe in the stage phase (the
+  // insert runs straight from the staged tile, no survivor queue) unless the
+  // filters keep <= 5% of the rows (then the probes and the insert run in the
+  // drain on the queued survivors). The build's pass fractions are estimated
+  // from column statistics until known.
+  if (!ctx->lambda.count(s.text)) ctx->lambda[s.text] = build_lambda_estimate(ctx, s);
+  auto tu = shortlist ? ctx->tuned.end() : ctx->tuned.find(s.text);
+  int split = ctx->opt.probe_split >= -1 || s.split_hint >= -1 ? choose_split(ctx, s) : choose_build_split(ctx, s);
+  if (force_split >= -1) split = force_split < 0 ? (int)s.probes.size() : force_split;
+  else if (tu != ctx->tuned.end() && tu->second.split >= -1 && ctx->opt.probe_split < -1 && s.split_hint < -1)
+    split = tu->second.split < 0 ? (int)s.probes.size() : tu->second.split;
   if ((st = lower_probe(ctx, s, split, pd, &li, &err, &H))) return fail(ctx, st, err);
   for (int i = 0; i < pd->nht; i++) {
     const HashTable& h = ctx->hts[li.ht_ids[i]];
     li.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
   }
-  auto tu = shortlist ? ctx->tuned.end() : ctx->tuned.find(s.text);
   if (tu != ctx->tuned.end()) {
     const TunedShape& t = tu->second;
     *cfg = predict(ctx, *pd, li, std::max<int64_t>(pd->nrows, 1), t.tile_rows, t.stage_rows, t.depth, t.warps,
@@ -1587,38 +1593,51 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
   const HashTable H = ctx->hts[hi->second];
   if (H.kind != HT_DIRECT) return GPL_OK;
   ctx->tuned.erase(s.text);
-  PipeDesc pd;
-  Config c0;
-  std::vector<Config> cs;
-  gpl_status st = lower_build_pipe(ctx, s, H, &pd, &c0, &cs);
-  if (st) return st;
-  if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
-  {
-    LowerInfo lb;  // the build pipeline's facts for the warp variants (as lower_build_pipe computed them)
-    PipeDesc pb;
-    std::string e2;
-    const int split = ctx->opt.probe_split >= -1 || s.split_hint >= -1 ? choose_split(ctx, s)
-                                                                        : std::min<int>((int)s.probes.size(), MAXSP);
-    if (lower_probe(ctx, s, split, &pb, &lb, &e2, &H) == GPL_OK) {
-      for (int i = 0; i < pb.nht; i++) {
-        const HashTable& h = ctx->hts[lb.ht_ids[i]];
-        lb.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+  // candidates per probe split: every probe in the stage phase, and (a build
+  // with filters before its probes) the probes + insert in the queue phase
+  const int np = (int)s.probes.size();
+  std::vector<int> splits{-1};
+  if (np > 0 && !s.filters.empty() && ctx->opt.probe_split < -1 && s.split_hint < -1) splits.push_back(0);
+  std::vector<std::pair<Config, int>> cands;  // (shape, split)
+  for (int sp : splits) {
+    PipeDesc pd;
+    Config c0;
+    std::vector<Config> cs;
+    gpl_status st = lower_build_pipe(ctx, s, H, &pd, &c0, &cs, sp);
+    if (st) return st;
+    if (max_candidates > 0 && (int)cs.size() > max_candidates) cs.resize(max_candidates);
+    {
+      LowerInfo lb;  // the build pipeline's facts for the warp variants (as lower_build_pipe computed them)
+      PipeDesc pb;
+      std::string e2;
+      if (lower_probe(ctx, s, sp < 0 ? np : sp, &pb, &lb, &e2, &H) == GPL_OK) {
+        for (int i = 0; i < pb.nht; i++) {
+          const HashTable& h = ctx->hts[lb.ht_ids[i]];
+          lb.ht_bytes[i] = (int64_t)(h.kind == HT_DIRECT ? h.bytes() : h.bytes() / 2);
+        }
+        with_warp_variants(ctx, pb, lb, pb.nrows, &cs);
       }
-      with_warp_variants(ctx, pb, lb, pb.nrows, &cs);
     }
+    bool has0 = false;
+    for (const Config& c : cs)
+      has0 |= c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
+              c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack && c.ndrain == c0.ndrain;
+    if (!has0) cs.insert(cs.begin(), c0);
+    for (const Config& c : cs) cands.push_back({c, sp});
   }
-  bool has0 = false;
-  for (const Config& c : cs)
-    has0 |= c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
-            c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack && c.ndrain == c0.ndrain;
-  if (!has0) cs.insert(cs.begin(), c0);
+  // the model's own pick (its split, its shape): the model-predicted build time reported
+  PipeDesc pm;
+  Config cm;
+  if (gpl_status st = lower_build_pipe(ctx, s, H, &pm, &cm)) return st;
+  const int sm = pm.nsprobe == pm.nprobe && pm.nresid == 0 ? -1 : pm.nsprobe;
+  gpl_status st = GPL_OK;
   cudaEvent_t a = nullptr, b = nullptr;
   CK(cudaEventCreate(&a));
   CK(cudaEventCreate(&b));
   double best_ms = 1e300, m0 = -1;
   TunedShape best;
-  for (const Config& c : cs) {
-    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, -2, c.npack, c.ndrain};
+  for (const auto& [c, sp] : cands) {
+    TunedShape t{c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, sp, c.npack, c.ndrain};
     ctx->tuned[s.text] = t;
     ctx->build_cache.erase(text);
     std::vector<float> ms;
@@ -1640,8 +1659,8 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
       continue;
     }
     std::sort(ms.begin(), ms.end());
-    if (m0 < 0 && c.tile_rows == c0.tile_rows && c.stage_rows == c0.stage_rows && c.depth == c0.depth &&
-        c.warps == c0.warps && c.ctas_per_sm == c0.ctas_per_sm && c.npack == c0.npack && c.ndrain == c0.ndrain)
+    if (m0 < 0 && sp == sm && c.tile_rows == cm.tile_rows && c.stage_rows == cm.stage_rows && c.depth == cm.depth &&
+        c.warps == cm.warps && c.ctas_per_sm == cm.ctas_per_sm && c.npack == cm.npack && c.ndrain == cm.ndrain)
       m0 = ms[1];
     if (ms[1] < best_ms) {
       best_ms = ms[1];

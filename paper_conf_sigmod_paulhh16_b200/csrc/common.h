@@ -213,7 +213,10 @@ struct PipeDesc {
   // ins_dense (clustered build): the key column is sorted and the domain is its [min, max], so each
   // packet writes its whole cell range — its rows' cells (0 when a row fails) and the key gaps between
   // them — with plain stores: no atomics and no clear pass (P:147's blocking build, B200 form)
-  int32_t ins_kcol, ins_pcol, ins_psreg, ins_dense;
+  // ins_q: the insert runs in the queue phase (drain) from queue fields (queue-phase probes or
+  // residuals before it); a dense build then zero-fills each packet's cell range in the stage phase
+  // (ins_kcol: the staged key column) and the drain writes the surviving rows' cells
+  int32_t ins_kcol, ins_pcol, ins_psreg, ins_dense, ins_q;
   long long ins_kmin, ins_pay_base;                            // run-time (table bases)
   unsigned long long ins_nslots;
   void* ins_slots;

@@ -122,7 +122,7 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   c.feasible = c.smem <= ctx->smem_optin && k * (c.smem + 1024) <= 228 * 1024 && W >= 1 &&
                W <= pipeline_max_consumer_warps() && depth >= 2 && k * (W + 1) * 32 <= 2048 &&
                k * (W + 1) * 32 * regs_need <= 65536 && (npack == 1 || npack == 2) && ndrain >= 0 &&
-               ndrain <= 4 && W - ndrain >= 1 && (ndrain == 0 || (d.npush > 0 && !(d.sink != SINK_AGG && d.ins_kcol >= 0)));
+               ndrain <= 4 && W - ndrain >= 1 && (ndrain == 0 || (d.npush > 0 && !(d.sink != SINK_AGG && d.ins_kcol >= 0 && !d.ins_q) && !d.ins_dense));
   const double B = (ctx->opt.hbm_gbs > 0 ? ctx->opt.hbm_gbs : ctx->hbm_gbs) * 1e9;
   c.bw_gbs = B / 1e9;
   // bytes per row: staged columns, plus one 32-B sector per surviving row of
@@ -302,7 +302,8 @@ bool choose_config(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, i
   std::vector<int> Ks = o.ctas_per_sm > 0 ? std::vector<int>{(int)o.ctas_per_sm} : std::vector<int>{1, 2};
   std::vector<int> Ps = o.packets > 0 ? std::vector<int>{(int)o.packets} : std::vector<int>{1, 2};
   // drain warps only for a segment with a queue phase (not a stage-phase insert)
-  const bool can_drain = d.npush > 0 && !(d.sink != SINK_AGG && d.ins_kcol >= 0);
+  // (a dense build's cells are written by the warp that zero-filled their packet: no drain warps)
+  const bool can_drain = d.npush > 0 && !(d.sink != SINK_AGG && d.ins_kcol >= 0 && !d.ins_q) && !d.ins_dense;
   std::vector<int> Dr = !can_drain ? std::vector<int>{0}
                         : o.drain_warps >= 0 ? std::vector<int>{(int)o.drain_warps} : std::vector<int>{0, 1, 2};
   Config best;
@@ -435,6 +436,49 @@ int choose_split(const gpl_ctx* ctx, const Segment& s) {
     return std::min(np, MAXSP);
   }
   return nf ? 0 : std::min(np, MAXSP);
+}
+
+std::vector<double> build_lambda_estimate(const gpl_ctx* ctx, const Segment& s) {
+  std::vector<double> lam;
+  double frac = 1.0;
+  auto ti = ctx->tables.find(s.table);
+  for (const FilterIR& F : s.filters) {
+    double sel = 0.3;
+    const Column* c = ti != ctx->tables.end() ? ti->second.find(F.col) : nullptr;
+    if (c && c->vmax >= c->vmin) {
+      const long double dom = (long double)c->vmax - (long double)c->vmin + 1;
+      if (F.kind == F_RANGE) {
+        const long double lo = std::max<long double>(F.lo, c->vmin), hi = std::min<long double>(F.hi, c->vmax);
+        sel = hi >= lo ? (double)((hi - lo + 1) / dom) : 0.0;
+      } else if (F.kind == F_MASK) {
+        int in = 0;
+        for (int b = 0; b < 64; b++)
+          if (((F.mask >> b) & 1ull) && b >= c->vmin && b <= c->vmax) in++;
+        sel = std::min(1.0, (double)(in / dom));
+      } else {
+        sel = 1.0 - (double)(1 / dom);
+      }
+    }
+    frac *= sel;
+    lam.push_back(frac);
+  }
+  for (size_t p = 0; p < s.probes.size(); p++) {
+    if (s.probes[p].kind != P_MARK) frac *= 0.3;
+    lam.push_back(frac);
+  }
+  for (size_t r = 0; r < s.wheres.size(); r++) {
+    frac *= 0.3;
+    lam.push_back(frac);
+  }
+  return lam;
+}
+
+int choose_build_split(const gpl_ctx* ctx, const Segment& s) {
+  const int np = (int)s.probes.size(), nf = (int)s.filters.size();
+  if (np == 0 || nf == 0) return std::min(np, MAXSP);
+  auto it = ctx->lambda.find(s.text);
+  const std::vector<double> lam = it != ctx->lambda.end() ? it->second : build_lambda_estimate(ctx, s);
+  return (int)lam.size() >= nf && lam[nf - 1] <= 0.05 ? 0 : std::min(np, MAXSP);
 }
 
 }  // namespace gpl

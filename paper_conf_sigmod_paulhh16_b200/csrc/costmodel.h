@@ -47,4 +47,17 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
 // fractions (the paper profiles the first tile) or a heuristic.
 int choose_split(const gpl_ctx* ctx, const Segment& s);
 
+// A build segment's pass fractions before its first run: each filter's
+// selectivity from its column's [min, max] under the uniformity assumption
+// (the textbook optimizer estimate; the paper takes a plan's statistics as
+// given), a probe's hit fraction 0.3. Cumulative, one per operator.
+std::vector<double> build_lambda_estimate(const gpl_ctx* ctx, const Segment& s);
+
+// A build's probe split: the probes move to the queue phase (the insert then
+// runs in the drain) when the filters keep at most 5% of the rows, else every
+// probe runs in the stage phase (measured on B200, SF 100: with the model's
+// shapes the queue split loses at 15-30% survival, Q5 0.51 vs 0.55 ms, Q8 0.59
+// vs 0.69; gpl_autotune measures both splits).
+int choose_build_split(const gpl_ctx* ctx, const Segment& s);
+
 }  // namespace gpl

@@ -184,6 +184,7 @@ std::string shape_source(const PipeDesc& d) {
   I("ins_width", d.ins_width);
   I("ins_kcol", d.ins_kcol);
   I("ins_dense", d.ins_dense);
+  I("ins_q", d.ins_q);
   I("static_tiles", d.static_tiles);
   I("nparts", d.nparts);
   I("part_shift", d.part_shift);

@@ -456,6 +456,9 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
   std::set<std::string> lazy;
   std::map<std::string, int> lazy_at;  // lazy column -> queue probe it is gathered before (np: the tail)
   const int nf0 = (int)s.filters.size();
+  // (not in build segments: measured on B200, SF 100 Q5 HT_O, a late-gathered
+  // build key costs a dependent gather per packet for the dense zero fill's
+  // boundary keys, 0.45 -> 0.62 ms)
   if (!ins && !part && !T.derived && ctx->opt.lazy_columns != 0 && T.nrows < (1ll << 31)) {
     auto lit = ctx->lambda.find(s.text);
     const std::vector<double>* lam =
@@ -683,9 +686,11 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->ins_kmin = ins->dkmin;
     d->ins_nslots = ins->dnslots;
     d->ins_pay_base = ins->pay_base;
-    d->ins_kcol = d->ins_pcol = d->ins_psreg = -1;
+    d->ins_pcol = d->ins_psreg = -1;
+    d->ins_kcol = cidx[s.key[0]];  // staged (a dense build's zero fill reads it in the stage phase)
+    d->ins_q = 1;
     if (sp == np && s.wheres.empty()) {  // every probe in the stage phase: insert from the staged tile
-      d->ins_kcol = cidx[s.key[0]];
+      d->ins_q = 0;
       if (ins->has_payload) {
         if (pay_slot) d->ins_psreg = slot_of[s.payload.name];
         else d->ins_pcol = cidx[s.payload.name];

@@ -365,6 +365,48 @@ __device__ __forceinline__ void insert_cells(const PipeDesc& d, const PipeDesc& 
   if (dup) atomicOr(d.err, ERR_DUPKEY);
 }
 
+// Dense (clustered) build: the cells of N qualifying rows by plain stores. The
+// key column is strictly increasing, so no other row writes these cells; the
+// packet's zero fill (the key gaps and failing rows) precedes them in the warp.
+template <int N>
+__device__ __forceinline__ void dense_cells(const PipeDesc& d, const PipeDesc& K, const long long (&key)[N],
+                                            const long long (&pay)[N], const bool (&act)[N]) {
+  char* cells = (char*)d.ins_slots;
+#pragma unroll
+  for (int j = 0; j < N; j++) {
+    if (!act[j]) continue;
+    long long pv = pay[j];
+    if (K.ins_ptransform == G_YEAR) pv = (int)pv / 10000;
+    const uint32_t v = (uint32_t)(pv - d.ins_pay_base + 1);
+    const long long c = key[j] - d.ins_kmin;
+    if (K.ins_width == 1) cells[c] = (char)v;
+    else if (K.ins_width == 2) ((unsigned short*)cells)[c] = (unsigned short)v;
+    else ((uint32_t*)cells)[c] = v;
+  }
+}
+
+// A dense build's zero fill of one 128-row packet: the cells from its first
+// row's key to the next packet's first key (the next stage's, at a stage end),
+// aligned 16-B stores inside, byte stores at the edges it shares with its
+// neighbours. Every cell of the domain is written exactly once per build.
+__device__ __forceinline__ void dense_zero_fill(const PipeDesc& d, const PipeDesc& K, uint32_t sb, int pb, int n,
+                                                int ins_knext, int lane) {
+  const uint32_t kcol_sa = smem_base() + sb + (uint32_t)K.coloff[K.ins_kcol];
+  const int first = lds_s32(kcol_sa + (uint32_t)pb * 4u);
+  const int next = pb + 128 < n ? lds_s32(kcol_sa + (uint32_t)(pb + 128) * 4u) : ins_knext;
+  const int w = K.ins_width;
+  char* cells = (char*)d.ins_slots;
+  const long long blo = ((long long)first - d.ins_kmin) * w, bhi = ((long long)next - d.ins_kmin) * w;
+  const long long alo = (blo + 15) & ~15ll, ahi = bhi & ~15ll;
+  if (alo < ahi) {
+    for (long long b = alo + lane * 16; b < ahi; b += 512) *(uint4*)(cells + b) = make_uint4(0u, 0u, 0u, 0u);
+    for (long long b = blo + lane; b < alo; b += 32) cells[b] = 0;
+    for (long long b = ahi + lane; b < bhi; b += 32) cells[b] = 0;
+  } else {
+    for (long long b = blo + lane; b < bhi; b += 32) cells[b] = 0;
+  }
+}
+
 // Queue phase on up to RPL*32 queued survivors starting at qhead: lane `lane`
 // owns entries qhead + j*32 + lane (j < RPL) that are < n. Remaining probes,
 // where residuals, group-by and the exact aggregation (A5-A7).
@@ -486,7 +528,13 @@ __device__ GPL_DRAIN_INLINE void drain(const PipeDesc& d, uint32_t qb, int qhead
         kx[j] = fget(K.ins_kfield, j);
         px[j] = K.ins_pfield >= 0 ? fget(K.ins_pfield, j) : 0;
       }
-      insert_cells<RPL>(d, K, kx, px, p);
+      if (K.ins_dense) {
+        // dense build, queue-phase insert: the stage phase zero-filled this row's
+        // packet range (same warp, ordered by the __syncwarp before the drain)
+        dense_cells<RPL>(d, K, kx, px, p);
+      } else {
+        insert_cells<RPL>(d, K, kx, px, p);
+      }
       return;
     }
     // the Listings' SELECT expression of row j (exact int64, bounded by the lowering)
@@ -939,7 +987,7 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
   for (int i = 0; i < MAXF + MAXSP; i++) lc[i] = 0;
   // rows this warp queued = the pass count of the last stage-phase operator
-  const bool kQueueCounts = !(K.sink != SINK_AGG && K.ins_kcol >= 0);  // (a stage-phase sink queues nothing)
+  const bool kQueueCounts = !(K.sink != SINK_AGG && K.ins_kcol >= 0 && !K.ins_q);  // (a stage-phase sink queues nothing)
   unsigned long long queued = 0;
   for (;;) {
     mbar_wait(&full[slot], phase);
@@ -1083,7 +1131,15 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           }
         continue;
       }
-      if (K.sink == SINK_INSERT && K.ins_kcol >= 0) {
+      if (K.sink == SINK_INSERT && K.ins_q && K.ins_dense) {
+        // dense build with a queue-phase insert: zero-fill every live packet's
+        // cell range now; the drain writes the cells of the rows that survive
+#pragma unroll
+        for (int q = 0; q < NPMAX; q++)
+          if (live[q]) dense_zero_fill(d, K, sb, (it0 + q * Ws) << 7, n, ins_knext, lane);
+        __syncwarp();  // the zero fill is ordered before this warp's drains
+      }
+      if (K.sink == SINK_INSERT && K.ins_kcol >= 0 && !K.ins_q) {
         // build segment with every probe in the stage phase: insert straight
         // from the staged tile (no survivor queue), all rows' atomics in flight
         long long kx[NR], px[NR];
@@ -1116,21 +1172,9 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
           for (int q = 0; q < NPMAX; q++) {
             if (!live[q]) continue;
-            const int pb = (it0 + q * Ws) << 7;  // the packet's first row in the stage
-            const uint32_t kcol_sa = smem_base() + sb + (uint32_t)K.coloff[K.ins_kcol];
-            const int first = lds_s32(kcol_sa + (uint32_t)pb * 4u);
-            const int next = pb + 128 < n ? lds_s32(kcol_sa + (uint32_t)(pb + 128) * 4u) : ins_knext;
+            dense_zero_fill(d, K, sb, (it0 + q * Ws) << 7, n, ins_knext, lane);
             const int w = K.ins_width;
             char* cells = (char*)d.ins_slots;
-            const long long blo = ((long long)first - d.ins_kmin) * w, bhi = ((long long)next - d.ins_kmin) * w;
-            const long long alo = (blo + 15) & ~15ll, ahi = bhi & ~15ll;
-            if (alo < ahi) {
-              for (long long b = alo + lane * 16; b < ahi; b += 512) *(uint4*)(cells + b) = make_uint4(0u, 0u, 0u, 0u);
-              for (long long b = blo + lane; b < alo; b += 32) cells[b] = 0;
-              for (long long b = ahi + lane; b < bhi; b += 32) cells[b] = 0;
-            } else {
-              for (long long b = blo + lane; b < bhi; b += 32) cells[b] = 0;
-            }
             __syncwarp();  // the zero fill is ordered before the cells below (same warp)
 #pragma unroll
             for (int j = 0; j < RPL; j++) {

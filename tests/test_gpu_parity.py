@@ -766,19 +766,27 @@ def test_dense_clustered_build_exact(ctx, q):
     o_orderkey, customer by c_custkey, supplier by s_suppkey) writes every cell of its domain with plain
     stores (no clear, no atomics); results equal the atomic build's and the oracle's, also on a ragged
     orders table (rows dropped: the domain and the packet ranges change) and after a duplicate key makes
-    the column non-strict (the atomic build then detects it)."""
+    the column non-strict (the atomic build then detects it); with the builds' probes in the stage phase
+    (insert from the staged tile) and in the queue phase (zero fill per packet, cells from the drain)."""
     db = tpchgen.generate(0.05, seed=29)
     o = _oracle(q, db)
     if q == "Q3":
         o = oracle.order_limit("Q3", oracle.run("Q3", db))
     try:
-        for dense in (1, 0, 1):
+        # probe_split 0: the builds' probes run in the queue phase, so a dense build zero-fills in the
+        # stage phase and its drain writes the surviving rows' cells
+        # (and with late materialisation forced in the probe segment)
+        for dense, split, lazy in ((1, -2, -1), (0, -2, -1), (1, 0, -1), (0, 0, -1), (1, 0, 1), (0, 0, 1), (1, -1, -1)):
             ctx.set_option("dense_build", dense)
+            ctx.set_option("probe_split", split)
+            ctx.set_option("lazy_columns", lazy)
             for _ in range(2):
                 r = _gpu(ctx, db, q)
-                assert r.keys == o.keys and r.aggs == o.aggs, (q, dense)
+                assert r.keys == o.keys and r.aggs == o.aggs, (q, dense, split, lazy)
     finally:
         ctx.set_option("dense_build", 1)
+        ctx.set_option("probe_split", -2)
+        ctx.set_option("lazy_columns", -1)
     # ragged: drop every 7th order (and its lineitems stay: FK misses drop them)
     db2 = tpchgen.generate(0.05, seed=29)
     keep = np.arange(db2.nrows("orders")) % 7 != 3
