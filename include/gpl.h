@@ -321,7 +321,14 @@ gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t
  * not depend on each other on two lanes, default; 0 = one chain),
  * "hash_slots_log2" (hash group-by table of 2^v slots; 0 = sized from the
  * plan's last run, default), "use_profile" (1 = the model fits its consumer cost to the plan's first
- * timed run after its λ profile, Table 2 "profiling input", default).
+ * timed run after its λ profile, Table 2 "profiling input", default),
+ * "dense_build" (1 = a DIRECT build keyed by a strictly increasing column writes
+ * its cell ranges densely, default; 0 = atomic inserts into a cleared table),
+ * "nibble_cells" (1 = DIRECT payloads of at most 15 values in 4-bit cells; 0 =
+ * byte cells, default), "lazy_columns" (late materialisation: -1 = from the
+ * plan's pass fractions, default; 0 = off; 1 = every eligible column).
+ * Builds take "probe_split" too (a DIRECT build's probes and insert in the
+ * stage phase or the queue phase; gpl_autotune measures both).
  * value < 0 restores automatic selection. */
 gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value);
 

@@ -260,6 +260,11 @@ __global__ void __launch_bounds__(kThreads) build_insert_kernel(const __grid_con
         const uint32_t v = (uint32_t)(payv[j] - d.pay_base + 1);
         if (d.width == 4) {
           if (atomicCAS((uint32_t*)d.slots + idx, 0u, v) != 0u) atomicOr(d.err, ERR_DUPKEY);
+        } else if (d.width == W_NIBBLE) {
+          const unsigned long long byte = idx >> 1;
+          uint32_t* w = (uint32_t*)((char*)d.slots + (byte & ~3ull));
+          const uint32_t sh = (uint32_t)(byte & 3ull) * 8u + (uint32_t)(idx & 1ull) * 4u;
+          if (atomicOr(w, v << sh) & (0xFu << sh)) atomicOr(d.err, ERR_DUPKEY);
         } else {
           const unsigned long long byte = idx * (unsigned long long)d.width;
           uint32_t* w = (uint32_t*)((char*)d.slots + (byte & ~3ull));

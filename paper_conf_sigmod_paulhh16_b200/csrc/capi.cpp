@@ -467,6 +467,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
     o.drain_warps = v < 0 ? -1 : v;
   } else if (k == "dense_build") {
     o.dense_build = v != 0 ? 1 : 0;
+  } else if (k == "nibble_cells") {
+    o.nibble_cells = v != 0 ? 1 : 0;
   } else if (k == "reg_fields") {
     o.reg_fields = v != 0 ? 1 : 0;
   } else if (k == "zone_restrict") {
@@ -1091,9 +1093,14 @@ GPL_API gpl_status gpl_build_hash(gpl_ctx* ctx, const char* build_segment, int32
     P.pgrid = cfg.grid;
     P.clear_bytes = direct_counter_off(H.bytes()) + 16;
     P.clear_off = 0;
-    if (pd.ins_dense) {  // the build writes every cell: clear only its tile counter
-      P.clear_off = direct_counter_off(H.bytes());
-      P.clear_bytes = 16;
+    if (pd.ins_dense) {
+      // the build writes every cell: clear only the bytes past the domain's
+      // last cell (a clustered probe stages 16-B rounded ranges, so they must
+      // read as empty) and the tile counter; 8-B granular (the query graph's
+      // clear kernel), the few cells below it are rewritten by the build
+      const size_t last = H.width == W_NIBBLE ? (size_t)(H.dnslots >> 1) : (size_t)H.dnslots * (size_t)H.width;
+      P.clear_off = last & ~(size_t)7;
+      P.clear_bytes = direct_counter_off(H.bytes()) + 16 - P.clear_off;
     }
   }
   P.desc = d;

@@ -47,14 +47,17 @@ struct Filt {
 // Hashed kinds: open addressing, linear probing, power-of-two slots:
 //   SET32 4 B {key}, MAP32 8 B {key, payload}, MAP64 16 B {key64, payload64}.
 // DIRECT: direct-addressed array over a dense key domain [kmin, kmin+nslots)
-//   (a collision-free perfect hash): width 0 = bitmap set, else 1/2/4-byte
-//   cells holding payload - pay_base + 1 (0 = empty).
+//   (a collision-free perfect hash): width 0 = bitmap set, W_NIBBLE = 4-bit
+//   cells (two per byte, the even cell in the low nibble; payload ranges of at
+//   most 15 values: nation keys, years), else 1/2/4-byte cells; a cell holds
+//   payload - pay_base + 1 (0 = empty).
 // MULTI (non-unique build keys): CSR over a dense key
 //   domain — slots = uint32 offsets[nslots + 1], pay = int32 payload[count];
 //   key k's matches are pay[off[k - kmin] .. off[k - kmin + 1]) (fan-out join).
 // PART: not a hash table — the output of a partition segment (a derived table), registered by name so
 //   the query's segment bookkeeping (graphs, caches) treats it like a build.
 enum : int32_t { HT_SET32 = 0, HT_MAP32 = 1, HT_MAP64 = 2, HT_DIRECT = 3, HT_MULTI = 4, HT_PART = 5 };
+constexpr int32_t W_NIBBLE = 3;  // DIRECT cell width code of 4-bit cells (not a byte count)
 enum : int32_t { H_MULT = 0, H_ORDERED = 1 };
 
 // Device-resident header, written by the build's count and size kernels and

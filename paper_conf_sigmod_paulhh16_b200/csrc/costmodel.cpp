@@ -56,7 +56,7 @@ int cl_cap_bytes(const PipeDesc& d, int S) {
   if (d.cl_probe < 0) return 0;
   const int w = d.ht[d.probe[d.cl_probe].ht].width;
   const int kpr = d.cl_kpr > 0 ? d.cl_kpr : 4;
-  return align128((w == 0 ? (kpr * S + 7) / 8 : kpr * S * w) + 32);
+  return align128((w == 0 ? (kpr * S + 7) / 8 : w == W_NIBBLE ? (kpr * S + 1) / 2 : kpr * S * w) + 32);
 }
 
 int smem_bytes(const PipeDesc& d, const LowerInfo& li, int stage_rows, int depth, int warps, int ndrain) {

@@ -69,7 +69,8 @@ struct HashTable {
   size_t aux_alloc = 0;
   size_t bytes() const {
     if (kind == HT_MULTI) return (dnslots + 1) * 4;
-    if (kind == HT_DIRECT) return width == 0 ? (dnslots + 31) / 32 * 4 : (dnslots * width + 3) / 4 * 4;
+    if (kind == HT_DIRECT)
+      return width == 0 ? (dnslots + 31) / 32 * 4 : width == W_NIBBLE ? (dnslots + 7) / 8 * 4 : (dnslots * width + 3) / 4 * 4;
     return (size_t)cap_slots * (kind == HT_SET32 ? 4 : kind == HT_MAP32 ? 8 : 16);
   }
   HTRef ref() const { return HTRef{slots, hdr, kind, hash, dkmin, dnslots, pay_base, width, 0, pay}; }
@@ -210,6 +211,11 @@ struct Options {
   int64_t graph_branches = 1;  // whole-query graph: independent build segments on two capture lanes
   int64_t drain_warps = -1;    // operator-specialised drain warps (NEXT-1): -1 = the model's choice
   int64_t dense_build = 1;     // sorted-key DIRECT builds write their cell ranges densely (no clear, no atomics)
+  // DIRECT payloads of <= 15 values in 4-bit cells (1) or byte cells (0, default). Measured on B200,
+  // SF 100, autotuned shapes: Q7 step 2.15 -> 2.00 ms (kernel 1.32 -> 1.20), Q9 1.085 -> 1.073, but
+  // Q5 1.32 -> 1.39 and Q8 1.71 -> 1.73: the nibble extraction in the clustered probe and the dense
+  // build's byte assembly cost more issue slots than the halved cell bytes save there.
+  int64_t nibble_cells = 0;
   int64_t reg_fields = 1;      // JIT kernels keep drain-produced queue fields in registers
   int64_t zone_restrict = 1;   // scan only the row range of range filters on sorted columns
   int64_t agg_mode = -1;       // dense group accumulators: -1 exactness-driven choice, 2 = force global int128 atomics

@@ -61,7 +61,8 @@ __device__ __forceinline__ bool direct_probe(const HTP& h, unsigned long long ke
     return (w >> (idx & 31)) & 1u;
   }
   uint32_t v;
-  if (h.width == 1) v = __ldg((const unsigned char*)h.slots + idx);
+  if (h.width == W_NIBBLE) v = ((uint32_t)__ldg((const unsigned char*)h.slots + (idx >> 1)) >> ((idx & 1) * 4)) & 0xFu;
+  else if (h.width == 1) v = __ldg((const unsigned char*)h.slots + idx);
   else if (h.width == 2) v = __ldg((const unsigned short*)h.slots + idx);
   else v = __ldg((const uint32_t*)h.slots + idx);
   *payload = (long long)v - 1 + h.pay_base;
@@ -136,7 +137,11 @@ __device__ __forceinline__ void ht_probe_n(const HTP& h, const int kind, const i
       for (int j = 0; j < R; j++) { hit[j] = v[j] != 0; pay[j] = 1; }
       return;
     }
-    if (width == 1) {
+    if (width == W_NIBBLE) {
+#pragma unroll
+      for (int j = 0; j < R; j++)
+        v[j] = in[j] ? ((uint32_t)__ldg((const unsigned char*)h.slots + (idx[j] >> 1)) >> ((idx[j] & 1) * 4)) & 0xFu : 0u;
+    } else if (width == 1) {
 #pragma unroll
       for (int j = 0; j < R; j++) v[j] = in[j] ? (uint32_t)__ldg((const unsigned char*)h.slots + idx[j]) : 0u;
     } else if (width == 2) {

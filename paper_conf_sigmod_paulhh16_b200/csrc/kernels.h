@@ -10,7 +10,9 @@ namespace gpl {
 
 // Bytes of a DIRECT table (bitmap when width == 0), 4-byte granular.
 inline unsigned long long direct_bytes(int width, unsigned long long nslots) {
-  return width == 0 ? (nslots + 31) / 32 * 4 : (nslots * (unsigned long long)width + 3) / 4 * 4;
+  return width == 0 ? (nslots + 31) / 32 * 4
+         : width == W_NIBBLE ? (nslots + 7) / 8 * 4
+                             : (nslots * (unsigned long long)width + 3) / 4 * 4;
 }
 
 // A1 build segment. `trivial` (no filter, no probe): every row is inserted,

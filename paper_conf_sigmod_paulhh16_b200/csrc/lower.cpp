@@ -185,6 +185,28 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
       shape->pay_min = cols[d->pay_ref]->vmin;
       shape->pay_max = cols[d->pay_ref]->vmax;
     }
+    // the segment's filters on the payload's column bound the inserted values
+    // (Q5: c_nationkey in the nations of ASIA -> [8, 21], so 4-bit cells)
+    if (d->pay_kind == PAY_COL || d->pay_kind == PAY_YEARCOL)
+      for (const FilterIR& F : s.filters) {
+        if (F.col != s.payload.name) continue;
+        long long lo = F.lo, hi = F.hi;
+        if (F.kind == F_MASK) {
+          if (!F.mask) continue;
+          lo = __builtin_ctzll(F.mask);
+          hi = 63 - __builtin_clzll(F.mask);
+        } else if (F.kind != F_RANGE) {
+          continue;
+        }
+        if (d->pay_kind == PAY_YEARCOL) {  // yyyymmdd dates -> years
+          lo = lo == INT64_MIN ? lo : lo / 10000;
+          hi = hi == INT64_MAX ? hi : hi / 10000;
+        }
+        if (std::max<long long>(lo, shape->pay_min) <= std::min<long long>(hi, shape->pay_max)) {
+          shape->pay_min = std::max<long long>(lo, shape->pay_min);
+          shape->pay_max = std::min<long long>(hi, shape->pay_max);
+        }
+      }
   }
   int load = ctx->opt.hash_load_pct > 0 ? (int)ctx->opt.hash_load_pct : s.load_pct;
   if (shape->key_arity == 2) shape->kind = HT_MAP64;
@@ -235,11 +257,14 @@ gpl_status lower_build(gpl_ctx* ctx, const Segment& s, BuildDesc* d, HashTable* 
     int width = -1;
     if (!shape->has_payload) width = 0;
     else {
+      // cell values 1..(pay_max - pay_min + 1), 0 = empty: 4-bit cells when they
+      // fit (nation keys of a region, years), else the narrowest byte width
       const unsigned long long prange = (unsigned long long)(shape->pay_max - shape->pay_min) + 2ull;
-      width = prange <= 0xFFull ? 1 : prange <= 0xFFFFull ? 2 : prange <= 0xFFFFFFFFull ? 4 : -1;
+      width = prange <= 0x10ull && ctx->opt.nibble_cells != 0 ? W_NIBBLE
+              : prange <= 0xFFull ? 1 : prange <= 0xFFFFull ? 2 : prange <= 0xFFFFFFFFull ? 4 : -1;
     }
     if (width >= 0 && range <= (1ull << 31)) {
-      const unsigned long long dbytes = width == 0 ? (range + 31) / 32 * 4 : range * width;
+      const unsigned long long dbytes = width == 0 ? (range + 31) / 32 * 4 : width == W_NIBBLE ? (range + 1) / 2 : range * width;
       const unsigned long long hbytes = (unsigned long long)std::max<int64_t>(16, next_pow2((T.nrows * 100 + load - 1) / load)) *
                                         (shape->has_payload ? 8ull : 4ull);
       if (s.hash == 2 || dbytes <= (64ull << 20) || dbytes <= 2 * hbytes) {

@@ -234,6 +234,7 @@ __device__ __forceinline__ void probe_rows(const PipeDesc& K, const HTP& h, int 
       const uint32_t i = in ? (uint32_t)idx : last;
       uint32_t x;
       if (width == 0) x = (lds_u32(sso + (i >> 5) * 4) >> (i & 31)) & 1u;
+      else if (width == W_NIBBLE) x = (lds_u8(sso + (i >> 1)) >> ((i & 1) * 4)) & 0xFu;
       else if (width == 1) x = lds_u8(sso + i);
       else if (width == 2) x = lds_u16(sso + i * 2);
       else x = lds_u32(sso + i * 4);
@@ -269,6 +270,7 @@ __device__ __forceinline__ void probe_rows_cl(const PipeDesc& K, const HTP& h, i
     const bool in = act[j] && o < ncells;
     uint32_t v = 0;
     if (width == 0) v = in ? (lds_u32(sbase + (o >> 5) * 4) >> (o & 31)) & 1u : 0u;
+    else if (width == W_NIBBLE) v = in ? (lds_u8(sbase + (o >> 1)) >> ((o & 1) * 4)) & 0xFu : 0u;
     else if (width == 1) v = in ? lds_u8(sbase + o) : 0u;
     else if (width == 2) v = in ? lds_u16(sbase + o * 2) : 0u;
     else v = in ? lds_u32(sbase + o * 4) : 0u;
@@ -352,6 +354,11 @@ __device__ __forceinline__ void insert_cells(const PipeDesc& d, const PipeDesc& 
     if (K.ins_width == 4) {
       m[j] = 0xFFFFFFFFu;
       old[j] = atomicCAS((uint32_t*)d.ins_slots + ci[j], 0u, v);
+    } else if (K.ins_width == W_NIBBLE) {
+      const unsigned long long byte = ci[j] >> 1;
+      const uint32_t sh = (uint32_t)(byte & 3ull) * 8u + (uint32_t)(ci[j] & 1ull) * 4u;
+      m[j] = 0xFu << sh;
+      old[j] = atomicOr((uint32_t*)((char*)d.ins_slots + (byte & ~3ull)), v << sh);
     } else {
       const unsigned long long byte = ci[j] * (unsigned long long)K.ins_width;
       const uint32_t sh = (uint32_t)(byte & 3ull) * 8u;
@@ -363,6 +370,21 @@ __device__ __forceinline__ void insert_cells(const PipeDesc& d, const PipeDesc& 
 #pragma unroll
   for (int j = 0; j < N; j++) dup |= (old[j] & m[j]) != 0u;
   if (dup) atomicOr(d.err, ERR_DUPKEY);
+}
+
+// 4-bit cells: cell c is nibble (c & 1) of byte c >> 1; the word-level atomics
+// touch only that nibble's bits, so they commute with every other cell's update
+__device__ __forceinline__ uint32_t nibble_shift(long long c) {
+  return (uint32_t)((c >> 1) & 3ll) * 8u + (uint32_t)(c & 1ll) * 4u;
+}
+__device__ __forceinline__ uint32_t* nibble_word(char* cells, long long c) {
+  return (uint32_t*)(cells + ((c >> 1) & ~3ll));
+}
+__device__ __forceinline__ void nibble_or(char* cells, long long c, uint32_t v) {
+  if (v) atomicOr(nibble_word(cells, c), (v & 0xFu) << nibble_shift(c));
+}
+__device__ __forceinline__ void nibble_clear(char* cells, long long c) {
+  atomicAnd(nibble_word(cells, c), ~(0xFu << nibble_shift(c)));
 }
 
 // Dense (clustered) build: the cells of N qualifying rows by plain stores. The
@@ -379,7 +401,8 @@ __device__ __forceinline__ void dense_cells(const PipeDesc& d, const PipeDesc& K
     if (K.ins_ptransform == G_YEAR) pv = (int)pv / 10000;
     const uint32_t v = (uint32_t)(pv - d.ins_pay_base + 1);
     const long long c = key[j] - d.ins_kmin;
-    if (K.ins_width == 1) cells[c] = (char)v;
+    if (K.ins_width == W_NIBBLE) nibble_or(cells, c, v);  // (rows of one byte may sit in different lanes)
+    else if (K.ins_width == 1) cells[c] = (char)v;
     else if (K.ins_width == 2) ((unsigned short*)cells)[c] = (unsigned short)v;
     else ((uint32_t*)cells)[c] = v;
   }
@@ -389,14 +412,30 @@ __device__ __forceinline__ void dense_cells(const PipeDesc& d, const PipeDesc& K
 // row's key to the next packet's first key (the next stage's, at a stage end),
 // aligned 16-B stores inside, byte stores at the edges it shares with its
 // neighbours. Every cell of the domain is written exactly once per build.
+// 4-bit cells: the packet owns the bytes whose two cells are both in its range;
+// a byte it shares with a neighbouring packet (an odd first cell, an odd end)
+// has its own nibble cleared by an atomic, never a byte store.
 __device__ __forceinline__ void dense_zero_fill(const PipeDesc& d, const PipeDesc& K, uint32_t sb, int pb, int n,
-                                                int ins_knext, int lane) {
+                                                int ins_knext, int lane, long long* c0_out = nullptr,
+                                                long long* c1_out = nullptr) {
   const uint32_t kcol_sa = smem_base() + sb + (uint32_t)K.coloff[K.ins_kcol];
   const int first = lds_s32(kcol_sa + (uint32_t)pb * 4u);
   const int next = pb + 128 < n ? lds_s32(kcol_sa + (uint32_t)(pb + 128) * 4u) : ins_knext;
   const int w = K.ins_width;
   char* cells = (char*)d.ins_slots;
-  const long long blo = ((long long)first - d.ins_kmin) * w, bhi = ((long long)next - d.ins_kmin) * w;
+  const long long c0 = (long long)first - d.ins_kmin, c1 = (long long)next - d.ins_kmin;  // cells [c0, c1)
+  if (c0_out) *c0_out = c0;
+  if (c1_out) *c1_out = c1;
+  long long blo, bhi;
+  if (w == W_NIBBLE) {
+    blo = (c0 + 1) >> 1;
+    bhi = c1 >> 1;
+    if (lane == 0 && (c0 & 1)) nibble_clear(cells, c0);
+    if (lane == 1 && (c1 & 1)) nibble_clear(cells, c1 - 1);
+  } else {
+    blo = c0 * w;
+    bhi = c1 * w;
+  }
   const long long alo = (blo + 15) & ~15ll, ahi = bhi & ~15ll;
   if (alo < ahi) {
     for (long long b = alo + lane * 16; b < ahi; b += 512) *(uint4*)(cells + b) = make_uint4(0u, 0u, 0u, 0u);
@@ -869,8 +908,8 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
           chi = min(chi, (long long)H.nslots - 1);
           if (clo <= chi) {
             const int w = K.ht[K.probe[K.cl_probe].ht].width;
-            const long long blo = w == 0 ? (clo >> 5) * 4 : clo * w;
-            const long long bhi = w == 0 ? ((chi >> 5) + 1) * 4 : (chi + 1) * w;
+            const long long blo = w == 0 ? (clo >> 5) * 4 : w == W_NIBBLE ? clo >> 1 : clo * w;
+            const long long bhi = w == 0 ? ((chi >> 5) + 1) * 4 : w == W_NIBBLE ? (chi >> 1) + 1 : (chi + 1) * w;
             cl_start = blo & ~15ll;
             const long long sz = ((bhi + 15) & ~15ll) - cl_start;
             if (sz <= K.cl_cap) cl_size = (uint32_t)sz;
@@ -1007,8 +1046,11 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
       cl_size = h2.z;
       const int w = K.ht[K.probe[K.cl_probe].ht].width;
       const HTP& H = GPL_SP_HTP(K.cl_probe);
-      cl_k0 = (uint32_t)((long long)H.kmin + (w == 0 ? cl_start * 8 : cl_start / (w > 0 ? w : 1)));
-      cl_ncells = w == 0 ? (uint32_t)cl_size * 8u : (uint32_t)cl_size / (uint32_t)(w > 0 ? w : 1);
+      cl_k0 = (uint32_t)((long long)H.kmin + (w == 0 ? cl_start * 8 : w == W_NIBBLE ? cl_start * 2 : cl_start / (w > 0 ? w : 1)));
+      // (the 16-B rounded range may reach past the domain's last cell: those
+      // bytes are zero — the build clears them — so such keys miss)
+      cl_ncells = w == 0 ? (uint32_t)cl_size * 8u
+                  : w == W_NIBBLE ? (uint32_t)cl_size * 2u : (uint32_t)cl_size / (uint32_t)(w > 0 ? w : 1);
     }
     const int nit = (n + 127) >> 7;
     bool released = false;
@@ -1172,10 +1214,52 @@ __device__ __forceinline__ void pipeline_body(const PipeDesc& d) {
 #pragma unroll
           for (int q = 0; q < NPMAX; q++) {
             if (!live[q]) continue;
-            dense_zero_fill(d, K, sb, (it0 + q * Ws) << 7, n, ins_knext, lane);
+            long long c0, c1;
+            dense_zero_fill(d, K, sb, (it0 + q * Ws) << 7, n, ins_knext, lane, &c0, &c1);
             const int w = K.ins_width;
             char* cells = (char*)d.ins_slots;
             __syncwarp();  // the zero fill is ordered before the cells below (same warp)
+            if (w == W_NIBBLE) {
+              // 4-bit cells: the row of a byte's even cell writes the whole byte
+              // (its value | the next row's when that row holds the odd cell),
+              // the row of an odd cell only when the even cell has no row; the
+              // two bytes shared with the neighbouring packets take atomics
+              long long c[RPL];
+              uint32_t v[RPL];
+              bool ok[RPL];
+#pragma unroll
+              for (int j = 0; j < RPL; j++) {
+                ok[j] = r0q[q] + j < n;
+                c[j] = kx[q * RPL + j] - d.ins_kmin;
+                long long pv = px[q * RPL + j];
+                if (K.ins_ptransform == G_YEAR) pv = (int)pv / 10000;
+                v[j] = p[q * RPL + j] ? (uint32_t)(pv - d.ins_pay_base + 1) & 0xFu : 0u;
+              }
+              const long long cn = __shfl_down_sync(0xffffffffu, c[0], 1), cp = __shfl_up_sync(0xffffffffu, c[RPL - 1], 1);
+              const uint32_t vn = __shfl_down_sync(0xffffffffu, v[0], 1);
+              const bool okn = __shfl_down_sync(0xffffffffu, ok[0], 1) && lane < 31;
+              const bool okp = __shfl_up_sync(0xffffffffu, ok[RPL - 1], 1) && lane > 0;
+#pragma unroll
+              for (int j = 0; j < RPL; j++) {
+                if (!ok[j]) continue;
+                const long long cj = c[j];
+                if ((cj & 1) == 0) {
+                  if (cj + 1 == c1) {
+                    nibble_or(cells, cj, v[j]);  // shared with the next packet
+                  } else {
+                    const bool hn = j < RPL - 1 ? ok[j + 1] && c[j + 1] == cj + 1 : okn && cn == cj + 1;
+                    const uint32_t b = v[j] | ((hn ? (j < RPL - 1 ? v[j + 1] : vn) : 0u) << 4);
+                    if (b) cells[cj >> 1] = (char)b;
+                  }
+                } else if (cj == c0) {
+                  nibble_or(cells, cj, v[j]);  // shared with the previous packet
+                } else {
+                  const bool hp = j > 0 ? c[j - 1] == cj - 1 : okp && cp == cj - 1;
+                  if (!hp && v[j]) cells[cj >> 1] = (char)(v[j] << 4);
+                }
+              }
+              continue;
+            }
 #pragma unroll
             for (int j = 0; j < RPL; j++) {
               if (!p[q * RPL + j]) continue;

@@ -776,17 +776,22 @@ def test_dense_clustered_build_exact(ctx, q):
         # probe_split 0: the builds' probes run in the queue phase, so a dense build zero-fills in the
         # stage phase and its drain writes the surviving rows' cells
         # (and with late materialisation forced in the probe segment)
-        for dense, split, lazy in ((1, -2, -1), (0, -2, -1), (1, 0, -1), (0, 0, -1), (1, 0, 1), (0, 0, 1), (1, -1, -1)):
+        # nibble_cells 0/1: payloads of <= 15 values in byte or 4-bit cells (a dense 4-bit build writes
+        # whole bytes from the row of the even cell, atomics on the bytes shared between packets)
+        for dense, split, lazy, nib in ((1, -2, -1, 1), (0, -2, -1, 1), (1, 0, -1, 1), (0, 0, -1, 1), (1, 0, 1, 1),
+                                        (0, 0, 1, 1), (1, -2, -1, 0), (1, 0, -1, 0), (0, -2, -1, 0), (1, -1, -1, 1)):
             ctx.set_option("dense_build", dense)
             ctx.set_option("probe_split", split)
             ctx.set_option("lazy_columns", lazy)
+            ctx.set_option("nibble_cells", nib)
             for _ in range(2):
                 r = _gpu(ctx, db, q)
-                assert r.keys == o.keys and r.aggs == o.aggs, (q, dense, split, lazy)
+                assert r.keys == o.keys and r.aggs == o.aggs, (q, dense, split, lazy, nib)
     finally:
         ctx.set_option("dense_build", 1)
         ctx.set_option("probe_split", -2)
         ctx.set_option("lazy_columns", -1)
+        ctx.set_option("nibble_cells", 0)
     # ragged: drop every 7th order (and its lineitems stay: FK misses drop them)
     db2 = tpchgen.generate(0.05, seed=29)
     keep = np.arange(db2.nrows("orders")) % 7 != 3
@@ -901,3 +906,41 @@ def test_smem_groups_dense_warp_aggregation(ctx, date):
         assert r2.stats["agg_mode"] == 2 and (r2.keys, r2.aggs) == (r.keys, r.aggs)
     finally:
         ctx.set_option("agg_mode", -1)
+
+
+@pytest.mark.parametrize("sorted_fact", [True, False])
+def test_nibble_cells_random_gaps(ctx, sorted_fact):
+    """4-bit DIRECT cells (payloads of <= 15 values) under a dense (clustered) build whose key column has
+    random gaps, so 128-row packets start and end on odd and even cells (the bytes shared between packets
+    take atomics, the others whole-byte stores from the row of the even cell). Every key of the domain
+    (and a few outside it) is probed — by the clustered probe when the fact keys are sorted, by global
+    loads when shuffled — and the per-payload counts equal numpy's; byte cells (nibble_cells 0), the
+    atomic build (dense_build 0) and a queue-phase insert give the same."""
+    rng = np.random.default_rng(7 if sorted_fact else 8)
+    n = 300_001
+    k = (np.cumsum(rng.integers(1, 4, n)) + 1000).astype(np.int32)  # strictly increasing, gaps 1..3
+    pay = rng.integers(3, 17, n).astype(np.int32)  # 14 values -> 4-bit cells
+    f = rng.integers(0, 100, n).astype(np.int32)
+    ctx.load_columns("nt_dim", {"k": k, "p": pay, "f": f})
+    x = np.arange(int(k[0]) - 5, int(k[-1]) + 6, dtype=np.int32)
+    if not sorted_fact:
+        rng.shuffle(x)
+    ctx.load_columns("nt_fact", {"x": x})
+    plan = ("build NT\nscan nt_dim\nfilter f < 60\nkey k\npayload p\n\n"
+            "run nt_fact\nprobe NT x -> pv\ngroup pv 3 17\nagg count\n")
+    sel = f < 60
+    vals, cnts = np.unique(pay[sel], return_counts=True)
+    expect_keys, expect_aggs = [(int(v),) for v in vals], [[int(c)] for c in cnts]
+    try:
+        for nib, dense, split in ((1, 1, -2), (1, 1, 0), (0, 1, -2), (1, 0, -2), (1, 1, -2)):
+            ctx.set_option("nibble_cells", nib)
+            ctx.set_option("dense_build", dense)
+            ctx.set_option("probe_split", split)
+            for _ in range(2):
+                ctx.run_query(plan)
+                r = ctx.fetch_result()
+                assert r.keys == expect_keys and r.aggs == expect_aggs, (nib, dense, split)
+    finally:
+        ctx.set_option("nibble_cells", 0)
+        ctx.set_option("dense_build", 1)
+        ctx.set_option("probe_split", -2)
