@@ -2,7 +2,9 @@
 synccheck), bit-exact vs the oracle: the paper plans (clustered probe, late materialisation with
 gathers at first use, register drain fields), Q3's hash group-by (device top-k and the full device sort),
 QF's fan-out join (multi build, chained probe), operator-specialised drain warps D = 1 and 2, forced
-global int128 accumulators, a dense shared-memory group-by (lane-private copies), and the KBE / GPL (w/o CE) baselines. Eager runs and graph replays, SF 0.02."""
+global int128 accumulators, a dense shared-memory group-by (lane-private copies), builds with queue-phase
+probes and inserts, 4-bit cells (dense, atomic, random key gaps), and the KBE / GPL (w/o CE) baselines.
+Eager runs and graph replays, SF 0.02."""
 import os
 import sys
 
@@ -88,4 +90,34 @@ for _ in range(3):
 good = r.stats["agg_mode"] == 1 and {k[0]: tuple(a) for k, a in zip(r.keys, r.aggs)} == want
 ok &= good
 print("dense smem groups", "exact" if good else "MISMATCH")
+# builds with their probes and insert in the queue phase (a dense build zero-fills in the stage phase,
+# the drain writes the cells), and 4-bit cells (dense: whole-byte stores + atomics on shared bytes;
+# atomic builds; clustered and global probes)
+ctx.set_option("probe_split", 0)
+for q in ("Q5", "Q8"):
+    check("build_split=0", q, P.get(q))
+ctx.set_option("probe_split", -2)
+ctx.set_option("nibble_cells", 1)
+for q in ("Q5", "Q7", "Q9"):
+    check("nibble", q, P.get(q))
+ctx.set_option("dense_build", 0)
+check("nibble atomic", "Q7")
+ctx.set_option("dense_build", 1)
+import numpy as np  # noqa: E402
+rng = np.random.default_rng(5)
+k = (np.cumsum(rng.integers(1, 4, 20001)) + 1000).astype(np.int32)
+pay = rng.integers(3, 17, k.size).astype(np.int32)
+f = rng.integers(0, 100, k.size).astype(np.int32)
+ctx.load_columns("nt_dim", {"k": k, "p": pay, "f": f})
+ctx.load_columns("nt_fact", {"x": np.arange(int(k[0]) - 5, int(k[-1]) + 6, dtype=np.int32)})
+plan = ("build NT\nscan nt_dim\nfilter f < 60\nkey k\npayload p\n\n"
+        "run nt_fact\nprobe NT x -> pv\ngroup pv 3 17\nagg count\n")
+vals, cnts = np.unique(pay[f < 60], return_counts=True)
+for _ in range(3):
+    ctx.run_query(plan)
+    r = ctx.fetch_result()
+good = r.keys == [(int(v),) for v in vals] and r.aggs == [[int(c)] for c in cnts]
+ok &= good
+print("nibble random gaps", "exact" if good else "MISMATCH")
+ctx.set_option("nibble_cells", 0)
 sys.exit(0 if ok else 1)
