@@ -13,11 +13,11 @@ sf = float(sys.argv[2]) if len(sys.argv) > 2 else 0.1
 db = tpchgen.generate(sf, tables=sorted(set(queries.TABLES[q]) | {"region", "nation"}))
 ctx = gpl.Context(device=-1)
 queries.load_database(ctx, db)
-for kv in sys.argv[3:]:
-    k, v = kv.split("=")
-    ctx.set_option(k, int(v))
 segs = queries.segments(queries.plan_text(q, db))
 for s in segs[:-1]:
     ctx.build_hash(s)
+for kv in sys.argv[3:]:  # options of the probe segment (set after the builds)
+    k, v = kv.split("=")
+    ctx.set_option(k, int(v))
 print(ctx.choose_tile_rows(segs[-1]))
 ctx.compile_plan(segs[-1])
