@@ -1666,6 +1666,14 @@ static gpl_status tune_build(gpl_ctx* ctx, const std::string& text, void* flush,
       continue;
     }
     std::sort(ms.begin(), ms.end());
+    if (std::getenv("GPL_DEBUG_TUNE"))
+      std::fprintf(stderr, "[tune build %s] split %d tile %lld stage %d depth %d warps %d k %d pk %d: %.4f ms (pred %.4f)%s\n",
+                   s.name.c_str(), sp, (long long)c.tile_rows, c.stage_rows, c.depth, c.warps, c.ctas_per_sm, c.npack,
+                   ms[1], c.pred_ms,
+                   sp == sm && c.tile_rows == cm.tile_rows && c.stage_rows == cm.stage_rows && c.depth == cm.depth &&
+                           c.warps == cm.warps && c.ctas_per_sm == cm.ctas_per_sm && c.npack == cm.npack
+                       ? " <- model"
+                       : "");
     if (m0 < 0 && sp == sm && c.tile_rows == cm.tile_rows && c.stage_rows == cm.stage_rows && c.depth == cm.depth &&
         c.warps == cm.warps && c.ctas_per_sm == cm.ctas_per_sm && c.npack == cm.npack && c.ndrain == cm.ndrain)
       m0 = ms[1];
