@@ -208,6 +208,9 @@ def main():
                     help="pipeline shape: the A9 model's own pick after the plan's profiled runs (default), or "
                          "gpl_autotune's measured best of the model's shortlist")
     ap.add_argument("--no-autotune", action="store_true", help="(kept for scripts: same as --shape model)")
+    ap.add_argument("--collective", action="store_true",
+                    help="run the multi-rank merge (process group, all-gather of the partials, fixed-order merge) "
+                         "even at one rank: exercises the NCCL path on a one-GPU box")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -233,7 +236,10 @@ def main():
     # tensors) only to exercise the multi-rank path on a box with fewer GPUs
     backend = "nccl" if world <= ndev else "gloo"
     cdev = dev if backend == "nccl" else torch.device("cpu")
-    if world > 1:
+    multi = world > 1 or args.collective  # the collective merge path (also at one rank with --collective)
+    if multi:
+        for k, v in (("MASTER_ADDR", "127.0.0.1"), ("MASTER_PORT", "29517"), ("RANK", "0"), ("WORLD_SIZE", "1")):
+            os.environ.setdefault(k, v)
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=dev)
         else:
@@ -297,9 +303,9 @@ def main():
 
     def step():
         ctx.run_query(text, args.tile_rows)  # builds + fused run; a CUDA graph replay once warm
-        if world > 1 and hash_plan:
+        if multi and hash_plan:
             return hash_merge(ctx)
-        if world > 1:
+        if multi:
             nonlocal part_dev, gathered
             nb = ctx.partials_nbytes()
             if part_dev is None:
@@ -326,10 +332,10 @@ def main():
     # the plan (λ, then two timed runs for the model) and re-plan it once
     for _ in range(args.warmup if tuned else max(args.warmup, 6)):
         res = step()
-    res0 = ctx.fetch_result() if world == 1 else res
+    res0 = ctx.fetch_result() if not multi else res
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     step_ms, kern_ms = [], []
-    if world > 1:
+    if multi:
         dist.barrier()
     torch.cuda.synchronize()
     wall0 = time.time()
@@ -343,13 +349,13 @@ def main():
             step_ms.append(ev0.elapsed_time(ev1))
             kern_ms.append(res.stats["kernel_ms"])
     torch.cuda.synchronize()
-    if world > 1:
+    if multi:
         dist.barrier()
     wall = time.time() - wall0
     total_ms = sum(step_ms)
     kernel_avg = statistics.mean(kern_ms)
     stats = res0.stats
-    if world > 1:
+    if multi:
         t = torch.tensor([total_ms, kernel_avg], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms, kernel_avg = float(t[0]), float(t[1])
@@ -373,7 +379,7 @@ def main():
         def e2e_step():
             queries.load_database(ctx2, type("H", (), {"tables": pinned})(), borrow=False)
             ctx2.run_query(text, args.tile_rows)
-            if world == 1:
+            if not multi:
                 return ctx2.fetch_result()
             if hash_plan:
                 return hash_merge(ctx2)
@@ -398,7 +404,7 @@ def main():
         res_bytes = 16 + ctx2.fetch_groups().nbytes if hash_plan else ctx2.partials_nbytes()  # result rows / partials
         d2h = res_bytes + 16 * 8 + 4 + 16 * ncols  # + counters + errors + column min/max
         e_ms_v = statistics.mean(e_ms)
-        if world > 1:
+        if multi:
             t = torch.tensor([e_ms_v], dtype=torch.float64, device=cdev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_ms_v = float(t[0])
@@ -460,7 +466,7 @@ def main():
                                                "drain_warps")},
         "op_pass": stats["op_pass"],
         "collective": ((f"{backend} all_gather of hash group-by rows + gpl_merge_groups" if hash_plan else
-                        f"{backend} all_gather of int128 partials + fixed-order merge") if world > 1 else None),
+                        f"{backend} all_gather of int128 partials + fixed-order merge") if multi else None),
         "jit": stats.get("jit"),
         "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split",
                                               "builds_tuned", "build_ms_model", "build_ms")}
@@ -469,7 +475,7 @@ def main():
     if rank == 0:
         print(json.dumps(line), flush=True)
     ctx.close()
-    if world > 1:
+    if multi:
         dist.destroy_process_group()
     return 0
 
