@@ -240,6 +240,8 @@ def main():
     if multi:
         for k, v in (("MASTER_ADDR", "127.0.0.1"), ("MASTER_PORT", "29517"), ("RANK", "0"), ("WORLD_SIZE", "1")):
             os.environ.setdefault(k, v)
+        # NCCL's own log lines (e.g. its version banner) go to stderr: stdout carries the one JSON line
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=dev)
         else:

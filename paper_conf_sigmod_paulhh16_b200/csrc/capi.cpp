@@ -2002,24 +2002,13 @@ GPL_API gpl_status gpl_sync(gpl_ctx* ctx) {
   return take_device_errors(ctx);
 }
 
-GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
-  if (!ctx || !out) return GPL_E_ARG;
-  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
-  ctx->err.clear();
-  gpl_status st = check_dev(ctx);
-  if (st) return st;
-  if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run to fetch");
+// The host-visible side of a finished run (its counters are in h_stage after
+// a stream synchronise): kernel time, pass counts, the kernel's own bytes, and
+// the plan's λ profile / the model's profiling input while they are missing.
+static void observe_run(gpl_ctx* ctx) {
   const LowerInfo& li = ctx->last.run->li;
-  // one D2H: error bits, counter, op_pass and partials are contiguous
-  const size_t pbytes = run_pbytes(li);
-  // fused runs: the copy-out kernel already wrote the results to h_stage
-  if (!ctx->last.copied_out)
-    CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
-  CK(cudaStreamSynchronize(ctx->stream));
   const unsigned long long* hs = (const unsigned long long*)ctx->h_stage;
-  const unsigned int bits = (unsigned int)hs[0];
   const unsigned long long* ops = hs + 2;
-  const unsigned long long* part = hs + kScratchHead;
   gpl_stats& S = ctx->last.stats;
   if (ctx->last.timed) {
     float ms = 0;
@@ -2077,6 +2066,43 @@ GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
       ctx->profile[R.text] = p;
     }
   }
+}
+
+// Whether the plan of the last run still profiles (λ, then the model's two
+// profiled runs): its counters must then reach the host even when the caller
+// only takes the partials on the device (multi-rank merge).
+static bool run_profiling(gpl_ctx* ctx) {
+  if (ctx->last.kbe || !ctx->last.run) return false;
+  if (!ctx->lambda.count(ctx->last.run->text)) return true;
+  return ctx->last.timed && ctx->last.run->lambda_n > 0 &&
+         !profile_current(ctx, ctx->last.run->text, ctx->last.run->li.table);
+}
+
+// Bring the run's error bits, counters and partials to h_stage (one D2H unless
+// the fused run's copy-out kernel already wrote them) and synchronise.
+static gpl_status stage_run_to_host(gpl_ctx* ctx) {
+  const size_t pbytes = run_pbytes(ctx->last.run->li);
+  if (!ctx->last.copied_out)
+    CK(cudaMemcpyAsync(ctx->h_stage, ctx->d_scratch, kScratchHead * 8 + pbytes, cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  return GPL_OK;
+}
+
+GPL_API gpl_status gpl_fetch_result(gpl_ctx* ctx, gpl_result* out) {
+  if (!ctx || !out) return GPL_E_ARG;
+  if (gpl_status rs = resolve_pending(ctx)) return rs;  // loads still in flight (A0)
+  ctx->err.clear();
+  gpl_status st = check_dev(ctx);
+  if (st) return st;
+  if (!ctx->last.valid) return fail(ctx, GPL_E_STATE, "no run to fetch");
+  const LowerInfo& li = ctx->last.run->li;
+  // one D2H: error bits, counter, op_pass and partials are contiguous
+  if ((st = stage_run_to_host(ctx))) return st;
+  const unsigned long long* hs = (const unsigned long long*)ctx->h_stage;
+  const unsigned int bits = (unsigned int)hs[0];
+  const unsigned long long* part = hs + kScratchHead;
+  gpl_stats& S = ctx->last.stats;
+  observe_run(ctx);
   if (li.hash_group) {
     // distinct groups size the next run's table (load <= 1/2); an overflow
     // (ERR_CAPACITY) quadruples it
@@ -2111,6 +2137,13 @@ GPL_API gpl_status gpl_fetch_partials(gpl_ctx* ctx, void* dst, int32_t dst_on_de
   const size_t b = (size_t)ctx->last.run->li.ngroups_total * ctx->last.run->li.nagg * 16;
   *nbytes = b;
   if (cap_bytes < b || !dst) return fail(ctx, GPL_E_CAPACITY, "partials buffer too small");
+  // while the plan profiles (its first runs), the counters reach the host
+  // here too, so a multi-rank caller (which never fetches the rank's own
+  // result) gets the same λ-planned, profile-fitted plan as a single rank
+  if (run_profiling(ctx)) {
+    if ((st = stage_run_to_host(ctx))) return st;
+    observe_run(ctx);
+  }
   CK(cudaMemcpyAsync(dst, partials_ptr(ctx), b, dst_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
                      ctx->stream));
   if (!dst_on_device) CK(cudaStreamSynchronize(ctx->stream));
@@ -2161,6 +2194,10 @@ GPL_API gpl_status gpl_fetch_groups(gpl_ctx* ctx, int64_t* rows, int64_t cap_row
   if (!ctx->last.valid || !ctx->last.run || !ctx->last.run->li.hash_group)
     return fail(ctx, GPL_E_STATE, "gpl_fetch_groups: the last run is not a hash group-by");
   CK(cudaStreamSynchronize(ctx->stream));
+  if (run_profiling(ctx)) {  // a multi-rank caller profiles the plan through this call (see gpl_fetch_partials)
+    if ((st = stage_run_to_host(ctx))) return st;
+    observe_run(ctx);
+  }
   // an overflowed aggregation table holds an incomplete group set: never
   // returned as rows (whether or not gpl_fetch_result already took the bits)
   const gpl_status dev_st = take_device_errors(ctx);

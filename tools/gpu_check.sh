@@ -11,7 +11,7 @@ timeout 1200 python bench.py > $O/bench.json 2> $O/bench.err; head -c 400 $O/ben
 # the multi-rank merge path over NCCL at one rank (torchrun, process group, all-gather, fixed-order merge)
 timeout 1200 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29533 \
     bench.py --collective --steps 20 --no-cpu-baseline > $O/bench_collective.json 2> $O/bench_collective.err
-python -c "import json,sys; d=json.load(open('$O/bench_collective.json')); print('collective', d['collective'], d['ms_per_step'])"
+python -c "import json; d=[json.loads(l) for l in open('$O/bench_collective.json') if l.startswith('{')][0]; print('collective', d['collective'], d['ms_per_step'], d['kernel_ms'])"
 timeout 1500 python tools/kernel_ms.py 100 Q5 Q7 Q8 Q9 Q14 Q3 > $O/kernel_ms.txt 2>&1; grep SF $O/kernel_ms.txt
 # every kernel variant bit-exact (the compute-sanitizer driver, run plain: the pool has the sanitizer closed)
 timeout 900 python tools/sanitize_run.py > $O/variants.log 2>&1; echo "variants rc=$?" >> $O/variants.log; tail -3 $O/variants.log
