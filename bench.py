@@ -240,8 +240,11 @@ def main():
     if multi:
         for k, v in (("MASTER_ADDR", "127.0.0.1"), ("MASTER_PORT", "29517"), ("RANK", "0"), ("WORLD_SIZE", "1")):
             os.environ.setdefault(k, v)
-        # NCCL's own log lines (e.g. its version banner) go to stderr: stdout carries the one JSON line
-        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
+        # NCCL's own output (e.g. its version banner, printed to the process's stdout) goes to stderr:
+        # stdout carries only the one JSON line, written to the saved descriptor at the end
+        sys.stdout.flush()
+        json_fd = os.dup(1)
+        os.dup2(2, 1)
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=dev)
         else:
@@ -475,7 +478,11 @@ def main():
                      if tuned else None),
     }
     if rank == 0:
-        print(json.dumps(line), flush=True)
+        if multi:
+            sys.stdout.flush()
+            os.write(json_fd, (json.dumps(line) + "\n").encode())
+        else:
+            print(json.dumps(line), flush=True)
     ctx.close()
     if multi:
         dist.destroy_process_group()
