@@ -188,6 +188,9 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
     (p < d.nsprobe ? lat_stage : lat_queue) += p == d.cl_probe ? 40.0 : lat(li.probe_ht[p]);
   // lazy columns: one HBM gather round trip per drain (per 128 queued rows)
   if (!li.lazy_reach.empty()) lat_queue += 2000.0;
+  // a hash group-by sink: the group's slot load, the group count and the CAS
+  // that claims a new group are dependent round trips into a global table
+  if (d.agg_mode == AGG_HASH) lat_queue += 3 * 2000.0;
   // cycles per warp iteration of `npack` packets: the stage-phase probe
   // latency is paid once per iteration (all npack*4 loads of a lane in flight).
   // cons_rate(ka): fact rows per cycle per SM the consumer warps sustain with
@@ -279,8 +282,19 @@ Config predict(const gpl_ctx* ctx, const PipeDesc& d, const LowerInfo& li, int64
   // Eq 6 analog (ring handoff, ~mbarrier round trip per stage per CTA)
   const double stages_per_cta = (double)N / S / std::min<int64_t>(G, tiles);
   const double t_chan = stages_per_cta * 0.3e-6 / depth;
+  // Convoy (no drain warps): a warp draining 128 queued rows consumes none of
+  // its packets meanwhile; the ring's other depth - 1 stages cover up to
+  // (depth - 1) stage times of that, the rest stalls the CTA behind the slot
+  // the warp has not released (measured, SF 100 Q3: D = 2 drain warps 1.60 ms
+  // vs the best D = 0 shape 1.97 ms). Drains spread over the CTAs.
+  double t_convoy = 0;
+  if (ndrain == 0 && d.npush > 0 && qfrac > 0) {
+    const double t_drain = (lat_queue + queue_cost) * cf / f_sm;
+    const double drains_per_cta = (double)N * qfrac / 128.0 / (double)std::min<int64_t>(G, tiles);
+    t_convoy = drains_per_cta * std::max(0.0, t_drain - (depth - 1) * t_stage);
+  }
   // Eq 8/9 analog
-  const double tp = t_prod + t_chan, tc = t_cons;
+  const double tp = t_prod + t_chan, tc = t_cons + t_convoy;
   const double T = 0.5 * (tp + tc) + 0.5 * std::fabs(tp - tc);
   c.t_launch_ms = t0_cal >= 0 ? t0_cal : 4e-3 + 1e3 * (depth * t_stage);  // launch + prologue + ring fill
   c.t_stream_ms = 1e3 * (N * b / B);
