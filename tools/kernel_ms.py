@@ -45,5 +45,5 @@ for q in qs:
     b = r.stats["bytes_scanned"]
     print(f"{q} SF {sf}: step {st:.4f} ms, kernel {k:.4f} ms, own {b / 1e9:.3f} GB = {b / k / 1e6:.0f} GB/s "
           f"({b / k / 1e6 / 6544:.3f}), shape {r.stats['stage_rows']}x{r.stats['ring_depth']} "
-          f"W{r.stats['consumer_warps']} grid {r.stats['grid']} pk {r.stats['packets']}", flush=True)
+          f"W{r.stats['consumer_warps']} grid {r.stats['grid']} pk {r.stats['packets']} dr {r.stats['drain_warps']}", flush=True)
     ctx.close()
