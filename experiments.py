@@ -227,6 +227,11 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
         tw, rw = timed(True, (1 << 20) // bpr)
         # ... and with the paper's largest swept tile, 16 MB: fewer, larger tiles
         tw16, rw16 = timed(True, (16 << 20) // bpr)
+        # the same 1 MB / 16 MB tile loops launched kernel by kernel instead of replayed as one graph
+        ctx.set_option("kbe_graph", 0)
+        tl, _ = timed(True, (1 << 20) // bpr)
+        tl16, _ = timed(True, (16 << 20) // bpr)
+        ctx.set_option("kbe_graph", 1)
         assert (rf.keys, rf.aggs) == (rk.keys, rk.aggs) == (rw.keys, rw.aggs) == (rw16.keys, rw16.aggs), name
         inp = rf.stats.get("bytes_full_scan") or rf.stats["bytes_scanned"]  # the input: every column read, once
         ops = rf.stats["op_pass"]
@@ -237,6 +242,7 @@ def kbe_compare(sf=10.0, seed=20160626, reps=3, out=None):
                      "wo_ce_over_kbe": tw / tk, "wo_ce_intermediate_bytes": rw.stats["intermediate_bytes"],
                      "wo_ce_16mb_ms": tw16, "wo_ce_16mb_tile_rows": rw16.stats["tile_rows_used"],
                      "wo_ce_16mb_over_kbe": tw16 / tk,
+                     "wo_ce_launched_ms": tl, "wo_ce_16mb_launched_ms": tl16,
                      "fused_moved_bytes": rf.stats["bytes_scanned"], "fused_lazy_columns": rf.stats.get("lazy_columns"),
                      "fused_intermediate_bytes": rf.stats["intermediate_bytes"],
                      "kbe_intermediate_bytes": rk.stats["intermediate_bytes"],

@@ -398,6 +398,8 @@ GPL_API void gpl_destroy(gpl_ctx* ctx) {
     }
     if (ctx->d_scratch) cudaFree(ctx->d_scratch);
     for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
+    for (auto& kv : ctx->kbe_graphs)
+      if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
     if (ctx->h_stage) cudaFreeHost(ctx->h_stage);
     if (ctx->h_err) cudaFreeHost(ctx->h_err);
     if (ctx->h_minmax) cudaFreeHost(ctx->h_minmax);
@@ -449,6 +451,8 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
   } else if (k == "hash_load_pct") {
     if (v >= 0 && (v < 10 || v > 90)) return fail(ctx, GPL_E_ARG, "hash_load_pct in [10, 90]");
     o.hash_load_pct = v;
+  } else if (k == "kbe_graph") {
+    o.kbe_graph = v != 0 ? 1 : 0;
   } else if (k == "kbe_tile_rows") {
     if (v < 0) return fail(ctx, GPL_E_ARG, "kbe_tile_rows >= 0 (0 = whole input: KBE)");
     o.kbe_tile_rows = v;
@@ -1949,15 +1953,56 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
   const bool tiled = ctx->opt.kbe_tile_rows > 0;
   if (tiled && !ctx->d_kbe_bytes) CK(cudaMalloc(&ctx->d_kbe_bytes, sizeof(unsigned long long)));
   if (tiled) CK(cudaMemsetAsync(ctx->d_kbe_bytes, 0, sizeof(unsigned long long), ctx->stream));
+  auto tile_loop = [&](double* inter_out) -> cudaError_t {
+    for (long long r0 = 0; r0 < d.nrows || (r0 == 0 && d.nrows == 0); r0 += tile) {
+      dt = d;
+      dt.nrows = std::min<long long>(tile, d.nrows - r0);
+      for (int c = 0; c < d.ncols; c++) dt.col[c] = d.col[c] + r0 * d.colw[c];
+      double tb = 0;
+      cudaError_t e = run_kbe(dt, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &tb, tiled ? ctx->d_kbe_bytes : nullptr);
+      if (e != cudaSuccess) return e;
+      *inter_out += tb;
+      if (d.nrows == 0) break;
+    }
+    return cudaSuccess;
+  };
+  // GPL (w/o CE) on B200: the tiles' kernel sequence (map, scan, count, scatter
+  // per operator, device-side cardinalities) is launch-bound at small tiles, so
+  // the whole loop is captured once as a CUDA graph and replayed (the kernels
+  // still run one after another, tile by tile, intermediates materialised)
+  cudaStreamCaptureStatus capturing = cudaStreamCaptureStatusNone;
+  CK(cudaStreamIsCapturing(ctx->stream, &capturing));
+  const bool use_graph = tiled && ctx->opt.kbe_graph != 0 && d.nrows > tile && capturing == cudaStreamCaptureStatusNone;
+  gpl_ctx::KbeGraph* G = nullptr;
+  if (use_graph) {
+    G = &ctx->kbe_graphs[seg.text + "#" + std::to_string(tile)];
+    const std::vector<char> key((const char*)&d, (const char*)&d + sizeof(d));
+    if (!G->exec || G->desc != key || G->buf != ctx->kbe_buf || G->cap != ctx->kbe_cap || G->opt_version != ctx->opt_version) {
+      if (G->exec) cudaGraphExecDestroy(G->exec);
+      G->exec = nullptr;
+      double gi = 0;
+      CK(cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal));
+      const cudaError_t le = tile_loop(&gi);
+      cudaGraph_t graph = nullptr;
+      const cudaError_t ce = cudaStreamEndCapture(ctx->stream, &graph);
+      CK(le);
+      CK(ce);
+      const cudaError_t ie = cudaGraphInstantiate(&G->exec, graph, 0);
+      cudaGraphDestroy(graph);
+      CK(ie);
+      G->desc = key;
+      G->buf = ctx->kbe_buf;
+      G->cap = ctx->kbe_cap;
+      G->opt_version = ctx->opt_version;
+      G->inter = gi;
+    }
+  }
   CK(cudaEventRecord(ctx->ev0, ctx->stream));
-  for (long long r0 = 0; r0 < d.nrows || (r0 == 0 && d.nrows == 0); r0 += tile) {
-    dt = d;
-    dt.nrows = std::min<long long>(tile, d.nrows - r0);
-    for (int c = 0; c < d.ncols; c++) dt.col[c] = d.col[c] + r0 * d.colw[c];
-    double tb = 0;
-    CK(run_kbe(dt, ctx->sms, ctx->stream, ctx->kbe_buf, ctx->kbe_cap, &tb, tiled ? ctx->d_kbe_bytes : nullptr));
-    inter += tb;
-    if (d.nrows == 0) break;
+  if (G) {
+    CK(cudaGraphLaunch(G->exec, ctx->stream));
+    inter += G->inter;
+  } else {
+    CK(tile_loop(&inter));
   }
   CK(cudaEventRecord(ctx->ev1, ctx->stream));
   if (tiled) {  // the materialised bytes, read once after the run

@@ -203,6 +203,7 @@ struct Options {
   int64_t lazy_columns = -1;   // late materialisation: -1 auto (from λ), 0 off, 1 every eligible column
   int64_t build_pipeline = 1;
   int64_t clustered = 1;       // stage the cell range of a probe keyed by a sorted column (0: probe L2/HBM)
+  int64_t kbe_graph = 1;       // GPL (w/o CE): the tile loop replayed as one captured CUDA graph (0: launched)
   int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
   double hbm_gbs = -1;
   int64_t use_gamma = 1;       // the model uses the channel calibration Γ when one is loaded
@@ -297,4 +298,15 @@ struct gpl_ctx {
   // KBE scratch (gpl_run_plan_kbe)
   void* kbe_buf = nullptr;
   size_t kbe_cap = 0;
+  // GPL (w/o CE): the tile loop captured once per (plan, tile rows) and replayed while the lowered
+  // descriptor (pointers, sizes, shape), the scratch pool and the options are unchanged
+  struct KbeGraph {
+    cudaGraphExec_t exec = nullptr;
+    std::vector<char> desc;
+    void* buf = nullptr;
+    size_t cap = 0;
+    uint64_t opt_version = 0;
+    double inter = 0;
+  };
+  std::map<std::string, KbeGraph> kbe_graphs;
 };
