@@ -313,6 +313,7 @@ gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t
  * "build_pipeline" (1 = DIRECT build segments run through the fused pipeline
  * with an insert sink, default; 0 = the standalone build kernels),
  * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input),
+ * "kbe_graph" (1 = GPL (w/o CE)'s tile loop replayed as one captured CUDA graph, default; 0 = launched),
  * "use_gamma" (1 = the model uses the Γ calibration when loaded, default),
  * "drain_warps" (operator-specialised consumer warps, NEXT-1: of the
  * consumer warps, this many only run the queue phase of survivor packets the

@@ -333,18 +333,23 @@ def test_autotune_split_choice_exact(ctx):
 def test_gpl_without_ce_bit_identical(ctx, q):
     """GPL (w/o CE): the KBE kernel sequence run one tile at a
     time (ragged last tile) gives the same exact result as the whole-input KBE
-    and the fused pipeline."""
+    and the fused pipeline — replayed as a captured graph (repeated runs reuse
+    it) and launched kernel by kernel (kbe_graph 0)."""
     db = tpchgen.generate(0.05, seed=22)
     queries.load_database(ctx, db, queries.TABLES[q])
     o = _oracle(q, db, _params(q))
     try:
-        for tile in (1000, 7777, 1 << 22):
-            ctx.set_option("kbe_tile_rows", tile)
-            r = queries.run_query(ctx, q, db, _params(q), kbe=True)
-            assert r.keys == o.keys and r.aggs == o.aggs, (q, tile)
-            assert r.stats["tile_rows_used"] == min(tile, db.nrows("lineitem"))
+        for graph in (1, 0):
+            ctx.set_option("kbe_graph", graph)
+            for tile in (1000, 7777, 1 << 22, 1000):
+                for _ in range(2):
+                    ctx.set_option("kbe_tile_rows", tile)
+                    r = queries.run_query(ctx, q, db, _params(q), kbe=True)
+                    assert r.keys == o.keys and r.aggs == o.aggs, (q, tile, graph)
+                    assert r.stats["tile_rows_used"] == min(tile, db.nrows("lineitem"))
     finally:
         ctx.set_option("kbe_tile_rows", 0)
+        ctx.set_option("kbe_graph", 1)
 
 
 def test_fetch_after_unrelated_load(ctx):
