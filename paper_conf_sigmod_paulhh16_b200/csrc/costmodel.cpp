@@ -381,8 +381,12 @@ void apply_profile(const gpl_ctx* ctx, const PipeDesc& d, LowerInfo* li, const s
     return predict(ctx, d, *li, std::max<int64_t>(p.nrows, 1), p.tile_rows, p.stage_rows, p.depth, p.warps,
                    p.ctas_per_sm, p.npack, p.ndrain).pred_ms;
   };
-  // the prediction is non-decreasing in the factor: geometric bisection
-  const double lo = 0.05, hi = 50;
+  // the prediction is non-decreasing in the factor: geometric bisection. The
+  // factor is not taken below 0.3: a profiled run at the producer's bound only
+  // says the consumers kept up, and scaling their latency terms towards zero
+  // makes shapes with a few warps look as fast as many (measured, SF 100 Q9:
+  // a fitted 0.086 picked 4 consumer warps, 0.74 ms, over 12, 0.66 ms)
+  const double lo = 0.3, hi = 50;
   auto bisect = [](double a, double b, auto&& below) {  // below(x): the prediction at x is under the target
     for (int i = 0; i < 40; i++) {
       const double mid = std::sqrt(a * b);
