@@ -313,7 +313,7 @@ def knob_sweep(q="Q5", sf=1.0, seed=20160626, reps=3, out=None, setup=None):
     return summary
 
 
-def model_vs_autotune(qs=("Q5", "Q7", "Q8", "Q9", "Q14"), sf=100.0, seed=20160626, reps=5, out=None):
+def model_vs_autotune(qs=("Q5", "Q7", "Q8", "Q9", "Q14", "Q3"), sf=100.0, seed=20160626, reps=5, out=None):
     """A9 without autotune (config 4): the shape the re-derived model picks on its own (after the
     λ profile and the profiled run) vs the shape gpl_autotune measures best; kernel times
     (median of reps, L2 flushed), the model's Eq 10 error for its own pick, identical results."""
