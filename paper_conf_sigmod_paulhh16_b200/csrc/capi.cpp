@@ -781,6 +781,10 @@ static gpl_status lower_build_pipe(gpl_ctx* ctx, const Segment& s, const HashTab
   } else if (!choose_config(ctx, *pd, li, pd->nrows, 0, cfg, &err, shortlist)) {
     return fail(ctx, GPL_E_ARG, err);
   }
+  if (std::getenv("GPL_DEBUG_MODEL") && !shortlist)
+    std::fprintf(stderr, "build %s: split %d/%d tile %lld stage %d depth %d warps %d k %d pk %d pred %.4f ms%s\n",
+                 s.name.c_str(), pd->nsprobe, pd->nprobe, (long long)cfg->tile_rows, cfg->stage_rows, cfg->depth,
+                 cfg->warps, cfg->ctas_per_sm, cfg->npack, cfg->pred_ms, tu != ctx->tuned.end() ? " (pinned)" : "");
   apply_config(pd, li, *cfg);
   return GPL_OK;
 }
