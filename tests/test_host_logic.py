@@ -176,3 +176,30 @@ def test_jit_compiles_every_plan():
             if "NVRTC unavailable" in str(e):
                 pytest.skip(str(e))
             raise
+
+
+def test_jit_compiles_queue_builds_and_nibble_cells():
+    """NVRTC builds the kernels of the round-2 variants on a host-only context: DIRECT builds whose probes
+    and insert run in the queue phase (a dense build's zero fill in the stage phase, its cells from the
+    drain) and 4-bit cells (dense stage insert with whole-byte stores and edge atomics; clustered and
+    global probes of 4-bit tables)."""
+    db = tpchgen.generate(0.01, seed=2)
+    ctx = gpl.Context(device=-1)
+    queries.load_database(ctx, db)
+    try:
+        for nib, split in ((1, -2), (0, 0), (1, 0)):
+            ctx.set_option("nibble_cells", nib)
+            ctx.set_option("probe_split", split)
+            for q in ("Q5", "Q7", "Q9"):
+                segs = queries.segments(queries.plan_text(q, db))
+                for s in segs[:-1]:
+                    ctx.compile_plan(s)
+                    ctx.build_hash(s)
+                ctx.compile_plan(segs[-1])
+    except gpl.GplError as e:
+        if "NVRTC unavailable" in str(e):
+            pytest.skip(str(e))
+        raise
+    finally:
+        ctx.set_option("nibble_cells", 0)
+        ctx.set_option("probe_split", -2)
