@@ -1985,20 +1985,26 @@ GPL_API gpl_status gpl_run_plan_kbe(gpl_ctx* ctx, const char* probe_segment) {
       if (G->exec) cudaGraphExecDestroy(G->exec);
       G->exec = nullptr;
       double gi = 0;
-      CK(cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal));
-      const cudaError_t le = tile_loop(&gi);
       cudaGraph_t graph = nullptr;
-      const cudaError_t ce = cudaStreamEndCapture(ctx->stream, &graph);
-      CK(le);
-      CK(ce);
-      const cudaError_t ie = cudaGraphInstantiate(&G->exec, graph, 0);
-      cudaGraphDestroy(graph);
-      CK(ie);
-      G->desc = key;
-      G->buf = ctx->kbe_buf;
-      G->cap = ctx->kbe_cap;
-      G->opt_version = ctx->opt_version;
-      G->inter = gi;
+      // a stream that cannot be captured (the legacy default stream) or a graph
+      // that does not instantiate falls back to launching the loop
+      if (cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess) {
+        const cudaError_t le = tile_loop(&gi);
+        const cudaError_t ce = cudaStreamEndCapture(ctx->stream, &graph);
+        CK(le);
+        if (ce == cudaSuccess && graph && cudaGraphInstantiate(&G->exec, graph, 0) != cudaSuccess) G->exec = nullptr;
+        if (graph) cudaGraphDestroy(graph);
+      }
+      cudaGetLastError();
+      if (G->exec) {
+        G->desc = key;
+        G->buf = ctx->kbe_buf;
+        G->cap = ctx->kbe_cap;
+        G->opt_version = ctx->opt_version;
+        G->inter = gi;
+      } else {
+        G = nullptr;
+      }
     }
   }
   CK(cudaEventRecord(ctx->ev0, ctx->stream));
