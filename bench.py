@@ -188,8 +188,14 @@ def workload_config(args, rows_per_gpu, tile_rows):
             "seed": args.seed, "parallelism": f"dp{args.gpus} (order-key shards)" if args.gpus > 1 else "single",
             "l2": "flushed before every step (write of 2x L2); inputs are larger than L2",
             "tile_rows": tile_rows or "A9 cost model",
-            "shape": "gpl_autotune (model shortlist, measured)" if getattr(args, "shape", "model") == "autotune"
-            else "A9 cost model (profiled, no search)"}
+            "shape": SHAPE_NAMES[getattr(args, "shape", "model")]}
+
+
+SHAPE_NAMES = {
+    "model": "probe segment: A9 cost model (profiled, no search); build segments: gpl_autotune (measured)",
+    "model-all": "A9 cost model for every segment (profiled, no search)",
+    "autotune": "gpl_autotune (model shortlist, measured) for every segment",
+}
 
 
 def main():
@@ -204,10 +210,12 @@ def main():
     ap.add_argument("--tile-rows", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--shape", default="model", choices=["model", "autotune"],
-                    help="pipeline shape: the A9 model's own pick after the plan's profiled runs (default), or "
-                         "gpl_autotune's measured best of the model's shortlist")
-    ap.add_argument("--no-autotune", action="store_true", help="(kept for scripts: same as --shape model)")
+    ap.add_argument("--shape", default="model", choices=["model", "model-all", "autotune"],
+                    help="pipeline shapes: 'model' (default) = the A9 model's own pick for the probe segment (the "
+                         "paper's pipelined segment, tile size from the cost model) with the build segments' shapes "
+                         "measured by gpl_autotune; 'model-all' = the model's pick for every segment; 'autotune' = "
+                         "gpl_autotune's measured best of the model's shortlist for every segment")
+    ap.add_argument("--no-autotune", action="store_true", help="(kept for scripts: same as --shape model-all)")
     ap.add_argument("--collective", action="store_true",
                     help="run the multi-rank merge (process group, all-gather of the partials, fixed-order merge) "
                          "even at one rank: exercises the NCCL path on a one-GPU box")
@@ -328,14 +336,20 @@ def main():
             res = ctx.fetch_result()
         return res
 
-    # --shape autotune: measure the model's shortlist on the device (untimed); default: the model's own pick
+    # --shape autotune: measure the model's shortlist on the device (untimed) for every segment; model
+    # (default): the build segments only, the probe segment keeping the model's own pick; model-all: no search
     tuned = None
-    if args.shape == "autotune" and not args.no_autotune and args.tile_rows == 0:
+    if args.no_autotune:
+        args.shape = "model-all"
+    if args.shape in ("autotune", "model") and args.tile_rows == 0:
+        ctx.set_option("autotune_probe", 1 if args.shape == "autotune" else 0)
         tuned = ctx.autotune(text)
-        log(f"[rank {rank}] autotune: {tuned}")
+        log(f"[rank {rank}] autotune ({args.shape}): {tuned}")
+        if args.shape == "model":
+            tuned = None if not tuned else {k: tuned[k] for k in ("builds_tuned", "build_ms_model", "build_ms")}
     # warm-up: W steps; without autotune at least 6, since the first runs profile
     # the plan (λ, then two timed runs for the model) and re-plan it once
-    for _ in range(args.warmup if tuned else max(args.warmup, 6)):
+    for _ in range(args.warmup if args.shape == "autotune" else max(args.warmup, 6)):
         res = step()
     res0 = ctx.fetch_result() if not multi else res
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -473,9 +487,9 @@ def main():
         "collective": ((f"{backend} all_gather of hash group-by rows + gpl_merge_groups" if hash_plan else
                         f"{backend} all_gather of int128 partials + fixed-order merge") if multi else None),
         "jit": stats.get("jit"),
-        "autotune": ({k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split",
-                                              "builds_tuned", "build_ms_model", "build_ms")}
-                     if tuned else None),
+        "autotune": (tuned if args.shape == "model" else
+                     {k: tuned[k] for k in ("candidates", "measured_ms", "predicted_ms", "ctas_per_sm", "probe_split",
+                                            "builds_tuned", "build_ms_model", "build_ms")} if tuned else None),
     }
     if rank == 0:
         if multi:

@@ -314,6 +314,8 @@ gpl_status gpl_set_calibration(gpl_ctx* ctx, const gpl_gamma_point* pts, int32_t
  * with an insert sink, default; 0 = the standalone build kernels),
  * "kbe_tile_rows" (gpl_run_plan_kbe tile size; 0 = whole input),
  * "kbe_graph" (1 = GPL (w/o CE)'s tile loop replayed as one captured CUDA graph, default; 0 = launched),
+ * "autotune_probe" (1 = gpl_autotune measures the build segments and the probe segment, default; 0 = the
+ * build segments only, the probe segment keeping the A9 model's pick; changing it keeps pinned shapes),
  * "use_gamma" (1 = the model uses the Γ calibration when loaded, default),
  * "drain_warps" (operator-specialised consumer warps, NEXT-1: of the
  * consumer warps, this many only run the queue phase of survivor packets the

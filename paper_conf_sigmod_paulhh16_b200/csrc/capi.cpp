@@ -486,6 +486,10 @@ GPL_API gpl_status gpl_set_option(gpl_ctx* ctx, const char* key, int64_t value) 
     for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
     ctx->graphs.clear();
     return GPL_OK;
+  } else if (k == "autotune_probe") {
+    // only what gpl_autotune measures: plans and pinned shapes stay
+    o.autotune_probe = v != 0 ? 1 : 0;
+    return GPL_OK;
   } else if (k == "use_profile") {
     o.use_profile = v != 0 ? 1 : 0;
   } else if (k == "use_gamma") {
@@ -1728,6 +1732,19 @@ GPL_API gpl_status gpl_autotune(gpl_ctx* ctx, const char* plan, int32_t max_cand
   for (size_t i = 0; i + 1 < segs.size(); i++)
     if ((st = tune_build(ctx, segs[i], flush, fbytes, max_candidates, &build_ms_model, &build_ms, &builds_tuned)))
       return st;
+  if (!ctx->opt.autotune_probe) {
+    // the build segments only: the probe segment keeps the A9 model's own
+    // pick; query graphs recorded with the old build shapes are dropped
+    for (auto& kv : ctx->graphs) cudaGraphExecDestroy(kv.second);
+    ctx->graphs.clear();
+    if (out) {
+      *out = gpl_model_report{};
+      out->builds_tuned = builds_tuned;
+      out->build_ms_model = build_ms_model;
+      out->build_ms = build_ms;
+    }
+    return GPL_OK;
+  }
   const std::string& probe = segs.back();
   // one eager run profiles λ (the split and the model depend on it)
   if ((st = gpl_run_plan(ctx, probe.c_str(), 0))) return st;

@@ -203,6 +203,7 @@ struct Options {
   int64_t lazy_columns = -1;   // late materialisation: -1 auto (from λ), 0 off, 1 every eligible column
   int64_t build_pipeline = 1;
   int64_t clustered = 1;       // stage the cell range of a probe keyed by a sorted column (0: probe L2/HBM)
+  int64_t autotune_probe = 1;  // gpl_autotune: 1 = builds and the probe segment; 0 = the build segments only
   int64_t kbe_graph = 1;       // GPL (w/o CE): the tile loop replayed as one captured CUDA graph (0: launched)
   int64_t kbe_tile_rows = 0;   // gpl_run_plan_kbe: > 0 = GPL (w/o CE), the KBE sequence tile by tile  // DIRECT builds through the fused pipeline (0: build kernels)
   double hbm_gbs = -1;

@@ -1,6 +1,6 @@
 """Per-query probe-kernel and step times at one scale factor (the model's shapes, or gpl_autotune's with
 GPL_AUTOTUNE=1): median over 20 graph-replayed steps with L2 flushed, CUDA events on the library's stream.
-usage: [GPL_OPTS=k=v,...] [GPL_AUTOTUNE=1] python tools/kernel_ms.py SF Q5 Q7 ..."""
+usage: [GPL_OPTS=k=v,...] [GPL_AUTOTUNE=1|builds] python tools/kernel_ms.py SF Q5 Q7 ..."""
 import os
 import statistics
 import sys
@@ -27,7 +27,9 @@ for q in qs:
     for kv in filter(None, os.environ.get("GPL_OPTS", "").split(",")):  # e.g. GPL_OPTS=nibble_cells=0
         key, v = kv.split("=")
         ctx.set_option(key, int(v))
-    if os.environ.get("GPL_AUTOTUNE", "0") == "1":
+    mode = os.environ.get("GPL_AUTOTUNE", "0")  # 1: builds + probe measured; builds: the builds only
+    if mode in ("1", "builds"):
+        ctx.set_option("autotune_probe", 0 if mode == "builds" else 1)
         ctx.autotune(text)
     for _ in range(8):
         ctx.run_query(text)
