@@ -241,6 +241,26 @@ __device__ __forceinline__ void atomic_add_i128(unsigned long long* p, long long
   if (hi) gred_add_u64(p + 1, hi);
 }
 
+// The 128-bit sum of the lanes' int64 values (exact at any magnitude), and its
+// atomic addition into an int128 counter {lo, hi}.
+__device__ __forceinline__ void warp_sum_i128(long long v, unsigned long long& lo, long long& hi) {
+  lo = (unsigned long long)v;
+  hi = v < 0 ? -1ll : 0ll;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long l2 = __shfl_xor_sync(0xffffffffu, lo, o);
+    const long long h2 = __shfl_xor_sync(0xffffffffu, hi, o);
+    const unsigned long long s = lo + l2;
+    hi += h2 + (s < lo ? 1ll : 0ll);
+    lo = s;
+  }
+}
+__device__ __forceinline__ void atomic_add_i128_wide(unsigned long long* p, unsigned long long lo, long long hi) {
+  const unsigned long long old = gatom_add_u64(p, lo);
+  const unsigned long long h = (unsigned long long)hi + ((old + lo) < old ? 1ull : 0ull);
+  if (h) gred_add_u64(p + 1, h);
+}
+
 __device__ __forceinline__ long long warp_sum_i64(long long v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);

@@ -954,8 +954,12 @@ gpl_status lower_probe(gpl_ctx* ctx, const Segment& s, int split, PipeDesc* d, L
     d->agg_mode = AGG_HASH;
     d->flush_each_tile = 0;
   } else if (d->ngroups_total == 1) {
+    // a lane's register accumulator receives 4 rows of each 128-row packet (stage
+    // phase) or of each 128-entry drain, so at most nrows / 32 + 8 rows over the
+    // run; the warp's flush sums the lanes in 128 bits
     d->agg_mode = AGG_REG;
-    d->flush_each_tile = total >= lim ? 1 : 0;
+    const long double lane_total = ((long double)std::max<int64_t>(T.nrows, 1) / 32.0L + 8.0L) * std::max<long double>(li->maxabs, 1);
+    d->flush_each_tile = lane_total >= lim ? 1 : 0;
   } else {
     d->agg_mode = (total < lim && (int64_t)d->ngroups_total * d->nagg * 8 <= 48 * 1024) ? AGG_SMEM : AGG_GLOBAL;
     d->flush_each_tile = 0;

@@ -752,8 +752,11 @@ __device__ __forceinline__ void flush_reg(const PipeDesc& d, long long (&acc)[MA
 #pragma unroll
   for (int a = 0; a < MAXA; a++) {
     if (a < K.nagg) {
-      const long long s = warp_sum_i64(acc[a]);
-      if (lane == 0 && s != 0) atomic_add_i128(d.partials + 2 * a, s);
+      // (in 128 bits: each lane's accumulator is exact, the warp's sum may not fit int64)
+      unsigned long long lo;
+      long long hi;
+      warp_sum_i128(acc[a], lo, hi);
+      if (lane == 0 && (lo | (unsigned long long)hi) != 0) atomic_add_i128_wide(d.partials + 2 * a, lo, hi);
       acc[a] = 0;
     }
   }

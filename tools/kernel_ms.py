@@ -23,7 +23,7 @@ ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=
 for q in qs:
     ctx = gpl.Context(0, stream=stream)
     queries.load_database(ctx, db, queries.TABLES[q])
-    text = queries.plan_text(q, db)
+    text = queries.plan_text(q, db, (19981101,) if q == "L1" else None)  # L1: the non-empty 1998 variant (R1)
     for kv in filter(None, os.environ.get("GPL_OPTS", "").split(",")):  # e.g. GPL_OPTS=nibble_cells=0
         key, v = kv.split("=")
         ctx.set_option(key, int(v))
